@@ -1,0 +1,655 @@
+/*
+ * ss_oracle.c -- CPU ORACLE (TEST INFRASTRUCTURE ONLY; see ss_oracle.h).
+ *
+ * Plain, single-threaded, obviously-correct C following the definitions the
+ * product must reproduce.  The paper (SLAM-Share, CoNEXT'22) moves ORB-SLAM3's
+ * FAST detection and "search local points" onto a GPU (§4.2.1)
+ * but prints no arithmetic; every step below therefore follows the reading in
+ * SURVEY.md §8(c) (rows O0..O10), each of which DESIGN.md §3 lists.
+ *
+ * Build: gcc -O2 -ffp-contract=off -fPIC -shared (no SIMD intrinsics, no OpenMP).
+ * Nothing here is shared with the CUDA path.
+ *
+ * Parity pins (tests/test_oracle_*.py):
+ *   O0 params      : App. B tables of SURVEY.md (tests/golden/params_*.json)
+ *   O1 pyramid     : cv2.resize(INTER_LINEAR_EXACT), chained
+ *   O2 FAST M      : cv2.FAST(TYPE_9_16) thresholds/responses; exhaustive ring masks
+ *   O3 cells       : ORB-SLAM's per-cell cv2.FAST loop with iniTh/minTh fallback
+ *   O4 quadtree    : hand-worked cases (tests/golden/quadtree_cases.json) + invariants
+ *                    + an independent std::list-style transcription.  NO external
+ *                    reference exists (ORB-SLAM's tie-break is heap-address order):
+ *                    "parity unpinned" against ORB-SLAM itself, see DESIGN.md.
+ *   O5 orientation : closed form on intensity planes; rot90 permutation
+ *   O6 blur        : cv2.GaussianBlur(7x7, sigma 2, REFLECT_101)
+ *   O7 descriptor  : rot90 invariance (bit-exact); unrotated case = pattern lookups
+ *   O9/O10 match   : brute-force definitions in Python on small inputs
+ */
+#include "ss_oracle.h"
+
+#include <math.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include "brief_pattern_ref.inc"
+
+#define EDGE_THRESHOLD 19
+#define MIN_BORDER (EDGE_THRESHOLD - 3) /* 16 */
+#define CELL_W 30                       /* north_star: "per 30-px grid cell" */
+#define HALF_PATCH 15
+
+static int imin(int a, int b) { return a < b ? a : b; }
+static int imax(int a, int b) { return a > b ? a : b; }
+
+/* ---------------------------------------------------------------- O0 params */
+/* S8c O0: f32 scale chain, rne level sizes, ORB-SLAM per-level feature split. */
+int ref_params_init(int32_t w, int32_t h, int32_t nf, int32_t L, float sf, int32_t ini, int32_t mn,
+                    ref_params* p) {
+  if (!p || L < 1 || L > REF_MAX_LEVELS || w < 64 || h < 64 || w > 2048 || h > 2048 || nf < 1 ||
+      !(sf > 1.0f) || ini < 1 || mn < 1 || ini > 254 || mn > 254)
+    return -1;
+  memset(p, 0, sizeof(*p));
+  p->width = w; p->height = h; p->n_features = nf; p->n_levels = L; p->scale_factor = sf;
+  p->ini_th_fast = ini; p->min_th_fast = mn;
+  p->scale[0] = 1.0f;
+  for (int l = 1; l < L; l++) p->scale[l] = p->scale[l - 1] * sf;
+  for (int l = 0; l < L; l++) p->inv_scale[l] = 1.0f / p->scale[l];
+  for (int l = 0; l < L; l++) {
+    float fw = (float)w * p->inv_scale[l];
+    float fh = (float)h * p->inv_scale[l];
+    p->level_w[l] = (int32_t)lrintf(fw);
+    p->level_h[l] = (int32_t)lrintf(fh);
+  }
+  float factor = 1.0f / sf;
+  float nd = (float)nf * (1.0f - factor) / (1.0f - (float)pow((double)factor, (double)L));
+  int sum = 0;
+  for (int l = 0; l < L - 1; l++) {
+    p->n_per_level[l] = (int32_t)lrintf(nd);
+    sum += p->n_per_level[l];
+    nd *= factor;
+  }
+  p->n_per_level[L - 1] = imax(nf - sum, 0);
+  int cap = 0;
+  for (int l = 0; l < L; l++) {
+    int lw = p->level_w[l], lh = p->level_h[l];
+    int maxBX = lw - EDGE_THRESHOLD + 3, maxBY = lh - EDGE_THRESHOLD + 3;
+    float width = (float)(maxBX - MIN_BORDER), height = (float)(maxBY - MIN_BORDER);
+    int ncols = (int)(width / (float)CELL_W), nrows = (int)(height / (float)CELL_W);
+    if (ncols < 1 || nrows < 1) return -1;
+    p->cell_cols[l] = ncols; p->cell_rows[l] = nrows;
+    p->cell_w[l] = (int)ceilf(width / (float)ncols);
+    p->cell_h[l] = (int)ceilf(height / (float)nrows);
+    int nini = (int)roundf(width / height); /* std::round: half away from zero */
+    if (nini < 1 || nini > 62) return -1;
+    p->n_ini[l] = nini;
+    /* S8c O4: <= N+2 after phase 1/2, but the first unconditional split can give 4*nIni. */
+    p->level_cap[l] = imax(p->n_per_level[l] + 2, 4 * nini);
+    cap += p->level_cap[l];
+  }
+  p->kp_capacity = cap;
+  return 0;
+}
+
+/* ---------------------------------------------------------------- O1 pyramid */
+/* S8c O1: bit-exact INTER_LINEAR_EXACT (8-bit weights, f64 source mapping, rne weights). */
+static void linear_coeffs(int d, int sn, int dn, int* s0, int* s1, int* w1) {
+  double f = ((double)d + 0.5) * ((double)sn / (double)dn) - 0.5;
+  double fl = floor(f);
+  int s = (int)fl;
+  double a = f - fl;
+  if (s < 0) { s = 0; a = 0.0; }
+  if (s >= sn - 1) { s = sn - 1; a = 0.0; }
+  *s0 = s;
+  *s1 = imin(s + 1, sn - 1);
+  *w1 = (int)lrint(a * 256.0); /* round half even */
+}
+
+void ref_resize_linear_exact(const uint8_t* src, int sw, int sh, int sp, uint8_t* dst, int dw, int dh,
+                             int dp) {
+  for (int y = 0; y < dh; y++) {
+    int y0, y1, wy1;
+    linear_coeffs(y, sh, dh, &y0, &y1, &wy1);
+    int wy0 = 256 - wy1;
+    for (int x = 0; x < dw; x++) {
+      int x0, x1, wx1;
+      linear_coeffs(x, sw, dw, &x0, &x1, &wx1);
+      int wx0 = 256 - wx1;
+      int h0 = wx0 * src[y0 * sp + x0] + wx1 * src[y0 * sp + x1];
+      int h1 = wx0 * src[y1 * sp + x0] + wx1 * src[y1 * sp + x1];
+      int v = wy0 * h0 + wy1 * h1;
+      dst[y * dp + x] = (uint8_t)((v + (1 << 15)) >> 16);
+    }
+  }
+}
+
+int64_t ref_pyramid_bytes(const ref_params* p) {
+  int64_t s = 0;
+  for (int l = 0; l < p->n_levels; l++) s += (int64_t)p->level_w[l] * p->level_h[l];
+  return s;
+}
+
+void ref_pyramid(const ref_params* p, const uint8_t* img, int pitch, uint8_t* out) {
+  int64_t off = 0, prev = 0;
+  for (int l = 0; l < p->n_levels; l++) {
+    int w = p->level_w[l], h = p->level_h[l];
+    if (l == 0) {
+      for (int y = 0; y < h; y++) memcpy(out + (int64_t)y * w, img + (int64_t)y * pitch, (size_t)w);
+    } else {
+      ref_resize_linear_exact(out + prev, p->level_w[l - 1], p->level_h[l - 1], p->level_w[l - 1],
+                              out + off, w, h, w);
+    }
+    prev = off;
+    off += (int64_t)w * h;
+  }
+}
+
+/* ---------------------------------------------------------------- O2 FAST */
+/* OpenCV offsets16 order, (dx, dy). FAST-9/16 [38]. */
+static const int RING[16][2] = {{0, 3},  {1, 3},   {2, 2},   {3, 1},   {3, 0},  {3, -1},
+                                {2, -2}, {1, -3},  {0, -3},  {-1, -3}, {-2, -2}, {-3, -1},
+                                {-3, 0}, {-3, 1},  {-2, 2},  {-1, 3}};
+
+/* M(p) = max_s max( min_{k<9} d_{s+k}, min_{k<9} -d_{s+k} ),  d_k = I(p) - I(p + R_k).
+ * corner at threshold t  <=>  M > t ;  OpenCV response = M - 1. */
+static int fast_M_at(const uint8_t* img, int pitch, int x, int y) {
+  int c = img[y * pitch + x];
+  int d[16];
+  for (int k = 0; k < 16; k++) d[k] = c - img[(y + RING[k][1]) * pitch + x + RING[k][0]];
+  int best = -1000;
+  for (int s = 0; s < 16; s++) {
+    int mn = 1000, mx = 1000;
+    for (int k = 0; k < 9; k++) {
+      int v = d[(s + k) & 15];
+      if (v < mn) mn = v;
+      if (-v < mx) mx = -v;
+    }
+    if (mn > best) best = mn;
+    if (mx > best) best = mx;
+  }
+  return best;
+}
+
+void ref_fast_M(const uint8_t* img, int w, int h, int pitch, uint8_t* out) {
+  memset(out, 0, (size_t)w * h);
+  for (int y = 3; y < h - 3; y++)
+    for (int x = 3; x < w - 3; x++) {
+      int m = fast_M_at(img, pitch, x, y);
+      out[y * w + x] = (uint8_t)(m < 0 ? 0 : m);
+    }
+}
+
+/* ---------------------------------------------------------------- O3 cells */
+/* ORB-SLAM's per-cell FAST (cv::FAST on the cell ROI, nonmax on) with the iniTh ->
+ * minTh fallback [ext], restated: in the detect window D of the cell, keep p with
+ * M(p) > t that beats every 8-neighbour inside D (S8c O3). Rank = cell row-major, y, x. */
+int ref_cell_candidates(const ref_params* p, int l, const uint8_t* M, int32_t* lx, int32_t* ly,
+                        int32_t* score, int cap) {
+  int w = p->level_w[l], h = p->level_h[l];
+  int maxBX = w - EDGE_THRESHOLD + 3, maxBY = h - EDGE_THRESHOLD + 3;
+  int wc = p->cell_w[l], hc = p->cell_h[l];
+  int n = 0;
+  (void)h;
+  for (int i = 0; i < p->cell_rows[l]; i++) {
+    int iniY = MIN_BORDER + i * hc;
+    if (iniY >= maxBY - 3) continue;
+    int maxY = imin(iniY + hc + 6, maxBY);
+    for (int j = 0; j < p->cell_cols[l]; j++) {
+      int iniX = MIN_BORDER + j * wc;
+      if (iniX >= maxBX - 6) continue;
+      int maxX = imin(iniX + wc + 6, maxBX);
+      int x0 = iniX + 3, x1 = maxX - 3, y0 = iniY + 3, y1 = maxY - 3;
+      int thr[2] = {p->ini_th_fast, p->min_th_fast};
+      for (int pass = 0; pass < 2; pass++) {
+        int found = 0;
+        for (int y = y0; y < y1; y++)
+          for (int x = x0; x < x1; x++) {
+            int m = M[y * w + x];
+            if (m <= thr[pass]) continue;
+            int keep = 1;
+            for (int dy = -1; dy <= 1 && keep; dy++)
+              for (int dx = -1; dx <= 1; dx++) {
+                if (!dx && !dy) continue;
+                int qx = x + dx, qy = y + dy;
+                if (qx < x0 || qx >= x1 || qy < y0 || qy >= y1) continue; /* outside D: ignored */
+                if (M[qy * w + qx] >= m) { keep = 0; break; }
+              }
+            if (!keep) continue;
+            if (n >= cap) return -1;
+            lx[n] = x; ly[n] = y; score[n] = m; n++;
+            found++;
+          }
+        if (found) break;
+      }
+    }
+  }
+  return n;
+}
+
+/* ---------------------------------------------------------------- O4 quadtree */
+/* Literal transcription of ORB-SLAM's DistributeOctTree [ext] (S8c O4): f32 root
+ * geometry, ceil halving, phase 1 (split every multi-key node) and phase 2 (split
+ * largest nodes first until N), "no progress" stop, per-node max response with ties to
+ * the first key in parent order.  Reading: equal-size nodes in phase 2 are ordered by
+ * (UL.y, UL.x, first-key rank) instead of heap address.  parity unpinned vs ORB-SLAM. */
+typedef struct {
+  int ulx, uly, urx, blx, bly; /* UR.y == UL.y, BR = (UR.x, BL.y) */
+  int* keys;                   /* indices into the input, in parent order */
+  int n;
+  int nomore;
+} qnode;
+
+typedef struct {
+  qnode* v;
+  int n, cap;
+} qlist;
+
+static void qpush(qlist* L, qnode nd) {
+  if (L->n == L->cap) {
+    L->cap = L->cap ? 2 * L->cap : 64;
+    L->v = (qnode*)realloc(L->v, sizeof(qnode) * (size_t)L->cap);
+  }
+  L->v[L->n++] = nd;
+}
+
+static void qdivide(const qnode* nd, const int32_t* kx, const int32_t* ky, qnode ch[4]) {
+  int halfX = (int)ceilf((float)(nd->urx - nd->ulx) / 2);
+  int halfY = (int)ceilf((float)(nd->bly - nd->uly) / 2);
+  /* n1 TL, n2 TR, n3 BL, n4 BR (ORB-SLAM ExtractorNode::DivideNode) */
+  ch[0].ulx = nd->ulx;         ch[0].uly = nd->uly;         ch[0].urx = nd->ulx + halfX;
+  ch[0].blx = nd->ulx;         ch[0].bly = nd->uly + halfY;
+  ch[1].ulx = nd->ulx + halfX; ch[1].uly = nd->uly;         ch[1].urx = nd->urx;
+  ch[1].blx = nd->ulx + halfX; ch[1].bly = nd->uly + halfY;
+  ch[2].ulx = nd->ulx;         ch[2].uly = nd->uly + halfY; ch[2].urx = nd->ulx + halfX;
+  ch[2].blx = nd->blx;         ch[2].bly = nd->bly;
+  ch[3].ulx = nd->ulx + halfX; ch[3].uly = nd->uly + halfY; ch[3].urx = nd->urx;
+  ch[3].blx = nd->ulx + halfX; ch[3].bly = nd->bly;
+  for (int c = 0; c < 4; c++) {
+    ch[c].keys = (int*)malloc(sizeof(int) * (size_t)(nd->n > 0 ? nd->n : 1));
+    ch[c].n = 0;
+    ch[c].nomore = 0;
+  }
+  int midx = nd->ulx + halfX, midy = nd->uly + halfY;
+  for (int i = 0; i < nd->n; i++) {
+    int k = nd->keys[i];
+    int c;
+    if (kx[k] < midx) c = (ky[k] < midy) ? 0 : 2;
+    else c = (ky[k] < midy) ? 1 : 3;
+    ch[c].keys[ch[c].n++] = k;
+  }
+  for (int c = 0; c < 4; c++)
+    if (ch[c].n == 1) ch[c].nomore = 1;
+}
+
+/* phase-2 order: size desc, UL.y asc, UL.x asc, first-key rank asc (reading) */
+static const qnode* g_sort_base;
+static int cmp_phase2(const void* a, const void* b) {
+  const qnode* A = &g_sort_base[*(const int*)a];
+  const qnode* B = &g_sort_base[*(const int*)b];
+  if (A->n != B->n) return A->n > B->n ? -1 : 1;
+  if (A->uly != B->uly) return A->uly < B->uly ? -1 : 1;
+  if (A->ulx != B->ulx) return A->ulx < B->ulx ? -1 : 1;
+  return A->keys[0] < B->keys[0] ? -1 : (A->keys[0] > B->keys[0] ? 1 : 0);
+}
+
+/* Splits node index `idx` of *nodes (marking it dead, n = -1) and appends the non-empty
+ * children; indices of children with > 1 key are appended to *expand. Returns #children. */
+static int split_node(qlist* nodes, int idx, const int32_t* kx, const int32_t* ky, int** expand,
+                      int* nexp, int* expcap) {
+  qnode ch[4];
+  qnode parent = nodes->v[idx];
+  qdivide(&parent, kx, ky, ch);
+  free(parent.keys);
+  nodes->v[idx].keys = NULL;
+  nodes->v[idx].n = -1; /* dead */
+  int made = 0;
+  for (int c = 0; c < 4; c++) {
+    if (ch[c].n > 0) {
+      qpush(nodes, ch[c]);
+      made++;
+      if (ch[c].n > 1) {
+        if (*nexp == *expcap) {
+          *expcap = *expcap ? 2 * *expcap : 64;
+          *expand = (int*)realloc(*expand, sizeof(int) * (size_t)*expcap);
+        }
+        (*expand)[(*nexp)++] = nodes->n - 1;
+      }
+    } else {
+      free(ch[c].keys);
+    }
+  }
+  return made;
+}
+
+int ref_distribute(const int32_t* kx, const int32_t* ky, const int32_t* score, int n, int width,
+                   int height, int N, int32_t* out_idx) {
+  if (n <= 0) return 0;
+  int nIni = (int)roundf((float)width / (float)height);
+  if (nIni < 1) return -1;
+  float hX = (float)width / (float)nIni;
+  qlist nodes = {0, 0, 0};
+  int alive = 0;
+  /* roots */
+  int root0 = 0;
+  for (int i = 0; i < nIni; i++) {
+    qnode r;
+    r.ulx = (int)(hX * (float)i);
+    r.uly = 0;
+    r.urx = (int)(hX * (float)(i + 1));
+    r.blx = r.ulx;
+    r.bly = height;
+    r.keys = (int*)malloc(sizeof(int) * (size_t)n);
+    r.n = 0;
+    r.nomore = 0;
+    qpush(&nodes, r);
+  }
+  for (int k = 0; k < n; k++) {
+    int ri = (int)((float)kx[k] / hX);
+    if (ri > nIni - 1) ri = nIni - 1; /* unreachable for widths <= 2048; kept defined */
+    nodes.v[root0 + ri].keys[nodes.v[root0 + ri].n++] = k;
+  }
+  for (int i = 0; i < nIni; i++) {
+    qnode* r = &nodes.v[i];
+    if (r->n == 0) { free(r->keys); r->keys = NULL; r->n = -1; }
+    else { if (r->n == 1) r->nomore = 1; alive++; }
+  }
+  int* expand = NULL;
+  int nexp = 0, expcap = 0;
+  int finish = 0;
+  while (!finish) {
+    int prevSize = alive;
+    int nToExpand;
+    nexp = 0;
+    int cur = nodes.n;
+    for (int i = 0; i < cur; i++) {
+      if (nodes.v[i].n < 0 || nodes.v[i].nomore) continue;
+      int made = split_node(&nodes, i, kx, ky, &expand, &nexp, &expcap);
+      alive += made - 1;
+    }
+    nToExpand = nexp;
+    if (alive >= N || alive == prevSize) {
+      finish = 1;
+    } else if (alive + nToExpand * 3 > N) {
+      while (!finish) {
+        prevSize = alive;
+        int nprev = nexp;
+        int* prev = (int*)malloc(sizeof(int) * (size_t)(nprev > 0 ? nprev : 1));
+        memcpy(prev, expand, sizeof(int) * (size_t)nprev);
+        nexp = 0;
+        g_sort_base = nodes.v;
+        qsort(prev, (size_t)nprev, sizeof(int), cmp_phase2);
+        for (int j = 0; j < nprev; j++) {
+          int made = split_node(&nodes, prev[j], kx, ky, &expand, &nexp, &expcap);
+          alive += made - 1;
+          g_sort_base = nodes.v; /* nodes.v may have been reallocated */
+          if (alive >= N) break;
+        }
+        free(prev);
+        if (alive >= N || alive == prevSize) finish = 1;
+      }
+    }
+  }
+  /* retain the best key of each node: max score, ties -> first key (smallest rank) */
+  int m = 0;
+  for (int i = 0; i < nodes.n; i++) {
+    qnode* nd = &nodes.v[i];
+    if (nd->n < 0) continue;
+    int best = nd->keys[0];
+    for (int t = 1; t < nd->n; t++)
+      if (score[nd->keys[t]] > score[best]) best = nd->keys[t];
+    out_idx[m++] = best;
+    free(nd->keys);
+  }
+  free(nodes.v);
+  free(expand);
+  return m;
+}
+
+/* ---------------------------------------------------------------- O5 orientation */
+/* umax built as ORB-SLAM's ORBextractor constructor does [ext]; 749-px disk. */
+static void build_umax(int umax[HALF_PATCH + 1]) {
+  int vmax = (int)floor(HALF_PATCH * sqrt(2.f) / 2 + 1);
+  int vmin = (int)ceil(HALF_PATCH * sqrt(2.f) / 2);
+  const double hp2 = HALF_PATCH * HALF_PATCH;
+  int v, v0;
+  for (v = 0; v <= vmax; ++v) umax[v] = (int)lrint(sqrt(hp2 - v * v));
+  for (v = HALF_PATCH, v0 = 0; v >= vmin; --v) {
+    while (umax[v0] == umax[v0 + 1]) ++v0;
+    umax[v] = v0;
+    ++v0;
+  }
+}
+
+/* "Oriented FAST": intensity-centroid moments over the disk (S8c O5). */
+void ref_moments(const uint8_t* img, int pitch, int lx, int ly, int32_t* m10, int32_t* m01) {
+  int umax[HALF_PATCH + 1];
+  build_umax(umax);
+  int64_t a = 0, b = 0;
+  for (int v = -HALF_PATCH; v <= HALF_PATCH; v++) {
+    int d = umax[v < 0 ? -v : v];
+    for (int u = -d; u <= d; u++) {
+      int I = img[(ly + v) * pitch + lx + u];
+      a += (int64_t)u * I;
+      b += (int64_t)v * I;
+    }
+  }
+  *m10 = (int32_t)a;
+  *m01 = (int32_t)b;
+}
+
+/* angle = atan2(m01, m10) in degrees, [0, 360); (0,0) -> 0 (S8c O5 reading). */
+float ref_angle_deg(int32_t m10, int32_t m01) {
+  if (m10 == 0 && m01 == 0) return 0.0f;
+  double a = atan2((double)m01, (double)m10) * (180.0 / 3.14159265358979323846);
+  if (a < 0) a += 360.0;
+  float f = (float)a;
+  if (f >= 360.0f) f = 0.0f;
+  return f;
+}
+
+/* ---------------------------------------------------------------- O6 blur */
+/* GaussianBlur(7x7, sigma=2, REFLECT_101) bit-exact fixed point: Q8 taps, exact
+ * horizontal sum, vertical (sum + 2^15) >> 16 (S8c O6). */
+static const int BLUR_K[7] = {18, 34, 48, 56, 48, 34, 18};
+
+static int reflect101(int i, int n) {
+  while (i < 0 || i >= n) {
+    if (i < 0) i = -i;
+    if (i >= n) i = 2 * n - 2 - i;
+  }
+  return i;
+}
+
+void ref_blur(const uint8_t* img, int w, int h, int pitch, uint8_t* out, int opitch) {
+  int* hs = (int*)malloc(sizeof(int) * (size_t)w * h);
+  for (int y = 0; y < h; y++)
+    for (int x = 0; x < w; x++) {
+      int s = 0;
+      for (int j = 0; j < 7; j++) s += BLUR_K[j] * img[y * pitch + reflect101(x + j - 3, w)];
+      hs[y * w + x] = s;
+    }
+  for (int y = 0; y < h; y++)
+    for (int x = 0; x < w; x++) {
+      int64_t s = 0;
+      for (int i = 0; i < 7; i++) s += (int64_t)BLUR_K[i] * hs[reflect101(y + i - 3, h) * w + x];
+      out[y * opitch + x] = (uint8_t)((s + (1 << 15)) >> 16);
+    }
+  free(hs);
+}
+
+/* ---------------------------------------------------------------- O7 descriptor */
+/* Exact round-half-even of z / sqrt(r2), r2 > 0, by plain integer search (S8c O7). */
+int32_t ref_rhe_div_sqrt(int64_t z, int64_t r2) {
+  int neg = z < 0;
+  int64_t a = neg ? -z : z;
+  int64_t A = 4 * a * a; /* (2a)^2 */
+  int64_t k = 0;
+  while ((2 * k + 1) * (2 * k + 1) * r2 < A) k++; /* a/r in (k-1/2, k+1/2] */
+  if ((2 * k + 1) * (2 * k + 1) * r2 == A && (k & 1)) k++; /* a/r == k+1/2: to even */
+  return (int32_t)(neg ? -k : k);
+}
+
+/* Rotated BRIEF: offsets (x cos - y sin, x sin + y cos) with cos = m10/r,
+ * sin = m01/r, exactly rounded; bit b = B(p_2b) < B(p_2b+1), LSB first. */
+void ref_descriptor(const uint8_t* B, int pitch, int lx, int ly, int32_t m10, int32_t m01,
+                    uint8_t out[32]) {
+  int64_t r2 = (int64_t)m10 * m10 + (int64_t)m01 * m01;
+  memset(out, 0, 32);
+  for (int b = 0; b < 256; b++) {
+    int v[2];
+    for (int e = 0; e < 2; e++) {
+      int px = REF_BRIEF_PATTERN[4 * b + 2 * e], py = REF_BRIEF_PATTERN[4 * b + 2 * e + 1];
+      int ox, oy;
+      if (r2 == 0) { ox = px; oy = py; }
+      else {
+        ox = ref_rhe_div_sqrt((int64_t)px * m10 - (int64_t)py * m01, r2);
+        oy = ref_rhe_div_sqrt((int64_t)px * m01 + (int64_t)py * m10, r2);
+      }
+      v[e] = B[(ly + oy) * pitch + lx + ox];
+    }
+    if (v[0] < v[1]) out[b >> 3] |= (uint8_t)(1u << (b & 7));
+  }
+}
+
+/* ---------------------------------------------------------------- O1..O8 */
+typedef struct { int lx, ly, score; } selkp;
+static int cmp_yx(const void* a, const void* b) {
+  const selkp* A = (const selkp*)a; const selkp* B = (const selkp*)b;
+  if (A->ly != B->ly) return A->ly < B->ly ? -1 : 1;
+  return A->lx < B->lx ? -1 : (A->lx > B->lx ? 1 : 0);
+}
+
+int ref_orb_extract(const ref_params* p, const uint8_t* img, int pitch, ref_keypoint* kps,
+                    uint8_t* desc, int32_t* counts) {
+  int64_t pb = ref_pyramid_bytes(p);
+  uint8_t* pyr = (uint8_t*)malloc((size_t)pb);
+  ref_pyramid(p, img, pitch, pyr);
+  int64_t off = 0;
+  int total = 0;
+  counts[0] = 0;
+  for (int l = 0; l < p->n_levels; l++) {
+    int w = p->level_w[l], h = p->level_h[l];
+    const uint8_t* lev = pyr + off;
+    uint8_t* M = (uint8_t*)malloc((size_t)w * h);
+    ref_fast_M(lev, w, h, w, M);
+    int cap = w * h;
+    int32_t* cx = (int32_t*)malloc(sizeof(int32_t) * (size_t)cap * 3);
+    int32_t *cy = cx + cap, *cs = cx + 2 * cap;
+    int nc = ref_cell_candidates(p, l, M, cx, cy, cs, cap);
+    int32_t* kx = (int32_t*)malloc(sizeof(int32_t) * (size_t)(nc > 0 ? nc : 1) * 3);
+    int32_t *ky = kx + (nc > 0 ? nc : 1), *sel = kx + 2 * (nc > 0 ? nc : 1);
+    for (int i = 0; i < nc; i++) { kx[i] = cx[i] - MIN_BORDER; ky[i] = cy[i] - MIN_BORDER; }
+    int maxBX = w - EDGE_THRESHOLD + 3, maxBY = h - EDGE_THRESHOLD + 3;
+    int ns = ref_distribute(kx, ky, cs, nc, maxBX - MIN_BORDER, maxBY - MIN_BORDER,
+                            p->n_per_level[l], sel);
+    if (ns > p->level_cap[l] || total + ns > p->kp_capacity) { ns = -1; }
+    if (ns < 0) { free(kx); free(cx); free(M); free(pyr); return -1; }
+    selkp* s = (selkp*)malloc(sizeof(selkp) * (size_t)(ns > 0 ? ns : 1));
+    for (int i = 0; i < ns; i++) { s[i].lx = cx[sel[i]]; s[i].ly = cy[sel[i]]; s[i].score = cs[sel[i]]; }
+    qsort(s, (size_t)ns, sizeof(selkp), cmp_yx);
+    uint8_t* blur = (uint8_t*)malloc((size_t)w * h);
+    ref_blur(lev, w, h, w, blur, w);
+    for (int i = 0; i < ns; i++) {
+      ref_keypoint* k = &kps[total + i];
+      int32_t m10, m01;
+      ref_moments(lev, w, s[i].lx, s[i].ly, &m10, &m01);
+      k->x = (float)s[i].lx * p->scale[l];
+      k->y = (float)s[i].ly * p->scale[l];
+      k->angle_deg = ref_angle_deg(m10, m01);
+      k->lx = (uint16_t)s[i].lx; k->ly = (uint16_t)s[i].ly;
+      k->level = (uint8_t)l; k->response = (uint8_t)(s[i].score - 1);
+      k->reserved = 0;
+      ref_descriptor(blur, w, s[i].lx, s[i].ly, m10, m01, desc + (size_t)(total + i) * 32);
+    }
+    total += ns;
+    counts[l + 1] = total;
+    free(blur); free(s); free(kx); free(cx); free(M);
+    off += (int64_t)w * h;
+  }
+  free(pyr);
+  return total;
+}
+
+/* ---------------------------------------------------------------- O9 / O10 */
+int32_t ref_hamming(const uint8_t* a, const uint8_t* b) {
+  int d = 0;
+  for (int i = 0; i < 32; i++) {
+    uint8_t x = a[i] ^ b[i];
+    for (int j = 0; j < 8; j++) d += (x >> j) & 1;
+  }
+  return d;
+}
+
+/* ORB-SLAM SearchByProjection (local map points) [ext], the paper's "search local
+ * points": window + level gate + taken mask -> Hamming top-2 by (d, k) ->
+ * d <= th and (levels differ or den*d1 <= num*d2); dedup keeps min (d, q) (S8c O9). */
+void ref_match_window(const ref_params* p, int F, const ref_keypoint* kps, const uint8_t* desc,
+                      const int32_t* counts, const uint8_t* taken, int nq, const ref_query* q,
+                      const uint8_t* qdesc, int th, int num, int den, int dedup, ref_match* out) {
+  int L = p->n_levels, cap = p->kp_capacity;
+  for (int i = 0; i < nq; i++) {
+    int d1 = 256, d2 = 256, k1 = -1, k2 = -1;
+    int f = q[i].frame;
+    if (f >= 0 && f < F) {
+      int n = counts[f * (L + 1) + L];
+      for (int k = 0; k < n; k++) {
+        const ref_keypoint* kp = &kps[(size_t)f * cap + k];
+        if (kp->level < q[i].pred_level - 1 || kp->level > q[i].pred_level) continue;
+        if (taken && taken[(size_t)f * cap + k]) continue;
+        float dx = kp->x - q[i].u, dy = kp->y - q[i].v;
+        if (!(fabsf(dx) < q[i].radius && fabsf(dy) < q[i].radius)) continue;
+        int d = ref_hamming(qdesc + (size_t)i * 32, desc + ((size_t)f * cap + k) * 32);
+        /* keep the two smallest (d, k); k increases so ties keep the earlier k */
+        if (d < d1) { d2 = d1; k2 = k1; d1 = d; k1 = k; }
+        else if (d < d2) { d2 = d; k2 = k; }
+      }
+    }
+    int accept = 0;
+    if (k1 >= 0 && d1 <= th) {
+      int lev1 = kps[(size_t)f * cap + k1].level;
+      int lev2 = k2 >= 0 ? kps[(size_t)f * cap + k2].level : -1;
+      if (lev1 != lev2 || den * d1 <= num * d2) accept = 1;
+    }
+    out[i].idx = accept ? k1 : -1;
+    out[i].dist = d1;
+    out[i].dist2 = d2;
+  }
+  if (!dedup) return;
+  /* winner[f][k] = the claimant query with the smallest (dist, query index) */
+  int* winner = (int*)malloc(sizeof(int) * (size_t)(F > 0 ? F : 1) * (size_t)cap);
+  for (size_t t = 0; t < (size_t)F * cap; t++) winner[t] = -1;
+  for (int i = 0; i < nq; i++) {
+    if (out[i].idx < 0) continue;
+    size_t slot = (size_t)q[i].frame * cap + out[i].idx;
+    int w = winner[slot];
+    if (w < 0 || out[i].dist < out[w].dist || (out[i].dist == out[w].dist && i < w)) winner[slot] = i;
+  }
+  for (int i = 0; i < nq; i++) {
+    if (out[i].idx < 0) continue;
+    if (winner[(size_t)q[i].frame * cap + out[i].idx] != i) out[i].idx = -1;
+  }
+  free(winner);
+}
+
+/* Brute force keypoint -> map (ORB-SLAM relocalisation thresholds [ext], S8c O10):
+ * top-2 by (d, m); accept iff d1 <= th and den*d1 < num*d2. */
+void ref_match_brute(const ref_params* p, int F, const uint8_t* desc, const int32_t* counts, int n_map,
+                     const uint8_t* map_desc, int th, int num, int den, int k0, int k1,
+                     ref_match* out) {
+  int L = p->n_levels, cap = p->kp_capacity;
+  for (int f = 0; f < F; f++) {
+    int n = counts[f * (L + 1) + L];
+    for (int k = k0; k < k1 && k < cap; k++) {
+      ref_match* o = &out[(size_t)f * cap + k];
+      o->idx = -1; o->dist = 256; o->dist2 = 256;
+      if (k >= n) continue;
+      const uint8_t* a = desc + ((size_t)f * cap + k) * 32;
+      int d1 = 256, d2 = 256, m1 = -1;
+      for (int m = 0; m < n_map; m++) {
+        int d = ref_hamming(a, map_desc + (size_t)m * 32);
+        if (d < d1) { d2 = d1; d1 = d; m1 = m; }
+        else if (d < d2) { d2 = d; }
+      }
+      o->dist = d1; o->dist2 = d2;
+      if (m1 >= 0 && d1 <= th && den * d1 < num * d2) o->idx = m1;
+    }
+  }
+}

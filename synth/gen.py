@@ -1,0 +1,159 @@
+"""Synthetic textured frames and map-point queries (SURVEY.md §8(d) recipe).
+
+Frames: uniform base U(80,170) + bicubic-upsampled value noise (cells 96/24/6 px,
+amplitudes 40/30/20) + ~400*(W*H/360960) opaque convex polygons (radius U(5,40), 3-6
+vertices, gray U(30,225)) + two flat 100x80 patches (force the minTh fallback) +
+N(0,3) pixel noise, rounded and clipped.  Seeds: splitmix64(cfg<<40 | client<<20 | frame)
+into numpy PCG64.  KITTI right image = left warped by a piecewise-constant disparity
+field (0..48 px) + N(0,2).
+"""
+from __future__ import annotations
+
+import cv2
+import numpy as np
+
+SHAPES = {"euroc": (752, 480), "tum": (640, 480), "kitti": (1241, 376)}
+_MASK64 = (1 << 64) - 1
+
+
+def _splitmix64(x: int) -> int:
+    x = (x + 0x9E3779B97F4A7C15) & _MASK64
+    z = x
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & _MASK64
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & _MASK64
+    return z ^ (z >> 31)
+
+
+def frame_seed(cfg: int, client: int, frame: int) -> int:
+    return _splitmix64((cfg << 40) | (client << 20) | frame)
+
+
+def _rng(seed: int) -> np.random.Generator:
+    return np.random.Generator(np.random.PCG64(seed))
+
+
+def _value_noise(rng, w, h, cell, amp):
+    gw, gh = w // cell + 3, h // cell + 3
+    g = rng.uniform(-1.0, 1.0, size=(gh, gw)).astype(np.float32)
+    up = cv2.resize(g, (gw * cell, gh * cell), interpolation=cv2.INTER_CUBIC)
+    return amp * up[:h, :w]
+
+
+def make_frame(width: int, height: int, seed: int) -> np.ndarray:
+    rng = _rng(seed)
+    img = np.full((height, width), rng.uniform(80, 170), np.float32)
+    for cell, amp in ((96, 40.0), (24, 30.0), (6, 20.0)):
+        img += _value_noise(rng, width, height, cell, amp)
+    img = np.clip(img, 0, 255)
+    n_poly = int(round(400 * width * height / 360960.0))
+    for _ in range(n_poly):
+        cx, cy = rng.uniform(0, width), rng.uniform(0, height)
+        r = rng.uniform(5, 40)
+        nv = int(rng.integers(3, 7))
+        ang = np.sort(rng.uniform(0, 2 * np.pi, nv))
+        pts = np.stack([cx + r * np.cos(ang), cy + r * np.sin(ang)], 1).round().astype(np.int32)
+        cv2.fillPoly(img, [pts], float(rng.uniform(30, 225)))
+    for _ in range(2):
+        x0 = int(rng.integers(0, max(1, width - 100)))
+        y0 = int(rng.integers(0, max(1, height - 80)))
+        img[y0:y0 + 80, x0:x0 + 100] = rng.uniform(60, 200)
+    img += rng.normal(0.0, 3.0, size=img.shape).astype(np.float32)
+    return np.clip(np.rint(img), 0, 255).astype(np.uint8)
+
+
+def make_frames(width: int, height: int, n: int, cfg: int = 0, client0: int = 0, frame0: int = 0,
+                per_client: bool = True) -> np.ndarray:
+    """n frames: client c = client0 + i (per_client) or frame index frame0 + i."""
+    out = np.empty((n, height, width), np.uint8)
+    for i in range(n):
+        c, f = (client0 + i, frame0) if per_client else (client0, frame0 + i)
+        out[i] = make_frame(width, height, frame_seed(cfg, c, f))
+    return out
+
+
+def make_stereo_pair(width: int, height: int, seed: int):
+    left = make_frame(width, height, seed)
+    rng = _rng(seed ^ 0x5EED)
+    right = np.empty_like(left)
+    band = 0
+    while band < height:
+        bh = int(rng.integers(16, 64))
+        xs = 0
+        while xs < width:
+            bw = int(rng.integers(32, 160))
+            disp = int(rng.integers(0, 49))
+            x1 = min(width, xs + bw)
+            src = np.clip(np.arange(xs, x1) + disp, 0, width - 1)
+            right[band:band + bh, xs:x1] = left[band:band + bh][:, src]
+            xs = x1
+        band += bh
+    right = np.clip(np.rint(right + rng.normal(0, 2.0, size=right.shape)), 0, 255).astype(np.uint8)
+    return left, right
+
+
+def flip_bits(desc: np.ndarray, p: float, rng: np.random.Generator) -> np.ndarray:
+    bits = np.unpackbits(desc, axis=-1, bitorder="little")
+    mask = (rng.random(bits.shape) < p).astype(np.uint8)
+    return np.packbits(bits ^ mask, axis=-1, bitorder="little")
+
+
+def make_queries(kps: np.ndarray, desc: np.ndarray, counts: np.ndarray, n_levels: int,
+                 scale: np.ndarray, n_per_level: np.ndarray, width: int, height: int,
+                 n_queries_per_frame: int, th: float, seed: int, query_dtype, taken_frac=0.10,
+                 true_frac=0.60):
+    """Map-point queries for the windowed matcher, per frame.
+
+    kps [F,cap] (keypoint records: x, y, level), desc [F,cap,32], counts [F,L+1].
+    Returns (queries [F*Q] query_dtype, qdesc [F*Q,32] u8, taken [F,cap] u8)."""
+    rng = _rng(seed)
+    F, cap = kps.shape
+    Q = n_queries_per_frame
+    queries = np.zeros(F * Q, query_dtype)
+    qdesc = np.zeros((F * Q, 32), np.uint8)
+    taken = np.zeros((F, cap), np.uint8)
+    pl = np.asarray(n_per_level, np.float64)
+    pl = pl / pl.sum()
+    scale = np.asarray(scale, np.float32)
+    for f in range(F):
+        n = int(counts[f, n_levels])
+        base = f * Q
+        nt = min(int(true_frac * n), Q)
+        sel = rng.permutation(n)[:nt] if n else np.zeros(0, np.int64)
+        taken[f, :n] = rng.random(n) < taken_frac
+        q = queries[base:base + Q]
+        q["frame"] = f
+        if nt:
+            k = kps[f, sel]
+            q["u"][:nt] = k["x"] + rng.normal(0, 1.0, nt).astype(np.float32)
+            q["v"][:nt] = k["y"] + rng.normal(0, 1.0, nt).astype(np.float32)
+            lev = k["level"].astype(np.int32) + (rng.random(nt) >= 0.8)
+            q["pred_level"][:nt] = np.minimum(lev, n_levels - 1)
+            qdesc[base:base + nt] = flip_bits(desc[f, sel], 0.06, rng)
+        nd = Q - nt
+        q["u"][nt:] = rng.uniform(0, width, nd).astype(np.float32)
+        q["v"][nt:] = rng.uniform(0, height, nd).astype(np.float32)
+        q["pred_level"][nt:] = rng.choice(n_levels, size=nd, p=pl)
+        hard = rng.random(nd) < 0.5
+        rnd = rng.integers(0, 256, size=(nd, 32), dtype=np.uint8)
+        if n:
+            other = desc[f, rng.integers(0, n, nd)]
+            rnd[hard] = flip_bits(other[hard], 0.25, rng)
+        qdesc[base + nt:base + Q] = rnd
+        fac = np.where(rng.random(Q) < 0.5, 2.5, 4.0).astype(np.float32)
+        q["radius"] = np.float32(th) * fac * scale[q["pred_level"]]
+        perm = rng.permutation(Q)
+        queries[base:base + Q] = q[perm]
+        qdesc[base:base + Q] = qdesc[base:base + Q][perm]
+    return queries, qdesc, taken
+
+
+def make_brute_map(desc_list, n_map: int, seed: int, n_from_kps: int | None = None) -> np.ndarray:
+    """Shared-map descriptors: perturbed copies of client keypoint descriptors (p=0.06 flips)
+    plus uniform random descriptors, shuffled."""
+    rng = _rng(seed)
+    pool = np.concatenate([d for d in desc_list], 0) if desc_list else np.zeros((0, 32), np.uint8)
+    nk = min(len(pool), n_map if n_from_kps is None else n_from_kps)
+    part = flip_bits(pool[rng.permutation(len(pool))[:nk]], 0.06, rng) if nk else np.zeros((0, 32), np.uint8)
+    rnd = rng.integers(0, 256, size=(n_map - nk, 32), dtype=np.uint8)
+    m = np.concatenate([part, rnd], 0)
+    return np.ascontiguousarray(m[rng.permutation(n_map)])
