@@ -1,0 +1,171 @@
+/*
+ * ss.h -- C ABI of libss: batched ORB extraction + tracking-time descriptor matching on
+ * B200 (sm_100a), the data-parallel hot path of SLAM-Share's GPU tracking
+ * (Dhakal et al., CoNEXT'22): "the parallelization of FAST corner detection ... with the
+ * GPU" (§4.2.1) and the "local tracking CUDA kernel" that parallelises
+ * search-local-points (L168), run for many clients at once ("spatio-temporal sharing of
+ * the GPU ... on the data received from multiple client updates", L170).
+ *
+ * The paper fixes no arithmetic; each entry point cites the DESIGN.md §3 reading
+ * (= SURVEY.md §8(c) row O0..O10) that defines it.
+ *
+ * Conventions
+ *  - Every function returns ss_status; nothing aborts or throws across the ABI.
+ *  - "device pointer" = CUDA global memory of the ctx's device; "host pointer" = CPU memory.
+ *  - Calls taking a stream only ENQUEUE work on it (no host synchronisation, no allocation);
+ *    outputs are valid once the stream reaches the call.  Inputs must stay valid until then.
+ *  - The caller owns every input/output buffer; an ss_ctx owns only its scratch, sized at
+ *    ss_create.  One ctx may be used by one host thread / stream at a time.
+ *  - Argument and capacity errors are detected synchronously (SS_EINVAL / SS_ECAPACITY),
+ *    before anything is enqueued.  SS_ECUDA = a CUDA API or launch error (message in
+ *    ss_last_error).  Kernels never write outside the documented output extents.
+ */
+#ifndef SS_H
+#define SS_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  SS_OK = 0,
+  SS_EINVAL = -1,       /* bad argument / shape / params mismatch                       */
+  SS_ECAPACITY = -2,    /* more frames / queries / map entries than the ctx was sized for */
+  SS_ECUDA = -3,        /* CUDA runtime or launch error                                   */
+  SS_EUNSUPPORTED = -4  /* valid request this build does not implement                   */
+} ss_status;
+
+typedef struct ss_ctx ss_ctx; /* opaque */
+typedef void* ss_stream_t;    /* a cudaStream_t (NULL = legacy default stream) */
+
+#define SS_MAX_LEVELS 8
+#define SS_DESC_BYTES 32
+
+/* ORB parameters (DESIGN.md §3 O0).  Fill with ss_orb_params_init, then treat read-only:
+ * scale[l] = f32(scale[l-1]*scale_factor); inv_scale[l] = f32(1/scale[l]);
+ * level_w/h[l] = rne(f32(W*inv_scale[l])); n_per_level = ORB-SLAM's geometric split of
+ * n_features; cells = 30-px FAST grid of each level (cols, rows, cell w, cell h);
+ * n_ini = quadtree root count; level_cap[l] = max(n_per_level[l]+2, 4*n_ini[l]) = the most
+ * keypoints the distribution can keep on level l; kp_capacity = sum of level_cap. */
+typedef struct {
+  int32_t width, height, n_features, n_levels;
+  float scale_factor;
+  int32_t ini_th_fast, min_th_fast;
+  float scale[SS_MAX_LEVELS], inv_scale[SS_MAX_LEVELS];
+  int32_t level_w[SS_MAX_LEVELS], level_h[SS_MAX_LEVELS], n_per_level[SS_MAX_LEVELS];
+  int32_t cell_cols[SS_MAX_LEVELS], cell_rows[SS_MAX_LEVELS];
+  int32_t cell_w[SS_MAX_LEVELS], cell_h[SS_MAX_LEVELS];
+  int32_t n_ini[SS_MAX_LEVELS];
+  int32_t level_cap[SS_MAX_LEVELS];
+  int32_t kp_capacity;
+} ss_orb_params;
+
+/* One ORB keypoint, 20 bytes.  Per frame, keypoints are in canonical order
+ * (level, ly, lx) (DESIGN.md §3 O8). */
+typedef struct {
+  float x, y;            /* level-0 coordinates: f32(lx) * scale[level] (one f32 multiply)   */
+  float angle_deg;       /* intensity-centroid angle atan2(m01, m10) in [0, 360) (O5)        */
+  uint16_t lx, ly;       /* integer pixel on its pyramid level                              */
+  uint8_t level;         /* pyramid level                                                   */
+  uint8_t response;      /* FAST score = M - 1 (O2)                                         */
+  uint16_t reserved;     /* 0                                                               */
+} ss_keypoint;
+
+/* A local-map point projected into a frame (the caller's frustum test, ORB-SLAM
+ * isInFrustum): frame index, predicted position (level-0 px), predicted level, window
+ * half-size r (level-0 px).  20 bytes. */
+typedef struct {
+  int32_t frame;
+  float u, v;
+  int32_t pred_level;
+  float radius;
+} ss_mp_query;
+
+/* A match: idx = keypoint index within its frame (WINDOW) or map index (BRUTE), -1 = none;
+ * dist / dist2 = best / second-best Hamming distance over the candidates (256 = none). */
+typedef struct {
+  int32_t idx;
+  int32_t dist;
+  int32_t dist2;
+} ss_match;
+
+#define SS_MATCH_WINDOW 0 /* one result per query: search local points (O9)       */
+#define SS_MATCH_BRUTE 1  /* one result per frame keypoint vs the whole map (O10) */
+
+typedef struct {
+  int32_t mode;      /* SS_MATCH_WINDOW or SS_MATCH_BRUTE                                       */
+  int32_t th;        /* accept only d1 <= th (WINDOW: ORB-SLAM TH_HIGH 100; BRUTE: TH_LOW 50)   */
+  int32_t ratio_num; /* ratio = num/den; WINDOW: den*d1 <= num*d2 unless the two best lie on   */
+  int32_t ratio_den; /*   different levels (4/5); BRUTE: den*d1 < num*d2 (3/4)                  */
+  int32_t dedup;     /* WINDOW: 1 = a keypoint claimed by several queries keeps min (d, query)  */
+} ss_match_cfg;
+
+/* O0.  Validates 64 <= w,h <= 2048, 1 <= n_levels <= 8, scale_factor > 1, 1 <= thresholds
+ * <= 254, every level >= 30 px of FAST grid in each direction and 1 <= n_ini <= 62.
+ * Host only; never touches the GPU.  Returns SS_EINVAL (out untouched) on rejection. */
+ss_status ss_orb_params_init(int32_t width, int32_t height, int32_t n_features, int32_t n_levels,
+                             float scale_factor, int32_t ini_th_fast, int32_t min_th_fast,
+                             ss_orb_params* out);
+
+/* Create a context on `device` for frames of shape p (p must equal what
+ * ss_orb_params_init returns for its own first seven fields, else SS_EINVAL).
+ * max_frames bounds n_frames per call, max_queries the WINDOW query count and max_map the
+ * BRUTE map size (0 = that mode unused).  Allocates all scratch here (none per call). */
+ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, int32_t max_queries,
+                    int32_t max_map, ss_ctx** out);
+ss_status ss_destroy(ss_ctx* ctx);
+
+/* Message of the last failing call on this host thread (ctx may be NULL).  Never NULL. */
+const char* ss_last_error(const ss_ctx* ctx);
+
+/* O1..O8 for n_frames frames of the ctx's shape (FAST on the GPU; the rest
+ * of ORB, L87, on the GPU as well).  Device pointers:
+ *   d_frames : u8 gray frames, frame f row y at d_frames + f*frame_stride + y*pitch
+ *              (pitch >= width, frame_stride >= height*pitch)
+ *   d_kps    : [n_frames][kp_capacity] ss_keypoint      (slots >= count are left untouched)
+ *   d_desc   : [n_frames][kp_capacity][32] u8, bit b of byte i = comparison 8i+b   (O7)
+ *   d_counts : [n_frames][n_levels+1] i32 prefix offsets: level l is [counts[l], counts[l+1])
+ * Bit-exact with the oracle except angle_deg (|err| <= 1e-4 rad).  Deterministic. */
+ss_status ss_orb_extract(ss_ctx* ctx, int32_t n_frames, const uint8_t* d_frames, int64_t frame_stride,
+                         int32_t pitch, ss_keypoint* d_kps, uint8_t* d_desc, int32_t* d_counts,
+                         ss_stream_t stream);
+
+/* O9 / O10 on the outputs of ss_orb_extract (same layouts).  Device pointers:
+ * WINDOW ("search local points"):
+ *   d_kp_taken [n_frames][kp_capacity] u8 (non-zero = keypoint already matched; may be NULL),
+ *   d_queries [n_queries], d_map_desc [n_queries][32] (the map points' descriptors),
+ *   d_out [n_queries]: candidates = keypoints of frame q.frame with level in
+ *   [pred_level-1, pred_level], |x-u| < r and |y-v| < r (f32), not taken; top-2 by
+ *   (distance, index); accepted as in ss_match_cfg; queries with an out-of-range frame
+ *   get {-1, 256, 256}.
+ * BRUTE: d_kp_taken and d_queries ignored (n_queries must be 0); d_map_desc [n_map][32];
+ *   d_out [n_frames][kp_capacity]: per keypoint, top-2 over the map by (distance, index);
+ *   slots >= the frame's count get {-1, 256, 256}. */
+ss_status ss_match_projection(ss_ctx* ctx, int32_t n_frames, const ss_keypoint* d_kps,
+                              const uint8_t* d_desc, const int32_t* d_counts,
+                              const uint8_t* d_kp_taken, int32_t n_queries,
+                              const ss_mp_query* d_queries, const uint8_t* d_map_desc, int32_t n_map,
+                              const ss_match_cfg* cfg, ss_match* d_out, ss_stream_t stream);
+
+/* ---- debug / test hooks (synchronise the ctx's device; not for the hot path) ---- */
+
+/* Device pointer + pitch of pyramid level `level` (>= 1) of frame slot `frame` as left by the
+ * last ss_orb_extract (level 0 is the caller's frame). */
+ss_status ss_debug_level(ss_ctx* ctx, int32_t frame, int32_t level, const uint8_t** d_ptr,
+                         int32_t* pitch);
+
+/* FAST candidates (O3) of (frame, level) from the last ss_orb_extract, in rank order
+ * (cells row-major, then y, then x), copied to host arrays of capacity `cap`
+ * (h_lx, h_ly: pixel; h_score: M).  *n = count; SS_ECAPACITY if count > cap. */
+ss_status ss_debug_candidates(ss_ctx* ctx, int32_t frame, int32_t level, int32_t* h_lx, int32_t* h_ly,
+                              int32_t* h_score, int32_t cap, int32_t* n);
+
+/* Number of (frame, level) distributions of the last ss_orb_extract that exceeded the
+ * in-shared-memory capacity and took the global-memory path (for tests/benchmarks). */
+ss_status ss_debug_overflow_count(ss_ctx* ctx, int32_t* n);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SS_H */

@@ -1,0 +1,192 @@
+// k_describe.cu -- S5+S6+S7+S8: orientation, 7x7 blur, rotated BRIEF and output packing
+// (DESIGN.md §3 O5-O8; "Oriented FAST and Rotated BRIEF").
+//
+// One warp per output keypoint slot.  The warp stages the 43x43 raw patch around the
+// keypoint (REFLECT_101 at the level border, which the blur needs) in shared memory and
+// derives everything from it: intensity-centroid moments over the 749-px disk (unblurred),
+// the 37x37 blurred patch (Q8 taps [18,34,48,56,48,34,18], exact horizontal sums, vertical
+// (sum + 2^15) >> 16), and the 256 comparisons at the pattern points rotated by
+// (cos, sin) = (m10, m01)/sqrt(m10^2 + m01^2), each offset rounded half-to-even EXACTLY
+// (float estimate + int64 fix-up).  Blurring only the patch replaces a whole-level blur
+// pass and its HBM round trip.  Output position = the keypoint's canonical index, so the
+// per-level counts of the distribution become the prefix offsets written to d_counts.
+#include "brief_pattern.inc"
+#include "ss_internal.h"
+
+namespace ss {
+
+namespace {
+
+constexpr int DESC_WARPS = 8;
+constexpr int PR = 43;  // raw patch: radius 21 (18 max sample offset + 3 blur taps)
+constexpr int PP = 44;
+constexpr int BR = 37;  // blurred patch: radius 18
+constexpr int HP = 37;  // pitch (u16) of the horizontal pass [43][37]
+constexpr int BP = 40;
+constexpr int PER_WARP = ((PR * PP + PR * HP * 2 + BR * BP) + 127) & ~127;
+
+__constant__ int c_umax[16] = {15, 15, 15, 15, 14, 14, 14, 13, 13, 12, 11, 10, 9, 8, 6, 3};
+
+__device__ __forceinline__ int reflect101(int i, int n) {
+  i = i < 0 ? -i : i;
+  return i >= n ? 2 * n - 2 - i : i;
+}
+
+// Exact round-half-even of z / sqrt(r2), r2 > 0: float estimate, then the integer test
+// (2k-1)^2 r2 < 4 z^2 <= (2k+1)^2 r2 selects k; a tie 4z^2 == (2k+1)^2 r2 goes to even.
+__device__ __forceinline__ int rhe_div_sqrt(long long z, long long r2, float inv_r) {
+  const long long a = z < 0 ? -z : z;
+  const long long A = 4 * a * a;
+  int k = __float2int_rn((float)a * inv_r);
+  while (k > 0 && (long long)(2 * k - 1) * (2 * k - 1) * r2 >= A) k--;
+  while ((long long)(2 * k + 1) * (2 * k + 1) * r2 < A) k++;
+  if ((k & 1) && (long long)(2 * k + 1) * (2 * k + 1) * r2 == A) k++;
+  return z < 0 ? -k : k;
+}
+
+__global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, FrameSrc src,
+                                                                   const uint32_t* __restrict__ selected,
+                                                                   const int32_t* __restrict__ sel_counts,
+                                                                   const int8_t* __restrict__ pattern,
+                                                                   ss_keypoint* __restrict__ kps,
+                                                                   uint8_t* __restrict__ desc,
+                                                                   int32_t* __restrict__ counts) {
+  extern __shared__ __align__(16) uint8_t sm[];  // DESC_WARPS * PER_WARP
+  __shared__ int8_t pat[1024];
+  __shared__ int off[kMaxLevels + 1];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int f = blockIdx.y;
+  const int L = g.L;
+  for (int i = threadIdx.x; i < 1024; i += blockDim.x) pat[i] = pattern[i];
+  if (threadIdx.x == 0) {
+    int s = 0;
+    off[0] = 0;
+    for (int l = 0; l < L; l++) {
+      s += sel_counts[f * L + l];
+      off[l + 1] = s;
+    }
+  }
+  __syncthreads();
+  if (blockIdx.x == 0 && threadIdx.x <= L) counts[f * (L + 1) + threadIdx.x] = off[threadIdx.x];
+  const int i = blockIdx.x * DESC_WARPS + warp;
+  if (i >= off[L]) return;  // warp-uniform; only warp-level sync below
+  int l = 0;
+  while (i >= off[l + 1]) l++;
+  const uint32_t packed = selected[(int64_t)f * g.kp_capacity + g.cap_off[l] + (i - off[l])];
+  const int lx = key_lx(packed), ly = key_ly(packed), M = key_m(packed);
+  const uint8_t* img;
+  int ip;
+  if (l == 0) {
+    img = src.frames + (int64_t)f * src.stride;
+    ip = src.pitch;
+  } else {
+    img = src.pyr + (int64_t)f * g.pyr_frame_bytes + g.lvl_off[l];
+    ip = g.pitch[l];
+  }
+  const int w = g.w[l], h = g.h[l];
+  uint8_t* P = sm + warp * PER_WARP;
+  uint16_t* Hs = reinterpret_cast<uint16_t*>(P + PR * PP);
+  uint8_t* B = reinterpret_cast<uint8_t*>(Hs + PR * HP);
+  // raw patch, REFLECT_101 outside the level
+  for (int r = 0; r < PR; r++) {
+    const uint8_t* row = img + (int64_t)reflect101(ly - 21 + r, h) * ip;
+    for (int c = lane; c < PR; c += 32) P[r * PP + c] = __ldg(row + reflect101(lx - 21 + c, w));
+  }
+  __syncwarp();
+  // moments over the disk |u| <= umax[|v|] (always inside the level: 19 <= lx < w-19)
+  int m10 = 0, m01 = 0;
+  {
+    const int u = lane - 15;
+    if (lane < 31) {
+      for (int v = -15; v <= 15; v++) {
+        const int um = c_umax[v < 0 ? -v : v];
+        if (u >= -um && u <= um) {
+          const int I = P[(21 + v) * PP + 21 + u];
+          m10 += u * I;
+          m01 += v * I;
+        }
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      m10 += __shfl_xor_sync(0xFFFFFFFFu, m10, o);
+      m01 += __shfl_xor_sync(0xFFFFFFFFu, m01, o);
+    }
+  }
+  // horizontal blur pass: Hs[r][c] = sum_j k_j P[r][c + j], c in [0, 37)
+  for (int idx = lane; idx < PR * BR; idx += 32) {
+    const int r = idx / BR, c = idx - r * BR;
+    const uint8_t* p = P + r * PP + c;
+    Hs[r * HP + c] = (uint16_t)(18 * (p[0] + p[6]) + 34 * (p[1] + p[5]) + 48 * (p[2] + p[4]) + 56 * p[3]);
+  }
+  __syncwarp();
+  for (int idx = lane; idx < BR * BR; idx += 32) {
+    const int r = idx / BR, c = idx - r * BR;
+    const uint16_t* p = Hs + r * HP + c;
+    const int s = 18 * ((int)p[0] + p[6 * HP]) + 34 * ((int)p[HP] + p[5 * HP]) + 48 * ((int)p[2 * HP] + p[4 * HP]) +
+                  56 * (int)p[3 * HP];
+    B[r * BP + c] = (uint8_t)((s + (1 << 15)) >> 16);
+  }
+  __syncwarp();
+  // rotated BRIEF: lane = output byte; bit t compares points 2b, 2b+1 with b = 8*lane + t
+  const long long r2 = (long long)m10 * m10 + (long long)m01 * m01;
+  const float inv_r = r2 ? rsqrtf((float)r2) : 0.f;
+  uint32_t byte = 0;
+#pragma unroll 2
+  for (int t = 0; t < 8; t++) {
+    const int b = lane * 8 + t;
+    int v[2];
+#pragma unroll
+    for (int e = 0; e < 2; e++) {
+      const int px = pat[4 * b + 2 * e], py = pat[4 * b + 2 * e + 1];
+      int ox = px, oy = py;
+      if (r2) {
+        ox = rhe_div_sqrt((long long)px * m10 - (long long)py * m01, r2, inv_r);
+        oy = rhe_div_sqrt((long long)px * m01 + (long long)py * m10, r2, inv_r);
+      }
+      v[e] = B[(18 + oy) * BP + 18 + ox];
+    }
+    byte |= (uint32_t)(v[0] < v[1]) << t;
+  }
+  const int64_t o = (int64_t)f * g.kp_capacity + i;
+  desc[o * SS_DESC_BYTES + lane] = (uint8_t)byte;
+  if (lane == 0) {
+    float ang = 0.f;
+    if (m10 != 0 || m01 != 0) {
+      double a = atan2((double)m01, (double)m10) * (180.0 / 3.14159265358979323846);
+      if (a < 0) a += 360.0;
+      ang = (float)a;
+      if (ang >= 360.0f) ang = 0.0f;
+    }
+    ss_keypoint kp;
+    kp.x = __fmul_rn((float)lx, g.scale[l]);
+    kp.y = __fmul_rn((float)ly, g.scale[l]);
+    kp.angle_deg = ang;
+    kp.lx = (uint16_t)lx;
+    kp.ly = (uint16_t)ly;
+    kp.level = (uint8_t)l;
+    kp.response = (uint8_t)(M - 1);
+    kp.reserved = 0;
+    kps[o] = kp;
+  }
+}
+
+}  // namespace
+
+const int* brief_pattern_host() { return SS_BRIEF_PATTERN_HOST; }
+
+cudaError_t launch_describe(const Geom& g, int n_frames, FrameSrc src, const uint32_t* selected,
+                            const int32_t* sel_counts, const int8_t* pattern, ss_keypoint* kps, uint8_t* desc,
+                            int32_t* counts, cudaStream_t s) {
+  const size_t smem = (size_t)DESC_WARPS * PER_WARP;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaFuncSetAttribute(describe_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    attr_set = true;
+  }
+  dim3 grid((g.kp_capacity + DESC_WARPS - 1) / DESC_WARPS, n_frames);
+  describe_kernel<<<grid, DESC_WARPS * 32, smem, s>>>(g, src, selected, sel_counts, pattern, kps, desc, counts);
+  return cudaGetLastError();
+}
+
+}  // namespace ss

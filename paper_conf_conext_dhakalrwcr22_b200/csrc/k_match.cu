@@ -1,0 +1,218 @@
+// k_match.cu -- S9 windowed matcher ("search local points") and S10
+// brute-force matcher (DESIGN.md §3 O9, O10).
+//
+// WINDOW: one thread per map-point query.  Keypoints are in canonical (level, ly, lx)
+// order, so on each level of the gate [l-1, l] the rows with |y - v| < r (f32) form one
+// contiguous run found by two binary searches on the exact predicate; the run is scanned
+// with the exact |x - u| < r test, the taken mask, and a 256-bit Hamming distance
+// (8 x POPC over 2 x 16-byte loads).  Top-2 by (distance, index) with strict updates in
+// increasing index order; ORB-SLAM's accept rule; a keypoint claimed by several accepted
+// queries keeps the min (distance, query) (atomicMin on packed u64, then a resolve pass).
+// BRUTE: map tiles staged in shared memory, one thread per frame keypoint keeps a packed
+// (distance << 32 | map index) top-2 per map split; a merge kernel takes the two smallest.
+#include "ss_internal.h"
+
+namespace ss {
+
+namespace {
+
+__device__ __forceinline__ int hamming256(const uint4 a0, const uint4 a1, const uint4 b0, const uint4 b1) {
+  return __popc(a0.x ^ b0.x) + __popc(a0.y ^ b0.y) + __popc(a0.z ^ b0.z) + __popc(a0.w ^ b0.w) +
+         __popc(a1.x ^ b1.x) + __popc(a1.y ^ b1.y) + __popc(a1.z ^ b1.z) + __popc(a1.w ^ b1.w);
+}
+
+__global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const ss_keypoint* __restrict__ kps,
+                                                           const uint8_t* __restrict__ desc,
+                                                           const int32_t* __restrict__ counts,
+                                                           const uint8_t* __restrict__ taken, int nq,
+                                                           const ss_mp_query* __restrict__ q,
+                                                           const uint8_t* __restrict__ qdesc, ss_match_cfg cfg,
+                                                           unsigned long long* __restrict__ claim,
+                                                           ss_match* __restrict__ out) {
+  const int qi = blockIdx.x * blockDim.x + threadIdx.x;
+  if (qi >= nq) return;
+  const ss_mp_query Q = q[qi];
+  const int L = g.L, cap = g.kp_capacity;
+  int d1 = 256, d2 = 256, k1 = -1, k2 = -1;
+  const int f = Q.frame;
+  if (f >= 0 && f < F) {
+    const uint4* qd = reinterpret_cast<const uint4*>(qdesc + (int64_t)qi * SS_DESC_BYTES);
+    const uint4 qa = qd[0], qb = qd[1];
+    const int32_t* cnt = counts + f * (L + 1);
+    const ss_keypoint* fk = kps + (int64_t)f * cap;
+    const uint4* fd = reinterpret_cast<const uint4*>(desc + (int64_t)f * cap * SS_DESC_BYTES);
+    const uint8_t* ft = taken ? taken + (int64_t)f * cap : nullptr;
+    const float r = Q.radius, nr = -Q.radius;
+    const int l0 = max(Q.pred_level - 1, 0), l1 = min(Q.pred_level, L - 1);
+    for (int l = l0; l <= l1; l++) {
+      int lo = cnt[l], hi = cnt[l + 1];
+      // first k with (y_k - v) > -r
+      int a = lo, b = hi;
+      while (a < b) {
+        const int m = (a + b) >> 1;
+        if (__fsub_rn(fk[m].y, Q.v) > nr) b = m; else a = m + 1;
+      }
+      const int kb = a;
+      a = kb;
+      b = hi;
+      // first k with (y_k - v) >= r
+      while (a < b) {
+        const int m = (a + b) >> 1;
+        if (__fsub_rn(fk[m].y, Q.v) >= r) b = m; else a = m + 1;
+      }
+      const int ke = a;
+      for (int k = kb; k < ke; k++) {
+        const float dx = __fsub_rn(fk[k].x, Q.u);
+        if (!(fabsf(dx) < r)) continue;
+        if (ft && ft[k]) continue;
+        const int d = hamming256(qa, qb, fd[2 * k], fd[2 * k + 1]);
+        if (d < d1) {
+          d2 = d1; k2 = k1; d1 = d; k1 = k;
+        } else if (d < d2) {
+          d2 = d; k2 = k;
+        }
+      }
+    }
+  }
+  bool accept = false;
+  if (k1 >= 0 && d1 <= cfg.th) {
+    const int lev1 = kps[(int64_t)f * cap + k1].level;
+    const int lev2 = k2 >= 0 ? (int)kps[(int64_t)f * cap + k2].level : -1;
+    accept = (lev1 != lev2) || (cfg.ratio_den * d1 <= cfg.ratio_num * d2);
+  }
+  ss_match m;
+  m.idx = accept ? k1 : -1;
+  m.dist = d1;
+  m.dist2 = d2;
+  out[qi] = m;
+  if (accept && cfg.dedup)
+    atomicMin(claim + (int64_t)f * cap + k1, ((unsigned long long)d1 << 32) | (unsigned)qi);
+}
+
+__global__ void __launch_bounds__(256) match_window_resolve(int nq, const ss_mp_query* __restrict__ q, int cap,
+                                                            const unsigned long long* __restrict__ claim,
+                                                            ss_match* __restrict__ out) {
+  const int qi = blockIdx.x * blockDim.x + threadIdx.x;
+  if (qi >= nq) return;
+  const ss_match m = out[qi];
+  if (m.idx < 0) return;
+  const unsigned long long mine = ((unsigned long long)m.dist << 32) | (unsigned)qi;
+  if (claim[(int64_t)q[qi].frame * cap + m.idx] != mine) out[qi].idx = -1;
+}
+
+constexpr int BQ = 128;    // keypoints per CTA (one per thread)
+constexpr int BTILE = 256;  // map descriptors per shared-memory tile
+
+__global__ void __launch_bounds__(BQ) match_brute_partial(Geom g, int F, const uint8_t* __restrict__ desc,
+                                                          const int32_t* __restrict__ counts, int n_map,
+                                                          const uint8_t* __restrict__ map_desc, int splits,
+                                                          unsigned long long* __restrict__ partial) {
+  __shared__ uint4 tile[BTILE * 2];
+  const int cap = g.kp_capacity, L = g.L;
+  const int gq = blockIdx.x * BQ + threadIdx.x;  // global keypoint slot f*cap + k
+  const int split = blockIdx.y;
+  const int per = (n_map + splits - 1) / splits;
+  const int m0 = split * per, m1 = min(n_map, m0 + per);
+  bool valid = false;
+  uint4 a0 = make_uint4(0, 0, 0, 0), a1 = a0;
+  if (gq < F * cap) {
+    const int f = gq / cap, k = gq - f * cap;
+    valid = k < counts[f * (L + 1) + L];
+    if (valid) {
+      const uint4* p = reinterpret_cast<const uint4*>(desc + (int64_t)gq * SS_DESC_BYTES);
+      a0 = p[0];
+      a1 = p[1];
+    }
+  }
+  unsigned long long b1 = ~0ull, b2 = ~0ull;
+  for (int t0 = m0; t0 < m1; t0 += BTILE) {
+    const int nt = min(BTILE, m1 - t0);
+    __syncthreads();
+    const uint4* src = reinterpret_cast<const uint4*>(map_desc + (int64_t)t0 * SS_DESC_BYTES);
+    for (int i = threadIdx.x; i < nt * 2; i += BQ) tile[i] = src[i];
+    __syncthreads();
+    if (valid) {
+      for (int j = 0; j < nt; j++) {
+        const int d = hamming256(a0, a1, tile[2 * j], tile[2 * j + 1]);
+        const unsigned long long key = ((unsigned long long)d << 32) | (unsigned)(t0 + j);
+        if (key < b1) {
+          b2 = b1;
+          b1 = key;
+        } else if (key < b2) {
+          b2 = key;
+        }
+      }
+    }
+  }
+  if (gq < F * cap) {
+    partial[((int64_t)gq * splits + split) * 2] = b1;
+    partial[((int64_t)gq * splits + split) * 2 + 1] = b2;
+  }
+}
+
+__global__ void __launch_bounds__(256) match_brute_merge(Geom g, int F, const int32_t* __restrict__ counts,
+                                                         int splits, const unsigned long long* __restrict__ partial,
+                                                         ss_match_cfg cfg, ss_match* __restrict__ out) {
+  const int gq = blockIdx.x * blockDim.x + threadIdx.x;
+  const int cap = g.kp_capacity, L = g.L;
+  if (gq >= F * cap) return;
+  const int f = gq / cap, k = gq - f * cap;
+  ss_match m;
+  m.idx = -1;
+  m.dist = 256;
+  m.dist2 = 256;
+  if (k < counts[f * (L + 1) + L]) {
+    unsigned long long b1 = ~0ull, b2 = ~0ull;
+    for (int s = 0; s < splits * 2; s++) {
+      const unsigned long long key = partial[(int64_t)gq * splits * 2 + s];
+      if (key < b1) {
+        b2 = b1;
+        b1 = key;
+      } else if (key < b2) {
+        b2 = key;
+      }
+    }
+    const int d1 = b1 == ~0ull ? 256 : (int)(b1 >> 32);
+    const int d2 = b2 == ~0ull ? 256 : (int)(b2 >> 32);
+    m.dist = d1;
+    m.dist2 = d2;
+    if (b1 != ~0ull && d1 <= cfg.th && cfg.ratio_den * d1 < cfg.ratio_num * d2) m.idx = (int)(b1 & 0xFFFFFFFFu);
+  }
+  out[gq] = m;
+}
+
+}  // namespace
+
+cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* kps, const uint8_t* desc,
+                                const int32_t* counts, const uint8_t* taken, int n_queries, const ss_mp_query* q,
+                                const uint8_t* qdesc, ss_match_cfg cfg, unsigned long long* claim, ss_match* out,
+                                cudaStream_t s) {
+  if (n_queries <= 0) return cudaSuccess;
+  if (cfg.dedup) {
+    cudaError_t e = cudaMemsetAsync(claim, 0xFF, (size_t)n_frames * g.kp_capacity * sizeof(unsigned long long), s);
+    if (e != cudaSuccess) return e;
+  }
+  const int blocks = (n_queries + 255) / 256;
+  match_window_kernel<<<blocks, 256, 0, s>>>(g, n_frames, kps, desc, counts, taken, n_queries, q, qdesc, cfg, claim,
+                                             out);
+  if (cfg.dedup) match_window_resolve<<<blocks, 256, 0, s>>>(n_queries, q, g.kp_capacity, claim, out);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_match_brute(const Geom& g, int n_frames, const uint8_t* desc, const int32_t* counts, int n_map,
+                               const uint8_t* map_desc, ss_match_cfg cfg, unsigned long long* partial, int max_splits,
+                               ss_match* out, cudaStream_t s) {
+  const int nslots = n_frames * g.kp_capacity;
+  if (nslots <= 0) return cudaSuccess;
+  const int qblocks = (nslots + BQ - 1) / BQ;
+  // enough CTAs for ~4 waves on 148 SMs, each split >= one tile
+  int splits = (4 * 148 + qblocks - 1) / qblocks;
+  splits = max(1, min(splits, max_splits));
+  splits = max(1, min(splits, (n_map + BTILE - 1) / BTILE));
+  dim3 grid(qblocks, splits);
+  match_brute_partial<<<grid, BQ, 0, s>>>(g, n_frames, desc, counts, n_map, map_desc, splits, partial);
+  match_brute_merge<<<(nslots + 255) / 256, 256, 0, s>>>(g, n_frames, counts, splits, partial, cfg, out);
+  return cudaGetLastError();
+}
+
+}  // namespace ss

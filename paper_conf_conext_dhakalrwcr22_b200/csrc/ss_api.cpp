@@ -1,0 +1,440 @@
+// ss_api.cpp -- host side of libss: parameter derivation, validation, scratch ownership and
+// the launch sequence of each C-ABI entry point (include/ss.h).  No per-call allocation,
+// no host synchronisation on the hot path; every entry point returns a status.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "ss_internal.h"
+
+using namespace ss;
+
+namespace {
+
+thread_local std::string g_err = "no error";
+
+ss_status fail(ss_status st, const std::string& msg) {
+  g_err = msg;
+  return st;
+}
+
+#define SS_CUDA_TRY(expr)                                                                    \
+  do {                                                                                       \
+    cudaError_t _e = (expr);                                                                 \
+    if (_e != cudaSuccess) return fail(SS_ECUDA, std::string(#expr) + ": " + cudaGetErrorString(_e)); \
+  } while (0)
+
+int imax(int a, int b) { return a > b ? a : b; }
+int imin(int a, int b) { return a < b ? a : b; }
+
+// O0: ORB-SLAM's ORBextractor constructor quantities in f32 (see ss.h).
+ss_status params_init(int32_t W, int32_t H, int32_t nf, int32_t L, float sf, int32_t ini, int32_t mn,
+                      ss_orb_params* p) {
+  if (L < 1 || L > SS_MAX_LEVELS) return fail(SS_EINVAL, "n_levels must be in [1, 8]");
+  if (W < 64 || H < 64 || W > 2048 || H > 2048) return fail(SS_EINVAL, "width/height must be in [64, 2048]");
+  if (nf < 1) return fail(SS_EINVAL, "n_features must be >= 1");
+  if (!(sf > 1.0f)) return fail(SS_EINVAL, "scale_factor must be > 1");
+  if (ini < 1 || mn < 1 || ini > 254 || mn > 254) return fail(SS_EINVAL, "FAST thresholds must be in [1, 254]");
+  ss_orb_params q;
+  std::memset(&q, 0, sizeof(q));
+  q.width = W;
+  q.height = H;
+  q.n_features = nf;
+  q.n_levels = L;
+  q.scale_factor = sf;
+  q.ini_th_fast = ini;
+  q.min_th_fast = mn;
+  volatile float s = 1.0f;  // keep every product a separate f32 rounding
+  q.scale[0] = 1.0f;
+  for (int l = 1; l < L; l++) {
+    s = s * sf;
+    q.scale[l] = s;
+  }
+  for (int l = 0; l < L; l++) {
+    volatile float inv = 1.0f / q.scale[l];
+    q.inv_scale[l] = inv;
+    volatile float fw = (float)W * q.inv_scale[l];
+    volatile float fh = (float)H * q.inv_scale[l];
+    q.level_w[l] = (int32_t)std::nearbyint((float)fw);  // round half even (default mode)
+    q.level_h[l] = (int32_t)std::nearbyint((float)fh);
+  }
+  const float factor = 1.0f / sf;
+  volatile float num = (float)nf * (1.0f - factor);
+  volatile float den = 1.0f - (float)std::pow((double)factor, (double)L);
+  volatile float per = num / den;
+  int sum = 0;
+  for (int l = 0; l < L - 1; l++) {
+    q.n_per_level[l] = (int32_t)std::nearbyint((float)per);
+    sum += q.n_per_level[l];
+    per = per * factor;
+  }
+  q.n_per_level[L - 1] = imax(nf - sum, 0);
+  int cap = 0;
+  for (int l = 0; l < L; l++) {
+    const int maxbx = q.level_w[l] - kEdgeThreshold + 3, maxby = q.level_h[l] - kEdgeThreshold + 3;
+    const float width = (float)(maxbx - kMinBorder), height = (float)(maxby - kMinBorder);
+    const int cols = (int)(width / (float)kCellPx), rows = (int)(height / (float)kCellPx);
+    if (cols < 1 || rows < 1) return fail(SS_EINVAL, "a pyramid level is smaller than one FAST cell");
+    q.cell_cols[l] = cols;
+    q.cell_rows[l] = rows;
+    q.cell_w[l] = (int)std::ceil(width / (float)cols);
+    q.cell_h[l] = (int)std::ceil(height / (float)rows);
+    const int nini = (int)std::round(width / height);  // half away from zero
+    if (nini < 1 || nini > 62) return fail(SS_EINVAL, "level aspect ratio outside the quadtree's root range");
+    q.n_ini[l] = nini;
+    q.level_cap[l] = imax(q.n_per_level[l] + 2, 4 * nini);
+    cap += q.level_cap[l];
+  }
+  q.kp_capacity = cap;
+  *p = q;
+  return SS_OK;
+}
+
+// Bilinear source coordinate of destination index d (INTER_LINEAR_EXACT): packed
+// x0 | wx1 << 16 | (x1 - x0) << 25 with wx1 = rne(frac * 256).
+uint32_t lin_coef(int d, int sn, int dn) {
+  volatile double ratio = (double)sn / (double)dn;
+  volatile double fx = ((double)d + 0.5) * ratio;
+  double f = fx - 0.5;
+  double fl = std::floor(f);
+  int x0 = (int)fl;
+  double frac = f - fl;
+  if (x0 < 0) { x0 = 0; frac = 0.0; }
+  if (x0 >= sn - 1) { x0 = sn - 1; frac = 0.0; }
+  const int w1 = (int)std::nearbyint(frac * 256.0);
+  const int x1 = imin(x0 + 1, sn - 1);
+  return (uint32_t)x0 | ((uint32_t)w1 << 16) | ((uint32_t)(x1 - x0) << 25);
+}
+
+}  // namespace
+
+struct ss_ctx {
+  int device = 0;
+  ss_orb_params p{};
+  Geom g{};
+  int max_frames = 0, max_queries = 0, max_map = 0, max_splits = 0;
+  std::vector<CellInfo> cells_h;
+  // device scratch
+  CellInfo* cells = nullptr;
+  uint32_t* xytab = nullptr;  // per level l >= 1: xtab [w_l], ytab [h_l]
+  std::vector<int64_t> xoff, yoff;
+  uint8_t* pyr = nullptr;
+  uint32_t* slots = nullptr;
+  int32_t* cell_counts = nullptr;
+  uint32_t* selected = nullptr;
+  int32_t* sel_counts = nullptr;
+  uint8_t* ovf = nullptr;
+  int64_t ovf_frame_bytes = 0;
+  int64_t* ovf_level_off = nullptr;
+  int32_t* ovf_counter = nullptr;  // [0] overflowed levels, [1] capacity violations
+  int8_t* pattern = nullptr;
+  unsigned long long* claim = nullptr;
+  unsigned long long* partial = nullptr;
+  // last extract (debug hooks)
+  const uint8_t* last_frames = nullptr;
+  int64_t last_stride = 0;
+  int32_t last_pitch = 0;
+  int last_n = 0;
+};
+
+namespace {
+
+void free_ctx(ss_ctx* c) {
+  if (!c) return;
+  cudaSetDevice(c->device);
+  void* ptrs[] = {c->cells, c->xytab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
+                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial};
+  for (void* q : ptrs)
+    if (q) cudaFree(q);
+  delete c;
+}
+
+template <typename T>
+cudaError_t dalloc(T** p, size_t bytes) {
+  return cudaMalloc(reinterpret_cast<void**>(p), bytes > 0 ? bytes : 16);
+}
+
+}  // namespace
+
+extern "C" {
+
+ss_status ss_orb_params_init(int32_t width, int32_t height, int32_t n_features, int32_t n_levels, float scale_factor,
+                             int32_t ini_th_fast, int32_t min_th_fast, ss_orb_params* out) {
+  if (!out) return fail(SS_EINVAL, "out is NULL");
+  return params_init(width, height, n_features, n_levels, scale_factor, ini_th_fast, min_th_fast, out);
+}
+
+const char* ss_last_error(const ss_ctx*) { return g_err.c_str(); }
+
+ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, int32_t max_queries, int32_t max_map,
+                    ss_ctx** out) {
+  if (!p || !out) return fail(SS_EINVAL, "NULL argument");
+  *out = nullptr;
+  if (max_frames < 1 || max_queries < 0 || max_map < 0) return fail(SS_EINVAL, "bad capacities");
+  ss_orb_params q;
+  ss_status st = params_init(p->width, p->height, p->n_features, p->n_levels, p->scale_factor, p->ini_th_fast,
+                             p->min_th_fast, &q);
+  if (st != SS_OK) return st;
+  if (std::memcmp(&q, p, sizeof(q)) != 0) return fail(SS_EINVAL, "params differ from ss_orb_params_init's");
+  int ndev = 0;
+  SS_CUDA_TRY(cudaGetDeviceCount(&ndev));
+  if (device < 0 || device >= ndev) return fail(SS_EINVAL, "no such device");
+  SS_CUDA_TRY(cudaSetDevice(device));
+  ss_ctx* c = new (std::nothrow) ss_ctx();
+  if (!c) return fail(SS_ECUDA, "host allocation failed");
+  c->device = device;
+  c->p = q;
+  c->max_frames = max_frames;
+  c->max_queries = max_queries;
+  c->max_map = max_map;
+  Geom& g = c->g;
+  const int L = q.n_levels;
+  g.L = L;
+  g.W = q.width;
+  g.H = q.height;
+  g.ini_th = q.ini_th_fast;
+  g.min_th = q.min_th_fast;
+  int64_t poff = 0;
+  int cap_off = 0, slot_off = 0, max_rw = 0, max_rh = 0;
+  for (int l = 0; l < L; l++) {
+    g.w[l] = q.level_w[l];
+    g.h[l] = q.level_h[l];
+    g.scale[l] = q.scale[l];
+    g.pitch[l] = (g.w[l] + 15) & ~15;
+    g.lvl_off[l] = 0;
+    if (l >= 1) {
+      g.lvl_off[l] = poff;
+      poff += ((int64_t)g.pitch[l] * g.h[l] + 127) & ~(int64_t)127;
+    }
+    g.N[l] = q.n_per_level[l];
+    g.cap[l] = q.level_cap[l];
+    g.cap_off[l] = cap_off;
+    cap_off += q.level_cap[l];
+    g.nini[l] = q.n_ini[l];
+    const int maxbx = g.w[l] - kEdgeThreshold + 3, maxby = g.h[l] - kEdgeThreshold + 3;
+    g.qw[l] = maxbx - kMinBorder;
+    g.qh[l] = maxby - kMinBorder;
+    volatile float hx = (float)g.qw[l] / (float)g.nini[l];
+    g.hX[l] = hx;
+    g.qrounds[l] = kQuadRounds;
+    // active FAST cells, row-major (DESIGN.md §3 O3)
+    g.cell_first[l] = (int)c->cells_h.size();
+    g.level_slot_off[l] = slot_off;
+    const int wc = q.cell_w[l], hc = q.cell_h[l];
+    for (int i = 0; i < q.cell_rows[l]; i++) {
+      const int iniY = kMinBorder + i * hc;
+      if (iniY >= maxby - 3) continue;
+      const int maxY = imin(iniY + hc + 6, maxby);
+      for (int j = 0; j < q.cell_cols[l]; j++) {
+        const int iniX = kMinBorder + j * wc;
+        if (iniX >= maxbx - 6) continue;
+        const int maxX = imin(iniX + wc + 6, maxbx);
+        CellInfo ci;
+        ci.level = l;
+        ci.x0 = iniX + 3;
+        ci.y0 = iniY + 3;
+        ci.x1 = maxX - 3;
+        ci.y1 = maxY - 3;
+        const int dw = ci.x1 - ci.x0, dh = ci.y1 - ci.y0;
+        ci.slot_off = slot_off;
+        ci.slot_cap = ((dw + 1) / 2) * ((dh + 1) / 2);
+        ci.pad = 0;
+        slot_off += ci.slot_cap;
+        max_rw = imax(max_rw, dw + 6);
+        max_rh = imax(max_rh, dh + 6);
+        c->cells_h.push_back(ci);
+      }
+    }
+    g.ncells[l] = (int)c->cells_h.size() - g.cell_first[l];
+    g.level_slots[l] = slot_off - g.level_slot_off[l];
+    if (g.ncells[l] > 4608) {
+      free_ctx(c);
+      return fail(SS_EUNSUPPORTED, "more than 4608 FAST cells on one level");
+    }
+  }
+  g.pyr_frame_bytes = poff;
+  g.total_cells = (int)c->cells_h.size();
+  g.slots_per_frame = slot_off;
+  g.kp_capacity = q.kp_capacity;
+  g.max_rw = max_rw;
+  g.max_rh = max_rh;
+  if (max_rw > 64 || max_rh > 64) {
+    free_ctx(c);
+    return fail(SS_EUNSUPPORTED, "FAST cell larger than 58x58 px");
+  }
+  // coefficient tables for levels >= 1
+  std::vector<uint32_t> tab;
+  c->xoff.assign(L, 0);
+  c->yoff.assign(L, 0);
+  for (int l = 1; l < L; l++) {
+    c->xoff[l] = (int64_t)tab.size();
+    for (int x = 0; x < g.w[l]; x++) tab.push_back(lin_coef(x, g.w[l - 1], g.w[l]));
+    c->yoff[l] = (int64_t)tab.size();
+    for (int y = 0; y < g.h[l]; y++) tab.push_back(lin_coef(y, g.h[l - 1], g.h[l]));
+  }
+  // overflow scratch layout
+  std::vector<int64_t> ovf_off(L, 0);
+  int64_t ob = 0;
+  for (int l = 0; l < L; l++) {
+    ovf_off[l] = ob;
+    ob += distribute_ovf_bytes(g.level_slots[l]);
+  }
+  c->ovf_frame_bytes = ob;
+  c->max_splits = 16;
+  std::vector<int8_t> pat(1024);
+  const int* ph = brief_pattern_host();
+  for (int i = 0; i < 1024; i++) pat[i] = (int8_t)ph[i];
+  const int64_t F = max_frames;
+  cudaError_t e = cudaSuccess;
+#define ALLOC(ptr, bytes)                          \
+  if (e == cudaSuccess) e = dalloc(&(ptr), (bytes));
+  ALLOC(c->cells, sizeof(CellInfo) * c->cells_h.size());
+  ALLOC(c->xytab, sizeof(uint32_t) * tab.size());
+  ALLOC(c->pyr, F * g.pyr_frame_bytes);
+  ALLOC(c->slots, sizeof(uint32_t) * F * g.slots_per_frame);
+  ALLOC(c->cell_counts, sizeof(int32_t) * F * g.total_cells);
+  ALLOC(c->selected, sizeof(uint32_t) * F * g.kp_capacity);
+  ALLOC(c->sel_counts, sizeof(int32_t) * F * L);
+  ALLOC(c->ovf, F * c->ovf_frame_bytes);
+  ALLOC(c->ovf_level_off, sizeof(int64_t) * L);
+  ALLOC(c->ovf_counter, sizeof(int32_t) * 2);
+  ALLOC(c->pattern, 1024);
+  ALLOC(c->claim, sizeof(unsigned long long) * F * g.kp_capacity);
+  if (max_map > 0) ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
+#undef ALLOC
+  if (e == cudaSuccess) e = cudaMemcpy(c->cells, c->cells_h.data(), sizeof(CellInfo) * c->cells_h.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess && !tab.empty()) e = cudaMemcpy(c->xytab, tab.data(), sizeof(uint32_t) * tab.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(c->ovf_level_off, ovf_off.data(), sizeof(int64_t) * L, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(c->pattern, pat.data(), 1024, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemset(c->ovf_counter, 0, sizeof(int32_t) * 2);
+  if (e == cudaSuccess) e = cudaMemset(c->sel_counts, 0, sizeof(int32_t) * F * L);
+  if (e != cudaSuccess) {
+    std::string m = std::string("ss_create: ") + cudaGetErrorString(e);
+    free_ctx(c);
+    return fail(SS_ECUDA, m);
+  }
+  *out = c;
+  return SS_OK;
+}
+
+ss_status ss_destroy(ss_ctx* ctx) {
+  if (!ctx) return fail(SS_EINVAL, "NULL ctx");
+  free_ctx(ctx);
+  return SS_OK;
+}
+
+ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, int64_t frame_stride, int32_t pitch,
+                         ss_keypoint* d_kps, uint8_t* d_desc, int32_t* d_counts, ss_stream_t stream) {
+  if (!c) return fail(SS_EINVAL, "NULL ctx");
+  if (n_frames < 0) return fail(SS_EINVAL, "n_frames < 0");
+  if (n_frames > c->max_frames) return fail(SS_ECAPACITY, "n_frames exceeds the ctx's max_frames");
+  if (n_frames == 0) return SS_OK;
+  if (!d_frames || !d_kps || !d_desc || !d_counts) return fail(SS_EINVAL, "NULL buffer");
+  if (pitch < c->g.W) return fail(SS_EINVAL, "pitch < width");
+  if (n_frames > 1 && frame_stride < (int64_t)pitch * c->g.H) return fail(SS_EINVAL, "frame_stride < height*pitch");
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  const Geom& g = c->g;
+  FrameSrc src{d_frames, frame_stride, pitch, c->pyr};
+  SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 2, s));
+  for (int l = 1; l < g.L; l++)
+    SS_CUDA_TRY(launch_pyramid_level(g, l, n_frames, src, c->xytab + c->xoff[l], c->xytab + c->yoff[l], s));
+  SS_CUDA_TRY(launch_fast_cells(g, n_frames, src, c->cells, c->slots, c->cell_counts, s));
+  SS_CUDA_TRY(launch_distribute(g, n_frames, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
+                                c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, s));
+  SS_CUDA_TRY(launch_describe(g, n_frames, src, c->selected, c->sel_counts, c->pattern, d_kps, d_desc, d_counts, s));
+  c->last_frames = d_frames;
+  c->last_stride = frame_stride;
+  c->last_pitch = pitch;
+  c->last_n = n_frames;
+  return SS_OK;
+}
+
+ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_kps, const uint8_t* d_desc,
+                              const int32_t* d_counts, const uint8_t* d_kp_taken, int32_t n_queries,
+                              const ss_mp_query* d_queries, const uint8_t* d_map_desc, int32_t n_map,
+                              const ss_match_cfg* cfg, ss_match* d_out, ss_stream_t stream) {
+  if (!c || !cfg) return fail(SS_EINVAL, "NULL ctx/cfg");
+  if (n_frames < 0 || n_queries < 0 || n_map < 0) return fail(SS_EINVAL, "negative size");
+  if (n_frames > c->max_frames) return fail(SS_ECAPACITY, "n_frames exceeds the ctx's max_frames");
+  if (cfg->ratio_den <= 0 || cfg->ratio_num < 0) return fail(SS_EINVAL, "bad ratio");
+  if (!d_kps || !d_desc || !d_counts || !d_out) return fail(SS_EINVAL, "NULL buffer");
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  if (cfg->mode == SS_MATCH_WINDOW) {
+    if (n_queries > c->max_queries) return fail(SS_ECAPACITY, "n_queries exceeds the ctx's max_queries");
+    if (n_queries > 0 && (!d_queries || !d_map_desc)) return fail(SS_EINVAL, "NULL queries");
+    SS_CUDA_TRY(launch_match_window(c->g, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_queries, d_queries,
+                                    d_map_desc, *cfg, c->claim, d_out, s));
+    return SS_OK;
+  }
+  if (cfg->mode == SS_MATCH_BRUTE) {
+    if (n_queries != 0) return fail(SS_EINVAL, "BRUTE mode takes no queries");
+    if (n_map > c->max_map) return fail(SS_ECAPACITY, "n_map exceeds the ctx's max_map");
+    if (n_map > 0 && !d_map_desc) return fail(SS_EINVAL, "NULL map");
+    if (n_frames == 0) return SS_OK;
+    SS_CUDA_TRY(launch_match_brute(c->g, n_frames, d_desc, d_counts, n_map, d_map_desc, *cfg, c->partial,
+                                   c->max_splits, d_out, s));
+    return SS_OK;
+  }
+  return fail(SS_EINVAL, "unknown match mode");
+}
+
+ss_status ss_debug_level(ss_ctx* c, int32_t frame, int32_t level, const uint8_t** d_ptr, int32_t* pitch) {
+  if (!c || !d_ptr || !pitch) return fail(SS_EINVAL, "NULL argument");
+  if (frame < 0 || frame >= c->max_frames || level < 1 || level >= c->g.L) return fail(SS_EINVAL, "bad frame/level");
+  *d_ptr = c->pyr + (int64_t)frame * c->g.pyr_frame_bytes + c->g.lvl_off[level];
+  *pitch = c->g.pitch[level];
+  return SS_OK;
+}
+
+ss_status ss_debug_candidates(ss_ctx* c, int32_t frame, int32_t level, int32_t* h_lx, int32_t* h_ly, int32_t* h_score,
+                              int32_t cap, int32_t* n) {
+  if (!c || !n) return fail(SS_EINVAL, "NULL argument");
+  if (frame < 0 || frame >= c->max_frames || level < 0 || level >= c->g.L) return fail(SS_EINVAL, "bad frame/level");
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  SS_CUDA_TRY(cudaDeviceSynchronize());
+  const Geom& g = c->g;
+  const int c0 = g.cell_first[level], nc = g.ncells[level];
+  std::vector<int32_t> cnt(nc);
+  SS_CUDA_TRY(cudaMemcpy(cnt.data(), c->cell_counts + (int64_t)frame * g.total_cells + c0, sizeof(int32_t) * nc,
+                         cudaMemcpyDeviceToHost));
+  std::vector<uint32_t> sl(g.level_slots[level]);
+  SS_CUDA_TRY(cudaMemcpy(sl.data(), c->slots + (int64_t)frame * g.slots_per_frame + g.level_slot_off[level],
+                         sizeof(uint32_t) * sl.size(), cudaMemcpyDeviceToHost));
+  int k = 0;
+  for (int i = 0; i < nc; i++) {
+    const CellInfo& ci = c->cells_h[c0 + i];
+    for (int j = 0; j < cnt[i]; j++) {
+      if (k < cap) {
+        const uint32_t v = sl[ci.slot_off - g.level_slot_off[level] + j];
+        if (h_lx) h_lx[k] = key_lx(v);
+        if (h_ly) h_ly[k] = key_ly(v);
+        if (h_score) h_score[k] = key_m(v);
+      }
+      k++;
+    }
+  }
+  *n = k;
+  if (k > cap) return fail(SS_ECAPACITY, "more candidates than cap");
+  return SS_OK;
+}
+
+ss_status ss_debug_overflow_count(ss_ctx* c, int32_t* n) {
+  if (!c || !n) return fail(SS_EINVAL, "NULL argument");
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  SS_CUDA_TRY(cudaDeviceSynchronize());
+  int32_t v[2];
+  SS_CUDA_TRY(cudaMemcpy(v, c->ovf_counter, sizeof(v), cudaMemcpyDeviceToHost));
+  *n = v[0];
+  if (v[1] != 0) return fail(SS_ECAPACITY, "a level kept more keypoints than its level_cap (bug)");
+  return SS_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,93 @@
+// ss_internal.h -- product-internal types shared by the host layer (ss_api.cpp) and the
+// sm_100a kernels.  Nothing here is shared with oracle/ (the CPU checker).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/ss.h"
+
+namespace ss {
+
+constexpr int kMaxLevels = SS_MAX_LEVELS;
+constexpr int kEdgeThreshold = 19;  // ORB-SLAM EDGE_THRESHOLD [ext]
+constexpr int kMinBorder = kEdgeThreshold - 3;
+constexpr int kCellPx = 30;         // FAST grid cell (north_star "per 30-px grid cell")
+constexpr int kQuadRounds = 13;     // quadtree path depth stored per key (levels <= 2048 px)
+
+// One FAST cell: detect window D = [x0,x1) x [y0,y1) of its level (DESIGN.md §3 O3) and
+// the range of its candidate slots inside a frame's slot array.
+struct CellInfo {
+  int32_t level;
+  int32_t x0, y0, x1, y1;
+  int32_t slot_off;  // entries from the start of the frame's slot array
+  int32_t slot_cap;  // ceil(Dw/2)*ceil(Dh/2): strict 8-neighbour maxima per 2x2 block <= 1
+  int32_t pad;
+};
+
+// Everything the kernels need to know about the frame shape, by value in kernel params.
+struct Geom {
+  int32_t L, W, H;
+  int32_t ini_th, min_th;
+  int32_t w[kMaxLevels], h[kMaxLevels];
+  int32_t pitch[kMaxLevels];        // pyramid scratch pitch of level l (l >= 1)
+  int64_t lvl_off[kMaxLevels];      // byte offset of level l in a frame's pyramid scratch
+  int64_t pyr_frame_bytes;
+  float scale[kMaxLevels];
+  int32_t cell_first[kMaxLevels];   // first active cell of level l in the cell table
+  int32_t ncells[kMaxLevels];       // active cells of level l (row-major, skipped cells removed)
+  int32_t total_cells;              // per frame
+  int32_t slots_per_frame;          // candidate slot entries per frame
+  int32_t level_slot_off[kMaxLevels], level_slots[kMaxLevels];
+  int32_t N[kMaxLevels];            // distribution target n_per_level
+  int32_t cap[kMaxLevels];          // level_cap
+  int32_t cap_off[kMaxLevels];      // offset of level l in a frame's selected-key scratch
+  int32_t kp_capacity;
+  int32_t nini[kMaxLevels];
+  float hX[kMaxLevels];             // f32(qw / nIni)
+  int32_t qw[kMaxLevels], qh[kMaxLevels];  // quadtree box (maxBorder - minBorder)
+  int32_t qrounds[kMaxLevels];      // quadtree rounds that can still separate keys on level l
+  int32_t max_rw, max_rh;           // largest FAST input region (D + 3-px halo) of any cell
+};
+
+// Where the frames of one call live.  Level 0 is the caller's frame (no copy).
+struct FrameSrc {
+  const uint8_t* frames;
+  int64_t stride;
+  int32_t pitch;
+  uint8_t* pyr;  // pyramid scratch (levels >= 1)
+};
+
+// Candidate / selected key: (ly << 19) | (lx << 8) | M  (lx, ly < 2048, M = FAST score + 1).
+__host__ __device__ inline uint32_t pack_key(int lx, int ly, int m) {
+  return ((uint32_t)ly << 19) | ((uint32_t)lx << 8) | (uint32_t)m;
+}
+__host__ __device__ inline int key_lx(uint32_t k) { return (int)((k >> 8) & 0x7FF); }
+__host__ __device__ inline int key_ly(uint32_t k) { return (int)(k >> 19); }
+__host__ __device__ inline int key_m(uint32_t k) { return (int)(k & 0xFF); }
+
+// ---- launchers (one per kernel; each returns cudaGetLastError()) ----
+cudaError_t launch_pyramid_level(const Geom& g, int level, int n_frames, FrameSrc src,
+                                 const uint32_t* xtab, const uint32_t* ytab, cudaStream_t s);
+cudaError_t launch_fast_cells(const Geom& g, int n_frames, FrameSrc src, const CellInfo* cells,
+                              uint32_t* slots, int32_t* cell_counts, cudaStream_t s);
+cudaError_t launch_distribute(const Geom& g, int n_frames, const CellInfo* cells, const uint32_t* slots,
+                              const int32_t* cell_counts, uint32_t* selected, int32_t* sel_counts,
+                              uint8_t* ovf, int64_t ovf_frame_bytes, const int64_t* ovf_level_off,
+                              int32_t* ovf_counter, cudaStream_t s);
+cudaError_t launch_describe(const Geom& g, int n_frames, FrameSrc src, const uint32_t* selected,
+                            const int32_t* sel_counts, const int8_t* pattern, ss_keypoint* kps, uint8_t* desc,
+                            int32_t* counts, cudaStream_t s);
+// The rotated-BRIEF pattern (1024 ints: 256 pairs x 2 points x (x, y)), host copy.
+const int* brief_pattern_host();
+cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* kps, const uint8_t* desc,
+                                const int32_t* counts, const uint8_t* taken, int n_queries,
+                                const ss_mp_query* q, const uint8_t* qdesc, ss_match_cfg cfg,
+                                unsigned long long* claim, ss_match* out, cudaStream_t s);
+cudaError_t launch_match_brute(const Geom& g, int n_frames, const uint8_t* desc, const int32_t* counts,
+                               int n_map, const uint8_t* map_desc, ss_match_cfg cfg,
+                               unsigned long long* partial, int max_splits, ss_match* out, cudaStream_t s);
+
+// Overflow scratch bytes the distribution needs for a level with `slots` candidate slots.
+int64_t distribute_ovf_bytes(int64_t slots);
+
+}  // namespace ss

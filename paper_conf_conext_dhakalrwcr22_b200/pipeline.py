@@ -1,0 +1,89 @@
+"""Torch-buffer convenience layer over the C ABI (argument marshalling only).
+
+``OrbPipeline`` owns one ss_ctx plus torch CUDA output buffers sized for ``max_frames``:
+    kps    [max_frames, kp_capacity] ss_keypoint  (as a uint8 [.., 20] tensor)
+    desc   [max_frames, kp_capacity, 32] uint8
+    counts [max_frames, n_levels + 1] int32
+and exposes extract / match calls that enqueue on a torch stream.
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+from . import ss
+
+
+class OrbPipeline:
+    def __init__(self, width: int, height: int, n_features: int = 1000, n_levels: int = 8,
+                 scale_factor: float = 1.2, ini_th: int = 20, min_th: int = 7, max_frames: int = 4,
+                 max_queries: int = 0, max_map: int = 0, device: int = 0):
+        if not torch.cuda.is_available():
+            raise RuntimeError("OrbPipeline needs a CUDA device (no CPU fallback by design)")
+        self.device = torch.device("cuda", device)
+        self.params = ss.ss_orb_params_init(width, height, n_features, n_levels, scale_factor, ini_th, min_th)
+        self.ctx = ss.ss_create(device, self.params, max_frames, max_queries, max_map)
+        self.width, self.height = width, height
+        self.n_levels = n_levels
+        self.cap = self.params.kp_capacity
+        self.max_frames = max_frames
+        self.kps = torch.zeros((max_frames, self.cap, 20), dtype=torch.uint8, device=self.device)
+        self.desc = torch.zeros((max_frames, self.cap, ss.DESC_BYTES), dtype=torch.uint8, device=self.device)
+        self.counts = torch.zeros((max_frames, n_levels + 1), dtype=torch.int32, device=self.device)
+
+    def close(self):
+        if self.ctx:
+            ss.ss_destroy(self.ctx)
+            self.ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # -- hot path -------------------------------------------------------------------
+    def extract(self, frames: torch.Tensor, stream: torch.cuda.Stream | None = None, n_frames: int | None = None):
+        """frames: uint8 CUDA tensor [B, H, pitch] (row pitch = frames.stride(1))."""
+        assert frames.dtype == torch.uint8 and frames.is_cuda and frames.dim() == 3
+        assert frames.stride(2) == 1
+        B = frames.shape[0] if n_frames is None else n_frames
+        stream = stream or torch.cuda.current_stream(self.device)
+        ss.ss_orb_extract(self.ctx, B, frames, frames.stride(0), frames.stride(1), self.kps, self.desc,
+                          self.counts, stream)
+
+    def match_window(self, n_frames: int, queries: torch.Tensor, qdesc: torch.Tensor, out: torch.Tensor,
+                     taken: torch.Tensor | None = None, cfg: ss.ss_match_cfg | None = None,
+                     stream: torch.cuda.Stream | None = None):
+        cfg = cfg or ss.window_cfg()
+        stream = stream or torch.cuda.current_stream(self.device)
+        nq = queries.numel() // 20 if queries.dtype == torch.uint8 else queries.shape[0]
+        ss.ss_match_projection(self.ctx, n_frames, self.kps, self.desc, self.counts, taken, nq, queries, qdesc,
+                               0, cfg, out, stream)
+
+    def match_brute(self, n_frames: int, map_desc: torch.Tensor, out: torch.Tensor,
+                    cfg: ss.ss_match_cfg | None = None, stream: torch.cuda.Stream | None = None):
+        cfg = cfg or ss.brute_cfg()
+        stream = stream or torch.cuda.current_stream(self.device)
+        ss.ss_match_projection(self.ctx, n_frames, self.kps, self.desc, self.counts, None, 0, None, map_desc,
+                               map_desc.shape[0], cfg, out, stream)
+
+    # -- host views (synchronising; tests / examples) -------------------------------
+    def results(self, n_frames: int):
+        torch.cuda.synchronize(self.device)
+        kps = self.kps[:n_frames].cpu().numpy().view(ss.KEYPOINT_DTYPE).reshape(n_frames, self.cap)
+        return kps, self.desc[:n_frames].cpu().numpy(), self.counts[:n_frames].cpu().numpy()
+
+
+def to_device_records(arr: np.ndarray, device) -> torch.Tensor:
+    """numpy structured array -> uint8 CUDA tensor with the same bytes."""
+    raw = np.ascontiguousarray(arr).view(np.uint8).reshape(len(arr), -1)
+    return torch.from_numpy(raw.copy()).to(device)
+
+
+def match_out(n: int, device) -> torch.Tensor:
+    return torch.zeros((n, 3), dtype=torch.int32, device=device)
+
+
+def match_records(t: torch.Tensor) -> np.ndarray:
+    return t.cpu().numpy().astype(np.int32).view(ss.MATCH_DTYPE).reshape(-1)

@@ -1,0 +1,177 @@
+"""Thin ctypes binding of libss (include/ss.h).  Argument marshalling only: every step of
+the ORB extract + match path runs in the sm_100a kernels of csrc/.  There is no CPU
+fallback: if libss.so is missing or no GPU is present, calls raise.
+
+torch is used only for device memory (tensor.data_ptr()) and streams (cuda_stream handles).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libss.so")
+MAX_LEVELS = 8
+DESC_BYTES = 32
+
+SS_OK, SS_EINVAL, SS_ECAPACITY, SS_ECUDA, SS_EUNSUPPORTED = 0, -1, -2, -3, -4
+SS_MATCH_WINDOW, SS_MATCH_BRUTE = 0, 1
+_STATUS = {0: "SS_OK", -1: "SS_EINVAL", -2: "SS_ECAPACITY", -3: "SS_ECUDA", -4: "SS_EUNSUPPORTED"}
+
+
+class SSError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class ss_orb_params(C.Structure):
+    _fields_ = [("width", C.c_int32), ("height", C.c_int32), ("n_features", C.c_int32),
+                ("n_levels", C.c_int32), ("scale_factor", C.c_float),
+                ("ini_th_fast", C.c_int32), ("min_th_fast", C.c_int32),
+                ("scale", C.c_float * MAX_LEVELS), ("inv_scale", C.c_float * MAX_LEVELS),
+                ("level_w", C.c_int32 * MAX_LEVELS), ("level_h", C.c_int32 * MAX_LEVELS),
+                ("n_per_level", C.c_int32 * MAX_LEVELS),
+                ("cell_cols", C.c_int32 * MAX_LEVELS), ("cell_rows", C.c_int32 * MAX_LEVELS),
+                ("cell_w", C.c_int32 * MAX_LEVELS), ("cell_h", C.c_int32 * MAX_LEVELS),
+                ("n_ini", C.c_int32 * MAX_LEVELS), ("level_cap", C.c_int32 * MAX_LEVELS),
+                ("kp_capacity", C.c_int32)]
+
+    def as_dict(self) -> dict:
+        out = {}
+        for name, _ in self._fields_:
+            v = getattr(self, name)
+            out[name] = list(v) if hasattr(v, "__len__") else v
+        return out
+
+
+class ss_match_cfg(C.Structure):
+    _fields_ = [("mode", C.c_int32), ("th", C.c_int32), ("ratio_num", C.c_int32),
+                ("ratio_den", C.c_int32), ("dedup", C.c_int32)]
+
+
+# numpy views of the 20-/20-/12-byte records of ss.h
+KEYPOINT_DTYPE = np.dtype([("x", "<f4"), ("y", "<f4"), ("angle_deg", "<f4"), ("lx", "<u2"),
+                           ("ly", "<u2"), ("level", "u1"), ("response", "u1"), ("reserved", "<u2")])
+QUERY_DTYPE = np.dtype([("frame", "<i4"), ("u", "<f4"), ("v", "<f4"), ("pred_level", "<i4"),
+                        ("radius", "<f4")])
+MATCH_DTYPE = np.dtype([("idx", "<i4"), ("dist", "<i4"), ("dist2", "<i4")])
+
+_lib = None
+
+
+def lib():
+    """Load libss.so (built by build.py).  Raises if it is missing -- no fallback."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"libss.so not built ({LIB_PATH}); run __graft_entry__.build()")
+        L = C.CDLL(LIB_PATH)
+        P, i32, i64 = C.c_void_p, C.c_int32, C.c_int64
+        L.ss_orb_params_init.argtypes = [i32, i32, i32, i32, C.c_float, i32, i32, C.POINTER(ss_orb_params)]
+        L.ss_create.argtypes = [i32, C.POINTER(ss_orb_params), i32, i32, i32, C.POINTER(P)]
+        L.ss_destroy.argtypes = [P]
+        L.ss_last_error.argtypes = [P]
+        L.ss_last_error.restype = C.c_char_p
+        L.ss_orb_extract.argtypes = [P, i32, P, i64, i32, P, P, P, P]
+        L.ss_match_projection.argtypes = [P, i32, P, P, P, P, i32, P, P, i32, C.POINTER(ss_match_cfg), P, P]
+        L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
+        L.ss_debug_candidates.argtypes = [P, i32, i32, P, P, P, i32, C.POINTER(i32)]
+        L.ss_debug_overflow_count.argtypes = [P, C.POINTER(i32)]
+        for fn in ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_orb_extract", "ss_match_projection",
+                   "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count"):
+            getattr(L, fn).restype = C.c_int
+        _lib = L
+    return _lib
+
+
+EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "ss_orb_extract",
+            "ss_match_projection", "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count")
+
+
+def _check(status: int, ctx=None):
+    if status != SS_OK:
+        raise SSError(status, lib().ss_last_error(ctx).decode())
+
+
+def _ptr(x) -> int | None:
+    """Device pointer of a torch tensor (or int / None)."""
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    return x.data_ptr()
+
+
+def _stream(s) -> int | None:
+    if s is None:
+        return None
+    if isinstance(s, int):
+        return s
+    return s.cuda_stream
+
+
+# ---- same names as the C ABI --------------------------------------------------------
+
+def ss_orb_params_init(width, height, n_features=1000, n_levels=8, scale_factor=1.2, ini_th_fast=20,
+                       min_th_fast=7) -> ss_orb_params:
+    p = ss_orb_params()
+    _check(lib().ss_orb_params_init(width, height, n_features, n_levels, scale_factor, ini_th_fast,
+                                    min_th_fast, C.byref(p)))
+    return p
+
+
+def ss_create(device: int, p: ss_orb_params, max_frames: int, max_queries: int = 0, max_map: int = 0) -> int:
+    ctx = C.c_void_p()
+    _check(lib().ss_create(device, C.byref(p), max_frames, max_queries, max_map, C.byref(ctx)))
+    return ctx.value
+
+
+def ss_destroy(ctx: int) -> None:
+    _check(lib().ss_destroy(ctx))
+
+
+def ss_last_error(ctx=None) -> str:
+    return lib().ss_last_error(ctx).decode()
+
+
+def ss_orb_extract(ctx, n_frames, d_frames, frame_stride, pitch, d_kps, d_desc, d_counts, stream=None):
+    _check(lib().ss_orb_extract(ctx, n_frames, _ptr(d_frames), frame_stride, pitch, _ptr(d_kps),
+                                _ptr(d_desc), _ptr(d_counts), _stream(stream)), ctx)
+
+
+def ss_match_projection(ctx, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_queries, d_queries,
+                        d_map_desc, n_map, cfg: ss_match_cfg, d_out, stream=None):
+    _check(lib().ss_match_projection(ctx, n_frames, _ptr(d_kps), _ptr(d_desc), _ptr(d_counts),
+                                     _ptr(d_kp_taken), n_queries, _ptr(d_queries), _ptr(d_map_desc), n_map,
+                                     C.byref(cfg), _ptr(d_out), _stream(stream)), ctx)
+
+
+def ss_debug_level(ctx, frame, level):
+    ptr, pitch = C.c_void_p(), C.c_int32()
+    _check(lib().ss_debug_level(ctx, frame, level, C.byref(ptr), C.byref(pitch)), ctx)
+    return ptr.value, pitch.value
+
+
+def ss_debug_candidates(ctx, frame, level, cap=1 << 21):
+    lx, ly, sc = (np.zeros(cap, np.int32) for _ in range(3))
+    n = C.c_int32()
+    _check(lib().ss_debug_candidates(ctx, frame, level, lx.ctypes.data, ly.ctypes.data, sc.ctypes.data, cap,
+                                     C.byref(n)), ctx)
+    return lx[:n.value].copy(), ly[:n.value].copy(), sc[:n.value].copy()
+
+
+def ss_debug_overflow_count(ctx) -> int:
+    n = C.c_int32()
+    _check(lib().ss_debug_overflow_count(ctx, C.byref(n)), ctx)
+    return n.value
+
+
+def window_cfg(th=100, ratio_num=4, ratio_den=5, dedup=1) -> ss_match_cfg:
+    return ss_match_cfg(SS_MATCH_WINDOW, th, ratio_num, ratio_den, dedup)
+
+
+def brute_cfg(th=50, ratio_num=3, ratio_den=4) -> ss_match_cfg:
+    return ss_match_cfg(SS_MATCH_BRUTE, th, ratio_num, ratio_den, 0)

@@ -1,0 +1,220 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle on identical seeded
+inputs.  Bar: pyramid, FAST candidates, selected keypoints, descriptors,
+counts and matches bit-exact; angle within 1e-4 rad (circular)."""
+import numpy as np
+import pytest
+
+import synth
+
+pytestmark = pytest.mark.gpu
+
+ANGLE_TOL_RAD = 1e-4
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_conext_dhakalrwcr22_b200 import build as b
+    b.build()
+    return torch
+
+
+def _pipe(torch_cuda, w, h, nf=1000, L=8, max_frames=4, max_queries=0, max_map=0):
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import OrbPipeline
+    return OrbPipeline(w, h, nf, L, max_frames=max_frames, max_queries=max_queries, max_map=max_map)
+
+
+def _upload(torch, frames, pitch=None):
+    B, H, W = frames.shape
+    pitch = pitch or W
+    buf = np.zeros((B, H, pitch), np.uint8)
+    buf[:, :, :W] = frames
+    return torch.from_numpy(buf).cuda()
+
+
+def assert_extract_equal(gk, gd, gc, rk, rd, rc, where=""):
+    np.testing.assert_array_equal(gc, rc, err_msg=f"counts {where}")
+    n = int(rc[-1])
+    g, r = gk[:n], rk[:n]
+    for fld in ("lx", "ly", "level", "response", "reserved", "x", "y"):
+        np.testing.assert_array_equal(g[fld], r[fld], err_msg=f"{fld} {where}")
+    da = np.radians(np.abs(g["angle_deg"].astype(np.float64) - r["angle_deg"].astype(np.float64)))
+    da = np.minimum(da, 2 * np.pi - da)
+    assert da.max(initial=0) <= ANGLE_TOL_RAD, f"angle {where}: {da.max()}"
+    assert ((g["angle_deg"] >= 0) & (g["angle_deg"] < 360)).all()
+    np.testing.assert_array_equal(gd[:n], rd[:n], err_msg=f"desc {where}")
+
+
+def _d2h(ptr, nbytes):
+    import ctypes
+    rt = ctypes.CDLL("libcudart.so.12")
+    out = np.empty(nbytes, np.uint8)
+    rc = rt.cudaMemcpy(ctypes.c_void_p(out.ctypes.data), ctypes.c_void_p(ptr), ctypes.c_size_t(nbytes),
+                       ctypes.c_int(2))
+    assert rc == 0
+    return out
+
+
+def test_pyramid_bit_exact(torch_cuda, ref):
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    for (w, h, L) in ((752, 480, 8), (333, 217, 3), (1241, 376, 8)):
+        frames = synth.make_frames(w, h, 2, cfg=11)
+        pipe = _pipe(torch, w, h, 200, L, max_frames=2)
+        pipe.extract(_upload(torch, frames, pitch=w + 13))
+        torch.cuda.synchronize()
+        p = ref.params(w, h, 200, n_levels=L)
+        for b in range(2):
+            want = ref.pyramid(p, frames[b])
+            for l in range(1, L):
+                ptr, pitch = ss.ss_debug_level(pipe.ctx, b, l)
+                lw, lh = p.level_w[l], p.level_h[l]
+                got = _d2h(ptr, lh * pitch).reshape(lh, pitch)[:, :lw]
+                np.testing.assert_array_equal(got, want[l], err_msg=f"{w}x{h} frame {b} level {l}")
+        pipe.close()
+
+
+@pytest.mark.parametrize("shape", ["euroc", "tum", "kitti"])
+def test_candidates_bit_exact(torch_cuda, ref, shape):
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    w, h = synth.SHAPES[shape]
+    frames = synth.make_frames(w, h, 2, cfg=12)
+    pipe = _pipe(torch, w, h, 1000, 8, max_frames=2)
+    pipe.extract(_upload(torch, frames))
+    p = ref.params(w, h, 1000)
+    for b in range(2):
+        levels = ref.pyramid(p, frames[b])
+        for l in range(8):
+            rl = ref.cell_candidates(p, l, ref.fast_M(levels[l]))
+            gl = ss.ss_debug_candidates(pipe.ctx, b, l)
+            for i, name in enumerate(("lx", "ly", "M")):
+                np.testing.assert_array_equal(gl[i], rl[i], err_msg=f"{shape} frame {b} level {l} {name}")
+    pipe.close()
+
+
+@pytest.mark.parametrize("w,h,nf,L,B", [(200, 160, 150, 3, 3), (320, 240, 300, 4, 2), (333, 217, 250, 3, 1),
+                                        (752, 480, 1000, 8, 4), (640, 480, 1000, 8, 2), (1241, 376, 2000, 8, 2),
+                                        (752, 480, 1250, 8, 1)])
+def test_extract_bit_exact(torch_cuda, ref, w, h, nf, L, B):
+    torch = torch_cuda
+    frames = synth.make_frames(w, h, B, cfg=13, client0=w)
+    pipe = _pipe(torch, w, h, nf, L, max_frames=B)
+    pipe.extract(_upload(torch, frames, pitch=(w + 63) // 64 * 64))
+    gk, gd, gc = pipe.results(B)
+    p = ref.params(w, h, nf, n_levels=L)
+    for b in range(B):
+        rk, rd, rc = ref.orb_extract(p, frames[b])
+        assert_extract_equal(gk[b], gd[b], gc[b], rk, rd, rc, f"{w}x{h} frame {b}")
+    assert sum(int(c[-1]) for c in gc) > 0
+    pipe.close()
+
+
+def test_batch_position_invariance(torch_cuda):
+    torch = torch_cuda
+    w, h = synth.SHAPES["euroc"]
+    frames = synth.make_frames(w, h, 4, cfg=14)
+    pipe = _pipe(torch, w, h, 1000, 8, max_frames=4)
+    pipe.extract(_upload(torch, frames))
+    k1, d1, c1 = pipe.results(4)
+    perm = [2, 0, 3, 1]
+    pipe.extract(_upload(torch, frames[perm]))
+    k2, d2, c2 = pipe.results(4)
+    for i, j in enumerate(perm):
+        n = c1[j][-1]
+        assert (c2[i] == c1[j]).all()
+        assert (k2[i][:n] == k1[j][:n]).all() and (d2[i][:n] == d1[j][:n]).all()
+    pipe.extract(_upload(torch, frames[1:2]), n_frames=1)
+    k3, d3, c3 = pipe.results(1)
+    assert (c3[0] == c1[1]).all() and (k3[0][: c1[1][-1]] == k1[1][: c1[1][-1]]).all()
+    pipe.close()
+
+
+def test_edge_frames(torch_cuda, ref):
+    """Flat frame (no candidates anywhere), a checkerboard and a noise frame whose level-0
+    candidates overflow shared memory (global-memory distribution path)."""
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    w, h = 752, 480
+    rng = np.random.default_rng(3)
+    flat = np.full((h, w), 97, np.uint8)
+    checker = ((np.indices((h, w)).sum(0) // 3) % 2 * 200 + 20).astype(np.uint8)
+    noise = rng.integers(0, 256, size=(h, w), dtype=np.uint8)
+    frames = np.stack([flat, checker, noise])
+    pipe = _pipe(torch, w, h, 1000, 8, max_frames=3)
+    pipe.extract(_upload(torch, frames))
+    gk, gd, gc = pipe.results(3)
+    assert ss.ss_debug_overflow_count(pipe.ctx) >= 1
+    p = ref.params(w, h, 1000)
+    for b in range(3):
+        rk, rd, rc = ref.orb_extract(p, frames[b])
+        assert_extract_equal(gk[b], gd[b], gc[b], rk, rd, rc, f"edge frame {b}")
+    assert gc[0][-1] == 0
+    pipe.close()
+
+
+def _window_inputs(ref, p, frames, n_q, th, seed):
+    from oracle import QUERY_DTYPE
+    rk, rd, rc = ref.orb_extract_batch(p, frames)
+    q, qd, taken = synth.make_queries(rk, rd, rc, p.n_levels, np.array(p.scale[:p.n_levels]),
+                                      np.array(p.n_per_level[:p.n_levels]), p.width, p.height, n_q, th, seed,
+                                      QUERY_DTYPE)
+    return rk, rd, rc, q, qd, taken
+
+
+@pytest.mark.parametrize("shape,nq,th", [("euroc", 5000, 1.0), ("tum", 3000, 3.0)])
+def test_window_match_bit_exact(torch_cuda, ref, shape, nq, th):
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import match_out, match_records, to_device_records
+    w, h = synth.SHAPES[shape]
+    B = 2
+    frames = synth.make_frames(w, h, B, cfg=15)
+    p = ref.params(w, h, 1000)
+    rk, rd, rc, q, qd, taken = _window_inputs(ref, p, frames, nq, th, 7)
+    q[::97]["frame"] = B + 3  # invalid frames
+    q[1::89]["pred_level"] = 7
+    pipe = _pipe(torch, w, h, 1000, 8, max_frames=B, max_queries=len(q))
+    pipe.extract(_upload(torch, frames))  # GPU extraction feeds the GPU matcher
+    gk, gd, gc = pipe.results(B)
+    for b in range(B):
+        assert_extract_equal(gk[b], gd[b], gc[b], rk[b], rd[b], rc[b])
+    dq = to_device_records(q, "cuda")
+    dqd = torch.from_numpy(qd).cuda()
+    dt = torch.from_numpy(taken).cuda()
+    for dedup in (1, 0):
+        for tk in (dt, None):
+            out = match_out(len(q), "cuda")
+            pipe.match_window(B, dq, dqd, out, taken=tk, cfg=ss.window_cfg(dedup=dedup))
+            got = match_records(out)
+            want = ref.match_window(p, rk, rd, rc, None if tk is None else taken, q, qd, 100, 4, 5, dedup)
+            np.testing.assert_array_equal(got, want)
+            if dedup and tk is not None:
+                assert (got["idx"] >= 0).sum() > len(q) // 10
+    pipe.close()
+
+
+def test_brute_match_bit_exact(torch_cuda, ref):
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import match_records
+    w, h = synth.SHAPES["euroc"]
+    B = 2
+    frames = synth.make_frames(w, h, B, cfg=16)
+    p = ref.params(w, h, 1250)
+    rk, rd, rc = ref.orb_extract_batch(p, frames)
+    for n_map in (1, 300, 20000):
+        mp = synth.make_brute_map([rd[b][: rc[b][-1]] for b in range(B)], n_map, seed=n_map,
+                                  n_from_kps=min(n_map, 800))
+        pipe = _pipe(torch, w, h, 1250, 8, max_frames=B, max_map=n_map)
+        pipe.extract(_upload(torch, frames))
+        out = torch.zeros((B * p.kp_capacity, 3), dtype=torch.int32, device="cuda")
+        pipe.match_brute(B, torch.from_numpy(mp).cuda(), out)
+        got = match_records(out).reshape(B, p.kp_capacity)
+        k1 = p.kp_capacity if n_map <= 300 else 60
+        want = ref.match_brute(p, rd, rc, mp, 50, 3, 4, 0, k1)
+        np.testing.assert_array_equal(got[:, :k1], want[:, :k1])
+        if n_map == 20000:
+            assert (got["idx"] >= 0).sum() > 100
+        pipe.close()
