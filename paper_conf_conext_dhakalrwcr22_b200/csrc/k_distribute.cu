@@ -305,7 +305,7 @@ __global__ void __launch_bounds__(DT, 1)
   // ---- 5. partial phase-2 round at depth D: order the multi-key nodes, split a prefix ----
   if (partial) {
     for (int i = tid; i < n; i += DT) {
-      if (i != 0 && a.dd[i] <= D) continue;
+      if (i != 0 && a.dd[i] > D) continue;  // not a depth-D node head
       int size = 1, c = 1;
       uint32_t minrank = a.rank[i];
       for (int j = i + 1; j < n && a.dd[j] > D; j++) {
@@ -348,7 +348,7 @@ __global__ void __launch_bounds__(DT, 1)
   uint32_t* kept = a.key;  // keys are no longer needed
   __syncthreads();
   for (int i = tid; i < n; i += DT) {
-    if (i != 0 && a.dd[i] <= dlim) continue;
+    if (i != 0 && a.dd[i] > dlim) continue;  // not a final node head
     const bool split = partial && (a.splitf[i] & 0x80);
     int best_m = -1;
     uint32_t best_r = 0;
