@@ -1,0 +1,600 @@
+"""bench.py -- batched ORB extract + match frames/s (and per-frame p50/p99 latency) on B200.
+
+Contract: ``python bench.py --gpus N --steps K --warmup W`` (torchrun for
+N > 1, one rank per GPU, NCCL) prints ONE JSON line on rank 0.  A step = one tick of the
+configured workload: every client on this rank submits one frame, the frames are ORB-extracted
+(pyramid, FAST, quadtree, orientation, blur, BRIEF) and matched (windowed search-local-points
+or brute force) through the C ABI.  Clients are sharded over ranks (weak scaling); with N > 1
+per-frame results are gathered to rank 0 (the map owner) over NCCL on a side stream.
+
+``--impl reference`` times the CPU oracle (oracle/, the checker) on the box's host cores on a
+bounded sample of the same workload and prints the same line with "impl": "reference".
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+METRIC = "batched ORB extract+match frames/sec at 1/2/4/8 B200; per-frame p50 latency ms"
+CONFIGS = {
+    "c1": dict(shape="euroc", clients=1, nf=1000, mode="window", queries=5000, th=1.0, map=0,
+               desc="c1: single synthetic 752x480 frame, 8 levels x1.2, 1000 ORB features, windowed match vs 5k map points"),
+    "c2": dict(shape="euroc", clients=4, nf=1000, mode="window", queries=5000, th=1.0, map=0,
+               desc="c2: EuRoC-shaped 752x480 mono stream, 4 concurrent clients per GPU, 1000 features/frame, "
+                    "windowed search-local-points vs 5k map points per client"),
+    "c3": dict(shape="tum", clients=16, nf=1000, mode="window", queries=50000, th=3.0, map=0,
+               desc="c3: TUM-RGBD-shaped 640x480, 16 clients per GPU, 1000 features, windowed match vs 50k map points"),
+    "c4": dict(shape="kitti", clients=8, stereo=True, nf=2000, mode="window", queries=10000, th=1.0, map=0,
+               desc="c4: KITTI-shaped 1241x376 stereo pairs, 8 clients per GPU, 2000 features/image, "
+                    "windowed match vs 10k map points (left image)"),
+    "c5": dict(shape="euroc", clients=8, nf=1250, mode="brute", queries=0, th=0.0, map=200000,
+               desc="c5: EuRoC-shaped clients (8 per GPU, 64 over 8xB200), 1250 features, brute-force Hamming "
+                    "vs a 200k shared-map descriptor set"),
+}
+CFG_ID = {"c1": 1, "c2": 2, "c3": 3, "c4": 4, "c5": 5}
+
+
+# ----------------------------------------------------------------------------- helpers
+def client_ids(rank: int, world: int, clients_per_rank: int) -> list[int]:
+    """Weak scaling: rank r owns clients [r*C, (r+1)*C) (disjoint, covering all)."""
+    return list(range(rank * clients_per_rank, (rank + 1) * clients_per_rank))
+
+
+def _gen_frame(args):
+    w, h, seed, stereo = args
+    if stereo:
+        l, r = synth.make_stereo_pair(w, h, seed)
+        return np.stack([l, r])
+    return synth.make_frame(w, h, seed)[None]
+
+
+def make_ring_frames(cfg: dict, clients: list[int], n_slots: int, workers: int) -> np.ndarray:
+    """[n_slots, images_per_step, H, W] u8, slot s = frame index s of every client."""
+    w, h = synth.SHAPES[cfg["shape"]]
+    stereo = bool(cfg.get("stereo"))
+    jobs = [(w, h, synth.frame_seed(CFG_ID[cfg["name"]], c, s), stereo) for s in range(n_slots) for c in clients]
+    if workers > 1 and len(jobs) > 8:
+        import multiprocessing as mp
+        with mp.get_context("fork").Pool(workers) as pool:
+            imgs = pool.map(_gen_frame, jobs, chunksize=max(1, len(jobs) // (4 * workers)))
+    else:
+        imgs = [_gen_frame(j) for j in jobs]
+    per = 2 if stereo else 1
+    out = np.stack(imgs).reshape(n_slots, len(clients) * per, h, w)
+    return out
+
+
+class ClockSampler:
+    """NVML sampling of SM clock + clock-event reasons during the timed region."""
+    BAD = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown"}
+    NAMES = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+             0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+             0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, device_index: int, period_s: float = 0.002):
+        self.samples, self.reasons, self.ok = [], 0, False
+        self.period = period_s
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover - depends on the box
+            self.err = str(e)
+        self._stop = threading.Event()
+        self._t = None
+
+    def _reason_bits(self):
+        nv = self.nv
+        fn = getattr(nv, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+            getattr(nv, "nvmlDeviceGetCurrentClocksThrottleReasons")
+        return fn(self.h)
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                self.reasons |= int(self._reason_bits())
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self) -> dict:
+        if not self.ok:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "error": getattr(self, "err", "nvml")}
+        reasons = [n for b, n in self.NAMES.items() if self.reasons & b and b != 0x1]
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None, "sm_max_mhz": self.max_mhz,
+                "reasons": reasons, "samples": len(self.samples),
+                "rejected": any(self.reasons & b for b in self.BAD)}
+
+
+def measured_peaks() -> dict:
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return {"hbm_gbs": float(d["hbm_gbs"]), "src": "measured (MEASURED_PEAKS.json)"}
+    except Exception:
+        return {"hbm_gbs": 6650.0, "src": "fallback (B200_PROFILING.md)"}
+
+
+# ----------------------------------------------------------------------------- algorithmic work
+def kernel_work(name: str, p, B: int, n_cand: int, n_kps: int, nq: int, n_map: int) -> tuple[str, float]:
+    """(bound, algorithmic bytes) per launch -- DESIGN.md §6 work model."""
+    W = [p.level_w[l] * p.level_h[l] for l in range(p.n_levels)]
+    if name.startswith("pyramid_l"):
+        l = int(name[len("pyramid_l"):])
+        return "hbm", float(B * (W[l - 1] + W[l]))
+    if name == "fast_cells":  # read every level once, write the candidates
+        return "hbm", float(B * sum(W) + 4 * n_cand)
+    if name == "distribute":  # read candidates, write kept keys
+        return "hbm", float(4 * n_cand + 4 * n_kps)
+    if name == "describe":  # 43x43 patch per keypoint (L2 gathers) + 52 B written per keypoint
+        return "hbm", float(n_kps * (43 * 43 + 4 + 52))
+    if name == "match_window":  # query 20 B + descriptor 32 B read, 12 B written
+        return "hbm", float(nq * 64)
+    if name == "match_resolve":
+        return "hbm", float(nq * 12)
+    if name == "brute_partial":
+        return "popc", float(n_kps) * n_map  # distances
+    return "hbm", 0.0
+
+
+# ----------------------------------------------------------------------------- our arm
+def run_ours(args, cfg):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import OrbPipeline, to_device_records
+
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    w, h = synth.SHAPES[cfg["shape"]]
+    clients = client_ids(rank, world, cfg["clients"])
+    per_client = 2 if cfg.get("stereo") else 1
+    B = len(clients) * per_client  # images per step on this rank
+    L = 8
+    Q = cfg["queries"] * len(clients)
+    window = cfg["mode"] == "window"
+    pipe = OrbPipeline(w, h, cfg["nf"], L, max_frames=B, max_queries=max(Q, 1), max_map=cfg["map"], device=local)
+    p = pipe.params
+    cap = p.kp_capacity
+    props = torch.cuda.get_device_properties(dev)
+    l2 = getattr(props, "L2_cache_size", 126 * 2 ** 20)
+    slot_bytes = B * h * w + (Q * 52 + B * cap if window else 0)
+    n_slots = int(min(256, max(4, math.ceil(2 * l2 / slot_bytes))))
+    if args.ring:
+        n_slots = args.ring
+    workers = max(1, min(32, (os.cpu_count() or 2) // max(1, world)))
+    t_setup = time.time()
+    frames_h = make_ring_frames(dict(cfg, name=args.config), clients, n_slots, workers)
+    frames = torch.from_numpy(frames_h).to(dev)  # [R, B, H, W]
+    stream = torch.cuda.Stream(dev)
+    out_rows = Q if window else B * cap
+    out = torch.zeros((max(out_rows, 1), 3), dtype=torch.int32, device=dev)
+    queries = qdesc = taken = map_desc = None
+    kp_rng = np.random.default_rng(1234 + rank)
+    if window:
+        queries = torch.zeros((n_slots, Q, 20), dtype=torch.uint8, device=dev)
+        qdesc = torch.zeros((n_slots, Q, 32), dtype=torch.uint8, device=dev)
+        taken = torch.zeros((n_slots, B, cap), dtype=torch.uint8, device=dev)
+        q_host = []
+        for s in range(n_slots):
+            with torch.cuda.stream(stream):
+                pipe.extract(frames[s], stream=stream)
+            stream.synchronize()
+            kps, desc, counts = pipe.results(B)
+            sel = list(range(0, B, per_client))  # queries against the left / mono image
+            qq, qd, tk = synth.make_queries(kps[sel], desc[sel], counts[sel], L, np.array(p.scale[:L]),
+                                            np.array(p.n_per_level[:L]), w, h, cfg["queries"], cfg["th"],
+                                            seed=synth.frame_seed(CFG_ID[args.config], 1 << 16 | rank, s),
+                                            query_dtype=ss.QUERY_DTYPE)
+            qq["frame"] = qq["frame"] * per_client
+            tk_full = np.zeros((B, cap), np.uint8)
+            tk_full[sel] = tk
+            queries[s] = to_device_records(qq, dev)
+            qdesc[s] = torch.from_numpy(qd).to(dev)
+            taken[s] = torch.from_numpy(tk_full).to(dev)
+            if s < 16:
+                q_host.append((qq, qd, tk_full))
+    else:
+        # shared map: rank 0 builds it from its clients' first-slot keypoints, broadcast once
+        with torch.cuda.stream(stream):
+            pipe.extract(frames[0], stream=stream)
+        stream.synchronize()
+        kps, desc, counts = pipe.results(B)
+        mp = synth.make_brute_map([desc[b][: counts[b][-1]] for b in range(B)], cfg["map"], seed=77,
+                                  n_from_kps=int(0.4 * cfg["map"]))
+        map_desc = torch.from_numpy(mp).to(dev)
+        if world > 1:
+            dist.broadcast(map_desc, src=0)
+        q_host = None
+    torch.cuda.synchronize(dev)
+
+    # --- one CUDA graph per ring slot, with profiling events recorded inside it
+    names = ss.extract_kernel_names(L) + (["gap"] + ss.window_kernel_names(True) if window
+                                          else ["gap"] + ss.brute_kernel_names())
+    n_ev = len(names) + 1
+    events = [[torch.cuda.Event(enable_timing=True) for _ in range(n_ev)] for _ in range(n_slots)]
+    graphs = []
+    for s in range(n_slots):
+        g = torch.cuda.CUDAGraph()
+        ss.ss_profile_events(pipe.ctx, events[s])
+        with torch.cuda.graph(g, stream=stream):
+            pipe.extract(frames[s], stream=stream)
+            if window:
+                pipe.match_window(B, queries[s], qdesc[s], out, taken=taken[s], stream=stream)
+            else:
+                pipe.match_brute(B, map_desc, out, stream=stream)
+        assert ss.ss_profile_next(pipe.ctx) == n_ev, (ss.ss_profile_next(pipe.ctx), n_ev)
+        ss.ss_profile_events(pipe.ctx, [])
+        graphs.append(g)
+    setup_s = time.time() - t_setup
+
+    # --- optional gather of per-frame results to rank 0 (map owner), off the critical path
+    gather_stream = torch.cuda.Stream(dev) if world > 1 else None
+    gathered = None
+    if world > 1:
+        slot_elems = pipe.kps[:B].numel() + pipe.desc[:B].numel() + pipe.counts[:B].numel() * 4 + out.numel() * 4
+        send = torch.zeros(slot_elems, dtype=torch.uint8, device=dev)
+        gathered = torch.zeros((world, slot_elems), dtype=torch.uint8, device=dev) if rank == 0 else None
+
+    def gather_step(done_ev):
+        gather_stream.wait_event(done_ev)
+        with torch.cuda.stream(gather_stream):
+            parts = [pipe.kps[:B].reshape(-1), pipe.desc[:B].reshape(-1), pipe.counts[:B].view(torch.uint8).reshape(-1),
+                     out.view(torch.uint8).reshape(-1)]
+            torch.cat(parts, out=send)
+            dist.gather(send, list(gathered.unbind(0)) if rank == 0 else None, dst=0)
+
+    def run_steps(s0, n):
+        for i in range(n):
+            s = (s0 + i) % n_slots
+            graphs[s].replay()
+            if world > 1:
+                ev = torch.cuda.Event()
+                ev.record(stream)
+                gather_step(ev)
+
+    W_, K = args.warmup, args.steps
+    with torch.cuda.stream(stream):
+        run_steps(0, W_)
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    sampler = ClockSampler(local)
+    with sampler:
+        torch.cuda.synchronize(dev)
+        with torch.cuda.stream(stream):
+            t0.record(stream)
+            run_steps(W_, K)
+            t1.record(stream)
+        torch.cuda.synchronize(dev)
+        if gather_stream is not None:
+            gather_stream.synchronize()
+    if world > 1:
+        dist.barrier()
+    T_ms = t0.elapsed_time(t1)
+    T_max = T_ms
+    if world > 1:
+        tt = torch.tensor([T_ms], device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        T_max = float(tt.item())
+
+    # --- per-kernel times from the graphs' last replays inside the timed region
+    timed_slots = sorted({(W_ + i) % n_slots for i in range(K)})
+    per_kernel = {n: [] for n in names}
+    step_ms = []
+    for s in timed_slots:
+        ev = events[s]
+        for i, n in enumerate(names):
+            per_kernel[n].append(ev[i].elapsed_time(ev[i + 1]))
+        step_ms.append(ev[0].elapsed_time(ev[-1]))
+    avg_us = {n: 1000.0 * float(np.mean(v)) for n, v in per_kernel.items() if n != "gap"}
+
+    # --- work model for the roofline of the dominant kernel
+    kps_h, desc_h, counts_h = pipe.results(B)  # last step's outputs
+    n_kps = int(counts_h[:, -1].sum())
+    n_cand = 0
+    for b in range(B):
+        for l in range(L):
+            n_cand += len(ss.ss_debug_candidates(pipe.ctx, b, l)[0])
+    dom = max(avg_us, key=avg_us.get)
+    bound, work = kernel_work(dom, p, B, n_cand, n_kps, Q, cfg["map"])
+    peaks = measured_peaks()
+    step_share = avg_us[dom] / (1000.0 * float(np.mean(step_ms)))
+    if bound == "hbm":
+        achieved = work / (avg_us[dom] * 1e-6) / 1e9
+        roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": achieved / peaks["hbm_gbs"], "traffic": None, "kernel": dom, "peak_src": peaks["src"],
+                "share_of_step": step_share}
+    else:
+        popc_peak = 148 * 16 * 1.965 / 8  # Tdist/s at the 1965 MHz max SM clock
+        achieved = work / (avg_us[dom] * 1e-6) / 1e12
+        roof = {"bound": "alu", "achieved": achieved, "peak": popc_peak, "unit": "Tdist/s",
+                "frac": achieved / popc_peak, "traffic": None, "kernel": dom,
+                "peak_src": "derived: 148 SM x 16 POPC/clk x clock / 8 POPC per distance", "share_of_step": step_share}
+    traffic_file = os.path.join(ROOT, "profiles", "dram_traffic_r01.json")
+    if os.path.exists(traffic_file):
+        try:
+            with open(traffic_file) as f:
+                tr = json.load(f).get(args.config, {}).get(dom)
+            if tr is not None:
+                roof["traffic"] = tr
+        except Exception:
+            pass
+
+    # --- e2e through the public API with host buffers (pinned), copies inside the timed region
+    e2e = run_e2e(args, pipe, frames_h, q_host, map_desc, out, B, Q, window, dev, stream)
+
+    frames_per_step = B * world
+    value = frames_per_step * K / (T_max / 1000.0)
+    launches_per_step = (L - 1) + 3 + (2 if window else 2)
+    res = {
+        "metric": METRIC, "value": value, "unit": "frames/s", "n_gpus": world, "steps": K, "warmup": W_,
+        "ms_per_step": T_max / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "u8", "data": "synthetic",
+        "config": {"workload": cfg["desc"], "config": args.config, "frames_per_step": frames_per_step,
+                   "images_per_step_per_gpu": B, "features_per_image": cfg["nf"],
+                   "queries_per_step_per_gpu": Q if window else 0, "map_size": cfg["map"],
+                   "parallelism": f"dp{world} (clients sharded over GPUs)",
+                   "l2": f"inputs ring of {n_slots} distinct slots = {n_slots * slot_bytes / 2**20:.0f} MiB "
+                         f"> L2 {l2 / 2**20:.0f} MiB (no flush)",
+                   "cuda_graphs": True, "setup_s": round(setup_s, 1)},
+        "latency_ms": {"p50": float(np.percentile(step_ms, 50)), "p99": float(np.percentile(step_ms, 99)),
+                       "samples": len(step_ms), "note": "per-frame latency = its tick's device time (frames of a tick are processed together)"},
+        "kernels_us": avg_us,
+        "roofline": roof,
+        "e2e": e2e,
+        "gpu_launches": launches_per_step * K * world,
+        "clocks": sampler.summary(),
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        res["cpu_baseline"] = cpu_baseline(args, cfg, frames_h, q_host, budget_s=args.cpu_budget)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    pipe.close()
+    if rank == 0:
+        print(json.dumps(res), flush=True)
+
+
+def run_e2e(args, pipe, frames_h, q_host, map_desc, out, B, Q, window, dev, stream):
+    import torch
+
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import match_records  # noqa: F401
+    n_host = min(len(frames_h), 8)
+    fr = [torch.from_numpy(frames_h[s]).pin_memory() for s in range(n_host)]
+    dfr = torch.empty_like(fr[0], device=dev)
+    if window:
+        qh = [torch.from_numpy(np.ascontiguousarray(q_host[s % len(q_host)][0]).view(np.uint8).reshape(Q, 20)).pin_memory()
+              for s in range(n_host)]
+        qdh = [torch.from_numpy(q_host[s % len(q_host)][1]).pin_memory() for s in range(n_host)]
+        tkh = [torch.from_numpy(q_host[s % len(q_host)][2]).pin_memory() for s in range(n_host)]
+        dq, dqd, dtk = (torch.empty_like(x[0], device=dev) for x in (qh, qdh, tkh))
+    kps_h = torch.empty(pipe.kps[:B].shape, dtype=torch.uint8).pin_memory()
+    desc_h = torch.empty(pipe.desc[:B].shape, dtype=torch.uint8).pin_memory()
+    cnt_h = torch.empty(pipe.counts[:B].shape, dtype=torch.int32).pin_memory()
+    out_h = torch.empty(out.shape, dtype=torch.int32).pin_memory()
+    h2d = fr[0].numel() + ((qh[0].numel() + qdh[0].numel() + tkh[0].numel()) if window else 0)
+    d2h = kps_h.numel() + desc_h.numel() + cnt_h.numel() * 4 + out_h.numel() * 4
+
+    def step(s):
+        i = s % n_host
+        dfr.copy_(fr[i], non_blocking=True)
+        if window:
+            dq.copy_(qh[i], non_blocking=True)
+            dqd.copy_(qdh[i], non_blocking=True)
+            dtk.copy_(tkh[i], non_blocking=True)
+        pipe.extract(dfr, stream=stream)
+        if window:
+            pipe.match_window(B, dq, dqd, out, taken=dtk, stream=stream)
+        else:
+            pipe.match_brute(B, map_desc, out, stream=stream)
+        kps_h.copy_(pipe.kps[:B], non_blocking=True)
+        desc_h.copy_(pipe.desc[:B], non_blocking=True)
+        cnt_h.copy_(pipe.counts[:B], non_blocking=True)
+        out_h.copy_(out, non_blocking=True)
+
+    K = max(1, min(args.steps, 200))
+    with torch.cuda.stream(stream):
+        for s in range(3):
+            step(s)
+        torch.cuda.synchronize(dev)
+        t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        t0.record(stream)
+        for s in range(K):
+            step(s)
+        t1.record(stream)
+    torch.cuda.synchronize(dev)
+    ms = t0.elapsed_time(t1)
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    return {"value": B * world * K / (ms / 1000.0), "unit": "frames/s", "h2d_bytes_per_step": int(h2d),
+            "d2h_bytes_per_step": int(d2h), "steps": K, "ms_per_step": ms / K,
+            "path": "pinned host -> H2D -> ss_orb_extract -> ss_match_projection -> D2H (C ABI, no graphs)"}
+
+
+# ----------------------------------------------------------------------------- oracle (CPU) legs
+def _oracle_job(job):
+    import oracle
+    (w, h, nf, frame, qq, qd, tk, mode, mp) = job
+    p = oracle.params(w, h, nf)
+    t = time.perf_counter()
+    kps, desc, counts = oracle.orb_extract(p, frame)
+    if mode == "window" and qq is not None:
+        q1 = qq.copy()
+        q1["frame"] = 0
+        oracle.match_window(p, kps[None], desc[None], counts[None], tk[None], q1, qd)
+    elif mode == "brute" and mp is not None:
+        oracle.match_brute(p, desc[None], counts[None], mp, k0=0, k1=4)
+    return time.perf_counter() - t
+
+
+def _jobs_for(cfg, frames_h, q_host, n, w, h, mp=None):
+    jobs = []
+    S, Bimg = frames_h.shape[:2]
+    per_client = 2 if cfg.get("stereo") else 1
+    i = 0
+    while len(jobs) < n:
+        s, b = (i // Bimg) % S, i % Bimg
+        qq = qd = tk = None
+        if cfg["mode"] == "window" and q_host and b % per_client == 0:
+            qs, qds, tks = q_host[s % len(q_host)]
+            c = b // per_client
+            sel = qs["frame"] == b
+            qq, qd, tk = qs[sel], qds[sel], tks[b]
+            _ = c
+        jobs.append((w, h, cfg["nf"], frames_h[s, b], qq, qd, tk, cfg["mode"], mp))
+        i += 1
+    return jobs
+
+
+def cpu_baseline(args, cfg, frames_h, q_host, budget_s=15.0, mp=None):
+    import multiprocessing as mpx
+
+    import oracle
+    oracle.build()
+    w, h = synth.SHAPES[cfg["shape"]]
+    cores = len(os.sched_getaffinity(0))
+    probe = _oracle_job(_jobs_for(cfg, frames_h, q_host, 1, w, h, mp)[0])
+    n = max(cores, int(budget_s * cores / max(probe, 1e-3)))
+    jobs = _jobs_for(cfg, frames_h, q_host, n, w, h, mp)
+    t = time.perf_counter()
+    with mpx.get_context("fork").Pool(cores) as pool:
+        per = pool.map(_oracle_job, jobs, chunksize=1)
+    wall = time.perf_counter() - t
+    return {"value": len(jobs) / wall, "unit": "frames/s", "cores": cores, "kind": "oracle",
+            "sample": f"{len(jobs)} frames of the {args.config} workload (extract + its {cfg['queries']} "
+                      f"{cfg['mode']} queries each), one single-threaded oracle process per core",
+            "median_frame_s_single_core": float(np.median(per)),
+            "cpu": _cpu_model()}
+
+
+def _cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+def run_reference(args, cfg):
+    """The CPU oracle as the reference arm: each step = one bounded sample of the workload."""
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    if rank != 0:
+        return
+    import multiprocessing as mpx
+
+    import oracle
+    oracle.build()
+    w, h = synth.SHAPES[cfg["shape"]]
+    clients = client_ids(0, 1, cfg["clients"])
+    frames_h = make_ring_frames(dict(cfg, name=args.config), clients, 2, max(1, os.cpu_count() or 1))
+    q_host = None
+    mp = None
+    if cfg["mode"] == "window":
+        p = oracle.params(w, h, cfg["nf"])
+        q_host = []
+        per_client = 2 if cfg.get("stereo") else 1
+        for s in range(frames_h.shape[0]):
+            kps, desc, counts = oracle.orb_extract_batch(p, frames_h[s][::per_client])
+            qq, qd, tk = synth.make_queries(kps, desc, counts, 8, np.array(p.scale[:8]), np.array(p.n_per_level[:8]),
+                                            w, h, cfg["queries"], cfg["th"],
+                                            seed=synth.frame_seed(CFG_ID[args.config], 1 << 16, s),
+                                            query_dtype=oracle.QUERY_DTYPE)
+            qq["frame"] = qq["frame"] * per_client
+            tkf = np.zeros((frames_h.shape[1], p.kp_capacity), np.uint8)
+            tkf[::per_client] = tk
+            q_host.append((qq, qd, tkf))
+    else:
+        p = oracle.params(w, h, cfg["nf"])
+        kps, desc, counts = oracle.orb_extract_batch(p, frames_h[0])
+        mp = synth.make_brute_map([desc[b][: counts[b][-1]] for b in range(len(desc))], cfg["map"], seed=77,
+                                  n_from_kps=int(0.4 * cfg["map"]))
+    cores = len(os.sched_getaffinity(0))
+    B = frames_h.shape[1]
+    probe = _oracle_job(_jobs_for(cfg, frames_h, q_host, 1, w, h, mp)[0])
+    # frames per step: the tick's B frames, reduced so that the whole run stays within ~3 minutes
+    per_step_budget = 170.0 / max(1, args.steps + args.warmup)
+    n_frames = int(max(1, min(B, per_step_budget * cores / max(probe, 1e-3))))
+    jobs_all = _jobs_for(cfg, frames_h, q_host, n_frames * (args.steps + args.warmup), w, h, mp)
+    times = []
+    with mpx.get_context("fork").Pool(min(cores, n_frames)) as pool:
+        for s in range(args.warmup + args.steps):
+            jobs = jobs_all[s * n_frames:(s + 1) * n_frames]
+            t = time.perf_counter()
+            pool.map(_oracle_job, jobs, chunksize=1)
+            if s >= args.warmup:
+                times.append(time.perf_counter() - t)
+    T = sum(times)
+    value = n_frames * len(times) / T
+    res = {"impl": "reference", "metric": METRIC, "value": value, "unit": "frames/s", "n_gpus": world,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * T / len(times),
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+           "config": {"workload": cfg["desc"], "config": args.config, "frames_per_step": n_frames,
+                      "parallelism": "CPU oracle, one single-threaded process per core"},
+           "cpu_baseline": {"value": value, "unit": "frames/s", "cores": min(cores, n_frames), "kind": "oracle",
+                            "sample": f"{n_frames} of the tick's {B} frames per step (extract + "
+                                      f"{cfg['queries']} {cfg['mode']} queries each)", "cpu": _cpu_model()},
+           "e2e": {"value": value, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(res), flush=True)
+
+
+def main(argv=None):
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", choices=sorted(CONFIGS), default="c2")
+    ap.add_argument("--ring", type=int, default=0, help="override the number of input ring slots")
+    ap.add_argument("--cpu-budget", type=float, default=15.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args(argv)
+    assert args.warmup >= 3, "at least 3 warm-up steps"
+    cfg = CONFIGS[args.config]
+    if args.impl == "reference":
+        run_reference(args, cfg)
+    else:
+        run_ours(args, cfg)
+
+
+if __name__ == "__main__":
+    main()

@@ -148,6 +148,20 @@ ss_status ss_match_projection(ss_ctx* ctx, int32_t n_frames, const ss_keypoint* 
                               const ss_mp_query* d_queries, const uint8_t* d_map_desc, int32_t n_map,
                               const ss_match_cfg* cfg, ss_match* d_out, ss_stream_t stream);
 
+/* ---- profiling hook (bench.py; does not synchronise) ---- */
+
+/* When n_events > 0, every following ss_orb_extract / ss_match_projection records the
+ * caller's events (cudaEvent_t handles created with timing enabled; host array copied) on
+ * its stream: the next unused event before its first operation, then one after every
+ * kernel it launches, continuing across calls until the next ss_profile_events call
+ * (n_events = 0 disables; events beyond n_events are not recorded).  Kernel order:
+ * extract = pyramid level 1..L-1, fast_cells, distribute, describe; WINDOW match =
+ * match_window[, match_resolve if dedup]; BRUTE = brute_partial, brute_merge.  Works
+ * under CUDA-graph stream capture (the records become graph event nodes).
+ * *next_index (may be NULL) receives the index of the next event to be recorded. */
+ss_status ss_profile_events(ss_ctx* ctx, void* const* events, int32_t n_events);
+ss_status ss_profile_next(ss_ctx* ctx, int32_t* next_index);
+
 /* ---- debug / test hooks (synchronise the ctx's device; not for the hot path) ---- */
 
 /* Device pointer + pitch of pyramid level `level` (>= 1) of frame slot `frame` as left by the

@@ -192,25 +192,38 @@ cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* 
     cudaError_t e = cudaMemsetAsync(claim, 0xFF, (size_t)n_frames * g.kp_capacity * sizeof(unsigned long long), s);
     if (e != cudaSuccess) return e;
   }
-  const int blocks = (n_queries + 255) / 256;
-  match_window_kernel<<<blocks, 256, 0, s>>>(g, n_frames, kps, desc, counts, taken, n_queries, q, qdesc, cfg, claim,
-                                             out);
-  if (cfg.dedup) match_window_resolve<<<blocks, 256, 0, s>>>(n_queries, q, g.kp_capacity, claim, out);
+  match_window_kernel<<<(n_queries + 255) / 256, 256, 0, s>>>(g, n_frames, kps, desc, counts, taken, n_queries, q,
+                                                              qdesc, cfg, claim, out);
   return cudaGetLastError();
 }
 
-cudaError_t launch_match_brute(const Geom& g, int n_frames, const uint8_t* desc, const int32_t* counts, int n_map,
-                               const uint8_t* map_desc, ss_match_cfg cfg, unsigned long long* partial, int max_splits,
-                               ss_match* out, cudaStream_t s) {
+cudaError_t launch_match_resolve(const Geom& g, int n_queries, const ss_mp_query* q, const unsigned long long* claim,
+                                 ss_match* out, cudaStream_t s) {
+  if (n_queries <= 0) return cudaSuccess;
+  match_window_resolve<<<(n_queries + 255) / 256, 256, 0, s>>>(n_queries, q, g.kp_capacity, claim, out);
+  return cudaGetLastError();
+}
+
+int brute_splits(const Geom& g, int n_frames, int n_map, int max_splits) {
   const int nslots = n_frames * g.kp_capacity;
-  if (nslots <= 0) return cudaSuccess;
   const int qblocks = (nslots + BQ - 1) / BQ;
   // enough CTAs for ~4 waves on 148 SMs, each split >= one tile
   int splits = (4 * 148 + qblocks - 1) / qblocks;
   splits = max(1, min(splits, max_splits));
-  splits = max(1, min(splits, (n_map + BTILE - 1) / BTILE));
-  dim3 grid(qblocks, splits);
+  return max(1, min(splits, (n_map + BTILE - 1) / BTILE));
+}
+
+cudaError_t launch_brute_partial(const Geom& g, int n_frames, const uint8_t* desc, const int32_t* counts, int n_map,
+                                 const uint8_t* map_desc, int splits, unsigned long long* partial, cudaStream_t s) {
+  const int nslots = n_frames * g.kp_capacity;
+  dim3 grid((nslots + BQ - 1) / BQ, splits);
   match_brute_partial<<<grid, BQ, 0, s>>>(g, n_frames, desc, counts, n_map, map_desc, splits, partial);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_brute_merge(const Geom& g, int n_frames, const int32_t* counts, int splits,
+                               const unsigned long long* partial, ss_match_cfg cfg, ss_match* out, cudaStream_t s) {
+  const int nslots = n_frames * g.kp_capacity;
   match_brute_merge<<<(nslots + 255) / 256, 256, 0, s>>>(g, n_frames, counts, splits, partial, cfg, out);
   return cudaGetLastError();
 }

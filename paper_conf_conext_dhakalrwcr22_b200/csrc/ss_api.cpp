@@ -136,6 +136,9 @@ struct ss_ctx {
   int8_t* pattern = nullptr;
   unsigned long long* claim = nullptr;
   unsigned long long* partial = nullptr;
+  // profiling hook
+  std::vector<cudaEvent_t> prof;
+  size_t prof_next = 0;
   // last extract (debug hooks)
   const uint8_t* last_frames = nullptr;
   int64_t last_stride = 0;
@@ -144,6 +147,10 @@ struct ss_ctx {
 };
 
 namespace {
+
+inline void prof_mark(ss_ctx* c, cudaStream_t s) {
+  if (c->prof_next < c->prof.size()) cudaEventRecord(c->prof[c->prof_next++], s);
+}
 
 void free_ctx(ss_ctx* c) {
   if (!c) return;
@@ -342,13 +349,19 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   const Geom& g = c->g;
   FrameSrc src{d_frames, frame_stride, pitch, c->pyr};
+  prof_mark(c, s);
   SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 2, s));
-  for (int l = 1; l < g.L; l++)
+  for (int l = 1; l < g.L; l++) {
     SS_CUDA_TRY(launch_pyramid_level(g, l, n_frames, src, c->xytab + c->xoff[l], c->xytab + c->yoff[l], s));
+    prof_mark(c, s);
+  }
   SS_CUDA_TRY(launch_fast_cells(g, n_frames, src, c->cells, c->slots, c->cell_counts, s));
+  prof_mark(c, s);
   SS_CUDA_TRY(launch_distribute(g, n_frames, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
                                 c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, s));
+  prof_mark(c, s);
   SS_CUDA_TRY(launch_describe(g, n_frames, src, c->selected, c->sel_counts, c->pattern, d_kps, d_desc, d_counts, s));
+  prof_mark(c, s);
   c->last_frames = d_frames;
   c->last_stride = frame_stride;
   c->last_pitch = pitch;
@@ -370,8 +383,15 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
   if (cfg->mode == SS_MATCH_WINDOW) {
     if (n_queries > c->max_queries) return fail(SS_ECAPACITY, "n_queries exceeds the ctx's max_queries");
     if (n_queries > 0 && (!d_queries || !d_map_desc)) return fail(SS_EINVAL, "NULL queries");
+    if (n_queries == 0) return SS_OK;
+    prof_mark(c, s);
     SS_CUDA_TRY(launch_match_window(c->g, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_queries, d_queries,
                                     d_map_desc, *cfg, c->claim, d_out, s));
+    prof_mark(c, s);
+    if (cfg->dedup) {
+      SS_CUDA_TRY(launch_match_resolve(c->g, n_queries, d_queries, c->claim, d_out, s));
+      prof_mark(c, s);
+    }
     return SS_OK;
   }
   if (cfg->mode == SS_MATCH_BRUTE) {
@@ -379,11 +399,29 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
     if (n_map > c->max_map) return fail(SS_ECAPACITY, "n_map exceeds the ctx's max_map");
     if (n_map > 0 && !d_map_desc) return fail(SS_EINVAL, "NULL map");
     if (n_frames == 0) return SS_OK;
-    SS_CUDA_TRY(launch_match_brute(c->g, n_frames, d_desc, d_counts, n_map, d_map_desc, *cfg, c->partial,
-                                   c->max_splits, d_out, s));
+    const int splits = brute_splits(c->g, n_frames, n_map, c->max_splits);
+    prof_mark(c, s);
+    SS_CUDA_TRY(launch_brute_partial(c->g, n_frames, d_desc, d_counts, n_map, d_map_desc, splits, c->partial, s));
+    prof_mark(c, s);
+    SS_CUDA_TRY(launch_brute_merge(c->g, n_frames, d_counts, splits, c->partial, *cfg, d_out, s));
+    prof_mark(c, s);
     return SS_OK;
   }
   return fail(SS_EINVAL, "unknown match mode");
+}
+
+ss_status ss_profile_events(ss_ctx* c, void* const* events, int32_t n_events) {
+  if (!c || n_events < 0 || (n_events > 0 && !events)) return fail(SS_EINVAL, "bad profiling events");
+  c->prof.assign(n_events, nullptr);
+  for (int i = 0; i < n_events; i++) c->prof[i] = reinterpret_cast<cudaEvent_t>(events[i]);
+  c->prof_next = 0;
+  return SS_OK;
+}
+
+ss_status ss_profile_next(ss_ctx* c, int32_t* next_index) {
+  if (!c) return fail(SS_EINVAL, "NULL ctx");
+  if (next_index) *next_index = (int32_t)c->prof_next;
+  return SS_OK;
 }
 
 ss_status ss_debug_level(ss_ctx* c, int32_t frame, int32_t level, const uint8_t** d_ptr, int32_t* pitch) {

@@ -83,9 +83,15 @@ cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* 
                                 const int32_t* counts, const uint8_t* taken, int n_queries,
                                 const ss_mp_query* q, const uint8_t* qdesc, ss_match_cfg cfg,
                                 unsigned long long* claim, ss_match* out, cudaStream_t s);
-cudaError_t launch_match_brute(const Geom& g, int n_frames, const uint8_t* desc, const int32_t* counts,
-                               int n_map, const uint8_t* map_desc, ss_match_cfg cfg,
-                               unsigned long long* partial, int max_splits, ss_match* out, cudaStream_t s);
+cudaError_t launch_match_resolve(const Geom& g, int n_queries, const ss_mp_query* q,
+                                 const unsigned long long* claim, ss_match* out, cudaStream_t s);
+int brute_splits(const Geom& g, int n_frames, int n_map, int max_splits);
+cudaError_t launch_brute_partial(const Geom& g, int n_frames, const uint8_t* desc, const int32_t* counts,
+                                 int n_map, const uint8_t* map_desc, int splits, unsigned long long* partial,
+                                 cudaStream_t s);
+cudaError_t launch_brute_merge(const Geom& g, int n_frames, const int32_t* counts, int splits,
+                               const unsigned long long* partial, ss_match_cfg cfg, ss_match* out,
+                               cudaStream_t s);
 
 // Overflow scratch bytes the distribution needs for a level with `slots` candidate slots.
 int64_t distribute_ovf_bytes(int64_t slots);

@@ -80,15 +80,19 @@ def lib():
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
         L.ss_debug_candidates.argtypes = [P, i32, i32, P, P, P, i32, C.POINTER(i32)]
         L.ss_debug_overflow_count.argtypes = [P, C.POINTER(i32)]
+        L.ss_profile_events.argtypes = [P, C.POINTER(P), i32]
+        L.ss_profile_next.argtypes = [P, C.POINTER(i32)]
         for fn in ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_orb_extract", "ss_match_projection",
-                   "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count"):
+                   "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
+                   "ss_profile_next"):
             getattr(L, fn).restype = C.c_int
         _lib = L
     return _lib
 
 
 EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "ss_orb_extract",
-            "ss_match_projection", "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count")
+            "ss_match_projection", "ss_profile_events", "ss_profile_next", "ss_debug_level",
+            "ss_debug_candidates", "ss_debug_overflow_count")
 
 
 def _check(status: int, ctx=None):
@@ -147,6 +151,32 @@ def ss_match_projection(ctx, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_qu
     _check(lib().ss_match_projection(ctx, n_frames, _ptr(d_kps), _ptr(d_desc), _ptr(d_counts),
                                      _ptr(d_kp_taken), n_queries, _ptr(d_queries), _ptr(d_map_desc), n_map,
                                      C.byref(cfg), _ptr(d_out), _stream(stream)), ctx)
+
+
+def ss_profile_events(ctx, events) -> None:
+    """events: list of torch.cuda.Event (timing enabled) or raw cudaEvent_t ints; [] disables."""
+    handles = [e if isinstance(e, int) else e.cuda_event for e in events]
+    arr = (C.c_void_p * max(1, len(handles)))(*handles)
+    _check(lib().ss_profile_events(ctx, arr, len(handles)), ctx)
+
+
+def ss_profile_next(ctx) -> int:
+    n = C.c_int32()
+    _check(lib().ss_profile_next(ctx, C.byref(n)), ctx)
+    return n.value
+
+
+def extract_kernel_names(n_levels: int) -> list[str]:
+    """Names of the intervals between consecutive profiling events of one extract call."""
+    return [f"pyramid_l{l}" for l in range(1, n_levels)] + ["fast_cells", "distribute", "describe"]
+
+
+def window_kernel_names(dedup: bool = True) -> list[str]:
+    return ["match_window"] + (["match_resolve"] if dedup else [])
+
+
+def brute_kernel_names() -> list[str]:
+    return ["brute_partial", "brute_merge"]
 
 
 def ss_debug_level(ctx, frame, level):
