@@ -55,6 +55,25 @@ def client_ids(rank: int, world: int, clients_per_rank: int) -> list[int]:
     return list(range(rank * clients_per_rank, (rank + 1) * clients_per_rank))
 
 
+def pack_results(parts) -> "torch.Tensor":
+    """Flatten one tick's per-frame results (uint8 views) into one send slot."""
+    import torch
+    return torch.cat([t.reshape(-1).view(torch.uint8) for t in parts])
+
+
+def gather_to_owner(send, rank: int, world: int):
+    """Per-tick result hand-off to the map-owning rank 0 (north_star: NCCL gather off the
+    critical path; gloo on CPU in tests).  Returns the per-rank slots on rank 0, else None."""
+    import torch
+    import torch.distributed as dist
+    if rank == 0:
+        bufs = [torch.empty_like(send) for _ in range(world)]
+        dist.gather(send, bufs, dst=0)
+        return bufs
+    dist.gather(send, None, dst=0)
+    return None
+
+
 def _gen_frame(args):
     w, h, seed, stereo = args
     if stereo:
@@ -266,19 +285,12 @@ def run_ours(args, cfg):
 
     # --- optional gather of per-frame results to rank 0 (map owner), off the critical path
     gather_stream = torch.cuda.Stream(dev) if world > 1 else None
-    gathered = None
-    if world > 1:
-        slot_elems = pipe.kps[:B].numel() + pipe.desc[:B].numel() + pipe.counts[:B].numel() * 4 + out.numel() * 4
-        send = torch.zeros(slot_elems, dtype=torch.uint8, device=dev)
-        gathered = torch.zeros((world, slot_elems), dtype=torch.uint8, device=dev) if rank == 0 else None
 
     def gather_step(done_ev):
+        # side stream: waits for the tick, packs its results and gathers them to rank 0
         gather_stream.wait_event(done_ev)
         with torch.cuda.stream(gather_stream):
-            parts = [pipe.kps[:B].reshape(-1), pipe.desc[:B].reshape(-1), pipe.counts[:B].view(torch.uint8).reshape(-1),
-                     out.view(torch.uint8).reshape(-1)]
-            torch.cat(parts, out=send)
-            dist.gather(send, list(gathered.unbind(0)) if rank == 0 else None, dst=0)
+            gather_to_owner(pack_results([pipe.kps[:B], pipe.desc[:B], pipe.counts[:B], out]), rank, world)
 
     def run_steps(s0, n):
         for i in range(n):

@@ -60,7 +60,9 @@ def build(force: bool = False, verbose: bool = False) -> str:
                 sys.stderr.write(log)
     if force or jobs or not _newer(LIB, objs):
         tmp = LIB + f".tmp{os.getpid()}"
-        run([nvcc] + ARCH + ["-shared", "-cudart", "static", "-o", tmp] + objs)
+        # dynamic cudart: the process must share ONE runtime with torch, otherwise stream handles
+        # created by torch are "invalid resource handle" inside libss
+        run([nvcc] + ARCH + ["-shared", "-cudart", "shared", "-o", tmp] + objs)
         os.replace(tmp, LIB)
     return LIB
 

@@ -148,6 +148,14 @@ struct ss_ctx {
 
 namespace {
 
+// Clears any stale error left in this thread by unrelated runtime calls (so that a launch
+// check reports only our own launches) and validates the caller's stream handle.
+cudaError_t check_stream(cudaStream_t s) {
+  (void)cudaGetLastError();
+  unsigned int flags = 0;
+  return cudaStreamGetFlags(s, &flags);
+}
+
 inline void prof_mark(ss_ctx* c, cudaStream_t s) {
   if (c->prof_next < c->prof.size()) cudaEventRecord(c->prof[c->prof_next++], s);
 }
@@ -347,6 +355,7 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   if (n_frames > 1 && frame_stride < (int64_t)pitch * c->g.H) return fail(SS_EINVAL, "frame_stride < height*pitch");
   SS_CUDA_TRY(cudaSetDevice(c->device));
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  SS_CUDA_TRY(check_stream(s));
   const Geom& g = c->g;
   FrameSrc src{d_frames, frame_stride, pitch, c->pyr};
   prof_mark(c, s);
@@ -380,6 +389,7 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
   if (!d_kps || !d_desc || !d_counts || !d_out) return fail(SS_EINVAL, "NULL buffer");
   SS_CUDA_TRY(cudaSetDevice(c->device));
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  SS_CUDA_TRY(check_stream(s));
   if (cfg->mode == SS_MATCH_WINDOW) {
     if (n_queries > c->max_queries) return fail(SS_ECAPACITY, "n_queries exceeds the ctx's max_queries");
     if (n_queries > 0 && (!d_queries || !d_map_desc)) return fail(SS_EINVAL, "NULL queries");

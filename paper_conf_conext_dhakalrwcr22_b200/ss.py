@@ -68,6 +68,10 @@ def lib():
     if _lib is None:
         if not os.path.exists(LIB_PATH):
             raise ImportError(f"libss.so not built ({LIB_PATH}); run __graft_entry__.build()")
+        try:  # load torch's libcudart first so that libss binds to the same CUDA runtime
+            import torch  # noqa: F401
+        except Exception:
+            pass
         L = C.CDLL(LIB_PATH)
         P, i32, i64 = C.c_void_p, C.c_int32, C.c_int64
         L.ss_orb_params_init.argtypes = [i32, i32, i32, i32, C.c_float, i32, i32, C.POINTER(ss_orb_params)]
