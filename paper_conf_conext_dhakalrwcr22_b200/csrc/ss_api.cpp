@@ -148,12 +148,12 @@ struct ss_ctx {
 
 namespace {
 
-// Clears any stale error left in this thread by unrelated runtime calls (so that a launch
-// check reports only our own launches) and validates the caller's stream handle.
-cudaError_t check_stream(cudaStream_t s) {
+// Clears any stale error left in this thread by unrelated runtime calls, so that the launch
+// checks report only our own launches.  (No stream query here: it is illegal while the caller
+// captures the stream into a CUDA graph.)
+cudaError_t check_stream(cudaStream_t) {
   (void)cudaGetLastError();
-  unsigned int flags = 0;
-  return cudaStreamGetFlags(s, &flags);
+  return cudaSuccess;
 }
 
 inline void prof_mark(ss_ctx* c, cudaStream_t s) {
