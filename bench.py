@@ -268,6 +268,10 @@ def run_ours(args, cfg):
                                           else ["gap"] + ss.brute_kernel_names())
     n_ev = len(names) + 1
     events = [[torch.cuda.Event(enable_timing=True) for _ in range(n_ev)] for _ in range(n_slots)]
+    for evs in events:  # torch creates the CUDA event lazily, at its first record
+        for e in evs:
+            e.record(stream)
+    stream.synchronize()
     graphs = []
     for s in range(n_slots):
         g = torch.cuda.CUDAGraph()

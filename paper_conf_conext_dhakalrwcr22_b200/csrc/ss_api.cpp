@@ -422,6 +422,8 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
 
 ss_status ss_profile_events(ss_ctx* c, void* const* events, int32_t n_events) {
   if (!c || n_events < 0 || (n_events > 0 && !events)) return fail(SS_EINVAL, "bad profiling events");
+  for (int i = 0; i < n_events; i++)
+    if (!events[i]) return fail(SS_EINVAL, "NULL event handle (torch creates events lazily: record once first)");
   c->prof.assign(n_events, nullptr);
   for (int i = 0; i < n_events; i++) c->prof[i] = reinterpret_cast<cudaEvent_t>(events[i]);
   c->prof_next = 0;

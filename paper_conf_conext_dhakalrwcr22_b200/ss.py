@@ -160,6 +160,8 @@ def ss_match_projection(ctx, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_qu
 def ss_profile_events(ctx, events) -> None:
     """events: list of torch.cuda.Event (timing enabled) or raw cudaEvent_t ints; [] disables."""
     handles = [e if isinstance(e, int) else e.cuda_event for e in events]
+    if any(not h for h in handles):
+        raise SSError(SS_EINVAL, "event not created yet (record a torch.cuda.Event once before passing it)")
     arr = (C.c_void_p * max(1, len(handles)))(*handles)
     _check(lib().ss_profile_events(ctx, arr, len(handles)), ctx)
 
