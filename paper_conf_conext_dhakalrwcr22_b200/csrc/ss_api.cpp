@@ -157,7 +157,9 @@ cudaError_t check_stream(cudaStream_t) {
 }
 
 inline void prof_mark(ss_ctx* c, cudaStream_t s) {
-  if (c->prof_next < c->prof.size()) cudaEventRecord(c->prof[c->prof_next++], s);
+  // External: under stream capture the record becomes a real graph event node (a plain
+  // record would only be a capture-internal dependency and could not be timed).
+  if (c->prof_next < c->prof.size()) cudaEventRecordWithFlags(c->prof[c->prof_next++], s, cudaEventRecordExternal);
 }
 
 void free_ctx(ss_ctx* c) {
