@@ -120,8 +120,10 @@ struct ss_ctx {
   Geom g{};
   int max_frames = 0, max_queries = 0, max_map = 0, max_splits = 0;
   std::vector<CellInfo> cells_h;
+  std::vector<BandInfo> bands_h;
   // device scratch
   CellInfo* cells = nullptr;
+  BandInfo* bands = nullptr;
   uint32_t* xytab = nullptr;  // per level l >= 1: xtab [w_l], ytab [h_l]
   std::vector<int64_t> xoff, yoff;
   uint8_t* pyr = nullptr;
@@ -165,7 +167,7 @@ inline void prof_mark(ss_ctx* c, cudaStream_t s) {
 void free_ctx(ss_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->device);
-  void* ptrs[] = {c->cells, c->xytab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
+  void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
                   c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial};
   for (void* q : ptrs)
     if (q) cudaFree(q);
@@ -277,14 +279,45 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   }
   g.pyr_frame_bytes = poff;
   g.total_cells = (int)c->cells_h.size();
+  // bands = rows of cells (same level and detect rows), biggest levels first in the grid
+  g.max_band_w = g.max_band_h = g.max_cell_w = 0;
+  for (size_t i = 0; i < c->cells_h.size(); i++) {
+    const CellInfo& ci = c->cells_h[i];
+    g.max_cell_w = imax(g.max_cell_w, ci.x1 - ci.x0);
+    if (c->bands_h.empty() || c->bands_h.back().level != ci.level || c->bands_h.back().y0 != ci.y0) {
+      BandInfo b;
+      b.level = ci.level;
+      b.y0 = ci.y0;
+      b.y1 = ci.y1;
+      b.x0 = ci.x0;
+      b.x1 = ci.x1;
+      b.cell_first = (int)i;
+      b.ncells = 0;
+      b.pad = 0;
+      c->bands_h.push_back(b);
+    }
+    BandInfo& b = c->bands_h.back();
+    if (ci.x0 != b.x1 && b.ncells > 0) {
+      free_ctx(c);
+      return fail(SS_EUNSUPPORTED, "FAST cell windows of a row do not tile");
+    }
+    b.x1 = ci.x1;
+    b.ncells++;
+    g.max_band_w = imax(g.max_band_w, b.x1 - b.x0);
+    g.max_band_h = imax(g.max_band_h, b.y1 - b.y0);
+  }
+  g.total_bands = (int)c->bands_h.size();
+  {
+    int rp, mbw, rb, mb, nb;
+    if (fast_smem_bytes(g, &rp, &mbw, &rb, &mb, &nb) > 227 * 1024) {
+      free_ctx(c);
+      return fail(SS_EUNSUPPORTED, "a FAST band does not fit in shared memory");
+    }
+  }
   g.slots_per_frame = slot_off;
   g.kp_capacity = q.kp_capacity;
   g.max_rw = max_rw;
   g.max_rh = max_rh;
-  if (max_rw > 64 || max_rh > 64) {
-    free_ctx(c);
-    return fail(SS_EUNSUPPORTED, "FAST cell larger than 58x58 px");
-  }
   // coefficient tables for levels >= 1
   std::vector<uint32_t> tab;
   c->xoff.assign(L, 0);
@@ -312,6 +345,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
 #define ALLOC(ptr, bytes)                          \
   if (e == cudaSuccess) e = dalloc(&(ptr), (bytes));
   ALLOC(c->cells, sizeof(CellInfo) * c->cells_h.size());
+  ALLOC(c->bands, sizeof(BandInfo) * c->bands_h.size());
   ALLOC(c->xytab, sizeof(uint32_t) * tab.size());
   ALLOC(c->pyr, F * g.pyr_frame_bytes);
   ALLOC(c->slots, sizeof(uint32_t) * F * g.slots_per_frame);
@@ -326,6 +360,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (max_map > 0) ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
 #undef ALLOC
   if (e == cudaSuccess) e = cudaMemcpy(c->cells, c->cells_h.data(), sizeof(CellInfo) * c->cells_h.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(c->bands, c->bands_h.data(), sizeof(BandInfo) * c->bands_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess && !tab.empty()) e = cudaMemcpy(c->xytab, tab.data(), sizeof(uint32_t) * tab.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->ovf_level_off, ovf_off.data(), sizeof(int64_t) * L, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->pattern, pat.data(), 1024, cudaMemcpyHostToDevice);
@@ -366,7 +401,7 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
     SS_CUDA_TRY(launch_pyramid_level(g, l, n_frames, src, c->xytab + c->xoff[l], c->xytab + c->yoff[l], s));
     prof_mark(c, s);
   }
-  SS_CUDA_TRY(launch_fast_cells(g, n_frames, src, c->cells, c->slots, c->cell_counts, s));
+  SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands, c->cells, c->slots, c->cell_counts, s));
   prof_mark(c, s);
   SS_CUDA_TRY(launch_distribute(g, n_frames, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
                                 c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, s));

@@ -24,6 +24,17 @@ struct CellInfo {
   int32_t pad;
 };
 
+// One row of FAST cells of one level ("band"): the cells' detect windows share rows
+// [y0, y1) and tile columns [x0, x1); cells [cell_first, cell_first + ncells) of the table.
+struct BandInfo {
+  int32_t level;
+  int32_t y0, y1;
+  int32_t x0, x1;
+  int32_t cell_first;
+  int32_t ncells;
+  int32_t pad;
+};
+
 // Everything the kernels need to know about the frame shape, by value in kernel params.
 struct Geom {
   int32_t L, W, H;
@@ -47,6 +58,9 @@ struct Geom {
   int32_t qw[kMaxLevels], qh[kMaxLevels];  // quadtree box (maxBorder - minBorder)
   int32_t qrounds[kMaxLevels];      // quadtree rounds that can still separate keys on level l
   int32_t max_rw, max_rh;           // largest FAST input region (D + 3-px halo) of any cell
+  int32_t total_bands;              // rows of FAST cells over all levels, per frame
+  int32_t max_band_w, max_band_h;   // widest band (detect columns) / tallest band (detect rows)
+  int32_t max_cell_w;               // widest cell detect window
 };
 
 // Where the frames of one call live.  Level 0 is the caller's frame (no copy).
@@ -68,8 +82,9 @@ __host__ __device__ inline int key_m(uint32_t k) { return (int)(k & 0xFF); }
 // ---- launchers (one per kernel; each returns cudaGetLastError()) ----
 cudaError_t launch_pyramid_level(const Geom& g, int level, int n_frames, FrameSrc src,
                                  const uint32_t* xtab, const uint32_t* ytab, cudaStream_t s);
-cudaError_t launch_fast_cells(const Geom& g, int n_frames, FrameSrc src, const CellInfo* cells,
-                              uint32_t* slots, int32_t* cell_counts, cudaStream_t s);
+cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands,
+                              const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s);
+size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int* mband_bytes, int* nball);
 cudaError_t launch_distribute(const Geom& g, int n_frames, const CellInfo* cells, const uint32_t* slots,
                               const int32_t* cell_counts, uint32_t* selected, int32_t* sel_counts,
                               uint8_t* ovf, int64_t ovf_frame_bytes, const int64_t* ovf_level_off,
