@@ -19,7 +19,7 @@ namespace {
 
 constexpr int DESC_WARPS = 8;
 constexpr int PR = 43;  // raw patch: radius 21 (18 max sample offset + 3 blur taps)
-constexpr int PP = 44;
+constexpr int PP = 64;  // raw patch pitch: a 16-B aligned 64-B window covers the 43 B row
 constexpr int BR = 37;  // blurred patch: radius 18
 constexpr int HP = 37;  // pitch (u16) of the horizontal pass [43][37]
 constexpr int BP = 40;
@@ -84,13 +84,27 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
     ip = g.pitch[l];
   }
   const int w = g.w[l], h = g.h[l];
-  uint8_t* P = sm + warp * PER_WARP;
-  uint16_t* Hs = reinterpret_cast<uint16_t*>(P + PR * PP);
+  uint8_t* Pw = sm + warp * PER_WARP;
+  uint16_t* Hs = reinterpret_cast<uint16_t*>(Pw + PR * PP);
   uint8_t* B = reinterpret_cast<uint8_t*>(Hs + PR * HP);
-  // raw patch, REFLECT_101 outside the level
-  for (int r = 0; r < PR; r++) {
-    const uint8_t* row = img + (int64_t)reflect101(ly - 21 + r, h) * ip;
-    for (int c = lane; c < PR; c += 32) P[r * PP + c] = __ldg(row + reflect101(lx - 21 + c, w));
+  const uint8_t* p0 = img + (int64_t)(ly - 21) * ip + (lx - 21);
+  const int sh = (int)(reinterpret_cast<uintptr_t>(p0) & 15);
+  const uint8_t* P;  // P[r * PP + c] = raw patch pixel (ly - 21 + r, lx - 21 + c)
+  if ((ip & 15) == 0 && lx >= 21 && ly >= 21 && ly + 21 < h && lx - 21 - sh + 64 <= ip) {
+    // interior: 43 rows x four aligned 16-B chunks, all loads in flight at once
+    const uint4* base = reinterpret_cast<const uint4*>(p0 - sh);
+    for (int i = lane; i < PR * 4; i += 32) {
+      const int r = i >> 2, c = i & 3;
+      *reinterpret_cast<uint4*>(Pw + r * PP + 16 * c) = __ldg(base + (int64_t)r * (ip >> 4) + c);
+    }
+    P = Pw + sh;
+  } else {
+    // near the level border: REFLECT_101 (the blur's border rule), byte loads
+    for (int i = lane; i < PR * PR; i += 32) {
+      const int r = i / PR, c = i - r * PR;
+      Pw[r * PP + c] = __ldg(img + (int64_t)reflect101(ly - 21 + r, h) * ip + reflect101(lx - 21 + c, w));
+    }
+    P = Pw;
   }
   __syncwarp();
   // moments over the disk |u| <= umax[|v|] (always inside the level: 19 <= lx < w-19)

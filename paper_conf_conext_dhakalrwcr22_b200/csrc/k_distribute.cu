@@ -18,7 +18,7 @@
 //    written in canonical (ly, lx) order.
 // Levels with more candidates than fit in shared memory (adversarial noise images) run
 // the same code on global scratch with a 1-bit-per-pass LSD split sort (slow, correct,
-// never truncated).
+// never truncated).  tests/test_quadtree_reformulation.py is a CPU model of this kernel.
 #include <cub/block/block_radix_sort.cuh>
 #include <cub/block/block_scan.cuh>
 
@@ -29,33 +29,29 @@ namespace ss {
 namespace {
 
 constexpr int DT = 1024;
-constexpr int DIPT = 8;
-constexpr int DCAP = DT * DIPT;
+constexpr int DCAP = DT * 8;
 constexpr int MAX_CELLS = 4608;
 constexpr int REC_CAP_SMEM = DCAP / 2;
 
-typedef cub::BlockRadixSort<uint32_t, DT, DIPT, uint32_t> BRS;
+typedef cub::BlockRadixSort<uint32_t, DT, 2, uint32_t> BRS2;
+typedef cub::BlockRadixSort<uint32_t, DT, 4, uint32_t> BRS4;
+typedef cub::BlockRadixSort<uint32_t, DT, 8, uint32_t> BRS8;
 typedef cub::BlockScan<int, DT> BScan;
 
-struct Arr {
-  uint32_t* cand;   // [n] packed candidates, rank order
-  uint32_t* key;    // [n] sorted keys (later: unsorted kept keys)
-  uint32_t* rank;   // [n] rank of the i-th sorted key
-  uint8_t* dd;      // [n] separation round of sorted neighbours (i >= 1)
-  uint8_t* splitf;  // [n] at depth-d heads: child count | 0x80 if split
-  uint64_t* rec;    // [rec_cap] partial-round order keys
-  int32_t* rec_head;
-  int32_t* order;
-  uint32_t* key2;   // overflow path: ping-pong buffers of the split sort
-  uint32_t* rank2;
-};
-
-constexpr size_t kSmemCells = MAX_CELLS * 4;
-constexpr size_t kSmemArrays = (size_t)DCAP * 12;
+constexpr size_t cmax(size_t a, size_t b) { return a > b ? a : b; }
+constexpr size_t kSmemCells = (size_t)(MAX_CELLS + 1) * 4 * 2;  // offsets + slot offsets
+constexpr size_t kSmemArrays = (size_t)DCAP * 12;                // cand, key, rank
 constexpr size_t kUnionPost = (size_t)DCAP * 2 + (size_t)REC_CAP_SMEM * 16;
-constexpr size_t kUnion = sizeof(typename BRS::TempStorage) > kUnionPost ? sizeof(typename BRS::TempStorage) : kUnionPost;
+constexpr size_t kUnion = cmax(cmax(sizeof(BRS8::TempStorage), sizeof(BRS4::TempStorage)),
+                               cmax(sizeof(BRS2::TempStorage), kUnionPost));
 constexpr size_t kSmemTotal = kSmemCells + kSmemArrays + kUnion;
-static_assert(kSmemTotal <= 227 * 1024, "distribution smem budget");
+static_assert(kSmemTotal <= 220 * 1024, "distribution smem budget");
+
+struct Shared {
+  BScan::TempStorage scan;
+  int sh[8];
+  int H[16], G[17], S[15], E[15];
+};
 
 __device__ __forceinline__ void root_geom(const Geom& g, int l, int ri, int& ulx, int& urx) {
   ulx = __float2int_rz(__fmul_rn(g.hX[l], (float)ri));
@@ -98,15 +94,24 @@ __device__ __forceinline__ void node_ul(const Geom& g, int l, uint32_t key, int 
 
 __device__ __forceinline__ int sep_round(uint32_t a, uint32_t b) {
   const uint32_t x = a ^ b;
-  if (x >> 26) return 0;         // different roots
-  if (x == 0) return 14;         // never separated (cannot happen for distinct pixels)
+  if (x >> 26) return 0;  // different roots
+  if (x == 0) return 14;  // never separated (cannot happen for distinct pixels)
   return ((__clz((int)x) - 6) >> 1) + 1;
+}
+
+// warp-aggregated shared-memory histogram increment (bin < 0: no-op); whole warp calls
+__device__ __forceinline__ void hist_add(int* hist, int bin) {
+  const unsigned act = __ballot_sync(0xFFFFFFFFu, bin >= 0);
+  if (bin >= 0) {
+    const unsigned peers = __match_any_sync(act, bin);
+    if ((int)(threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(&hist[bin], __popc(peers));
+  }
 }
 
 // Stable LSD split sort of (k, v) on bits [b0, b1), ping-ponging with (k2, v2); on return
 // (k, v) name the sorted buffers.  Used only for levels that overflow shared memory.
-__device__ void split_sort_global(uint32_t*& k, uint32_t*& v, uint32_t*& k2, uint32_t*& v2, int n, int b0,
-                                  int b1, BScan::TempStorage& tmp) {
+__device__ void split_sort_global(uint32_t*& k, uint32_t*& v, uint32_t*& k2, uint32_t*& v2, int n, int b0, int b1,
+                                  BScan::TempStorage& tmp) {
   const int tid = threadIdx.x;
   for (int b = b0; b < b1; b++) {
     int z = 0;
@@ -133,245 +138,224 @@ __device__ void split_sort_global(uint32_t*& k, uint32_t*& v, uint32_t*& k2, uin
   }
 }
 
-__global__ void __launch_bounds__(DT, 1)
-    distribute_kernel(Geom g, const CellInfo* __restrict__ cells, const uint32_t* __restrict__ slots,
-                      const int32_t* __restrict__ cell_counts, uint32_t* __restrict__ selected,
-                      int32_t* __restrict__ sel_counts, uint8_t* ovf, int64_t ovf_frame_bytes,
-                      const int64_t* __restrict__ ovf_level_off, int32_t* ovf_counter) {
-  extern __shared__ __align__(16) uint8_t sm[];
-  __shared__ typename BScan::TempStorage scan_tmp;
-  __shared__ int sh[8];
-  __shared__ int H[16], G[17], S[15], E[15];
-  const int l = blockIdx.x, f = blockIdx.y, tid = threadIdx.x;
-  const int warp = tid >> 5, lane = tid & 31;
-  const int ncells = g.ncells[l];
-  const int c0 = g.cell_first[l];
-  const int N = g.N[l];
-  int32_t* cell_off = reinterpret_cast<int32_t*>(sm);
-  const int32_t* cc = cell_counts + (int64_t)f * g.total_cells + c0;
+template <int ITEMS, typename BRS>
+__device__ __forceinline__ void block_sort(const Geom& g, int l, const uint32_t* cand, uint32_t* key, uint32_t* rank,
+                                           int n, int end_bit, void* tmp) {
+  uint32_t kk[ITEMS], vv[ITEMS];
+#pragma unroll
+  for (int i = 0; i < ITEMS; i++) {
+    const int idx = threadIdx.x * ITEMS + i;
+    kk[i] = idx < n ? make_key(g, l, cand[idx]) : 0xFFFFFFFFu;
+    vv[i] = (uint32_t)idx;
+  }
+  BRS(*reinterpret_cast<typename BRS::TempStorage*>(tmp)).Sort(kk, vv, 0, end_bit);
+  __syncthreads();
+#pragma unroll
+  for (int i = 0; i < ITEMS; i++) {
+    const int idx = threadIdx.x * ITEMS + i;
+    if (idx < n) {
+      key[idx] = kk[i];
+      rank[idx] = vv[i];
+    }
+  }
+}
 
-  // ---- 1. candidate offsets per cell (rank order = cells row-major, then raster) ----
-  {
-    const int cpt = (ncells + DT - 1) / DT;
-    int s = 0;
-    for (int j = 0; j < cpt; j++) {
-      const int c = tid * cpt + j;
-      if (c < ncells) s += cc[c];
-    }
-    int ex, tot;
-    BScan(scan_tmp).ExclusiveSum(s, ex, tot);
-    for (int j = 0; j < cpt; j++) {
-      const int c = tid * cpt + j;
-      if (c < ncells) {
-        cell_off[c] = ex;
-        ex += cc[c];
-      }
-    }
-    if (tid == 0) {
-      sh[0] = tot;
-      for (int i = 0; i < 15; i++) H[i] = 0;
-      H[15] = 0;
-      for (int i = 0; i < 17; i++) G[i] = 0;
-      sh[1] = 0;  // partial-round record count
-      sh[2] = 0;  // kept keys
-    }
-    __syncthreads();
-  }
-  const int n = sh[0];
-  uint32_t* sel_out = selected + (int64_t)f * g.kp_capacity + g.cap_off[l];
-  if (n == 0) {
-    if (tid == 0) sel_counts[f * g.L + l] = 0;
-    return;
-  }
-  const bool big = n > DCAP;
-  Arr a;
-  if (!big) {
+// Everything after the cell-offset scan.  SMEM selects shared-memory arrays (compile-time,
+// so the compiler emits LDS/STS) or the global overflow scratch.
+template <bool SMEM>
+__device__ __forceinline__ void distribute_body(const Geom& g, int l, int f, int n, uint8_t* sm, Shared& S_,
+                                                const int32_t* cell_off, const int32_t* cell_slot,
+                                                const uint32_t* __restrict__ slots, uint32_t* __restrict__ selected,
+                                                int32_t* __restrict__ sel_counts, uint8_t* ovf_base,
+                                                int32_t* ovf_counter) {
+  const int tid = threadIdx.x;
+  const int ncells = g.ncells[l];
+  const int N = g.N[l];
+  uint32_t *cand, *key, *rank, *key2 = nullptr, *rank2 = nullptr;
+  uint8_t *dd, *splitf;
+  uint64_t* rec;
+  int32_t *rec_head, *order;
+  void* sort_tmp = nullptr;
+  if (SMEM) {
     uint8_t* p = sm + kSmemCells;
-    a.cand = reinterpret_cast<uint32_t*>(p);
-    a.key = a.cand + DCAP;
-    a.rank = a.key + DCAP;
-    uint8_t* u = reinterpret_cast<uint8_t*>(a.rank + DCAP);
-    a.rec = reinterpret_cast<uint64_t*>(u);
-    a.rec_head = reinterpret_cast<int32_t*>(a.rec + REC_CAP_SMEM);
-    a.order = a.rec_head + REC_CAP_SMEM;
-    a.dd = reinterpret_cast<uint8_t*>(a.order + REC_CAP_SMEM);
-    a.splitf = a.dd + DCAP;
-    a.key2 = a.rank2 = nullptr;
+    cand = reinterpret_cast<uint32_t*>(p);
+    key = cand + DCAP;
+    rank = key + DCAP;
+    uint8_t* u = reinterpret_cast<uint8_t*>(rank + DCAP);
+    sort_tmp = u;
+    rec = reinterpret_cast<uint64_t*>(u);
+    rec_head = reinterpret_cast<int32_t*>(rec + REC_CAP_SMEM);
+    order = rec_head + REC_CAP_SMEM;
+    dd = reinterpret_cast<uint8_t*>(order + REC_CAP_SMEM);
+    splitf = dd + DCAP;
   } else {
-    uint8_t* p = ovf + (int64_t)f * ovf_frame_bytes + ovf_level_off[l];
     const int64_t cap = g.level_slots[l];
-    a.cand = reinterpret_cast<uint32_t*>(p);
-    a.key = a.cand + cap;
-    a.rank = a.key + cap;
-    a.key2 = a.rank + cap;
-    a.rank2 = a.key2 + cap;
-    a.rec = reinterpret_cast<uint64_t*>(a.rank2 + cap + (cap & 1));
-    a.rec_head = reinterpret_cast<int32_t*>(a.rec + (cap / 2 + 1));
-    a.order = a.rec_head + (cap / 2 + 1);
-    a.dd = reinterpret_cast<uint8_t*>(a.order + (cap / 2 + 1));
-    a.splitf = a.dd + cap;
+    const int64_t rc = cap / 2 + 1;
+    cand = reinterpret_cast<uint32_t*>(ovf_base);
+    key = cand + cap;
+    rank = key + cap;
+    key2 = rank + cap;
+    rank2 = key2 + cap;
+    rec = reinterpret_cast<uint64_t*>(rank2 + cap + (cap & 1));
+    rec_head = reinterpret_cast<int32_t*>(rec + rc);
+    order = rec_head + rc;
+    dd = reinterpret_cast<uint8_t*>(order + rc);
+    splitf = dd + cap;
     if (tid == 0) atomicAdd(ovf_counter, 1);
   }
 
-  // ---- 2. gather candidates into rank order (one warp per cell) ----
+  // ---- 2. gather candidates into rank order (cells row-major, raster inside a cell) ----
   {
     const uint32_t* fs = slots + (int64_t)f * g.slots_per_frame;
-    for (int c = warp; c < ncells; c += DT / 32) {
-      const int cnt = cc[c];
-      const int off = cell_off[c];
-      const uint32_t* src = fs + cells[c0 + c].slot_off;
-      for (int j = lane; j < cnt; j += 32) a.cand[off + j] = src[j];
+    for (int i = tid; i < n; i += DT) {
+      int lo = 0, hi = ncells - 1;  // last cell with cell_off[c] <= i
+      while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (cell_off[mid] <= i) lo = mid; else hi = mid - 1;
+      }
+      cand[i] = fs[cell_slot[lo] + (i - cell_off[lo])];
     }
     __syncthreads();
   }
 
   // ---- 3. quadtree keys + stable sort by key (value = rank) ----
   const int end_bit = 26 + (32 - __clz(max(g.nini[l] - 1, 1)));
-  const int begin_bit = 0;
-  if (!big) {
-    uint32_t kk[DIPT], vv[DIPT];
-#pragma unroll
-    for (int i = 0; i < DIPT; i++) {
-      const int idx = tid * DIPT + i;
-      kk[i] = idx < n ? make_key(g, l, a.cand[idx]) : 0xFFFFFFFFu;
-      vv[i] = (uint32_t)idx;
-    }
-    __syncthreads();
-    BRS(*reinterpret_cast<typename BRS::TempStorage*>(sm + kSmemCells + kSmemArrays)).Sort(kk, vv, begin_bit, end_bit);
-    __syncthreads();
-#pragma unroll
-    for (int i = 0; i < DIPT; i++) {
-      const int idx = tid * DIPT + i;
-      if (idx < n) {
-        a.key[idx] = kk[i];
-        a.rank[idx] = vv[i];
-      }
-    }
+  if (SMEM) {
+    if (n <= DT * 2) block_sort<2, BRS2>(g, l, cand, key, rank, n, end_bit, sort_tmp);
+    else if (n <= DT * 4) block_sort<4, BRS4>(g, l, cand, key, rank, n, end_bit, sort_tmp);
+    else block_sort<8, BRS8>(g, l, cand, key, rank, n, end_bit, sort_tmp);
     __syncthreads();
   } else {
     for (int i = tid; i < n; i += DT) {
-      a.key[i] = make_key(g, l, a.cand[i]);
-      a.rank[i] = (uint32_t)i;
+      key[i] = make_key(g, l, cand[i]);
+      rank[i] = (uint32_t)i;
     }
     __syncthreads();
-    split_sort_global(a.key, a.rank, a.key2, a.rank2, n, begin_bit, end_bit, scan_tmp);
+    split_sort_global(key, rank, key2, rank2, n, 0, end_bit, S_.scan);
   }
 
   // ---- 4. separation rounds + histograms -> S_r, E_r for every depth ----
-  for (int i = tid; i < n; i += DT) a.dd[i] = i ? (uint8_t)sep_round(a.key[i - 1], a.key[i]) : 0;
+  for (int i = tid; i < n; i += DT) dd[i] = i ? (uint8_t)sep_round(key[i - 1], key[i]) : 0;
   __syncthreads();
-  for (int i = tid; i < n; i += DT) {
-    const int lo = i ? (int)a.dd[i] : -1;
-    const int hi = (i + 1 < n) ? (int)a.dd[i + 1] : -1;
-    if (i) atomicAdd(&H[lo], 1);
-    atomicAdd(&G[max(lo, hi) + 1], 1);
+  for (int base = 0; base < n; base += DT) {
+    const int i = base + tid;
+    int hb = -1, gb = -1;
+    if (i < n) {
+      const int lo = i ? (int)dd[i] : -1;
+      const int hi = (i + 1 < n) ? (int)dd[i + 1] : -1;
+      hb = lo;
+      gb = max(lo, hi) + 1;
+    }
+    hist_add(S_.H, hb);
+    hist_add(S_.G, gb);
   }
   __syncthreads();
   if (tid == 0) {
-    int s = 1, single = G[0];
+    int s = 1, single = S_.G[0];
     for (int r = 0; r <= 13; r++) {
-      s += H[r];
-      single += G[r + 1];
-      S[r] = s;
-      E[r] = s - single;
+      s += S_.H[r];
+      single += S_.G[r + 1];
+      S_.S[r] = s;
+      S_.E[r] = s - single;
     }
-    S[14] = S[13];
-    E[14] = E[13];
+    S_.S[14] = S_.S[13];
+    S_.E[14] = S_.E[13];
     // ORB-SLAM's loop, on node counts only (phase 1 then phase 2 stop rules)
     int D = 1, partial = 0, r = 0;
     for (;;) {
-      const int nx = S[min(r + 1, 14)];
-      if (nx >= N || nx == S[r]) { D = r + 1; break; }
-      if (nx + 3 * E[min(r + 1, 14)] > N) {
+      const int nx = S_.S[min(r + 1, 14)];
+      if (nx >= N || nx == S_.S[r]) { D = r + 1; break; }
+      if (nx + 3 * S_.E[min(r + 1, 14)] > N) {
         int d = r + 1;
         for (;;) {
-          const int s2 = S[min(d + 1, 14)];
+          const int s2 = S_.S[min(d + 1, 14)];
           if (s2 >= N) { D = d; partial = 1; break; }
-          if (s2 == S[min(d, 14)]) { D = d + 1; break; }
+          if (s2 == S_.S[min(d, 14)]) { D = d + 1; break; }
           d++;
         }
         break;
       }
       r++;
     }
-    sh[3] = min(D, 14);
-    sh[4] = partial;
+    S_.sh[3] = min(D, 14);
+    S_.sh[4] = partial;
   }
   __syncthreads();
-  const int D = sh[3];
-  const bool partial = sh[4] != 0;
+  const int D = S_.sh[3];
+  const bool partial = S_.sh[4] != 0;
   const int dlim = min(D, 13);
 
   // ---- 5. partial phase-2 round at depth D: order the multi-key nodes, split a prefix ----
   if (partial) {
     for (int i = tid; i < n; i += DT) {
-      if (i != 0 && a.dd[i] > D) continue;  // not a depth-D node head
+      if (i != 0 && dd[i] > D) continue;  // not a depth-D node head
       int size = 1, c = 1;
-      uint32_t minrank = a.rank[i];
-      for (int j = i + 1; j < n && a.dd[j] > D; j++) {
+      uint32_t minrank = rank[i];
+      for (int j = i + 1; j < n && dd[j] > D; j++) {
         size++;
-        minrank = min(minrank, a.rank[j]);
-        c += (a.dd[j] == D + 1);
+        minrank = min(minrank, rank[j]);
+        c += (dd[j] == D + 1);
       }
-      a.splitf[i] = 0;
+      splitf[i] = 0;
       if (size > 1) {
-        const int e = atomicAdd(&sh[1], 1);
+        const int e = atomicAdd(&S_.sh[1], 1);
         int ulx, uly;
-        node_ul(g, l, a.key[i], D, ulx, uly);
-        a.rec[e] = ((uint64_t)(0x1FFFFF - size) << 43) | ((uint64_t)uly << 32) | ((uint64_t)ulx << 20) |
-                   (uint64_t)minrank;
-        a.rec_head[e] = i;
-        a.splitf[i] = (uint8_t)c;
+        node_ul(g, l, key[i], D, ulx, uly);
+        rec[e] = ((uint64_t)(0x1FFFFF - size) << 43) | ((uint64_t)uly << 32) | ((uint64_t)ulx << 20) |
+                 (uint64_t)minrank;
+        rec_head[e] = i;
+        splitf[i] = (uint8_t)c;
       }
     }
     __syncthreads();
-    const int ne = sh[1];
+    const int ne = S_.sh[1];
     for (int e = tid; e < ne; e += DT) {
-      const uint64_t k = a.rec[e];
+      const uint64_t k = rec[e];
       int pos = 0;
-      for (int e2 = 0; e2 < ne; e2++) pos += a.rec[e2] < k;
-      a.order[pos] = e;
+      for (int e2 = 0; e2 < ne; e2++) pos += rec[e2] < k;
+      order[pos] = e;
     }
     __syncthreads();
     if (tid == 0) {
-      int acc = S[D];
+      int acc = S_.S[D];
       for (int t = 0; t < ne && acc < N; t++) {
-        const int h = a.rec_head[a.order[t]];
-        acc += (a.splitf[h] & 0x7F) - 1;
-        a.splitf[h] |= 0x80;
+        const int h = rec_head[order[t]];
+        acc += (splitf[h] & 0x7F) - 1;
+        splitf[h] |= 0x80;
       }
     }
     __syncthreads();
   }
 
   // ---- 6. one key per final node: max score, ties -> lowest rank ----
-  uint32_t* kept = a.key;  // keys are no longer needed
+  uint32_t* kept = key;  // keys are no longer needed
   __syncthreads();
   for (int i = tid; i < n; i += DT) {
-    if (i != 0 && a.dd[i] > dlim) continue;  // not a final node head
-    const bool split = partial && (a.splitf[i] & 0x80);
+    if (i != 0 && dd[i] > dlim) continue;  // not a final node head
+    const bool split = partial && (splitf[i] & 0x80);
     int best_m = -1;
     uint32_t best_r = 0;
-    for (int j = i; j < n && (j == i || a.dd[j] > dlim); j++) {
-      if (j != i && split && a.dd[j] == D + 1) {
-        const int p = atomicAdd(&sh[2], 1);
-        kept[p] = a.cand[best_r];
+    for (int j = i; j < n && (j == i || dd[j] > dlim); j++) {
+      if (j != i && split && dd[j] == D + 1) {
+        const int p = atomicAdd(&S_.sh[2], 1);
+        kept[p] = cand[best_r];
         best_m = -1;
       }
-      const uint32_t r = a.rank[j];
-      const int m = key_m(a.cand[r]);
+      const uint32_t r = rank[j];
+      const int m = key_m(cand[r]);
       if (m > best_m || (m == best_m && r < best_r)) {
         best_m = m;
         best_r = r;
       }
     }
-    const int p = atomicAdd(&sh[2], 1);
-    kept[p] = a.cand[best_r];
+    const int p = atomicAdd(&S_.sh[2], 1);
+    kept[p] = cand[best_r];
   }
   __syncthreads();
-  const int nk = sh[2];
+  const int nk = S_.sh[2];
   const int nk_w = min(nk, g.cap[l]);
   // ---- 7. canonical (ly, lx) order, into the frame's selected scratch ----
+  uint32_t* sel_out = selected + (int64_t)f * g.kp_capacity + g.cap_off[l];
   for (int t = tid; t < nk; t += DT) {
     const uint32_t k = kept[t] >> 8;
     int pos = 0;
@@ -382,6 +366,63 @@ __global__ void __launch_bounds__(DT, 1)
     sel_counts[f * g.L + l] = nk_w;
     if (nk > g.cap[l]) atomicAdd(ovf_counter + 1, 1);  // impossible by the O4 bound; reported
   }
+}
+
+__global__ void __launch_bounds__(DT, 1)
+    distribute_kernel(Geom g, const CellInfo* __restrict__ cells, const uint32_t* __restrict__ slots,
+                      const int32_t* __restrict__ cell_counts, uint32_t* __restrict__ selected,
+                      int32_t* __restrict__ sel_counts, uint8_t* ovf, int64_t ovf_frame_bytes,
+                      const int64_t* __restrict__ ovf_level_off, int32_t* ovf_counter) {
+  extern __shared__ __align__(16) uint8_t sm[];
+  __shared__ Shared S_;
+  const int l = blockIdx.x, f = blockIdx.y, tid = threadIdx.x;
+  const int ncells = g.ncells[l];
+  const int c0 = g.cell_first[l];
+  int32_t* cell_off = reinterpret_cast<int32_t*>(sm);
+  int32_t* cell_slot = cell_off + MAX_CELLS + 1;
+  const int32_t* cc = cell_counts + (int64_t)f * g.total_cells + c0;
+
+  // ---- 1. candidate offsets per cell (rank order = cells row-major, then raster) ----
+  {
+    const int cpt = (ncells + DT - 1) / DT;  // <= 5 (MAX_CELLS)
+    int cnt[5];
+    int s = 0;
+#pragma unroll
+    for (int j = 0; j < 5; j++) {
+      const int c = tid * cpt + j;
+      cnt[j] = (j < cpt && c < ncells) ? cc[c] : 0;
+      s += cnt[j];
+    }
+    int ex, tot;
+    BScan(S_.scan).ExclusiveSum(s, ex, tot);
+#pragma unroll
+    for (int j = 0; j < 5; j++) {
+      const int c = tid * cpt + j;
+      if (j < cpt && c < ncells) {
+        cell_off[c] = ex;
+        cell_slot[c] = cells[c0 + c].slot_off;
+        ex += cnt[j];
+      }
+    }
+    if (tid == 0) {
+      S_.sh[0] = tot;
+      S_.sh[1] = 0;  // partial-round record count
+      S_.sh[2] = 0;  // kept keys
+    }
+    if (tid < 16) S_.H[tid] = 0;
+    if (tid < 17) S_.G[tid] = 0;
+    __syncthreads();
+  }
+  const int n = S_.sh[0];
+  if (n == 0) {
+    if (tid == 0) sel_counts[f * g.L + l] = 0;
+    return;
+  }
+  if (n <= DCAP)
+    distribute_body<true>(g, l, f, n, sm, S_, cell_off, cell_slot, slots, selected, sel_counts, nullptr, ovf_counter);
+  else
+    distribute_body<false>(g, l, f, n, sm, S_, cell_off, cell_slot, slots, selected, sel_counts,
+                           ovf + (int64_t)f * ovf_frame_bytes + ovf_level_off[l], ovf_counter);
 }
 
 }  // namespace

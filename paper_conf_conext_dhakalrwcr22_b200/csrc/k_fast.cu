@@ -4,18 +4,20 @@
 //
 // One CTA per *band* = one row of 30-px FAST cells of one level of one frame (the cells of a
 // row share their detect rows, and their detect windows tile [x0, x1) without gaps):
-//  1. stage the band + 3-px ring halo in shared memory with 16-byte coalesced loads;
-//  2. every warp walks band rows 32 pixels at a time: an 8-point pre-test (any 9-arc of the
-//     ring contains 4 consecutive even ring positions) rejects ~80 % of pixels; survivors are
-//     compacted into a per-warp queue with ballots and scored 32 at a time by the full arc test
-//     on packed 16x2 lanes (DPX VIMNMX3.U16x2) -> M map of the band in shared memory;
-//  3. one warp per cell: strict 8-neighbour maxima inside the cell's window (neighbours in the
-//     next cell are ignored: per-cell ROI semantics), the cell's threshold (iniTh if any
-//     survivor beats it, else minTh), compaction in raster order by ballot prefix counts.
+//  1. stage the band + ring halo in shared memory with 16-byte coalesced loads;
+//  2. the score M of EVERY band pixel, four horizontally adjacent pixels per thread: the 16
+//     ring values of the 4 pixels are 16 byte-permutes of a sliding 7-row x 3-word register
+//     window (3 shared loads per row step), unpacked into two 16x2 lanes, and the cyclic
+//     min/max over the 16 arcs of 9 runs on DPX three-way min/max (VIMNMX3.U16x2) -- no
+//     pre-test, no divergence, one 32-bit store of 4 scores;
+//  3. one warp per cell, one lane per cell row: strict 8-neighbour maxima inside the cell's
+//     window (neighbours in the next cell are ignored: per-cell ROI semantics) as 64-bit row
+//     masks, the cell's threshold (iniTh if any maximum beats it, else minTh), and the
+//     survivors written in raster order (warp prefix sum of the row counts).
 //
 //   M(p) = max_s max( min_{k<9} d_{s+k}, min_{k<9} -d_{s+k} ),  d_k = I(p) - I(p + R_k)
-//   corner at t <=> M > t; pixels with M <= minTh are stored as 0 (they can neither be
-//   candidates nor suppress one: a candidate has M > minTh).
+//   corner at t <=> M > t (stored clamped to >= 0; scores <= minTh can neither be candidates
+//   nor suppress one, so no thresholding is needed before the NMS).
 #include "ss_internal.h"
 
 namespace ss {
@@ -23,85 +25,85 @@ namespace ss {
 namespace {
 
 constexpr int FB_WARPS = 16;
-constexpr int QCAP = 64;  // per-warp queue of pre-test survivors
+constexpr int FB_THREADS = FB_WARPS * 32;
+constexpr int ROWS_PER_TASK = 8;
 
-__device__ __forceinline__ uint32_t swap16(uint32_t v) { return __byte_perm(v, 0, 0x1032); }
+__device__ __forceinline__ uint32_t lo_pair(uint32_t w) { return __byte_perm(w, 0, 0x7270); }  // bytes 0, 2
+__device__ __forceinline__ uint32_t hi_pair(uint32_t w) { return __byte_perm(w, 0, 0x7371); }  // bytes 1, 3
 
-// 8-point necessary condition for M > t: four cyclically consecutive even ring positions
-// all brighter than I+t or all darker than I-t.
-__device__ __forceinline__ bool pretest8(const uint8_t* c, int p, int t) {
-  const int cv = c[0];
-  const int e0 = c[3 * p], e1 = c[2 * p + 2], e2 = c[3], e3 = c[-2 * p + 2];
-  const int e4 = c[-3 * p], e5 = c[-2 * p - 2], e6 = c[-3], e7 = c[2 * p - 2];
-  const int hi = cv + t, lo = cv - t;
-  unsigned b = (unsigned)(e0 > hi) | ((unsigned)(e1 > hi) << 1) | ((unsigned)(e2 > hi) << 2) |
-               ((unsigned)(e3 > hi) << 3) | ((unsigned)(e4 > hi) << 4) | ((unsigned)(e5 > hi) << 5) |
-               ((unsigned)(e6 > hi) << 6) | ((unsigned)(e7 > hi) << 7);
-  unsigned d = (unsigned)(e0 < lo) | ((unsigned)(e1 < lo) << 1) | ((unsigned)(e2 < lo) << 2) |
-               ((unsigned)(e3 < lo) << 3) | ((unsigned)(e4 < lo) << 4) | ((unsigned)(e5 < lo) << 5) |
-               ((unsigned)(e6 < lo) << 6) | ((unsigned)(e7 < lo) << 7);
-  b |= b << 8;
-  d |= d << 8;
-  const unsigned rb = b & (b >> 1) & (b >> 2) & (b >> 3);
-  const unsigned rd = d & (d >> 1) & (d >> 2) & (d >> 3);
-  return ((rb | rd) & 0xFFu) != 0u;
+// Cyclic arc min/max of one 16x2 pair of pixels.  d[k] = c - r_k + 256 (both lanes).
+// Returns max(max_s min9 d, 512 - min_s max9 d) clamped to >= 256, i.e. M + 256 >= 256.
+__device__ __forceinline__ uint32_t arc_score2(const uint32_t (&d)[16]) {
+  uint32_t mn3[16], mx3[16];
+#pragma unroll
+  for (int k = 0; k < 16; k++) {
+    mn3[k] = __vimin3_u16x2(d[k], d[(k + 1) & 15], d[(k + 2) & 15]);
+    mx3[k] = __vimax3_u16x2(d[k], d[(k + 1) & 15], d[(k + 2) & 15]);
+  }
+  uint32_t mn9[16], mx9[16];
+#pragma unroll
+  for (int s = 0; s < 16; s++) {
+    mn9[s] = __vimin3_u16x2(mn3[s], mn3[(s + 3) & 15], mn3[(s + 6) & 15]);
+    mx9[s] = __vimax3_u16x2(mx3[s], mx3[(s + 3) & 15], mx3[(s + 6) & 15]);
+  }
+  const uint32_t a1 = __vimax3_u16x2(__vimax3_u16x2(mn9[0], mn9[1], mn9[2]), __vimax3_u16x2(mn9[3], mn9[4], mn9[5]),
+                                     __vimax3_u16x2(mn9[6], mn9[7], mn9[8]));
+  const uint32_t a2 = __vimax3_u16x2(__vimax3_u16x2(mn9[9], mn9[10], mn9[11]),
+                                     __vimax3_u16x2(mn9[12], mn9[13], mn9[14]), mn9[15]);
+  const uint32_t z1 = __vimin3_u16x2(__vimin3_u16x2(mx9[0], mx9[1], mx9[2]), __vimin3_u16x2(mx9[3], mx9[4], mx9[5]),
+                                     __vimin3_u16x2(mx9[6], mx9[7], mx9[8]));
+  const uint32_t z2 = __vimin3_u16x2(__vimin3_u16x2(mx9[9], mx9[10], mx9[11]),
+                                     __vimin3_u16x2(mx9[12], mx9[13], mx9[14]), mx9[15]);
+  const uint32_t maxmin = __vimax3_u16x2(a1, a2, a2);                 // max_s min9(d) + 256 (dark ring)
+  const uint32_t minmax = __vimin3_u16x2(z1, z2, z2);                 // min_s max9(d) + 256 (bright ring)
+  return __vimax3_u16x2(maxmin, 0x02000200u - minmax, 0x01000100u);  // max(.., 256 + max(0, ..))
 }
 
-// Full arc test: M clamped to 0 when <= tmin.  c = centre pixel in the staged band (pitch p).
-__device__ __forceinline__ int fast_M(const uint8_t* c, int p, int tmin) {
-  const int cv = c[0];
-  // ring in OpenCV offsets16 order: (0,3) (1,3) (2,2) (3,1) (3,0) (3,-1) (2,-2) (1,-3) ...
-  const int r0 = c[3 * p], r1 = c[3 * p + 1], r2 = c[2 * p + 2], r3 = c[p + 3];
-  const int r4 = c[3], r5 = c[-p + 3], r6 = c[-2 * p + 2], r7 = c[-3 * p + 1];
-  const int r8 = c[-3 * p], r9 = c[-3 * p - 1], r10 = c[-2 * p - 2], r11 = c[-p - 3];
-  const int r12 = c[-3], r13 = c[p - 3], r14 = c[2 * p - 2], r15 = c[3 * p - 1];
-  // biased differences d'_k = cv - r_k + 256 in [1, 511], packed (d'_k, d'_{k+8})
-  const uint32_t cc = (uint32_t)(cv + 256) * 0x10001u;
-  uint32_t q[16];
-  q[0] = cc - ((uint32_t)r0 | ((uint32_t)r8 << 16));
-  q[1] = cc - ((uint32_t)r1 | ((uint32_t)r9 << 16));
-  q[2] = cc - ((uint32_t)r2 | ((uint32_t)r10 << 16));
-  q[3] = cc - ((uint32_t)r3 | ((uint32_t)r11 << 16));
-  q[4] = cc - ((uint32_t)r4 | ((uint32_t)r12 << 16));
-  q[5] = cc - ((uint32_t)r5 | ((uint32_t)r13 << 16));
-  q[6] = cc - ((uint32_t)r6 | ((uint32_t)r14 << 16));
-  q[7] = cc - ((uint32_t)r7 | ((uint32_t)r15 << 16));
+// M of 4 horizontally adjacent pixels from the 7-row window W[dy + 3][0..2] (columns
+// gx-4 .. gx+7 of rows y-3 .. y+3), packed as 4 bytes (pixel i in byte i).
+__device__ __forceinline__ uint32_t fast_M4(const uint32_t (&W)[7][3]) {
+  uint32_t R[16];
+  R[0] = W[6][1];                              // ( 0, 3)
+  R[1] = __byte_perm(W[6][1], W[6][2], 0x4321);  // ( 1, 3)
+  R[2] = __byte_perm(W[5][1], W[5][2], 0x5432);  // ( 2, 2)
+  R[3] = __byte_perm(W[4][1], W[4][2], 0x6543);  // ( 3, 1)
+  R[4] = __byte_perm(W[3][1], W[3][2], 0x6543);  // ( 3, 0)
+  R[5] = __byte_perm(W[2][1], W[2][2], 0x6543);  // ( 3,-1)
+  R[6] = __byte_perm(W[1][1], W[1][2], 0x5432);  // ( 2,-2)
+  R[7] = __byte_perm(W[0][1], W[0][2], 0x4321);  // ( 1,-3)
+  R[8] = W[0][1];                              // ( 0,-3)
+  R[9] = __byte_perm(W[0][0], W[0][1], 0x6543);  // (-1,-3)
+  R[10] = __byte_perm(W[1][0], W[1][1], 0x5432); // (-2,-2)
+  R[11] = __byte_perm(W[2][0], W[2][1], 0x4321); // (-3,-1)
+  R[12] = __byte_perm(W[3][0], W[3][1], 0x4321); // (-3, 0)
+  R[13] = __byte_perm(W[4][0], W[4][1], 0x4321); // (-3, 1)
+  R[14] = __byte_perm(W[5][0], W[5][1], 0x5432); // (-2, 2)
+  R[15] = __byte_perm(W[6][0], W[6][1], 0x6543); // (-1, 3)
+  const uint32_t C = W[3][1];
+  uint32_t d[16];
+  const uint32_t clo = lo_pair(C) + 0x01000100u;
 #pragma unroll
-  for (int k = 0; k < 8; k++) q[k + 8] = swap16(q[k]);
-  // windows of 9: lo half = window s, hi half = window s+8
-  uint32_t mn3[14], mx3[14];
+  for (int k = 0; k < 16; k++) d[k] = clo - lo_pair(R[k]);
+  const uint32_t slo = arc_score2(d) - 0x01000100u;  // pixels 0, 2
+  const uint32_t chi = hi_pair(C) + 0x01000100u;
 #pragma unroll
-  for (int k = 0; k < 14; k++) {
-    mn3[k] = __vimin3_u16x2(q[k], q[k + 1], q[k + 2]);
-    mx3[k] = __vimax3_u16x2(q[k], q[k + 1], q[k + 2]);
-  }
-  uint32_t mn9[8], mx9[8];
-#pragma unroll
-  for (int s = 0; s < 8; s++) {
-    mn9[s] = __vimin3_u16x2(mn3[s], mn3[s + 3], mn3[s + 6]);
-    mx9[s] = __vimax3_u16x2(mx3[s], mx3[s + 3], mx3[s + 6]);
-  }
-  const uint32_t a = __vimax3_u16x2(__vimax3_u16x2(mn9[0], mn9[1], mn9[2]), __vimax3_u16x2(mn9[3], mn9[4], mn9[5]),
-                                    __vimax3_u16x2(mn9[6], mn9[7], mn9[7]));
-  const uint32_t z = __vimin3_u16x2(__vimin3_u16x2(mx9[0], mx9[1], mx9[2]), __vimin3_u16x2(mx9[3], mx9[4], mx9[5]),
-                                    __vimin3_u16x2(mx9[6], mx9[7], mx9[7]));
-  const int maxmin = max((int)(a & 0xFFFF), (int)(a >> 16));  // max_s min9(d') (dark ring)
-  const int minmax = min((int)(z & 0xFFFF), (int)(z >> 16));  // min_s max9(d') (bright ring)
-  const int M = max(maxmin - 256, 256 - minmax);
-  return M > tmin ? M : 0;
+  for (int k = 0; k < 16; k++) d[k] = chi - hi_pair(R[k]);
+  const uint32_t shi = arc_score2(d) - 0x01000100u;  // pixels 1, 3
+  return __byte_perm(slo, shi, 0x6240);
 }
 
-__global__ void __launch_bounds__(FB_WARPS * 32) fast_bands_kernel(Geom g, FrameSrc src,
-                                                                   const BandInfo* __restrict__ bands,
-                                                                   const CellInfo* __restrict__ cells,
-                                                                   uint32_t* __restrict__ slots,
-                                                                   int32_t* __restrict__ cell_counts, int rp, int mbw,
-                                                                   int region_bytes, int mband_bytes, int nball) {
+__global__ void __launch_bounds__(FB_THREADS) fast_bands_kernel(Geom g, FrameSrc src,
+                                                                const BandInfo* __restrict__ bands,
+                                                                const CellInfo* __restrict__ cells,
+                                                                uint32_t* __restrict__ slots,
+                                                                int32_t* __restrict__ cell_counts, int rp, int mbw,
+                                                                int region_bytes) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const BandInfo bd = bands[blockIdx.x];
   const int f = blockIdx.y;
   const int l = bd.level;
+  const int tmin = g.min_th, tini = g.ini_th;
   const uint8_t* img;
   int ip;
   if (l == 0) {
@@ -111,126 +113,133 @@ __global__ void __launch_bounds__(FB_WARPS * 32) fast_bands_kernel(Geom g, Frame
     img = src.pyr + (int64_t)f * g.pyr_frame_bytes + g.lvl_off[l];
     ip = g.pitch[l];
   }
-  uint8_t* reg = smem;                                   // [RH][rp] staged band + halo
-  uint8_t* Mb = smem + region_bytes;                     // [Dh + 2][mbw] M map (zero border rows)
-  uint32_t* queue = reinterpret_cast<uint32_t*>(Mb + mband_bytes) + warp * QCAP;
-  uint32_t* ball = reinterpret_cast<uint32_t*>(Mb + mband_bytes) + FB_WARPS * QCAP + warp * nball;
-  const int Dw = bd.x1 - bd.x0, Dh = bd.y1 - bd.y0;
-  const int RH = Dh + 6;
-  const int xs = bd.x0 - 3;       // first staged column
-  const int xa = xs & ~15;        // 16-byte aligned start
-  const int shift = xs - xa;      // staged column of level column x = x - xa
-  const int nchunk = (shift + Dw + 6 + 15) >> 4;
-  const uint8_t* row0 = img + (int64_t)(bd.y0 - 3) * ip;
-  // ---- 1. stage the band + halo (coalesced 16-B loads when the rows are 16-B aligned) ----
+  uint8_t* reg = smem;                 // [Dh + 6][rp] staged band; staged column s <-> level column xa + s
+  uint8_t* Mb = smem + region_bytes;   // [Dh + 2][mbw] scores; same columns, zero rows above/below
+  const int Dh = bd.y1 - bd.y0;
+  const int xa = ((bd.x0 - 3) & ~15) - 16;              // >= 0: x0 >= 19
+  const int g0 = ((bd.x0 - xa) & ~3), g1 = (bd.x1 - xa + 3) & ~3;  // 4-px groups covering [x0, x1)
+  const int sw = (g1 + 4 + 15) & ~15;                   // staged columns [0, sw)
+  const uint8_t* row0 = img + (int64_t)(bd.y0 - 3) * ip + xa;
+  // ---- 1. stage rows y0-3 .. y1+2, columns xa .. xa+sw-1 (all inside the level row) ----
+  const int nchunk = sw >> 4;
   if ((ip & 15) == 0 && (reinterpret_cast<uintptr_t>(img) & 15) == 0) {
-    for (int i = threadIdx.x; i < RH * nchunk; i += blockDim.x) {
+    for (int i = threadIdx.x; i < (Dh + 6) * nchunk; i += FB_THREADS) {
       const int r = i / nchunk, c = i - r * nchunk;
-      const uint4 v = __ldg(reinterpret_cast<const uint4*>(row0 + (int64_t)r * ip + xa) + c);
-      *reinterpret_cast<uint4*>(reg + r * rp + 16 * c) = v;
+      *reinterpret_cast<uint4*>(reg + r * rp + 16 * c) =
+          __ldg(reinterpret_cast<const uint4*>(row0 + (int64_t)r * ip) + c);
     }
   } else {
-    for (int i = threadIdx.x; i < RH * (Dw + 6); i += blockDim.x) {
-      const int r = i / (Dw + 6), c = i - r * (Dw + 6);
-      reg[r * rp + shift + c] = __ldg(row0 + (int64_t)r * ip + xs + c);
+    for (int i = threadIdx.x; i < (Dh + 6) * sw; i += FB_THREADS) {
+      const int r = i / sw, c = i - r * sw;
+      reg[r * rp + c] = __ldg(row0 + (int64_t)r * ip + c);
     }
   }
-  for (int i = threadIdx.x; i < mband_bytes / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(Mb)[i] = 0u;
+  // zero border rows of the score map
+  for (int i = threadIdx.x; i < mbw / 4; i += FB_THREADS) {
+    reinterpret_cast<uint32_t*>(Mb)[i] = 0u;
+    reinterpret_cast<uint32_t*>(Mb + (Dh + 1) * mbw)[i] = 0u;
+  }
   __syncthreads();
-  // ---- 2. M map: 8-point pre-test, warp-queue compaction, full arc test ----
-  const int tmin = g.min_th, tini = g.ini_th;
-  const unsigned lt = (1u << lane) - 1u;
-  int qn = 0;
-  auto drain = [&](int cnt) {  // score queue entries [0, cnt)
-    if (lane < cnt) {
-      const uint32_t e = queue[lane];
-      const int x = (int)(e & 0xFFFF), y = (int)(e >> 16);  // band-relative D coordinates
-      const int m = fast_M(reg + (y + 3) * rp + (x + 3 + shift), rp, tmin);
-      Mb[(y + 1) * mbw + x + 1] = (uint8_t)m;
-    }
-  };
-  for (int y = warp; y < Dh; y += FB_WARPS) {
-    const uint8_t* rowc = reg + (y + 3) * rp + 3 + shift;
-    for (int xc = 0; xc < Dw; xc += 32) {
-      const int x = xc + lane;
-      const bool pass = x < Dw && pretest8(rowc + x, rp, tmin);
-      const unsigned msk = __ballot_sync(0xFFFFFFFFu, pass);
-      if (pass) queue[qn + __popc(msk & lt)] = ((uint32_t)y << 16) | (uint32_t)x;
-      qn += __popc(msk);
-      __syncwarp();
-      if (qn >= 32) {
-        drain(32);
-        __syncwarp();
-        if (lane < qn - 32) queue[lane] = queue[32 + lane];
-        qn -= 32;
-        __syncwarp();
+  // ---- 2. scores of all band pixels, 4 per thread, ROWS_PER_TASK rows per task ----
+  {
+    const int ng = (g1 - g0) >> 2;
+    const int nrt = (Dh + ROWS_PER_TASK - 1) / ROWS_PER_TASK;
+    for (int t = threadIdx.x; t < ng * nrt; t += FB_THREADS) {
+      const int gc = g0 + 4 * (t % ng);
+      const int ys = (t / ng) * ROWS_PER_TASK;
+      uint32_t W[7][3];
+      // staged row of band row y is y + 3; rows y-3..y+3 -> staged rows y..y+6
+#pragma unroll
+      for (int r = 0; r < 6; r++) {
+        const uint32_t* p = reinterpret_cast<const uint32_t*>(reg + (ys + r) * rp + gc - 4);
+        W[r + 1][0] = p[0];
+        W[r + 1][1] = p[1];
+        W[r + 1][2] = p[2];
+      }
+#pragma unroll
+      for (int i = 0; i < ROWS_PER_TASK; i++) {  // fully unrolled: the window shift is renaming
+        const int y = ys + i;
+        if (y >= Dh) break;
+#pragma unroll
+        for (int r = 0; r < 6; r++) {
+          W[r][0] = W[r + 1][0];
+          W[r][1] = W[r + 1][1];
+          W[r][2] = W[r + 1][2];
+        }
+        const uint32_t* p = reinterpret_cast<const uint32_t*>(reg + (y + 6) * rp + gc - 4);
+        W[6][0] = p[0];
+        W[6][1] = p[1];
+        W[6][2] = p[2];
+        *reinterpret_cast<uint32_t*>(Mb + (y + 1) * mbw + gc) = fast_M4(W);
       }
     }
   }
-  drain(qn);
   __syncthreads();
-  // ---- 3. per cell: strict maxima inside the cell window, threshold choice, compaction ----
+  // ---- 3. per cell (warp), per row (lane): strict maxima, threshold choice, raster output ----
   for (int j = warp; j < bd.ncells; j += FB_WARPS) {
     const int ci = bd.cell_first + j;
     const CellInfo c = cells[ci];
-    const int cx0 = c.x0 - bd.x0, cx1 = c.x1 - bd.x0;  // band-relative cell columns
-    const int cw = cx1 - cx0;
-    const int nxc = (cw + 31) >> 5;
-    bool any_ini = false;
-    int nch = 0;
-    for (int y = 0; y < Dh; y++) {
-      for (int xc = 0; xc < cw; xc += 32, nch++) {
-        const int x = cx0 + xc + lane;
-        bool kmin = false, kini = false;
-        if (xc + lane < cw) {
-          const uint8_t* p = Mb + (y + 1) * mbw + x + 1;
-          const int m = p[0];
+    const int cx0 = c.x0 - xa, cw = c.x1 - c.x0;  // staged columns [cx0, cx0 + cw), cw < 64
+    unsigned long long kmin[2] = {0ull, 0ull}, kini[2] = {0ull, 0ull};
+#pragma unroll
+    for (int hh = 0; hh < 2; hh++) {
+      const int y = lane + 32 * hh;
+      if (y < Dh) {
+        const uint8_t* rowp = Mb + (y + 1) * mbw + cx0;
+        for (int x = 0; x < cw; x++) {
+          const int m = rowp[x];
           if (m > tmin) {
-            const bool lok = x > cx0, rok = x < cx1 - 1;  // neighbours in other cells are ignored
+            const uint8_t* p = rowp + x;
             bool mx = m > p[-mbw] && m > p[mbw];
-            if (lok) mx = mx && m > p[-mbw - 1] && m > p[-1] && m > p[mbw - 1];
-            if (rok) mx = mx && m > p[-mbw + 1] && m > p[1] && m > p[mbw + 1];
-            kmin = mx;
-            kini = mx && m > tini;
+            if (x > 0) mx = mx && m > p[-mbw - 1] && m > p[-1] && m > p[mbw - 1];
+            if (x < cw - 1) mx = mx && m > p[-mbw + 1] && m > p[1] && m > p[mbw + 1];
+            if (mx) {
+              kmin[hh] |= 1ull << x;
+              if (m > tini) kini[hh] |= 1ull << x;
+            }
           }
         }
-        const unsigned bmin = __ballot_sync(0xFFFFFFFFu, kmin);
-        const unsigned bini = __ballot_sync(0xFFFFFFFFu, kini);
-        if (lane == 0) {
-          ball[2 * nch] = bmin;
-          ball[2 * nch + 1] = bini;
-        }
-        any_ini |= (bini != 0u);
       }
     }
-    __syncwarp();
-    const int sel = any_ini ? 1 : 0;
+    const bool any_ini = __any_sync(0xFFFFFFFFu, (kini[0] | kini[1]) != 0ull);
     uint32_t* out = slots + (int64_t)f * g.slots_per_frame + c.slot_off;
-    int cnt = 0;
-    for (int ch = 0; ch < nch; ch++) {
-      const unsigned b = ball[2 * ch + sel];
-      if ((b >> lane) & 1u) {
-        const int y = ch / nxc, xc = (ch - y * nxc) * 32;
-        const int x = cx0 + xc + lane;
-        out[cnt + __popc(b & lt)] = pack_key(bd.x0 + x, bd.y0 + y, Mb[(y + 1) * mbw + x + 1]);
+    int base = 0;
+#pragma unroll
+    for (int hh = 0; hh < 2; hh++) {
+      unsigned long long sel = any_ini ? kini[hh] : kmin[hh];
+      const int cnt = __popcll(sel);
+      int incl = cnt;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int v = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+        if (lane >= o) incl += v;
       }
-      cnt += __popc(b);
+      int pos = base + incl - cnt;
+      const int y = lane + 32 * hh;
+      while (sel) {
+        const int x = __ffsll((long long)sel) - 1;
+        sel &= sel - 1;
+        out[pos++] = pack_key(c.x0 + x, bd.y0 + y, Mb[(y + 1) * mbw + cx0 + x]);
+      }
+      base += __shfl_sync(0xFFFFFFFFu, incl, 31);
     }
-    if (lane == 0) cell_counts[(int64_t)f * g.total_cells + ci] = cnt;
-    __syncwarp();
+    if (lane == 0) cell_counts[(int64_t)f * g.total_cells + ci] = base;
   }
 }
 
 }  // namespace
 
 size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int* mband_bytes, int* nball) {
-  // widest band + halo, 16-B aligned staging with up to 15 B of lead-in
-  *rp = ((g.max_band_w + 6 + 15 + 15) / 16) * 16;
+  // staged columns: up to 16 + 15 lead-in, the band, 4-px group round-up and a 4-B right guard
+  const int sw = ((g.max_band_w + 31 + 3 + 4 + 4) + 15) & ~15;
+  *rp = sw + 16;
   *region_bytes = ((g.max_band_h + 6) * *rp + 15) & ~15;
-  *mbw = (g.max_band_w + 2 + 3) & ~3;
-  *mband_bytes = ((g.max_band_h + 2) * *mbw + 15) & ~15;
-  *nball = 2 * g.max_band_h * ((g.max_cell_w + 31) / 32);
-  return (size_t)*region_bytes + *mband_bytes + (size_t)FB_WARPS * QCAP * 4 + (size_t)FB_WARPS * *nball * 4;
+  int m = (sw + 3) & ~3;
+  if (((m >> 2) & 1) == 0) m += 4;  // odd word pitch: lane-per-row reads hit distinct banks
+  *mbw = m;
+  *mband_bytes = ((g.max_band_h + 2) * m + 15) & ~15;
+  *nball = 0;
+  return (size_t)*region_bytes + *mband_bytes;
 }
 
 cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands,
@@ -243,7 +252,7 @@ cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const B
     attr_set = true;
   }
   dim3 grid(g.total_bands, n_frames);
-  fast_bands_kernel<<<grid, FB_WARPS * 32, smem, s>>>(g, src, bands, cells, slots, cell_counts, rp, mbw, rb, mb, nb);
+  fast_bands_kernel<<<grid, FB_THREADS, smem, s>>>(g, src, bands, cells, slots, cell_counts, rp, mbw, rb);
   return cudaGetLastError();
 }
 

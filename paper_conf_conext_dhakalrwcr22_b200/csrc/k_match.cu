@@ -1,12 +1,13 @@
 // k_match.cu -- S9 windowed matcher ("search local points") and S10
 // brute-force matcher (DESIGN.md §3 O9, O10).
 //
-// WINDOW: one thread per map-point query.  Keypoints are in canonical (level, ly, lx)
+// WINDOW: eight lanes per map-point query.  Keypoints are in canonical (level, ly, lx)
 // order, so on each level of the gate [l-1, l] the rows with |y - v| < r (f32) form one
 // contiguous run found by two binary searches on the exact predicate; the run is scanned
 // with the exact |x - u| < r test, the taken mask, and a 256-bit Hamming distance
-// (8 x POPC over 2 x 16-byte loads).  Top-2 by (distance, index) with strict updates in
-// increasing index order; ORB-SLAM's accept rule; a keypoint claimed by several accepted
+// (8 x POPC over 2 x 16-byte loads); the eight lanes split the run and merge their packed
+// (distance << 32 | index) top-2 by shuffles, i.e. top-2 by (distance, index); ORB-SLAM's
+// accept rule; a keypoint claimed by several accepted
 // queries keeps the min (distance, query) (atomicMin on packed u64, then a resolve pass).
 // BRUTE: map tiles staged in shared memory, one thread per frame keypoint keeps a packed
 // (distance << 32 | map index) top-2 per map split; a merge kernel takes the two smallest.
@@ -21,6 +22,17 @@ __device__ __forceinline__ int hamming256(const uint4 a0, const uint4 a1, const 
          __popc(a1.x ^ b1.x) + __popc(a1.y ^ b1.y) + __popc(a1.z ^ b1.z) + __popc(a1.w ^ b1.w);
 }
 
+constexpr int WG = 8;  // lanes cooperating on one query
+
+// top-2 of two packed (distance << 32 | index) pairs
+__device__ __forceinline__ void merge_top2(unsigned long long& a1, unsigned long long& a2, unsigned long long b1,
+                                           unsigned long long b2) {
+  const unsigned long long lo = a1 < b1 ? a1 : b1, hi = a1 < b1 ? b1 : a1;
+  const unsigned long long s2 = a2 < b2 ? a2 : b2;
+  a1 = lo;
+  a2 = hi < s2 ? hi : s2;
+}
+
 __global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const ss_keypoint* __restrict__ kps,
                                                            const uint8_t* __restrict__ desc,
                                                            const int32_t* __restrict__ counts,
@@ -29,11 +41,13 @@ __global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const 
                                                            const uint8_t* __restrict__ qdesc, ss_match_cfg cfg,
                                                            unsigned long long* __restrict__ claim,
                                                            ss_match* __restrict__ out) {
-  const int qi = blockIdx.x * blockDim.x + threadIdx.x;
-  if (qi >= nq) return;
+  const int gt = blockIdx.x * blockDim.x + threadIdx.x;
+  const int qi = gt / WG, sub = gt % WG;
+  const unsigned gmask = 0xFFu << ((threadIdx.x & 31) & ~(WG - 1));
+  if (qi >= nq) return;  // whole groups exit together (WG divides 32)
   const ss_mp_query Q = q[qi];
   const int L = g.L, cap = g.kp_capacity;
-  int d1 = 256, d2 = 256, k1 = -1, k2 = -1;
+  unsigned long long b1 = ~0ull, b2 = ~0ull;  // (distance << 32 | keypoint index)
   const int f = Q.frame;
   if (f >= 0 && f < F) {
     const uint4* qd = reinterpret_cast<const uint4*>(qdesc + (int64_t)qi * SS_DESC_BYTES);
@@ -45,35 +59,43 @@ __global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const 
     const float r = Q.radius, nr = -Q.radius;
     const int l0 = max(Q.pred_level - 1, 0), l1 = min(Q.pred_level, L - 1);
     for (int l = l0; l <= l1; l++) {
-      int lo = cnt[l], hi = cnt[l + 1];
-      // first k with (y_k - v) > -r
+      const int lo = cnt[l], hi = cnt[l + 1];
+      // rows with |y - v| < r form one run [kb, ke) (y non-decreasing, f32 subtract monotone)
       int a = lo, b = hi;
-      while (a < b) {
+      while (a < b) {  // first k with (y_k - v) > -r
         const int m = (a + b) >> 1;
         if (__fsub_rn(fk[m].y, Q.v) > nr) b = m; else a = m + 1;
       }
       const int kb = a;
-      a = kb;
       b = hi;
-      // first k with (y_k - v) >= r
-      while (a < b) {
+      while (a < b) {  // first k with (y_k - v) >= r
         const int m = (a + b) >> 1;
         if (__fsub_rn(fk[m].y, Q.v) >= r) b = m; else a = m + 1;
       }
       const int ke = a;
-      for (int k = kb; k < ke; k++) {
+      for (int k = kb + sub; k < ke; k += WG) {
         const float dx = __fsub_rn(fk[k].x, Q.u);
         if (!(fabsf(dx) < r)) continue;
         if (ft && ft[k]) continue;
         const int d = hamming256(qa, qb, fd[2 * k], fd[2 * k + 1]);
-        if (d < d1) {
-          d2 = d1; k2 = k1; d1 = d; k1 = k;
-        } else if (d < d2) {
-          d2 = d; k2 = k;
+        const unsigned long long key = ((unsigned long long)d << 32) | (unsigned)k;
+        if (key < b1) {
+          b2 = b1;
+          b1 = key;
+        } else if (key < b2) {
+          b2 = key;
         }
       }
     }
   }
+#pragma unroll
+  for (int o = WG / 2; o > 0; o >>= 1) {
+    const unsigned long long o1 = __shfl_xor_sync(gmask, b1, o), o2 = __shfl_xor_sync(gmask, b2, o);
+    merge_top2(b1, b2, o1, o2);
+  }
+  if (sub != 0) return;
+  const int d1 = b1 == ~0ull ? 256 : (int)(b1 >> 32), d2 = b2 == ~0ull ? 256 : (int)(b2 >> 32);
+  const int k1 = b1 == ~0ull ? -1 : (int)(b1 & 0xFFFFFFFFu), k2 = b2 == ~0ull ? -1 : (int)(b2 & 0xFFFFFFFFu);
   bool accept = false;
   if (k1 >= 0 && d1 <= cfg.th) {
     const int lev1 = kps[(int64_t)f * cap + k1].level;
@@ -192,8 +214,9 @@ cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* 
     cudaError_t e = cudaMemsetAsync(claim, 0xFF, (size_t)n_frames * g.kp_capacity * sizeof(unsigned long long), s);
     if (e != cudaSuccess) return e;
   }
-  match_window_kernel<<<(n_queries + 255) / 256, 256, 0, s>>>(g, n_frames, kps, desc, counts, taken, n_queries, q,
-                                                              qdesc, cfg, claim, out);
+  const int64_t threads = (int64_t)n_queries * WG;
+  match_window_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, s>>>(g, n_frames, kps, desc, counts, taken,
+                                                                        n_queries, q, qdesc, cfg, claim, out);
   return cudaGetLastError();
 }
 
