@@ -39,7 +39,7 @@ typedef cub::BlockRadixSort<uint32_t, DT, 8, uint32_t> BRS8;
 typedef cub::BlockScan<int, DT> BScan;
 
 constexpr size_t cmax(size_t a, size_t b) { return a > b ? a : b; }
-constexpr size_t kSmemCells = (size_t)(MAX_CELLS + 1) * 4 * 2;  // offsets + slot offsets
+constexpr size_t kSmemCells = ((size_t)(MAX_CELLS + 1) * 4 * 2 + 127) & ~(size_t)127;  // offsets + slot offsets
 constexpr size_t kSmemArrays = (size_t)DCAP * 12;                // cand, key, rank
 constexpr size_t kUnionPost = (size_t)DCAP * 2 + (size_t)REC_CAP_SMEM * 16;
 constexpr size_t kUnion = cmax(cmax(sizeof(BRS8::TempStorage), sizeof(BRS4::TempStorage)),
