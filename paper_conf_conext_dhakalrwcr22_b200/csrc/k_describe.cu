@@ -90,7 +90,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
   const uint8_t* p0 = img + (int64_t)(ly - 21) * ip + (lx - 21);
   const int sh = (int)(reinterpret_cast<uintptr_t>(p0) & 15);
   const uint8_t* P;  // P[r * PP + c] = raw patch pixel (ly - 21 + r, lx - 21 + c)
-  if ((ip & 15) == 0 && lx >= 21 && ly >= 21 && ly + 21 < h && lx - 21 - sh + 64 <= ip) {
+  if ((ip & 15) == 0 && lx >= 21 && lx + 21 < w && ly >= 21 && ly + 21 < h && lx - 21 - sh + 64 <= ip) {
     // interior: 43 rows x four aligned 16-B chunks, all loads in flight at once
     const uint4* base = reinterpret_cast<const uint4*>(p0 - sh);
     for (int i = lane; i < PR * 4; i += 32) {
