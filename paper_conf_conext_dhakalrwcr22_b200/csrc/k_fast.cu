@@ -2,8 +2,9 @@
 // iniThFAST -> minThFAST fallback (DESIGN.md §3 O2, O3; "parallelization of
 // FAST corner detection ... with the GPU").
 //
-// One CTA per *band* = one row of 30-px FAST cells of one level of one frame (the cells of a
-// row share their detect rows, and their detect windows tile [x0, x1) without gaps):
+// One CTA per *segment* = up to 8 consecutive 30-px FAST cells of one cell row of one level
+// of one frame (the cells of a row share their detect rows and their detect windows tile
+// [x0, x1) without gaps):
 //  1. stage the band + ring halo in shared memory with 16-byte coalesced loads;
 //  2. the score M of EVERY band pixel, four horizontally adjacent pixels per thread: the 16
 //     ring values of the 4 pixels are 16 byte-permutes of a sliding 7-row x 3-word register
@@ -24,7 +25,7 @@ namespace ss {
 
 namespace {
 
-constexpr int FB_WARPS = 16;
+constexpr int FB_WARPS = 8;
 constexpr int FB_THREADS = FB_WARPS * 32;
 constexpr int ROWS_PER_TASK = 8;
 

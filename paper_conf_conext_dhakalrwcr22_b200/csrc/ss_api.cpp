@@ -279,12 +279,15 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   }
   g.pyr_frame_bytes = poff;
   g.total_cells = (int)c->cells_h.size();
-  // bands = rows of cells (same level and detect rows), biggest levels first in the grid
+  // FAST work units: runs of <= kSegCells consecutive cells of one row (same level and detect
+  // rows; their windows tile [x0, x1)), biggest levels first in the grid
+  const int kSegCells = 8;
   g.max_band_w = g.max_band_h = g.max_cell_w = 0;
   for (size_t i = 0; i < c->cells_h.size(); i++) {
     const CellInfo& ci = c->cells_h[i];
     g.max_cell_w = imax(g.max_cell_w, ci.x1 - ci.x0);
-    if (c->bands_h.empty() || c->bands_h.back().level != ci.level || c->bands_h.back().y0 != ci.y0) {
+    if (c->bands_h.empty() || c->bands_h.back().level != ci.level || c->bands_h.back().y0 != ci.y0 ||
+        c->bands_h.back().ncells == kSegCells) {
       BandInfo b;
       b.level = ci.level;
       b.y0 = ci.y0;
