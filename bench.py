@@ -168,9 +168,8 @@ def measured_peaks() -> dict:
 def kernel_work(name: str, p, B: int, n_cand: int, n_kps: int, nq: int, n_map: int) -> tuple[str, float]:
     """(bound, algorithmic bytes) per launch -- DESIGN.md §6 work model."""
     W = [p.level_w[l] * p.level_h[l] for l in range(p.n_levels)]
-    if name.startswith("pyramid_l"):
-        l = int(name[len("pyramid_l"):])
-        return "hbm", float(B * (W[l - 1] + W[l]))
+    if name == "pyramid":  # every level l >= 1 reads level l-1 once and is written once
+        return "hbm", float(B * sum(W[l - 1] + W[l] for l in range(1, p.n_levels)))
     if name == "fast_bands":  # read every level once, write the candidates
         return "hbm", float(B * sum(W) + 4 * n_cand)
     if name == "distribute":  # read candidates, write kept keys
@@ -392,7 +391,7 @@ def run_ours(args, cfg):
 
     frames_per_step = B * world
     value = frames_per_step * K / (T_max / 1000.0)
-    launches_per_step = (L - 1) + 3 + (2 if window else 2)
+    launches_per_step = 4 + 2  # pyramid, fast, distribute, describe + two matcher kernels
     res = {
         "metric": METRIC, "value": value, "unit": "frames/s", "n_gpus": world, "steps": K, "warmup": W_,
         "ms_per_step": T_max / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,

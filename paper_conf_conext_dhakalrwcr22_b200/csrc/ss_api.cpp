@@ -136,6 +136,7 @@ struct ss_ctx {
   int64_t* ovf_level_off = nullptr;
   int32_t* ovf_counter = nullptr;  // [0] overflowed levels, [1] capacity violations
   int8_t* pattern = nullptr;
+  int* pyr_flags = nullptr;  // pyramid dataflow: ticket + per-(frame, level, band) ready flags
   unsigned long long* claim = nullptr;
   unsigned long long* partial = nullptr;
   // profiling hook
@@ -168,7 +169,7 @@ void free_ctx(ss_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->device);
   void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
-                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial};
+                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->pyr_flags};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   delete c;
@@ -330,6 +331,17 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     for (int x = 0; x < g.w[l]; x++) tab.push_back(lin_coef(x, g.w[l - 1], g.w[l]));
     c->yoff[l] = (int64_t)tab.size();
     for (int y = 0; y < g.h[l]; y++) tab.push_back(lin_coef(y, g.h[l - 1], g.h[l]));
+    // the dataflow pyramid stages the source rows of one output band in shared memory
+    const int br = pyramid_band_rows();
+    for (int r0 = 0; r0 < g.h[l]; r0 += br) {
+      const int r1 = imin(r0 + br, g.h[l]) - 1;
+      const uint32_t a = tab[c->yoff[l] + r0], b = tab[c->yoff[l] + r1];
+      const int span = (int)((b & 0xFFFF) + (b >> 25)) - (int)(a & 0xFFFF) + 1;
+      if (span > pyramid_max_src_rows()) {
+        free_ctx(c);
+        return fail(SS_EUNSUPPORTED, "scale_factor too large for the pyramid's 8-row tiles");
+      }
+    }
   }
   // overflow scratch layout
   std::vector<int64_t> ovf_off(L, 0);
@@ -359,6 +371,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->ovf_level_off, sizeof(int64_t) * L);
   ALLOC(c->ovf_counter, sizeof(int32_t) * 2);
   ALLOC(c->pattern, 1024);
+  ALLOC(c->pyr_flags, sizeof(int) * (1 + F * pyramid_flags_per_frame(g)));
   ALLOC(c->claim, sizeof(unsigned long long) * F * g.kp_capacity);
   if (max_map > 0) ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
 #undef ALLOC
@@ -400,10 +413,8 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   FrameSrc src{d_frames, frame_stride, pitch, c->pyr};
   prof_mark(c, s);
   SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 2, s));
-  for (int l = 1; l < g.L; l++) {
-    SS_CUDA_TRY(launch_pyramid_level(g, l, n_frames, src, c->xytab + c->xoff[l], c->xytab + c->yoff[l], s));
-    prof_mark(c, s);
-  }
+  SS_CUDA_TRY(launch_pyramid(g, n_frames, src, c->xytab, c->xoff.data(), c->yoff.data(), c->pyr_flags, s));
+  prof_mark(c, s);
   SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands, c->cells, c->slots, c->cell_counts, s));
   prof_mark(c, s);
   SS_CUDA_TRY(launch_distribute(g, n_frames, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,

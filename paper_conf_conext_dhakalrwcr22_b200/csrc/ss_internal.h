@@ -80,8 +80,13 @@ __host__ __device__ inline int key_ly(uint32_t k) { return (int)(k >> 19); }
 __host__ __device__ inline int key_m(uint32_t k) { return (int)(k & 0xFF); }
 
 // ---- launchers (one per kernel; each returns cudaGetLastError()) ----
-cudaError_t launch_pyramid_level(const Geom& g, int level, int n_frames, FrameSrc src,
-                                 const uint32_t* xtab, const uint32_t* ytab, cudaStream_t s);
+// All pyramid levels of all frames in one dataflow launch; ticket_and_flags = [1 + n_frames *
+// pyramid_flags_per_frame] ints of scratch (zeroed by the launcher on the stream).
+cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const uint32_t* xytab, const int64_t* xoff,
+                           const int64_t* yoff, int* ticket_and_flags, cudaStream_t s);
+int pyramid_flags_per_frame(const Geom& g);
+int pyramid_max_src_rows();
+int pyramid_band_rows();
 cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands,
                               const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s);
 size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int* mband_bytes, int* nball);

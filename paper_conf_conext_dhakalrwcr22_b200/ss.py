@@ -174,7 +174,7 @@ def ss_profile_next(ctx) -> int:
 
 def extract_kernel_names(n_levels: int) -> list[str]:
     """Names of the intervals between consecutive profiling events of one extract call."""
-    return [f"pyramid_l{l}" for l in range(1, n_levels)] + ["fast_bands", "distribute", "describe"]
+    return ["pyramid", "fast_bands", "distribute", "describe"]
 
 
 def window_kernel_names(dedup: bool = True) -> list[str]:
