@@ -5,9 +5,9 @@
 // keypoint (REFLECT_101 at the level border, which the blur needs) in shared memory and
 // derives everything from it: intensity-centroid moments over the 749-px disk (unblurred),
 // the 37x37 blurred patch (Q8 taps [18,34,48,56,48,34,18], exact horizontal sums, vertical
-// (sum + 2^15) >> 16), and the 256 comparisons at the pattern points rotated by
-// (cos, sin) = (m10, m01)/sqrt(m10^2 + m01^2), each offset rounded half-to-even EXACTLY
-// (float estimate + int64 fix-up).  Blurring only the patch replaces a whole-level blur
+// (sum + 2^15) >> 16, computed as two sliding-window passes), and the 256 comparisons at the
+// pattern points rotated by (cos, sin) = (m10, m01)/sqrt(m10^2 + m01^2), each offset rounded
+// half-to-even EXACTLY (f32 estimate; int64 test only within 1e-4 of a tie).  Blurring only the patch replaces a whole-level blur
 // pass and its HBM round trip.  Output position = the keypoint's canonical index, so the
 // per-level counts of the distribution become the prefix offsets written to d_counts.
 #include "brief_pattern.inc"
@@ -21,9 +21,9 @@ constexpr int DESC_WARPS = 8;
 constexpr int PR = 43;  // raw patch: radius 21 (18 max sample offset + 3 blur taps)
 constexpr int PP = 64;  // raw patch pitch: a 16-B aligned 64-B window covers the 43 B row
 constexpr int BR = 37;  // blurred patch: radius 18
-constexpr int HP = 37;  // pitch (u16) of the horizontal pass [43][37]
-constexpr int BP = 40;
-constexpr int PER_WARP = ((PR * PP + PR * HP * 2 + BR * BP) + 127) & ~127;
+constexpr int VP = 46;  // pitch (u16) of the vertical pass V[37][43]: 23 words (odd) per row
+constexpr int BP = 44;  // pitch of the blurred patch B[37][37]: 11 words (odd) per row
+constexpr int PER_WARP = ((PR * PP + BR * VP * 2 + BR * BP) + 127) & ~127;
 
 __constant__ int c_umax[16] = {15, 15, 15, 15, 14, 14, 14, 13, 13, 12, 11, 10, 9, 8, 6, 3};
 
@@ -32,16 +32,25 @@ __device__ __forceinline__ int reflect101(int i, int n) {
   return i >= n ? 2 * n - 2 - i : i;
 }
 
-// Exact round-half-even of z / sqrt(r2), r2 > 0: float estimate, then the integer test
-// (2k-1)^2 r2 < 4 z^2 <= (2k+1)^2 r2 selects k; a tie 4z^2 == (2k+1)^2 r2 goes to even.
-__device__ __forceinline__ int rhe_div_sqrt(long long z, long long r2, float inv_r) {
+// Exact round-half-even of z / sqrt(r2), r2 > 0, |z| < 2^31.  Fast path: t = z * (1/r) in
+// f32 is within 4e-6 of z/r (|z/r| <= 19), so rint(t) is the exact answer unless t lies
+// within 1e-4 of a half-integer; then the integer test (2k-1)^2 r2 < 4 z^2 <= (2k+1)^2 r2
+// selects k and a tie 4z^2 == (2k+1)^2 r2 goes to even.
+__device__ __noinline__ int rhe_exact(long long z, long long r2, int k) {
   const long long a = z < 0 ? -z : z;
   const long long A = 4 * a * a;
-  int k = __float2int_rn((float)a * inv_r);
+  k = k < 0 ? -k : k;
   while (k > 0 && (long long)(2 * k - 1) * (2 * k - 1) * r2 >= A) k--;
   while ((long long)(2 * k + 1) * (2 * k + 1) * r2 < A) k++;
   if ((k & 1) && (long long)(2 * k + 1) * (2 * k + 1) * r2 == A) k++;
   return z < 0 ? -k : k;
+}
+
+__device__ __forceinline__ int rhe_div_sqrt(int z, long long r2, float inv_r) {
+  const float t = __fmul_rn((float)z, inv_r);
+  const float k = rintf(t);
+  if (fabsf(fabsf(t - k) - 0.5f) > 1e-4f) return (int)k;
+  return rhe_exact(z, r2, (int)k);
 }
 
 __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, FrameSrc src,
@@ -85,8 +94,8 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
   }
   const int w = g.w[l], h = g.h[l];
   uint8_t* Pw = sm + warp * PER_WARP;
-  uint16_t* Hs = reinterpret_cast<uint16_t*>(Pw + PR * PP);
-  uint8_t* B = reinterpret_cast<uint8_t*>(Hs + PR * HP);
+  uint16_t* V = reinterpret_cast<uint16_t*>(Pw + PR * PP);
+  uint8_t* B = reinterpret_cast<uint8_t*>(V + BR * VP);
   const uint8_t* p0 = img + (int64_t)(ly - 21) * ip + (lx - 21);
   const int sh = (int)(reinterpret_cast<uintptr_t>(p0) & 15);
   const uint8_t* P;  // P[r * PP + c] = raw patch pixel (ly - 21 + r, lx - 21 + c)
@@ -127,24 +136,35 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
       m01 += __shfl_xor_sync(0xFFFFFFFFu, m01, o);
     }
   }
-  // horizontal blur pass: Hs[r][c] = sum_j k_j P[r][c + j], c in [0, 37)
-  for (int idx = lane; idx < PR * BR; idx += 32) {
-    const int r = idx / BR, c = idx - r * BR;
-    const uint8_t* p = P + r * PP + c;
-    Hs[r * HP + c] = (uint16_t)(18 * (p[0] + p[6]) + 34 * (p[1] + p[5]) + 48 * (p[2] + p[4]) + 56 * p[3]);
+  // separable blur; all sums are exact integers until the final rounding, so the vertical
+  // pass may come first: V[r][x] = sum_i k_i P[r + i][x] (lane = column, sliding over rows),
+  // then B[r][c] = (sum_j k_j V[r][c + j] + 2^15) >> 16 (lane = row, sliding over columns)
+  for (int x = lane; x < PR; x += 32) {
+    int p0 = P[0 * PP + x], p1 = P[1 * PP + x], p2 = P[2 * PP + x], p3 = P[3 * PP + x];
+    int p4 = P[4 * PP + x], p5 = P[5 * PP + x];
+#pragma unroll 4
+    for (int r = 0; r < BR; r++) {
+      const int p6 = P[(r + 6) * PP + x];
+      V[r * VP + x] = (uint16_t)(18 * (p0 + p6) + 34 * (p1 + p5) + 48 * (p2 + p4) + 56 * p3);
+      p0 = p1; p1 = p2; p2 = p3; p3 = p4; p4 = p5; p5 = p6;
+    }
   }
   __syncwarp();
-  for (int idx = lane; idx < BR * BR; idx += 32) {
-    const int r = idx / BR, c = idx - r * BR;
-    const uint16_t* p = Hs + r * HP + c;
-    const int s = 18 * ((int)p[0] + p[6 * HP]) + 34 * ((int)p[HP] + p[5 * HP]) + 48 * ((int)p[2 * HP] + p[4 * HP]) +
-                  56 * (int)p[3 * HP];
-    B[r * BP + c] = (uint8_t)((s + (1 << 15)) >> 16);
+  for (int r = lane; r < BR; r += 32) {
+    const uint16_t* vr = V + r * VP;
+    int v0 = vr[0], v1 = vr[1], v2 = vr[2], v3 = vr[3], v4 = vr[4], v5 = vr[5];
+#pragma unroll 4
+    for (int c = 0; c < BR; c++) {
+      const int v6 = vr[c + 6];
+      const int sum = 18 * (v0 + v6) + 34 * (v1 + v5) + 48 * (v2 + v4) + 56 * v3;
+      B[r * BP + c] = (uint8_t)((sum + (1 << 15)) >> 16);
+      v0 = v1; v1 = v2; v2 = v3; v3 = v4; v4 = v5; v5 = v6;
+    }
   }
   __syncwarp();
   // rotated BRIEF: lane = output byte; bit t compares points 2b, 2b+1 with b = 8*lane + t
   const long long r2 = (long long)m10 * m10 + (long long)m01 * m01;
-  const float inv_r = r2 ? rsqrtf((float)r2) : 0.f;
+  const float inv_r = r2 ? (float)(1.0 / sqrt((double)r2)) : 0.f;
   uint32_t byte = 0;
 #pragma unroll 2
   for (int t = 0; t < 8; t++) {
@@ -155,8 +175,8 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
       const int px = pat[4 * b + 2 * e], py = pat[4 * b + 2 * e + 1];
       int ox = px, oy = py;
       if (r2) {
-        ox = rhe_div_sqrt((long long)px * m10 - (long long)py * m01, r2, inv_r);
-        oy = rhe_div_sqrt((long long)px * m01 + (long long)py * m10, r2, inv_r);
+        ox = rhe_div_sqrt(px * m10 - py * m01, r2, inv_r);  // |.| <= 13 * 2 * 1248480 < 2^31
+        oy = rhe_div_sqrt(px * m01 + py * m10, r2, inv_r);
       }
       v[e] = B[(18 + oy) * BP + 18 + ox];
     }
