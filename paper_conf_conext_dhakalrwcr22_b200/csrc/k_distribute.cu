@@ -46,6 +46,8 @@ constexpr size_t kUnion = cmax(cmax(sizeof(BRS8::TempStorage), sizeof(BRS4::Temp
                                cmax(sizeof(BRS2::TempStorage), kUnionPost));
 constexpr size_t kSmemTotal = kSmemCells + kSmemArrays + kUnion;
 static_assert(kSmemTotal <= 220 * 1024, "distribution smem budget");
+static_assert((size_t)DCAP * 4 + kUnion >= (5464 + 4096 * 2 + 1024) * 4 + 1024 * (8 + 4 + 4 + 1) + 1024,
+              "dense fast-path workspace must fit in the rank + union region");
 
 struct Shared {
   BScan::TempStorage scan;
@@ -167,7 +169,7 @@ __device__ __forceinline__ void distribute_body(const Geom& g, int l, int f, int
                                                 const int32_t* cell_off, const int32_t* cell_slot,
                                                 const uint32_t* __restrict__ slots, uint32_t* __restrict__ selected,
                                                 int32_t* __restrict__ sel_counts, uint8_t* ovf_base,
-                                                int32_t* ovf_counter) {
+                                                int32_t* ovf_counter, bool gathered) {
   const int tid = threadIdx.x;
   const int ncells = g.ncells[l];
   const int N = g.N[l];
@@ -205,7 +207,7 @@ __device__ __forceinline__ void distribute_body(const Geom& g, int l, int f, int
   }
 
   // ---- 2. gather candidates into rank order (cells row-major, raster inside a cell) ----
-  {
+  if (!gathered) {
     const uint32_t* fs = slots + (int64_t)f * g.slots_per_frame;
     for (int i = tid; i < n; i += DT) {
       int lo = 0, hi = ncells - 1;  // last cell with cell_off[c] <= i
@@ -368,6 +370,187 @@ __device__ __forceinline__ void distribute_body(const Geom& g, int l, int f, int
   }
 }
 
+// Fast path for the usual case (n <= DCAP and the stop rules settle at depth <= R, R = the
+// deepest level whose nIni * 4^R node grid fits a dense table): the depth-r node of a key is
+// the dense index key >> (26 - 2r), so node counts per depth are shared-memory histograms
+// (no sort at all); ORB-SLAM's stop rules run on S_r = #non-empty bins, E_r = #bins >= 2;
+// the partial phase-2 round ranks the multi-key bins; the best key of every final node is
+// an atomicMax of (score << 20 | ~rank).  Returns false (nothing written) when the rules
+// need a depth beyond R -- the caller then runs the sort-based body on the same candidates.
+constexpr int DENSE_BINS = 4096;      // nIni * 4^R <= DENSE_BINS
+constexpr int DENSE_TOTAL = 5464;     // sum_{r<=R} nIni * 4^r <= 4/3 DENSE_BINS
+constexpr int DENSE_REC = 1024;       // multi-key bins at the partial depth (<= DENSE_BINS / 4)
+
+__device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* cand, uint32_t* key, uint8_t* ws,
+                           Shared& S_, uint32_t* __restrict__ selected, int32_t* __restrict__ sel_counts,
+                           int32_t* ovf_counter) {
+  const int tid = threadIdx.x;
+  const int N = g.N[l];
+  const int nini = g.nini[l];
+  int R = 0;
+  while (R < 6 && nini << (2 * (R + 1)) <= DENSE_BINS) R++;
+  uint32_t* cnt = reinterpret_cast<uint32_t*>(ws);          // [DENSE_TOTAL] per-depth bins
+  uint32_t* best0 = cnt + DENSE_TOTAL;                        // [DENSE_BINS] depth D
+  uint32_t* best1 = best0 + DENSE_BINS;                       // [DENSE_BINS] depth D + 1
+  uint32_t* first = best1 + DENSE_BINS;                       // [DENSE_BINS / 4] first rank, depth D
+  uint64_t* rec = reinterpret_cast<uint64_t*>(first + DENSE_BINS / 4);  // [DENSE_REC]
+  int32_t* recnode = reinterpret_cast<int32_t*>(rec + DENSE_REC);
+  int32_t* order = recnode + DENSE_REC;
+  uint8_t* recch = reinterpret_cast<uint8_t*>(order + DENSE_REC);
+  uint8_t* split = recch + DENSE_REC;                         // [DENSE_BINS / 4]
+  int off[8], sz[8];
+  {
+    int o = 0;
+    for (int r = 0; r <= R; r++) {
+      off[r] = o;
+      sz[r] = nini << (2 * r);
+      o += sz[r];
+    }
+    for (int i = tid; i < o; i += DT) cnt[i] = 0u;
+    if (tid < 8) {
+      S_.H[tid] = 0;  // non-empty bins per depth
+      S_.G[tid] = 0;  // bins with >= 2 keys per depth
+    }
+  }
+  for (int i = tid; i < n; i += DT) key[i] = make_key(g, l, cand[i]);
+  __syncthreads();
+  for (int i = tid; i < n; i += DT) {
+    const uint32_t k = key[i];
+    for (int r = 0; r <= R; r++) atomicAdd(&cnt[off[r] + (int)(k >> (26 - 2 * r))], 1u);
+  }
+  __syncthreads();
+  for (int r = 0; r <= R; r++) {
+    int nz = 0, mu = 0;
+    for (int b = tid; b < sz[r]; b += DT) {
+      const uint32_t c = cnt[off[r] + b];
+      nz += c > 0u;
+      mu += c > 1u;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      nz += __shfl_xor_sync(0xFFFFFFFFu, nz, o);
+      mu += __shfl_xor_sync(0xFFFFFFFFu, mu, o);
+    }
+    if ((tid & 31) == 0) {
+      if (nz) atomicAdd(&S_.H[r], nz);
+      if (mu) atomicAdd(&S_.G[r], mu);
+    }
+  }
+  __syncthreads();
+  if (tid == 0) {
+    // ORB-SLAM's loop on node counts (as in the sort path); -1 = a depth > R is needed
+    int D = -1, partial = 0, r = 0;
+    for (;;) {
+      if (r + 1 > R) break;
+      const int nx = S_.H[r + 1];
+      if (nx >= N || nx == S_.H[r]) { D = r + 1; break; }
+      if (nx + 3 * S_.G[r + 1] > N) {
+        int d = r + 1;
+        for (;;) {
+          if (d + 1 > R) { d = -1; break; }
+          const int s2 = S_.H[d + 1];
+          if (s2 >= N) { partial = 1; break; }
+          if (s2 == S_.H[d]) { d = d + 1; break; }
+          d++;
+        }
+        D = d;
+        break;
+      }
+      r++;
+    }
+    S_.sh[3] = D;
+    S_.sh[4] = partial;
+    S_.sh[1] = 0;  // records
+    S_.sh[2] = 0;  // kept keys
+  }
+  __syncthreads();
+  const int D = S_.sh[3];
+  if (D < 0) return false;
+  const bool partial = S_.sh[4] != 0;
+  const int szD = nini << (2 * D);
+  for (int b = tid; b < szD; b += DT) best0[b] = 0u;
+  if (partial) {
+    for (int b = tid; b < 4 * szD; b += DT) best1[b] = 0u;
+    for (int b = tid; b < szD; b += DT) {
+      first[b] = 0xFFFFFFFFu;
+      split[b] = 0;
+    }
+    __syncthreads();
+    for (int i = tid; i < n; i += DT) atomicMin(&first[key[i] >> (26 - 2 * D)], (uint32_t)i);
+    __syncthreads();
+    // the multi-key nodes at depth D, ordered by (size desc, UL.y, UL.x, first-key rank)
+    const uint32_t* cD = cnt + off[D];
+    const uint32_t* cD1 = cnt + off[D + 1];
+    for (int b = tid; b < szD; b += DT) {
+      const uint32_t c = cD[b];
+      if (c > 1u) {
+        const int ch = (cD1[4 * b] > 0u) + (cD1[4 * b + 1] > 0u) + (cD1[4 * b + 2] > 0u) + (cD1[4 * b + 3] > 0u);
+        int ulx, uly;
+        node_ul(g, l, (uint32_t)b << (26 - 2 * D), D, ulx, uly);
+        const int e = atomicAdd(&S_.sh[1], 1);
+        rec[e] = ((uint64_t)(0x1FFFFF - c) << 43) | ((uint64_t)uly << 32) | ((uint64_t)ulx << 20) | (uint64_t)first[b];
+        recnode[e] = b;
+        recch[e] = (uint8_t)ch;
+      }
+    }
+    __syncthreads();
+    const int ne = S_.sh[1];
+    for (int e = tid; e < ne; e += DT) {
+      const uint64_t k = rec[e];
+      int pos = 0;
+      for (int e2 = 0; e2 < ne; e2++) pos += rec[e2] < k;
+      order[pos] = e;
+    }
+    __syncthreads();
+    if (tid == 0) {
+      int acc = S_.H[D];
+      for (int t = 0; t < ne && acc < N; t++) {
+        const int e = order[t];
+        acc += recch[e] - 1;
+        split[recnode[e]] = 1;
+      }
+    }
+  }
+  __syncthreads();
+  // best key of every final node: max score, ties -> lowest rank
+  for (int i = tid; i < n; i += DT) {
+    const uint32_t k = key[i];
+    const uint32_t v = ((uint32_t)key_m(cand[i]) << 20) | (0xFFFFFu - (uint32_t)i);
+    const int b = (int)(k >> (26 - 2 * D));
+    if (partial && split[b]) atomicMax(&best1[k >> (26 - 2 * (D + 1))], v);
+    else atomicMax(&best0[b], v);
+  }
+  __syncthreads();
+  uint32_t* kept = key;  // keys are no longer needed
+  const uint32_t* cD = cnt + off[D];
+  for (int b = tid; b < szD; b += DT) {
+    if (cD[b] == 0u) continue;
+    if (partial && split[b]) {
+      for (int q = 0; q < 4; q++) {
+        const uint32_t v = best1[4 * b + q];
+        if (v) kept[atomicAdd(&S_.sh[2], 1)] = cand[0xFFFFFu - (v & 0xFFFFFu)];
+      }
+    } else {
+      kept[atomicAdd(&S_.sh[2], 1)] = cand[0xFFFFFu - (best0[b] & 0xFFFFFu)];
+    }
+  }
+  __syncthreads();
+  const int nk = S_.sh[2];
+  const int nk_w = min(nk, g.cap[l]);
+  uint32_t* sel_out = selected + (int64_t)f * g.kp_capacity + g.cap_off[l];
+  for (int t = tid; t < nk; t += DT) {
+    const uint32_t k = kept[t] >> 8;
+    int pos = 0;
+    for (int u = 0; u < nk; u++) pos += (kept[u] >> 8) < k;
+    if (pos < nk_w) sel_out[pos] = kept[t];
+  }
+  if (tid == 0) {
+    sel_counts[f * g.L + l] = nk_w;
+    if (nk > g.cap[l]) atomicAdd(ovf_counter + 1, 1);
+  }
+  return true;
+}
+
 __global__ void __launch_bounds__(DT, 1)
     distribute_kernel(Geom g, const CellInfo* __restrict__ cells, const uint32_t* __restrict__ slots,
                       const int32_t* __restrict__ cell_counts, uint32_t* __restrict__ selected,
@@ -418,11 +601,38 @@ __global__ void __launch_bounds__(DT, 1)
     if (tid == 0) sel_counts[f * g.L + l] = 0;
     return;
   }
-  if (n <= DCAP)
-    distribute_body<true>(g, l, f, n, sm, S_, cell_off, cell_slot, slots, selected, sel_counts, nullptr, ovf_counter);
-  else
+  if (n <= DCAP) {
+    uint32_t* cand = reinterpret_cast<uint32_t*>(sm + kSmemCells);
+    uint32_t* key = cand + DCAP;
+    {  // gather candidates into rank order (cells row-major, raster inside a cell)
+      const uint32_t* fs = slots + (int64_t)f * g.slots_per_frame;
+      for (int i = tid; i < n; i += DT) {
+        int lo = 0, hi = ncells - 1;  // last cell with cell_off[c] <= i
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (cell_off[mid] <= i) lo = mid; else hi = mid - 1;
+        }
+        cand[i] = fs[cell_slot[lo] + (i - cell_off[lo])];
+      }
+      __syncthreads();
+    }
+    if (dense_body(g, l, f, n, cand, key, reinterpret_cast<uint8_t*>(key + DCAP), S_, selected, sel_counts,
+                   ovf_counter))
+      return;
+    __syncthreads();
+    if (tid < 16) S_.H[tid] = 0;
+    if (tid < 17) S_.G[tid] = 0;
+    if (tid == 0) {
+      S_.sh[1] = 0;
+      S_.sh[2] = 0;
+    }
+    __syncthreads();
+    distribute_body<true>(g, l, f, n, sm, S_, cell_off, cell_slot, slots, selected, sel_counts, nullptr, ovf_counter,
+                          true);
+  } else {
     distribute_body<false>(g, l, f, n, sm, S_, cell_off, cell_slot, slots, selected, sel_counts,
-                           ovf + (int64_t)f * ovf_frame_bytes + ovf_level_off[l], ovf_counter);
+                           ovf + (int64_t)f * ovf_frame_bytes + ovf_level_off[l], ovf_counter, false);
+  }
 }
 
 }  // namespace

@@ -93,7 +93,7 @@ __device__ __forceinline__ uint32_t fast_M4(const uint32_t (&W)[7][3]) {
   return __byte_perm(slo, shi, 0x6240);
 }
 
-__global__ void __launch_bounds__(FB_THREADS) fast_bands_kernel(Geom g, FrameSrc src,
+__global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(Geom g, FrameSrc src,
                                                                 const BandInfo* __restrict__ bands,
                                                                 const CellInfo* __restrict__ cells,
                                                                 uint32_t* __restrict__ slots,
@@ -187,17 +187,27 @@ __global__ void __launch_bounds__(FB_THREADS) fast_bands_kernel(Geom g, FrameSrc
       const int y = lane + 32 * hh;
       if (y < Dh) {
         const uint8_t* rowp = Mb + (y + 1) * mbw + cx0;
-        for (int x = 0; x < cw; x++) {
-          const int m = rowp[x];
-          if (m > tmin) {
-            const uint8_t* p = rowp + x;
-            bool mx = m > p[-mbw] && m > p[mbw];
-            if (x > 0) mx = mx && m > p[-mbw - 1] && m > p[-1] && m > p[mbw - 1];
-            if (x < cw - 1) mx = mx && m > p[-mbw + 1] && m > p[1] && m > p[mbw + 1];
-            if (mx) {
-              kmin[hh] |= 1ull << x;
-              if (m > tini) kini[hh] |= 1ull << x;
-            }
+        // pass 1: scores above minTh (independent loads, 8 per step), pass 2: their neighbours
+        unsigned long long cand = 0ull;
+        for (int x0 = 0; x0 < cw; x0 += 8) {
+          int m[8];
+#pragma unroll
+          for (int q = 0; q < 8; q++) m[q] = rowp[x0 + q];  // row has >= 8 B of slack past cw
+#pragma unroll
+          for (int q = 0; q < 8; q++)
+            if (m[q] > tmin && x0 + q < cw) cand |= 1ull << (x0 + q);
+        }
+        while (cand) {
+          const int x = __ffsll((long long)cand) - 1;
+          cand &= cand - 1;
+          const uint8_t* p = rowp + x;
+          const int m = p[0];
+          bool mx = m > p[-mbw] && m > p[mbw];
+          if (x > 0) mx = mx && m > p[-mbw - 1] && m > p[-1] && m > p[mbw - 1];
+          if (x < cw - 1) mx = mx && m > p[-mbw + 1] && m > p[1] && m > p[mbw + 1];
+          if (mx) {
+            kmin[hh] |= 1ull << x;
+            if (m > tini) kini[hh] |= 1ull << x;
           }
         }
       }
@@ -235,7 +245,7 @@ size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int*
   const int sw = ((g.max_band_w + 31 + 3 + 4 + 4) + 15) & ~15;
   *rp = sw + 16;
   *region_bytes = ((g.max_band_h + 6) * *rp + 15) & ~15;
-  int m = (sw + 3) & ~3;
+  int m = (sw + 8 + 3) & ~3;  // + 8: the NMS reads 8 scores per step past a cell's last column
   if (((m >> 2) & 1) == 0) m += 4;  // odd word pitch: lane-per-row reads hit distinct banks
   *mbw = m;
   *mband_bytes = ((g.max_band_h + 2) * m + 15) & ~15;
