@@ -136,7 +136,10 @@ struct ss_ctx {
   int64_t* ovf_level_off = nullptr;
   int32_t* ovf_counter = nullptr;  // [0] overflowed levels, [1] capacity violations
   int8_t* pattern = nullptr;
-  int* pyr_flags = nullptr;  // pyramid dataflow: ticket + per-(frame, level, band) ready flags
+  PyrStrip* pyr_strips = nullptr;  // pyramid work units
+  int n_pyr_strips = 0;
+  int pyr_buf_bytes = 0;
+  PyrTabs pyr_tabs{};
   unsigned long long* claim = nullptr;
   unsigned long long* partial = nullptr;
   // profiling hook
@@ -169,7 +172,7 @@ void free_ctx(ss_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->device);
   void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
-                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->pyr_flags};
+                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->pyr_strips};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   delete c;
@@ -331,17 +334,52 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     for (int x = 0; x < g.w[l]; x++) tab.push_back(lin_coef(x, g.w[l - 1], g.w[l]));
     c->yoff[l] = (int64_t)tab.size();
     for (int y = 0; y < g.h[l]; y++) tab.push_back(lin_coef(y, g.h[l - 1], g.h[l]));
-    // the dataflow pyramid stages the source rows of one output band in shared memory
-    const int br = pyramid_band_rows();
-    for (int r0 = 0; r0 < g.h[l]; r0 += br) {
-      const int r1 = imin(r0 + br, g.h[l]) - 1;
-      const uint32_t a = tab[c->yoff[l] + r0], b = tab[c->yoff[l] + r1];
-      const int span = (int)((b & 0xFFFF) + (b >> 25)) - (int)(a & 0xFFFF) + 1;
-      if (span > pyramid_max_src_rows()) {
-        free_ctx(c);
-        return fail(SS_EUNSUPPORTED, "scale_factor too large for the pyramid's 8-row tiles");
+  }
+  // pyramid strips: the fewest vertical strips whose two level buffers fit in shared memory
+  std::vector<PyrStrip> strips;
+  int pyr_buf = 0;
+  for (int S = imax(1, (g.W + 95) / 96); S <= 64; S++) {
+    strips.assign(S, PyrStrip{});
+    int need = 0;
+    for (int si = 0; si < S; si++) {
+      PyrStrip& st = strips[si];
+      for (int l = 0; l < kMaxLevels; l++) st.c0[l] = st.c1[l] = st.p0[l] = st.p1[l] = 0;
+      for (int l = L - 1; l >= 1; l--) {
+        st.p0[l] = (int)((int64_t)si * g.w[l] / S);
+        st.p1[l] = (int)((int64_t)(si + 1) * g.w[l] / S);
+        int lo = st.p0[l], hi = st.p1[l];
+        if (l + 1 < L && st.c1[l + 1] > st.c0[l + 1]) {
+          const uint32_t a = tab[c->xoff[l + 1] + st.c0[l + 1]], b = tab[c->xoff[l + 1] + st.c1[l + 1] - 1];
+          lo = imin(lo, (int)(a & 0xFFFF));
+          hi = imax(hi, (int)(b & 0xFFFF) + (int)(b >> 25) + 1);
+        }
+        st.c0[l] = lo;
+        st.c1[l] = hi;
       }
+      {
+        const uint32_t a = tab[c->xoff[1] + st.c0[1]], b = tab[c->xoff[1] + st.c1[1] - 1];
+        st.c0[0] = (int)(a & 0xFFFF);
+        st.c1[0] = (int)(b & 0xFFFF) + (int)(b >> 25) + 1;
+      }
+      const int a0 = st.c0[0] & ~15;
+      need = imax(need, g.h[0] * (((st.c1[0] - a0) + 15) & ~15));
+      for (int l = 1; l < L; l++) need = imax(need, g.h[l] * (((st.c1[l] - st.c0[l]) + 3) & ~3));
     }
+    need = (need + 15) & ~15;
+    if (2 * need <= 220 * 1024) {
+      pyr_buf = need;
+      break;
+    }
+  }
+  if (pyr_buf == 0) {
+    free_ctx(c);
+    return fail(SS_EUNSUPPORTED, "pyramid strips do not fit in shared memory");
+  }
+  c->n_pyr_strips = (int)strips.size();
+  c->pyr_buf_bytes = pyr_buf;
+  for (int l = 0; l < kMaxLevels; l++) {
+    c->pyr_tabs.xoff[l] = l < L ? c->xoff[l] : 0;
+    c->pyr_tabs.yoff[l] = l < L ? c->yoff[l] : 0;
   }
   // overflow scratch layout
   std::vector<int64_t> ovf_off(L, 0);
@@ -371,7 +409,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->ovf_level_off, sizeof(int64_t) * L);
   ALLOC(c->ovf_counter, sizeof(int32_t) * 2);
   ALLOC(c->pattern, 1024);
-  ALLOC(c->pyr_flags, sizeof(int) * (1 + F * pyramid_flags_per_frame(g)));
+  ALLOC(c->pyr_strips, sizeof(PyrStrip) * strips.size());
   ALLOC(c->claim, sizeof(unsigned long long) * F * g.kp_capacity);
   if (max_map > 0) ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
 #undef ALLOC
@@ -379,6 +417,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (e == cudaSuccess) e = cudaMemcpy(c->bands, c->bands_h.data(), sizeof(BandInfo) * c->bands_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess && !tab.empty()) e = cudaMemcpy(c->xytab, tab.data(), sizeof(uint32_t) * tab.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->ovf_level_off, ovf_off.data(), sizeof(int64_t) * L, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(c->pyr_strips, strips.data(), sizeof(PyrStrip) * strips.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->pattern, pat.data(), 1024, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemset(c->ovf_counter, 0, sizeof(int32_t) * 2);
   if (e == cudaSuccess) e = cudaMemset(c->sel_counts, 0, sizeof(int32_t) * F * L);
@@ -413,7 +452,8 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   FrameSrc src{d_frames, frame_stride, pitch, c->pyr};
   prof_mark(c, s);
   SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 2, s));
-  SS_CUDA_TRY(launch_pyramid(g, n_frames, src, c->xytab, c->xoff.data(), c->yoff.data(), c->pyr_flags, s));
+  SS_CUDA_TRY(launch_pyramid(g, n_frames, src, c->pyr_strips, c->n_pyr_strips, c->xytab, c->pyr_tabs,
+                             c->pyr_buf_bytes, s));
   prof_mark(c, s);
   SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands, c->cells, c->slots, c->cell_counts, s));
   prof_mark(c, s);

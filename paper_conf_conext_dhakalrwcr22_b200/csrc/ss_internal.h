@@ -80,13 +80,18 @@ __host__ __device__ inline int key_ly(uint32_t k) { return (int)(k >> 19); }
 __host__ __device__ inline int key_m(uint32_t k) { return (int)(k & 0xFF); }
 
 // ---- launchers (one per kernel; each returns cudaGetLastError()) ----
-// All pyramid levels of all frames in one dataflow launch; ticket_and_flags = [1 + n_frames *
-// pyramid_flags_per_frame] ints of scratch (zeroed by the launcher on the stream).
-cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const uint32_t* xytab, const int64_t* xoff,
-                           const int64_t* yoff, int* ticket_and_flags, cudaStream_t s);
-int pyramid_flags_per_frame(const Geom& g);
-int pyramid_max_src_rows();
-int pyramid_band_rows();
+// Pyramid work unit: one vertical strip of every level.  Level l's cone [c0, c1) = the
+// columns the CTA computes (its own partition [p0, p1) widened by what level l+1 reads);
+// c0[0]/c1[0] = the level-0 columns it stages.
+struct PyrStrip {
+  int32_t c0[kMaxLevels], c1[kMaxLevels], p0[kMaxLevels], p1[kMaxLevels];
+};
+struct PyrTabs {
+  int64_t xoff[kMaxLevels], yoff[kMaxLevels];  // offsets of level l's x / y coefficient tables
+};
+// All levels of all frames in one launch, one CTA per (strip, frame), buffers in shared memory.
+cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const PyrStrip* strips, int n_strips,
+                           const uint32_t* xytab, PyrTabs tabs, int buf_bytes, cudaStream_t s);
 cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands,
                               const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s);
 size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int* mband_bytes, int* nball);
