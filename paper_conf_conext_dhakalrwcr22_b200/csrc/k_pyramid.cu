@@ -60,20 +60,30 @@ __global__ void __launch_bounds__(PT) pyramid_strips_kernel(Geom g, FrameSrc src
     uint8_t* dst = src.pyr + (int64_t)f * g.pyr_frame_bytes + g.lvl_off[l];
     const int dp = g.pitch[l];
     const int p0 = st.p0[l], p1 = st.p1[l];
-    for (int i = threadIdx.x; i < hl * wdt; i += PT) {
-      const int y = i / wdt, xx = i - y * wdt;
-      const int x = c0 + xx;
-      const uint32_t cy = __ldg(ytab + y), cx = __ldg(xtab + x);
+    const int ng = (wdt + 3) >> 2;  // 4 output columns per thread step
+    for (int i = threadIdx.x; i < hl * ng; i += PT) {
+      const int y = i / ng, gx = (i - y * ng) * 4;
+      const uint32_t cy = __ldg(ytab + y);
       const int y0 = (int)(cy & 0xFFFF), wy1 = (int)((cy >> 16) & 0x1FF), y1 = y0 + (int)(cy >> 25);
-      const int x0 = (int)(cx & 0xFFFF) - a, wx1 = (int)((cx >> 16) & 0x1FF), x1 = x0 + (int)(cx >> 25);
-      const uint8_t* r0 = A + y0 * pa;
-      const uint8_t* r1 = A + y1 * pa;
-      const int wx0 = 256 - wx1;
-      const int h0 = wx0 * r0[x0] + wx1 * r0[x1];
-      const int h1 = wx0 * r1[x0] + wx1 * r1[x1];
-      const int v = ((256 - wy1) * h0 + wy1 * h1 + (1 << 15)) >> 16;
-      Bf[y * pb + xx] = (uint8_t)v;
-      if (x >= p0 && x < p1) dst[(int64_t)y * dp + x] = (uint8_t)v;
+      const uint8_t* r0 = A + y0 * pa - a;
+      const uint8_t* r1 = A + y1 * pa - a;
+      uint8_t* brow = Bf + y * pb;
+      uint8_t* drow = dst + (int64_t)y * dp;
+#pragma unroll
+      for (int q = 0; q < 4; q++) {
+        const int xx = gx + q;
+        if (xx < wdt) {
+          const int x = c0 + xx;
+          const uint32_t cx = __ldg(xtab + x);
+          const int x0 = (int)(cx & 0xFFFF), wx1 = (int)((cx >> 16) & 0x1FF), x1 = x0 + (int)(cx >> 25);
+          const int wx0 = 256 - wx1;
+          const int h0 = wx0 * r0[x0] + wx1 * r0[x1];
+          const int h1 = wx0 * r1[x0] + wx1 * r1[x1];
+          const int v = ((256 - wy1) * h0 + wy1 * h1 + (1 << 15)) >> 16;
+          brow[xx] = (uint8_t)v;
+          if (x >= p0 && x < p1) drow[x] = (uint8_t)v;
+        }
+      }
     }
     __syncthreads();
     uint8_t* t = A;

@@ -338,7 +338,10 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   // pyramid strips: the fewest vertical strips whose two level buffers fit in shared memory
   std::vector<PyrStrip> strips;
   int pyr_buf = 0;
-  for (int S = imax(1, (g.W + 95) / 96); S <= 64; S++) {
+  // more strips than the smem bound needs, so that a batch fills the GPU (>= ~2 CTAs per SM);
+  // the price is the recomputed cone halo (~10 columns per side on level 1)
+  const int s_fill = imin(32, (2 * 148 + max_frames - 1) / max_frames);
+  for (int S = imax(s_fill, (g.W + 95) / 96); S <= 64; S++) {
     strips.assign(S, PyrStrip{});
     int need = 0;
     for (int si = 0; si < S; si++) {
