@@ -165,23 +165,27 @@ def measured_peaks() -> dict:
 
 
 # ----------------------------------------------------------------------------- algorithmic work
-def kernel_work(name: str, p, B: int, n_cand: int, n_kps: int, nq: int, n_map: int) -> tuple[str, float]:
-    """(bound, algorithmic bytes) per launch -- DESIGN.md §6 work model."""
+def kernel_work(name: str, p, B: int, cand_l: list, kps_l: list, nq: int, n_map: int) -> tuple[str, float]:
+    """(bound, algorithmic bytes or work) per launch -- DESIGN.md §6 work model.
+    cand_l / kps_l: candidates / kept keypoints per level summed over the batch."""
     W = [p.level_w[l] * p.level_h[l] for l in range(p.n_levels)]
+    L = p.n_levels
     if name == "pyramid":  # every level l >= 1 reads level l-1 once and is written once
-        return "hbm", float(B * sum(W[l - 1] + W[l] for l in range(1, p.n_levels)))
-    if name == "fast_bands":  # read every level once, write the candidates
-        return "hbm", float(B * sum(W) + 4 * n_cand)
-    if name == "distribute":  # read candidates, write kept keys
-        return "hbm", float(4 * n_cand + 4 * n_kps)
+        return "hbm", float(B * sum(W[l - 1] + W[l] for l in range(1, L)))
+    if name in ("fast_l0", "fast_l1plus"):  # read the level pixels, write 4 B per candidate
+        ls = [0] if name == "fast_l0" else list(range(1, L))
+        return "hbm", float(sum(B * W[l] + 4 * cand_l[l] for l in ls))
+    if name in ("distribute_l0", "distribute_l1plus"):  # read candidates, write kept keys
+        ls = [0] if name == "distribute_l0" else list(range(1, L))
+        return "hbm", float(sum(4 * cand_l[l] + 4 * kps_l[l] for l in ls))
     if name == "describe":  # 43x43 patch per keypoint (L2 gathers) + 52 B written per keypoint
-        return "hbm", float(n_kps * (43 * 43 + 4 + 52))
+        return "hbm", float(sum(kps_l) * (43 * 43 + 4 + 52))
     if name == "match_window":  # query 20 B + descriptor 32 B read, 12 B written
         return "hbm", float(nq * 64)
     if name == "match_resolve":
         return "hbm", float(nq * 12)
     if name == "brute_partial":
-        return "popc", float(n_kps) * n_map  # distances
+        return "popc", float(sum(kps_l)) * n_map  # distances
     return "hbm", 0.0
 
 
@@ -264,9 +268,9 @@ def run_ours(args, cfg):
 
     # --- one CUDA graph per ring slot (plain, timed) + an instrumented twin whose profiling
     #     events (recorded inside the graph) give every kernel's duration
-    names = ss.extract_kernel_names(L) + (["gap"] + ss.window_kernel_names(True) if window
-                                          else ["gap"] + ss.brute_kernel_names())
-    n_ev = len(names) + 1
+    mode = ss.SS_MATCH_WINDOW if window else ss.SS_MATCH_BRUTE
+    intervals = ss.EXTRACT_INTERVALS + ss.match_intervals(mode, True, base=ss.EXTRACT_EVENTS)
+    n_ev = ss.EXTRACT_EVENTS + ss.match_events(mode, True)
     events = [[torch.cuda.Event(enable_timing=True) for _ in range(n_ev)] for _ in range(n_slots)]
     for evs in events:  # torch creates the CUDA event lazily, at its first record
         for e in evs:
@@ -345,24 +349,21 @@ def run_ours(args, cfg):
         run_steps(W_, K, graphs_prof)
     torch.cuda.synchronize(dev)
     prof_slots = sorted({(W_ + i) % n_slots for i in range(K)})
-    per_kernel = {n: [] for n in names}
+    per_kernel = {n: [] for n, _, _ in intervals}
     prof_step_ms = []
     for s in prof_slots:
         ev = events[s]
-        for i, n in enumerate(names):
-            per_kernel[n].append(ev[i].elapsed_time(ev[i + 1]))
+        for n, starts, end in intervals:  # an interval starts at the latest of its start events
+            per_kernel[n].append(min(ev[i].elapsed_time(ev[end]) for i in starts))
         prof_step_ms.append(ev[0].elapsed_time(ev[-1]))
-    avg_us = {n: 1000.0 * float(np.mean(v)) for n, v in per_kernel.items() if n != "gap"}
+    avg_us = {n: 1000.0 * float(np.mean(v)) for n, v in per_kernel.items()}
 
     # --- work model for the roofline of the dominant kernel
     kps_h, desc_h, counts_h = pipe.results(B)  # last step's outputs
-    n_kps = int(counts_h[:, -1].sum())
-    n_cand = 0
-    for b in range(B):
-        for l in range(L):
-            n_cand += len(ss.ss_debug_candidates(pipe.ctx, b, l)[0])
+    kps_l = [int((counts_h[:, l + 1] - counts_h[:, l]).sum()) for l in range(L)]
+    cand_l = [sum(len(ss.ss_debug_candidates(pipe.ctx, b, l)[0]) for b in range(B)) for l in range(L)]
     dom = max(avg_us, key=avg_us.get)
-    bound, work = kernel_work(dom, p, B, n_cand, n_kps, Q, cfg["map"])
+    bound, work = kernel_work(dom, p, B, cand_l, kps_l, Q, cfg["map"])
     peaks = measured_peaks()
     step_share = avg_us[dom] / (1000.0 * float(np.mean(prof_step_ms)))
     if bound == "hbm":
@@ -391,7 +392,7 @@ def run_ours(args, cfg):
 
     frames_per_step = B * world
     value = frames_per_step * K / (T_max / 1000.0)
-    launches_per_step = 4 + 2  # pyramid, fast, distribute, describe + two matcher kernels
+    launches_per_step = 6 + 2  # pyramid, 2x fast, 2x distribute, describe + two matcher kernels
     res = {
         "metric": METRIC, "value": value, "unit": "frames/s", "n_gpus": world, "steps": K, "warmup": W_,
         "ms_per_step": T_max / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,

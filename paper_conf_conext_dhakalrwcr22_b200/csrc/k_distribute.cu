@@ -555,10 +555,10 @@ __global__ void __launch_bounds__(DT, 1)
     distribute_kernel(Geom g, const CellInfo* __restrict__ cells, const uint32_t* __restrict__ slots,
                       const int32_t* __restrict__ cell_counts, uint32_t* __restrict__ selected,
                       int32_t* __restrict__ sel_counts, uint8_t* ovf, int64_t ovf_frame_bytes,
-                      const int64_t* __restrict__ ovf_level_off, int32_t* ovf_counter) {
+                      const int64_t* __restrict__ ovf_level_off, int32_t* ovf_counter, int level0) {
   extern __shared__ __align__(16) uint8_t sm[];
   __shared__ Shared S_;
-  const int l = blockIdx.x, f = blockIdx.y, tid = threadIdx.x;
+  const int l = level0 + blockIdx.x, f = blockIdx.y, tid = threadIdx.x;
   const int ncells = g.ncells[l];
   const int c0 = g.cell_first[l];
   int32_t* cell_off = reinterpret_cast<int32_t*>(sm);
@@ -644,18 +644,19 @@ int64_t distribute_ovf_bytes(int64_t slots) {
   return (b + 255) & ~(int64_t)255;
 }
 
-cudaError_t launch_distribute(const Geom& g, int n_frames, const CellInfo* cells, const uint32_t* slots,
-                              const int32_t* cell_counts, uint32_t* selected, int32_t* sel_counts, uint8_t* ovf,
-                              int64_t ovf_frame_bytes, const int64_t* ovf_level_off, int32_t* ovf_counter,
+cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_levels, const CellInfo* cells,
+                              const uint32_t* slots, const int32_t* cell_counts, uint32_t* selected, int32_t* sel_counts,
+                              uint8_t* ovf, int64_t ovf_frame_bytes, const int64_t* ovf_level_off, int32_t* ovf_counter,
                               cudaStream_t s) {
+  if (n_levels <= 0) return cudaSuccess;
   static bool attr_set = false;
   if (!attr_set) {
     cudaFuncSetAttribute(distribute_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemTotal);
     attr_set = true;
   }
-  dim3 grid(g.L, n_frames);
+  dim3 grid(n_levels, n_frames);
   distribute_kernel<<<grid, DT, kSmemTotal, s>>>(g, cells, slots, cell_counts, selected, sel_counts, ovf,
-                                                 ovf_frame_bytes, ovf_level_off, ovf_counter);
+                                                 ovf_frame_bytes, ovf_level_off, ovf_counter, level0);
   return cudaGetLastError();
 }
 

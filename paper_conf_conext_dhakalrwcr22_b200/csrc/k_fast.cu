@@ -253,8 +253,9 @@ size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int*
   return (size_t)*region_bytes + *mband_bytes;
 }
 
-cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands,
+cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands, int n_bands,
                               const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s) {
+  if (n_bands <= 0) return cudaSuccess;
   int rp, mbw, rb, mb, nb;
   const size_t smem = fast_smem_bytes(g, &rp, &mbw, &rb, &mb, &nb);
   static bool attr_set = false;
@@ -262,7 +263,7 @@ cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const B
     cudaFuncSetAttribute(fast_bands_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     attr_set = true;
   }
-  dim3 grid(g.total_bands, n_frames);
+  dim3 grid(n_bands, n_frames);
   fast_bands_kernel<<<grid, FB_THREADS, smem, s>>>(g, src, bands, cells, slots, cell_counts, rp, mbw, rb);
   return cudaGetLastError();
 }

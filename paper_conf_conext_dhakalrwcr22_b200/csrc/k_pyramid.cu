@@ -23,11 +23,14 @@ __global__ void __launch_bounds__(PT) pyramid_strips_kernel(Geom g, FrameSrc src
                                                             const uint32_t* __restrict__ xytab, PyrTabs tabs,
                                                             int buf_bytes) {
   extern __shared__ __align__(16) uint8_t sm[];
-  const PyrStrip st = strips[blockIdx.x];
+  __shared__ PyrStrip st;
   const int f = blockIdx.y;
-  uint8_t* A = sm;              // level l-1 cone, rows x [c0 - a, c1 - a)
-  uint8_t* Bf = sm + buf_bytes; // level l cone
-  // ---- stage the level-0 cone (all rows): columns [a0, c1_0) with a0 = c0_0 rounded down to 16 ----
+  if (threadIdx.x < (int)(sizeof(PyrStrip) / 4))
+    reinterpret_cast<int32_t*>(&st)[threadIdx.x] = reinterpret_cast<const int32_t*>(strips + blockIdx.x)[threadIdx.x];
+  __syncthreads();
+  uint8_t* A = sm;               // level l-1 cone, staged columns [a, a + pa)
+  uint8_t* Bf = sm + buf_bytes;  // level l cone
+  // ---- stage the level-0 cone (all rows): columns [a, c1_0) with a = c0_0 rounded down to 16 ----
   int a = st.c0[0] & ~15;
   int pa = ((st.c1[0] - a) + 15) & ~15;  // staged pitch
   {
@@ -50,38 +53,36 @@ __global__ void __launch_bounds__(PT) pyramid_strips_kernel(Geom g, FrameSrc src
   }
   __syncthreads();
   for (int l = 1; l < g.L; l++) {
-    const int c0 = st.c0[l], c1 = st.c1[l];
-    const int b = c0;  // level l cone starts at column c0 (byte layout, no alignment needed)
-    const int pb = ((c1 - b) + 3) & ~3;
-    const int wdt = c1 - c0;
+    const int c0 = st.c0[l], wdt = st.c1[l] - c0;
+    const int pb = (wdt + 3) & ~3;
     const uint32_t* xtab = xytab + tabs.xoff[l];
     const uint32_t* ytab = xytab + tabs.yoff[l];
     const int hl = g.h[l];
     uint8_t* dst = src.pyr + (int64_t)f * g.pyr_frame_bytes + g.lvl_off[l];
     const int dp = g.pitch[l];
     const int p0 = st.p0[l], p1 = st.p1[l];
-    const int ng = (wdt + 3) >> 2;  // 4 output columns per thread step
-    for (int i = threadIdx.x; i < hl * ng; i += PT) {
-      const int y = i / ng, gx = (i - y * ng) * 4;
-      const uint32_t cy = __ldg(ytab + y);
-      const int y0 = (int)(cy & 0xFFFF), wy1 = (int)((cy >> 16) & 0x1FF), y1 = y0 + (int)(cy >> 25);
-      const uint8_t* r0 = A + y0 * pa - a;
-      const uint8_t* r1 = A + y1 * pa - a;
-      uint8_t* brow = Bf + y * pb;
-      uint8_t* drow = dst + (int64_t)y * dp;
-#pragma unroll
-      for (int q = 0; q < 4; q++) {
-        const int xx = gx + q;
-        if (xx < wdt) {
-          const int x = c0 + xx;
-          const uint32_t cx = __ldg(xtab + x);
-          const int x0 = (int)(cx & 0xFFFF), wx1 = (int)((cx >> 16) & 0x1FF), x1 = x0 + (int)(cx >> 25);
-          const int wx0 = 256 - wx1;
+    // thread = one column of the cone (coefficients loaded once), rows strided by the
+    // number of column groups the CTA covers at once
+    const int nx = wdt < PT ? wdt : PT;
+    const int rstep = PT / nx;
+    const int ty = threadIdx.x / nx;
+    if (ty < rstep) {
+      for (int xx = threadIdx.x - ty * nx; xx < wdt; xx += nx) {
+        const int x = c0 + xx;
+        const uint32_t cx = __ldg(xtab + x);
+        const int x0 = (int)(cx & 0xFFFF) - a, wx1 = (int)((cx >> 16) & 0x1FF), x1 = x0 + (int)(cx >> 25);
+        const int wx0 = 256 - wx1;
+        const bool own = x >= p0 && x < p1;
+        for (int y = ty; y < hl; y += rstep) {
+          const uint32_t cy = __ldg(ytab + y);
+          const int y0 = (int)(cy & 0xFFFF), wy1 = (int)((cy >> 16) & 0x1FF), y1 = y0 + (int)(cy >> 25);
+          const uint8_t* r0 = A + y0 * pa;
+          const uint8_t* r1 = A + y1 * pa;
           const int h0 = wx0 * r0[x0] + wx1 * r0[x1];
           const int h1 = wx0 * r1[x0] + wx1 * r1[x1];
           const int v = ((256 - wy1) * h0 + wy1 * h1 + (1 << 15)) >> 16;
-          brow[xx] = (uint8_t)v;
-          if (x >= p0 && x < p1) drow[x] = (uint8_t)v;
+          Bf[y * pb + xx] = (uint8_t)v;
+          if (own) dst[(int64_t)y * dp + x] = (uint8_t)v;
         }
       }
     }
@@ -89,7 +90,7 @@ __global__ void __launch_bounds__(PT) pyramid_strips_kernel(Geom g, FrameSrc src
     uint8_t* t = A;
     A = Bf;
     Bf = t;
-    a = b;
+    a = c0;
     pa = pb;
   }
 }

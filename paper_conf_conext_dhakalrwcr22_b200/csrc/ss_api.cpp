@@ -142,6 +142,9 @@ struct ss_ctx {
   PyrTabs pyr_tabs{};
   unsigned long long* claim = nullptr;
   unsigned long long* partial = nullptr;
+  // level 0 (FAST + distribution) runs on `aux`, concurrently with the pyramid and levels >= 1
+  cudaStream_t aux = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   // profiling hook
   std::vector<cudaEvent_t> prof;
   size_t prof_next = 0;
@@ -175,6 +178,9 @@ void free_ctx(ss_ctx* c) {
                   c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->pyr_strips};
   for (void* q : ptrs)
     if (q) cudaFree(q);
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_join) cudaEventDestroy(c->ev_join);
+  if (c->aux) cudaStreamDestroy(c->aux);
   delete c;
 }
 
@@ -314,6 +320,8 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     g.max_band_h = imax(g.max_band_h, b.y1 - b.y0);
   }
   g.total_bands = (int)c->bands_h.size();
+  g.level0_bands = 0;
+  for (const BandInfo& b : c->bands_h) g.level0_bands += (b.level == 0);
   {
     int rp, mbw, rb, mb, nb;
     if (fast_smem_bytes(g, &rp, &mbw, &rb, &mb, &nb) > 227 * 1024) {
@@ -423,6 +431,9 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (e == cudaSuccess) e = cudaMemcpy(c->pyr_strips, strips.data(), sizeof(PyrStrip) * strips.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->pattern, pat.data(), 1024, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemset(c->ovf_counter, 0, sizeof(int32_t) * 2);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaMemset(c->sel_counts, 0, sizeof(int32_t) * F * L);
   if (e != cudaSuccess) {
     std::string m = std::string("ss_create: ") + cudaGetErrorString(e);
@@ -453,18 +464,32 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   SS_CUDA_TRY(check_stream(s));
   const Geom& g = c->g;
   FrameSrc src{d_frames, frame_stride, pitch, c->pyr};
-  prof_mark(c, s);
+  // fork: level 0 needs no pyramid, so its FAST + distribution overlap the pyramid and the
+  // levels above it; join before describe (which needs every level's counts)
+  prof_mark(c, s);                                                             // e0
   SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 2, s));
+  SS_CUDA_TRY(cudaEventRecord(c->ev_fork, s));
+  SS_CUDA_TRY(cudaStreamWaitEvent(c->aux, c->ev_fork, 0));
+  prof_mark(c, c->aux);                                                        // e1
+  SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands, g.level0_bands, c->cells, c->slots, c->cell_counts,
+                                c->aux));
+  prof_mark(c, c->aux);                                                        // e2
+  SS_CUDA_TRY(launch_distribute(g, n_frames, 0, 1, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts,
+                                c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, c->aux));
+  prof_mark(c, c->aux);                                                        // e3
+  SS_CUDA_TRY(cudaEventRecord(c->ev_join, c->aux));
   SS_CUDA_TRY(launch_pyramid(g, n_frames, src, c->pyr_strips, c->n_pyr_strips, c->xytab, c->pyr_tabs,
                              c->pyr_buf_bytes, s));
-  prof_mark(c, s);
-  SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands, c->cells, c->slots, c->cell_counts, s));
-  prof_mark(c, s);
-  SS_CUDA_TRY(launch_distribute(g, n_frames, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
-                                c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, s));
-  prof_mark(c, s);
+  prof_mark(c, s);                                                             // e4
+  SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands + g.level0_bands, g.total_bands - g.level0_bands,
+                                c->cells, c->slots, c->cell_counts, s));
+  prof_mark(c, s);                                                             // e5
+  SS_CUDA_TRY(launch_distribute(g, n_frames, 1, g.L - 1, c->cells, c->slots, c->cell_counts, c->selected,
+                                c->sel_counts, c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, s));
+  prof_mark(c, s);                                                             // e6
+  SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join, 0));
   SS_CUDA_TRY(launch_describe(g, n_frames, src, c->selected, c->sel_counts, c->pattern, d_kps, d_desc, d_counts, s));
-  prof_mark(c, s);
+  prof_mark(c, s);                                                             // e7
   c->last_frames = d_frames;
   c->last_stride = frame_stride;
   c->last_pitch = pitch;

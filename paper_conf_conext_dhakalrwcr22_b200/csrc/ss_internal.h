@@ -58,7 +58,8 @@ struct Geom {
   int32_t qw[kMaxLevels], qh[kMaxLevels];  // quadtree box (maxBorder - minBorder)
   int32_t qrounds[kMaxLevels];      // quadtree rounds that can still separate keys on level l
   int32_t max_rw, max_rh;           // largest FAST input region (D + 3-px halo) of any cell
-  int32_t total_bands;              // rows of FAST cells over all levels, per frame
+  int32_t total_bands;              // FAST work units (cell-row segments) over all levels, per frame
+  int32_t level0_bands;             // ... of which on level 0 (they come first)
   int32_t max_band_w, max_band_h;   // widest band (detect columns) / tallest band (detect rows)
   int32_t max_cell_w;               // widest cell detect window
 };
@@ -92,13 +93,13 @@ struct PyrTabs {
 // All levels of all frames in one launch, one CTA per (strip, frame), buffers in shared memory.
 cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const PyrStrip* strips, int n_strips,
                            const uint32_t* xytab, PyrTabs tabs, int buf_bytes, cudaStream_t s);
-cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands,
+cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands, int n_bands,
                               const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s);
 size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int* mband_bytes, int* nball);
-cudaError_t launch_distribute(const Geom& g, int n_frames, const CellInfo* cells, const uint32_t* slots,
-                              const int32_t* cell_counts, uint32_t* selected, int32_t* sel_counts,
-                              uint8_t* ovf, int64_t ovf_frame_bytes, const int64_t* ovf_level_off,
-                              int32_t* ovf_counter, cudaStream_t s);
+cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_levels, const CellInfo* cells,
+                              const uint32_t* slots, const int32_t* cell_counts, uint32_t* selected,
+                              int32_t* sel_counts, uint8_t* ovf, int64_t ovf_frame_bytes,
+                              const int64_t* ovf_level_off, int32_t* ovf_counter, cudaStream_t s);
 cudaError_t launch_describe(const Geom& g, int n_frames, FrameSrc src, const uint32_t* selected,
                             const int32_t* sel_counts, const int8_t* pattern, ss_keypoint* kps, uint8_t* desc,
                             int32_t* counts, cudaStream_t s);

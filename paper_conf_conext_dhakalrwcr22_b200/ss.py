@@ -172,17 +172,23 @@ def ss_profile_next(ctx) -> int:
     return n.value
 
 
-def extract_kernel_names(n_levels: int) -> list[str]:
-    """Names of the intervals between consecutive profiling events of one extract call."""
-    return ["pyramid", "fast_bands", "distribute", "describe"]
+EXTRACT_EVENTS = 8  # profiling events one ss_orb_extract records (include/ss.h)
+# (name, start events (latest wins), end event) of one extract, indices into its events
+EXTRACT_INTERVALS = [("fast_l0", (1,), 2), ("distribute_l0", (2,), 3), ("pyramid", (0,), 4),
+                     ("fast_l1plus", (4,), 5), ("distribute_l1plus", (5,), 6), ("describe", (3, 6), 7)]
 
 
-def window_kernel_names(dedup: bool = True) -> list[str]:
-    return ["match_window"] + (["match_resolve"] if dedup else [])
+def match_events(mode: int, dedup: bool = True) -> int:
+    return 3 if mode == SS_MATCH_BRUTE else (3 if dedup else 2)
 
 
-def brute_kernel_names() -> list[str]:
-    return ["brute_partial", "brute_merge"]
+def match_intervals(mode: int, dedup: bool = True, base: int = 0):
+    if mode == SS_MATCH_BRUTE:
+        return [("brute_partial", (base,), base + 1), ("brute_merge", (base + 1,), base + 2)]
+    out = [("match_window", (base,), base + 1)]
+    if dedup:
+        out.append(("match_resolve", (base + 1,), base + 2))
+    return out
 
 
 def ss_debug_level(ctx, frame, level):
