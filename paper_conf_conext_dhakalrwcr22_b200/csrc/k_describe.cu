@@ -139,17 +139,25 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
   // separable blur; all sums are exact integers until the final rounding, so the vertical
   // pass may come first: V[r][x] = sum_i k_i P[r + i][x] (lane = column, sliding over rows),
   // then B[r][c] = (sum_j k_j V[r][c + j] + 2^15) >> 16 (lane = row, sliding over columns)
-  for (int x = lane; x < PR; x += 32) {
-    int p0 = P[0 * PP + x], p1 = P[1 * PP + x], p2 = P[2 * PP + x], p3 = P[3 * PP + x];
-    int p4 = P[4 * PP + x], p5 = P[5 * PP + x];
+  // pass 1 on packed column pairs: lane covers columns 2*lane, 2*lane + 1 as two 16-bit lanes
+  // of one register (a weighted sum is <= 255 * 256, so the halves never carry)
+  if (lane < (PR + 1) / 2) {
+    const uint16_t* pc = reinterpret_cast<const uint16_t*>(P - (reinterpret_cast<uintptr_t>(P) & 1)) + lane;
+    const int odd = (int)(reinterpret_cast<uintptr_t>(P) & 1);
+    auto ld2 = [&](int r) -> uint32_t {  // bytes (r, 2 lane), (r, 2 lane + 1) -> (lo16, hi16)
+      if (!odd) return __byte_perm((uint32_t)pc[r * (PP / 2)], 0, 0x7170);
+      const uint32_t w = (uint32_t)pc[r * (PP / 2)] | ((uint32_t)pc[r * (PP / 2) + 1] << 16);
+      return __byte_perm(w, 0, 0x7271);
+    };
+    uint32_t q0 = ld2(0), q1 = ld2(1), q2 = ld2(2), q3 = ld2(3), q4 = ld2(4), q5 = ld2(5);
+    uint32_t* V32 = reinterpret_cast<uint32_t*>(V) + lane;
 #pragma unroll 4
     for (int r = 0; r < BR; r++) {
-      const int p6 = P[(r + 6) * PP + x];
-      V[r * VP + x] = (uint16_t)(18 * (p0 + p6) + 34 * (p1 + p5) + 48 * (p2 + p4) + 56 * p3);
-      p0 = p1; p1 = p2; p2 = p3; p3 = p4; p4 = p5; p5 = p6;
+      const uint32_t q6 = ld2(r + 6);
+      V32[r * (VP / 2)] = 18u * (q0 + q6) + 34u * (q1 + q5) + 48u * (q2 + q4) + 56u * q3;
+      q0 = q1; q1 = q2; q2 = q3; q3 = q4; q4 = q5; q5 = q6;
     }
   }
-  __syncwarp();
   for (int r = lane; r < BR; r += 32) {
     const uint16_t* vr = V + r * VP;
     int v0 = vr[0], v1 = vr[1], v2 = vr[2], v3 = vr[3], v4 = vr[4], v5 = vr[5];
@@ -215,7 +223,8 @@ cudaError_t launch_describe(const Geom& g, int n_frames, FrameSrc src, const uin
   const size_t smem = (size_t)DESC_WARPS * PER_WARP;
   static bool attr_set = false;
   if (!attr_set) {
-    cudaFuncSetAttribute(describe_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(describe_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
     attr_set = true;
   }
   dim3 grid((g.kp_capacity + DESC_WARPS - 1) / DESC_WARPS, n_frames);

@@ -651,7 +651,8 @@ cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_lev
   if (n_levels <= 0) return cudaSuccess;
   static bool attr_set = false;
   if (!attr_set) {
-    cudaFuncSetAttribute(distribute_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemTotal);
+    cudaError_t e = cudaFuncSetAttribute(distribute_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemTotal);
+    if (e != cudaSuccess) return e;
     attr_set = true;
   }
   dim3 grid(n_levels, n_frames);

@@ -260,7 +260,8 @@ cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const B
   const size_t smem = fast_smem_bytes(g, &rp, &mbw, &rb, &mb, &nb);
   static bool attr_set = false;
   if (!attr_set) {
-    cudaFuncSetAttribute(fast_bands_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaError_t e = cudaFuncSetAttribute(fast_bands_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 224 * 1024);
+    if (e != cudaSuccess) return e;
     attr_set = true;
   }
   dim3 grid(n_bands, n_frames);

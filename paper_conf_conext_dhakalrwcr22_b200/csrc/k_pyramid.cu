@@ -102,7 +102,9 @@ cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const PyrS
   if (g.L < 2) return cudaSuccess;
   static bool attr_set = false;
   if (!attr_set) {
-    cudaFuncSetAttribute(pyramid_strips_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    // dynamic + static shared memory must stay <= 227 KB
+    cudaError_t e = cudaFuncSetAttribute(pyramid_strips_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 224 * 1024);
+    if (e != cudaSuccess) return e;
     attr_set = true;
   }
   dim3 grid(n_strips, n_frames);
