@@ -4,112 +4,114 @@
 // the host precomputes (x0, wx1, x1-x0) with wx1 = rne(frac * 256); then
 //   out = ((256-wy1)*(wx0*s[y0][x0] + wx1*s[y0][x1]) + wy1*(...row y1...) + 2^15) >> 16.
 //
-// The chain level 1 -> ... -> level L-1 is latency-bound (7 dependent steps over ~1 MB per
-// frame), so one launch builds every level of every frame, one CTA per (vertical strip,
-// frame), entirely in shared memory: the CTA stages the level-0 columns its strip's
-// dependency cone needs, then computes each level over the cone (its own strip widened by
-// the source columns the next level reads) from the previous level in shared memory,
-// writing only its own strip to HBM.  Strips are independent -- cone columns are recomputed
-// by neighbours, never read from them -- so no inter-CTA synchronisation is needed.
+// One launch per level (levels are chained), all frames at once, 128x32 output tiles: the
+// CTA stages the source rectangle the tile reads (<= 48 x 208 B) in shared memory with
+// 16-byte coalesced loads and writes 4 output pixels per thread with one 32-bit store.
+// The chain runs on the main stream while level 0's FAST and distribution run on a second
+// stream (ss_api.cpp), so its latency is off the critical path.
 #include "ss_internal.h"
 
 namespace ss {
 
 namespace {
 
-constexpr int PT = 1024;
+constexpr int TW = 128, TH = 32, PT = 256;
+constexpr int SRC_ROWS = 48, SRC_PITCH = 208;  // >= TH*scale+2 rows, >= TW*scale+2+15 (aligned) cols
 
-__global__ void __launch_bounds__(PT) pyramid_strips_kernel(Geom g, FrameSrc src, const PyrStrip* __restrict__ strips,
-                                                            const uint32_t* __restrict__ xytab, PyrTabs tabs,
-                                                            int buf_bytes) {
-  extern __shared__ __align__(16) uint8_t sm[];
-  __shared__ PyrStrip st;
-  const int f = blockIdx.y;
-  if (threadIdx.x < (int)(sizeof(PyrStrip) / 4))
-    reinterpret_cast<int32_t*>(&st)[threadIdx.x] = reinterpret_cast<const int32_t*>(strips + blockIdx.x)[threadIdx.x];
-  __syncthreads();
-  uint8_t* A = sm;               // level l-1 cone, staged columns [a, a + pa)
-  uint8_t* Bf = sm + buf_bytes;  // level l cone
-  // ---- stage the level-0 cone (all rows): columns [a, c1_0) with a = c0_0 rounded down to 16 ----
-  int a = st.c0[0] & ~15;
-  int pa = ((st.c1[0] - a) + 15) & ~15;  // staged pitch
-  {
-    const uint8_t* s0 = src.frames + (int64_t)f * src.stride;
-    const int h = g.h[0];
-    if ((src.pitch & 15) == 0 && (reinterpret_cast<uintptr_t>(s0) & 15) == 0) {
-      const int nch = pa >> 4;
-      for (int i = threadIdx.x; i < h * nch; i += PT) {
-        const int r = i / nch, c = i - r * nch;
-        *reinterpret_cast<uint4*>(A + r * pa + 16 * c) =
-            __ldg(reinterpret_cast<const uint4*>(s0 + (int64_t)r * src.pitch + a) + c);
-      }
-    } else {
-      const int wdt = st.c1[0] - a;
-      for (int i = threadIdx.x; i < h * wdt; i += PT) {
-        const int r = i / wdt, c = i - r * wdt;
-        A[r * pa + c] = __ldg(s0 + (int64_t)r * src.pitch + a + c);
-      }
+__global__ void __launch_bounds__(PT) pyramid_level_kernel(Geom g, int l, FrameSrc src, const uint32_t* __restrict__ xtab,
+                                                           const uint32_t* __restrict__ ytab) {
+  __shared__ __align__(16) uint8_t s_src[SRC_ROWS * SRC_PITCH];
+  __shared__ uint32_t s_x[TW];
+  const int f = blockIdx.z;
+  const int dw = g.w[l], dh = g.h[l];
+  const int tx0 = blockIdx.x * TW, ty0 = blockIdx.y * TH;
+  const int tx1 = min(tx0 + TW, dw), ty1 = min(ty0 + TH, dh);
+  const uint8_t* s;
+  int sp;
+  if (l == 1) {
+    s = src.frames + (int64_t)f * src.stride;
+    sp = src.pitch;
+  } else {
+    s = src.pyr + (int64_t)f * g.pyr_frame_bytes + g.lvl_off[l - 1];
+    sp = g.pitch[l - 1];
+  }
+  // source rectangle: rows [sy0, sy1], columns [sx0, sx1] (sx0 aligned down to 16)
+  const uint32_t cy0 = __ldg(ytab + ty0), cy1 = __ldg(ytab + ty1 - 1);
+  const int sy0 = (int)(cy0 & 0xFFFF), sy1 = (int)(cy1 & 0xFFFF) + (int)(cy1 >> 25);
+  const uint32_t cx0 = __ldg(xtab + tx0), cx1 = __ldg(xtab + tx1 - 1);
+  const int sx0 = (int)(cx0 & 0xFFFF) & ~15, sx1 = (int)(cx1 & 0xFFFF) + (int)(cx1 >> 25);
+  if (threadIdx.x < TW) s_x[threadIdx.x] = tx0 + (int)threadIdx.x < dw ? __ldg(xtab + tx0 + threadIdx.x) : 0u;
+  const int nrows = sy1 - sy0 + 1;
+  if ((sp & 15) == 0 && (reinterpret_cast<uintptr_t>(s) & 15) == 0) {
+    const int nch = (sx1 - sx0 + 16) >> 4;
+    for (int i = threadIdx.x; i < nrows * nch; i += PT) {
+      const int r = i / nch, c = i - r * nch;
+      *reinterpret_cast<uint4*>(s_src + r * SRC_PITCH + 16 * c) =
+          __ldg(reinterpret_cast<const uint4*>(s + (int64_t)(sy0 + r) * sp + sx0) + c);
+    }
+  } else {
+    const int ncol = sx1 - sx0 + 1;
+    for (int i = threadIdx.x; i < nrows * ncol; i += PT) {
+      const int r = i / ncol, c = i - r * ncol;
+      s_src[r * SRC_PITCH + c] = __ldg(s + (int64_t)(sy0 + r) * sp + sx0 + c);
     }
   }
   __syncthreads();
-  for (int l = 1; l < g.L; l++) {
-    const int c0 = st.c0[l], wdt = st.c1[l] - c0;
-    const int pb = (wdt + 3) & ~3;
-    const uint32_t* xtab = xytab + tabs.xoff[l];
-    const uint32_t* ytab = xytab + tabs.yoff[l];
-    const int hl = g.h[l];
-    uint8_t* dst = src.pyr + (int64_t)f * g.pyr_frame_bytes + g.lvl_off[l];
-    const int dp = g.pitch[l];
-    const int p0 = st.p0[l], p1 = st.p1[l];
-    // thread = one column of the cone (coefficients loaded once), rows strided by the
-    // number of column groups the CTA covers at once
-    const int nx = wdt < PT ? wdt : PT;
-    const int rstep = PT / nx;
-    const int ty = threadIdx.x / nx;
-    if (ty < rstep) {
-      for (int xx = threadIdx.x - ty * nx; xx < wdt; xx += nx) {
-        const int x = c0 + xx;
-        const uint32_t cx = __ldg(xtab + x);
-        const int x0 = (int)(cx & 0xFFFF) - a, wx1 = (int)((cx >> 16) & 0x1FF), x1 = x0 + (int)(cx >> 25);
-        const int wx0 = 256 - wx1;
-        const bool own = x >= p0 && x < p1;
-        for (int y = ty; y < hl; y += rstep) {
-          const uint32_t cy = __ldg(ytab + y);
-          const int y0 = (int)(cy & 0xFFFF), wy1 = (int)((cy >> 16) & 0x1FF), y1 = y0 + (int)(cy >> 25);
-          const uint8_t* r0 = A + y0 * pa;
-          const uint8_t* r1 = A + y1 * pa;
-          const int h0 = wx0 * r0[x0] + wx1 * r0[x1];
-          const int h1 = wx0 * r1[x0] + wx1 * r1[x1];
-          const int v = ((256 - wy1) * h0 + wy1 * h1 + (1 << 15)) >> 16;
-          Bf[y * pb + xx] = (uint8_t)v;
-          if (own) dst[(int64_t)y * dp + x] = (uint8_t)v;
-        }
-      }
+  uint8_t* d = src.pyr + (int64_t)f * g.pyr_frame_bytes + g.lvl_off[l];
+  const int dp = g.pitch[l];
+  const int gx = (threadIdx.x & 31) * 4;  // 32 threads x 4 px = one 128-px tile row
+  for (int y = ty0 + (threadIdx.x >> 5); y < ty1; y += PT / 32) {
+    const uint32_t cy = __ldg(ytab + y);
+    const int y0 = (int)(cy & 0xFFFF) - sy0, wy1 = (int)((cy >> 16) & 0x1FF), y1 = y0 + (int)(cy >> 25);
+    const uint8_t* r0 = s_src + y0 * SRC_PITCH - sx0;
+    const uint8_t* r1 = s_src + y1 * SRC_PITCH - sx0;
+    uint32_t packed = 0;
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+      const uint32_t cx = s_x[gx + q];
+      const int x0 = (int)(cx & 0xFFFF), wx1 = (int)((cx >> 16) & 0x1FF), x1 = x0 + (int)(cx >> 25);
+      const int wx0 = 256 - wx1;
+      const int h0 = wx0 * r0[x0] + wx1 * r0[x1];
+      const int h1 = wx0 * r1[x0] + wx1 * r1[x1];
+      packed |= (uint32_t)(((256 - wy1) * h0 + wy1 * h1 + (1 << 15)) >> 16) << (8 * q);
     }
-    __syncthreads();
-    uint8_t* t = A;
-    A = Bf;
-    Bf = t;
-    a = c0;
-    pa = pb;
+    const int x = tx0 + gx;
+    if (x >= tx1) continue;
+    uint8_t* drow = d + (int64_t)y * dp;
+    if (x + 4 <= tx1) {
+      *reinterpret_cast<uint32_t*>(drow + x) = packed;  // pitch is a multiple of 16
+    } else {
+      for (int q = 0; x + q < tx1; q++) drow[x + q] = (uint8_t)(packed >> (8 * q));
+    }
   }
 }
 
 }  // namespace
 
-cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const PyrStrip* strips, int n_strips,
-                           const uint32_t* xytab, PyrTabs tabs, int buf_bytes, cudaStream_t s) {
-  if (g.L < 2) return cudaSuccess;
-  static bool attr_set = false;
-  if (!attr_set) {
-    // dynamic + static shared memory must stay <= 227 KB
-    cudaError_t e = cudaFuncSetAttribute(pyramid_strips_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 224 * 1024);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
+// Whether every 128x32 tile's source rectangle fits the kernel's shared-memory staging.
+bool pyramid_tiles_fit(int dst_w, int dst_h, const uint32_t* xt, const uint32_t* yt) {
+  for (int ty0 = 0; ty0 < dst_h; ty0 += TH) {
+    const int ty1 = (ty0 + TH < dst_h ? ty0 + TH : dst_h) - 1;
+    const int rows = (int)(yt[ty1] & 0xFFFF) + (int)(yt[ty1] >> 25) - (int)(yt[ty0] & 0xFFFF) + 1;
+    if (rows > SRC_ROWS) return false;
   }
-  dim3 grid(n_strips, n_frames);
-  pyramid_strips_kernel<<<grid, PT, 2 * (size_t)buf_bytes, s>>>(g, src, strips, xytab, tabs, buf_bytes);
-  return cudaGetLastError();
+  for (int tx0 = 0; tx0 < dst_w; tx0 += TW) {
+    const int tx1 = (tx0 + TW < dst_w ? tx0 + TW : dst_w) - 1;
+    const int cols = (int)(xt[tx1] & 0xFFFF) + (int)(xt[tx1] >> 25) - ((int)(xt[tx0] & 0xFFFF) & ~15) + 1;
+    if (((cols + 15) & ~15) > SRC_PITCH) return false;
+  }
+  return true;
+}
+
+cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const uint32_t* xytab, PyrTabs tabs,
+                           cudaStream_t s) {
+  for (int l = 1; l < g.L; l++) {
+    dim3 grid((g.w[l] + TW - 1) / TW, (g.h[l] + TH - 1) / TH, n_frames);
+    pyramid_level_kernel<<<grid, PT, 0, s>>>(g, l, src, xytab + tabs.xoff[l], xytab + tabs.yoff[l]);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
 }
 
 }  // namespace ss

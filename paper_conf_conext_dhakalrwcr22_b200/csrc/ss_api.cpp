@@ -136,9 +136,6 @@ struct ss_ctx {
   int64_t* ovf_level_off = nullptr;
   int32_t* ovf_counter = nullptr;  // [0] overflowed levels, [1] capacity violations
   int8_t* pattern = nullptr;
-  PyrStrip* pyr_strips = nullptr;  // pyramid work units
-  int n_pyr_strips = 0;
-  int pyr_buf_bytes = 0;
   PyrTabs pyr_tabs{};
   unsigned long long* claim = nullptr;
   unsigned long long* partial = nullptr;
@@ -175,7 +172,7 @@ void free_ctx(ss_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->device);
   void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
-                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->pyr_strips};
+                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
@@ -343,51 +340,12 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     c->yoff[l] = (int64_t)tab.size();
     for (int y = 0; y < g.h[l]; y++) tab.push_back(lin_coef(y, g.h[l - 1], g.h[l]));
   }
-  // pyramid strips: the fewest vertical strips whose two level buffers fit in shared memory
-  std::vector<PyrStrip> strips;
-  int pyr_buf = 0;
-  // more strips than the smem bound needs, so that a batch fills the GPU (>= ~2 CTAs per SM);
-  // the price is the recomputed cone halo (~10 columns per side on level 1)
-  const int s_fill = imin(32, (2 * 148 + max_frames - 1) / max_frames);
-  for (int S = imax(s_fill, (g.W + 95) / 96); S <= 64; S++) {
-    strips.assign(S, PyrStrip{});
-    int need = 0;
-    for (int si = 0; si < S; si++) {
-      PyrStrip& st = strips[si];
-      for (int l = 0; l < kMaxLevels; l++) st.c0[l] = st.c1[l] = st.p0[l] = st.p1[l] = 0;
-      for (int l = L - 1; l >= 1; l--) {
-        st.p0[l] = (int)((int64_t)si * g.w[l] / S);
-        st.p1[l] = (int)((int64_t)(si + 1) * g.w[l] / S);
-        int lo = st.p0[l], hi = st.p1[l];
-        if (l + 1 < L && st.c1[l + 1] > st.c0[l + 1]) {
-          const uint32_t a = tab[c->xoff[l + 1] + st.c0[l + 1]], b = tab[c->xoff[l + 1] + st.c1[l + 1] - 1];
-          lo = imin(lo, (int)(a & 0xFFFF));
-          hi = imax(hi, (int)(b & 0xFFFF) + (int)(b >> 25) + 1);
-        }
-        st.c0[l] = lo;
-        st.c1[l] = hi;
-      }
-      {
-        const uint32_t a = tab[c->xoff[1] + st.c0[1]], b = tab[c->xoff[1] + st.c1[1] - 1];
-        st.c0[0] = (int)(a & 0xFFFF);
-        st.c1[0] = (int)(b & 0xFFFF) + (int)(b >> 25) + 1;
-      }
-      const int a0 = st.c0[0] & ~15;
-      need = imax(need, g.h[0] * (((st.c1[0] - a0) + 15) & ~15));
-      for (int l = 1; l < L; l++) need = imax(need, g.h[l] * (((st.c1[l] - st.c0[l]) + 3) & ~3));
-    }
-    need = (need + 15) & ~15;
-    if (2 * need <= 220 * 1024) {
-      pyr_buf = need;
-      break;
+  for (int l = 1; l < L; l++) {
+    if (!pyramid_tiles_fit(g.w[l], g.h[l], tab.data() + c->xoff[l], tab.data() + c->yoff[l])) {
+      free_ctx(c);
+      return fail(SS_EUNSUPPORTED, "scale_factor too large for the pyramid's shared-memory tiles");
     }
   }
-  if (pyr_buf == 0) {
-    free_ctx(c);
-    return fail(SS_EUNSUPPORTED, "pyramid strips do not fit in shared memory");
-  }
-  c->n_pyr_strips = (int)strips.size();
-  c->pyr_buf_bytes = pyr_buf;
   for (int l = 0; l < kMaxLevels; l++) {
     c->pyr_tabs.xoff[l] = l < L ? c->xoff[l] : 0;
     c->pyr_tabs.yoff[l] = l < L ? c->yoff[l] : 0;
@@ -420,7 +378,6 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->ovf_level_off, sizeof(int64_t) * L);
   ALLOC(c->ovf_counter, sizeof(int32_t) * 2);
   ALLOC(c->pattern, 1024);
-  ALLOC(c->pyr_strips, sizeof(PyrStrip) * strips.size());
   ALLOC(c->claim, sizeof(unsigned long long) * F * g.kp_capacity);
   if (max_map > 0) ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
 #undef ALLOC
@@ -428,7 +385,6 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (e == cudaSuccess) e = cudaMemcpy(c->bands, c->bands_h.data(), sizeof(BandInfo) * c->bands_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess && !tab.empty()) e = cudaMemcpy(c->xytab, tab.data(), sizeof(uint32_t) * tab.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->ovf_level_off, ovf_off.data(), sizeof(int64_t) * L, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMemcpy(c->pyr_strips, strips.data(), sizeof(PyrStrip) * strips.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->pattern, pat.data(), 1024, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemset(c->ovf_counter, 0, sizeof(int32_t) * 2);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking);
@@ -478,8 +434,7 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
                                 c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, c->aux));
   prof_mark(c, c->aux);                                                        // e3
   SS_CUDA_TRY(cudaEventRecord(c->ev_join, c->aux));
-  SS_CUDA_TRY(launch_pyramid(g, n_frames, src, c->pyr_strips, c->n_pyr_strips, c->xytab, c->pyr_tabs,
-                             c->pyr_buf_bytes, s));
+  SS_CUDA_TRY(launch_pyramid(g, n_frames, src, c->xytab, c->pyr_tabs, s));
   prof_mark(c, s);                                                             // e4
   SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands + g.level0_bands, g.total_bands - g.level0_bands,
                                 c->cells, c->slots, c->cell_counts, s));

@@ -81,18 +81,14 @@ __host__ __device__ inline int key_ly(uint32_t k) { return (int)(k >> 19); }
 __host__ __device__ inline int key_m(uint32_t k) { return (int)(k & 0xFF); }
 
 // ---- launchers (one per kernel; each returns cudaGetLastError()) ----
-// Pyramid work unit: one vertical strip of every level.  Level l's cone [c0, c1) = the
-// columns the CTA computes (its own partition [p0, p1) widened by what level l+1 reads);
-// c0[0]/c1[0] = the level-0 columns it stages.
-struct PyrStrip {
-  int32_t c0[kMaxLevels], c1[kMaxLevels], p0[kMaxLevels], p1[kMaxLevels];
-};
 struct PyrTabs {
   int64_t xoff[kMaxLevels], yoff[kMaxLevels];  // offsets of level l's x / y coefficient tables
 };
-// All levels of all frames in one launch, one CTA per (strip, frame), buffers in shared memory.
-cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const PyrStrip* strips, int n_strips,
-                           const uint32_t* xytab, PyrTabs tabs, int buf_bytes, cudaStream_t s);
+// Levels 1..L-1 of all frames, one launch per level, 128x32 output tiles.
+cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const uint32_t* xytab, PyrTabs tabs,
+                           cudaStream_t s);
+// Whether every tile's source rectangle fits the kernel's shared-memory staging.
+bool pyramid_tiles_fit(int dst_w, int dst_h, const uint32_t* xt, const uint32_t* yt);
 cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands, int n_bands,
                               const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s);
 size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int* mband_bytes, int* nball);
