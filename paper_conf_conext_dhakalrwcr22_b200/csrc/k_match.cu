@@ -24,6 +24,39 @@ __device__ __forceinline__ int hamming256(const uint4 a0, const uint4 a1, const 
 
 constexpr int WG = 8;  // lanes cooperating on one query
 
+__host__ __device__ __forceinline__ int row_off(const Geom& g, int l) {  // start of level l in a frame's row index
+  int o = 0;
+  for (int i = 0; i < l; i++) o += g.h[i] + 1;
+  return o;
+}
+
+// Per frame and level: rowidx[r] = index of the first keypoint with ly >= r (r in [0, h_l]),
+// from the canonical (level, ly, lx) order; plus the dedup claim table reset.
+__global__ void __launch_bounds__(256) match_prepare(Geom g, int F, const ss_keypoint* __restrict__ kps,
+                                                     const int32_t* __restrict__ counts, uint16_t* __restrict__ rowidx,
+                                                     int rows_per_frame, unsigned long long* __restrict__ claim,
+                                                     int dedup) {
+  const int cap = g.kp_capacity, L = g.L;
+  const int gt = blockIdx.x * blockDim.x + threadIdx.x;
+  if (gt >= F * cap) return;
+  if (dedup) claim[gt] = ~0ull;
+  const int f = gt / cap, k = gt - f * cap;
+  const int32_t* cnt = counts + f * (L + 1);
+  uint16_t* fr = rowidx + (int64_t)f * rows_per_frame;
+  if (k < L && cnt[k] == cnt[k + 1]) {  // empty level k: every row points at its (empty) range
+    uint16_t* ri = fr + row_off(g, k);
+    for (int r = 0; r <= g.h[k]; r++) ri[r] = (uint16_t)cnt[k];
+  }
+  if (k >= cnt[L]) return;
+  const ss_keypoint kp = kps[(int64_t)f * cap + k];
+  const int l = kp.level, ly = kp.ly;
+  uint16_t* ri = fr + row_off(g, l);
+  const int prev = k > cnt[l] ? (int)kps[(int64_t)f * cap + k - 1].ly : -1;
+  for (int r = prev + 1; r <= ly; r++) ri[r] = (uint16_t)k;
+  if (k == cnt[l + 1] - 1)
+    for (int r = ly + 1; r <= g.h[l]; r++) ri[r] = (uint16_t)(k + 1);
+}
+
 // top-2 of two packed (distance << 32 | index) pairs
 __device__ __forceinline__ void merge_top2(unsigned long long& a1, unsigned long long& a2, unsigned long long b1,
                                            unsigned long long b2) {
@@ -40,7 +73,8 @@ __global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const 
                                                            const ss_mp_query* __restrict__ q,
                                                            const uint8_t* __restrict__ qdesc, ss_match_cfg cfg,
                                                            unsigned long long* __restrict__ claim,
-                                                           ss_match* __restrict__ out) {
+                                                           ss_match* __restrict__ out,
+                                                           const uint16_t* __restrict__ rowidx, int rows_per_frame) {
   const int gt = blockIdx.x * blockDim.x + threadIdx.x;
   const int qi = gt / WG, sub = gt % WG;
   const unsigned gmask = 0xFFu << ((threadIdx.x & 31) & ~(WG - 1));
@@ -52,30 +86,25 @@ __global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const 
   if (f >= 0 && f < F) {
     const uint4* qd = reinterpret_cast<const uint4*>(qdesc + (int64_t)qi * SS_DESC_BYTES);
     const uint4 qa = qd[0], qb = qd[1];
-    const int32_t* cnt = counts + f * (L + 1);
     const ss_keypoint* fk = kps + (int64_t)f * cap;
     const uint4* fd = reinterpret_cast<const uint4*>(desc + (int64_t)f * cap * SS_DESC_BYTES);
     const uint8_t* ft = taken ? taken + (int64_t)f * cap : nullptr;
     const float r = Q.radius, nr = -Q.radius;
     const int l0 = max(Q.pred_level - 1, 0), l1 = min(Q.pred_level, L - 1);
+    (void)nr;
+    const uint16_t* fri = rowidx + (int64_t)f * rows_per_frame;
     for (int l = l0; l <= l1; l++) {
-      const int lo = cnt[l], hi = cnt[l + 1];
-      // rows with |y - v| < r form one run [kb, ke) (y non-decreasing, f32 subtract monotone)
-      int a = lo, b = hi;
-      while (a < b) {  // first k with (y_k - v) > -r
-        const int m = (a + b) >> 1;
-        if (__fsub_rn(fk[m].y, Q.v) > nr) b = m; else a = m + 1;
-      }
-      const int kb = a;
-      b = hi;
-      while (a < b) {  // first k with (y_k - v) >= r
-        const int m = (a + b) >> 1;
-        if (__fsub_rn(fk[m].y, Q.v) >= r) b = m; else a = m + 1;
-      }
-      const int ke = a;
+      // rows that can hold |y - v| < r, widened by one row each side (f32 rounding); the exact
+      // test below decides, so the superset only costs a few extra candidates
+      const float s_l = g.scale[l];
+      const int hl = g.h[l];
+      const int rlo = max(0, min(hl, (int)floorf(__fdiv_rn(__fsub_rn(Q.v, r), s_l)) - 1));
+      const int rhi = max(0, min(hl, (int)ceilf(__fdiv_rn(__fadd_rn(Q.v, r), s_l)) + 2));
+      const uint16_t* ri = fri + row_off(g, l);
+      const int kb = ri[rlo], ke = ri[rhi];
       for (int k = kb + sub; k < ke; k += WG) {
-        const float dx = __fsub_rn(fk[k].x, Q.u);
-        if (!(fabsf(dx) < r)) continue;
+        const float dx = __fsub_rn(fk[k].x, Q.u), dy = __fsub_rn(fk[k].y, Q.v);
+        if (!(fabsf(dx) < r && fabsf(dy) < r)) continue;
         if (ft && ft[k]) continue;
         const int d = hamming256(qa, qb, fd[2 * k], fd[2 * k + 1]);
         const unsigned long long key = ((unsigned long long)d << 32) | (unsigned)k;
@@ -205,18 +234,25 @@ __global__ void __launch_bounds__(256) match_brute_merge(Geom g, int F, const in
 
 }  // namespace
 
+int match_rows_per_frame(const Geom& g) { return row_off(g, g.L); }
+
+cudaError_t launch_match_prepare(const Geom& g, int n_frames, const ss_keypoint* kps, const int32_t* counts,
+                                 uint16_t* rowidx, unsigned long long* claim, int dedup, cudaStream_t s) {
+  const int n = n_frames * g.kp_capacity;
+  if (n <= 0) return cudaSuccess;
+  match_prepare<<<(n + 255) / 256, 256, 0, s>>>(g, n_frames, kps, counts, rowidx, match_rows_per_frame(g), claim,
+                                                dedup);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* kps, const uint8_t* desc,
                                 const int32_t* counts, const uint8_t* taken, int n_queries, const ss_mp_query* q,
                                 const uint8_t* qdesc, ss_match_cfg cfg, unsigned long long* claim, ss_match* out,
-                                cudaStream_t s) {
+                                const uint16_t* rowidx, cudaStream_t s) {
   if (n_queries <= 0) return cudaSuccess;
-  if (cfg.dedup) {
-    cudaError_t e = cudaMemsetAsync(claim, 0xFF, (size_t)n_frames * g.kp_capacity * sizeof(unsigned long long), s);
-    if (e != cudaSuccess) return e;
-  }
   const int64_t threads = (int64_t)n_queries * WG;
-  match_window_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, s>>>(g, n_frames, kps, desc, counts, taken,
-                                                                        n_queries, q, qdesc, cfg, claim, out);
+  match_window_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, s>>>(
+      g, n_frames, kps, desc, counts, taken, n_queries, q, qdesc, cfg, claim, out, rowidx, match_rows_per_frame(g));
   return cudaGetLastError();
 }
 

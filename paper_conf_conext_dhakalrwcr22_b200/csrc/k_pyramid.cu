@@ -40,7 +40,8 @@ __global__ void __launch_bounds__(PT) pyramid_level_kernel(Geom g, int l, FrameS
   const int sy0 = (int)(cy0 & 0xFFFF), sy1 = (int)(cy1 & 0xFFFF) + (int)(cy1 >> 25);
   const uint32_t cx0 = __ldg(xtab + tx0), cx1 = __ldg(xtab + tx1 - 1);
   const int sx0 = (int)(cx0 & 0xFFFF) & ~15, sx1 = (int)(cx1 & 0xFFFF) + (int)(cx1 >> 25);
-  if (threadIdx.x < TW) s_x[threadIdx.x] = tx0 + (int)threadIdx.x < dw ? __ldg(xtab + tx0 + threadIdx.x) : 0u;
+  // columns past the level edge reuse the last column's coefficients (computed, never stored)
+  if (threadIdx.x < TW) s_x[threadIdx.x] = __ldg(xtab + min(tx0 + (int)threadIdx.x, dw - 1));
   const int nrows = sy1 - sy0 + 1;
   if ((sp & 15) == 0 && (reinterpret_cast<uintptr_t>(s) & 15) == 0) {
     const int nch = (sx1 - sx0 + 16) >> 4;

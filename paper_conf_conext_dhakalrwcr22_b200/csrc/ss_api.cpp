@@ -138,6 +138,7 @@ struct ss_ctx {
   int8_t* pattern = nullptr;
   PyrTabs pyr_tabs{};
   unsigned long long* claim = nullptr;
+  uint16_t* rowidx = nullptr;  // WINDOW matcher: first keypoint per (frame, level, row)
   unsigned long long* partial = nullptr;
   // level 0 (FAST + distribution) runs on `aux`, concurrently with the pyramid and levels >= 1
   cudaStream_t aux = nullptr;
@@ -172,7 +173,7 @@ void free_ctx(ss_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->device);
   void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
-                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial};
+                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->rowidx};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
@@ -328,6 +329,10 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   }
   g.slots_per_frame = slot_off;
   g.kp_capacity = q.kp_capacity;
+  if (g.kp_capacity > 65535) {  // keypoint indices are 16-bit in the matcher's row index
+    free_ctx(c);
+    return fail(SS_EUNSUPPORTED, "kp_capacity above 65535");
+  }
   g.max_rw = max_rw;
   g.max_rh = max_rh;
   // coefficient tables for levels >= 1
@@ -379,6 +384,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->ovf_counter, sizeof(int32_t) * 2);
   ALLOC(c->pattern, 1024);
   ALLOC(c->claim, sizeof(unsigned long long) * F * g.kp_capacity);
+  ALLOC(c->rowidx, sizeof(uint16_t) * F * match_rows_per_frame(g));
   if (max_map > 0) ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
 #undef ALLOC
   if (e == cudaSuccess) e = cudaMemcpy(c->cells, c->cells_h.data(), sizeof(CellInfo) * c->cells_h.size(), cudaMemcpyHostToDevice);
@@ -469,8 +475,9 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
     if (n_queries > 0 && (!d_queries || !d_map_desc)) return fail(SS_EINVAL, "NULL queries");
     if (n_queries == 0) return SS_OK;
     prof_mark(c, s);
+    SS_CUDA_TRY(launch_match_prepare(c->g, n_frames, d_kps, d_counts, c->rowidx, c->claim, cfg->dedup, s));
     SS_CUDA_TRY(launch_match_window(c->g, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_queries, d_queries,
-                                    d_map_desc, *cfg, c->claim, d_out, s));
+                                    d_map_desc, *cfg, c->claim, d_out, c->rowidx, s));
     prof_mark(c, s);
     if (cfg->dedup) {
       SS_CUDA_TRY(launch_match_resolve(c->g, n_queries, d_queries, c->claim, d_out, s));

@@ -101,10 +101,15 @@ cudaError_t launch_describe(const Geom& g, int n_frames, FrameSrc src, const uin
                             int32_t* counts, cudaStream_t s);
 // The rotated-BRIEF pattern (1024 ints: 256 pairs x 2 points x (x, y)), host copy.
 const int* brief_pattern_host();
+// Row index of the keypoints (first keypoint per (frame, level, row)) + dedup claim reset.
+int match_rows_per_frame(const Geom& g);
+cudaError_t launch_match_prepare(const Geom& g, int n_frames, const ss_keypoint* kps, const int32_t* counts,
+                                 uint16_t* rowidx, unsigned long long* claim, int dedup, cudaStream_t s);
 cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* kps, const uint8_t* desc,
                                 const int32_t* counts, const uint8_t* taken, int n_queries,
                                 const ss_mp_query* q, const uint8_t* qdesc, ss_match_cfg cfg,
-                                unsigned long long* claim, ss_match* out, cudaStream_t s);
+                                unsigned long long* claim, ss_match* out, const uint16_t* rowidx,
+                                cudaStream_t s);
 cudaError_t launch_match_resolve(const Geom& g, int n_queries, const ss_mp_query* q,
                                  const unsigned long long* claim, ss_match* out, cudaStream_t s);
 int brute_splits(const Geom& g, int n_frames, int n_map, int max_splits);
