@@ -60,6 +60,8 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
                                                                    ss_keypoint* __restrict__ kps,
                                                                    uint8_t* __restrict__ desc,
                                                                    int32_t* __restrict__ counts) {
+  pdl_wait();
+  pdl_trigger();
   extern __shared__ __align__(16) uint8_t sm[];  // DESC_WARPS * PER_WARP
   __shared__ int8_t pat[1024];
   __shared__ int off[kMaxLevels + 1];
@@ -228,8 +230,9 @@ cudaError_t launch_describe(const Geom& g, int n_frames, FrameSrc src, const uin
     attr_set = true;
   }
   dim3 grid((g.kp_capacity + DESC_WARPS - 1) / DESC_WARPS, n_frames);
-  describe_kernel<<<grid, DESC_WARPS * 32, smem, s>>>(g, src, selected, sel_counts, pattern, kps, desc, counts);
-  return cudaGetLastError();
+  cudaError_t e = launch_pdl(describe_kernel, grid, dim3(DESC_WARPS * 32), smem, s, g, src, selected, sel_counts,
+                             pattern, kps, desc, counts);
+  return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 }  // namespace ss

@@ -556,6 +556,8 @@ __global__ void __launch_bounds__(DT, 1)
                       const int32_t* __restrict__ cell_counts, uint32_t* __restrict__ selected,
                       int32_t* __restrict__ sel_counts, uint8_t* ovf, int64_t ovf_frame_bytes,
                       const int64_t* __restrict__ ovf_level_off, int32_t* ovf_counter, int level0) {
+  pdl_wait();
+  pdl_trigger();
   extern __shared__ __align__(16) uint8_t sm[];
   __shared__ Shared S_;
   const int l = level0 + blockIdx.x, f = blockIdx.y, tid = threadIdx.x;
@@ -656,9 +658,9 @@ cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_lev
     attr_set = true;
   }
   dim3 grid(n_levels, n_frames);
-  distribute_kernel<<<grid, DT, kSmemTotal, s>>>(g, cells, slots, cell_counts, selected, sel_counts, ovf,
-                                                 ovf_frame_bytes, ovf_level_off, ovf_counter, level0);
-  return cudaGetLastError();
+  cudaError_t e = launch_pdl(distribute_kernel, grid, dim3(DT), kSmemTotal, s, g, cells, slots, cell_counts, selected,
+                             sel_counts, ovf, ovf_frame_bytes, ovf_level_off, ovf_counter, level0);
+  return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 }  // namespace ss

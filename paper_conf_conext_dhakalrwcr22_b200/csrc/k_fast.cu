@@ -99,6 +99,8 @@ __global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(Geom g, Frame
                                                                 uint32_t* __restrict__ slots,
                                                                 int32_t* __restrict__ cell_counts, int rp, int mbw,
                                                                 int region_bytes) {
+  pdl_wait();
+  pdl_trigger();
   extern __shared__ __align__(16) uint8_t smem[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const BandInfo bd = bands[blockIdx.x];
@@ -265,8 +267,9 @@ cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const B
     attr_set = true;
   }
   dim3 grid(n_bands, n_frames);
-  fast_bands_kernel<<<grid, FB_THREADS, smem, s>>>(g, src, bands, cells, slots, cell_counts, rp, mbw, rb);
-  return cudaGetLastError();
+  cudaError_t e = launch_pdl(fast_bands_kernel, grid, dim3(FB_THREADS), smem, s, g, src, bands, cells, slots,
+                             cell_counts, rp, mbw, rb);
+  return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 }  // namespace ss

@@ -36,6 +36,8 @@ __global__ void __launch_bounds__(256) match_prepare(Geom g, int F, const ss_key
                                                      const int32_t* __restrict__ counts, uint16_t* __restrict__ rowidx,
                                                      int rows_per_frame, unsigned long long* __restrict__ claim,
                                                      int dedup) {
+  pdl_wait();
+  pdl_trigger();
   const int cap = g.kp_capacity, L = g.L;
   const int gt = blockIdx.x * blockDim.x + threadIdx.x;
   if (gt >= F * cap) return;
@@ -75,6 +77,8 @@ __global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const 
                                                            unsigned long long* __restrict__ claim,
                                                            ss_match* __restrict__ out,
                                                            const uint16_t* __restrict__ rowidx, int rows_per_frame) {
+  pdl_wait();
+  pdl_trigger();
   const int gt = blockIdx.x * blockDim.x + threadIdx.x;
   const int qi = gt / WG, sub = gt % WG;
   const unsigned gmask = 0xFFu << ((threadIdx.x & 31) & ~(WG - 1));
@@ -143,6 +147,8 @@ __global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const 
 __global__ void __launch_bounds__(256) match_window_resolve(int nq, const ss_mp_query* __restrict__ q, int cap,
                                                             const unsigned long long* __restrict__ claim,
                                                             ss_match* __restrict__ out) {
+  pdl_wait();
+  pdl_trigger();
   const int qi = blockIdx.x * blockDim.x + threadIdx.x;
   if (qi >= nq) return;
   const ss_match m = out[qi];
@@ -158,6 +164,8 @@ __global__ void __launch_bounds__(BQ) match_brute_partial(Geom g, int F, const u
                                                           const int32_t* __restrict__ counts, int n_map,
                                                           const uint8_t* __restrict__ map_desc, int splits,
                                                           unsigned long long* __restrict__ partial) {
+  pdl_wait();
+  pdl_trigger();
   __shared__ uint4 tile[BTILE * 2];
   const int cap = g.kp_capacity, L = g.L;
   const int gq = blockIdx.x * BQ + threadIdx.x;  // global keypoint slot f*cap + k
@@ -204,6 +212,8 @@ __global__ void __launch_bounds__(BQ) match_brute_partial(Geom g, int F, const u
 __global__ void __launch_bounds__(256) match_brute_merge(Geom g, int F, const int32_t* __restrict__ counts,
                                                          int splits, const unsigned long long* __restrict__ partial,
                                                          ss_match_cfg cfg, ss_match* __restrict__ out) {
+  pdl_wait();
+  pdl_trigger();
   const int gq = blockIdx.x * blockDim.x + threadIdx.x;
   const int cap = g.kp_capacity, L = g.L;
   if (gq >= F * cap) return;
@@ -240,9 +250,9 @@ cudaError_t launch_match_prepare(const Geom& g, int n_frames, const ss_keypoint*
                                  uint16_t* rowidx, unsigned long long* claim, int dedup, cudaStream_t s) {
   const int n = n_frames * g.kp_capacity;
   if (n <= 0) return cudaSuccess;
-  match_prepare<<<(n + 255) / 256, 256, 0, s>>>(g, n_frames, kps, counts, rowidx, match_rows_per_frame(g), claim,
-                                                dedup);
-  return cudaGetLastError();
+  cudaError_t e = launch_pdl(match_prepare, dim3((n + 255) / 256), dim3(256), 0, s, g, n_frames, kps, counts, rowidx,
+                             match_rows_per_frame(g), claim, dedup);
+  return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* kps, const uint8_t* desc,
@@ -251,16 +261,18 @@ cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* 
                                 const uint16_t* rowidx, cudaStream_t s) {
   if (n_queries <= 0) return cudaSuccess;
   const int64_t threads = (int64_t)n_queries * WG;
-  match_window_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, s>>>(
-      g, n_frames, kps, desc, counts, taken, n_queries, q, qdesc, cfg, claim, out, rowidx, match_rows_per_frame(g));
-  return cudaGetLastError();
+  cudaError_t e = launch_pdl(match_window_kernel, dim3((unsigned)((threads + 255) / 256)), dim3(256), 0, s, g, n_frames,
+                             kps, desc, counts, taken, n_queries, q, qdesc, cfg, claim, out, rowidx,
+                             match_rows_per_frame(g));
+  return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 cudaError_t launch_match_resolve(const Geom& g, int n_queries, const ss_mp_query* q, const unsigned long long* claim,
                                  ss_match* out, cudaStream_t s) {
   if (n_queries <= 0) return cudaSuccess;
-  match_window_resolve<<<(n_queries + 255) / 256, 256, 0, s>>>(n_queries, q, g.kp_capacity, claim, out);
-  return cudaGetLastError();
+  cudaError_t e = launch_pdl(match_window_resolve, dim3((n_queries + 255) / 256), dim3(256), 0, s, n_queries, q,
+                             g.kp_capacity, (const unsigned long long*)claim, out);
+  return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 int brute_splits(const Geom& g, int n_frames, int n_map, int max_splits) {

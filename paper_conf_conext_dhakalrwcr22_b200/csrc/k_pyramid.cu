@@ -20,6 +20,8 @@ constexpr int SRC_ROWS = 48, SRC_PITCH = 208;  // >= TH*scale+2 rows, >= TW*scal
 
 __global__ void __launch_bounds__(PT) pyramid_level_kernel(Geom g, int l, FrameSrc src, const uint32_t* __restrict__ xtab,
                                                            const uint32_t* __restrict__ ytab) {
+  pdl_wait();
+  pdl_trigger();
   __shared__ __align__(16) uint8_t s_src[SRC_ROWS * SRC_PITCH];
   __shared__ uint32_t s_x[TW];
   const int f = blockIdx.z;
@@ -108,8 +110,8 @@ cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const uint
                            cudaStream_t s) {
   for (int l = 1; l < g.L; l++) {
     dim3 grid((g.w[l] + TW - 1) / TW, (g.h[l] + TH - 1) / TH, n_frames);
-    pyramid_level_kernel<<<grid, PT, 0, s>>>(g, l, src, xytab + tabs.xoff[l], xytab + tabs.yoff[l]);
-    cudaError_t e = cudaGetLastError();
+    cudaError_t e = launch_pdl(pyramid_level_kernel, grid, dim3(PT), 0, s, g, l, src, xytab + tabs.xoff[l], xytab + tabs.yoff[l]);
+    if (e == cudaSuccess) e = cudaGetLastError();
     if (e != cudaSuccess) return e;
   }
   return cudaSuccess;

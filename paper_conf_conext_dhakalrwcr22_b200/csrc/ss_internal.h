@@ -80,6 +80,31 @@ __host__ __device__ inline int key_lx(uint32_t k) { return (int)((k >> 8) & 0x7F
 __host__ __device__ inline int key_ly(uint32_t k) { return (int)(k >> 19); }
 __host__ __device__ inline int key_m(uint32_t k) { return (int)(k & 0xFF); }
 
+// ---- Programmatic Dependent Launch (sm_90+): every kernel of the chain is launched with
+// programmatic stream serialisation, lets its dependents launch as soon as all its CTAs are
+// resident (pdl_trigger) and waits for its predecessor's completion + memory (pdl_wait)
+// before touching its inputs.  This hides the launch latency between dependent kernels. ----
+#ifdef __CUDACC__
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                              Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
+#endif
+
 // ---- launchers (one per kernel; each returns cudaGetLastError()) ----
 struct PyrTabs {
   int64_t xoff[kMaxLevels], yoff[kMaxLevels];  // offsets of level l's x / y coefficient tables
