@@ -23,7 +23,9 @@ constexpr int PP = 64;  // raw patch pitch: a 16-B aligned 64-B window covers th
 constexpr int BR = 37;  // blurred patch: radius 18
 constexpr int VP = 46;  // pitch (u16) of the vertical pass V[37][43]: 23 words (odd) per row
 constexpr int BP = 44;  // pitch of the blurred patch B[37][37]: 11 words (odd) per row
-constexpr int PER_WARP = ((PR * PP + BR * VP * 2 + BR * BP) + 127) & ~127;
+// the blurred patch B reuses the raw patch's space (P is dead after the vertical pass)
+constexpr int PER_WARP = ((PR * PP + BR * VP * 2) + 127) & ~127;
+static_assert(BR * BP <= PR * PP, "B aliases P");
 
 __constant__ int c_umax[16] = {15, 15, 15, 15, 14, 14, 14, 13, 13, 12, 11, 10, 9, 8, 6, 3};
 
@@ -97,7 +99,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
   const int w = g.w[l], h = g.h[l];
   uint8_t* Pw = sm + warp * PER_WARP;
   uint16_t* V = reinterpret_cast<uint16_t*>(Pw + PR * PP);
-  uint8_t* B = reinterpret_cast<uint8_t*>(V + BR * VP);
+  uint8_t* B = Pw;  // written only after the vertical pass has consumed P (syncwarp between)
   const uint8_t* p0 = img + (int64_t)(ly - 21) * ip + (lx - 21);
   const int sh = (int)(reinterpret_cast<uintptr_t>(p0) & 15);
   const uint8_t* P;  // P[r * PP + c] = raw patch pixel (ly - 21 + r, lx - 21 + c)

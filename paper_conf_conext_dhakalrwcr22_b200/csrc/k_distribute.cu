@@ -60,7 +60,9 @@ __device__ __forceinline__ void root_geom(const Geom& g, int l, int ri, int& ulx
   urx = __float2int_rz(__fmul_rn(g.hX[l], (float)(ri + 1)));
 }
 
-__device__ __forceinline__ uint32_t make_key(const Geom& g, int l, uint32_t packed) {
+// key = root << 26 | quadrant path; `rounds` < 13 leaves the deeper path bits zero (the dense
+// path needs only depths <= R + 1)
+__device__ __forceinline__ uint32_t make_key(const Geom& g, int l, uint32_t packed, int rounds = kQuadRounds) {
   const int kx = key_lx(packed) - kMinBorder, ky = key_ly(packed) - kMinBorder;
   int ri = __float2int_rz(__fdiv_rn((float)kx, g.hX[l]));
   ri = min(ri, g.nini[l] - 1);
@@ -68,15 +70,14 @@ __device__ __forceinline__ uint32_t make_key(const Geom& g, int l, uint32_t pack
   root_geom(g, l, ri, ulx, urx);
   int uly = 0, bly = g.qh[l];
   uint32_t path = 0;
-#pragma unroll
-  for (int r = 0; r < kQuadRounds; r++) {
+  for (int r = 0; r < rounds; r++) {
     const int hx = (urx - ulx + 1) >> 1, hy = (bly - uly + 1) >> 1;  // ceil(w/2), w >= 0
     const int right = kx >= ulx + hx, down = ky >= uly + hy;
     path = (path << 2) | (uint32_t)(down * 2 + right);
     if (right) ulx += hx; else urx = ulx + hx;
     if (down) uly += hy; else bly = uly + hy;
   }
-  return ((uint32_t)ri << 26) | path;
+  return ((uint32_t)ri << 26) | (path << (2 * (kQuadRounds - rounds)));
 }
 
 // Upper-left corner of the depth-d node holding `key`.
@@ -412,13 +413,21 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
       S_.G[tid] = 0;  // bins with >= 2 keys per depth
     }
   }
-  for (int i = tid; i < n; i += DT) key[i] = make_key(g, l, cand[i]);
-  __syncthreads();
+  // keys to depth R + 1 (the partial round at D <= R - 1 looks at D + 1 <= R); only the deepest
+  // histogram takes atomics (few keys share a bin), shallower depths are sums of 4 children
   for (int i = tid; i < n; i += DT) {
-    const uint32_t k = key[i];
-    for (int r = 0; r <= R; r++) atomicAdd(&cnt[off[r] + (int)(k >> (26 - 2 * r))], 1u);
+    const uint32_t k = make_key(g, l, cand[i], R + 1);
+    key[i] = k;
+    atomicAdd(&cnt[off[R] + (int)(k >> (26 - 2 * R))], 1u);
   }
   __syncthreads();
+  for (int r = R - 1; r >= 0; r--) {
+    for (int b = tid; b < sz[r]; b += DT) {
+      const uint32_t* ch = cnt + off[r + 1] + 4 * b;
+      cnt[off[r] + b] = ch[0] + ch[1] + ch[2] + ch[3];
+    }
+    __syncthreads();
+  }
   for (int r = 0; r <= R; r++) {
     int nz = 0, mu = 0;
     for (int b = tid; b < sz[r]; b += DT) {
