@@ -154,13 +154,14 @@ ss_status ss_match_projection(ss_ctx* ctx, int32_t n_frames, const ss_keypoint* 
  * caller's events (cudaEvent_t handles created with timing enabled; host array copied) on
  * its stream: the next unused event before its first operation, then one after every
  * kernel it launches, continuing across calls until the next ss_profile_events call
- * (n_events = 0 disables; events beyond n_events are not recorded).  Record order of one
- * extract (level 0 runs on an internal stream forked from `stream` and joined before
- * describe): e0 start, e1 level-0 branch start, e2 after level-0 FAST, e3 after level-0
- * distribution, e4 after the pyramid, e5 after FAST of levels >= 1, e6 after their
- * distribution, e7 after describe.  WINDOW match: start, match_window[, match_resolve if
- * dedup]; BRUTE: start, brute_partial, brute_merge.  Works under CUDA-graph stream capture
- * (the records become graph event nodes).
+ * (n_events = 0 disables; events beyond n_events are not recorded).  One extract records a
+ * start event, then a (before, after) pair around every kernel launch on the stream it runs
+ * on, in this order: fast(level 0), distribute(level 0), then for l = 1..L-1: pyramid(l),
+ * fast(l), distribute(l); then describe: 1 + 6 L events for L levels.  Level l's FAST and
+ * distribution run on internal side streams
+ * forked from `stream`.  WINDOW match: a pair per kernel (match_prepare, match_window[,
+ * match_resolve if dedup]), preceded by nothing; BRUTE: pairs for brute_partial, brute_merge.
+ * Works under CUDA-graph stream capture (the records become graph event nodes).
  * *next_index (may be NULL) receives the index of the next event to be recorded. */
 ss_status ss_profile_events(ss_ctx* ctx, void* const* events, int32_t n_events);
 ss_status ss_profile_next(ss_ctx* ctx, int32_t* next_index);

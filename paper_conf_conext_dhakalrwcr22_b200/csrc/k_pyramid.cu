@@ -106,6 +106,14 @@ bool pyramid_tiles_fit(int dst_w, int dst_h, const uint32_t* xt, const uint32_t*
   return true;
 }
 
+cudaError_t launch_pyramid_level(const Geom& g, int l, int n_frames, FrameSrc src, const uint32_t* xytab, PyrTabs tabs,
+                                 cudaStream_t s) {
+  dim3 grid((g.w[l] + TW - 1) / TW, (g.h[l] + TH - 1) / TH, n_frames);
+  cudaError_t e = launch_pdl(pyramid_level_kernel, grid, dim3(PT), 0, s, g, l, src, xytab + tabs.xoff[l],
+                             xytab + tabs.yoff[l]);
+  return e != cudaSuccess ? e : cudaGetLastError();
+}
+
 cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const uint32_t* xytab, PyrTabs tabs,
                            cudaStream_t s) {
   for (int l = 1; l < g.L; l++) {

@@ -140,9 +140,11 @@ struct ss_ctx {
   unsigned long long* claim = nullptr;
   uint16_t* rowidx = nullptr;  // WINDOW matcher: first keypoint per (frame, level, row)
   unsigned long long* partial = nullptr;
-  // level 0 (FAST + distribution) runs on `aux`, concurrently with the pyramid and levels >= 1
-  cudaStream_t aux = nullptr;
-  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  // per-extract DAG: level 0's FAST + distribution on side stream 0 right away; level l >= 1's
+  // on side stream 1 + (l % kSideLevel) as soon as the pyramid (caller's stream) has level l
+  static constexpr int kSide = 4, kSideLevel = 3;
+  cudaStream_t side[kSide] = {};
+  cudaEvent_t ev_fork = nullptr, ev_level[kMaxLevels] = {}, ev_join[kSide] = {};
   // profiling hook
   std::vector<cudaEvent_t> prof;
   size_t prof_next = 0;
@@ -177,8 +179,12 @@ void free_ctx(ss_ctx* c) {
   for (void* q : ptrs)
     if (q) cudaFree(q);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
-  if (c->ev_join) cudaEventDestroy(c->ev_join);
-  if (c->aux) cudaStreamDestroy(c->aux);
+  for (cudaEvent_t e : c->ev_level)
+    if (e) cudaEventDestroy(e);
+  for (cudaEvent_t e : c->ev_join)
+    if (e) cudaEventDestroy(e);
+  for (cudaStream_t q : c->side)
+    if (q) cudaStreamDestroy(q);
   delete c;
 }
 
@@ -319,7 +325,13 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   }
   g.total_bands = (int)c->bands_h.size();
   g.level0_bands = 0;
-  for (const BandInfo& b : c->bands_h) g.level0_bands += (b.level == 0);
+  for (int l = 0; l < kMaxLevels; l++) g.band_first[l] = g.band_count[l] = 0;
+  for (size_t i = 0; i < c->bands_h.size(); i++) {
+    const int l = c->bands_h[i].level;
+    if (g.band_count[l] == 0) g.band_first[l] = (int)i;
+    g.band_count[l]++;
+  }
+  g.level0_bands = g.band_count[0];
   {
     int rp, mbw, rb, mb, nb;
     if (fast_smem_bytes(g, &rp, &mbw, &rb, &mb, &nb) > 227 * 1024) {
@@ -393,9 +405,13 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (e == cudaSuccess) e = cudaMemcpy(c->ovf_level_off, ovf_off.data(), sizeof(int64_t) * L, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->pattern, pat.data(), 1024, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemset(c->ovf_counter, 0, sizeof(int32_t) * 2);
-  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking);
+  for (int i = 0; i < ss_ctx::kSide && e == cudaSuccess; i++) {
+    e = cudaStreamCreateWithFlags(&c->side[i], cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_join[i], cudaEventDisableTiming);
+  }
+  for (int l = 0; l < kMaxLevels && e == cudaSuccess; l++)
+    e = cudaEventCreateWithFlags(&c->ev_level[l], cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);
-  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaMemset(c->sel_counts, 0, sizeof(int32_t) * F * L);
   if (e != cudaSuccess) {
     std::string m = std::string("ss_create: ") + cudaGetErrorString(e);
@@ -426,31 +442,47 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   SS_CUDA_TRY(check_stream(s));
   const Geom& g = c->g;
   FrameSrc src{d_frames, frame_stride, pitch, c->pyr};
-  // fork: level 0 needs no pyramid, so its FAST + distribution overlap the pyramid and the
-  // levels above it; join before describe (which needs every level's counts)
-  prof_mark(c, s);                                                             // e0
+  // DAG: level l's FAST + distribution run on a side stream as soon as level l exists (level
+  // 0 at once, levels >= 1 after their pyramid launch on the caller's stream); describe joins.
+  // Profiling events: start, then a (before, after) pair around every launch in this order:
+  // fast l0, distribute l0, then per level l >= 1: pyramid l, fast l, distribute l; describe.
+  prof_mark(c, s);
   SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 2, s));
   SS_CUDA_TRY(cudaEventRecord(c->ev_fork, s));
-  SS_CUDA_TRY(cudaStreamWaitEvent(c->aux, c->ev_fork, 0));
-  prof_mark(c, c->aux);                                                        // e1
-  SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands, g.level0_bands, c->cells, c->slots, c->cell_counts,
-                                c->aux));
-  prof_mark(c, c->aux);                                                        // e2
-  SS_CUDA_TRY(launch_distribute(g, n_frames, 0, 1, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts,
-                                c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, c->aux));
-  prof_mark(c, c->aux);                                                        // e3
-  SS_CUDA_TRY(cudaEventRecord(c->ev_join, c->aux));
-  SS_CUDA_TRY(launch_pyramid(g, n_frames, src, c->xytab, c->pyr_tabs, s));
-  prof_mark(c, s);                                                             // e4
-  SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands + g.level0_bands, g.total_bands - g.level0_bands,
-                                c->cells, c->slots, c->cell_counts, s));
-  prof_mark(c, s);                                                             // e5
-  SS_CUDA_TRY(launch_distribute(g, n_frames, 1, g.L - 1, c->cells, c->slots, c->cell_counts, c->selected,
-                                c->sel_counts, c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, s));
-  prof_mark(c, s);                                                             // e6
-  SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join, 0));
+  bool used[ss_ctx::kSide] = {};
+  auto level_branch = [&](int l, cudaStream_t q) -> cudaError_t {
+    prof_mark(c, q);
+    cudaError_t e = launch_fast_bands(g, n_frames, src, c->bands + g.band_first[l], g.band_count[l], c->cells,
+                                      c->slots, c->cell_counts, q);
+    if (e != cudaSuccess) return e;
+    prof_mark(c, q);
+    prof_mark(c, q);
+    e = launch_distribute(g, n_frames, l, 1, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
+                          c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, q);
+    prof_mark(c, q);
+    return e;
+  };
+  SS_CUDA_TRY(cudaStreamWaitEvent(c->side[0], c->ev_fork, 0));
+  used[0] = true;
+  SS_CUDA_TRY(level_branch(0, c->side[0]));
+  for (int l = 1; l < g.L; l++) {
+    prof_mark(c, s);
+    SS_CUDA_TRY(launch_pyramid_level(g, l, n_frames, src, c->xytab, c->pyr_tabs, s));
+    prof_mark(c, s);
+    SS_CUDA_TRY(cudaEventRecord(c->ev_level[l], s));
+    const int si = 1 + (l % ss_ctx::kSideLevel);
+    SS_CUDA_TRY(cudaStreamWaitEvent(c->side[si], c->ev_level[l], 0));
+    used[si] = true;
+    SS_CUDA_TRY(level_branch(l, c->side[si]));
+  }
+  for (int i = 0; i < ss_ctx::kSide; i++) {
+    if (!used[i]) continue;
+    SS_CUDA_TRY(cudaEventRecord(c->ev_join[i], c->side[i]));
+    SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[i], 0));
+  }
+  prof_mark(c, s);
   SS_CUDA_TRY(launch_describe(g, n_frames, src, c->selected, c->sel_counts, c->pattern, d_kps, d_desc, d_counts, s));
-  prof_mark(c, s);                                                             // e7
+  prof_mark(c, s);
   c->last_frames = d_frames;
   c->last_stride = frame_stride;
   c->last_pitch = pitch;
@@ -476,10 +508,13 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
     if (n_queries == 0) return SS_OK;
     prof_mark(c, s);
     SS_CUDA_TRY(launch_match_prepare(c->g, n_frames, d_kps, d_counts, c->rowidx, c->claim, cfg->dedup, s));
+    prof_mark(c, s);
+    prof_mark(c, s);
     SS_CUDA_TRY(launch_match_window(c->g, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_queries, d_queries,
                                     d_map_desc, *cfg, c->claim, d_out, c->rowidx, s));
     prof_mark(c, s);
     if (cfg->dedup) {
+      prof_mark(c, s);
       SS_CUDA_TRY(launch_match_resolve(c->g, n_queries, d_queries, c->claim, d_out, s));
       prof_mark(c, s);
     }
@@ -493,6 +528,7 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
     const int splits = brute_splits(c->g, n_frames, n_map, c->max_splits);
     prof_mark(c, s);
     SS_CUDA_TRY(launch_brute_partial(c->g, n_frames, d_desc, d_counts, n_map, d_map_desc, splits, c->partial, s));
+    prof_mark(c, s);
     prof_mark(c, s);
     SS_CUDA_TRY(launch_brute_merge(c->g, n_frames, d_counts, splits, c->partial, *cfg, d_out, s));
     prof_mark(c, s);

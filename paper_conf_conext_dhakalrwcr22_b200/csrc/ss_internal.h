@@ -60,6 +60,7 @@ struct Geom {
   int32_t max_rw, max_rh;           // largest FAST input region (D + 3-px halo) of any cell
   int32_t total_bands;              // FAST work units (cell-row segments) over all levels, per frame
   int32_t level0_bands;             // ... of which on level 0 (they come first)
+  int32_t band_first[kMaxLevels], band_count[kMaxLevels];  // FAST work units of level l
   int32_t max_band_w, max_band_h;   // widest band (detect columns) / tallest band (detect rows)
   int32_t max_cell_w;               // widest cell detect window
 };
@@ -112,6 +113,8 @@ struct PyrTabs {
 // Levels 1..L-1 of all frames, one launch per level, 128x32 output tiles.
 cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const uint32_t* xytab, PyrTabs tabs,
                            cudaStream_t s);
+cudaError_t launch_pyramid_level(const Geom& g, int l, int n_frames, FrameSrc src, const uint32_t* xytab, PyrTabs tabs,
+                                 cudaStream_t s);
 // Whether every tile's source rectangle fits the kernel's shared-memory staging.
 bool pyramid_tiles_fit(int dst_w, int dst_h, const uint32_t* xt, const uint32_t* yt);
 cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands, int n_bands,

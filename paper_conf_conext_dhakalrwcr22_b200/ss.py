@@ -172,23 +172,26 @@ def ss_profile_next(ctx) -> int:
     return n.value
 
 
-EXTRACT_EVENTS = 8  # profiling events one ss_orb_extract records (include/ss.h)
-# (name, start events (latest wins), end event) of one extract, indices into its events
-EXTRACT_INTERVALS = [("fast_l0", (1,), 2), ("distribute_l0", (2,), 3), ("pyramid", (0,), 4),
-                     ("fast_l1plus", (4,), 5), ("distribute_l1plus", (5,), 6), ("describe", (3, 6), 7)]
+def extract_kernels(n_levels: int) -> list[str]:
+    """Kernel launches of one ss_orb_extract in profiling-event order (include/ss.h)."""
+    out = ["fast_l0", "distribute_l0"]
+    for l in range(1, n_levels):
+        out += [f"pyramid_l{l}", f"fast_l{l}", f"distribute_l{l}"]
+    return out + ["describe"]
+
+
+def extract_events(n_levels: int) -> int:
+    return 1 + 2 * len(extract_kernels(n_levels))
+
+
+def match_kernels(mode: int, dedup: bool = True) -> list[str]:
+    if mode == SS_MATCH_BRUTE:
+        return ["brute_partial", "brute_merge"]
+    return ["match_prepare", "match_window"] + (["match_resolve"] if dedup else [])
 
 
 def match_events(mode: int, dedup: bool = True) -> int:
-    return 3 if mode == SS_MATCH_BRUTE else (3 if dedup else 2)
-
-
-def match_intervals(mode: int, dedup: bool = True, base: int = 0):
-    if mode == SS_MATCH_BRUTE:
-        return [("brute_partial", (base,), base + 1), ("brute_merge", (base + 1,), base + 2)]
-    out = [("match_window", (base,), base + 1)]
-    if dedup:
-        out.append(("match_resolve", (base + 1,), base + 2))
-    return out
+    return 2 * len(match_kernels(mode, dedup))
 
 
 def ss_debug_level(ctx, frame, level):
