@@ -413,6 +413,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
       S_.G[tid] = 0;  // bins with >= 2 keys per depth
     }
   }
+  __syncthreads();  // bins zeroed before any increment
   // keys to depth R + 1 (the partial round at D <= R - 1 looks at D + 1 <= R); only the deepest
   // histogram takes atomics (few keys share a bin), shallower depths are sums of 4 children
   for (int i = tid; i < n; i += DT) {
