@@ -49,6 +49,17 @@ static_assert(kSmemTotal <= 220 * 1024, "distribution smem budget");
 static_assert((size_t)DCAP * 4 + kUnion >= (5464 + 4096 * 2 + 1024) * 4 + 1024 * (8 + 4 + 4 + 1) + 1024,
               "dense fast-path workspace must fit in the rank + union region");
 
+__device__ __forceinline__ uint64_t gtimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// phase timestamps of one (frame, level) CTA (debug hook ss_debug_phase_times), thread 0 only
+#define SS_PHASE(i)                                  \
+  do {                                               \
+    if (phase_ts && threadIdx.x == 0) phase_ts[i] = gtimer(); \
+  } while (0)
+
 struct Shared {
   BScan::TempStorage scan;
   int sh[8];
@@ -384,7 +395,7 @@ constexpr int DENSE_REC = 1024;       // multi-key bins at the partial depth (<=
 
 __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* cand, uint32_t* key, uint8_t* ws,
                            Shared& S_, uint32_t* __restrict__ selected, int32_t* __restrict__ sel_counts,
-                           int32_t* ovf_counter) {
+                           int32_t* ovf_counter, uint64_t* phase_ts) {
   const int tid = threadIdx.x;
   const int N = g.N[l];
   const int nini = g.nini[l];
@@ -414,6 +425,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
     }
   }
   __syncthreads();  // bins zeroed before any increment
+  SS_PHASE(3);
   // keys to depth R + 1 (the partial round at D <= R - 1 looks at D + 1 <= R); only the deepest
   // histogram takes atomics (few keys share a bin), shallower depths are sums of 4 children
   for (int i = tid; i < n; i += DT) {
@@ -422,6 +434,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
     atomicAdd(&cnt[off[R] + (int)(k >> (26 - 2 * R))], 1u);
   }
   __syncthreads();
+  SS_PHASE(4);
   for (int r = R - 1; r >= 0; r--) {
     for (int b = tid; b < sz[r]; b += DT) {
       const uint32_t* ch = cnt + off[r + 1] + 4 * b;
@@ -475,6 +488,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
   }
   __syncthreads();
   const int D = S_.sh[3];
+  SS_PHASE(5);
   if (D < 0) return false;
   const bool partial = S_.sh[4] != 0;
   const int szD = nini << (2 * D);
@@ -522,6 +536,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
     }
   }
   __syncthreads();
+  SS_PHASE(6);
   // best key of every final node: max score, ties -> lowest rank
   for (int i = tid; i < n; i += DT) {
     const uint32_t k = key[i];
@@ -531,6 +546,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
     else atomicMax(&best0[b], v);
   }
   __syncthreads();
+  SS_PHASE(7);
   uint32_t* kept = key;  // keys are no longer needed
   const uint32_t* cD = cnt + off[D];
   for (int b = tid; b < szD; b += DT) {
@@ -547,6 +563,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
   __syncthreads();
   const int nk = S_.sh[2];
   const int nk_w = min(nk, g.cap[l]);
+  SS_PHASE(8);
   uint32_t* sel_out = selected + (int64_t)f * g.kp_capacity + g.cap_off[l];
   for (int t = tid; t < nk; t += DT) {
     const uint32_t k = kept[t] >> 8;
@@ -558,6 +575,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
     sel_counts[f * g.L + l] = nk_w;
     if (nk > g.cap[l]) atomicAdd(ovf_counter + 1, 1);
   }
+  SS_PHASE(9);
   return true;
 }
 
@@ -565,12 +583,15 @@ __global__ void __launch_bounds__(DT, 1)
     distribute_kernel(Geom g, const CellInfo* __restrict__ cells, const uint32_t* __restrict__ slots,
                       const int32_t* __restrict__ cell_counts, uint32_t* __restrict__ selected,
                       int32_t* __restrict__ sel_counts, uint8_t* ovf, int64_t ovf_frame_bytes,
-                      const int64_t* __restrict__ ovf_level_off, int32_t* ovf_counter, int level0) {
+                      const int64_t* __restrict__ ovf_level_off, int32_t* ovf_counter, int level0,
+                      uint64_t* phase_base) {
   pdl_wait();
   pdl_trigger();
   extern __shared__ __align__(16) uint8_t sm[];
   __shared__ Shared S_;
   const int l = level0 + blockIdx.x, f = blockIdx.y, tid = threadIdx.x;
+  uint64_t* phase_ts = phase_base ? phase_base + ((int64_t)f * g.L + l) * 16 : nullptr;
+  SS_PHASE(0);
   const int ncells = g.ncells[l];
   const int c0 = g.cell_first[l];
   int32_t* cell_off = reinterpret_cast<int32_t*>(sm);
@@ -609,6 +630,7 @@ __global__ void __launch_bounds__(DT, 1)
     __syncthreads();
   }
   const int n = S_.sh[0];
+  SS_PHASE(1);
   if (n == 0) {
     if (tid == 0) sel_counts[f * g.L + l] = 0;
     return;
@@ -628,8 +650,9 @@ __global__ void __launch_bounds__(DT, 1)
       }
       __syncthreads();
     }
+    SS_PHASE(2);
     if (dense_body(g, l, f, n, cand, key, reinterpret_cast<uint8_t*>(key + DCAP), S_, selected, sel_counts,
-                   ovf_counter))
+                   ovf_counter, phase_ts))
       return;
     __syncthreads();
     if (tid < 16) S_.H[tid] = 0;
@@ -659,7 +682,7 @@ int64_t distribute_ovf_bytes(int64_t slots) {
 cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_levels, const CellInfo* cells,
                               const uint32_t* slots, const int32_t* cell_counts, uint32_t* selected, int32_t* sel_counts,
                               uint8_t* ovf, int64_t ovf_frame_bytes, const int64_t* ovf_level_off, int32_t* ovf_counter,
-                              cudaStream_t s) {
+                              uint64_t* phase_ts, cudaStream_t s) {
   if (n_levels <= 0) return cudaSuccess;
   static bool attr_set = false;
   if (!attr_set) {
@@ -669,7 +692,7 @@ cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_lev
   }
   dim3 grid(n_levels, n_frames);
   cudaError_t e = launch_pdl(distribute_kernel, grid, dim3(DT), kSmemTotal, s, g, cells, slots, cell_counts, selected,
-                             sel_counts, ovf, ovf_frame_bytes, ovf_level_off, ovf_counter, level0);
+                             sel_counts, ovf, ovf_frame_bytes, ovf_level_off, ovf_counter, level0, phase_ts);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 

@@ -139,6 +139,7 @@ struct ss_ctx {
   PyrTabs pyr_tabs{};
   unsigned long long* claim = nullptr;
   uint16_t* rowidx = nullptr;  // WINDOW matcher: first keypoint per (frame, level, row)
+  uint64_t* phase_ts = nullptr;  // distribution phase timestamps [max_frames][L][16] (debug hook)
   unsigned long long* partial = nullptr;
   // per-extract DAG: level 0's FAST + distribution on side stream 0 right away; level l >= 1's
   // on side stream 1 + (l % kSideLevel) as soon as the pyramid (caller's stream) has level l
@@ -175,7 +176,7 @@ void free_ctx(ss_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->device);
   void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
-                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->rowidx};
+                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->rowidx, c->phase_ts};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
@@ -397,6 +398,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->pattern, 1024);
   ALLOC(c->claim, sizeof(unsigned long long) * F * g.kp_capacity);
   ALLOC(c->rowidx, sizeof(uint16_t) * F * match_rows_per_frame(g));
+  ALLOC(c->phase_ts, sizeof(uint64_t) * F * L * 16);
   if (max_map > 0) ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
 #undef ALLOC
   if (e == cudaSuccess) e = cudaMemcpy(c->cells, c->cells_h.data(), sizeof(CellInfo) * c->cells_h.size(), cudaMemcpyHostToDevice);
@@ -458,7 +460,7 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
     prof_mark(c, q);
     prof_mark(c, q);
     e = launch_distribute(g, n_frames, l, 1, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
-                          c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, q);
+                          c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, c->phase_ts, q);
     prof_mark(c, q);
     return e;
   };
@@ -590,6 +592,16 @@ ss_status ss_debug_candidates(ss_ctx* c, int32_t frame, int32_t level, int32_t* 
   }
   *n = k;
   if (k > cap) return fail(SS_ECAPACITY, "more candidates than cap");
+  return SS_OK;
+}
+
+ss_status ss_debug_phase_times(ss_ctx* c, int32_t frame, int32_t level, int64_t* h_ns, int32_t n) {
+  if (!c || !h_ns || n < 0 || n > 16) return fail(SS_EINVAL, "bad argument");
+  if (frame < 0 || frame >= c->max_frames || level < 0 || level >= c->g.L) return fail(SS_EINVAL, "bad frame/level");
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  SS_CUDA_TRY(cudaDeviceSynchronize());
+  SS_CUDA_TRY(cudaMemcpy(h_ns, c->phase_ts + ((int64_t)frame * c->g.L + level) * 16, sizeof(int64_t) * n,
+                         cudaMemcpyDeviceToHost));
   return SS_OK;
 }
 

@@ -123,7 +123,8 @@ size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int*
 cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_levels, const CellInfo* cells,
                               const uint32_t* slots, const int32_t* cell_counts, uint32_t* selected,
                               int32_t* sel_counts, uint8_t* ovf, int64_t ovf_frame_bytes,
-                              const int64_t* ovf_level_off, int32_t* ovf_counter, cudaStream_t s);
+                              const int64_t* ovf_level_off, int32_t* ovf_counter, uint64_t* phase_ts,
+                              cudaStream_t s);
 cudaError_t launch_describe(const Geom& g, int n_frames, FrameSrc src, const uint32_t* selected,
                             const int32_t* sel_counts, const int8_t* pattern, ss_keypoint* kps, uint8_t* desc,
                             int32_t* counts, cudaStream_t s);

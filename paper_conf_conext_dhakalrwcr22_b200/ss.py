@@ -85,10 +85,11 @@ def lib():
         L.ss_debug_candidates.argtypes = [P, i32, i32, P, P, P, i32, C.POINTER(i32)]
         L.ss_debug_overflow_count.argtypes = [P, C.POINTER(i32)]
         L.ss_profile_events.argtypes = [P, C.POINTER(P), i32]
+        L.ss_debug_phase_times.argtypes = [P, i32, i32, P, i32]
         L.ss_profile_next.argtypes = [P, C.POINTER(i32)]
         for fn in ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_orb_extract", "ss_match_projection",
                    "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
-                   "ss_profile_next"):
+                   "ss_profile_next", "ss_debug_phase_times"):
             getattr(L, fn).restype = C.c_int
         _lib = L
     return _lib
@@ -96,7 +97,7 @@ def lib():
 
 EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "ss_orb_extract",
             "ss_match_projection", "ss_profile_events", "ss_profile_next", "ss_debug_level",
-            "ss_debug_candidates", "ss_debug_overflow_count")
+            "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times")
 
 
 def _check(status: int, ctx=None):
@@ -206,6 +207,12 @@ def ss_debug_candidates(ctx, frame, level, cap=1 << 21):
     _check(lib().ss_debug_candidates(ctx, frame, level, lx.ctypes.data, ly.ctypes.data, sc.ctypes.data, cap,
                                      C.byref(n)), ctx)
     return lx[:n.value].copy(), ly[:n.value].copy(), sc[:n.value].copy()
+
+
+def ss_debug_phase_times(ctx, frame, level, n=10) -> np.ndarray:
+    out = np.zeros(n, np.int64)
+    _check(lib().ss_debug_phase_times(ctx, frame, level, out.ctypes.data, n), ctx)
+    return out
 
 
 def ss_debug_overflow_count(ctx) -> int:

@@ -218,3 +218,19 @@ def test_brute_match_bit_exact(torch_cuda, ref):
         if n_map == 20000:
             assert (got["idx"] >= 0).sum() > 100
         pipe.close()
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
+def test_compute_sanitizer_clean(torch_cuda, tool):
+    """No memory errors, shared-memory races or barrier misuse on a small extract + match."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    cs = "/usr/local/cuda/bin/compute-sanitizer"
+    r = subprocess.run([cs, "--tool", tool, "--error-exitcode", "9", sys.executable,
+                        os.path.join(root, "scripts", "sanitize_extract.py")],
+                       capture_output=True, text=True, timeout=900)
+    tail = (r.stdout + r.stderr)[-3000:]
+    assert r.returncode == 0 and "sanitize run ok" in r.stdout, tail
+    assert "ERROR SUMMARY: 0 errors" in r.stdout + r.stderr or "RACECHECK SUMMARY: 0 hazards" in r.stdout + r.stderr, tail
