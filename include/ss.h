@@ -156,11 +156,10 @@ ss_status ss_match_projection(ss_ctx* ctx, int32_t n_frames, const ss_keypoint* 
  * kernel it launches, continuing across calls until the next ss_profile_events call
  * (n_events = 0 disables; events beyond n_events are not recorded).  One extract records a
  * start event, then a (before, after) pair around every kernel launch on the stream it runs
- * on, in this order: fast(level 0), distribute(level 0), then for l = 1..L-1: pyramid(l),
- * fast(l), distribute(l); then describe: 1 + 6 L events for L levels.  Level l's FAST and
- * distribution run on internal side streams
- * forked from `stream`.  WINDOW match: a pair per kernel (match_prepare, match_window[,
- * match_resolve if dedup]), preceded by nothing; BRUTE: pairs for brute_partial, brute_merge.
+ * on, in this order: fast(level 0), distribute(level 0) [internal side stream forked from
+ * `stream`], pyramid(l) for l = 1..L-1, fast(levels >= 1), distribute(levels >= 1),
+ * describe: 1 + 2 (L + 4) events for L levels.  WINDOW match: a pair per kernel
+ * (match_prepare, match_window[, match_resolve if dedup]); BRUTE: brute_partial, brute_merge.
  * Works under CUDA-graph stream capture (the records become graph event nodes).
  * *next_index (may be NULL) receives the index of the next event to be recorded. */
 ss_status ss_profile_events(ss_ctx* ctx, void* const* events, int32_t n_events);

@@ -444,44 +444,39 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   SS_CUDA_TRY(check_stream(s));
   const Geom& g = c->g;
   FrameSrc src{d_frames, frame_stride, pitch, c->pyr};
-  // DAG: level l's FAST + distribution run on a side stream as soon as level l exists (level
-  // 0 at once, levels >= 1 after their pyramid launch on the caller's stream); describe joins.
+  // DAG: level 0's FAST + distribution run on side stream 0 (they need no pyramid) while the
+  // caller's stream builds levels 1..L-1 and runs their FAST + distribution (one launch each:
+  // per-level launches cost more in launch latency than the overlap saves); describe joins.
   // Profiling events: start, then a (before, after) pair around every launch in this order:
-  // fast l0, distribute l0, then per level l >= 1: pyramid l, fast l, distribute l; describe.
+  // fast l0, distribute l0, pyramid l1 .. l(L-1), fast l>=1, distribute l>=1, describe.
   prof_mark(c, s);
   SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 2, s));
   SS_CUDA_TRY(cudaEventRecord(c->ev_fork, s));
-  bool used[ss_ctx::kSide] = {};
-  auto level_branch = [&](int l, cudaStream_t q) -> cudaError_t {
-    prof_mark(c, q);
-    cudaError_t e = launch_fast_bands(g, n_frames, src, c->bands + g.band_first[l], g.band_count[l], c->cells,
-                                      c->slots, c->cell_counts, q);
-    if (e != cudaSuccess) return e;
-    prof_mark(c, q);
-    prof_mark(c, q);
-    e = launch_distribute(g, n_frames, l, 1, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
-                          c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, c->phase_ts, q);
-    prof_mark(c, q);
-    return e;
-  };
-  SS_CUDA_TRY(cudaStreamWaitEvent(c->side[0], c->ev_fork, 0));
-  used[0] = true;
-  SS_CUDA_TRY(level_branch(0, c->side[0]));
+  cudaStream_t q = c->side[0];
+  SS_CUDA_TRY(cudaStreamWaitEvent(q, c->ev_fork, 0));
+  prof_mark(c, q);
+  SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands, g.band_count[0], c->cells, c->slots, c->cell_counts, q));
+  prof_mark(c, q);
+  prof_mark(c, q);
+  SS_CUDA_TRY(launch_distribute(g, n_frames, 0, 1, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts,
+                                c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, c->phase_ts, q));
+  prof_mark(c, q);
+  SS_CUDA_TRY(cudaEventRecord(c->ev_join[0], q));
   for (int l = 1; l < g.L; l++) {
     prof_mark(c, s);
     SS_CUDA_TRY(launch_pyramid_level(g, l, n_frames, src, c->xytab, c->pyr_tabs, s));
     prof_mark(c, s);
-    SS_CUDA_TRY(cudaEventRecord(c->ev_level[l], s));
-    const int si = 1 + (l % ss_ctx::kSideLevel);
-    SS_CUDA_TRY(cudaStreamWaitEvent(c->side[si], c->ev_level[l], 0));
-    used[si] = true;
-    SS_CUDA_TRY(level_branch(l, c->side[si]));
   }
-  for (int i = 0; i < ss_ctx::kSide; i++) {
-    if (!used[i]) continue;
-    SS_CUDA_TRY(cudaEventRecord(c->ev_join[i], c->side[i]));
-    SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[i], 0));
-  }
+  prof_mark(c, s);
+  SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands + g.band_count[0], g.total_bands - g.band_count[0],
+                                c->cells, c->slots, c->cell_counts, s));
+  prof_mark(c, s);
+  prof_mark(c, s);
+  SS_CUDA_TRY(launch_distribute(g, n_frames, 1, g.L - 1, c->cells, c->slots, c->cell_counts, c->selected,
+                                c->sel_counts, c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter,
+                                c->phase_ts, s));
+  prof_mark(c, s);
+  SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[0], 0));
   prof_mark(c, s);
   SS_CUDA_TRY(launch_describe(g, n_frames, src, c->selected, c->sel_counts, c->pattern, d_kps, d_desc, d_counts, s));
   prof_mark(c, s);

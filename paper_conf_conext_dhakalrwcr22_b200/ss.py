@@ -175,10 +175,8 @@ def ss_profile_next(ctx) -> int:
 
 def extract_kernels(n_levels: int) -> list[str]:
     """Kernel launches of one ss_orb_extract in profiling-event order (include/ss.h)."""
-    out = ["fast_l0", "distribute_l0"]
-    for l in range(1, n_levels):
-        out += [f"pyramid_l{l}", f"fast_l{l}", f"distribute_l{l}"]
-    return out + ["describe"]
+    return (["fast_l0", "distribute_l0"] + [f"pyramid_l{l}" for l in range(1, n_levels)] +
+            ["fast_l1plus", "distribute_l1plus", "describe"])
 
 
 def extract_events(n_levels: int) -> int:
