@@ -162,6 +162,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
       q0 = q1; q1 = q2; q2 = q3; q3 = q4; q4 = q5; q5 = q6;
     }
   }
+  __syncwarp();  // V complete and P consumed before B (aliasing P) is written
   for (int r = lane; r < BR; r += 32) {
     const uint16_t* vr = V + r * VP;
     int v0 = vr[0], v1 = vr[1], v2 = vr[2], v3 = vr[3], v4 = vr[4], v5 = vr[5];
