@@ -180,7 +180,7 @@ ss_status ss_debug_candidates(ss_ctx* ctx, int32_t frame, int32_t level, int32_t
 
 /* Global-timer timestamps (ns) of the distribution phases of (frame, level) in the last
  * ss_orb_extract: [0] start, [1] candidate count known, [2] candidates gathered, [3] dense
- * tables cleared, [4] keys + deepest histogram, [5] stop rules evaluated, [6] partial round,
+ * tables cleared, [4] keys + per-depth node counts, [5] stop rules evaluated, [6] partial round,
  * [7] best keys, [8] kept keys listed, [9] written (dense path; unused slots unspecified). */
 ss_status ss_debug_phase_times(ss_ctx* ctx, int32_t frame, int32_t level, int64_t* h_ns, int32_t n);
 

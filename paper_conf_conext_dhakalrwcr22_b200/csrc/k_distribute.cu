@@ -391,12 +391,13 @@ __device__ __forceinline__ void distribute_body(const Geom& g, int l, int f, int
 // need a depth beyond R -- the caller then runs the sort-based body on the same candidates.
 constexpr int DENSE_BINS = 4096;      // nIni * 4^R <= DENSE_BINS
 constexpr int DENSE_TOTAL = 5464;     // sum_{r<=R} nIni * 4^r <= 4/3 DENSE_BINS
-constexpr int DENSE_REC = 1024;       // multi-key bins at the partial depth (<= DENSE_BINS / 4)
+constexpr int DENSE_REC = 1024;       // multi-key bins at the partial depth (<= DENSE_BINS / 4 = DT)
 
 __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* cand, uint32_t* key, uint8_t* ws,
                            Shared& S_, uint32_t* __restrict__ selected, int32_t* __restrict__ sel_counts,
                            int32_t* ovf_counter, uint64_t* phase_ts) {
-  const int tid = threadIdx.x;
+  typedef cub::BlockScan<int, DT> Scan;
+  const int tid = threadIdx.x, lane = tid & 31;
   const int N = g.N[l];
   const int nini = g.nini[l];
   int R = 0;
@@ -410,14 +411,10 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
   int32_t* order = recnode + DENSE_REC;
   uint8_t* recch = reinterpret_cast<uint8_t*>(order + DENSE_REC);
   uint8_t* split = recch + DENSE_REC;                         // [DENSE_BINS / 4]
-  int off[8], sz[8];
+  // bins of depth r start at off(r) = nini (4^r - 1) / 3
+  auto off = [&](int r) { return nini * (((1 << (2 * r)) - 1) / 3); };
   {
-    int o = 0;
-    for (int r = 0; r <= R; r++) {
-      off[r] = o;
-      sz[r] = nini << (2 * r);
-      o += sz[r];
-    }
+    const int o = off(R + 1);
     for (int i = tid; i < o; i += DT) cnt[i] = 0u;
     if (tid < 8) {
       S_.H[tid] = 0;  // non-empty bins per depth
@@ -426,40 +423,57 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
   }
   __syncthreads();  // bins zeroed before any increment
   SS_PHASE(3);
-  // keys to depth R + 1 (the partial round at D <= R - 1 looks at D + 1 <= R); only the deepest
-  // histogram takes atomics (few keys share a bin), shallower depths are sums of 4 children
-  for (int i = tid; i < n; i += DT) {
-    const uint32_t k = make_key(g, l, cand[i], R + 1);
-    key[i] = k;
-    atomicAdd(&cnt[off[R] + (int)(k >> (26 - 2 * R))], 1u);
+  // one pass: key to depth R (+1 spare round), one increment per depth; the value an
+  // increment returns says whether it opened a bin (S_r) or made it multi-key (E_r)
+  {
+    int nz[7] = {0, 0, 0, 0, 0, 0, 0}, mu[7] = {0, 0, 0, 0, 0, 0, 0};
+    for (int base = 0; base < n; base += DT) {
+      const int i = base + tid;
+      const bool act = i < n;
+      uint32_t k = 0;
+      if (act) {
+        k = make_key(g, l, cand[i], R + 1);
+        key[i] = k;
+      }
+#pragma unroll
+      for (int r = 0; r < 7; r++) {
+        if (r > R) break;
+        const int bin = off(r) + (int)(k >> (26 - 2 * r));
+        if (r < 3) {  // few bins: aggregate the warp's increments per bin first
+          const unsigned am = __ballot_sync(0xFFFFFFFFu, act);
+          if (act) {
+            const unsigned peers = __match_any_sync(am, bin);
+            const int leader = __ffs(peers) - 1, c = __popc(peers);
+            if (lane == leader) {
+              const uint32_t old = atomicAdd(&cnt[bin], (uint32_t)c);
+              nz[r] += old == 0u;
+              mu[r] += (old == 1u) || (old == 0u && c >= 2);
+            }
+          }
+        } else if (act) {
+          const uint32_t old = atomicAdd(&cnt[bin], 1u);
+          nz[r] += old == 0u;
+          mu[r] += old == 1u;
+        }
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < 7; r++) {
+      if (r > R) break;
+      int a = nz[r], m = mu[r];
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        a += __shfl_xor_sync(0xFFFFFFFFu, a, o);
+        m += __shfl_xor_sync(0xFFFFFFFFu, m, o);
+      }
+      if (lane == 0) {
+        if (a) atomicAdd(&S_.H[r], a);
+        if (m) atomicAdd(&S_.G[r], m);
+      }
+    }
   }
   __syncthreads();
   SS_PHASE(4);
-  for (int r = R - 1; r >= 0; r--) {
-    for (int b = tid; b < sz[r]; b += DT) {
-      const uint32_t* ch = cnt + off[r + 1] + 4 * b;
-      cnt[off[r] + b] = ch[0] + ch[1] + ch[2] + ch[3];
-    }
-    __syncthreads();
-  }
-  for (int r = 0; r <= R; r++) {
-    int nz = 0, mu = 0;
-    for (int b = tid; b < sz[r]; b += DT) {
-      const uint32_t c = cnt[off[r] + b];
-      nz += c > 0u;
-      mu += c > 1u;
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      nz += __shfl_xor_sync(0xFFFFFFFFu, nz, o);
-      mu += __shfl_xor_sync(0xFFFFFFFFu, mu, o);
-    }
-    if ((tid & 31) == 0) {
-      if (nz) atomicAdd(&S_.H[r], nz);
-      if (mu) atomicAdd(&S_.G[r], mu);
-    }
-  }
-  __syncthreads();
   if (tid == 0) {
     // ORB-SLAM's loop on node counts (as in the sort path); -1 = a depth > R is needed
     int D = -1, partial = 0, r = 0;
@@ -503,8 +517,8 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
     for (int i = tid; i < n; i += DT) atomicMin(&first[key[i] >> (26 - 2 * D)], (uint32_t)i);
     __syncthreads();
     // the multi-key nodes at depth D, ordered by (size desc, UL.y, UL.x, first-key rank)
-    const uint32_t* cD = cnt + off[D];
-    const uint32_t* cD1 = cnt + off[D + 1];
+    const uint32_t* cD = cnt + off(D);
+    const uint32_t* cD1 = cnt + off(D + 1);
     for (int b = tid; b < szD; b += DT) {
       const uint32_t c = cD[b];
       if (c > 1u) {
@@ -526,13 +540,15 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
       order[pos] = e;
     }
     __syncthreads();
-    if (tid == 0) {
-      int acc = S_.H[D];
-      for (int t = 0; t < ne && acc < N; t++) {
-        const int e = order[t];
-        acc += recch[e] - 1;
-        split[recnode[e]] = 1;
-      }
+    // split the prefix of that order that first brings the node count to >= N: an inclusive
+    // scan of (children - 1) over the sorted nodes (ne <= DENSE_REC = DT)
+    {
+      const int e = tid < ne ? order[tid] : 0;
+      const int inc = tid < ne ? (int)recch[e] - 1 : 0;
+      int ex, tot;
+      Scan(S_.scan).ExclusiveSum(inc, ex, tot);
+      // node t is split iff the nodes before it have not yet reached N
+      if (tid < ne && S_.H[D] + ex < N) split[recnode[e]] = 1;
     }
   }
   __syncthreads();
@@ -548,7 +564,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
   __syncthreads();
   SS_PHASE(7);
   uint32_t* kept = key;  // keys are no longer needed
-  const uint32_t* cD = cnt + off[D];
+  const uint32_t* cD = cnt + off(D);
   for (int b = tid; b < szD; b += DT) {
     if (cD[b] == 0u) continue;
     if (partial && split[b]) {
