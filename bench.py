@@ -440,7 +440,7 @@ def run_ours(args, cfg):
             pass
 
     # --- e2e through the public API with host buffers (pinned), copies inside the timed region
-    e2e = run_e2e(args, pipe, frames_h, q_host, map_desc, out, B, Q, window, dev, stream)
+    e2e = run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams)
 
     frames_per_step = B * world
     value = frames_per_step * K / (T_max / 1000.0)
@@ -481,58 +481,70 @@ def run_ours(args, cfg):
         print(json.dumps(res), flush=True)
 
 
-def run_e2e(args, pipe, frames_h, q_host, map_desc, out, B, Q, window, dev, stream):
+def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams):
+    """Same ticks through the C ABI from pinned host buffers: H2D of the tick's inputs, extract +
+    match, D2H of all results, every step inside the timed region; ticks round-robin over the
+    in-flight contexts/streams so copies of one tick overlap compute of another."""
     import torch
-
-    from paper_conf_conext_dhakalrwcr22_b200.pipeline import match_records  # noqa: F401
+    P = len(pipes)
     n_host = min(len(frames_h), 8)
     fr = [torch.from_numpy(frames_h[s]).pin_memory() for s in range(n_host)]
-    dfr = torch.empty_like(fr[0], device=dev)
     if window:
         qh = [torch.from_numpy(np.ascontiguousarray(q_host[s % len(q_host)][0]).view(np.uint8).reshape(Q, 20)).pin_memory()
               for s in range(n_host)]
         qdh = [torch.from_numpy(q_host[s % len(q_host)][1]).pin_memory() for s in range(n_host)]
         tkh = [torch.from_numpy(q_host[s % len(q_host)][2]).pin_memory() for s in range(n_host)]
-        dq, dqd, dtk = (torch.empty_like(x[0], device=dev) for x in (qh, qdh, tkh))
-    kps_h = torch.empty(pipe.kps[:B].shape, dtype=torch.uint8).pin_memory()
-    desc_h = torch.empty(pipe.desc[:B].shape, dtype=torch.uint8).pin_memory()
-    cnt_h = torch.empty(pipe.counts[:B].shape, dtype=torch.int32).pin_memory()
-    out_h = torch.empty(out.shape, dtype=torch.int32).pin_memory()
+    dev_in, host_out = [], []
+    for q in range(P):  # per in-flight context: device inputs, pinned host outputs
+        d = {"fr": torch.empty_like(fr[0], device=dev)}
+        if window:
+            d.update(q=torch.empty_like(qh[0], device=dev), qd=torch.empty_like(qdh[0], device=dev),
+                     tk=torch.empty_like(tkh[0], device=dev))
+        dev_in.append(d)
+        host_out.append([torch.empty(pipes[q].kps[:B].shape, dtype=torch.uint8).pin_memory(),
+                         torch.empty(pipes[q].desc[:B].shape, dtype=torch.uint8).pin_memory(),
+                         torch.empty(pipes[q].counts[:B].shape, dtype=torch.int32).pin_memory(),
+                         torch.empty(outs[q].shape, dtype=torch.int32).pin_memory()])
     h2d = fr[0].numel() + ((qh[0].numel() + qdh[0].numel() + tkh[0].numel()) if window else 0)
-    d2h = kps_h.numel() + desc_h.numel() + cnt_h.numel() * 4 + out_h.numel() * 4
+    d2h = sum(t.numel() * t.element_size() for t in host_out[0])
 
     def step(s):
-        i = s % n_host
-        dfr.copy_(fr[i], non_blocking=True)
-        if window:
-            dq.copy_(qh[i], non_blocking=True)
-            dqd.copy_(qdh[i], non_blocking=True)
-            dtk.copy_(tkh[i], non_blocking=True)
-        pipe.extract(dfr, stream=stream)
-        if window:
-            pipe.match_window(B, dq, dqd, out, taken=dtk, stream=stream)
-        else:
-            pipe.match_brute(B, map_desc, out, stream=stream)
-        kps_h.copy_(pipe.kps[:B], non_blocking=True)
-        desc_h.copy_(pipe.desc[:B], non_blocking=True)
-        cnt_h.copy_(pipe.counts[:B], non_blocking=True)
-        out_h.copy_(out, non_blocking=True)
+        i, q = s % n_host, s % P
+        d, (kh, dh, ch, oh), pp, ot = dev_in[q], host_out[q], pipes[q], outs[q]
+        with torch.cuda.stream(streams[q]):
+            d["fr"].copy_(fr[i], non_blocking=True)
+            if window:
+                d["q"].copy_(qh[i], non_blocking=True)
+                d["qd"].copy_(qdh[i], non_blocking=True)
+                d["tk"].copy_(tkh[i], non_blocking=True)
+            pp.extract(d["fr"], stream=streams[q])
+            if window:
+                pp.match_window(B, d["q"], d["qd"], ot, taken=d["tk"], stream=streams[q])
+            else:
+                pp.match_brute(B, map_desc, ot, stream=streams[q])
+            kh.copy_(pp.kps[:B], non_blocking=True)
+            dh.copy_(pp.desc[:B], non_blocking=True)
+            ch.copy_(pp.counts[:B], non_blocking=True)
+            oh.copy_(ot, non_blocking=True)
 
     K = max(1, min(args.steps, 200))
-    with torch.cuda.stream(stream):
-        for s in range(3):
-            step(s)
-        torch.cuda.synchronize(dev)
-        t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        t0.record(stream)
-        for s in range(K):
-            step(s)
-        t1.record(stream)
+    for s in range(3):
+        step(s)
+    torch.cuda.synchronize(dev)
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    t0.record(streams[0])
+    for q in range(1, P):
+        streams[q].wait_event(t0)
+    for s in range(K):
+        step(s)
+    for q in range(1, P):
+        streams[0].wait_stream(streams[q])
+    t1.record(streams[0])
     torch.cuda.synchronize(dev)
     ms = t0.elapsed_time(t1)
     world = int(os.environ.get("WORLD_SIZE", 1))
     return {"value": B * world * K / (ms / 1000.0), "unit": "frames/s", "h2d_bytes_per_step": int(h2d),
-            "d2h_bytes_per_step": int(d2h), "steps": K, "ms_per_step": ms / K,
+            "d2h_bytes_per_step": int(d2h), "steps": K, "ms_per_step": ms / K, "ticks_in_flight": P,
             "path": "pinned host -> H2D -> ss_orb_extract -> ss_match_projection -> D2H (C ABI, no graphs)"}
 
 
@@ -673,7 +685,7 @@ def main(argv=None):
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--config", choices=sorted(CONFIGS), default="c2")
     ap.add_argument("--ring", type=int, default=0, help="override the number of input ring slots")
-    ap.add_argument("--inflight", type=int, default=3, help="ticks in flight (contexts/streams)")
+    ap.add_argument("--inflight", type=int, default=4, help="ticks in flight (contexts/streams)")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args(argv)

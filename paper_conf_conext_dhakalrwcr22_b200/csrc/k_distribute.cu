@@ -423,39 +423,38 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
   }
   __syncthreads();  // bins zeroed before any increment
   SS_PHASE(3);
-  // one pass: key to depth R (+1 spare round), one increment per depth; the value an
-  // increment returns says whether it opened a bin (S_r) or made it multi-key (E_r)
+  // one pass over the keys in a scattered order (consecutive candidates share cells, hence
+  // bins): key to depth R (+1 spare round), one increment per depth >= r_lo; the value an
+  // increment returns says whether it opened a bin (S_r) or made it multi-key (E_r).  The few
+  // shallow bins (depth < r_lo) are sums of their 4 children, formed afterwards.
+  const int r_lo = R < 3 ? R : 3;
   {
     int nz[7] = {0, 0, 0, 0, 0, 0, 0}, mu[7] = {0, 0, 0, 0, 0, 0, 0};
-    for (int base = 0; base < n; base += DT) {
-      const int i = base + tid;
-      const bool act = i < n;
-      uint32_t k = 0;
-      if (act) {
-        k = make_key(g, l, cand[i], R + 1);
-        key[i] = k;
-      }
+    uint32_t stride = 1031u;
+    while ((uint32_t)n % stride == 0u) stride += 2u;  // an odd prime-ish step coprime with n
+    for (int j = tid; j < n; j += DT) {
+      const int i = (int)(((uint64_t)j * stride) % (uint32_t)n);
+      const uint32_t k = make_key(g, l, cand[i], R + 1);
+      key[i] = k;
 #pragma unroll
       for (int r = 0; r < 7; r++) {
-        if (r > R) break;
-        const int bin = off(r) + (int)(k >> (26 - 2 * r));
-        if (r < 3) {  // few bins: aggregate the warp's increments per bin first
-          const unsigned am = __ballot_sync(0xFFFFFFFFu, act);
-          if (act) {
-            const unsigned peers = __match_any_sync(am, bin);
-            const int leader = __ffs(peers) - 1, c = __popc(peers);
-            if (lane == leader) {
-              const uint32_t old = atomicAdd(&cnt[bin], (uint32_t)c);
-              nz[r] += old == 0u;
-              mu[r] += (old == 1u) || (old == 0u && c >= 2);
-            }
-          }
-        } else if (act) {
-          const uint32_t old = atomicAdd(&cnt[bin], 1u);
-          nz[r] += old == 0u;
-          mu[r] += old == 1u;
-        }
+        if (r < r_lo || r > R) continue;
+        const uint32_t old = atomicAdd(&cnt[off(r) + (int)(k >> (26 - 2 * r))], 1u);
+        nz[r] += old == 0u;
+        mu[r] += old == 1u;
       }
+    }
+    __syncthreads();
+    for (int r = r_lo - 1; r >= 0; r--) {
+      const int sz = nini << (2 * r);
+      for (int b = tid; b < sz; b += DT) {
+        const uint32_t* ch = cnt + off(r + 1) + 4 * b;
+        const uint32_t c = ch[0] + ch[1] + ch[2] + ch[3];
+        cnt[off(r) + b] = c;
+        nz[r] += c > 0u;
+        mu[r] += c > 1u;
+      }
+      __syncthreads();
     }
 #pragma unroll
     for (int r = 0; r < 7; r++) {
