@@ -155,9 +155,10 @@ ss_status ss_match_projection(ss_ctx* ctx, int32_t n_frames, const ss_keypoint* 
  * its stream: the next unused event before its first operation, then one after every
  * kernel it launches, continuing across calls until the next ss_profile_events call
  * (n_events = 0 disables; events beyond n_events are not recorded).  One extract records a
- * start event, then a (before, after) pair around every kernel launch on the stream it runs
- * on, in this order: fast(level 0), distribute(level 0) [internal side stream forked from
- * `stream`], pyramid(l) for l = 1..L-1, fast(levels >= 1), distribute(levels >= 1),
+ * start event, then a (before, after) pair around every kernel launch, in this order:
+ * fast(level 0), distribute(level 0), pyramid(l) for l = 1..L-1, fast(levels >= 1),
+ * distribute(levels >= 1), describe (while events are installed the level-0 branch runs in
+ * line on `stream` instead of on its side stream, so each kernel is timed alone):
  * describe: 1 + 2 (L + 4) events for L levels.  WINDOW match: a pair per kernel
  * (match_prepare, match_window[, match_resolve if dedup]); BRUTE: brute_partial, brute_merge.
  * Works under CUDA-graph stream capture (the records become graph event nodes).

@@ -433,7 +433,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
     uint32_t stride = 1031u;
     while ((uint32_t)n % stride == 0u) stride += 2u;  // an odd prime-ish step coprime with n
     for (int j = tid; j < n; j += DT) {
-      const int i = (int)(((uint64_t)j * stride) % (uint32_t)n);
+      const int i = (int)(((uint32_t)j * stride) % (uint32_t)n);  // j < 8192: no overflow
       const uint32_t k = make_key(g, l, cand[i], R + 1);
       key[i] = k;
 #pragma unroll

@@ -452,8 +452,10 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   prof_mark(c, s);
   SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 2, s));
   SS_CUDA_TRY(cudaEventRecord(c->ev_fork, s));
-  cudaStream_t q = c->side[0];
-  SS_CUDA_TRY(cudaStreamWaitEvent(q, c->ev_fork, 0));
+  // with profiling events installed the level-0 branch runs in line on `stream`, so every
+  // kernel is timed alone (the fork/join only changes overlap, not any kernel's work)
+  cudaStream_t q = c->prof.empty() ? c->side[0] : s;
+  if (q != s) SS_CUDA_TRY(cudaStreamWaitEvent(q, c->ev_fork, 0));
   prof_mark(c, q);
   SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands, g.band_count[0], c->cells, c->slots, c->cell_counts, q));
   prof_mark(c, q);
@@ -461,7 +463,7 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   SS_CUDA_TRY(launch_distribute(g, n_frames, 0, 1, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts,
                                 c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, c->phase_ts, q));
   prof_mark(c, q);
-  SS_CUDA_TRY(cudaEventRecord(c->ev_join[0], q));
+  if (q != s) SS_CUDA_TRY(cudaEventRecord(c->ev_join[0], q));
   for (int l = 1; l < g.L; l++) {
     prof_mark(c, s);
     SS_CUDA_TRY(launch_pyramid_level(g, l, n_frames, src, c->xytab, c->pyr_tabs, s));
@@ -476,7 +478,7 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
                                 c->sel_counts, c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter,
                                 c->phase_ts, s));
   prof_mark(c, s);
-  SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[0], 0));
+  if (q != s) SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[0], 0));
   prof_mark(c, s);
   SS_CUDA_TRY(launch_describe(g, n_frames, src, c->selected, c->sel_counts, c->pattern, d_kps, d_desc, d_counts, s));
   prof_mark(c, s);
