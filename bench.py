@@ -424,9 +424,9 @@ def run_ours(args, cfg):
                 "peak_src": "derived: 148 SM x 64 ALU lanes/clk x 1.965 GHz (DESIGN.md §6)",
                 "work": f"{FAST_OPS_PER_PX} ops per detect pixel", "share_of_step": step_share}
     else:
-        popc_peak = 148 * 16 * 1.965 / 8  # Tdist/s at the 1965 MHz max SM clock
-        achieved = work / (avg_us[dom] * 1e-6) / 1e12
-        roof = {"bound": "alu", "achieved": achieved, "peak": popc_peak, "unit": "Tdist/s",
+        popc_peak = 148 * 16 * 1.965 / 8  # Gdist/s at the 1965 MHz max SM clock
+        achieved = work / (avg_us[dom] * 1e-6) / 1e9
+        roof = {"bound": "alu", "achieved": achieved, "peak": popc_peak, "unit": "Gdist/s",
                 "frac": achieved / popc_peak, "traffic": None, "kernel": dom,
                 "peak_src": "derived: 148 SM x 16 POPC/clk x clock / 8 POPC per distance", "share_of_step": step_share}
     traffic_file = os.path.join(ROOT, "profiles", "dram_traffic_r01.json")

@@ -111,7 +111,10 @@ ss_status ss_orb_params_init(int32_t width, int32_t height, int32_t n_features, 
 /* Create a context on `device` for frames of shape p (p must equal what
  * ss_orb_params_init returns for its own first seven fields, else SS_EINVAL).
  * max_frames bounds n_frames per call, max_queries the WINDOW query count and max_map the
- * BRUTE map size (0 = that mode unused).  Allocates all scratch here (none per call). */
+ * BRUTE map size (0 = that mode unused).  Allocates all scratch here (none per call).
+ * SS_EUNSUPPORTED when this build's kernels cannot serve p: scale_factor above 4/3 (the
+ * pyramid kernel's source window), kp_capacity above 65535, or a FAST band / pyramid block
+ * that does not fit in shared memory. */
 ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, int32_t max_queries,
                     int32_t max_map, ss_ctx** out);
 ss_status ss_destroy(ss_ctx* ctx);
@@ -156,10 +159,10 @@ ss_status ss_match_projection(ss_ctx* ctx, int32_t n_frames, const ss_keypoint* 
  * kernel it launches, continuing across calls until the next ss_profile_events call
  * (n_events = 0 disables; events beyond n_events are not recorded).  One extract records a
  * start event, then a (before, after) pair around every kernel launch, in this order:
- * fast(level 0), distribute(level 0), pyramid(l) for l = 1..L-1, fast(levels >= 1),
- * distribute(levels >= 1), describe (while events are installed the level-0 branch runs in
- * line on `stream` instead of on its side stream, so each kernel is timed alone):
- * describe: 1 + 2 (L + 4) events for L levels.  WINDOW match: a pair per kernel
+ * fast(level 0), distribute(level 0), pyramid (levels 1..L-1, one launch), fast(levels >= 1),
+ * distribute(levels >= 1), describe -- 13 events (while events are installed the level-0
+ * branch runs in line on `stream` instead of on its side stream, so each kernel is timed
+ * alone).  WINDOW match: a pair per kernel
  * (match_prepare, match_window[, match_resolve if dedup]); BRUTE: brute_partial, brute_merge.
  * Works under CUDA-graph stream capture (the records become graph event nodes).
  * *next_index (may be NULL) receives the index of the next event to be recorded. */

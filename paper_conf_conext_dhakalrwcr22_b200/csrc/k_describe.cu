@@ -4,12 +4,14 @@
 // One warp per output keypoint slot.  The warp stages the 43x43 raw patch around the
 // keypoint (REFLECT_101 at the level border, which the blur needs) in shared memory and
 // derives everything from it: intensity-centroid moments over the 749-px disk (unblurred),
-// the 37x37 blurred patch (Q8 taps [18,34,48,56,48,34,18], exact horizontal sums, vertical
-// (sum + 2^15) >> 16, computed as two sliding-window passes), and the 256 comparisons at the
-// pattern points rotated by (cos, sin) = (m10, m01)/sqrt(m10^2 + m01^2), each offset rounded
-// half-to-even EXACTLY (f32 estimate; int64 test only within 1e-4 of a tie).  Blurring only the patch replaces a whole-level blur
-// pass and its HBM round trip.  Output position = the keypoint's canonical index, so the
-// per-level counts of the distribution become the prefix offsets written to d_counts.
+// the vertical blur pass over the patch (Q8 taps [18,34,48,56,48,34,18], exact sums, two
+// columns per register), and the 256 comparisons at the pattern points rotated by
+// (cos, sin) = (m10, m01)/sqrt(m10^2 + m01^2), each offset rounded half-to-even EXACTLY (f32
+// estimate; int64 test only within 1e-4 of a tie), with the horizontal blur pass and the
+// (sum + 2^15) >> 16 rounding evaluated at the 512 sample points only.  Blurring only what
+// the samples read replaces a whole-level blur pass and its HBM round trip.  Output
+// position = the keypoint's canonical index, so the per-level counts of the distribution
+// become the prefix offsets written to d_counts.
 #include "brief_pattern.inc"
 #include "ss_internal.h"
 
@@ -22,10 +24,7 @@ constexpr int PR = 43;  // raw patch: radius 21 (18 max sample offset + 3 blur t
 constexpr int PP = 64;  // raw patch pitch: a 16-B aligned 64-B window covers the 43 B row
 constexpr int BR = 37;  // blurred patch: radius 18
 constexpr int VP = 46;  // pitch (u16) of the vertical pass V[37][43]: 23 words (odd) per row
-constexpr int BP = 44;  // pitch of the blurred patch B[37][37]: 11 words (odd) per row
-// the blurred patch B reuses the raw patch's space (P is dead after the vertical pass)
 constexpr int PER_WARP = ((PR * PP + BR * VP * 2) + 127) & ~127;
-static_assert(BR * BP <= PR * PP, "B aliases P");
 
 __constant__ int c_umax[16] = {15, 15, 15, 15, 14, 14, 14, 13, 13, 12, 11, 10, 9, 8, 6, 3};
 
@@ -48,11 +47,17 @@ __device__ __noinline__ int rhe_exact(long long z, long long r2, int k) {
   return z < 0 ? -k : k;
 }
 
-__device__ __forceinline__ int rhe_div_sqrt(int z, long long r2, float inv_r) {
-  const float t = __fmul_rn((float)z, inv_r);
-  const float k = rintf(t);
-  if (fabsf(fabsf(t - k) - 0.5f) > 1e-4f) return (int)k;
-  return rhe_exact(z, r2, (int)k);
+// round-half-even of (a * m_a + b * m_b) / r for the rotated pattern offsets, r^2 = r2 > 0:
+// t = a * ca + b * cb in f32 (ca = m_a / r, cb = m_b / r; |t| <= 19, error < 1e-5), rounded
+// with the 1.5 * 2^23 trick (round-to-nearest-even, no conversion instructions); within 1e-4
+// of a half-integer the exact integer test decides.
+__device__ __forceinline__ int rhe_rot(int a, int b, float ca, float cb, int ma, int mb, long long r2) {
+  const float t = __fmaf_rn((float)a, ca, __fmul_rn((float)b, cb));
+  const float big = __fadd_rn(t, 12582912.0f);
+  const int k = __float_as_int(big) - 0x4B400000;
+  const float d = __fsub_rn(t, __fsub_rn(big, 12582912.0f));
+  if (fabsf(fabsf(d) - 0.5f) > 1e-4f) return k;
+  return rhe_exact((long long)a * ma + (long long)b * mb, r2, k);
 }
 
 __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, FrameSrc src,
@@ -99,7 +104,6 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
   const int w = g.w[l], h = g.h[l];
   uint8_t* Pw = sm + warp * PER_WARP;
   uint16_t* V = reinterpret_cast<uint16_t*>(Pw + PR * PP);
-  uint8_t* B = Pw;  // written only after the vertical pass has consumed P (syncwarp between)
   const uint8_t* p0 = img + (int64_t)(ly - 21) * ip + (lx - 21);
   const int sh = (int)(reinterpret_cast<uintptr_t>(p0) & 15);
   const uint8_t* P;  // P[r * PP + c] = raw patch pixel (ly - 21 + r, lx - 21 + c)
@@ -142,7 +146,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
   }
   // separable blur; all sums are exact integers until the final rounding, so the vertical
   // pass may come first: V[r][x] = sum_i k_i P[r + i][x] (lane = column, sliding over rows),
-  // then B[r][c] = (sum_j k_j V[r][c + j] + 2^15) >> 16 (lane = row, sliding over columns)
+  // then B[r][c] = (sum_j k_j V[r][c + j] + 2^15) >> 16 at the sample points (below)
   // pass 1 on packed column pairs: lane covers columns 2*lane, 2*lane + 1 as two 16-bit lanes
   // of one register (a weighted sum is <= 255 * 256, so the halves never carry)
   if (lane < (PR + 1) / 2) {
@@ -162,22 +166,13 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
       q0 = q1; q1 = q2; q2 = q3; q3 = q4; q4 = q5; q5 = q6;
     }
   }
-  __syncwarp();  // V complete and P consumed before B (aliasing P) is written
-  for (int r = lane; r < BR; r += 32) {
-    const uint16_t* vr = V + r * VP;
-    int v0 = vr[0], v1 = vr[1], v2 = vr[2], v3 = vr[3], v4 = vr[4], v5 = vr[5];
-#pragma unroll 4
-    for (int c = 0; c < BR; c++) {
-      const int v6 = vr[c + 6];
-      const int sum = 18 * (v0 + v6) + 34 * (v1 + v5) + 48 * (v2 + v4) + 56 * v3;
-      B[r * BP + c] = (uint8_t)((sum + (1 << 15)) >> 16);
-      v0 = v1; v1 = v2; v2 = v3; v3 = v4; v4 = v5; v5 = v6;
-    }
-  }
-  __syncwarp();
-  // rotated BRIEF: lane = output byte; bit t compares points 2b, 2b+1 with b = 8*lane + t
+  __syncwarp();  // V complete
+  // rotated BRIEF: lane = output byte; bit t compares points 2b, 2b+1 with b = 8*lane + t.
+  // The blurred value is needed only at the 512 sample points, so the horizontal pass runs
+  // there alone: B(oy, ox) = (sum_j k_j V[18 + oy][18 + ox + j] + 2^15) >> 16.
   const long long r2 = (long long)m10 * m10 + (long long)m01 * m01;
   const float inv_r = r2 ? (float)(1.0 / sqrt((double)r2)) : 0.f;
+  const float cs = (float)m10 * inv_r, sn = (float)m01 * inv_r;  // |m| < 2^24: exact conversions
   uint32_t byte = 0;
 #pragma unroll 2
   for (int t = 0; t < 8; t++) {
@@ -188,10 +183,12 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
       const int px = pat[4 * b + 2 * e], py = pat[4 * b + 2 * e + 1];
       int ox = px, oy = py;
       if (r2) {
-        ox = rhe_div_sqrt(px * m10 - py * m01, r2, inv_r);  // |.| <= 13 * 2 * 1248480 < 2^31
-        oy = rhe_div_sqrt(px * m01 + py * m10, r2, inv_r);
+        ox = rhe_rot(px, -py, cs, sn, m10, m01, r2);  // (px m10 - py m01) / r
+        oy = rhe_rot(px, py, sn, cs, m01, m10, r2);   // (px m01 + py m10) / r
       }
-      v[e] = B[(18 + oy) * BP + 18 + ox];
+      const uint16_t* vr = V + (18 + oy) * VP + 18 + ox;
+      const int sum = 18 * (vr[0] + vr[6]) + 34 * (vr[1] + vr[5]) + 48 * (vr[2] + vr[4]) + 56 * vr[3];
+      v[e] = (sum + (1 << 15)) >> 16;
     }
     byte |= (uint32_t)(v[0] < v[1]) << t;
   }

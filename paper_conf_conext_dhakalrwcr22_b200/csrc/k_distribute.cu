@@ -595,7 +595,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
 }
 
 __global__ void __launch_bounds__(DT, 1)
-    distribute_kernel(Geom g, const CellInfo* __restrict__ cells, const uint32_t* __restrict__ slots,
+    distribute_kernel(const __grid_constant__ Geom g, const CellInfo* __restrict__ cells, const uint32_t* __restrict__ slots,
                       const int32_t* __restrict__ cell_counts, uint32_t* __restrict__ selected,
                       int32_t* __restrict__ sel_counts, uint8_t* ovf, int64_t ovf_frame_bytes,
                       const int64_t* __restrict__ ovf_level_off, int32_t* ovf_counter, int level0,

@@ -93,7 +93,7 @@ __device__ __forceinline__ uint32_t fast_M4(const uint32_t (&W)[7][3]) {
   return __byte_perm(slo, shi, 0x6240);
 }
 
-__global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(Geom g, FrameSrc src,
+__global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(const __grid_constant__ Geom g, FrameSrc src,
                                                                 const BandInfo* __restrict__ bands,
                                                                 const CellInfo* __restrict__ cells,
                                                                 uint32_t* __restrict__ slots,

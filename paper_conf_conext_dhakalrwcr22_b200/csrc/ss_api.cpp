@@ -125,6 +125,9 @@ struct ss_ctx {
   CellInfo* cells = nullptr;
   BandInfo* bands = nullptr;
   uint32_t* xytab = nullptr;  // per level l >= 1: xtab [w_l], ytab [h_l]
+  PyrLvl* pyr_plan = nullptr;   // [pyr_blocks][L] fused-pyramid block records
+  uint4* pyr_gtab = nullptr;    // per level >= 1: 4-column group coefficients
+  int pyr_blocks = 0, pyr_buf0 = 0, pyr_buf1 = 0, pyr_smem = 0;
   std::vector<int64_t> xoff, yoff;
   uint8_t* pyr = nullptr;
   uint32_t* slots = nullptr;
@@ -136,7 +139,6 @@ struct ss_ctx {
   int64_t* ovf_level_off = nullptr;
   int32_t* ovf_counter = nullptr;  // [0] overflowed levels, [1] capacity violations
   int8_t* pattern = nullptr;
-  PyrTabs pyr_tabs{};
   unsigned long long* claim = nullptr;
   uint16_t* rowidx = nullptr;  // WINDOW matcher: first keypoint per (frame, level, row)
   uint64_t* phase_ts = nullptr;  // distribution phase timestamps [max_frames][L][16] (debug hook)
@@ -175,7 +177,7 @@ inline void prof_mark(ss_ctx* c, cudaStream_t s) {
 void free_ctx(ss_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->device);
-  void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
+  void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr_plan, c->pyr_gtab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
                   c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->rowidx, c->phase_ts};
   for (void* q : ptrs)
     if (q) cudaFree(q);
@@ -358,15 +360,26 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     c->yoff[l] = (int64_t)tab.size();
     for (int y = 0; y < g.h[l]; y++) tab.push_back(lin_coef(y, g.h[l - 1], g.h[l]));
   }
-  for (int l = 1; l < L; l++) {
-    if (!pyramid_tiles_fit(g.w[l], g.h[l], tab.data() + c->xoff[l], tab.data() + c->yoff[l])) {
-      free_ctx(c);
-      return fail(SS_EUNSUPPORTED, "scale_factor too large for the pyramid's shared-memory tiles");
-    }
+  std::vector<PyrLvl> plan;
+  std::vector<uint4> gtab;
+  std::vector<int64_t> goff;
+  if (L > 1 && !pyramid_groups(g, tab.data(), c->xoff.data(), &gtab, &goff)) {
+    free_ctx(c);
+    return fail(SS_EUNSUPPORTED, "scale_factor above 4/3 is not supported by the pyramid kernel");
   }
-  for (int l = 0; l < kMaxLevels; l++) {
-    c->pyr_tabs.xoff[l] = l < L ? c->xoff[l] : 0;
-    c->pyr_tabs.yoff[l] = l < L ? c->yoff[l] : 0;
+  // fused pyramid: blocks of about 128 x 96 level-0 pixels (more, smaller blocks if a
+  // block does not fit)
+  if (L > 1) {
+    int gx = (g.w[0] + 127) / 128, gy = (g.h[0] + 95) / 96;
+    while (!pyramid_plan(g, tab.data(), c->xoff.data(), c->yoff.data(), goff, gx, gy, &plan, &c->pyr_buf0,
+                         &c->pyr_buf1, &c->pyr_smem)) {
+      if (gx >= g.w[L - 1] / 4 || gy >= g.h[L - 1]) {
+        free_ctx(c);
+        return fail(SS_EUNSUPPORTED, "no pyramid block plan fits shared memory");
+      }
+      if (gx <= gy) gx++; else gy++;
+    }
+    c->pyr_blocks = gx * gy;
   }
   // overflow scratch layout
   std::vector<int64_t> ovf_off(L, 0);
@@ -387,6 +400,8 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->cells, sizeof(CellInfo) * c->cells_h.size());
   ALLOC(c->bands, sizeof(BandInfo) * c->bands_h.size());
   ALLOC(c->xytab, sizeof(uint32_t) * tab.size());
+  if (!plan.empty()) ALLOC(c->pyr_plan, sizeof(PyrLvl) * plan.size());
+  if (!gtab.empty()) ALLOC(c->pyr_gtab, sizeof(uint4) * gtab.size());
   ALLOC(c->pyr, F * g.pyr_frame_bytes);
   ALLOC(c->slots, sizeof(uint32_t) * F * g.slots_per_frame);
   ALLOC(c->cell_counts, sizeof(int32_t) * F * g.total_cells);
@@ -404,6 +419,10 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (e == cudaSuccess) e = cudaMemcpy(c->cells, c->cells_h.data(), sizeof(CellInfo) * c->cells_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->bands, c->bands_h.data(), sizeof(BandInfo) * c->bands_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess && !tab.empty()) e = cudaMemcpy(c->xytab, tab.data(), sizeof(uint32_t) * tab.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess && !plan.empty())
+    e = cudaMemcpy(c->pyr_plan, plan.data(), sizeof(PyrLvl) * plan.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess && !gtab.empty())
+    e = cudaMemcpy(c->pyr_gtab, gtab.data(), sizeof(uint4) * gtab.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->ovf_level_off, ovf_off.data(), sizeof(int64_t) * L, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->pattern, pat.data(), 1024, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemset(c->ovf_counter, 0, sizeof(int32_t) * 2);
@@ -448,7 +467,7 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   // caller's stream builds levels 1..L-1 and runs their FAST + distribution (one launch each:
   // per-level launches cost more in launch latency than the overlap saves); describe joins.
   // Profiling events: start, then a (before, after) pair around every launch in this order:
-  // fast l0, distribute l0, pyramid l1 .. l(L-1), fast l>=1, distribute l>=1, describe.
+  // fast l0, distribute l0, pyramid (levels 1..L-1, one launch), fast l>=1, distribute l>=1, describe.
   prof_mark(c, s);
   SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 2, s));
   SS_CUDA_TRY(cudaEventRecord(c->ev_fork, s));
@@ -464,11 +483,11 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
                                 c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, c->phase_ts, q));
   prof_mark(c, q);
   if (q != s) SS_CUDA_TRY(cudaEventRecord(c->ev_join[0], q));
-  for (int l = 1; l < g.L; l++) {
-    prof_mark(c, s);
-    SS_CUDA_TRY(launch_pyramid_level(g, l, n_frames, src, c->xytab, c->pyr_tabs, s));
-    prof_mark(c, s);
-  }
+  prof_mark(c, s);
+  if (g.L > 1)
+    SS_CUDA_TRY(launch_pyramid(g, n_frames, src, c->pyr_gtab, c->xytab, c->pyr_plan, c->pyr_blocks, c->pyr_buf0,
+                               c->pyr_buf1, c->pyr_smem, s));
+  prof_mark(c, s);
   prof_mark(c, s);
   SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands + g.band_count[0], g.total_bands - g.band_count[0],
                                 c->cells, c->slots, c->cell_counts, s));

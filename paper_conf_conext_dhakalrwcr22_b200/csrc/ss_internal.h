@@ -4,6 +4,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <vector>
+
 #include "../../include/ss.h"
 
 namespace ss {
@@ -107,16 +109,34 @@ inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, s
 #endif
 
 // ---- launchers (one per kernel; each returns cudaGetLastError()) ----
-struct PyrTabs {
-  int64_t xoff[kMaxLevels], yoff[kMaxLevels];  // offsets of level l's x / y coefficient tables
+// Fused pyramid plan (k_pyramid.cu).  Host-side rectangles per (block, level), half-open:
+// N = computed (owned + the halo deeper levels need), O = owned (stored).  Level 0: N only
+// (the staged footprint, x0 aligned down to 16).
+struct PyrRect {
+  int16_t nx0, nx1, ny0, ny1, ox0, ox1, oy0, oy1;
 };
-// Levels 1..L-1 of all frames, one launch per level, 128x32 output tiles.
-cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const uint32_t* xytab, PyrTabs tabs,
-                           cudaStream_t s);
-cudaError_t launch_pyramid_level(const Geom& g, int l, int n_frames, FrameSrc src, const uint32_t* xytab, PyrTabs tabs,
-                                 cudaStream_t s);
-// Whether every tile's source rectangle fits the kernel's shared-memory staging.
-bool pyramid_tiles_fit(int dst_w, int dst_h, const uint32_t* xt, const uint32_t* yt);
+// Device-side per (block, level >= 1) record, read as four int4 (entry 0: the staged
+// footprint nx0/ny0/rows, ngx = staged width, dpitch = staged pitch, soff = s_y base).
+struct __align__(16) PyrLvl {
+  int32_t nx0, ngx, ny0, rows;        // computed rectangle: x0, 4-column groups, y0, rows
+  int32_t ox0, ox1, oy0, oy1;         // owned rectangle
+  int32_t sx0, sy0, spitch, dpitch;   // source rectangle origin + pitches of the smem buffers
+  int32_t mr, soff, gg, yg;           // ceil(2^20/ngx) | rows-in-parallel << 21; s_g | s_y << 16
+                                      // offsets; first group / row coefficient in the tables
+};
+constexpr int kPyrSmemMax = 200 * 1024;
+// Per 4-column group coefficient table of every level >= 1 (goff[l] = level l's first
+// entry); false if scale_factor > 4/3 (a group's source bytes exceed the 6-byte window).
+bool pyramid_groups(const Geom& g, const uint32_t* tab, const int64_t* xoff, std::vector<uint4>* gtab,
+                    std::vector<int64_t>* goff);
+// Plan gx x gy blocks per frame; false if a block does not fit (shared memory, one
+// coefficient load per thread per level).
+bool pyramid_plan(const Geom& g, const uint32_t* tab, const int64_t* xoff, const int64_t* yoff,
+                  const std::vector<int64_t>& goff, int gx, int gy, std::vector<PyrLvl>* plan, int* buf0, int* buf1,
+                  int* smem);
+// Levels 1..L-1 of all frames in one launch (grid: n_blocks x n_frames).
+cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const uint4* gtab, const uint32_t* ytab,
+                           const PyrLvl* plan, int n_blocks, int buf0, int buf1, int smem, cudaStream_t s);
 cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands, int n_bands,
                               const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s);
 size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int* mband_bytes, int* nball);

@@ -13,6 +13,10 @@ fi
 timeout 900 python bench.py ${BENCH_ARGS:-} > $OUT/bench_$TAG.json 2> $OUT/bench_$TAG.err; echo "bench rc=$?"
 tail -c 3000 $OUT/bench_$TAG.json
 tail -5 $OUT/bench_$TAG.err
+for C in ${EXTRA_CONFIGS:-}; do
+  timeout 600 python bench.py --config $C --steps 50 --warmup 5 --no-cpu-baseline > $OUT/bench_${TAG}_$C.json 2> $OUT/bench_${TAG}_$C.err
+  echo "bench $C rc=$?"; tail -c 600 $OUT/bench_${TAG}_$C.json
+done
 if [ "${SKIP_NCU:-0}" != "1" ]; then
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_$TAG.csv \
      python bench.py --steps 20 --warmup 3 --ring 8 --no-cpu-baseline ${NCU_BENCH_ARGS:-} > $OUT/ncu_bench_$TAG.log 2>&1

@@ -60,10 +60,14 @@ def _d2h(ptr, nbytes):
 def test_pyramid_bit_exact(torch_cuda, ref):
     torch = torch_cuda
     from paper_conf_conext_dhakalrwcr22_b200 import ss
-    for (w, h, L) in ((752, 480, 8), (333, 217, 3), (1241, 376, 8)):
+    # unaligned pitch (byte staging) and 16-B aligned pitch (vector staging); ragged and large
+    # frames so the fused kernel's block plan has partial blocks and several block shapes
+    for (w, h, L, pitch) in ((752, 480, 8, 752 + 13), (752, 480, 8, 768), (333, 217, 3, 333 + 13),
+                             (1241, 376, 8, 1241 + 13), (1241, 376, 8, 1248), (1920, 1080, 8, 1920),
+                             (250, 170, 2, 256)):
         frames = synth.make_frames(w, h, 2, cfg=11)
         pipe = _pipe(torch, w, h, 200, L, max_frames=2)
-        pipe.extract(_upload(torch, frames, pitch=w + 13))
+        pipe.extract(_upload(torch, frames, pitch=pitch))
         torch.cuda.synchronize()
         p = ref.params(w, h, 200, n_levels=L)
         for b in range(2):
@@ -74,6 +78,33 @@ def test_pyramid_bit_exact(torch_cuda, ref):
                 got = _d2h(ptr, lh * pitch).reshape(lh, pitch)[:, :lw]
                 np.testing.assert_array_equal(got, want[l], err_msg=f"{w}x{h} frame {b} level {l}")
         pipe.close()
+
+
+def test_pyramid_other_scales(torch_cuda, ref):
+    """Scale factors other than 1.2 change every level's coefficient pattern and the fused
+    kernel's block halos; above 4/3 the kernel's 6-byte source window no longer holds and
+    ss_create must refuse (SS_EUNSUPPORTED) instead of computing wrong pixels."""
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import OrbPipeline
+    w, h = 752, 480
+    frames = synth.make_frames(w, h, 2, cfg=17)
+    for sf, L in ((1.05, 8), (1.3, 6), (1.33, 5)):
+        pipe = OrbPipeline(w, h, 300, L, scale_factor=sf, max_frames=2)
+        pipe.extract(_upload(torch, frames))
+        torch.cuda.synchronize()
+        p = ref.params(w, h, 300, n_levels=L, scale_factor=sf)
+        for b in range(2):
+            want = ref.pyramid(p, frames[b])
+            for l in range(1, L):
+                ptr, pitch = ss.ss_debug_level(pipe.ctx, b, l)
+                lw, lh = p.level_w[l], p.level_h[l]
+                got = _d2h(ptr, lh * pitch).reshape(lh, pitch)[:, :lw]
+                np.testing.assert_array_equal(got, want[l], err_msg=f"scale {sf} frame {b} level {l}")
+        pipe.close()
+    with pytest.raises(ss.SSError) as ei:
+        OrbPipeline(w, h, 300, 4, scale_factor=1.5, max_frames=1)
+    assert ei.value.status == ss.SS_EUNSUPPORTED
 
 
 @pytest.mark.parametrize("shape", ["euroc", "tum", "kitti"])
