@@ -72,10 +72,20 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
   extern __shared__ __align__(16) uint8_t sm[];  // DESC_WARPS * PER_WARP
   __shared__ int8_t pat[1024];
   __shared__ int off[kMaxLevels + 1];
+  __shared__ __align__(16) uint32_t s_wmask[16 * 8], s_wu[16 * 8];  // per |v|: 32 byte weights
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int f = blockIdx.y;
   const int L = g.L;
   for (int i = threadIdx.x; i < 1024; i += blockDim.x) pat[i] = pattern[i];
+  if (threadIdx.x < 256) {  // byte j = u + 15 of row |v|: inside the disk -> (1, u + 15), else 0
+    const int t = threadIdx.x >> 7, av = (threadIdx.x >> 3) & 15, k = threadIdx.x & 7;
+    uint32_t word = 0;
+    for (int b = 0; b < 4; b++) {
+      const int j = 4 * k + b, u = j - 15;
+      if (j <= 30 && u >= -c_umax[av] && u <= c_umax[av]) word |= (uint32_t)(t ? j : 1) << (8 * b);
+    }
+    (t ? s_wu : s_wmask)[(threadIdx.x & 127)] = word;
+  }
   if (threadIdx.x == 0) {
     int s = 0;
     off[0] = 0;
@@ -124,19 +134,34 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
     P = Pw;
   }
   __syncwarp();
-  // moments over the disk |u| <= umax[|v|] (always inside the level: 19 <= lx < w-19)
+  // moments over the disk |u| <= umax[|v|] (always inside the level: 19 <= lx < w-19):
+  // lane = row v; the row's 31 pixels (plus one zero-weight byte) as 8 words, dotted 4 bytes
+  // at a time with the disk mask (S0 = sum I) and with weights u + 15 (S1); m10 = sum of
+  // S1 - 15 S0, m01 = sum of v S0
   int m10 = 0, m01 = 0;
   {
-    const int u = lane - 15;
     if (lane < 31) {
-      for (int v = -15; v <= 15; v++) {
-        const int um = c_umax[v < 0 ? -v : v];
-        if (u >= -um && u <= um) {
-          const int I = P[(21 + v) * PP + 21 + u];
-          m10 += u * I;
-          m01 += v * I;
-        }
+      const int v = lane - 15, av = v < 0 ? -v : v;
+      const uint8_t* rp = P + (21 + v) * PP + 6;  // column u = -15
+      const uint32_t* wa = reinterpret_cast<const uint32_t*>(reinterpret_cast<uintptr_t>(rp) & ~(uintptr_t)3);
+      const uint32_t shb = 8u * (uint32_t)(reinterpret_cast<uintptr_t>(rp) & 3);
+      const uint4* wm = reinterpret_cast<const uint4*>(s_wmask + 8 * av);
+      const uint4* wu = reinterpret_cast<const uint4*>(s_wu + 8 * av);
+      const uint4 m0 = wm[0], m1 = wm[1], u0 = wu[0], u1 = wu[1];
+      const uint32_t mk[8] = {m0.x, m0.y, m0.z, m0.w, m1.x, m1.y, m1.z, m1.w};
+      const uint32_t uk[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
+      uint32_t w[9];
+#pragma unroll
+      for (int k = 0; k < 9; k++) w[k] = wa[k];
+      unsigned s0 = 0, s1 = 0;
+#pragma unroll
+      for (int k = 0; k < 8; k++) {
+        const uint32_t x = __funnelshift_r(w[k], w[k + 1], shb);
+        s0 = __dp4a(x, mk[k], s0);
+        s1 = __dp4a(x, uk[k], s1);
       }
+      m10 = (int)s1 - 15 * (int)s0;
+      m01 = v * (int)s0;
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
@@ -149,13 +174,12 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
   // then B[r][c] = (sum_j k_j V[r][c + j] + 2^15) >> 16 at the sample points (below)
   // pass 1 on packed column pairs: lane covers columns 2*lane, 2*lane + 1 as two 16-bit lanes
   // of one register (a weighted sum is <= 255 * 256, so the halves never carry)
-  if (lane < (PR + 1) / 2) {
-    const uint16_t* pc = reinterpret_cast<const uint16_t*>(P - (reinterpret_cast<uintptr_t>(P) & 1)) + lane;
-    const int odd = (int)(reinterpret_cast<uintptr_t>(P) & 1);
-    auto ld2 = [&](int r) -> uint32_t {  // bytes (r, 2 lane), (r, 2 lane + 1) -> (lo16, hi16)
-      if (!odd) return __byte_perm((uint32_t)pc[r * (PP / 2)], 0, 0x7170);
-      const uint32_t w = (uint32_t)pc[r * (PP / 2)] | ((uint32_t)pc[r * (PP / 2) + 1] << 16);
-      return __byte_perm(w, 0, 0x7271);
+  // column pairs start at an even address: V column x' holds patch column x' - podd
+  const int podd = (int)(reinterpret_cast<uintptr_t>(P) & 1);
+  if (lane < (PR + 2) / 2) {
+    const uint16_t* pc = reinterpret_cast<const uint16_t*>(P - podd) + lane;
+    auto ld2 = [&](int r) -> uint32_t {  // bytes (r, 2 lane - podd), (r, 2 lane + 1 - podd) -> (lo16, hi16)
+      return __byte_perm((uint32_t)pc[r * (PP / 2)], 0, 0x7170);
     };
     uint32_t q0 = ld2(0), q1 = ld2(1), q2 = ld2(2), q3 = ld2(3), q4 = ld2(4), q5 = ld2(5);
     uint32_t* V32 = reinterpret_cast<uint32_t*>(V) + lane;
@@ -186,7 +210,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
         ox = rhe_rot(px, -py, cs, sn, m10, m01, r2);  // (px m10 - py m01) / r
         oy = rhe_rot(px, py, sn, cs, m01, m10, r2);   // (px m01 + py m10) / r
       }
-      const uint16_t* vr = V + (18 + oy) * VP + 18 + ox;
+      const uint16_t* vr = V + (18 + oy) * VP + 18 + ox + podd;
       const int sum = 18 * (vr[0] + vr[6]) + 34 * (vr[1] + vr[5]) + 48 * (vr[2] + vr[4]) + 56 * vr[3];
       v[e] = (sum + (1 << 15)) >> 16;
     }
@@ -197,10 +221,10 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
   if (lane == 0) {
     float ang = 0.f;
     if (m10 != 0 || m01 != 0) {
-      double a = atan2((double)m01, (double)m10) * (180.0 / 3.14159265358979323846);
-      if (a < 0) a += 360.0;
-      ang = (float)a;
-      if (ang >= 360.0f) ang = 0.0f;
+      // f32 atan2 of exactly representable moments: |error| < 1e-6 rad (budget 1e-4)
+      float a = atan2f((float)m01, (float)m10) * 57.29577951308232f;
+      if (a < 0.f) a += 360.0f;
+      ang = a >= 360.0f ? 0.0f : a;
     }
     ss_keypoint kp;
     kp.x = __fmul_rn((float)lx, g.scale[l]);
