@@ -297,14 +297,27 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   g.pyr_frame_bytes = poff;
   g.total_cells = (int)c->cells_h.size();
   // FAST work units: runs of <= kSegCells consecutive cells of one row (same level and detect
-  // rows; their windows tile [x0, x1)), biggest levels first in the grid
+  // rows; their windows tile [x0, x1)), biggest levels first in the grid.  8 measured best
+  // on B200 (c2: 2..24 swept; smaller runs pay more halo, larger ones lose parallelism).
   const int kSegCells = 8;
   g.max_band_w = g.max_band_h = g.max_cell_w = 0;
+  // a row of n cells is cut into nseg = ceil(n / S) near-equal runs: cell k of the row goes
+  // to run floor(k * nseg / n)
+  std::vector<int> run_of(c->cells_h.size());
+  for (size_t r0 = 0; r0 < c->cells_h.size();) {
+    size_t r1 = r0;
+    while (r1 < c->cells_h.size() && c->cells_h[r1].level == c->cells_h[r0].level && c->cells_h[r1].y0 == c->cells_h[r0].y0)
+      r1++;
+    const int n = (int)(r1 - r0), S = kSegCells;
+    const int nseg = (n + S - 1) / S;
+    for (int k = 0; k < n; k++) run_of[r0 + k] = (int)((int64_t)k * nseg / n);
+    r0 = r1;
+  }
   for (size_t i = 0; i < c->cells_h.size(); i++) {
     const CellInfo& ci = c->cells_h[i];
     g.max_cell_w = imax(g.max_cell_w, ci.x1 - ci.x0);
     if (c->bands_h.empty() || c->bands_h.back().level != ci.level || c->bands_h.back().y0 != ci.y0 ||
-        c->bands_h.back().ncells == kSegCells) {
+        run_of[i] != run_of[i - 1]) {
       BandInfo b;
       b.level = ci.level;
       b.y0 = ci.y0;
