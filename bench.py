@@ -159,9 +159,12 @@ def measured_peaks() -> dict:
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
             d = json.load(f)
-        return {"hbm_gbs": float(d["hbm_gbs"]), "src": "measured (MEASURED_PEAKS.json)"}
+        return {"hbm_gbs": float(d["hbm_gbs"]), "src": "measured (MEASURED_PEAKS.json)",
+                "i8_tops": 2.0 * float(d["bf16_tflops"]),
+                "tc_src": "measured bf16 dense (MEASURED_PEAKS.json) x 2 (nominal int8:bf16 ratio, 4.5:2.25 POPS)"}
     except Exception:
-        return {"hbm_gbs": 6650.0, "src": "fallback (B200_PROFILING.md)"}
+        return {"hbm_gbs": 6650.0, "src": "fallback (B200_PROFILING.md)", "i8_tops": 4500.0,
+                "tc_src": "nominal int8 dense 4.5 POPS (fallback)"}
 
 
 # ----------------------------------------------------------------------------- algorithmic work
@@ -192,8 +195,11 @@ def kernel_work(name: str, p, B: int, cand_l: list, kps_l: list, nq: int, n_map:
         return "hbm", float(nq * 64)
     if name == "match_resolve":
         return "hbm", float(nq * 12)
-    if name == "brute_partial":
-        return "popc", float(sum(kps_l)) * n_map  # distances
+    if name == "brute_tc":  # s8 +-1 dot products on tcgen05: 2 x 256 ops per distance
+        return "tensor", float(sum(kps_l)) * n_map * 512.0
+    if name == "brute_expand":  # packed descriptors read (32 B/row), expanded s8 rows written (256 B/row)
+        slots = B * p.kp_capacity
+        return "hbm", float((slots + n_map) * (32 + 256))
     return "hbm", 0.0
 
 
@@ -423,12 +429,12 @@ def run_ours(args, cfg):
                 "frac": achieved / ALU_PEAK_TOPS, "traffic": None, "kernel": dom,
                 "peak_src": "derived: 148 SM x 64 ALU lanes/clk x 1.965 GHz (DESIGN.md §6)",
                 "work": f"{FAST_OPS_PER_PX} ops per detect pixel", "share_of_step": step_share}
-    else:
-        popc_peak = 148 * 16 * 1.965 / 8  # Gdist/s at the 1965 MHz max SM clock
-        achieved = work / (avg_us[dom] * 1e-6) / 1e9
-        roof = {"bound": "alu", "achieved": achieved, "peak": popc_peak, "unit": "Gdist/s",
-                "frac": achieved / popc_peak, "traffic": None, "kernel": dom,
-                "peak_src": "derived: 148 SM x 16 POPC/clk x clock / 8 POPC per distance", "share_of_step": step_share}
+    else:  # tensor: int8 dense peak = measured bf16 dense x 2 (the guide's nominal i8 : bf16 ratio)
+        achieved = work / (avg_us[dom] * 1e-6) / 1e12
+        roof = {"bound": "tensor", "achieved": achieved, "peak": peaks["i8_tops"], "unit": "TOPS",
+                "frac": achieved / peaks["i8_tops"], "traffic": None, "kernel": dom, "peak_src": peaks["tc_src"],
+                "work": "512 int8 ops per keypoint x map distance (256-long +-1 dot product)",
+                "share_of_step": step_share}
     traffic_file = os.path.join(ROOT, "profiles", "dram_traffic_r01.json")
     if os.path.exists(traffic_file):
         try:

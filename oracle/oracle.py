@@ -55,6 +55,12 @@ KEYPOINT_DTYPE = np.dtype([("x", "<f4"), ("y", "<f4"), ("angle_deg", "<f4"), ("l
 QUERY_DTYPE = np.dtype([("frame", "<i4"), ("u", "<f4"), ("v", "<f4"), ("pred_level", "<i4"),
                         ("radius", "<f4")])
 MATCH_DTYPE = np.dtype([("idx", "<i4"), ("dist", "<i4"), ("dist2", "<i4")])
+CAMERA_DTYPE = np.dtype([("R", "<f4", (9,)), ("t", "<f4", (3,)), ("ow", "<f4", (3,)), ("fx", "<f4"),
+                         ("fy", "<f4"), ("cx", "<f4"), ("cy", "<f4"), ("min_x", "<f4"), ("max_x", "<f4"),
+                         ("min_y", "<f4"), ("max_y", "<f4"), ("pad", "<f4")])
+MAP_POINT_DTYPE = np.dtype([("pos", "<f4", (3,)), ("normal", "<f4", (3,)), ("min_dist", "<f4"),
+                            ("max_dist", "<f4")])
+assert CAMERA_DTYPE.itemsize == 96 and MAP_POINT_DTYPE.itemsize == 32
 assert KEYPOINT_DTYPE.itemsize == 20 and QUERY_DTYPE.itemsize == 20 and MATCH_DTYPE.itemsize == 12
 
 _lib = None
@@ -88,6 +94,7 @@ def lib():
                                           C.c_int, C.c_int, C.c_int, C.c_int, P]
         _lib.ref_match_brute.argtypes = [C.POINTER(RefParams), C.c_int, P, P, C.c_int, P, C.c_int,
                                          C.c_int, C.c_int, C.c_int, C.c_int, P]
+        _lib.ref_project_points.argtypes = [C.POINTER(RefParams), C.c_int, P, C.c_int, P, P, C.c_float, P]
     return _lib
 
 
@@ -239,4 +246,15 @@ def match_brute(p: RefParams, desc, counts, map_desc, th=50, ratio_num=3, ratio_
     k1 = p.kp_capacity if k1 is None else k1
     lib().ref_match_brute(C.byref(p), F, _p(desc), _p(counts), len(map_desc), _p(map_desc), th,
                           ratio_num, ratio_den, k0, k1, _p(out))
+    return out
+
+
+def project_points(p: RefParams, cams, points, point_frame, th=1.0):
+    """O11: -> QUERY_DTYPE [n_points] (pred_level -1 / radius 0 = outside the frustum)."""
+    cams = np.ascontiguousarray(cams, dtype=CAMERA_DTYPE)
+    points = np.ascontiguousarray(points, dtype=MAP_POINT_DTYPE)
+    point_frame = np.ascontiguousarray(point_frame, dtype=np.int32)
+    out = np.zeros(len(points), QUERY_DTYPE)
+    lib().ref_project_points(C.byref(p), len(cams), _p(cams), len(points), _p(points), _p(point_frame),
+                             float(th), _p(out))
     return out

@@ -23,6 +23,10 @@
  *   O6 blur        : cv2.GaussianBlur(7x7, sigma 2, REFLECT_101)
  *   O7 descriptor  : rot90 invariance (bit-exact); unrotated case = pattern lookups
  *   O9/O10 match   : brute-force definitions in Python on small inputs
+ *   O11 projection : cv2.projectPoints (f64) on random poses; closed forms (optical axis,
+ *                    rot90 about z, viewCos = 1 along the normal); predicted level vs
+ *                    ceil(log(ratio)/log(1.2)) away from level boundaries; each culling
+ *                    rule isolated by a point that violates only it
  */
 #include "ss_oracle.h"
 
@@ -651,5 +655,54 @@ void ref_match_brute(const ref_params* p, int F, const uint8_t* desc, const int3
       o->dist = d1; o->dist2 = d2;
       if (m1 >= 0 && d1 <= th && den * d1 < num * d2) o->idx = m1;
     }
+  }
+}
+
+/* --------------------------------------------------------- O11 projection */
+/* ORB-SLAM3 Frame::isInFrustum + MapPoint::PredictScale + ORBmatcher::RadiusByViewingCos
+ * [ext]: the per-map-point step of "search local points" (§4.2.1) before the
+ * windowed match (O9).  f32 throughout, every operation rounded once in the order written
+ * (built with -ffp-contract=off; sums left to right).  Readings (DESIGN.md §3 item 11):
+ * the predicted level is the smallest n in [0, L-1] with ratio <= scale[n] (the f32 scale
+ * chain of O0), i.e. ceil(log(ratio)/log(sf)) clamped, decided by comparisons instead of a
+ * libm log; radius = f32(f32(rv * th) * scale[level]) with rv = 2.5 if viewCos > 0.998
+ * else 4.0; viewing-cosine limit 0.5; distance gate [0.8*min_dist, 1.2*max_dist]. */
+static float dot3(const float* a, const float* b) {
+  float s = a[0] * b[0];
+  s = s + a[1] * b[1];
+  s = s + a[2] * b[2];
+  return s;
+}
+
+void ref_project_points(const ref_params* p, int F, const ref_camera* cams, int n, const ref_map_point* pts,
+                        const int32_t* point_frame, float th, ref_query* out) {
+  int L = p->n_levels;
+  for (int i = 0; i < n; i++) {
+    ref_query* o = &out[i];
+    int f = point_frame[i];
+    o->frame = f; o->u = 0.0f; o->v = 0.0f; o->pred_level = -1; o->radius = 0.0f;
+    if (f < 0 || f >= F) continue;
+    const ref_camera* c = &cams[f];
+    const float* P = pts[i].pos;
+    float pc[3];
+    for (int r = 0; r < 3; r++) pc[r] = dot3(&c->R[3 * r], P) + c->t[r];
+    if (pc[2] < 0.0f) continue;                          /* behind the camera */
+    float u = c->fx * pc[0] / pc[2] + c->cx;              /* Pinhole::project */
+    float v = c->fy * pc[1] / pc[2] + c->cy;
+    if (u < c->min_x || u > c->max_x) continue;
+    if (v < c->min_y || v > c->max_y) continue;
+    float po[3] = {P[0] - c->ow[0], P[1] - c->ow[1], P[2] - c->ow[2]};
+    float dist = sqrtf(dot3(po, po));
+    float min_d = 0.8f * pts[i].min_dist, max_d = 1.2f * pts[i].max_dist;
+    if (dist < min_d || dist > max_d) continue;
+    float view_cos = dot3(po, pts[i].normal) / dist;
+    if (view_cos < 0.5f) continue;
+    float ratio = pts[i].max_dist / dist;                 /* PredictScale */
+    int level = L - 1;
+    for (int l = 0; l < L; l++)
+      if (ratio <= p->scale[l]) { level = l; break; }
+    float rv = view_cos > 0.998f ? 2.5f : 4.0f;           /* RadiusByViewingCos */
+    float r = rv * th;
+    o->u = u; o->v = v; o->pred_level = level; o->radius = r * p->scale[level];
   }
 }

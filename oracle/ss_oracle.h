@@ -85,6 +85,23 @@ void ref_match_brute(const ref_params* p, int n_frames, const uint8_t* desc, con
                      int n_map, const uint8_t* map_desc, int th, int ratio_num, int ratio_den,
                      int k0, int k1, ref_match* out);
 
+/* O11 (S9's input): local-map point -> frame projection ("isInFrustum").
+ * Camera: Pc = R*Pw + t (R row-major), pinhole fx, fy, cx, cy, bounds [min_x, max_x] x
+ * [min_y, max_y], camera centre ow.  96 bytes, same layout as ss_camera. */
+typedef struct {
+  float R[9], t[3], ow[3];
+  float fx, fy, cx, cy;
+  float min_x, max_x, min_y, max_y;
+  float pad;
+} ref_camera;
+/* 32 bytes, same layout as ss_map_point: world position, unit mean viewing direction,
+ * ORB-SLAM mfMinDistance / mfMaxDistance (scale-invariance distances). */
+typedef struct { float pos[3], normal[3], min_dist, max_dist; } ref_map_point;
+/* out[i]: frame = point_frame[i]; u, v, pred_level, radius when point i is in frame
+ * point_frame[i]'s frustum, else pred_level = -1, radius = 0, u = v = 0 (never matches). */
+void ref_project_points(const ref_params* p, int n_frames, const ref_camera* cams, int n_points,
+                        const ref_map_point* pts, const int32_t* point_frame, float th, ref_query* out);
+
 #ifdef __cplusplus
 }
 #endif

@@ -9,8 +9,8 @@
 // (distance << 32 | index) top-2 by shuffles, i.e. top-2 by (distance, index); ORB-SLAM's
 // accept rule; a keypoint claimed by several accepted
 // queries keeps the min (distance, query) (atomicMin on packed u64, then a resolve pass).
-// BRUTE: map tiles staged in shared memory, one thread per frame keypoint keeps a packed
-// (distance << 32 | map index) top-2 per map split; a merge kernel takes the two smallest.
+// BRUTE: the per-split partial top-2 comes from the tensor-core kernel (k_brute_tc.cu);
+// match_brute_merge takes the two smallest (distance << 32 | map index) and applies the rule.
 #include "ss_internal.h"
 
 namespace ss {
@@ -157,58 +157,6 @@ __global__ void __launch_bounds__(256) match_window_resolve(int nq, const ss_mp_
   if (claim[(int64_t)q[qi].frame * cap + m.idx] != mine) out[qi].idx = -1;
 }
 
-constexpr int BQ = 128;    // keypoints per CTA (one per thread)
-constexpr int BTILE = 256;  // map descriptors per shared-memory tile
-
-__global__ void __launch_bounds__(BQ) match_brute_partial(Geom g, int F, const uint8_t* __restrict__ desc,
-                                                          const int32_t* __restrict__ counts, int n_map,
-                                                          const uint8_t* __restrict__ map_desc, int splits,
-                                                          unsigned long long* __restrict__ partial) {
-  pdl_wait();
-  pdl_trigger();
-  __shared__ uint4 tile[BTILE * 2];
-  const int cap = g.kp_capacity, L = g.L;
-  const int gq = blockIdx.x * BQ + threadIdx.x;  // global keypoint slot f*cap + k
-  const int split = blockIdx.y;
-  const int per = (n_map + splits - 1) / splits;
-  const int m0 = split * per, m1 = min(n_map, m0 + per);
-  bool valid = false;
-  uint4 a0 = make_uint4(0, 0, 0, 0), a1 = a0;
-  if (gq < F * cap) {
-    const int f = gq / cap, k = gq - f * cap;
-    valid = k < counts[f * (L + 1) + L];
-    if (valid) {
-      const uint4* p = reinterpret_cast<const uint4*>(desc + (int64_t)gq * SS_DESC_BYTES);
-      a0 = p[0];
-      a1 = p[1];
-    }
-  }
-  unsigned long long b1 = ~0ull, b2 = ~0ull;
-  for (int t0 = m0; t0 < m1; t0 += BTILE) {
-    const int nt = min(BTILE, m1 - t0);
-    __syncthreads();
-    const uint4* src = reinterpret_cast<const uint4*>(map_desc + (int64_t)t0 * SS_DESC_BYTES);
-    for (int i = threadIdx.x; i < nt * 2; i += BQ) tile[i] = src[i];
-    __syncthreads();
-    if (valid) {
-      for (int j = 0; j < nt; j++) {
-        const int d = hamming256(a0, a1, tile[2 * j], tile[2 * j + 1]);
-        const unsigned long long key = ((unsigned long long)d << 32) | (unsigned)(t0 + j);
-        if (key < b1) {
-          b2 = b1;
-          b1 = key;
-        } else if (key < b2) {
-          b2 = key;
-        }
-      }
-    }
-  }
-  if (gq < F * cap) {
-    partial[((int64_t)gq * splits + split) * 2] = b1;
-    partial[((int64_t)gq * splits + split) * 2 + 1] = b2;
-  }
-}
-
 __global__ void __launch_bounds__(256) match_brute_merge(Geom g, int F, const int32_t* __restrict__ counts,
                                                          int splits, const unsigned long long* __restrict__ partial,
                                                          ss_match_cfg cfg, ss_match* __restrict__ out) {
@@ -273,23 +221,6 @@ cudaError_t launch_match_resolve(const Geom& g, int n_queries, const ss_mp_query
   cudaError_t e = launch_pdl(match_window_resolve, dim3((n_queries + 255) / 256), dim3(256), 0, s, n_queries, q,
                              g.kp_capacity, (const unsigned long long*)claim, out);
   return e != cudaSuccess ? e : cudaGetLastError();
-}
-
-int brute_splits(const Geom& g, int n_frames, int n_map, int max_splits) {
-  const int nslots = n_frames * g.kp_capacity;
-  const int qblocks = (nslots + BQ - 1) / BQ;
-  // enough CTAs for ~4 waves on 148 SMs, each split >= one tile
-  int splits = (4 * 148 + qblocks - 1) / qblocks;
-  splits = max(1, min(splits, max_splits));
-  return max(1, min(splits, (n_map + BTILE - 1) / BTILE));
-}
-
-cudaError_t launch_brute_partial(const Geom& g, int n_frames, const uint8_t* desc, const int32_t* counts, int n_map,
-                                 const uint8_t* map_desc, int splits, unsigned long long* partial, cudaStream_t s) {
-  const int nslots = n_frames * g.kp_capacity;
-  dim3 grid((nslots + BQ - 1) / BQ, splits);
-  match_brute_partial<<<grid, BQ, 0, s>>>(g, n_frames, desc, counts, n_map, map_desc, splits, partial);
-  return cudaGetLastError();
 }
 
 cudaError_t launch_brute_merge(const Geom& g, int n_frames, const int32_t* counts, int splits,

@@ -6,6 +6,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -143,6 +144,9 @@ struct ss_ctx {
   uint16_t* rowidx = nullptr;  // WINDOW matcher: first keypoint per (frame, level, row)
   uint64_t* phase_ts = nullptr;  // distribution phase timestamps [max_frames][L][16] (debug hook)
   unsigned long long* partial = nullptr;
+  int8_t* brute_qexp = nullptr;  // BRUTE: keypoint descriptors expanded to s8 +-1 (k_brute_tc.cu)
+  int8_t* brute_mexp = nullptr;  // BRUTE: map descriptors expanded to s8 +-1
+  int n_sm = 148;
   // per-extract DAG: level 0's FAST + distribution on side stream 0 right away; level l >= 1's
   // on side stream 1 + (l % kSideLevel) as soon as the pyramid (caller's stream) has level l
   static constexpr int kSide = 4, kSideLevel = 3;
@@ -178,7 +182,8 @@ void free_ctx(ss_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->device);
   void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr_plan, c->pyr_gtab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
-                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->rowidx, c->phase_ts};
+                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->rowidx, c->phase_ts,
+                  c->brute_qexp, c->brute_mexp};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
@@ -402,7 +407,11 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     ob += distribute_ovf_bytes(g.level_slots[l]);
   }
   c->ovf_frame_bytes = ob;
-  c->max_splits = 16;
+  c->max_splits = 64;
+  {
+    int nsm = 0;
+    if (cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, device) == cudaSuccess && nsm > 0) c->n_sm = nsm;
+  }
   std::vector<int8_t> pat(1024);
   const int* ph = brief_pattern_host();
   for (int i = 0; i < 1024; i++) pat[i] = (int8_t)ph[i];
@@ -427,7 +436,11 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->claim, sizeof(unsigned long long) * F * g.kp_capacity);
   ALLOC(c->rowidx, sizeof(uint16_t) * F * match_rows_per_frame(g));
   ALLOC(c->phase_ts, sizeof(uint64_t) * F * L * 16);
-  if (max_map > 0) ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
+  if (max_map > 0) {
+    ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
+    ALLOC(c->brute_qexp, brute_tc_query_bytes(F * g.kp_capacity));
+    ALLOC(c->brute_mexp, brute_tc_map_bytes(max_map));
+  }
 #undef ALLOC
   if (e == cudaSuccess) e = cudaMemcpy(c->cells, c->cells_h.data(), sizeof(CellInfo) * c->cells_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->bands, c->bands_h.data(), sizeof(BandInfo) * c->bands_h.size(), cudaMemcpyHostToDevice);
@@ -556,9 +569,13 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
     if (n_map > c->max_map) return fail(SS_ECAPACITY, "n_map exceeds the ctx's max_map");
     if (n_map > 0 && !d_map_desc) return fail(SS_EINVAL, "NULL map");
     if (n_frames == 0) return SS_OK;
-    const int splits = brute_splits(c->g, n_frames, n_map, c->max_splits);
+    const int n_slots = n_frames * c->g.kp_capacity;
+    const int splits = brute_tc_splits(n_slots, n_map, c->max_splits, c->n_sm);
     prof_mark(c, s);
-    SS_CUDA_TRY(launch_brute_partial(c->g, n_frames, d_desc, d_counts, n_map, d_map_desc, splits, c->partial, s));
+    SS_CUDA_TRY(launch_brute_expand(n_slots, d_desc, n_map, d_map_desc, c->brute_qexp, c->brute_mexp, s));
+    prof_mark(c, s);
+    prof_mark(c, s);
+    SS_CUDA_TRY(launch_brute_tc(n_slots, n_map, c->brute_qexp, c->brute_mexp, splits, c->partial, s));
     prof_mark(c, s);
     prof_mark(c, s);
     SS_CUDA_TRY(launch_brute_merge(c->g, n_frames, d_counts, splits, c->partial, *cfg, d_out, s));

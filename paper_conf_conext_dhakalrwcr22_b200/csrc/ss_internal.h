@@ -161,13 +161,19 @@ cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* 
                                 cudaStream_t s);
 cudaError_t launch_match_resolve(const Geom& g, int n_queries, const ss_mp_query* q,
                                  const unsigned long long* claim, ss_match* out, cudaStream_t s);
-int brute_splits(const Geom& g, int n_frames, int n_map, int max_splits);
-cudaError_t launch_brute_partial(const Geom& g, int n_frames, const uint8_t* desc, const int32_t* counts,
-                                 int n_map, const uint8_t* map_desc, int splits, unsigned long long* partial,
-                                 cudaStream_t s);
 cudaError_t launch_brute_merge(const Geom& g, int n_frames, const int32_t* counts, int splits,
                                const unsigned long long* partial, ss_match_cfg cfg, ss_match* out,
                                cudaStream_t s);
+// Tensor-core brute matcher (k_brute_tc.cu): expanded-operand scratch sizes, the map split
+// count (whole waves of one CTA per SM), and expand + tcgen05 partial top-2 (per-split partial
+// top-2, reduced by launch_brute_merge).
+int64_t brute_tc_query_bytes(int64_t n_slots);
+int64_t brute_tc_map_bytes(int64_t n_map);
+int brute_tc_splits(int n_slots, int n_map, int max_splits, int n_sm);
+cudaError_t launch_brute_expand(int n_slots, const uint8_t* desc, int n_map, const uint8_t* map_desc, int8_t* qexp,
+                                int8_t* mexp, cudaStream_t s);
+cudaError_t launch_brute_tc(int n_slots, int n_map, const int8_t* qexp, const int8_t* mexp, int splits,
+                            unsigned long long* partial, cudaStream_t s);
 
 // Overflow scratch bytes the distribution needs for a level with `slots` candidate slots.
 int64_t distribute_ovf_bytes(int64_t slots);

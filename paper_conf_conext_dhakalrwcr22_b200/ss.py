@@ -184,7 +184,7 @@ def extract_events(n_levels: int) -> int:
 
 def match_kernels(mode: int, dedup: bool = True) -> list[str]:
     if mode == SS_MATCH_BRUTE:
-        return ["brute_partial", "brute_merge"]
+        return ["brute_expand", "brute_tc", "brute_merge"]
     return ["match_prepare", "match_window"] + (["match_resolve"] if dedup else [])
 
 

@@ -17,7 +17,7 @@ METRICS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.
            "lts__t_sectors.sum"]
 SHORT = {"fast_bands_kernel": "fast", "distribute_kernel": "distribute", "pyramid_fused_kernel": "pyramid",
          "describe_kernel": "describe", "match_prepare": "match_prepare", "match_window_kernel": "match_window",
-         "match_window_resolve": "match_resolve", "match_brute_partial": "brute_partial",
+         "match_window_resolve": "match_resolve", "brute_tc_kernel": "brute_tc", "brute_expand_kernel": "brute_expand",
          "match_brute_merge": "brute_merge"}
 
 
