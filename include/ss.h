@@ -82,6 +82,25 @@ typedef struct {
   float radius;
 } ss_mp_query;
 
+/* A camera pose + pinhole intrinsics for ss_project_points (DESIGN.md §3 O11), 96 bytes:
+ * camera coordinates Pc = R * Pw + t (R row-major), camera centre ow = -R^T t (given, not
+ * recomputed), projection u = fx * Pc.x / Pc.z + cx, v = fy * Pc.y / Pc.z + cy, image bounds
+ * [min_x, max_x] x [min_y, max_y] (ORB-SLAM mnMinX..mnMaxY, level-0 px). */
+typedef struct {
+  float R[9], t[3], ow[3];
+  float fx, fy, cx, cy;
+  float min_x, max_x, min_y, max_y;
+  float pad;
+} ss_camera;
+
+/* A local-map point for ss_project_points (O11), 32 bytes: world position, unit mean viewing
+ * direction (ORB-SLAM mNormalVector), scale-invariance distances mfMinDistance /
+ * mfMaxDistance. */
+typedef struct {
+  float pos[3], normal[3];
+  float min_dist, max_dist;
+} ss_map_point;
+
 /* A match: idx = keypoint index within its frame (WINDOW) or map index (BRUTE), -1 = none;
  * dist / dist2 = best / second-best Hamming distance over the candidates (256 = none). */
 typedef struct {
@@ -151,6 +170,23 @@ ss_status ss_match_projection(ss_ctx* ctx, int32_t n_frames, const ss_keypoint* 
                               const ss_mp_query* d_queries, const uint8_t* d_map_desc, int32_t n_map,
                               const ss_match_cfg* cfg, ss_match* d_out, ss_stream_t stream);
 
+/* O11: the per-map-point half of "search local points" (ORB-SLAM3
+ * Frame::isInFrustum + MapPoint::PredictScale + ORBmatcher::RadiusByViewingCos): map point
+ * i is tested against the camera of frame d_point_frame[i] and written as WINDOW query i.
+ * Device pointers: d_cams [n_frames] ss_camera, d_points [n_points] ss_map_point,
+ * d_point_frame [n_points] i32, d_queries [n_points] ss_mp_query (output).  In the frustum
+ * (Pc.z >= 0, u, v inside the bounds, 0.8*min_dist <= |Pw - ow| <= 1.2*max_dist, viewing
+ * cosine >= 0.5): {frame, u, v, level, radius} with level = the smallest n in [0, L-1]
+ * with max_dist / dist <= scale[n] (else L-1) and radius = f32(f32(rv * th) * scale[level]),
+ * rv = 2.5 if the viewing cosine > 0.998 else 4.0.  Otherwise (or a frame index outside
+ * [0, n_frames)) {frame, 0, 0, -1, 0}, which ss_match_projection never matches.  Every f32
+ * operation is rounded once in the documented order (no contraction): bit-exact with the
+ * oracle.  The map points' descriptors are the queries' descriptors (same index).
+ * SS_EINVAL for negative sizes or NULL buffers with n_points > 0. */
+ss_status ss_project_points(ss_ctx* ctx, int32_t n_frames, const ss_camera* d_cams, int32_t n_points,
+                            const ss_map_point* d_points, const int32_t* d_point_frame, float th,
+                            ss_mp_query* d_queries, ss_stream_t stream);
+
 /* ---- profiling hook (bench.py; does not synchronise) ---- */
 
 /* When n_events > 0, every following ss_orb_extract / ss_match_projection records the
@@ -163,7 +199,8 @@ ss_status ss_match_projection(ss_ctx* ctx, int32_t n_frames, const ss_keypoint* 
  * distribute(levels >= 1), describe -- 13 events (while events are installed the level-0
  * branch runs in line on `stream` instead of on its side stream, so each kernel is timed
  * alone).  WINDOW match: a pair per kernel
- * (match_prepare, match_window[, match_resolve if dedup]); BRUTE: brute_partial, brute_merge.
+ * (match_prepare, match_window[, match_resolve if dedup]); BRUTE: brute_expand, brute_tc,
+ * brute_merge; ss_project_points: project.
  * Works under CUDA-graph stream capture (the records become graph event nodes).
  * *next_index (may be NULL) receives the index of the next event to be recorded. */
 ss_status ss_profile_events(ss_ctx* ctx, void* const* events, int32_t n_events);

@@ -585,6 +585,22 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
   return fail(SS_EINVAL, "unknown match mode");
 }
 
+ss_status ss_project_points(ss_ctx* c, int32_t n_frames, const ss_camera* d_cams, int32_t n_points,
+                            const ss_map_point* d_points, const int32_t* d_point_frame, float th,
+                            ss_mp_query* d_queries, ss_stream_t stream) {
+  if (!c) return fail(SS_EINVAL, "NULL ctx");
+  if (n_frames < 0 || n_points < 0) return fail(SS_EINVAL, "negative size");
+  if (n_points == 0) return SS_OK;
+  if (!d_points || !d_point_frame || !d_queries || (n_frames > 0 && !d_cams)) return fail(SS_EINVAL, "NULL buffer");
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  SS_CUDA_TRY(check_stream(s));
+  prof_mark(c, s);
+  SS_CUDA_TRY(launch_project(c->g, n_frames, d_cams, n_points, d_points, d_point_frame, th, d_queries, s));
+  prof_mark(c, s);
+  return SS_OK;
+}
+
 ss_status ss_profile_events(ss_ctx* c, void* const* events, int32_t n_events) {
   if (!c || n_events < 0 || (n_events > 0 && !events)) return fail(SS_EINVAL, "bad profiling events");
   for (int i = 0; i < n_events; i++)

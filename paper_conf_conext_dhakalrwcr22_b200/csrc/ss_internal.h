@@ -175,6 +175,10 @@ cudaError_t launch_brute_expand(int n_slots, const uint8_t* desc, int n_map, con
 cudaError_t launch_brute_tc(int n_slots, int n_map, const int8_t* qexp, const int8_t* mexp, int splits,
                             unsigned long long* partial, cudaStream_t s);
 
+// O11 local-map projection (k_project.cu): one thread per map point.
+cudaError_t launch_project(const Geom& g, int n_frames, const ss_camera* cams, int n_points, const ss_map_point* pts,
+                           const int32_t* point_frame, float th, ss_mp_query* out, cudaStream_t s);
+
 // Overflow scratch bytes the distribution needs for a level with `slots` candidate slots.
 int64_t distribute_ovf_bytes(int64_t slots);
 

@@ -68,6 +68,14 @@ class OrbPipeline:
         ss.ss_match_projection(self.ctx, n_frames, self.kps, self.desc, self.counts, None, 0, None, map_desc,
                                map_desc.shape[0], cfg, out, stream)
 
+    def project(self, n_frames: int, cams: torch.Tensor, points: torch.Tensor, point_frame: torch.Tensor,
+                out: torch.Tensor, th: float = 1.0, stream: torch.cuda.Stream | None = None):
+        """O11: cams uint8 [n_frames, 96] (ss_camera), points uint8 [n, 32] (ss_map_point),
+        point_frame int32 [n] -> out uint8 [n, 20] (ss_mp_query), the WINDOW queries."""
+        stream = stream or torch.cuda.current_stream(self.device)
+        n = point_frame.numel()
+        ss.ss_project_points(self.ctx, n_frames, cams, n, points, point_frame, th, out, stream)
+
     # -- host views (synchronising; tests / examples) -------------------------------
     def results(self, n_frames: int):
         torch.cuda.synchronize(self.device)

@@ -58,6 +58,11 @@ KEYPOINT_DTYPE = np.dtype([("x", "<f4"), ("y", "<f4"), ("angle_deg", "<f4"), ("l
 QUERY_DTYPE = np.dtype([("frame", "<i4"), ("u", "<f4"), ("v", "<f4"), ("pred_level", "<i4"),
                         ("radius", "<f4")])
 MATCH_DTYPE = np.dtype([("idx", "<i4"), ("dist", "<i4"), ("dist2", "<i4")])
+CAMERA_DTYPE = np.dtype([("R", "<f4", (9,)), ("t", "<f4", (3,)), ("ow", "<f4", (3,)), ("fx", "<f4"),
+                         ("fy", "<f4"), ("cx", "<f4"), ("cy", "<f4"), ("min_x", "<f4"), ("max_x", "<f4"),
+                         ("min_y", "<f4"), ("max_y", "<f4"), ("pad", "<f4")])
+MAP_POINT_DTYPE = np.dtype([("pos", "<f4", (3,)), ("normal", "<f4", (3,)), ("min_dist", "<f4"),
+                            ("max_dist", "<f4")])
 
 _lib = None
 
@@ -81,6 +86,7 @@ def lib():
         L.ss_last_error.restype = C.c_char_p
         L.ss_orb_extract.argtypes = [P, i32, P, i64, i32, P, P, P, P]
         L.ss_match_projection.argtypes = [P, i32, P, P, P, P, i32, P, P, i32, C.POINTER(ss_match_cfg), P, P]
+        L.ss_project_points.argtypes = [P, i32, P, i32, P, P, C.c_float, P, P]
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
         L.ss_debug_candidates.argtypes = [P, i32, i32, P, P, P, i32, C.POINTER(i32)]
         L.ss_debug_overflow_count.argtypes = [P, C.POINTER(i32)]
@@ -88,6 +94,7 @@ def lib():
         L.ss_debug_phase_times.argtypes = [P, i32, i32, P, i32]
         L.ss_profile_next.argtypes = [P, C.POINTER(i32)]
         for fn in ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_orb_extract", "ss_match_projection",
+                   "ss_project_points",
                    "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
                    "ss_profile_next", "ss_debug_phase_times"):
             getattr(L, fn).restype = C.c_int
@@ -96,7 +103,7 @@ def lib():
 
 
 EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "ss_orb_extract",
-            "ss_match_projection", "ss_profile_events", "ss_profile_next", "ss_debug_level",
+            "ss_match_projection", "ss_project_points", "ss_profile_events", "ss_profile_next", "ss_debug_level",
             "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times")
 
 
@@ -156,6 +163,11 @@ def ss_match_projection(ctx, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_qu
     _check(lib().ss_match_projection(ctx, n_frames, _ptr(d_kps), _ptr(d_desc), _ptr(d_counts),
                                      _ptr(d_kp_taken), n_queries, _ptr(d_queries), _ptr(d_map_desc), n_map,
                                      C.byref(cfg), _ptr(d_out), _stream(stream)), ctx)
+
+
+def ss_project_points(ctx, n_frames, d_cams, n_points, d_points, d_point_frame, th, d_queries, stream=None):
+    _check(lib().ss_project_points(ctx, n_frames, _ptr(d_cams), n_points, _ptr(d_points), _ptr(d_point_frame),
+                                   float(th), _ptr(d_queries), _stream(stream)), ctx)
 
 
 def ss_profile_events(ctx, events) -> None:
