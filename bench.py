@@ -3,8 +3,9 @@
 Contract: ``python bench.py --gpus N --steps K --warmup W`` (torchrun for
 N > 1, one rank per GPU, NCCL) prints ONE JSON line on rank 0.  A step = one tick of the
 configured workload: every client on this rank submits one frame, the frames are ORB-extracted
-(pyramid, FAST, quadtree, orientation, blur, BRIEF) and matched (windowed search-local-points
-or brute force) through the C ABI.  Clients are sharded over ranks (weak scaling); with N > 1
+(pyramid, FAST, quadtree, orientation, blur, BRIEF) and matched -- search local points (each
+client's local-map points projected into its frame, then windowed matching) or brute force --
+through the C ABI.  Clients are sharded over ranks (weak scaling); with N > 1
 per-frame results are gathered to rank 0 (the map owner) over NCCL on a side stream.
 
 ``--impl reference`` times the CPU oracle (oracle/, the checker) on the box's host cores on a
@@ -33,15 +34,15 @@ import synth  # noqa: E402
 METRIC = "batched ORB extract+match frames/sec at 1/2/4/8 B200; per-frame p50 latency ms"
 CONFIGS = {
     "c1": dict(shape="euroc", clients=1, nf=1000, mode="window", queries=5000, th=1.0, map=0,
-               desc="c1: single synthetic 752x480 frame, 8 levels x1.2, 1000 ORB features, windowed match vs 5k map points"),
+               desc="c1: single synthetic 752x480 frame, 8 levels x1.2, 1000 ORB features, search local points vs 5k local-map points (GPU projection + windowed match)"),
     "c2": dict(shape="euroc", clients=4, nf=1000, mode="window", queries=5000, th=1.0, map=0,
                desc="c2: EuRoC-shaped 752x480 mono stream, 4 concurrent clients per GPU, 1000 features/frame, "
-                    "windowed search-local-points vs 5k map points per client"),
+                    "search local points vs 5k local-map points per client (GPU projection + windowed match)"),
     "c3": dict(shape="tum", clients=16, nf=1000, mode="window", queries=50000, th=3.0, map=0,
-               desc="c3: TUM-RGBD-shaped 640x480, 16 clients per GPU, 1000 features, windowed match vs 50k map points"),
+               desc="c3: TUM-RGBD-shaped 640x480, 16 clients per GPU, 1000 features, search local points vs 50k local-map points (projection + windowed match)"),
     "c4": dict(shape="kitti", clients=8, stereo=True, nf=2000, mode="window", queries=10000, th=1.0, map=0,
                desc="c4: KITTI-shaped 1241x376 stereo pairs, 8 clients per GPU, 2000 features/image, "
-                    "windowed match vs 10k map points (left image)"),
+                    "search local points vs 10k local-map points (left image; projection + windowed match)"),
     "c5": dict(shape="euroc", clients=8, nf=1250, mode="brute", queries=0, th=0.0, map=200000,
                desc="c5: EuRoC-shaped clients (8 per GPU, 64 over 8xB200), 1250 features, brute-force Hamming "
                     "vs a 200k shared-map descriptor set"),
@@ -193,6 +194,8 @@ def kernel_work(name: str, p, B: int, cand_l: list, kps_l: list, nq: int, n_map:
         return "hbm", float(sum(kps_l) * (43 * 43 + 4 + 52))
     if name == "match_window":  # query 20 B + descriptor 32 B read, 12 B written
         return "hbm", float(nq * 64)
+    if name == "project":  # map point 32 B + frame index 4 B read, query 20 B written
+        return "hbm", float(nq * 56)
     if name == "match_resolve":
         return "hbm", float(nq * 12)
     if name == "brute_tc":  # s8 +-1 dot products on tcgen05: 2 x 256 ops per distance
@@ -230,7 +233,7 @@ def run_ours(args, cfg):
     cap = p.kp_capacity
     props = torch.cuda.get_device_properties(dev)
     l2 = getattr(props, "L2_cache_size", 126 * 2 ** 20)
-    slot_bytes = B * h * w + (Q * 52 + B * cap if window else 0)
+    slot_bytes = B * h * w + (Q * 68 + B * (cap + 96) if window else 0)
     n_slots = int(min(256, max(4, math.ceil(2 * l2 / slot_bytes))))
     if args.ring:
         n_slots = args.ring
@@ -241,10 +244,14 @@ def run_ours(args, cfg):
     stream = torch.cuda.Stream(dev)
     out_rows = Q if window else B * cap
     out = torch.zeros((max(out_rows, 1), 3), dtype=torch.int32, device=dev)
-    queries = qdesc = taken = map_desc = None
+    cams = points = point_frame = qdesc = taken = map_desc = None
     kp_rng = np.random.default_rng(1234 + rank)
     if window:
-        queries = torch.zeros((n_slots, Q, 20), dtype=torch.uint8, device=dev)
+        # "search local points" inputs per ring slot: a local map per frame (3D points,
+        # projected on the GPU by ss_project_points into the WINDOW queries), descriptors, mask
+        cams = torch.zeros((n_slots, B, 96), dtype=torch.uint8, device=dev)
+        points = torch.zeros((n_slots, Q, 32), dtype=torch.uint8, device=dev)
+        point_frame = torch.zeros((n_slots, Q), dtype=torch.int32, device=dev)
         qdesc = torch.zeros((n_slots, Q, 32), dtype=torch.uint8, device=dev)
         taken = torch.zeros((n_slots, B, cap), dtype=torch.uint8, device=dev)
         q_host = []
@@ -253,19 +260,23 @@ def run_ours(args, cfg):
                 pipe.extract(frames[s], stream=stream)
             stream.synchronize()
             kps, desc, counts = pipe.results(B)
-            sel = list(range(0, B, per_client))  # queries against the left / mono image
-            qq, qd, tk = synth.make_queries(kps[sel], desc[sel], counts[sel], L, np.array(p.scale[:L]),
-                                            np.array(p.n_per_level[:L]), w, h, cfg["queries"], cfg["th"],
-                                            seed=synth.frame_seed(CFG_ID[args.config], 1 << 16 | rank, s),
-                                            query_dtype=ss.QUERY_DTYPE)
-            qq["frame"] = qq["frame"] * per_client
+            sel = list(range(0, B, per_client))  # local maps of the left / mono images
+            cm, pt, pf, qd, tk = synth.make_local_map(kps[sel], desc[sel], counts[sel], L, p.scale_factor,
+                                                      np.array(p.n_per_level[:L]), w, h, cfg["shape"],
+                                                      cfg["queries"],
+                                                      seed=synth.frame_seed(CFG_ID[args.config], 1 << 16 | rank, s))
+            pf = pf * per_client
+            cm_full = np.zeros(B, synth.CAMERA_DTYPE)
+            cm_full[sel] = cm
             tk_full = np.zeros((B, cap), np.uint8)
             tk_full[sel] = tk
-            queries[s] = to_device_records(qq, dev)
+            cams[s] = torch.from_numpy(cm_full.view(np.uint8).reshape(B, 96).copy()).to(dev)
+            points[s] = torch.from_numpy(pt.view(np.uint8).reshape(Q, 32).copy()).to(dev)
+            point_frame[s] = torch.from_numpy(pf).to(dev)
             qdesc[s] = torch.from_numpy(qd).to(dev)
             taken[s] = torch.from_numpy(tk_full).to(dev)
             if s < 16:
-                q_host.append((qq, qd, tk_full))
+                q_host.append((cm_full, pt, pf, qd, tk_full))
     else:
         # shared map: rank 0 builds it from its clients' first-slot keypoints, broadcast once
         with torch.cuda.stream(stream):
@@ -283,11 +294,11 @@ def run_ours(args, cfg):
     # --- one CUDA graph per ring slot (plain, timed) + an instrumented twin whose profiling
     #     events (recorded inside the graph) give every kernel's duration
     mode = ss.SS_MATCH_WINDOW if window else ss.SS_MATCH_BRUTE
-    ek, mk = ss.extract_kernels(L), ss.match_kernels(mode, True)
+    ek, mk = ss.extract_kernels(L), (["project"] if window else []) + ss.match_kernels(mode, True)
     base = ss.extract_events(L)
     kernel_ev = [(n, 1 + 2 * i, 2 + 2 * i) for i, n in enumerate(ek)] + \
                 [(n, base + 2 * j, base + 2 * j + 1) for j, n in enumerate(mk)]
-    n_ev = base + ss.match_events(mode, True)
+    n_ev = base + 2 * len(mk)
     events = [[torch.cuda.Event(enable_timing=True) for _ in range(n_ev)] for _ in range(n_slots)]
     for evs in events:  # torch creates the CUDA event lazily, at its first record
         for e in evs:
@@ -300,6 +311,7 @@ def run_ours(args, cfg):
     pipes = [pipe] + [OrbPipeline(w, h, cfg["nf"], L, max_frames=B, max_queries=max(Q, 1), max_map=cfg["map"],
                                   device=local) for _ in range(P - 1)]
     outs = [out] + [torch.zeros_like(out) for _ in range(P - 1)]
+    qbufs = [torch.zeros((max(Q, 1), 20), dtype=torch.uint8, device=dev) for _ in range(P)]  # projected queries
     streams = [stream] + [torch.cuda.Stream(dev) for _ in range(P - 1)]
     for q in range(1, P):  # first call outside capture (kernel attributes)
         with torch.cuda.stream(streams[q]):
@@ -314,7 +326,8 @@ def run_ours(args, cfg):
         with torch.cuda.graph(g, stream=st):
             pp.extract(frames[s], stream=st)
             if window:
-                pp.match_window(B, queries[s], qdesc[s], ot, taken=taken[s], stream=st)
+                pp.project(B, cams[s], points[s], point_frame[s], qbufs[q], th=cfg["th"], stream=st)
+                pp.match_window(B, qbufs[q], qdesc[s], ot, taken=taken[s], stream=st)
             else:
                 pp.match_brute(B, map_desc, ot, stream=st)
         if prof:
@@ -446,7 +459,7 @@ def run_ours(args, cfg):
             pass
 
     # --- e2e through the public API with host buffers (pinned), copies inside the timed region
-    e2e = run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams)
+    e2e = run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=cfg["th"])
 
     frames_per_step = B * world
     value = frames_per_step * K / (T_max / 1000.0)
@@ -457,7 +470,7 @@ def run_ours(args, cfg):
         "dtype": "u8", "data": "synthetic",
         "config": {"workload": cfg["desc"], "config": args.config, "frames_per_step": frames_per_step,
                    "images_per_step_per_gpu": B, "features_per_image": cfg["nf"],
-                   "queries_per_step_per_gpu": Q if window else 0, "map_size": cfg["map"],
+                   "map_points_per_step_per_gpu": Q if window else 0, "map_size": cfg["map"],
                    "parallelism": f"dp{world} (clients sharded over GPUs)",
                    "l2": f"inputs ring of {n_slots} distinct slots = {n_slots * slot_bytes / 2**20:.0f} MiB "
                          f"> L2 {l2 / 2**20:.0f} MiB (no flush)",
@@ -487,7 +500,7 @@ def run_ours(args, cfg):
         print(json.dumps(res), flush=True)
 
 
-def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams):
+def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=1.0):
     """Same ticks through the C ABI from pinned host buffers: H2D of the tick's inputs, extract +
     match, D2H of all results, every step inside the timed region; ticks round-robin over the
     in-flight contexts/streams so copies of one tick overlap compute of another."""
@@ -495,23 +508,21 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
     P = len(pipes)
     n_host = min(len(frames_h), 8)
     fr = [torch.from_numpy(frames_h[s]).pin_memory() for s in range(n_host)]
-    if window:
-        qh = [torch.from_numpy(np.ascontiguousarray(q_host[s % len(q_host)][0]).view(np.uint8).reshape(Q, 20)).pin_memory()
-              for s in range(n_host)]
-        qdh = [torch.from_numpy(q_host[s % len(q_host)][1]).pin_memory() for s in range(n_host)]
-        tkh = [torch.from_numpy(q_host[s % len(q_host)][2]).pin_memory() for s in range(n_host)]
+    if window:  # per slot: cams, points, point_frame, qdesc, taken
+        hin = [[torch.from_numpy(np.ascontiguousarray(a).view(np.uint8).reshape(-1).copy()).pin_memory()
+                for a in q_host[s % len(q_host)]] for s in range(n_host)]
     dev_in, host_out = [], []
     for q in range(P):  # per in-flight context: device inputs, pinned host outputs
         d = {"fr": torch.empty_like(fr[0], device=dev)}
         if window:
-            d.update(q=torch.empty_like(qh[0], device=dev), qd=torch.empty_like(qdh[0], device=dev),
-                     tk=torch.empty_like(tkh[0], device=dev))
+            d["in"] = [torch.empty_like(a, device=dev) for a in hin[0]]
+            d["qb"] = torch.empty((Q, 20), dtype=torch.uint8, device=dev)
         dev_in.append(d)
         host_out.append([torch.empty(pipes[q].kps[:B].shape, dtype=torch.uint8).pin_memory(),
                          torch.empty(pipes[q].desc[:B].shape, dtype=torch.uint8).pin_memory(),
                          torch.empty(pipes[q].counts[:B].shape, dtype=torch.int32).pin_memory(),
                          torch.empty(outs[q].shape, dtype=torch.int32).pin_memory()])
-    h2d = fr[0].numel() + ((qh[0].numel() + qdh[0].numel() + tkh[0].numel()) if window else 0)
+    h2d = fr[0].numel() + (sum(a.numel() for a in hin[0]) if window else 0)
     d2h = sum(t.numel() * t.element_size() for t in host_out[0])
 
     def step(s):
@@ -520,12 +531,13 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
         with torch.cuda.stream(streams[q]):
             d["fr"].copy_(fr[i], non_blocking=True)
             if window:
-                d["q"].copy_(qh[i], non_blocking=True)
-                d["qd"].copy_(qdh[i], non_blocking=True)
-                d["tk"].copy_(tkh[i], non_blocking=True)
+                for dst, src in zip(d["in"], hin[i]):
+                    dst.copy_(src, non_blocking=True)
             pp.extract(d["fr"], stream=streams[q])
             if window:
-                pp.match_window(B, d["q"], d["qd"], ot, taken=d["tk"], stream=streams[q])
+                cm, pt, pf, qd, tk = d["in"]
+                pp.project(B, cm, pt.view(Q, 32), pf.view(torch.int32), d["qb"], th=th, stream=streams[q])
+                pp.match_window(B, d["qb"], qd.view(Q, 32), ot, taken=tk, stream=streams[q])
             else:
                 pp.match_brute(B, map_desc, ot, stream=streams[q])
             kh.copy_(pp.kps[:B], non_blocking=True)
@@ -551,40 +563,41 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
     world = int(os.environ.get("WORLD_SIZE", 1))
     return {"value": B * world * K / (ms / 1000.0), "unit": "frames/s", "h2d_bytes_per_step": int(h2d),
             "d2h_bytes_per_step": int(d2h), "steps": K, "ms_per_step": ms / K, "ticks_in_flight": P,
-            "path": "pinned host -> H2D -> ss_orb_extract -> ss_match_projection -> D2H (C ABI, no graphs)"}
+            "path": "pinned host -> H2D -> ss_orb_extract -> " + ("ss_project_points -> " if window else "") +
+                    "ss_match_projection -> D2H (C ABI, no graphs)"}
 
 
 # ----------------------------------------------------------------------------- oracle (CPU) legs
 def _oracle_job(job):
     import oracle
-    (w, h, nf, frame, qq, qd, tk, mode, mp) = job
+    (w, h, nf, frame, lm, mode, mp, th) = job
     p = oracle.params(w, h, nf)
     t = time.perf_counter()
     kps, desc, counts = oracle.orb_extract(p, frame)
-    if mode == "window" and qq is not None:
-        q1 = qq.copy()
-        q1["frame"] = 0
-        oracle.match_window(p, kps[None], desc[None], counts[None], tk[None], q1, qd)
+    if mode == "window" and lm is not None:
+        cm, pt, qd, tk = lm
+        q = oracle.project_points(p, cm[None], pt, np.zeros(len(pt), np.int32), th)
+        oracle.match_window(p, kps[None], desc[None], counts[None], tk[None], q, qd)
     elif mode == "brute" and mp is not None:
         oracle.match_brute(p, desc[None], counts[None], mp, k0=0, k1=4)
     return time.perf_counter() - t
 
 
 def _jobs_for(cfg, frames_h, q_host, n, w, h, mp=None):
+    """Oracle jobs: one frame each (extract, then its local map projected + matched, or its
+    first 4 keypoints brute-matched against the whole map)."""
     jobs = []
     S, Bimg = frames_h.shape[:2]
     per_client = 2 if cfg.get("stereo") else 1
     i = 0
     while len(jobs) < n:
         s, b = (i // Bimg) % S, i % Bimg
-        qq = qd = tk = None
+        lm = None
         if cfg["mode"] == "window" and q_host and b % per_client == 0:
-            qs, qds, tks = q_host[s % len(q_host)]
-            c = b // per_client
-            sel = qs["frame"] == b
-            qq, qd, tk = qs[sel], qds[sel], tks[b]
-            _ = c
-        jobs.append((w, h, cfg["nf"], frames_h[s, b], qq, qd, tk, cfg["mode"], mp))
+            cm, pt, pf, qd, tk = q_host[s % len(q_host)]
+            sel = pf == b
+            lm = (cm[b], pt[sel], qd[sel], tk[b])
+        jobs.append((w, h, cfg["nf"], frames_h[s, b], lm, cfg["mode"], mp, cfg["th"]))
         i += 1
     return jobs
 
@@ -604,8 +617,10 @@ def cpu_baseline(args, cfg, frames_h, q_host, budget_s=15.0, mp=None):
         per = pool.map(_oracle_job, jobs, chunksize=1)
     wall = time.perf_counter() - t
     return {"value": len(jobs) / wall, "unit": "frames/s", "cores": cores, "kind": "oracle",
-            "sample": f"{len(jobs)} frames of the {args.config} workload (extract + its {cfg['queries']} "
-                      f"{cfg['mode']} queries each), one single-threaded oracle process per core",
+            "sample": f"{len(jobs)} frames of the {args.config} workload (extract + " +
+                      (f"its {cfg['queries']}-point local map projected and window-matched" if cfg["mode"] == "window"
+                       else "4 keypoints brute-matched against the map") +
+                      " each), one single-threaded oracle process per core",
             "median_frame_s_single_core": float(np.median(per)),
             "cpu": _cpu_model()}
 
@@ -639,16 +654,18 @@ def run_reference(args, cfg):
         p = oracle.params(w, h, cfg["nf"])
         q_host = []
         per_client = 2 if cfg.get("stereo") else 1
+        B = frames_h.shape[1]
         for s in range(frames_h.shape[0]):
             kps, desc, counts = oracle.orb_extract_batch(p, frames_h[s][::per_client])
-            qq, qd, tk = synth.make_queries(kps, desc, counts, 8, np.array(p.scale[:8]), np.array(p.n_per_level[:8]),
-                                            w, h, cfg["queries"], cfg["th"],
-                                            seed=synth.frame_seed(CFG_ID[args.config], 1 << 16, s),
-                                            query_dtype=oracle.QUERY_DTYPE)
-            qq["frame"] = qq["frame"] * per_client
-            tkf = np.zeros((frames_h.shape[1], p.kp_capacity), np.uint8)
+            cm, pt, pf, qd, tk = synth.make_local_map(kps, desc, counts, 8, p.scale_factor,
+                                                      np.array(p.n_per_level[:8]), w, h, cfg["shape"],
+                                                      cfg["queries"], seed=synth.frame_seed(CFG_ID[args.config],
+                                                                                            1 << 16, s))
+            cmf = np.zeros(B, synth.CAMERA_DTYPE)
+            cmf[::per_client] = cm
+            tkf = np.zeros((B, p.kp_capacity), np.uint8)
             tkf[::per_client] = tk
-            q_host.append((qq, qd, tkf))
+            q_host.append((cmf, pt, pf * per_client, qd, tkf))
     else:
         p = oracle.params(w, h, cfg["nf"])
         kps, desc, counts = oracle.orb_extract_batch(p, frames_h[0])
@@ -677,8 +694,10 @@ def run_reference(args, cfg):
            "config": {"workload": cfg["desc"], "config": args.config, "frames_per_step": n_frames,
                       "parallelism": "CPU oracle, one single-threaded process per core"},
            "cpu_baseline": {"value": value, "unit": "frames/s", "cores": min(cores, n_frames), "kind": "oracle",
-                            "sample": f"{n_frames} of the tick's {B} frames per step (extract + "
-                                      f"{cfg['queries']} {cfg['mode']} queries each)", "cpu": _cpu_model()},
+                            "sample": f"{n_frames} of the tick's {B} frames per step (extract + " +
+                                      (f"{cfg['queries']}-point local map projected + window-matched"
+                                       if cfg["mode"] == "window" else "4 keypoints brute-matched") + " each)",
+                            "cpu": _cpu_model()},
            "e2e": {"value": value, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(res), flush=True)
 

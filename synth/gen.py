@@ -157,3 +157,112 @@ def make_brute_map(desc_list, n_map: int, seed: int, n_from_kps: int | None = No
     rnd = rng.integers(0, 256, size=(n_map - nk, 32), dtype=np.uint8)
     m = np.concatenate([part, rnd], 0)
     return np.ascontiguousarray(m[rng.permutation(n_map)])
+
+
+# Pinhole intrinsics (fx, fy, cx, cy) of the datasets the shapes stand for (EuRoC cam0, TUM
+# fr1, KITTI 00 left) -- input geometry only; the projection itself is the method's (O11).
+INTRINSICS = {"euroc": (458.654, 457.296, 367.215, 248.375), "tum": (517.306, 516.469, 318.643, 255.314),
+              "kitti": (718.856, 718.856, 607.1928, 185.2157)}
+CAMERA_DTYPE = np.dtype([("R", "<f4", (9,)), ("t", "<f4", (3,)), ("ow", "<f4", (3,)), ("fx", "<f4"),
+                         ("fy", "<f4"), ("cx", "<f4"), ("cy", "<f4"), ("min_x", "<f4"), ("max_x", "<f4"),
+                         ("min_y", "<f4"), ("max_y", "<f4"), ("pad", "<f4")])
+MAP_POINT_DTYPE = np.dtype([("pos", "<f4", (3,)), ("normal", "<f4", (3,)), ("min_dist", "<f4"),
+                            ("max_dist", "<f4")])
+
+
+def _rotation(rng) -> np.ndarray:
+    q = rng.normal(size=4)
+    q /= np.linalg.norm(q)
+    w, x, y, z = q
+    return np.array([[1 - 2 * (y * y + z * z), 2 * (x * y - z * w), 2 * (x * z + y * w)],
+                     [2 * (x * y + z * w), 1 - 2 * (x * x + z * z), 2 * (y * z - x * w)],
+                     [2 * (x * z - y * w), 2 * (y * z + x * w), 1 - 2 * (x * x + y * y)]])
+
+
+def _tilt(d: np.ndarray, deg: np.ndarray, rng) -> np.ndarray:
+    """Unit vectors at angle deg from the unit rows of d (random azimuth)."""
+    a = np.cross(d, rng.normal(size=d.shape))
+    a /= np.linalg.norm(a, axis=1, keepdims=True)
+    r = np.radians(deg)[:, None]
+    return d * np.cos(r) + np.cross(a, d) * np.sin(r)
+
+
+def make_local_map(kps: np.ndarray, desc: np.ndarray, counts: np.ndarray, n_levels: int, scale_factor: float,
+                   n_per_level: np.ndarray, width: int, height: int, shape: str, n_points_per_frame: int,
+                   seed: int, taken_frac=0.10, true_frac=0.60):
+    """Local-map points for "search local points" (O11 projection -> O9 windowed match), per
+    frame (SURVEY §8(d) query statistics, lifted to 3D):
+
+    * a random camera pose per frame, the dataset's intrinsics, bounds [0, W] x [0, H];
+    * true points (60 % of the frame's keypoints): the keypoint position + N(0, 1 px)
+      back-projected at depth U(2, 20), descriptor = the keypoint's with 6 % bit flips,
+      max_dist = dist * sf^(level' - 0.5) with level' = level (80 %) or level + 1 (so the
+      predicted level is level'), min_dist = max_dist / sf^(L-1), normal = the viewing ray
+      tilted by U(0, 3) deg (half: radius factor 2.5) or U(6, 50) deg (4.0);
+    * distractors: positions uniform over the image +-10 % at depth U(-2, 30) (some behind the
+      camera or outside the image), levels ~ N_l, tilt U(0, 70) deg (some beyond 60 deg),
+      half random descriptors, half hard negatives (another keypoint's, 25 % flips);
+    * 10 % of keypoints marked taken.
+
+    kps [F, cap] (x, y, level), desc [F, cap, 32], counts [F, L+1].
+    Returns (cams [F], points [F*Q], point_frame [F*Q] i32, qdesc [F*Q, 32] u8, taken [F, cap] u8)."""
+    rng = _rng(seed)
+    F, cap = kps.shape
+    Q = n_points_per_frame
+    fx, fy, cx, cy = INTRINSICS[shape]
+    cams = np.zeros(F, CAMERA_DTYPE)
+    pts = np.zeros(F * Q, MAP_POINT_DTYPE)
+    pf = np.repeat(np.arange(F, dtype=np.int32), Q)
+    qdesc = np.zeros((F * Q, 32), np.uint8)
+    taken = np.zeros((F, cap), np.uint8)
+    pl = np.asarray(n_per_level, np.float64)
+    pl = pl / pl.sum()
+    sf = float(scale_factor)
+    for f in range(F):
+        R, t = _rotation(rng), rng.normal(0, 3.0, 3)
+        ow = -R.T @ t
+        c = cams[f]
+        c["R"], c["t"], c["ow"] = R.astype(np.float32).ravel(), t.astype(np.float32), ow.astype(np.float32)
+        c["fx"], c["fy"], c["cx"], c["cy"] = fx, fy, cx, cy
+        c["min_x"], c["max_x"], c["min_y"], c["max_y"] = 0.0, width, 0.0, height
+        n = int(counts[f, n_levels])
+        nt = min(int(true_frac * n), Q)
+        sel = rng.permutation(n)[:nt] if n else np.zeros(0, np.int64)
+        taken[f, :n] = rng.random(n) < taken_frac
+        u = np.empty(Q)
+        v = np.empty(Q)
+        lev = np.empty(Q, np.int64)
+        k = kps[f, sel]
+        u[:nt] = k["x"] + rng.normal(0, 1.0, nt)
+        v[:nt] = k["y"] + rng.normal(0, 1.0, nt)
+        lev[:nt] = np.minimum(k["level"].astype(np.int64) + (rng.random(nt) >= 0.8), n_levels - 1)
+        nd = Q - nt
+        u[nt:] = rng.uniform(-0.1 * width, 1.1 * width, nd)
+        v[nt:] = rng.uniform(-0.1 * height, 1.1 * height, nd)
+        lev[nt:] = rng.choice(n_levels, size=nd, p=pl)
+        z = np.concatenate([rng.uniform(2.0, 20.0, nt), rng.uniform(-2.0, 30.0, nd)])
+        pc = np.stack([(u - cx) / fx * z, (v - cy) / fy * z, z], 1)
+        pw = (pc - t) @ R  # R^T (pc - t), row-wise
+        ray = pw - ow
+        dist = np.linalg.norm(ray, axis=1)
+        tilt = np.where(rng.random(Q) < 0.5, rng.uniform(0, 3, Q), rng.uniform(6, 50, Q))
+        tilt[nt:] = rng.uniform(0, 70, nd)
+        nrm = _tilt(ray / dist[:, None], tilt, rng)
+        p = pts[f * Q:(f + 1) * Q]
+        p["pos"] = pw.astype(np.float32)
+        p["normal"] = nrm.astype(np.float32)
+        p["max_dist"] = (dist * sf ** (lev - 0.5)).astype(np.float32)
+        p["min_dist"] = (p["max_dist"].astype(np.float64) / sf ** (n_levels - 1)).astype(np.float32)
+        qd = qdesc[f * Q:(f + 1) * Q]
+        if nt:
+            qd[:nt] = flip_bits(desc[f, sel], 0.06, rng)
+        rnd = rng.integers(0, 256, size=(nd, 32), dtype=np.uint8)
+        hard = rng.random(nd) < 0.5
+        if n:
+            other = desc[f, rng.integers(0, n, nd)]
+            rnd[hard] = flip_bits(other[hard], 0.25, rng)
+        qd[nt:] = rnd
+        perm = rng.permutation(Q)
+        pts[f * Q:(f + 1) * Q] = p[perm]
+        qdesc[f * Q:(f + 1) * Q] = qd[perm]
+    return cams, pts, pf, qdesc, taken

@@ -265,3 +265,37 @@ def test_compute_sanitizer_clean(torch_cuda, tool):
     tail = (r.stdout + r.stderr)[-3000:]
     assert r.returncode == 0 and "sanitize run ok" in r.stdout, tail
     assert "ERROR SUMMARY: 0 errors" in r.stdout + r.stderr or "RACECHECK SUMMARY: 0 hazards" in r.stdout + r.stderr, tail
+
+
+@pytest.mark.parametrize("shape,th", [("euroc", 1.0), ("tum", 3.0)])
+def test_search_local_points_chain(torch_cuda, ref, shape, th):
+    """The whole S9 step as bench.py runs it: GPU extract -> GPU projection of each frame's
+    local map (O11) -> GPU windowed match (O9), vs the oracle's extract -> project -> match."""
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import match_records
+    w, h = synth.SHAPES[shape]
+    B, Q = 3, 3000
+    frames = synth.make_frames(w, h, B, cfg=21)
+    p = ref.params(w, h, 1000)
+    rk, rd, rc = ref.orb_extract_batch(p, frames)
+    cams, pts, pf, qd, tk = synth.make_local_map(rk, rd, rc, 8, p.scale_factor, np.array(p.n_per_level[:8]),
+                                                 w, h, shape, Q, seed=5)
+    q_ref = ref.project_points(p, cams, pts, pf, th)
+    want = ref.match_window(p, rk, rd, rc, tk, q_ref, qd)
+    pipe = _pipe(torch, w, h, 1000, 8, max_frames=B, max_queries=B * Q)
+    pipe.extract(_upload(torch, frames))
+    qbuf = torch.zeros((B * Q, 20), dtype=torch.uint8, device="cuda")
+    pipe.project(B, torch.from_numpy(cams.view(np.uint8).reshape(B, 96).copy()).cuda(),
+                 torch.from_numpy(pts.view(np.uint8).reshape(-1, 32).copy()).cuda(), torch.from_numpy(pf).cuda(),
+                 qbuf, th=th)
+    out = torch.zeros((B * Q, 3), dtype=torch.int32, device="cuda")
+    pipe.match_window(B, qbuf, torch.from_numpy(qd).cuda(), out, taken=torch.from_numpy(tk).cuda())
+    got_q = qbuf.cpu().numpy().view(ref.QUERY_DTYPE).reshape(-1)
+    for fld in ("frame", "pred_level"):
+        np.testing.assert_array_equal(got_q[fld], q_ref[fld], err_msg=fld)
+    for fld in ("u", "v", "radius"):
+        np.testing.assert_array_equal(got_q[fld].view(np.uint32), q_ref[fld].view(np.uint32), err_msg=fld)
+    got = match_records(out)
+    np.testing.assert_array_equal(got, want)
+    assert (got["idx"] >= 0).sum() > 200
+    pipe.close()
