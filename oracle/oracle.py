@@ -94,6 +94,8 @@ def lib():
                                           C.c_int, C.c_int, C.c_int, C.c_int, P]
         _lib.ref_match_brute.argtypes = [C.POINTER(RefParams), C.c_int, P, P, C.c_int, P, C.c_int,
                                          C.c_int, C.c_int, C.c_int, C.c_int, P]
+        _lib.ref_stereo_match.argtypes = [C.POINTER(RefParams), P, P, C.c_int, P, P, P, P, P, P, C.c_float, C.c_float,
+                                          P, P, P]
         _lib.ref_project_points.argtypes = [C.POINTER(RefParams), C.c_int, P, C.c_int, P, P, C.c_float, P]
     return _lib
 
@@ -258,3 +260,18 @@ def project_points(p: RefParams, cams, points, point_frame, th=1.0):
     lib().ref_project_points(C.byref(p), len(cams), _p(cams), len(points), _p(points), _p(point_frame),
                              float(th), _p(out))
     return out
+
+
+def stereo_match(p: RefParams, left, right, kl, dl, cl, kr, dr, cr, bf, b):
+    """O12: one rectified pair -> (uright[cap] f32, depth[cap] f32, sad[cap] i32), -1 = none."""
+    left = np.ascontiguousarray(left, dtype=np.uint8)
+    right = np.ascontiguousarray(right, dtype=np.uint8)
+    assert left.shape == right.shape
+    cap = p.kp_capacity
+    ur = np.full(cap, -1.0, np.float32)
+    dp = np.full(cap, -1.0, np.float32)
+    sad = np.full(cap, -1, np.int32)
+    args = [np.ascontiguousarray(a) for a in (kl, dl, cl, kr, dr, cr)]
+    lib().ref_stereo_match(C.byref(p), _p(left), _p(right), left.shape[1], *[_p(a) for a in args],
+                           float(bf), float(b), _p(ur), _p(dp), _p(sad))
+    return ur, dp, sad

@@ -23,6 +23,9 @@
  *   O6 blur        : cv2.GaussianBlur(7x7, sigma 2, REFLECT_101)
  *   O7 descriptor  : rot90 invariance (bit-exact); unrotated case = pattern lookups
  *   O9/O10 match   : brute-force definitions in Python on small inputs
+ *   O12 stereo     : right image = left shifted by an integer disparity (uR within 0.5 px
+ *                    of uL - d, depth ~ bf/d); invariants (level gate, Hamming < 75,
+ *                    disparity range, outlier cut at 2.1 x the median SAD)
  *   O11 projection : cv2.projectPoints (f64) on random poses; closed forms (optical axis,
  *                    rot90 about z, viewCos = 1 along the normal); predicted level vs
  *                    ceil(log(ratio)/log(1.2)) away from level boundaries; each culling
@@ -705,4 +708,152 @@ void ref_project_points(const ref_params* p, int F, const ref_camera* cams, int 
     float r = rv * th;
     o->u = u; o->v = v; o->pred_level = level; o->radius = r * p->scale[level];
   }
+}
+
+/* ------------------------------------------------------------- O12 stereo */
+/* ORB-SLAM2 Frame::ComputeStereoMatches [ext] (the stereo tracking input of P:L163/L246;
+ * SURVEY §8(f) F1), step by step in ORB-SLAM's order:
+ *  1. every right keypoint iR is listed on rows floor(y - r) .. ceil(y + r), r = 2*scale[oct];
+ *  2. per left keypoint: candidates = the list of row (int)vL, in iR order; keep those on
+ *     octaves [oct-1, oct+1] with uL - maxD <= uR <= uL (maxD = bf/b, minD = 0); best =
+ *     first minimum Hamming distance below TH_HIGH = 100;
+ *  3. if best < (TH_HIGH + TH_LOW)/2 = 75: 11x11 SAD of the left window (centre-subtracted)
+ *     against right windows at scaleduR0 + inc, inc in [-5, 5] (centre-subtracted), on the
+ *     octave's pyramid level; rounded coordinates round(v * invScale[oct]) (half away from
+ *     zero); skip if iniu = scaleduR0 < 0 or endu = scaleduR0 + 11 >= level width (ORB-SLAM's
+ *     check, literally); first minimum SAD; reject inc = +-5; parabola
+ *     deltaR = (d1 - d3) / (2 (d1 + d3 - 2 d2)), reject |deltaR| > 1;
+ *     uR = scale[oct] * ((float)scaleduR0 + (float)inc + deltaR); disparity = uL - uR,
+ *     accept 0 <= disparity < maxD (<= 0 -> 0.01, uR = uL - 0.01 in double); depth = bf/disparity;
+ *  4. outliers: median = the SAD of element size/2 of the accepted (SAD, iL) sorted
+ *     ascending; reject every accepted match with SAD >= 1.5f*1.4f*median.
+ * Keypoint indices are the canonical (level, ly, lx) order.  SADs are exact integers. */
+static const uint8_t* ref_level_ptr(const ref_params* p, const uint8_t* pyr, int l) {
+  int64_t off = 0;
+  for (int i = 0; i < l; i++) off += (int64_t)p->level_w[i] * p->level_h[i];
+  return pyr + off;
+}
+
+static int cmp_pair(const void* a, const void* b) {
+  const int32_t* x = (const int32_t*)a;
+  const int32_t* y = (const int32_t*)b;
+  if (x[0] != y[0]) return x[0] < y[0] ? -1 : 1;
+  return x[1] < y[1] ? -1 : (x[1] > y[1]);
+}
+
+void ref_stereo_match(const ref_params* p, const uint8_t* left, const uint8_t* right, int pitch,
+                      const ref_keypoint* kl, const uint8_t* dl, const int32_t* cl,
+                      const ref_keypoint* kr, const uint8_t* dr, const int32_t* cr, float bf, float b,
+                      float* uright, float* depth, int32_t* sad) {
+  const int L = p->n_levels, H = p->height;
+  const int nl = cl[L], nr = cr[L];
+  int64_t pb = ref_pyramid_bytes(p);
+  uint8_t* pyl = (uint8_t*)malloc((size_t)pb);
+  uint8_t* pyr = (uint8_t*)malloc((size_t)pb);
+  ref_pyramid(p, left, pitch, pyl);
+  ref_pyramid(p, right, pitch, pyr);
+  /* 1. row lists */
+  int* rcount = (int*)calloc((size_t)H, sizeof(int));
+  int* rstart = (int*)malloc(sizeof(int) * (size_t)(H + 1));
+  for (int i = 0; i < nr; i++) {
+    float ky = kr[i].y, r = 2.0f * p->scale[kr[i].level];
+    int maxr = (int)ceilf(ky + r), minr = (int)floorf(ky - r);
+    for (int yi = minr; yi <= maxr; yi++)
+      if (yi >= 0 && yi < H) rcount[yi]++;
+  }
+  rstart[0] = 0;
+  for (int y = 0; y < H; y++) rstart[y + 1] = rstart[y] + rcount[y];
+  int* rlist = (int*)malloc(sizeof(int) * (size_t)(rstart[H] > 0 ? rstart[H] : 1));
+  memset(rcount, 0, sizeof(int) * (size_t)H);
+  for (int i = 0; i < nr; i++) {
+    float ky = kr[i].y, r = 2.0f * p->scale[kr[i].level];
+    int maxr = (int)ceilf(ky + r), minr = (int)floorf(ky - r);
+    for (int yi = minr; yi <= maxr; yi++) {
+      if (yi < 0 || yi >= H) continue;
+      rlist[rstart[yi] + rcount[yi]++] = i;
+    }
+  }
+  const float minD = 0.0f, maxD = bf / b;
+  const int thOrb = (100 + 50) / 2;
+  int32_t* acc = (int32_t*)malloc(sizeof(int32_t) * 2 * (size_t)(nl > 0 ? nl : 1));
+  int nacc = 0;
+  for (int iL = 0; iL < nl; iL++) {
+    uright[iL] = -1.0f; depth[iL] = -1.0f; sad[iL] = -1;
+    const ref_keypoint* k = &kl[iL];
+    const int lev = k->level;
+    const float vL = k->y, uL = k->x;
+    const int row = (int)vL;
+    if (row < 0 || row >= H || rcount[row] == 0) continue;
+    const float minU = uL - maxD, maxU = uL - minD;
+    if (maxU < 0) continue;
+    int bestDist = 100, bestIdxR = 0;
+    for (int c = 0; c < rcount[row]; c++) {
+      int iR = rlist[rstart[row] + c];
+      const ref_keypoint* q = &kr[iR];
+      if (q->level < lev - 1 || q->level > lev + 1) continue;
+      const float uR = q->x;
+      if (uR >= minU && uR <= maxU) {
+        int dist = ref_hamming(dl + (size_t)iL * 32, dr + (size_t)iR * 32);
+        if (dist < bestDist) { bestDist = dist; bestIdxR = iR; }
+      }
+    }
+    if (bestDist >= thOrb) continue;
+    /* 3. sub-pixel refinement by SAD on the octave's level */
+    const float uR0 = kr[bestIdxR].x;
+    const float sf = p->inv_scale[lev];
+    const int su = (int)roundf(uL * sf), sv = (int)roundf(vL * sf), su0 = (int)roundf(uR0 * sf);
+    const int w = 5, Lr = 5;
+    const int lw = p->level_w[lev];
+    const uint8_t* IL = ref_level_ptr(p, pyl, lev);
+    const uint8_t* IR = ref_level_ptr(p, pyr, lev);
+    const int iniu = su0 + Lr - w, endu = su0 + Lr + w + 1;
+    if (iniu < 0 || endu >= lw) continue;
+    float vd[11];
+    float best = 3.0e38f;
+    int bestinc = 0;
+    const int cL = IL[(size_t)sv * lw + su];
+    for (int inc = -Lr; inc <= Lr; inc++) {
+      const int cR = IR[(size_t)sv * lw + su0 + inc];
+      double s1 = 0.0;
+      for (int dy = -w; dy <= w; dy++)
+        for (int dx = -w; dx <= w; dx++) {
+          int a = IL[(size_t)(sv + dy) * lw + su + dx] - cL;
+          int bb = IR[(size_t)(sv + dy) * lw + su0 + inc + dx] - cR;
+          s1 += fabs((double)(a - bb));
+        }
+      float dist = (float)s1;
+      if (dist < best) { best = dist; bestinc = inc; }
+      vd[Lr + inc] = dist;
+    }
+    if (bestinc == -Lr || bestinc == Lr) continue;
+    const float d1 = vd[Lr + bestinc - 1], d2 = vd[Lr + bestinc], d3 = vd[Lr + bestinc + 1];
+    const float deltaR = (d1 - d3) / (2.0f * (d1 + d3 - 2.0f * d2));
+    if (deltaR < -1 || deltaR > 1) continue;
+    float bestuR = p->scale[lev] * ((float)su0 + (float)bestinc + deltaR);
+    float disparity = uL - bestuR;
+    if (disparity >= minD && disparity < maxD) {
+      if (disparity <= 0) {
+        disparity = 0.01;
+        bestuR = (float)((double)uL - 0.01);
+      }
+      depth[iL] = bf / disparity;
+      uright[iL] = bestuR;
+      sad[iL] = (int32_t)best;
+      acc[2 * nacc] = (int32_t)best;
+      acc[2 * nacc + 1] = iL;
+      nacc++;
+    }
+  }
+  /* 4. outlier cut */
+  if (nacc > 0) {
+    qsort(acc, (size_t)nacc, 2 * sizeof(int32_t), cmp_pair);
+    const int median = acc[2 * (nacc / 2)];
+    const float thDist = 1.5f * 1.4f * (float)median;
+    for (int i = nacc - 1; i >= 0; i--) {
+      if ((float)acc[2 * i] < thDist) break;
+      uright[acc[2 * i + 1]] = -1.0f;
+      depth[acc[2 * i + 1]] = -1.0f;
+    }
+  }
+  free(acc); free(rlist); free(rstart); free(rcount); free(pyl); free(pyr);
 }

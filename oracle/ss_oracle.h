@@ -102,6 +102,16 @@ typedef struct { float pos[3], normal[3], min_dist, max_dist; } ref_map_point;
 void ref_project_points(const ref_params* p, int n_frames, const ref_camera* cams, int n_points,
                         const ref_map_point* pts, const int32_t* point_frame, float th, ref_query* out);
 
+/* O12: ORB-SLAM2 Frame::ComputeStereoMatches for one rectified pair.
+ * left/right: level-0 images (pitch), keypoints/descriptors/counts of each image (O1..O8);
+ * bf = baseline x fx, b = baseline (maxD = bf / b).  Out: uright[kp_capacity],
+ * depth[kp_capacity] per LEFT keypoint (-1 = no stereo match; slots >= count untouched), and
+ * sad[kp_capacity] = the SAD of accepted matches before the outlier cut (-1 otherwise). */
+void ref_stereo_match(const ref_params* p, const uint8_t* left, const uint8_t* right, int pitch,
+                      const ref_keypoint* kl, const uint8_t* dl, const int32_t* cl,
+                      const ref_keypoint* kr, const uint8_t* dr, const int32_t* cr, float bf, float b,
+                      float* uright, float* depth, int32_t* sad);
+
 #ifdef __cplusplus
 }
 #endif
