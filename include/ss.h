@@ -187,6 +187,25 @@ ss_status ss_project_points(ss_ctx* ctx, int32_t n_frames, const ss_camera* d_ca
                             const ss_map_point* d_points, const int32_t* d_point_frame, float th,
                             ss_mp_query* d_queries, ss_stream_t stream);
 
+/* O12: stereo matching of rectified pairs (ORB-SLAM2 Frame::ComputeStereoMatches; the input
+ * of the paper's stereo tracking, PAPER.md L163 / L246), run after ss_orb_extract on the
+ * SAME ctx and frames: pair i = extracted frames 2i (left) and 2i+1 (right); d_frames,
+ * frame_stride, pitch, d_kps, d_desc, d_counts are that call's arguments (the pyramid levels
+ * >= 1 are read from the ctx's scratch, so no other ss_orb_extract may run on the ctx in
+ * between).  Per left keypoint iL (slot iL of pair i): d_uright[i][iL] = the right-image x
+ * coordinate (level-0 px, sub-pixel) and d_depth[i][iL] = bf / disparity, or -1 for both when
+ * there is no stereo match (slots >= the left count are left untouched).  Matching: right
+ * keypoints on octaves [o-1, o+1] whose row span [floor(y - 2 s), ceil(y + 2 s)] holds
+ * (int)vL, with uL - bf/baseline <= uR <= uL; smallest Hamming (lowest index on ties) below
+ * 100, kept if < 75; 11x11 centre-subtracted SAD over shifts [-5, 5] on octave o's level,
+ * parabola sub-pixel offset, disparity in [0, bf/baseline); then every match whose SAD is
+ * >= 1.5f*1.4f*(median accepted SAD) is dropped.  Bit-exact with the oracle (DESIGN.md §3
+ * item 12).  SS_EINVAL for bad sizes, pitches, NULL buffers or bf / baseline <= 0;
+ * SS_ECAPACITY if 2*n_pairs > max_frames. */
+ss_status ss_stereo_match(ss_ctx* ctx, int32_t n_pairs, const uint8_t* d_frames, int64_t frame_stride, int32_t pitch,
+                          const ss_keypoint* d_kps, const uint8_t* d_desc, const int32_t* d_counts, float bf,
+                          float baseline, float* d_uright, float* d_depth, ss_stream_t stream);
+
 /* ---- profiling hook (bench.py; does not synchronise) ---- */
 
 /* When n_events > 0, every following ss_orb_extract / ss_match_projection records the
@@ -200,7 +219,7 @@ ss_status ss_project_points(ss_ctx* ctx, int32_t n_frames, const ss_camera* d_ca
  * branch runs in line on `stream` instead of on its side stream, so each kernel is timed
  * alone).  WINDOW match: a pair per kernel
  * (match_prepare, match_window[, match_resolve if dedup]); BRUTE: brute_expand, brute_tc,
- * brute_merge; ss_project_points: project.
+ * brute_merge; ss_project_points: project; ss_stereo_match: stereo_prepare, stereo, stereo_outliers.
  * Works under CUDA-graph stream capture (the records become graph event nodes).
  * *next_index (may be NULL) receives the index of the next event to be recorded. */
 ss_status ss_profile_events(ss_ctx* ctx, void* const* events, int32_t n_events);

@@ -144,6 +144,7 @@ struct ss_ctx {
   uint16_t* rowidx = nullptr;  // WINDOW matcher: first keypoint per (frame, level, row)
   uint64_t* phase_ts = nullptr;  // distribution phase timestamps [max_frames][L][16] (debug hook)
   unsigned long long* partial = nullptr;
+  int32_t* stereo_sad = nullptr;  // O12: accepted SAD per left keypoint [max_frames/2][cap]
   int8_t* brute_qexp = nullptr;  // BRUTE: keypoint descriptors expanded to s8 +-1 (k_brute_tc.cu)
   int8_t* brute_mexp = nullptr;  // BRUTE: map descriptors expanded to s8 +-1
   int n_sm = 148;
@@ -183,7 +184,7 @@ void free_ctx(ss_ctx* c) {
   cudaSetDevice(c->device);
   void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr_plan, c->pyr_gtab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
                   c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->rowidx, c->phase_ts,
-                  c->brute_qexp, c->brute_mexp};
+                  c->brute_qexp, c->brute_mexp, c->stereo_sad};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
@@ -247,6 +248,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     g.w[l] = q.level_w[l];
     g.h[l] = q.level_h[l];
     g.scale[l] = q.scale[l];
+    g.inv_scale[l] = q.inv_scale[l];
     g.pitch[l] = (g.w[l] + 15) & ~15;
     g.lvl_off[l] = 0;
     if (l >= 1) {
@@ -436,6 +438,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->claim, sizeof(unsigned long long) * F * g.kp_capacity);
   ALLOC(c->rowidx, sizeof(uint16_t) * F * match_rows_per_frame(g));
   ALLOC(c->phase_ts, sizeof(uint64_t) * F * L * 16);
+  ALLOC(c->stereo_sad, sizeof(int32_t) * ((F + 1) / 2) * g.kp_capacity);
   if (max_map > 0) {
     ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
     ALLOC(c->brute_qexp, brute_tc_query_bytes(F * g.kp_capacity));
@@ -583,6 +586,34 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
     return SS_OK;
   }
   return fail(SS_EINVAL, "unknown match mode");
+}
+
+ss_status ss_stereo_match(ss_ctx* c, int32_t n_pairs, const uint8_t* d_frames, int64_t frame_stride, int32_t pitch,
+                          const ss_keypoint* d_kps, const uint8_t* d_desc, const int32_t* d_counts, float bf,
+                          float baseline, float* d_uright, float* d_depth, ss_stream_t stream) {
+  if (!c) return fail(SS_EINVAL, "NULL ctx");
+  if (n_pairs < 0) return fail(SS_EINVAL, "negative size");
+  if (2 * (int64_t)n_pairs > c->max_frames) return fail(SS_ECAPACITY, "2 * n_pairs exceeds the ctx's max_frames");
+  if (n_pairs == 0) return SS_OK;
+  if (!d_frames || !d_kps || !d_desc || !d_counts || !d_uright || !d_depth) return fail(SS_EINVAL, "NULL buffer");
+  if (pitch < c->g.W || frame_stride < (int64_t)c->g.H * pitch) return fail(SS_EINVAL, "bad pitch / frame stride");
+  if (!(bf > 0.0f) || !(baseline > 0.0f)) return fail(SS_EINVAL, "bf and baseline must be > 0");
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  SS_CUDA_TRY(check_stream(s));
+  const float maxD = bf / baseline;  // ORB-SLAM: maxD = mbf / minZ, minZ = mb
+  FrameSrc src{d_frames, frame_stride, pitch, c->pyr};
+  prof_mark(c, s);
+  SS_CUDA_TRY(launch_match_prepare(c->g, 2 * n_pairs, d_kps, d_counts, c->rowidx, c->claim, 0, s));
+  prof_mark(c, s);
+  prof_mark(c, s);
+  SS_CUDA_TRY(launch_stereo(c->g, n_pairs, src, d_kps, d_desc, d_counts, c->rowidx, match_rows_per_frame(c->g), bf,
+                            maxD, d_uright, d_depth, c->stereo_sad, s));
+  prof_mark(c, s);
+  prof_mark(c, s);
+  SS_CUDA_TRY(launch_stereo_outliers(c->g, n_pairs, d_counts, c->stereo_sad, d_uright, d_depth, s));
+  prof_mark(c, s);
+  return SS_OK;
 }
 
 ss_status ss_project_points(ss_ctx* c, int32_t n_frames, const ss_camera* d_cams, int32_t n_points,

@@ -46,6 +46,7 @@ struct Geom {
   int64_t lvl_off[kMaxLevels];      // byte offset of level l in a frame's pyramid scratch
   int64_t pyr_frame_bytes;
   float scale[kMaxLevels];
+  float inv_scale[kMaxLevels];      // f32(1 / scale[l]) (O0)
   int32_t cell_first[kMaxLevels];   // first active cell of level l in the cell table
   int32_t ncells[kMaxLevels];       // active cells of level l (row-major, skipped cells removed)
   int32_t total_cells;              // per frame
@@ -178,6 +179,13 @@ cudaError_t launch_brute_tc(int n_slots, int n_map, const int8_t* qexp, const in
 // O11 local-map projection (k_project.cu): one thread per map point.
 cudaError_t launch_project(const Geom& g, int n_frames, const ss_camera* cams, int n_points, const ss_map_point* pts,
                            const int32_t* point_frame, float th, ss_mp_query* out, cudaStream_t s);
+
+// O12 stereo matching (k_stereo.cu): one warp per left keypoint, then the per-pair outlier cut.
+cudaError_t launch_stereo(const Geom& g, int n_pairs, FrameSrc src, const ss_keypoint* kps, const uint8_t* desc,
+                          const int32_t* counts, const uint16_t* rowidx, int rows_per_frame, float bf, float maxD,
+                          float* uright, float* depth, int32_t* sad, cudaStream_t s);
+cudaError_t launch_stereo_outliers(const Geom& g, int n_pairs, const int32_t* counts, const int32_t* sad,
+                                   float* uright, float* depth, cudaStream_t s);
 
 // Overflow scratch bytes the distribution needs for a level with `slots` candidate slots.
 int64_t distribute_ovf_bytes(int64_t slots);

@@ -76,6 +76,14 @@ class OrbPipeline:
         n = point_frame.numel()
         ss.ss_project_points(self.ctx, n_frames, cams, n, points, point_frame, th, out, stream)
 
+    def stereo(self, frames: torch.Tensor, bf: float, baseline: float, uright: torch.Tensor, depth: torch.Tensor,
+               n_pairs: int | None = None, stream: torch.cuda.Stream | None = None):
+        """O12 after extract(frames) of pairs (2i left, 2i+1 right): uright / depth f32 [n_pairs, cap]."""
+        stream = stream or torch.cuda.current_stream(self.device)
+        n_pairs = frames.shape[0] // 2 if n_pairs is None else n_pairs
+        ss.ss_stereo_match(self.ctx, n_pairs, frames, frames.stride(0), frames.stride(1), self.kps, self.desc,
+                           self.counts, bf, baseline, uright, depth, stream)
+
     # -- host views (synchronising; tests / examples) -------------------------------
     def results(self, n_frames: int):
         torch.cuda.synchronize(self.device)

@@ -87,6 +87,7 @@ def lib():
         L.ss_orb_extract.argtypes = [P, i32, P, i64, i32, P, P, P, P]
         L.ss_match_projection.argtypes = [P, i32, P, P, P, P, i32, P, P, i32, C.POINTER(ss_match_cfg), P, P]
         L.ss_project_points.argtypes = [P, i32, P, i32, P, P, C.c_float, P, P]
+        L.ss_stereo_match.argtypes = [P, i32, P, i64, i32, P, P, P, C.c_float, C.c_float, P, P, P]
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
         L.ss_debug_candidates.argtypes = [P, i32, i32, P, P, P, i32, C.POINTER(i32)]
         L.ss_debug_overflow_count.argtypes = [P, C.POINTER(i32)]
@@ -94,7 +95,7 @@ def lib():
         L.ss_debug_phase_times.argtypes = [P, i32, i32, P, i32]
         L.ss_profile_next.argtypes = [P, C.POINTER(i32)]
         for fn in ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_orb_extract", "ss_match_projection",
-                   "ss_project_points",
+                   "ss_project_points", "ss_stereo_match",
                    "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
                    "ss_profile_next", "ss_debug_phase_times"):
             getattr(L, fn).restype = C.c_int
@@ -103,7 +104,7 @@ def lib():
 
 
 EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "ss_orb_extract",
-            "ss_match_projection", "ss_project_points", "ss_profile_events", "ss_profile_next", "ss_debug_level",
+            "ss_match_projection", "ss_project_points", "ss_stereo_match", "ss_profile_events", "ss_profile_next", "ss_debug_level",
             "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times")
 
 
@@ -163,6 +164,13 @@ def ss_match_projection(ctx, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_qu
     _check(lib().ss_match_projection(ctx, n_frames, _ptr(d_kps), _ptr(d_desc), _ptr(d_counts),
                                      _ptr(d_kp_taken), n_queries, _ptr(d_queries), _ptr(d_map_desc), n_map,
                                      C.byref(cfg), _ptr(d_out), _stream(stream)), ctx)
+
+
+def ss_stereo_match(ctx, n_pairs, d_frames, frame_stride, pitch, d_kps, d_desc, d_counts, bf, baseline, d_uright,
+                    d_depth, stream=None):
+    _check(lib().ss_stereo_match(ctx, n_pairs, _ptr(d_frames), frame_stride, pitch, _ptr(d_kps), _ptr(d_desc),
+                                 _ptr(d_counts), float(bf), float(baseline), _ptr(d_uright), _ptr(d_depth),
+                                 _stream(stream)), ctx)
 
 
 def ss_project_points(ctx, n_frames, d_cams, n_points, d_points, d_point_frame, th, d_queries, stream=None):
