@@ -42,7 +42,8 @@ CONFIGS = {
                desc="c3: TUM-RGBD-shaped 640x480, 16 clients per GPU, 1000 features, search local points vs 50k local-map points (projection + windowed match)"),
     "c4": dict(shape="kitti", clients=8, stereo=True, nf=2000, mode="window", queries=10000, th=1.0, map=0,
                desc="c4: KITTI-shaped 1241x376 stereo pairs, 8 clients per GPU, 2000 features/image, "
-                    "search local points vs 10k local-map points (left image; projection + windowed match)"),
+                    "ORB-SLAM stereo matching of every pair + search local points vs 10k local-map points "
+                    "(left image; projection + windowed match)"),
     "c5": dict(shape="euroc", clients=8, nf=1250, mode="brute", queries=0, th=0.0, map=200000,
                desc="c5: EuRoC-shaped clients (8 per GPU, 64 over 8xB200), 1250 features, brute-force Hamming "
                     "vs a 200k shared-map descriptor set"),
@@ -194,6 +195,8 @@ def kernel_work(name: str, p, B: int, cand_l: list, kps_l: list, nq: int, n_map:
         return "hbm", float(sum(kps_l) * (43 * 43 + 4 + 52))
     if name == "match_window":  # query 20 B + descriptor 32 B read, 12 B written
         return "hbm", float(nq * 64)
+    if name == "stereo":  # per left keypoint: its record + descriptor, 11x11 + 11x21 SAD pixels
+        return "hbm", float(sum(kps_l)) / 2 * (20 + 32 + 121 + 231)  # half of the images are left ones
     if name == "project":  # map point 32 B + frame index 4 B read, query 20 B written
         return "hbm", float(nq * 56)
     if name == "match_resolve":
@@ -294,7 +297,12 @@ def run_ours(args, cfg):
     # --- one CUDA graph per ring slot (plain, timed) + an instrumented twin whose profiling
     #     events (recorded inside the graph) give every kernel's duration
     mode = ss.SS_MATCH_WINDOW if window else ss.SS_MATCH_BRUTE
-    ek, mk = ss.extract_kernels(L), (["project"] if window else []) + ss.match_kernels(mode, True)
+    stereo = bool(cfg.get("stereo"))
+    ek = ss.extract_kernels(L)
+    mk = (["stereo_prepare", "stereo", "stereo_outliers"] if stereo else []) + (["project"] if window else []) + \
+        ss.match_kernels(mode, True)
+    BASE_M = synth.STEREO_BASELINE.get(cfg["shape"], 0.0)
+    BF = float(np.float32(synth.INTRINSICS[cfg["shape"]][0] * BASE_M))
     base = ss.extract_events(L)
     kernel_ev = [(n, 1 + 2 * i, 2 + 2 * i) for i, n in enumerate(ek)] + \
                 [(n, base + 2 * j, base + 2 * j + 1) for j, n in enumerate(mk)]
@@ -312,6 +320,9 @@ def run_ours(args, cfg):
                                   device=local) for _ in range(P - 1)]
     outs = [out] + [torch.zeros_like(out) for _ in range(P - 1)]
     qbufs = [torch.zeros((max(Q, 1), 20), dtype=torch.uint8, device=dev) for _ in range(P)]  # projected queries
+    npairs = B // 2 if stereo else 0
+    st_out = [(torch.zeros((max(npairs, 1), cap), dtype=torch.float32, device=dev),
+               torch.zeros((max(npairs, 1), cap), dtype=torch.float32, device=dev)) for _ in range(P)]
     streams = [stream] + [torch.cuda.Stream(dev) for _ in range(P - 1)]
     for q in range(1, P):  # first call outside capture (kernel attributes)
         with torch.cuda.stream(streams[q]):
@@ -325,6 +336,8 @@ def run_ours(args, cfg):
             ss.ss_profile_events(pp.ctx, events[s])
         with torch.cuda.graph(g, stream=st):
             pp.extract(frames[s], stream=st)
+            if stereo:
+                pp.stereo(frames[s], BF, BASE_M, st_out[q][0], st_out[q][1], stream=st)
             if window:
                 pp.project(B, cams[s], points[s], point_frame[s], qbufs[q], th=cfg["th"], stream=st)
                 pp.match_window(B, qbufs[q], qdesc[s], ot, taken=taken[s], stream=st)
@@ -459,7 +472,8 @@ def run_ours(args, cfg):
             pass
 
     # --- e2e through the public API with host buffers (pinned), copies inside the timed region
-    e2e = run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=cfg["th"])
+    e2e = run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=cfg["th"],
+                  stereo=(BF, BASE_M, st_out) if stereo else None)
 
     frames_per_step = B * world
     value = frames_per_step * K / (T_max / 1000.0)
@@ -500,7 +514,7 @@ def run_ours(args, cfg):
         print(json.dumps(res), flush=True)
 
 
-def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=1.0):
+def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=1.0, stereo=None):
     """Same ticks through the C ABI from pinned host buffers: H2D of the tick's inputs, extract +
     match, D2H of all results, every step inside the timed region; ticks round-robin over the
     in-flight contexts/streams so copies of one tick overlap compute of another."""
@@ -521,19 +535,23 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
         host_out.append([torch.empty(pipes[q].kps[:B].shape, dtype=torch.uint8).pin_memory(),
                          torch.empty(pipes[q].desc[:B].shape, dtype=torch.uint8).pin_memory(),
                          torch.empty(pipes[q].counts[:B].shape, dtype=torch.int32).pin_memory(),
-                         torch.empty(outs[q].shape, dtype=torch.int32).pin_memory()])
+                         torch.empty(outs[q].shape, dtype=torch.int32).pin_memory()] +
+                        ([torch.empty(t.shape, dtype=torch.float32).pin_memory() for t in stereo[2][q]] if stereo else []))
     h2d = fr[0].numel() + (sum(a.numel() for a in hin[0]) if window else 0)
     d2h = sum(t.numel() * t.element_size() for t in host_out[0])
 
     def step(s):
         i, q = s % n_host, s % P
-        d, (kh, dh, ch, oh), pp, ot = dev_in[q], host_out[q], pipes[q], outs[q]
+        d, pp, ot = dev_in[q], pipes[q], outs[q]
+        kh, dh, ch, oh = host_out[q][:4]
         with torch.cuda.stream(streams[q]):
             d["fr"].copy_(fr[i], non_blocking=True)
             if window:
                 for dst, src in zip(d["in"], hin[i]):
                     dst.copy_(src, non_blocking=True)
             pp.extract(d["fr"], stream=streams[q])
+            if stereo:
+                pp.stereo(d["fr"], stereo[0], stereo[1], stereo[2][q][0], stereo[2][q][1], stream=streams[q])
             if window:
                 cm, pt, pf, qd, tk = d["in"]
                 pp.project(B, cm, pt.view(Q, 32), pf.view(torch.int32), d["qb"], th=th, stream=streams[q])
@@ -544,6 +562,9 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
             dh.copy_(pp.desc[:B], non_blocking=True)
             ch.copy_(pp.counts[:B], non_blocking=True)
             oh.copy_(ot, non_blocking=True)
+            if stereo:
+                host_out[q][4].copy_(stereo[2][q][0], non_blocking=True)
+                host_out[q][5].copy_(stereo[2][q][1], non_blocking=True)
 
     K = max(1, min(args.steps, 200))
     for s in range(3):
@@ -563,17 +584,25 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
     world = int(os.environ.get("WORLD_SIZE", 1))
     return {"value": B * world * K / (ms / 1000.0), "unit": "frames/s", "h2d_bytes_per_step": int(h2d),
             "d2h_bytes_per_step": int(d2h), "steps": K, "ms_per_step": ms / K, "ticks_in_flight": P,
-            "path": "pinned host -> H2D -> ss_orb_extract -> " + ("ss_project_points -> " if window else "") +
+            "path": "pinned host -> H2D -> ss_orb_extract -> " + ("ss_stereo_match -> " if stereo else "") +
+                    ("ss_project_points -> " if window else "") +
                     "ss_match_projection -> D2H (C ABI, no graphs)"}
 
 
 # ----------------------------------------------------------------------------- oracle (CPU) legs
 def _oracle_job(job):
     import oracle
-    (w, h, nf, frame, lm, mode, mp, th) = job
+    (w, h, nf, frame, lm, mode, mp, th, right) = job
     p = oracle.params(w, h, nf)
     t = time.perf_counter()
+    if frame is None:  # the right image of a stereo pair: handled by its left image's job
+        return 0.0
     kps, desc, counts = oracle.orb_extract(p, frame)
+    if right is not None:  # stereo pair: extract the right image, then O12
+        kr, dr, cr = oracle.orb_extract(p, right)
+        base = synth.STEREO_BASELINE["kitti"]
+        bf = float(np.float32(synth.INTRINSICS["kitti"][0] * base))
+        oracle.stereo_match(p, frame, right, kps, desc, counts, kr, dr, cr, bf, base)
     if mode == "window" and lm is not None:
         cm, pt, qd, tk = lm
         q = oracle.project_points(p, cm[None], pt, np.zeros(len(pt), np.int32), th)
@@ -597,7 +626,12 @@ def _jobs_for(cfg, frames_h, q_host, n, w, h, mp=None):
             cm, pt, pf, qd, tk = q_host[s % len(q_host)]
             sel = pf == b
             lm = (cm[b], pt[sel], qd[sel], tk[b])
-        jobs.append((w, h, cfg["nf"], frames_h[s, b], lm, cfg["mode"], mp, cfg["th"]))
+        if per_client == 2:  # stereo: the left image's job covers the pair
+            left = b % 2 == 0
+            jobs.append((w, h, cfg["nf"], frames_h[s, b] if left else None, lm, cfg["mode"], mp, cfg["th"],
+                         frames_h[s, b + 1] if left else None))
+        else:
+            jobs.append((w, h, cfg["nf"], frames_h[s, b], lm, cfg["mode"], mp, cfg["th"], None))
         i += 1
     return jobs
 
@@ -618,6 +652,7 @@ def cpu_baseline(args, cfg, frames_h, q_host, budget_s=15.0, mp=None):
     wall = time.perf_counter() - t
     return {"value": len(jobs) / wall, "unit": "frames/s", "cores": cores, "kind": "oracle",
             "sample": f"{len(jobs)} frames of the {args.config} workload (extract + " +
+                      ("stereo matching of each pair + " if cfg.get("stereo") else "") +
                       (f"its {cfg['queries']}-point local map projected and window-matched" if cfg["mode"] == "window"
                        else "4 keypoints brute-matched against the map") +
                       " each), one single-threaded oracle process per core",

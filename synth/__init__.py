@@ -6,5 +6,5 @@ matching, no projection): it only draws frames, map-point queries, local-map poi
 and statistics of the paper's workloads (recipe: SURVEY.md §8(d), restated in DESIGN.md §4).
 """
 from .gen import (SHAPES, frame_seed, make_frame, make_frames, make_stereo_pair, make_queries,
-                  make_brute_map, flip_bits, make_local_map, INTRINSICS, CAMERA_DTYPE,
+                  make_brute_map, flip_bits, make_local_map, INTRINSICS, STEREO_BASELINE, CAMERA_DTYPE,
                   MAP_POINT_DTYPE)  # noqa: F401

@@ -163,6 +163,8 @@ def make_brute_map(desc_list, n_map: int, seed: int, n_from_kps: int | None = No
 # fr1, KITTI 00 left) -- input geometry only; the projection itself is the method's (O11).
 INTRINSICS = {"euroc": (458.654, 457.296, 367.215, 248.375), "tum": (517.306, 516.469, 318.643, 255.314),
               "kitti": (718.856, 718.856, 607.1928, 185.2157)}
+# rectified stereo baseline (m) of the stereo shape (KITTI 00: bf = fx * b = 386.1448)
+STEREO_BASELINE = {"kitti": 0.5371657}
 CAMERA_DTYPE = np.dtype([("R", "<f4", (9,)), ("t", "<f4", (3,)), ("ow", "<f4", (3,)), ("fx", "<f4"),
                          ("fy", "<f4"), ("cx", "<f4"), ("cy", "<f4"), ("min_x", "<f4"), ("max_x", "<f4"),
                          ("min_y", "<f4"), ("max_y", "<f4"), ("pad", "<f4")])
