@@ -515,56 +515,66 @@ def run_ours(args, cfg):
 
 
 def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=1.0, stereo=None):
-    """Same ticks through the C ABI from pinned host buffers: H2D of the tick's inputs, extract +
-    match, D2H of all results, every step inside the timed region; ticks round-robin over the
-    in-flight contexts/streams so copies of one tick overlap compute of another."""
+    """Same ticks end to end from pinned host buffers through ONE C-ABI call per tick
+    (ss_track_tick: H2D of the tick's frames and local maps, extract, stereo, projection +
+    match or brute match, D2H of every output), all inside the timed region; ticks
+    round-robin over the in-flight contexts/streams so copies of one tick overlap compute of
+    another."""
+
     import torch
+
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
     P = len(pipes)
     n_host = min(len(frames_h), 8)
-    fr = [torch.from_numpy(frames_h[s]).pin_memory() for s in range(n_host)]
-    if window:  # per slot: cams, points, point_frame, qdesc, taken
-        hin = [[torch.from_numpy(np.ascontiguousarray(a).view(np.uint8).reshape(-1).copy()).pin_memory()
-                for a in q_host[s % len(q_host)]] for s in range(n_host)]
-    dev_in, host_out = [], []
-    for q in range(P):  # per in-flight context: device inputs, pinned host outputs
-        d = {"fr": torch.empty_like(fr[0], device=dev)}
-        if window:
-            d["in"] = [torch.empty_like(a, device=dev) for a in hin[0]]
-            d["qb"] = torch.empty((Q, 20), dtype=torch.uint8, device=dev)
-        dev_in.append(d)
-        host_out.append([torch.empty(pipes[q].kps[:B].shape, dtype=torch.uint8).pin_memory(),
-                         torch.empty(pipes[q].desc[:B].shape, dtype=torch.uint8).pin_memory(),
-                         torch.empty(pipes[q].counts[:B].shape, dtype=torch.int32).pin_memory(),
-                         torch.empty(outs[q].shape, dtype=torch.int32).pin_memory()] +
-                        ([torch.empty(t.shape, dtype=torch.float32).pin_memory() for t in stereo[2][q]] if stereo else []))
+    cap = pipes[0].cap
+    L = pipes[0].n_levels
+    H, W = frames_h.shape[2], frames_h.shape[3]
+
+    def pinned(a):
+        return torch.from_numpy(np.ascontiguousarray(a).view(np.uint8).reshape(-1).copy()).pin_memory()
+
+    fr = [pinned(frames_h[s]) for s in range(n_host)]
+    hin = [[pinned(a) for a in q_host[s % len(q_host)]] for s in range(n_host)] if window else None
+    rows = Q if window else B * cap
+    host_out = []
+    for q in range(P):
+        o = {"kps": torch.empty(B * cap * 20, dtype=torch.uint8).pin_memory(),
+             "desc": torch.empty(B * cap * 32, dtype=torch.uint8).pin_memory(),
+             "counts": torch.empty(B * (L + 1), dtype=torch.int32).pin_memory(),
+             "matches": torch.empty(rows * 3, dtype=torch.int32).pin_memory()}
+        if stereo:
+            o["uright"] = torch.empty((B // 2) * cap, dtype=torch.float32).pin_memory()
+            o["depth"] = torch.empty((B // 2) * cap, dtype=torch.float32).pin_memory()
+        host_out.append(o)
+    cfg = ss.window_cfg() if window else ss.brute_cfg()
+    ios = []
+    for q in range(P):
+        row = []
+        for i in range(n_host):
+            io = ss.ss_tick_io()
+            io.frames, io.frame_stride, io.pitch = fr[i].data_ptr(), H * W, W
+            if stereo:
+                io.bf, io.baseline = stereo[0], stereo[1]
+            if window:
+                cm, pt, pf, qd, tk = hin[i]
+                io.cams, io.n_points, io.points, io.point_frame = cm.data_ptr(), Q, pt.data_ptr(), pf.data_ptr()
+                io.point_desc, io.taken, io.th = qd.data_ptr(), tk.data_ptr(), th
+            else:
+                io.d_map_desc, io.n_map = map_desc.data_ptr(), map_desc.shape[0]
+            o = host_out[q]
+            io.kps, io.desc, io.counts = o["kps"].data_ptr(), o["desc"].data_ptr(), o["counts"].data_ptr()
+            io.matches = o["matches"].data_ptr()
+            if stereo:
+                io.uright, io.depth = o["uright"].data_ptr(), o["depth"].data_ptr()
+            row.append(io)
+        ios.append(row)
     h2d = fr[0].numel() + (sum(a.numel() for a in hin[0]) if window else 0)
-    d2h = sum(t.numel() * t.element_size() for t in host_out[0])
+    d2h = sum(t.numel() * t.element_size() for t in host_out[0].values())
+    handles = [st.cuda_stream for st in streams]
 
     def step(s):
         i, q = s % n_host, s % P
-        d, pp, ot = dev_in[q], pipes[q], outs[q]
-        kh, dh, ch, oh = host_out[q][:4]
-        with torch.cuda.stream(streams[q]):
-            d["fr"].copy_(fr[i], non_blocking=True)
-            if window:
-                for dst, src in zip(d["in"], hin[i]):
-                    dst.copy_(src, non_blocking=True)
-            pp.extract(d["fr"], stream=streams[q])
-            if stereo:
-                pp.stereo(d["fr"], stereo[0], stereo[1], stereo[2][q][0], stereo[2][q][1], stream=streams[q])
-            if window:
-                cm, pt, pf, qd, tk = d["in"]
-                pp.project(B, cm, pt.view(Q, 32), pf.view(torch.int32), d["qb"], th=th, stream=streams[q])
-                pp.match_window(B, d["qb"], qd.view(Q, 32), ot, taken=tk, stream=streams[q])
-            else:
-                pp.match_brute(B, map_desc, ot, stream=streams[q])
-            kh.copy_(pp.kps[:B], non_blocking=True)
-            dh.copy_(pp.desc[:B], non_blocking=True)
-            ch.copy_(pp.counts[:B], non_blocking=True)
-            oh.copy_(ot, non_blocking=True)
-            if stereo:
-                host_out[q][4].copy_(stereo[2][q][0], non_blocking=True)
-                host_out[q][5].copy_(stereo[2][q][1], non_blocking=True)
+        ss.ss_track_tick(pipes[q].ctx, B, cfg, ios[q][i], handles[q])
 
     K = max(1, min(args.steps, 200))
     for s in range(3):
@@ -584,9 +594,10 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
     world = int(os.environ.get("WORLD_SIZE", 1))
     return {"value": B * world * K / (ms / 1000.0), "unit": "frames/s", "h2d_bytes_per_step": int(h2d),
             "d2h_bytes_per_step": int(d2h), "steps": K, "ms_per_step": ms / K, "ticks_in_flight": P,
-            "path": "pinned host -> H2D -> ss_orb_extract -> " + ("ss_stereo_match -> " if stereo else "") +
-                    ("ss_project_points -> " if window else "") +
-                    "ss_match_projection -> D2H (C ABI, no graphs)"}
+            "path": "pinned host -> ss_track_tick (one C-ABI call per tick: H2D, ss_orb_extract, " +
+                    ("ss_stereo_match, " if stereo else "") +
+                    ("ss_project_points, ss_match_projection WINDOW" if window else "ss_match_projection BRUTE") +
+                    ", D2H of all outputs; no graphs)"}
 
 
 # ----------------------------------------------------------------------------- oracle (CPU) legs

@@ -206,6 +206,51 @@ ss_status ss_stereo_match(ss_ctx* ctx, int32_t n_pairs, const uint8_t* d_frames,
                           const ss_keypoint* d_kps, const uint8_t* d_desc, const int32_t* d_counts, float bf,
                           float baseline, float* d_uright, float* d_depth, ss_stream_t stream);
 
+/* ---- one tracking tick from host memory (the native executor of a client batch) ---- */
+
+/* Inputs and outputs of ss_track_tick, all HOST pointers (page-locked memory makes the copies
+ * asynchronous; pageable memory works but the copies then block).  NULL = unused. */
+typedef struct {
+  /* n_frames frames, frame f row y at frames + f*frame_stride + y*pitch (pitch >= width) */
+  const uint8_t* frames;
+  int64_t frame_stride;
+  int32_t pitch;
+  /* stereo (O12): bf > 0 and baseline > 0 match pairs (2i, 2i+1); 0 = no stereo */
+  float bf, baseline;
+  /* WINDOW (search local points, O11 + O9): cams [n_frames], points / point_frame /
+   * point_desc [n_points], taken [n_frames][kp_capacity] (may be NULL), projection th */
+  const ss_camera* cams;
+  int32_t n_points;
+  const ss_map_point* points;
+  const int32_t* point_frame;
+  const uint8_t* point_desc;
+  const uint8_t* taken;
+  float th;
+  /* BRUTE (O10): a DEVICE-resident map [n_map][32] (a shared map is uploaded once) */
+  const uint8_t* d_map_desc;
+  int32_t n_map;
+  /* outputs: kps [n_frames][kp_capacity], desc [n_frames][kp_capacity][32], counts
+   * [n_frames][n_levels+1], matches [n_points] (WINDOW) or [n_frames][kp_capacity] (BRUTE),
+   * uright / depth [n_frames/2][kp_capacity] (stereo).  Any output may be NULL (not copied). */
+  ss_keypoint* kps;
+  uint8_t* desc;
+  int32_t* counts;
+  ss_match* matches;
+  float* uright;
+  float* depth;
+} ss_tick_io;
+
+/* One tick of the hot path for a batch of client frames, enqueued on `stream` from a single
+ * call: host -> device copies into ctx-owned staging buffers (sized at ss_create: max_frames
+ * frames, max_queries points), ss_orb_extract, ss_stereo_match (if io->bf > 0),
+ * ss_project_points + ss_match_projection WINDOW (cfg->mode == SS_MATCH_WINDOW, n_points > 0)
+ * or ss_match_projection BRUTE (cfg->mode == SS_MATCH_BRUTE), device -> host copies of the
+ * outputs.  Asynchronous: outputs are valid once the stream reaches the end of the call; the
+ * caller must not reuse the ctx for another tick before then.  Same results and errors as
+ * the individual calls (SS_ECAPACITY when n_frames > max_frames or n_points > max_queries). */
+ss_status ss_track_tick(ss_ctx* ctx, int32_t n_frames, const ss_match_cfg* cfg, const ss_tick_io* io,
+                        ss_stream_t stream);
+
 /* ---- profiling hook (bench.py; does not synchronise) ---- */
 
 /* When n_events > 0, every following ss_orb_extract / ss_match_projection records the

@@ -145,6 +145,21 @@ struct ss_ctx {
   uint64_t* phase_ts = nullptr;  // distribution phase timestamps [max_frames][L][16] (debug hook)
   unsigned long long* partial = nullptr;
   int32_t* stereo_sad = nullptr;  // O12: accepted SAD per left keypoint [max_frames/2][cap]
+  // ss_track_tick staging (device copies of the host inputs / outputs of a tick)
+  uint8_t* io_frames = nullptr;   // [max_frames][H][io_pitch]
+  int32_t io_pitch = 0;
+  ss_keypoint* io_kps = nullptr;
+  uint8_t* io_desc = nullptr;
+  int32_t* io_counts = nullptr;
+  ss_camera* io_cams = nullptr;
+  ss_map_point* io_points = nullptr;
+  int32_t* io_pf = nullptr;
+  uint8_t* io_pdesc = nullptr;
+  uint8_t* io_taken = nullptr;
+  ss_mp_query* io_queries = nullptr;
+  ss_match* io_matches = nullptr;
+  float* io_uright = nullptr;
+  float* io_depth = nullptr;
   int8_t* brute_qexp = nullptr;  // BRUTE: keypoint descriptors expanded to s8 +-1 (k_brute_tc.cu)
   int8_t* brute_mexp = nullptr;  // BRUTE: map descriptors expanded to s8 +-1
   int n_sm = 148;
@@ -184,7 +199,9 @@ void free_ctx(ss_ctx* c) {
   cudaSetDevice(c->device);
   void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr_plan, c->pyr_gtab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
                   c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->rowidx, c->phase_ts,
-                  c->brute_qexp, c->brute_mexp, c->stereo_sad};
+                  c->brute_qexp, c->brute_mexp, c->stereo_sad, c->io_frames, c->io_kps, c->io_desc, c->io_counts,
+                  c->io_cams, c->io_points, c->io_pf, c->io_pdesc, c->io_taken, c->io_queries, c->io_matches,
+                  c->io_uright, c->io_depth};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
@@ -439,6 +456,23 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->rowidx, sizeof(uint16_t) * F * match_rows_per_frame(g));
   ALLOC(c->phase_ts, sizeof(uint64_t) * F * L * 16);
   ALLOC(c->stereo_sad, sizeof(int32_t) * ((F + 1) / 2) * g.kp_capacity);
+  c->io_pitch = (g.W + 15) & ~15;
+  {
+    const int64_t Qm = std::max<int64_t>(max_queries, 1);
+    ALLOC(c->io_frames, (size_t)F * g.H * c->io_pitch);
+    ALLOC(c->io_kps, sizeof(ss_keypoint) * F * g.kp_capacity);
+    ALLOC(c->io_desc, (size_t)F * g.kp_capacity * SS_DESC_BYTES);
+    ALLOC(c->io_counts, sizeof(int32_t) * F * (L + 1));
+    ALLOC(c->io_cams, sizeof(ss_camera) * F);
+    ALLOC(c->io_points, sizeof(ss_map_point) * Qm);
+    ALLOC(c->io_pf, sizeof(int32_t) * Qm);
+    ALLOC(c->io_pdesc, (size_t)Qm * SS_DESC_BYTES);
+    ALLOC(c->io_taken, (size_t)F * g.kp_capacity);
+    ALLOC(c->io_queries, sizeof(ss_mp_query) * Qm);
+    ALLOC(c->io_matches, sizeof(ss_match) * std::max<int64_t>(Qm, F * g.kp_capacity));
+    ALLOC(c->io_uright, sizeof(float) * ((F + 1) / 2) * g.kp_capacity);
+    ALLOC(c->io_depth, sizeof(float) * ((F + 1) / 2) * g.kp_capacity);
+  }
   if (max_map > 0) {
     ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
     ALLOC(c->brute_qexp, brute_tc_query_bytes(F * g.kp_capacity));
@@ -629,6 +663,84 @@ ss_status ss_project_points(ss_ctx* c, int32_t n_frames, const ss_camera* d_cams
   prof_mark(c, s);
   SS_CUDA_TRY(launch_project(c->g, n_frames, d_cams, n_points, d_points, d_point_frame, th, d_queries, s));
   prof_mark(c, s);
+  return SS_OK;
+}
+
+ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, const ss_tick_io* io,
+                        ss_stream_t stream) {
+  if (!c || !cfg || !io) return fail(SS_EINVAL, "NULL ctx/cfg/io");
+  if (n_frames < 0 || io->n_points < 0 || io->n_map < 0) return fail(SS_EINVAL, "negative size");
+  if (n_frames > c->max_frames) return fail(SS_ECAPACITY, "n_frames exceeds the ctx's max_frames");
+  if (n_frames == 0) return SS_OK;
+  if (!io->frames) return fail(SS_EINVAL, "NULL frames");
+  const Geom& g = c->g;
+  if (io->pitch < g.W || (n_frames > 1 && io->frame_stride < (int64_t)io->pitch * g.H))
+    return fail(SS_EINVAL, "bad pitch / frame stride");
+  const bool stereo = io->bf > 0.0f;
+  if (stereo && (n_frames & 1)) return fail(SS_EINVAL, "stereo needs an even frame count");
+  const bool window = cfg->mode == SS_MATCH_WINDOW && io->n_points > 0;
+  if (window) {
+    if (io->n_points > c->max_queries) return fail(SS_ECAPACITY, "n_points exceeds the ctx's max_queries");
+    if (!io->cams || !io->points || !io->point_frame || !io->point_desc) return fail(SS_EINVAL, "NULL window input");
+  }
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  const int cap = g.kp_capacity, L = g.L, P = c->io_pitch;
+  const int64_t fstride = (int64_t)g.H * P;
+  // host -> device
+  if (io->frame_stride == (int64_t)io->pitch * g.H || n_frames == 1) {
+    SS_CUDA_TRY(cudaMemcpy2DAsync(c->io_frames, P, io->frames, io->pitch, g.W, (size_t)g.H * n_frames,
+                                  cudaMemcpyHostToDevice, s));
+  } else {
+    for (int f = 0; f < n_frames; f++)
+      SS_CUDA_TRY(cudaMemcpy2DAsync(c->io_frames + f * fstride, P, io->frames + f * io->frame_stride, io->pitch, g.W,
+                                    g.H, cudaMemcpyHostToDevice, s));
+  }
+  if (window) {
+    const int64_t n = io->n_points;
+    SS_CUDA_TRY(cudaMemcpyAsync(c->io_cams, io->cams, sizeof(ss_camera) * n_frames, cudaMemcpyHostToDevice, s));
+    SS_CUDA_TRY(cudaMemcpyAsync(c->io_points, io->points, sizeof(ss_map_point) * n, cudaMemcpyHostToDevice, s));
+    SS_CUDA_TRY(cudaMemcpyAsync(c->io_pf, io->point_frame, sizeof(int32_t) * n, cudaMemcpyHostToDevice, s));
+    SS_CUDA_TRY(cudaMemcpyAsync(c->io_pdesc, io->point_desc, (size_t)n * SS_DESC_BYTES, cudaMemcpyHostToDevice, s));
+    if (io->taken)
+      SS_CUDA_TRY(cudaMemcpyAsync(c->io_taken, io->taken, (size_t)n_frames * cap, cudaMemcpyHostToDevice, s));
+  }
+  // the hot path
+  ss_status st = ss_orb_extract(c, n_frames, c->io_frames, fstride, P, c->io_kps, c->io_desc, c->io_counts, stream);
+  if (st != SS_OK) return st;
+  if (stereo) {
+    st = ss_stereo_match(c, n_frames / 2, c->io_frames, fstride, P, c->io_kps, c->io_desc, c->io_counts, io->bf,
+                         io->baseline, c->io_uright, c->io_depth, stream);
+    if (st != SS_OK) return st;
+  }
+  int64_t n_matches = 0;
+  if (window) {
+    st = ss_project_points(c, n_frames, c->io_cams, io->n_points, c->io_points, c->io_pf, io->th, c->io_queries,
+                           stream);
+    if (st != SS_OK) return st;
+    st = ss_match_projection(c, n_frames, c->io_kps, c->io_desc, c->io_counts, io->taken ? c->io_taken : nullptr,
+                             io->n_points, c->io_queries, c->io_pdesc, 0, cfg, c->io_matches, stream);
+    if (st != SS_OK) return st;
+    n_matches = io->n_points;
+  } else if (cfg->mode == SS_MATCH_BRUTE) {
+    st = ss_match_projection(c, n_frames, c->io_kps, c->io_desc, c->io_counts, nullptr, 0, nullptr, io->d_map_desc,
+                             io->n_map, cfg, c->io_matches, stream);
+    if (st != SS_OK) return st;
+    n_matches = (int64_t)n_frames * cap;
+  }
+  // device -> host
+  if (io->kps)
+    SS_CUDA_TRY(cudaMemcpyAsync(io->kps, c->io_kps, sizeof(ss_keypoint) * n_frames * cap, cudaMemcpyDeviceToHost, s));
+  if (io->desc)
+    SS_CUDA_TRY(cudaMemcpyAsync(io->desc, c->io_desc, (size_t)n_frames * cap * SS_DESC_BYTES, cudaMemcpyDeviceToHost, s));
+  if (io->counts)
+    SS_CUDA_TRY(cudaMemcpyAsync(io->counts, c->io_counts, sizeof(int32_t) * n_frames * (L + 1), cudaMemcpyDeviceToHost, s));
+  if (io->matches && n_matches > 0)
+    SS_CUDA_TRY(cudaMemcpyAsync(io->matches, c->io_matches, sizeof(ss_match) * n_matches, cudaMemcpyDeviceToHost, s));
+  if (stereo && io->uright)
+    SS_CUDA_TRY(cudaMemcpyAsync(io->uright, c->io_uright, sizeof(float) * (n_frames / 2) * cap, cudaMemcpyDeviceToHost, s));
+  if (stereo && io->depth)
+    SS_CUDA_TRY(cudaMemcpyAsync(io->depth, c->io_depth, sizeof(float) * (n_frames / 2) * cap, cudaMemcpyDeviceToHost, s));
   return SS_OK;
 }
 

@@ -52,6 +52,17 @@ class ss_match_cfg(C.Structure):
                 ("ratio_den", C.c_int32), ("dedup", C.c_int32)]
 
 
+class ss_tick_io(C.Structure):
+    """Host-side inputs / outputs of ss_track_tick (ss.h); pointer fields take addresses."""
+    _fields_ = [("frames", C.c_void_p), ("frame_stride", C.c_int64), ("pitch", C.c_int32),
+                ("bf", C.c_float), ("baseline", C.c_float),
+                ("cams", C.c_void_p), ("n_points", C.c_int32), ("points", C.c_void_p),
+                ("point_frame", C.c_void_p), ("point_desc", C.c_void_p), ("taken", C.c_void_p),
+                ("th", C.c_float), ("d_map_desc", C.c_void_p), ("n_map", C.c_int32),
+                ("kps", C.c_void_p), ("desc", C.c_void_p), ("counts", C.c_void_p), ("matches", C.c_void_p),
+                ("uright", C.c_void_p), ("depth", C.c_void_p)]
+
+
 # numpy views of the 20-/20-/12-byte records of ss.h
 KEYPOINT_DTYPE = np.dtype([("x", "<f4"), ("y", "<f4"), ("angle_deg", "<f4"), ("lx", "<u2"),
                            ("ly", "<u2"), ("level", "u1"), ("response", "u1"), ("reserved", "<u2")])
@@ -88,6 +99,7 @@ def lib():
         L.ss_match_projection.argtypes = [P, i32, P, P, P, P, i32, P, P, i32, C.POINTER(ss_match_cfg), P, P]
         L.ss_project_points.argtypes = [P, i32, P, i32, P, P, C.c_float, P, P]
         L.ss_stereo_match.argtypes = [P, i32, P, i64, i32, P, P, P, C.c_float, C.c_float, P, P, P]
+        L.ss_track_tick.argtypes = [P, i32, C.POINTER(ss_match_cfg), C.POINTER(ss_tick_io), P]
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
         L.ss_debug_candidates.argtypes = [P, i32, i32, P, P, P, i32, C.POINTER(i32)]
         L.ss_debug_overflow_count.argtypes = [P, C.POINTER(i32)]
@@ -95,7 +107,7 @@ def lib():
         L.ss_debug_phase_times.argtypes = [P, i32, i32, P, i32]
         L.ss_profile_next.argtypes = [P, C.POINTER(i32)]
         for fn in ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_orb_extract", "ss_match_projection",
-                   "ss_project_points", "ss_stereo_match",
+                   "ss_project_points", "ss_stereo_match", "ss_track_tick",
                    "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
                    "ss_profile_next", "ss_debug_phase_times"):
             getattr(L, fn).restype = C.c_int
@@ -104,7 +116,7 @@ def lib():
 
 
 EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "ss_orb_extract",
-            "ss_match_projection", "ss_project_points", "ss_stereo_match", "ss_profile_events", "ss_profile_next", "ss_debug_level",
+            "ss_match_projection", "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_profile_events", "ss_profile_next", "ss_debug_level",
             "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times")
 
 
@@ -164,6 +176,10 @@ def ss_match_projection(ctx, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_qu
     _check(lib().ss_match_projection(ctx, n_frames, _ptr(d_kps), _ptr(d_desc), _ptr(d_counts),
                                      _ptr(d_kp_taken), n_queries, _ptr(d_queries), _ptr(d_map_desc), n_map,
                                      C.byref(cfg), _ptr(d_out), _stream(stream)), ctx)
+
+
+def ss_track_tick(ctx, n_frames, cfg: ss_match_cfg, io: ss_tick_io, stream=None):
+    _check(lib().ss_track_tick(ctx, n_frames, C.byref(cfg), C.byref(io), _stream(stream)), ctx)
 
 
 def ss_stereo_match(ctx, n_pairs, d_frames, frame_stride, pitch, d_kps, d_desc, d_counts, bf, baseline, d_uright,

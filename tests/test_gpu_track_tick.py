@@ -1,0 +1,117 @@
+"""ss_track_tick (one C-ABI call per tick from host memory) vs the oracle: keypoints,
+descriptors, counts, stereo u_right / depth and window matches (search local points) of a
+KITTI-shaped stereo batch, and brute matches of an EuRoC batch, bit-exact (angle <= 1e-4 rad)."""
+import numpy as np
+import pytest
+
+import synth
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_conext_dhakalrwcr22_b200 import build as b
+    b.build()
+    return torch
+
+
+def _check_extract(p, kps, desc, counts, frames, ref):
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    out = []
+    for f in range(len(frames)):
+        rk, rd, rc = ref.orb_extract(p, frames[f])
+        n = int(rc[-1])
+        gk = kps[f].view(ss.KEYPOINT_DTYPE)
+        np.testing.assert_array_equal(counts[f], rc)
+        for fld in ("lx", "ly", "level", "response", "x", "y"):
+            np.testing.assert_array_equal(gk[fld][:n], rk[fld][:n], err_msg=fld)
+        da = np.radians(np.abs(gk["angle_deg"][:n].astype(np.float64) - rk["angle_deg"][:n]))
+        assert np.minimum(da, 2 * np.pi - da).max(initial=0) <= 1e-4
+        np.testing.assert_array_equal(desc[f][:n], rd[:n])
+        out.append((rk, rd, rc))
+    return out
+
+
+def test_track_tick_stereo_window(torch_cuda, ref):
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import OrbPipeline
+    w, h = synth.SHAPES["kitti"]
+    frames = np.stack([im for i in range(2) for im in synth.make_stereo_pair(w, h, seed=90 + i)])
+    B, Q, nf = 4, 2000, 2000
+    p = ref.params(w, h, nf)
+    cap = p.kp_capacity
+    rk, rd, rc = ref.orb_extract_batch(p, frames)
+    cm, pt, pf, qd, tk = synth.make_local_map(rk[::2], rd[::2], rc[::2], 8, p.scale_factor,
+                                              np.array(p.n_per_level[:8]), w, h, "kitti", Q // 2, seed=9)
+    pf = pf * 2
+    cams = np.zeros(B, synth.CAMERA_DTYPE)
+    cams[::2] = cm
+    taken = np.zeros((B, cap), np.uint8)
+    taken[::2] = tk
+    base = synth.STEREO_BASELINE["kitti"]
+    bf = float(np.float32(synth.INTRINSICS["kitti"][0] * base))
+    pin = lambda a: torch.from_numpy(np.ascontiguousarray(a).view(np.uint8).reshape(-1).copy()).pin_memory()
+    hf, hc, hp, hpf, hqd, htk = (pin(a) for a in (frames, cams, pt, pf, qd, taken))
+    o = {k: torch.zeros(n, dtype=torch.uint8).pin_memory()
+         for k, n in (("kps", B * cap * 20), ("desc", B * cap * 32), ("counts", B * 9 * 4), ("matches", Q * 12),
+                      ("uright", 2 * cap * 4), ("depth", 2 * cap * 4))}
+    io = ss.ss_tick_io()
+    io.frames, io.frame_stride, io.pitch, io.bf, io.baseline = hf.data_ptr(), h * w, w, bf, base
+    io.cams, io.n_points, io.points, io.point_frame = hc.data_ptr(), Q, hp.data_ptr(), hpf.data_ptr()
+    io.point_desc, io.taken, io.th = hqd.data_ptr(), htk.data_ptr(), 1.0
+    for k in o:
+        setattr(io, k, o[k].data_ptr())
+    pipe = OrbPipeline(w, h, nf, 8, max_frames=B, max_queries=Q)
+    ss.ss_track_tick(pipe.ctx, B, ss.window_cfg(), io)
+    torch.cuda.synchronize()
+    kps = o["kps"].numpy().reshape(B, cap, 20)
+    desc = o["desc"].numpy().reshape(B, cap, 32)
+    counts = o["counts"].numpy().view(np.int32).reshape(B, 9)
+    _check_extract(p, kps, desc, counts, frames, ref)
+    ur = o["uright"].numpy().view(np.float32).reshape(2, cap)
+    dp = o["depth"].numpy().view(np.float32).reshape(2, cap)
+    for i in range(2):
+        u_w, d_w, _ = ref.stereo_match(p, frames[2 * i], frames[2 * i + 1], rk[2 * i], rd[2 * i], rc[2 * i],
+                                       rk[2 * i + 1], rd[2 * i + 1], rc[2 * i + 1], bf, base)
+        n = int(rc[2 * i][-1])
+        np.testing.assert_array_equal(ur[i, :n].view(np.uint32), u_w[:n].view(np.uint32))
+        np.testing.assert_array_equal(dp[i, :n].view(np.uint32), d_w[:n].view(np.uint32))
+    q = ref.project_points(p, cams, pt, pf, 1.0)
+    want = ref.match_window(p, rk, rd, rc, taken, q, qd)
+    got = o["matches"].numpy().view(ref.MATCH_DTYPE).reshape(-1)
+    np.testing.assert_array_equal(got, want)
+    assert (got["idx"] >= 0).sum() > 100
+    pipe.close()
+
+
+def test_track_tick_brute(torch_cuda, ref):
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import OrbPipeline
+    w, h = synth.SHAPES["euroc"]
+    B, nf, n_map = 3, 1250, 3000
+    frames = synth.make_frames(w, h, B, cfg=5)
+    p = ref.params(w, h, nf)
+    cap = p.kp_capacity
+    rk, rd, rc = ref.orb_extract_batch(p, frames)
+    mp = synth.make_brute_map([rd[b][: rc[b][-1]] for b in range(B)], n_map, seed=3, n_from_kps=1000)
+    d_map = torch.from_numpy(mp).cuda()
+    hf = torch.from_numpy(frames.copy()).pin_memory()
+    hm = torch.zeros(B * cap * 12, dtype=torch.uint8).pin_memory()
+    io = ss.ss_tick_io()
+    io.frames, io.frame_stride, io.pitch = hf.data_ptr(), h * w, w
+    io.d_map_desc, io.n_map, io.matches = d_map.data_ptr(), n_map, hm.data_ptr()
+    pipe = OrbPipeline(w, h, nf, 8, max_frames=B, max_map=n_map)
+    ss.ss_track_tick(pipe.ctx, B, ss.brute_cfg(), io)
+    torch.cuda.synchronize()
+    got = hm.numpy().view(ref.MATCH_DTYPE).reshape(B, cap)
+    want = ref.match_brute(p, rd, rc, mp, 50, 3, 4)
+    for b in range(B):
+        n = int(rc[b][-1])
+        np.testing.assert_array_equal(got[b, :n], want[b, :n])
+    pipe.close()
