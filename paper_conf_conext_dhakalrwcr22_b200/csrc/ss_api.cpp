@@ -685,12 +685,16 @@ ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, co
   }
   SS_CUDA_TRY(cudaSetDevice(c->device));
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-  const int cap = g.kp_capacity, L = g.L, P = c->io_pitch;
-  const int64_t fstride = (int64_t)g.H * P;
-  // host -> device
-  if (io->frame_stride == (int64_t)io->pitch * g.H || n_frames == 1) {
-    SS_CUDA_TRY(cudaMemcpy2DAsync(c->io_frames, P, io->frames, io->pitch, g.W, (size_t)g.H * n_frames,
-                                  cudaMemcpyHostToDevice, s));
+  const int cap = g.kp_capacity, L = g.L;
+  // host -> device.  Frames stored densely (pitch <= the staging pitch, frame_stride = H *
+  // pitch) go in ONE linear copy and keep their pitch; anything else is repacked by 2-D
+  // copies (a 2-D copy moves row by row, several times slower for 0.3-0.5 MB frames).
+  int P = c->io_pitch;
+  int64_t fstride = (int64_t)g.H * P;
+  if (io->pitch <= c->io_pitch && (n_frames == 1 || io->frame_stride == (int64_t)io->pitch * g.H)) {
+    P = io->pitch;
+    fstride = (int64_t)g.H * P;
+    SS_CUDA_TRY(cudaMemcpyAsync(c->io_frames, io->frames, (size_t)fstride * n_frames, cudaMemcpyHostToDevice, s));
   } else {
     for (int f = 0; f < n_frames; f++)
       SS_CUDA_TRY(cudaMemcpy2DAsync(c->io_frames + f * fstride, P, io->frames + f * io->frame_stride, io->pitch, g.W,

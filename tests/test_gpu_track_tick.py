@@ -25,7 +25,7 @@ def _check_extract(p, kps, desc, counts, frames, ref):
     for f in range(len(frames)):
         rk, rd, rc = ref.orb_extract(p, frames[f])
         n = int(rc[-1])
-        gk = kps[f].view(ss.KEYPOINT_DTYPE)
+        gk = np.ascontiguousarray(kps[f]).reshape(-1).view(ss.KEYPOINT_DTYPE)
         np.testing.assert_array_equal(counts[f], rc)
         for fld in ("lx", "ly", "level", "response", "x", "y"):
             np.testing.assert_array_equal(gk[fld][:n], rk[fld][:n], err_msg=fld)
