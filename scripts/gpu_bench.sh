@@ -21,7 +21,7 @@ if [ "${SKIP_NCU:-0}" != "1" ]; then
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_$TAG.csv \
      python bench.py --steps 20 --warmup 3 --ring 8 --no-cpu-baseline ${NCU_BENCH_ARGS:-} > $OUT/ncu_bench_$TAG.log 2>&1
   echo "ncu list rc=$?"
-  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:"${NCU_KERNELS:-fast_bands|distribute|describe|match_window|pyramid}" \
+  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:"${NCU_KERNELS:-fast_bands|distribute|describe|match_window|pyramid|project|match_prepare|match_window_resolve}" \
      -s ${NCU_SKIP:-40} -c ${NCU_COUNT:-12} -o $OUT/prof_$TAG -f \
      python bench.py --steps 20 --warmup 3 --ring 8 --no-cpu-baseline ${NCU_BENCH_ARGS:-} > $OUT/ncu_full_$TAG.log 2>&1
   echo "ncu full rc=$?"
