@@ -88,6 +88,8 @@ def lib():
         _lib.ref_rhe_div_sqrt.restype = i32
         _lib.ref_descriptor.argtypes = [P, C.c_int, C.c_int, C.c_int, i32, i32, P]
         _lib.ref_orb_extract.argtypes = [C.POINTER(RefParams), P, C.c_int, P, P, P]
+        _lib.ref_orb_extract_mode.argtypes = [C.POINTER(RefParams), P, C.c_int, C.c_int, P, P, P]
+        _lib.ref_distribute_grid.argtypes = [C.POINTER(RefParams), C.c_int, P, P, P, C.c_int, C.c_int, P]
         _lib.ref_hamming.argtypes = [P, P]
         _lib.ref_hamming.restype = i32
         _lib.ref_match_window.argtypes = [C.POINTER(RefParams), C.c_int, P, P, P, P, C.c_int, P, P,
@@ -190,26 +192,27 @@ def descriptor(blurred: np.ndarray, lx: int, ly: int, m10: int, m01: int) -> np.
     return out
 
 
-def orb_extract(p: RefParams, img: np.ndarray):
-    """One frame -> (keypoints[kp_capacity] KEYPOINT_DTYPE, desc[kp_capacity,32], counts[L+1])."""
+def orb_extract(p: RefParams, img: np.ndarray, mode: int = 0):
+    """One frame -> (keypoints[kp_capacity] KEYPOINT_DTYPE, desc[kp_capacity,32], counts[L+1]).
+    mode 0 = quadtree distribution (O4), 1 = grid top-N (O4g)."""
     img = np.ascontiguousarray(img, dtype=np.uint8)
     kps = np.zeros(p.kp_capacity, KEYPOINT_DTYPE)
     desc = np.zeros((p.kp_capacity, 32), np.uint8)
     counts = np.zeros(p.n_levels + 1, np.int32)
-    n = lib().ref_orb_extract(C.byref(p), _p(img), img.shape[1], _p(kps), _p(desc), _p(counts))
+    n = lib().ref_orb_extract_mode(C.byref(p), _p(img), img.shape[1], mode, _p(kps), _p(desc), _p(counts))
     if n < 0:
         raise RuntimeError("oracle extraction exceeded capacity")
     return kps, desc, counts
 
 
-def orb_extract_batch(p: RefParams, frames: np.ndarray):
+def orb_extract_batch(p: RefParams, frames: np.ndarray, mode: int = 0):
     """frames [B,H,W] -> kps [B,cap], desc [B,cap,32], counts [B,L+1]."""
     B = frames.shape[0]
     kps = np.zeros((B, p.kp_capacity), KEYPOINT_DTYPE)
     desc = np.zeros((B, p.kp_capacity, 32), np.uint8)
     counts = np.zeros((B, p.n_levels + 1), np.int32)
     for b in range(B):
-        kps[b], desc[b], counts[b] = orb_extract(p, frames[b])
+        kps[b], desc[b], counts[b] = orb_extract(p, frames[b], mode)
     return kps, desc, counts
 
 
@@ -275,3 +278,11 @@ def stereo_match(p: RefParams, left, right, kl, dl, cl, kr, dr, cr, bf, b):
     lib().ref_stereo_match(C.byref(p), _p(left), _p(right), left.shape[1], *[_p(a) for a in args],
                            float(bf), float(b), _p(ur), _p(dp), _p(sad))
     return ur, dp, sad
+
+
+def distribute_grid(p: RefParams, level: int, lx, ly, score, N: int) -> np.ndarray:
+    """O4g: indices (into the rank-ordered candidates) of the keys grid top-N keeps."""
+    lx, ly, score = (np.ascontiguousarray(a, dtype=np.int32) for a in (lx, ly, score))
+    out = np.zeros(max(len(lx), 1), np.int32)
+    n = lib().ref_distribute_grid(C.byref(p), level, _p(lx), _p(ly), _p(score), len(lx), N, _p(out))
+    return out[:n]

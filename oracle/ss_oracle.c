@@ -517,6 +517,57 @@ void ref_descriptor(const uint8_t* B, int pitch, int lx, int ly, int32_t m10, in
 }
 
 /* ---------------------------------------------------------------- O1..O8 */
+/* ------------------------------------------------ O4g grid top-N distribution */
+/* The north_star's alternative to the quadtree ("a per-level quadtree (or grid top-N)
+ * distribution"), reading (DESIGN.md §3 item 13): on level l with N
+ * = n_per_level[l] and the O3 candidates in rank order,
+ *   K = number of FAST cells with at least one candidate, q = ceil(N / K);
+ *   every cell keeps its q best candidates by (score desc, rank asc);
+ *   if more than N remain, the N best of them by (score desc, rank asc) are kept.
+ * A candidate's cell is (i, j) = ((ly - 16 - 3) / cell_h, (lx - 16 - 3) / cell_w), the O3
+ * detect-window tiling.  Returns the number kept (<= N); out_idx = indices into the input.
+ * Parity: no external reference exists (the definition is ours): hand-worked cases and
+ * invariants in tests/test_oracle_grid.py. */
+typedef struct { int score, rank, cell; } gcand;
+static int cmp_gcand(const void* a, const void* b) {  /* cell, then score desc, then rank */
+  const gcand* A = (const gcand*)a; const gcand* B = (const gcand*)b;
+  if (A->cell != B->cell) return A->cell < B->cell ? -1 : 1;
+  if (A->score != B->score) return A->score > B->score ? -1 : 1;
+  return A->rank < B->rank ? -1 : (A->rank > B->rank);
+}
+static int cmp_gbest(const void* a, const void* b) {  /* score desc, then rank */
+  const gcand* A = (const gcand*)a; const gcand* B = (const gcand*)b;
+  if (A->score != B->score) return A->score > B->score ? -1 : 1;
+  return A->rank < B->rank ? -1 : (A->rank > B->rank);
+}
+
+int ref_distribute_grid(const ref_params* p, int l, const int32_t* lx, const int32_t* ly, const int32_t* score,
+                        int n, int N, int32_t* out_idx) {
+  if (n <= 0 || N <= 0) return 0;
+  gcand* c = (gcand*)malloc(sizeof(gcand) * (size_t)n);
+  for (int i = 0; i < n; i++) {
+    int ci = (ly[i] - MIN_BORDER - 3) / p->cell_h[l], cj = (lx[i] - MIN_BORDER - 3) / p->cell_w[l];
+    c[i].score = score[i]; c[i].rank = i; c[i].cell = ci * p->cell_cols[l] + cj;
+  }
+  qsort(c, (size_t)n, sizeof(gcand), cmp_gcand);
+  int K = 0;
+  for (int i = 0; i < n; i++) if (i == 0 || c[i].cell != c[i - 1].cell) K++;
+  int q = (N + K - 1) / K;
+  gcand* pool = (gcand*)malloc(sizeof(gcand) * (size_t)n);
+  int np = 0, run = 0;
+  for (int i = 0; i < n; i++) {
+    run = (i > 0 && c[i].cell == c[i - 1].cell) ? run + 1 : 0;
+    if (run < q) pool[np++] = c[i];
+  }
+  if (np > N) {
+    qsort(pool, (size_t)np, sizeof(gcand), cmp_gbest);
+    np = N;
+  }
+  for (int i = 0; i < np; i++) out_idx[i] = pool[i].rank;
+  free(pool); free(c);
+  return np;
+}
+
 typedef struct { int lx, ly, score; } selkp;
 static int cmp_yx(const void* a, const void* b) {
   const selkp* A = (const selkp*)a; const selkp* B = (const selkp*)b;
@@ -524,8 +575,8 @@ static int cmp_yx(const void* a, const void* b) {
   return A->lx < B->lx ? -1 : (A->lx > B->lx ? 1 : 0);
 }
 
-int ref_orb_extract(const ref_params* p, const uint8_t* img, int pitch, ref_keypoint* kps,
-                    uint8_t* desc, int32_t* counts) {
+int ref_orb_extract_mode(const ref_params* p, const uint8_t* img, int pitch, int mode, ref_keypoint* kps,
+                         uint8_t* desc, int32_t* counts) {
   int64_t pb = ref_pyramid_bytes(p);
   uint8_t* pyr = (uint8_t*)malloc((size_t)pb);
   ref_pyramid(p, img, pitch, pyr);
@@ -545,8 +596,9 @@ int ref_orb_extract(const ref_params* p, const uint8_t* img, int pitch, ref_keyp
     int32_t *ky = kx + (nc > 0 ? nc : 1), *sel = kx + 2 * (nc > 0 ? nc : 1);
     for (int i = 0; i < nc; i++) { kx[i] = cx[i] - MIN_BORDER; ky[i] = cy[i] - MIN_BORDER; }
     int maxBX = w - EDGE_THRESHOLD + 3, maxBY = h - EDGE_THRESHOLD + 3;
-    int ns = ref_distribute(kx, ky, cs, nc, maxBX - MIN_BORDER, maxBY - MIN_BORDER,
-                            p->n_per_level[l], sel);
+    int ns = mode == 1 ? ref_distribute_grid(p, l, cx, cy, cs, nc, p->n_per_level[l], sel)
+                       : ref_distribute(kx, ky, cs, nc, maxBX - MIN_BORDER, maxBY - MIN_BORDER,
+                                        p->n_per_level[l], sel);
     if (ns > p->level_cap[l] || total + ns > p->kp_capacity) { ns = -1; }
     if (ns < 0) { free(kx); free(cx); free(M); free(pyr); return -1; }
     selkp* s = (selkp*)malloc(sizeof(selkp) * (size_t)(ns > 0 ? ns : 1));
@@ -573,6 +625,11 @@ int ref_orb_extract(const ref_params* p, const uint8_t* img, int pitch, ref_keyp
   }
   free(pyr);
   return total;
+}
+
+int ref_orb_extract(const ref_params* p, const uint8_t* img, int pitch, ref_keypoint* kps,
+                    uint8_t* desc, int32_t* counts) {
+  return ref_orb_extract_mode(p, img, pitch, 0, kps, desc, counts);
 }
 
 /* ---------------------------------------------------------------- O9 / O10 */

@@ -72,6 +72,12 @@ int32_t ref_rhe_div_sqrt(int64_t z, int64_t r2);
 void ref_descriptor(const uint8_t* blurred, int pitch, int lx, int ly, int32_t m10, int32_t m01,
                     uint8_t out[32]);
 /* O1..O8 for one frame.  kps[kp_capacity], desc[kp_capacity*32], counts[n_levels+1] (prefix). */
+/* O4g grid top-N (mode 1 of ref_orb_extract_mode): indices of the kept candidates. */
+int ref_distribute_grid(const ref_params* p, int level, const int32_t* lx, const int32_t* ly,
+                        const int32_t* score, int n, int N, int32_t* out_idx);
+/* O1..O8 with distribution mode 0 = quadtree (O4), 1 = grid top-N (O4g). */
+int ref_orb_extract_mode(const ref_params* p, const uint8_t* img, int pitch, int mode,
+                         ref_keypoint* kps, uint8_t* desc, int32_t* counts);
 int ref_orb_extract(const ref_params* p, const uint8_t* img, int pitch,
                     ref_keypoint* kps, uint8_t* desc, int32_t* counts);
 int32_t ref_hamming(const uint8_t* a, const uint8_t* b);
