@@ -232,6 +232,8 @@ def run_ours(args, cfg):
     Q = cfg["queries"] * len(clients)
     window = cfg["mode"] == "window"
     pipe = OrbPipeline(w, h, cfg["nf"], L, max_frames=B, max_queries=max(Q, 1), max_map=cfg["map"], device=local)
+    dist_mode = ss.SS_DIST_GRID_TOPN if args.dist == "grid" else ss.SS_DIST_QUADTREE
+    pipe.set_distribution(dist_mode)
     p = pipe.params
     cap = p.kp_capacity
     props = torch.cuda.get_device_properties(dev)
@@ -318,6 +320,8 @@ def run_ours(args, cfg):
     P = max(1, args.inflight)
     pipes = [pipe] + [OrbPipeline(w, h, cfg["nf"], L, max_frames=B, max_queries=max(Q, 1), max_map=cfg["map"],
                                   device=local) for _ in range(P - 1)]
+    for pp in pipes:
+        pp.set_distribution(dist_mode)
     outs = [out] + [torch.zeros_like(out) for _ in range(P - 1)]
     qbufs = [torch.zeros((max(Q, 1), 20), dtype=torch.uint8, device=dev) for _ in range(P)]  # projected queries
     npairs = B // 2 if stereo else 0
@@ -488,7 +492,8 @@ def run_ours(args, cfg):
                    "parallelism": f"dp{world} (clients sharded over GPUs)",
                    "l2": f"inputs ring of {n_slots} distinct slots = {n_slots * slot_bytes / 2**20:.0f} MiB "
                          f"> L2 {l2 / 2**20:.0f} MiB (no flush)",
-                   "cuda_graphs": True, "ticks_in_flight": P, "setup_s": round(setup_s, 1)},
+                   "cuda_graphs": True, "ticks_in_flight": P, "setup_s": round(setup_s, 1),
+                   "distribution": "grid top-N (O4g)" if args.dist == "grid" else "quadtree (O4)"},
         "latency_ms": {"p50": float(np.percentile(step_ms, 50)), "p99": float(np.percentile(step_ms, 99)),
                        "samples": len(step_ms),
                        "note": f"per-frame latency = its tick's device time from start to end on its stream "
@@ -759,6 +764,8 @@ def main(argv=None):
     ap.add_argument("--inflight", type=int, default=4, help="ticks in flight (contexts/streams)")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--dist", choices=["quadtree", "grid"], default="quadtree",
+                    help="keypoint distribution: ORB-SLAM quadtree (O4) or grid top-N (O4g)")
     args = ap.parse_args(argv)
     assert args.warmup >= 3, "at least 3 warm-up steps"
     cfg = CONFIGS[args.config]

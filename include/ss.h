@@ -206,6 +206,15 @@ ss_status ss_stereo_match(ss_ctx* ctx, int32_t n_pairs, const uint8_t* d_frames,
                           const ss_keypoint* d_kps, const uint8_t* d_desc, const int32_t* d_counts, float bf,
                           float baseline, float* d_uright, float* d_depth, ss_stream_t stream);
 
+/* Keypoint distribution of the following ss_orb_extract calls on ctx (default quadtree):
+ * SS_DIST_QUADTREE = ORB-SLAM's DistributeOctTree reading (O4); SS_DIST_GRID_TOPN = grid
+ * top-N (O4g: K = FAST cells with a candidate, q = ceil(N_l / K), each cell keeps its q best
+ * by (score desc, rank asc), then the N_l best of those; <= N_l keypoints per level).
+ * SS_EINVAL for an unknown mode.  Host only. */
+#define SS_DIST_QUADTREE 0
+#define SS_DIST_GRID_TOPN 1
+ss_status ss_set_distribution(ss_ctx* ctx, int32_t mode);
+
 /* ---- one tracking tick from host memory (the native executor of a client batch) ---- */
 
 /* Inputs and outputs of ss_track_tick, all HOST pointers (page-locked memory makes the copies

@@ -144,6 +144,7 @@ struct ss_ctx {
   uint16_t* rowidx = nullptr;  // WINDOW matcher: first keypoint per (frame, level, row)
   uint64_t* phase_ts = nullptr;  // distribution phase timestamps [max_frames][L][16] (debug hook)
   unsigned long long* partial = nullptr;
+  int dist_mode = SS_DIST_QUADTREE;  // ss_set_distribution
   int32_t* stereo_sad = nullptr;  // O12: accepted SAD per left keypoint [max_frames/2][cap]
   // ss_track_tick staging (device copies of the host inputs / outputs of a tick)
   uint8_t* io_frames = nullptr;   // [max_frames][H][io_pitch]
@@ -542,8 +543,12 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands, g.band_count[0], c->cells, c->slots, c->cell_counts, q));
   prof_mark(c, q);
   prof_mark(c, q);
-  SS_CUDA_TRY(launch_distribute(g, n_frames, 0, 1, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts,
-                                c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, c->phase_ts, q));
+  if (c->dist_mode == SS_DIST_GRID_TOPN)
+    SS_CUDA_TRY(launch_distribute_grid(g, n_frames, 0, 1, c->cells, c->slots, c->cell_counts, c->selected,
+                                       c->sel_counts, q));
+  else
+    SS_CUDA_TRY(launch_distribute(g, n_frames, 0, 1, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts,
+                                  c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, c->phase_ts, q));
   prof_mark(c, q);
   if (q != s) SS_CUDA_TRY(cudaEventRecord(c->ev_join[0], q));
   prof_mark(c, s);
@@ -556,9 +561,13 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
                                 c->cells, c->slots, c->cell_counts, s));
   prof_mark(c, s);
   prof_mark(c, s);
-  SS_CUDA_TRY(launch_distribute(g, n_frames, 1, g.L - 1, c->cells, c->slots, c->cell_counts, c->selected,
-                                c->sel_counts, c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter,
-                                c->phase_ts, s));
+  if (c->dist_mode == SS_DIST_GRID_TOPN)
+    SS_CUDA_TRY(launch_distribute_grid(g, n_frames, 1, g.L - 1, c->cells, c->slots, c->cell_counts, c->selected,
+                                       c->sel_counts, s));
+  else
+    SS_CUDA_TRY(launch_distribute(g, n_frames, 1, g.L - 1, c->cells, c->slots, c->cell_counts, c->selected,
+                                  c->sel_counts, c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter,
+                                  c->phase_ts, s));
   prof_mark(c, s);
   if (q != s) SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[0], 0));
   prof_mark(c, s);
@@ -663,6 +672,13 @@ ss_status ss_project_points(ss_ctx* c, int32_t n_frames, const ss_camera* d_cams
   prof_mark(c, s);
   SS_CUDA_TRY(launch_project(c->g, n_frames, d_cams, n_points, d_points, d_point_frame, th, d_queries, s));
   prof_mark(c, s);
+  return SS_OK;
+}
+
+ss_status ss_set_distribution(ss_ctx* c, int32_t mode) {
+  if (!c) return fail(SS_EINVAL, "NULL ctx");
+  if (mode != SS_DIST_QUADTREE && mode != SS_DIST_GRID_TOPN) return fail(SS_EINVAL, "unknown distribution mode");
+  c->dist_mode = mode;
   return SS_OK;
 }
 

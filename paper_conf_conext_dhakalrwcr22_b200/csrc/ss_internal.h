@@ -180,6 +180,11 @@ cudaError_t launch_brute_tc(int n_slots, int n_map, const int8_t* qexp, const in
 cudaError_t launch_project(const Geom& g, int n_frames, const ss_camera* cams, int n_points, const ss_map_point* pts,
                            const int32_t* point_frame, float th, ss_mp_query* out, cudaStream_t s);
 
+// O4g grid top-N distribution (k_grid.cu), same outputs as launch_distribute.
+cudaError_t launch_distribute_grid(const Geom& g, int n_frames, int level0, int n_levels, const CellInfo* cells,
+                                   const uint32_t* slots, const int32_t* cell_counts, uint32_t* selected,
+                                   int32_t* sel_counts, cudaStream_t s);
+
 // O12 stereo matching (k_stereo.cu): one warp per left keypoint, then the per-pair outlier cut.
 cudaError_t launch_stereo(const Geom& g, int n_pairs, FrameSrc src, const ss_keypoint* kps, const uint8_t* desc,
                           const int32_t* counts, const uint16_t* rowidx, int rows_per_frame, float bf, float maxD,

@@ -31,6 +31,10 @@ class OrbPipeline:
         self.desc = torch.zeros((max_frames, self.cap, ss.DESC_BYTES), dtype=torch.uint8, device=self.device)
         self.counts = torch.zeros((max_frames, n_levels + 1), dtype=torch.int32, device=self.device)
 
+    def set_distribution(self, mode: int):
+        """ss.SS_DIST_QUADTREE (default) or ss.SS_DIST_GRID_TOPN for the following extracts."""
+        ss.ss_set_distribution(self.ctx, mode)
+
     def close(self):
         if self.ctx:
             ss.ss_destroy(self.ctx)

@@ -18,6 +18,7 @@ DESC_BYTES = 32
 
 SS_OK, SS_EINVAL, SS_ECAPACITY, SS_ECUDA, SS_EUNSUPPORTED = 0, -1, -2, -3, -4
 SS_MATCH_WINDOW, SS_MATCH_BRUTE = 0, 1
+SS_DIST_QUADTREE, SS_DIST_GRID_TOPN = 0, 1
 _STATUS = {0: "SS_OK", -1: "SS_EINVAL", -2: "SS_ECAPACITY", -3: "SS_ECUDA", -4: "SS_EUNSUPPORTED"}
 
 
@@ -99,6 +100,7 @@ def lib():
         L.ss_match_projection.argtypes = [P, i32, P, P, P, P, i32, P, P, i32, C.POINTER(ss_match_cfg), P, P]
         L.ss_project_points.argtypes = [P, i32, P, i32, P, P, C.c_float, P, P]
         L.ss_stereo_match.argtypes = [P, i32, P, i64, i32, P, P, P, C.c_float, C.c_float, P, P, P]
+        L.ss_set_distribution.argtypes = [P, i32]
         L.ss_track_tick.argtypes = [P, i32, C.POINTER(ss_match_cfg), C.POINTER(ss_tick_io), P]
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
         L.ss_debug_candidates.argtypes = [P, i32, i32, P, P, P, i32, C.POINTER(i32)]
@@ -107,7 +109,7 @@ def lib():
         L.ss_debug_phase_times.argtypes = [P, i32, i32, P, i32]
         L.ss_profile_next.argtypes = [P, C.POINTER(i32)]
         for fn in ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_orb_extract", "ss_match_projection",
-                   "ss_project_points", "ss_stereo_match", "ss_track_tick",
+                   "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_set_distribution",
                    "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
                    "ss_profile_next", "ss_debug_phase_times"):
             getattr(L, fn).restype = C.c_int
@@ -116,7 +118,8 @@ def lib():
 
 
 EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "ss_orb_extract",
-            "ss_match_projection", "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_profile_events", "ss_profile_next", "ss_debug_level",
+            "ss_match_projection", "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_set_distribution",
+            "ss_profile_events", "ss_profile_next", "ss_debug_level",
             "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times")
 
 
@@ -176,6 +179,10 @@ def ss_match_projection(ctx, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_qu
     _check(lib().ss_match_projection(ctx, n_frames, _ptr(d_kps), _ptr(d_desc), _ptr(d_counts),
                                      _ptr(d_kp_taken), n_queries, _ptr(d_queries), _ptr(d_map_desc), n_map,
                                      C.byref(cfg), _ptr(d_out), _stream(stream)), ctx)
+
+
+def ss_set_distribution(ctx, mode: int) -> None:
+    _check(lib().ss_set_distribution(ctx, mode), ctx)
 
 
 def ss_track_tick(ctx, n_frames, cfg: ss_match_cfg, io: ss_tick_io, stream=None):
