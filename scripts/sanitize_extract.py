@@ -1,4 +1,6 @@
-"""Small extract + window match for compute-sanitizer runs (memcheck / racecheck / synccheck).
+"""Small runs of every kernel for compute-sanitizer (memcheck / racecheck / synccheck): extract
+(quadtree and grid top-N), window match, projection, stereo, brute force (tensor cores;
+skipped when SANITIZE_BRUTE=0) and one ss_track_tick.
 
 usage: compute-sanitizer --tool racecheck python scripts/sanitize_extract.py
 """
@@ -33,6 +35,44 @@ def main():
     qd = rng.integers(0, 256, (512, 32), dtype=np.uint8)
     out = match_out(512, "cuda")
     pipe.match_window(B, to_device_records(q, "cuda"), torch.from_numpy(qd).cuda(), out)
+    # projection of a small local map, then the projected queries
+    cams = np.zeros(B, synth.CAMERA_DTYPE)
+    cams["R"] = np.eye(3, dtype=np.float32).ravel()
+    cams["fx"], cams["fy"], cams["cx"], cams["cy"] = 300.0, 300.0, w / 2, h / 2
+    cams["max_x"], cams["max_y"] = w, h
+    pts = np.zeros(512, synth.MAP_POINT_DTYPE)
+    pts["pos"] = np.stack([rng.uniform(-2, 2, 512), rng.uniform(-2, 2, 512), rng.uniform(-1, 8, 512)], 1)
+    pts["normal"] = [0.0, 0.0, 1.0]
+    pts["min_dist"], pts["max_dist"] = 0.5, 6.0
+    pf = rng.integers(-1, B + 1, 512).astype(np.int32)
+    qb = torch.zeros((512, 20), dtype=torch.uint8, device="cuda")
+    pipe.project(B, torch.from_numpy(cams.view(np.uint8).reshape(B, -1).copy()).cuda(),
+                 torch.from_numpy(pts.view(np.uint8).reshape(512, -1).copy()).cuda(), torch.from_numpy(pf).cuda(), qb)
+    pipe.match_window(B, qb, torch.from_numpy(qd).cuda(), out)
+    # stereo on the (frame 0, frame 1) pair
+    d_frames = torch.from_numpy(frames).cuda()
+    ur = torch.zeros((1, pipe.cap), dtype=torch.float32, device="cuda")
+    dp = torch.zeros_like(ur)
+    pipe.extract(d_frames)
+    pipe.stereo(d_frames, 200.0, 0.5, ur, dp)
+    # grid top-N distribution
+    pipe.set_distribution(ss.SS_DIST_GRID_TOPN)
+    pipe.extract(d_frames)
+    pipe.set_distribution(ss.SS_DIST_QUADTREE)
+    if os.environ.get("SANITIZE_BRUTE", "1") == "1":
+        mp = rng.integers(0, 256, (300, 32), dtype=np.uint8)
+        bp = OrbPipeline(w, h, 300, 4, max_frames=B, max_map=300)
+        bp.extract(d_frames)
+        bo = torch.zeros((B * bp.cap, 3), dtype=torch.int32, device="cuda")
+        bp.match_brute(B, torch.from_numpy(mp).cuda(), bo)
+        torch.cuda.synchronize()
+        bp.close()
+    # one tick from host memory
+    hf = torch.from_numpy(frames.copy()).pin_memory()
+    hk = torch.zeros(B * pipe.cap * 20, dtype=torch.uint8).pin_memory()
+    io = ss.ss_tick_io()
+    io.frames, io.frame_stride, io.pitch, io.kps = hf.data_ptr(), h * w, w, hk.data_ptr()
+    ss.ss_track_tick(pipe.ctx, B, ss.window_cfg(), io)
     torch.cuda.synchronize()
     print("sanitize run ok", int(counts[:, -1].sum()), "keypoints")
 
