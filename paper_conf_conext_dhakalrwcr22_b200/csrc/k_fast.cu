@@ -12,8 +12,9 @@
 //     min/max over the 16 arcs of 9 runs on DPX three-way min/max (VIMNMX3.U16x2) -- no
 //     pre-test, no divergence, one 32-bit store of 4 scores;
 //  3. one warp per cell, one lane per cell row: strict 8-neighbour maxima inside the cell's
-//     window (neighbours in the next cell are ignored: per-cell ROI semantics) as 64-bit row
-//     masks, the cell's threshold (iniTh if any maximum beats it, else minTh), and the
+//     window (neighbours in the next cell are ignored: per-cell ROI semantics), four columns
+//     per step as 16x2 three-way max trees over cell-masked neighbour words, as 64-bit row
+//     masks; the cell's threshold (iniTh if any maximum beats it, else minTh), and the
 //     survivors written in raster order (warp prefix sum of the row counts).
 //
 //   M(p) = max_s max( min_{k<9} d_{s+k}, min_{k<9} -d_{s+k} ),  d_k = I(p) - I(p + R_k)
@@ -188,29 +189,47 @@ __global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(const __grid_
     for (int hh = 0; hh < 2; hh++) {
       const int y = lane + 32 * hh;
       if (y < Dh) {
-        const uint8_t* rowp = Mb + (y + 1) * mbw + cx0;
-        // pass 1: scores above minTh (independent loads, 8 per step), pass 2: their neighbours
-        unsigned long long cand = 0ull;
-        for (int x0 = 0; x0 < cw; x0 += 8) {
-          int m[8];
+        // strict 8-neighbour maxima of the row, four columns per step on 16x2 lanes: words
+        // A_j = cell columns [4j-4, 4j) of rows y-1, y, y+1 with every byte outside the cell
+        // zeroed (ROI semantics: neighbours in other cells are ignored; a zero never beats a
+        // score > minTh), so the test needs no edge cases.
+        const int base = cx0 - 4, a0 = base & ~3;
+        const uint32_t sh = 8u * (uint32_t)(base & 3);
+        const uint32_t* pr0 = reinterpret_cast<const uint32_t*>(Mb + y * mbw + a0);
+        const uint32_t* pr1 = reinterpret_cast<const uint32_t*>(Mb + (y + 1) * mbw + a0);
+        const uint32_t* pr2 = reinterpret_cast<const uint32_t*>(Mb + (y + 2) * mbw + a0);
+        auto aword = [&](const uint32_t* pr, int j) -> uint32_t {
+          const int valid = cw - (4 * j - 4);  // bytes of A_j inside the cell (j >= 1)
+          const uint32_t v = __funnelshift_r(pr[j], pr[j + 1], sh);
+          return valid >= 4 ? v : (valid <= 0 ? 0u : v & (0xFFFFFFFFu >> (8 * (4 - valid))));
+        };
+        uint32_t p0 = 0u, p1 = 0u, p2 = 0u;  // A_k of rows y-1, y, y+1
+        uint32_t c0w = aword(pr0, 1), c1w = aword(pr1, 1), c2w = aword(pr2, 1);  // A_{k+1}
+        const uint32_t tmin1 = (uint32_t)(tmin + 1) * 0x10001u, tini1 = (uint32_t)(tini + 1) * 0x10001u;
+        const int nk = (cw + 3) >> 2;
+        for (int k = 0; k < nk; k++) {
+          const uint32_t n0 = aword(pr0, k + 2), n1 = aword(pr1, k + 2), n2 = aword(pr2, k + 2);
+          const uint32_t L0 = __byte_perm(p0, c0w, 0x6543), R0 = __byte_perm(c0w, n0, 0x4321);
+          const uint32_t L1 = __byte_perm(p1, c1w, 0x6543), R1 = __byte_perm(c1w, n1, 0x4321);
+          const uint32_t L2 = __byte_perm(p2, c2w, 0x6543), R2 = __byte_perm(c2w, n2, 0x4321);
+          uint32_t bmin = 0u, bini = 0u;
 #pragma unroll
-          for (int q = 0; q < 8; q++) m[q] = rowp[x0 + q];  // row has >= 8 B of slack past cw
-#pragma unroll
-          for (int q = 0; q < 8; q++)
-            if (m[q] > tmin && x0 + q < cw) cand |= 1ull << (x0 + q);
-        }
-        while (cand) {
-          const int x = __ffsll((long long)cand) - 1;
-          cand &= cand - 1;
-          const uint8_t* p = rowp + x;
-          const int m = p[0];
-          bool mx = m > p[-mbw] && m > p[mbw];
-          if (x > 0) mx = mx && m > p[-mbw - 1] && m > p[-1] && m > p[mbw - 1];
-          if (x < cw - 1) mx = mx && m > p[-mbw + 1] && m > p[1] && m > p[mbw + 1];
-          if (mx) {
-            kmin[hh] |= 1ull << x;
-            if (m > tini) kini[hh] |= 1ull << x;
+          for (int half = 0; half < 2; half++) {  // lanes: pixels (0, 2), then (1, 3)
+            const uint32_t sel = half ? 0x7371u : 0x7270u;
+            const uint32_t C = __byte_perm(c1w, 0, sel) | 0x80008000u;
+            const uint32_t nb =
+                __vimax3_u16x2(__vimax3_u16x2(__byte_perm(c0w, 0, sel), __byte_perm(L0, 0, sel), __byte_perm(R0, 0, sel)),
+                               __vimax3_u16x2(__byte_perm(c2w, 0, sel), __byte_perm(L2, 0, sel), __byte_perm(R2, 0, sel)),
+                               __vimax3_u16x2(__byte_perm(L1, 0, sel), __byte_perm(R1, 0, sel), 0u));
+            const uint32_t ok = (C - nb - 0x00010001u) & (C - tmin1) & 0x80008000u;  // > neighbours, > minTh
+            const uint32_t oi = ok & (C - tini1);                                       // and > iniTh
+            bmin |= ((ok >> 15) & 1u) << half | ((ok >> 31) & 1u) << (2 + half);
+            bini |= ((oi >> 15) & 1u) << half | ((oi >> 31) & 1u) << (2 + half);
           }
+          kmin[hh] |= (unsigned long long)bmin << (4 * k);
+          kini[hh] |= (unsigned long long)bini << (4 * k);
+          p0 = c0w, p1 = c1w, p2 = c2w;
+          c0w = n0, c1w = n1, c2w = n2;
         }
       }
     }
@@ -250,7 +269,7 @@ size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int*
   int m = (sw + 8 + 3) & ~3;  // + 8: the NMS reads 8 scores per step past a cell's last column
   if (((m >> 2) & 1) == 0) m += 4;  // odd word pitch: lane-per-row reads hit distinct banks
   *mbw = m;
-  *mband_bytes = ((g.max_band_h + 2) * m + 15) & ~15;
+  *mband_bytes = ((g.max_band_h + 2) * m + 16 + 15) & ~15;  // + 16: the NMS word reads pass the last row
   *nball = 0;
   return (size_t)*region_bytes + *mband_bytes;
 }
