@@ -60,6 +60,8 @@ CAMERA_DTYPE = np.dtype([("R", "<f4", (9,)), ("t", "<f4", (3,)), ("ow", "<f4", (
                          ("min_y", "<f4"), ("max_y", "<f4"), ("pad", "<f4")])
 MAP_POINT_DTYPE = np.dtype([("pos", "<f4", (3,)), ("normal", "<f4", (3,)), ("min_dist", "<f4"),
                             ("max_dist", "<f4")])
+FRAME_POINT_DTYPE = np.dtype([("pos", "<f4", (3,)), ("angle_deg", "<f4"), ("octave", "<i4"), ("reserved", "<i4")])
+assert FRAME_POINT_DTYPE.itemsize == 24
 assert CAMERA_DTYPE.itemsize == 96 and MAP_POINT_DTYPE.itemsize == 32
 assert KEYPOINT_DTYPE.itemsize == 20 and QUERY_DTYPE.itemsize == 20 and MATCH_DTYPE.itemsize == 12
 
@@ -98,6 +100,10 @@ def lib():
                                          C.c_int, C.c_int, C.c_int, C.c_int, P]
         _lib.ref_stereo_match.argtypes = [C.POINTER(RefParams), P, P, C.c_int, P, P, P, P, P, P, C.c_float, C.c_float,
                                           P, P, P]
+        _lib.ref_match_last_frame.argtypes = [C.POINTER(RefParams), C.c_int, P, P, C.c_float, P, P, P, P, P, P, P,
+                                              C.c_float, C.c_int, C.c_int, C.c_int, P, P]
+        _lib.ref_lf_rot_bin.argtypes = [C.c_float, C.c_float]
+        _lib.ref_lf_rot_bin.restype = C.c_int
         _lib.ref_project_points.argtypes = [C.POINTER(RefParams), C.c_int, P, C.c_int, P, P, C.c_float, P]
     return _lib
 
@@ -286,3 +292,29 @@ def distribute_grid(p: RefParams, level: int, lx, ly, score, N: int) -> np.ndarr
     out = np.zeros(max(len(lx), 1), np.int32)
     n = lib().ref_distribute_grid(C.byref(p), level, _p(lx), _p(ly), _p(score), len(lx), N, _p(out))
     return out[:n]
+
+
+def match_last_frame(p: RefParams, cams, last_cams, mb, kps, desc, counts, taken, pt_off, points, pdesc, th=15.0,
+                     th_high=100, check_orientation=1, min_matches=20):
+    """O13: -> (MATCH_DTYPE [n_points], kept matches per frame i32 [F])."""
+    cams = np.ascontiguousarray(cams, dtype=CAMERA_DTYPE)
+    lc = None if last_cams is None else np.ascontiguousarray(last_cams, dtype=CAMERA_DTYPE)
+    kps = np.ascontiguousarray(kps)
+    desc = np.ascontiguousarray(desc, dtype=np.uint8)
+    counts = np.ascontiguousarray(counts, dtype=np.int32)
+    tk = None if taken is None else np.ascontiguousarray(taken, dtype=np.uint8)
+    pt_off = np.ascontiguousarray(pt_off, dtype=np.int32)
+    points = np.ascontiguousarray(points, dtype=FRAME_POINT_DTYPE)
+    pdesc = np.ascontiguousarray(pdesc, dtype=np.uint8).reshape(-1, 32)
+    F = len(cams)
+    assert len(pt_off) == F + 1 and pt_off[-1] == len(points) == len(pdesc)
+    out = np.zeros(len(points), MATCH_DTYPE)
+    nm = np.zeros(F, np.int32)
+    lib().ref_match_last_frame(C.byref(p), F, _p(cams), None if lc is None else _p(lc), float(mb), _p(kps), _p(desc),
+                               _p(counts), None if tk is None else _p(tk), _p(pt_off), _p(points), _p(pdesc),
+                               float(th), int(th_high), int(check_orientation), int(min_matches), _p(out), _p(nm))
+    return out, nm
+
+
+def lf_rot_bin(angle_last: float, angle_cur: float) -> int:
+    return int(lib().ref_lf_rot_bin(float(angle_last), float(angle_cur)))

@@ -30,6 +30,10 @@
  *                    rot90 about z, viewCos = 1 along the normal); predicted level vs
  *                    ceil(log(ratio)/log(1.2)) away from level boundaries; each culling
  *                    rule isolated by a point that violates only it
+ *   O13 last frame : integer image shift of a fronto-parallel plane (every level-0 keypoint
+ *                    matched to its shifted twin at d = 0, rotation bin 0); hand-worked
+ *                    three-maxima / dedup / TH_HIGH / level-gate / retry cases; rotation-bin
+ *                    closed forms; numpy brute force of steps 1-4
  */
 #include "ss_oracle.h"
 
@@ -913,4 +917,150 @@ void ref_stereo_match(const ref_params* p, const uint8_t* left, const uint8_t* r
     }
   }
   free(acc); free(rlist); free(rstart); free(rcount); free(pyl); free(pyr);
+}
+
+/* ------------------------------------------- O13 frame-to-frame projection matching */
+/* ORB-SLAM2/3 ORBmatcher::SearchByProjection(CurrentFrame, LastFrame, th, bMono) as called by
+ * Tracking::TrackWithMotionModel [ext]: the "ORB-Matching" step of the paper's tracking-time
+ * breakdown (§5, Fig. 8: "feature extraction (ORB-Extraction), feature matching
+ * (ORB-Matching), pose prediction, and finally search local point").  SURVEY §8(f) F2;
+ * readings in DESIGN.md §3 item 14.  Per frame f, its last-frame points
+ * [pt_off[f], pt_off[f+1]) (a map point seen in the previous frame: world position, the
+ * previous keypoint's octave and angle), in ORB-SLAM's order:
+ *  1. Pc = R*Pw + t (O11's arithmetic); skip if Pc.z < 0; u = fx*X/Z + cx, v = fy*Y/Z + cy;
+ *     skip if outside [min_x, max_x] x [min_y, max_y];
+ *  2. radius = f32(th * scale[octave]); stereo direction (only when mb > 0 and last cameras
+ *     are given): tlc = R_last * ow_cur + t_last, forward iff tlc.z > mb, backward iff
+ *     -tlc.z > mb; level gate: forward [octave, L-1], backward [0, octave], else
+ *     [octave-1, octave+1] (GetFeaturesInArea(u, v, r, minLevel, maxLevel));
+ *  3. candidates: keypoints of frame f in the gate with |x-u| < r and |y-v| < r (f32), not
+ *     taken; best / second by (Hamming, keypoint index); accept iff best <= th_high
+ *     (TH_HIGH = 100; no ratio test in this matcher);
+ *  4. reading of ORB-SLAM's sequential claim (a keypoint matched by an earlier point is
+ *     skipped by later ones): every point is evaluated independently, then a keypoint claimed
+ *     by several accepted points keeps the min (distance, point index) (as O9);
+ *  5. rotation consistency (mbCheckOrientation): rot = angle_last - angle_cur (f32), +360 if
+ *     negative, bin = roundf(rot * f32(1/30)) (HISTO_LENGTH = 30, factor = 1.0f/HISTO_LENGTH,
+ *     literally), 30 -> 0; ComputeThreeMaxima (strict >, earlier bin wins ties; drop the 2nd /
+ *     3rd maximum when below 0.1f * max1); matches in other bins are removed;
+ *  6. if min_matches > 0 and the frame kept fewer than min_matches matches, the whole frame is
+ *     matched again from step 1 with radius factor 2*th (TrackWithMotionModel's retry), and
+ *     the second result stands.
+ * Output per point: idx = keypoint index or -1, dist / dist2 = best / second distance of the
+ * last pass that evaluated it (256 = none).  Points whose octave is outside [0, L-1] have no
+ * candidates. */
+#define HISTO_LENGTH 30
+
+static void lf_three_maxima(const int* hist, int* ind1, int* ind2, int* ind3) {
+  int max1 = 0, max2 = 0, max3 = 0;
+  *ind1 = *ind2 = *ind3 = -1;
+  for (int i = 0; i < HISTO_LENGTH; i++) {
+    int s = hist[i];
+    if (s > max1) { max3 = max2; max2 = max1; max1 = s; *ind3 = *ind2; *ind2 = *ind1; *ind1 = i; }
+    else if (s > max2) { max3 = max2; max2 = s; *ind3 = *ind2; *ind2 = i; }
+    else if (s > max3) { max3 = s; *ind3 = i; }
+  }
+  if ((float)max2 < 0.1f * (float)max1) { *ind2 = -1; *ind3 = -1; }
+  else if ((float)max3 < 0.1f * (float)max1) { *ind3 = -1; }
+}
+
+int ref_lf_rot_bin(float angle_last, float angle_cur) {
+  const float factor = 1.0f / HISTO_LENGTH;
+  float rot = angle_last - angle_cur;
+  if (rot < 0.0f) rot = rot + 360.0f;
+  float t = rot * factor;
+  int bin = (int)roundf(t);
+  if (bin == HISTO_LENGTH) bin = 0;
+  return bin;
+}
+
+/* one pass over frame f's points with window factor th; returns the kept match count */
+static int lf_frame_pass(const ref_params* p, int f, const ref_camera* c, int dir, const ref_keypoint* kps,
+                         const uint8_t* desc, const int32_t* counts, const uint8_t* taken, int i0, int i1,
+                         const ref_frame_point* pts, const uint8_t* pdesc, float th, int th_high,
+                         int check_orientation, ref_match* out, int* winner) {
+  int L = p->n_levels, cap = p->kp_capacity;
+  int n = counts[f * (L + 1) + L];
+  const ref_keypoint* fk = &kps[(size_t)f * cap];
+  for (int i = i0; i < i1; i++) {
+    out[i].idx = -1; out[i].dist = 256; out[i].dist2 = 256;
+    int o = pts[i].octave;
+    if (o < 0 || o >= L) continue;
+    const float* P = pts[i].pos;
+    float pc[3];
+    for (int r = 0; r < 3; r++) pc[r] = dot3(&c->R[3 * r], P) + c->t[r];
+    if (pc[2] < 0.0f) continue;
+    float u = c->fx * pc[0] / pc[2] + c->cx;
+    float v = c->fy * pc[1] / pc[2] + c->cy;
+    if (u < c->min_x || u > c->max_x) continue;
+    if (v < c->min_y || v > c->max_y) continue;
+    float radius = th * p->scale[o];
+    int lmin, lmax;
+    if (dir == 1) { lmin = o; lmax = L - 1; }
+    else if (dir == 2) { lmin = 0; lmax = o; }
+    else { lmin = o - 1; lmax = o + 1; }
+    int d1 = 256, d2 = 256, k1 = -1;
+    for (int k = 0; k < n; k++) {
+      if (fk[k].level < lmin || fk[k].level > lmax) continue;
+      if (taken && taken[(size_t)f * cap + k]) continue;
+      float dx = fk[k].x - u, dy = fk[k].y - v;
+      if (!(fabsf(dx) < radius && fabsf(dy) < radius)) continue;
+      int d = ref_hamming(pdesc + (size_t)i * 32, desc + ((size_t)f * cap + k) * 32);
+      if (d < d1) { d2 = d1; d1 = d; k1 = k; }
+      else if (d < d2) { d2 = d; }
+    }
+    out[i].dist = d1; out[i].dist2 = d2;
+    if (k1 >= 0 && d1 <= th_high) out[i].idx = k1;
+  }
+  /* step 4: dedup, min (distance, point index) per keypoint */
+  for (int k = 0; k < cap; k++) winner[k] = -1;
+  for (int i = i0; i < i1; i++) {
+    int k = out[i].idx;
+    if (k < 0) continue;
+    int w = winner[k];
+    if (w < 0 || out[i].dist < out[w].dist || (out[i].dist == out[w].dist && i < w)) winner[k] = i;
+  }
+  for (int i = i0; i < i1; i++)
+    if (out[i].idx >= 0 && winner[out[i].idx] != i) out[i].idx = -1;
+  /* step 5: rotation consistency */
+  if (check_orientation) {
+    int hist[HISTO_LENGTH] = {0};
+    for (int i = i0; i < i1; i++)
+      if (out[i].idx >= 0) hist[ref_lf_rot_bin(pts[i].angle_deg, fk[out[i].idx].angle_deg)]++;
+    int a, b, d;
+    lf_three_maxima(hist, &a, &b, &d);
+    for (int i = i0; i < i1; i++) {
+      if (out[i].idx < 0) continue;
+      int bin = ref_lf_rot_bin(pts[i].angle_deg, fk[out[i].idx].angle_deg);
+      if (bin != a && bin != b && bin != d) out[i].idx = -1;
+    }
+  }
+  int kept = 0;
+  for (int i = i0; i < i1; i++) kept += out[i].idx >= 0;
+  return kept;
+}
+
+void ref_match_last_frame(const ref_params* p, int F, const ref_camera* cams, const ref_camera* last_cams, float mb,
+                          const ref_keypoint* kps, const uint8_t* desc, const int32_t* counts, const uint8_t* taken,
+                          const int32_t* pt_off, const ref_frame_point* pts, const uint8_t* pdesc, float th,
+                          int th_high, int check_orientation, int min_matches, ref_match* out, int32_t* n_matches) {
+  int cap = p->kp_capacity;
+  int* winner = (int*)malloc(sizeof(int) * (size_t)(cap > 0 ? cap : 1));
+  for (int f = 0; f < F; f++) {
+    const ref_camera* c = &cams[f];
+    int dir = 0;
+    if (mb > 0.0f && last_cams) {
+      const ref_camera* cl = &last_cams[f];
+      float tz = dot3(&cl->R[6], c->ow) + cl->t[2];
+      if (tz > mb) dir = 1;
+      else if (-tz > mb) dir = 2;
+    }
+    int kept = lf_frame_pass(p, f, c, dir, kps, desc, counts, taken, pt_off[f], pt_off[f + 1], pts, pdesc, th,
+                             th_high, check_orientation, out, winner);
+    if (min_matches > 0 && kept < min_matches)
+      kept = lf_frame_pass(p, f, c, dir, kps, desc, counts, taken, pt_off[f], pt_off[f + 1], pts, pdesc,
+                           2.0f * th, th_high, check_orientation, out, winner);
+    if (n_matches) n_matches[f] = kept;
+  }
+  free(winner);
 }

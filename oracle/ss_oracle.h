@@ -118,6 +118,20 @@ void ref_stereo_match(const ref_params* p, const uint8_t* left, const uint8_t* r
                       const ref_keypoint* kr, const uint8_t* dr, const int32_t* cr, float bf, float b,
                       float* uright, float* depth, int32_t* sad);
 
+/* O13 ("ORB-Matching" of P:L254 Fig. 8): ORB-SLAM SearchByProjection of the
+ * last frame's map points into the current frame (TrackWithMotionModel).  24 bytes, same
+ * layout as ss_frame_point: world position, the last keypoint's angle (deg) and octave. */
+typedef struct { float pos[3]; float angle_deg; int32_t octave; int32_t reserved; } ref_frame_point;
+/* Points of frame f = [pt_off[f], pt_off[f+1]); last_cams may be NULL (mono); mb > 0 enables the
+ * stereo forward/backward level gate.  out[pt_off[F]]; n_matches[F] (may be NULL) = kept per frame. */
+void ref_match_last_frame(const ref_params* p, int n_frames, const ref_camera* cams, const ref_camera* last_cams,
+                          float mb, const ref_keypoint* kps, const uint8_t* desc, const int32_t* counts,
+                          const uint8_t* taken, const int32_t* pt_off, const ref_frame_point* pts,
+                          const uint8_t* pdesc, float th, int th_high, int check_orientation, int min_matches,
+                          ref_match* out, int32_t* n_matches);
+/* the rotation-histogram bin of step 5 */
+int ref_lf_rot_bin(float angle_last, float angle_cur);
+
 #ifdef __cplusplus
 }
 #endif

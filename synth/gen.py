@@ -268,3 +268,80 @@ def make_local_map(kps: np.ndarray, desc: np.ndarray, counts: np.ndarray, n_leve
         pts[f * Q:(f + 1) * Q] = p[perm]
         qdesc[f * Q:(f + 1) * Q] = qd[perm]
     return cams, pts, pf, qdesc, taken
+
+
+FRAME_POINT_DTYPE = np.dtype([("pos", "<f4", (3,)), ("angle_deg", "<f4"), ("octave", "<i4"), ("reserved", "<i4")])
+
+
+def _camera(c, R, t, shape, width, height):
+    fx, fy, cx, cy = INTRINSICS[shape]
+    c["R"], c["t"], c["ow"] = R.astype(np.float32).ravel(), t.astype(np.float32), (-R.T @ t).astype(np.float32)
+    c["fx"], c["fy"], c["cx"], c["cy"] = fx, fy, cx, cy
+    c["min_x"], c["max_x"], c["min_y"], c["max_y"] = 0.0, width, 0.0, height
+
+
+def make_last_frame(kps: np.ndarray, desc: np.ndarray, counts: np.ndarray, n_levels: int, n_per_level: np.ndarray,
+                    width: int, height: int, shape: str, n_points_per_frame: int, seed: int, true_frac=0.70,
+                    pos_sigma=1.5, stereo_z=0.0):
+    """The previous frame's tracked map points for frame-to-frame matching (O13, ORB-SLAM
+    TrackWithMotionModel), per frame:
+
+    * the current camera: a random pose and the dataset's intrinsics, bounds [0, W] x [0, H];
+      the last camera: the current one moved by stereo_z * U(-2, 2) along its optical axis
+      (0 = the same pose; the stereo forward / backward gate needs |motion| > baseline);
+    * true points (70 % of Q, at most the keypoint count): a keypoint's position +
+      N(0, pos_sigma px) back-projected at depth U(2, 20), octave = its level (80 %) or
+      level -+ 1 (clamped), angle = the keypoint's + a per-frame in-plane rotation U(-20, 20)
+      deg + N(0, 4) deg (mod 360), descriptor with 6 % bit flips;
+    * distractors: positions uniform over the image +-10 % at depth U(-2, 30), octave ~ N_l,
+      uniform angle, half random descriptors, half hard negatives (25 % flips).
+
+    Returns (cams [F], last_cams [F], pt_off [F+1] i32, points [F*Q] FRAME_POINT_DTYPE,
+    pdesc [F*Q, 32] u8); frame f's points are [pt_off[f], pt_off[f+1])."""
+    rng = _rng(seed)
+    F, cap = kps.shape
+    Q = n_points_per_frame
+    fx, fy, cx, cy = INTRINSICS[shape]
+    cams = np.zeros(F, CAMERA_DTYPE)
+    last = np.zeros(F, CAMERA_DTYPE)
+    pts = np.zeros(F * Q, FRAME_POINT_DTYPE)
+    pdesc = np.zeros((F * Q, 32), np.uint8)
+    pl = np.asarray(n_per_level, np.float64)
+    pl = pl / pl.sum()
+    for f in range(F):
+        R, t = _rotation(rng), rng.normal(0, 3.0, 3)
+        _camera(cams[f], R, t, shape, width, height)
+        tl = t + np.array([0.0, 0.0, stereo_z * rng.uniform(-2.0, 2.0)])
+        _camera(last[f], R, tl, shape, width, height)
+        n = int(counts[f, n_levels])
+        nt = min(int(true_frac * Q), n)
+        sel = rng.permutation(n)[:nt] if n else np.zeros(0, np.int64)
+        k = kps[f, sel]
+        u = np.concatenate([k["x"] + rng.normal(0, pos_sigma, nt), rng.uniform(-0.1 * width, 1.1 * width, Q - nt)])
+        v = np.concatenate([k["y"] + rng.normal(0, pos_sigma, nt), rng.uniform(-0.1 * height, 1.1 * height, Q - nt)])
+        z = np.concatenate([rng.uniform(2.0, 20.0, nt), rng.uniform(-2.0, 30.0, Q - nt)])
+        pc = np.stack([(u - cx) / fx * z, (v - cy) / fy * z, z], 1)
+        pw = (pc - t) @ R
+        oct_t = k["level"].astype(np.int64) + np.where(rng.random(nt) < 0.8, 0, rng.choice([-1, 1], nt))
+        octv = np.concatenate([np.clip(oct_t, 0, n_levels - 1), rng.choice(n_levels, size=Q - nt, p=pl)])
+        rot = rng.uniform(-20.0, 20.0)
+        ang = np.concatenate([k["angle_deg"] + rot + rng.normal(0, 4.0, nt), rng.uniform(0, 360, Q - nt)])
+        pd = np.zeros((Q, 32), np.uint8)
+        if nt:
+            pd[:nt] = flip_bits(desc[f, sel], 0.06, rng)
+        nd = Q - nt
+        rnd = rng.integers(0, 256, size=(nd, 32), dtype=np.uint8)
+        hard = rng.random(nd) < 0.5
+        if n:
+            other = desc[f, rng.integers(0, n, nd)]
+            rnd[hard] = flip_bits(other[hard], 0.25, rng)
+        pd[nt:] = rnd
+        p = np.zeros(Q, FRAME_POINT_DTYPE)
+        p["pos"] = pw.astype(np.float32)
+        p["angle_deg"] = np.mod(ang, 360.0).astype(np.float32) % np.float32(360.0)
+        p["octave"] = octv
+        perm = rng.permutation(Q)
+        pts[f * Q:(f + 1) * Q] = p[perm]
+        pdesc[f * Q:(f + 1) * Q] = pd[perm]
+    pt_off = (np.arange(F + 1) * Q).astype(np.int32)
+    return cams, last, pt_off, pts, pdesc
