@@ -206,6 +206,49 @@ ss_status ss_stereo_match(ss_ctx* ctx, int32_t n_pairs, const uint8_t* d_frames,
                           const ss_keypoint* d_kps, const uint8_t* d_desc, const int32_t* d_counts, float bf,
                           float baseline, float* d_uright, float* d_depth, ss_stream_t stream);
 
+/* A map point seen in the previous frame, for ss_match_last_frame (O13), 24 bytes: world
+ * position, the angle (deg, [0, 360)) and octave of the previous frame's keypoint it was matched
+ * to (ORB-SLAM LastFrame.mvKeysUn[i].angle / .octave). */
+typedef struct {
+  float pos[3];
+  float angle_deg;
+  int32_t octave;
+  int32_t reserved;
+} ss_frame_point;
+
+/* O13: frame-to-frame projection matching, ORB-SLAM SearchByProjection(CurrentFrame,
+ * LastFrame, th, bMono) as run by TrackWithMotionModel -- the "ORB-Matching" step of the
+ * paper's tracking-time breakdown (§5, Fig. 8); DESIGN.md §3 item 14.  Run after
+ * ss_orb_extract (same layouts).  Device pointers:
+ *   d_cams [n_frames]        current camera of each frame (the motion-model pose)
+ *   d_last_cams [n_frames]   previous camera of each frame, or NULL (only read when mb > 0)
+ *   d_kp_taken               [n_frames][kp_capacity] u8 or NULL (non-zero = not a candidate)
+ *   d_point_offsets [n_frames+1] i32: frame f's points are [off[f], off[f+1]), off[0] = 0,
+ *                            non-decreasing (the host never reads it: no synchronisation)
+ *   d_points / d_point_desc  [off[n_frames]] ss_frame_point / [off[n_frames]][32] u8
+ *   d_out [off[n_frames]]    per point: idx = keypoint index in its frame or -1; dist / dist2 =
+ *                            best / second Hamming distance over its candidates (256 = none)
+ *   d_n_matches [n_frames]   kept matches per frame, or NULL
+ * Per point: Pc = R*Pw + t, skip if Pc.z < 0, u = fx*X/Z + cx, v = fy*Y/Z + cy inside the
+ * bounds; window r = th * scale[octave] (|x-u| < r and |y-v| < r, f32); levels [o-1, o+1], or,
+ * when mb > 0 (stereo baseline) and the current camera centre seen from the last camera has
+ * z > mb, [o, L-1] (forward), or z < -mb, [0, o] (backward); best by (distance, index),
+ * accepted iff <= th_high (TH_HIGH = 100).  A keypoint claimed by several points keeps the
+ * min (distance, point).  check_orientation != 0: rotation histogram of (angle_last -
+ * angle_cur) with ORB-SLAM's bin = roundf(rot * (1.0f/30)), matches outside the three
+ * largest bins (ComputeThreeMaxima, 10 % rule) rejected.  min_matches > 0: a frame keeping
+ * fewer matches is redone with window factor 2*th (TrackWithMotionModel's retry).  Points
+ * with an octave outside [0, L-1] get {-1, 256, 256}.  Bit-exact with the oracle.
+ * SS_EINVAL for negative sizes, NULL buffers, th <= 0; SS_ECAPACITY if n_frames > max_frames.
+ * Uses the ctx's matcher scratch (row index, claims): not concurrently with another match
+ * call on the same ctx. */
+ss_status ss_match_last_frame(ss_ctx* ctx, int32_t n_frames, const ss_camera* d_cams, const ss_camera* d_last_cams,
+                              float mb, const ss_keypoint* d_kps, const uint8_t* d_desc, const int32_t* d_counts,
+                              const uint8_t* d_kp_taken, const int32_t* d_point_offsets,
+                              const ss_frame_point* d_points, const uint8_t* d_point_desc, float th,
+                              int32_t th_high, int32_t check_orientation, int32_t min_matches, ss_match* d_out,
+                              int32_t* d_n_matches, ss_stream_t stream);
+
 /* Keypoint distribution of the following ss_orb_extract calls on ctx (default quadtree):
  * SS_DIST_QUADTREE = ORB-SLAM's DistributeOctTree reading (O4); SS_DIST_GRID_TOPN = grid
  * top-N (O4g: K = FAST cells with a candidate, q = ceil(N_l / K), each cell keeps its q best
@@ -273,7 +316,8 @@ ss_status ss_track_tick(ss_ctx* ctx, int32_t n_frames, const ss_match_cfg* cfg, 
  * branch runs in line on `stream` instead of on its side stream, so each kernel is timed
  * alone).  WINDOW match: a pair per kernel
  * (match_prepare, match_window[, match_resolve if dedup]); BRUTE: brute_expand, brute_tc,
- * brute_merge; ss_project_points: project; ss_stereo_match: stereo_prepare, stereo, stereo_outliers.
+ * brute_merge; ss_project_points: project; ss_stereo_match: stereo_prepare, stereo, stereo_outliers;
+ * ss_match_last_frame: lastframe.
  * Works under CUDA-graph stream capture (the records become graph event nodes).
  * *next_index (may be NULL) receives the index of the next event to be recorded. */
 ss_status ss_profile_events(ss_ctx* ctx, void* const* events, int32_t n_events);

@@ -11,24 +11,13 @@
 // queries keeps the min (distance, query) (atomicMin on packed u64, then a resolve pass).
 // BRUTE: the per-split partial top-2 comes from the tensor-core kernel (k_brute_tc.cu);
 // match_brute_merge takes the two smallest (distance << 32 | map index) and applies the rule.
-#include "ss_internal.h"
+#include "match_common.cuh"
 
 namespace ss {
 
 namespace {
 
-__device__ __forceinline__ int hamming256(const uint4 a0, const uint4 a1, const uint4 b0, const uint4 b1) {
-  return __popc(a0.x ^ b0.x) + __popc(a0.y ^ b0.y) + __popc(a0.z ^ b0.z) + __popc(a0.w ^ b0.w) +
-         __popc(a1.x ^ b1.x) + __popc(a1.y ^ b1.y) + __popc(a1.z ^ b1.z) + __popc(a1.w ^ b1.w);
-}
-
 constexpr int WG = 8;  // lanes cooperating on one query
-
-__host__ __device__ __forceinline__ int row_off(const Geom& g, int l) {  // start of level l in a frame's row index
-  int o = 0;
-  for (int i = 0; i < l; i++) o += g.h[i] + 1;
-  return o;
-}
 
 // Per frame and level: rowidx[r] = index of the first keypoint with ly >= r (r in [0, h_l]),
 // from the canonical (level, ly, lx) order; plus the dedup claim table reset.
@@ -43,29 +32,7 @@ __global__ void __launch_bounds__(256) match_prepare(Geom g, int F, const ss_key
   if (gt >= F * cap) return;
   if (dedup) claim[gt] = ~0ull;
   const int f = gt / cap, k = gt - f * cap;
-  const int32_t* cnt = counts + f * (L + 1);
-  uint16_t* fr = rowidx + (int64_t)f * rows_per_frame;
-  if (k < L && cnt[k] == cnt[k + 1]) {  // empty level k: every row points at its (empty) range
-    uint16_t* ri = fr + row_off(g, k);
-    for (int r = 0; r <= g.h[k]; r++) ri[r] = (uint16_t)cnt[k];
-  }
-  if (k >= cnt[L]) return;
-  const ss_keypoint kp = kps[(int64_t)f * cap + k];
-  const int l = kp.level, ly = kp.ly;
-  uint16_t* ri = fr + row_off(g, l);
-  const int prev = k > cnt[l] ? (int)kps[(int64_t)f * cap + k - 1].ly : -1;
-  for (int r = prev + 1; r <= ly; r++) ri[r] = (uint16_t)k;
-  if (k == cnt[l + 1] - 1)
-    for (int r = ly + 1; r <= g.h[l]; r++) ri[r] = (uint16_t)(k + 1);
-}
-
-// top-2 of two packed (distance << 32 | index) pairs
-__device__ __forceinline__ void merge_top2(unsigned long long& a1, unsigned long long& a2, unsigned long long b1,
-                                           unsigned long long b2) {
-  const unsigned long long lo = a1 < b1 ? a1 : b1, hi = a1 < b1 ? b1 : a1;
-  const unsigned long long s2 = a2 < b2 ? a2 : b2;
-  a1 = lo;
-  a2 = hi < s2 ? hi : s2;
+  rowidx_fill(g, kps + (int64_t)f * cap, counts + f * (L + 1), rowidx + (int64_t)f * rows_per_frame, k);
 }
 
 __global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const ss_keypoint* __restrict__ kps,
@@ -100,10 +67,8 @@ __global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const 
     for (int l = l0; l <= l1; l++) {
       // rows that can hold |y - v| < r, widened by one row each side (f32 rounding); the exact
       // test below decides, so the superset only costs a few extra candidates
-      const float s_l = g.scale[l];
-      const int hl = g.h[l];
-      const int rlo = max(0, min(hl, (int)floorf(__fdiv_rn(__fsub_rn(Q.v, r), s_l)) - 1));
-      const int rhi = max(0, min(hl, (int)ceilf(__fdiv_rn(__fadd_rn(Q.v, r), s_l)) + 2));
+      int rlo, rhi;
+      window_rows(g, l, Q.v, r, &rlo, &rhi);
       const uint16_t* ri = fri + row_off(g, l);
       const int kb = ri[rlo], ke = ri[rhi];
       for (int k = kb + sub; k < ke; k += WG) {

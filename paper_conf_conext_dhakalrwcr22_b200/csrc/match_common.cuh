@@ -1,0 +1,58 @@
+// match_common.cuh -- device helpers shared by the matchers (k_match.cu, k_lastframe.cu):
+// 256-bit Hamming distance, the per-(frame, level, row) keypoint row index, packed top-2.
+#pragma once
+#include "ss_internal.h"
+
+namespace ss {
+
+__device__ __forceinline__ int hamming256(const uint4 a0, const uint4 a1, const uint4 b0, const uint4 b1) {
+  return __popc(a0.x ^ b0.x) + __popc(a0.y ^ b0.y) + __popc(a0.z ^ b0.z) + __popc(a0.w ^ b0.w) +
+         __popc(a1.x ^ b1.x) + __popc(a1.y ^ b1.y) + __popc(a1.z ^ b1.z) + __popc(a1.w ^ b1.w);
+}
+
+__host__ __device__ __forceinline__ int row_off(const Geom& g, int l) {  // start of level l in a frame's row index
+  int o = 0;
+  for (int i = 0; i < l; i++) o += g.h[i] + 1;
+  return o;
+}
+
+// Row-index entries owned by slot k of one frame (keypoints in canonical (level, ly, lx)
+// order): ri_l[r] = index of the first keypoint of level l with ly >= r, r in [0, h_l].
+// Slot k < L also fills the rows of an empty level k.  fk = the frame's keypoints, cnt = its
+// prefix counts, fr = its row index.
+__device__ __forceinline__ void rowidx_fill(const Geom& g, const ss_keypoint* __restrict__ fk,
+                                            const int32_t* __restrict__ cnt, uint16_t* __restrict__ fr, int k) {
+  const int L = g.L;
+  if (k < L && cnt[k] == cnt[k + 1]) {  // empty level k: every row points at its (empty) range
+    uint16_t* ri = fr + row_off(g, k);
+    for (int r = 0; r <= g.h[k]; r++) ri[r] = (uint16_t)cnt[k];
+  }
+  if (k >= cnt[L]) return;
+  const ss_keypoint kp = fk[k];
+  const int l = kp.level, ly = kp.ly;
+  uint16_t* ri = fr + row_off(g, l);
+  const int prev = k > cnt[l] ? (int)fk[k - 1].ly : -1;
+  for (int r = prev + 1; r <= ly; r++) ri[r] = (uint16_t)k;
+  if (k == cnt[l + 1] - 1)
+    for (int r = ly + 1; r <= g.h[l]; r++) ri[r] = (uint16_t)(k + 1);
+}
+
+// Rows [rlo, rhi) of level l (clamped to [0, h_l]) that can hold |y - v| < r, widened by one
+// row each side for f32 rounding; the exact test on each keypoint decides.
+__device__ __forceinline__ void window_rows(const Geom& g, int l, float v, float r, int* rlo, int* rhi) {
+  const float s_l = g.scale[l];
+  const int hl = g.h[l];
+  *rlo = max(0, min(hl, (int)floorf(__fdiv_rn(__fsub_rn(v, r), s_l)) - 1));
+  *rhi = max(0, min(hl, (int)ceilf(__fdiv_rn(__fadd_rn(v, r), s_l)) + 2));
+}
+
+// top-2 of two packed (distance << 32 | index) pairs
+__device__ __forceinline__ void merge_top2(unsigned long long& a1, unsigned long long& a2, unsigned long long b1,
+                                           unsigned long long b2) {
+  const unsigned long long lo = a1 < b1 ? a1 : b1, hi = a1 < b1 ? b1 : a1;
+  const unsigned long long s2 = a2 < b2 ? a2 : b2;
+  a1 = lo;
+  a2 = hi < s2 ? hi : s2;
+}
+
+}  // namespace ss

@@ -675,6 +675,30 @@ ss_status ss_project_points(ss_ctx* c, int32_t n_frames, const ss_camera* d_cams
   return SS_OK;
 }
 
+ss_status ss_match_last_frame(ss_ctx* c, int32_t n_frames, const ss_camera* d_cams, const ss_camera* d_last_cams,
+                              float mb, const ss_keypoint* d_kps, const uint8_t* d_desc, const int32_t* d_counts,
+                              const uint8_t* d_kp_taken, const int32_t* d_point_offsets,
+                              const ss_frame_point* d_points, const uint8_t* d_point_desc, float th,
+                              int32_t th_high, int32_t check_orientation, int32_t min_matches, ss_match* d_out,
+                              int32_t* d_n_matches, ss_stream_t stream) {
+  if (!c) return fail(SS_EINVAL, "NULL ctx");
+  if (n_frames < 0) return fail(SS_EINVAL, "negative size");
+  if (n_frames > c->max_frames) return fail(SS_ECAPACITY, "n_frames exceeds the ctx's max_frames");
+  if (!(th > 0.0f)) return fail(SS_EINVAL, "th must be > 0");
+  if (n_frames == 0) return SS_OK;
+  if (!d_cams || !d_kps || !d_desc || !d_counts || !d_point_offsets || !d_points || !d_point_desc || !d_out)
+    return fail(SS_EINVAL, "NULL buffer");
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  SS_CUDA_TRY(check_stream(s));
+  prof_mark(c, s);
+  SS_CUDA_TRY(launch_lastframe(c->g, n_frames, d_cams, mb > 0.0f ? d_last_cams : nullptr, mb, d_kps, d_desc, d_counts,
+                               d_kp_taken, d_point_offsets, d_points, d_point_desc, th, th_high, check_orientation,
+                               min_matches, d_out, d_n_matches, c->claim, c->rowidx, s));
+  prof_mark(c, s);
+  return SS_OK;
+}
+
 ss_status ss_set_distribution(ss_ctx* c, int32_t mode) {
   if (!c) return fail(SS_EINVAL, "NULL ctx");
   if (mode != SS_DIST_QUADTREE && mode != SS_DIST_GRID_TOPN) return fail(SS_EINVAL, "unknown distribution mode");

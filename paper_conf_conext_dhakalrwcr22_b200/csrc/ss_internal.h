@@ -192,6 +192,13 @@ cudaError_t launch_stereo(const Geom& g, int n_pairs, FrameSrc src, const ss_key
 cudaError_t launch_stereo_outliers(const Geom& g, int n_pairs, const int32_t* counts, const int32_t* sad,
                                    float* uright, float* depth, cudaStream_t s);
 
+// O13 frame-to-frame projection matching (k_lastframe.cu): one cluster of CTAs per frame.
+cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams, const ss_camera* last_cams, float mb,
+                             const ss_keypoint* kps, const uint8_t* desc, const int32_t* counts, const uint8_t* taken,
+                             const int32_t* pt_off, const ss_frame_point* pts, const uint8_t* pdesc, float th,
+                             int th_high, int check_orientation, int min_matches, ss_match* out, int32_t* n_matches,
+                             unsigned long long* claim, uint16_t* rowidx, cudaStream_t s);
+
 // Overflow scratch bytes the distribution needs for a level with `slots` candidate slots.
 int64_t distribute_ovf_bytes(int64_t slots);
 

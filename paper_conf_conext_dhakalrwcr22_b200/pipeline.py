@@ -88,6 +88,19 @@ class OrbPipeline:
         ss.ss_stereo_match(self.ctx, n_pairs, frames, frames.stride(0), frames.stride(1), self.kps, self.desc,
                            self.counts, bf, baseline, uright, depth, stream)
 
+    def match_last_frame(self, n_frames: int, cams: torch.Tensor, point_offsets: torch.Tensor, points: torch.Tensor,
+                         pdesc: torch.Tensor, out: torch.Tensor, n_matches: torch.Tensor | None = None,
+                         last_cams: torch.Tensor | None = None, mb: float = 0.0, th: float = 15.0, th_high: int = 100,
+                         check_orientation: bool = True, min_matches: int = 20, taken: torch.Tensor | None = None,
+                         stream: torch.cuda.Stream | None = None):
+        """O13 after extract(): cams / last_cams uint8 [n_frames, 96] (ss_camera), point_offsets int32
+        [n_frames+1], points uint8 [n, 24] (ss_frame_point), pdesc uint8 [n, 32] -> out int32 [n, 3]
+        (ss_match), n_matches int32 [n_frames]."""
+        stream = stream or torch.cuda.current_stream(self.device)
+        ss.ss_match_last_frame(self.ctx, n_frames, cams, last_cams, mb, self.kps, self.desc, self.counts, taken,
+                               point_offsets, points, pdesc, th, th_high, int(check_orientation), min_matches, out,
+                               n_matches, stream)
+
     # -- host views (synchronising; tests / examples) -------------------------------
     def results(self, n_frames: int):
         torch.cuda.synchronize(self.device)

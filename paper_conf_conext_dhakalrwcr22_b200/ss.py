@@ -75,6 +75,7 @@ CAMERA_DTYPE = np.dtype([("R", "<f4", (9,)), ("t", "<f4", (3,)), ("ow", "<f4", (
                          ("min_y", "<f4"), ("max_y", "<f4"), ("pad", "<f4")])
 MAP_POINT_DTYPE = np.dtype([("pos", "<f4", (3,)), ("normal", "<f4", (3,)), ("min_dist", "<f4"),
                             ("max_dist", "<f4")])
+FRAME_POINT_DTYPE = np.dtype([("pos", "<f4", (3,)), ("angle_deg", "<f4"), ("octave", "<i4"), ("reserved", "<i4")])
 
 _lib = None
 
@@ -100,6 +101,8 @@ def lib():
         L.ss_match_projection.argtypes = [P, i32, P, P, P, P, i32, P, P, i32, C.POINTER(ss_match_cfg), P, P]
         L.ss_project_points.argtypes = [P, i32, P, i32, P, P, C.c_float, P, P]
         L.ss_stereo_match.argtypes = [P, i32, P, i64, i32, P, P, P, C.c_float, C.c_float, P, P, P]
+        L.ss_match_last_frame.argtypes = [P, i32, P, P, C.c_float, P, P, P, P, P, P, P, C.c_float, i32, i32, i32,
+                                          P, P, P]
         L.ss_set_distribution.argtypes = [P, i32]
         L.ss_track_tick.argtypes = [P, i32, C.POINTER(ss_match_cfg), C.POINTER(ss_tick_io), P]
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
@@ -110,7 +113,7 @@ def lib():
         L.ss_profile_next.argtypes = [P, C.POINTER(i32)]
         for fn in ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_orb_extract", "ss_match_projection",
                    "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_set_distribution",
-                   "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
+                   "ss_match_last_frame", "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
                    "ss_profile_next", "ss_debug_phase_times"):
             getattr(L, fn).restype = C.c_int
         _lib = L
@@ -119,7 +122,7 @@ def lib():
 
 EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "ss_orb_extract",
             "ss_match_projection", "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_set_distribution",
-            "ss_profile_events", "ss_profile_next", "ss_debug_level",
+            "ss_match_last_frame", "ss_profile_events", "ss_profile_next", "ss_debug_level",
             "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times")
 
 
@@ -199,6 +202,16 @@ def ss_stereo_match(ctx, n_pairs, d_frames, frame_stride, pitch, d_kps, d_desc, 
 def ss_project_points(ctx, n_frames, d_cams, n_points, d_points, d_point_frame, th, d_queries, stream=None):
     _check(lib().ss_project_points(ctx, n_frames, _ptr(d_cams), n_points, _ptr(d_points), _ptr(d_point_frame),
                                    float(th), _ptr(d_queries), _stream(stream)), ctx)
+
+
+def ss_match_last_frame(ctx, n_frames, d_cams, d_last_cams, mb, d_kps, d_desc, d_counts, d_kp_taken, d_point_offsets,
+                        d_points, d_point_desc, th, th_high, check_orientation, min_matches, d_out, d_n_matches=None,
+                        stream=None):
+    _check(lib().ss_match_last_frame(ctx, n_frames, _ptr(d_cams), _ptr(d_last_cams), float(mb), _ptr(d_kps),
+                                     _ptr(d_desc), _ptr(d_counts), _ptr(d_kp_taken), _ptr(d_point_offsets),
+                                     _ptr(d_points), _ptr(d_point_desc), float(th), int(th_high),
+                                     int(check_orientation), int(min_matches), _ptr(d_out), _ptr(d_n_matches),
+                                     _stream(stream)), ctx)
 
 
 def ss_profile_events(ctx, events) -> None:
