@@ -33,16 +33,19 @@ import synth  # noqa: E402
 
 METRIC = "batched ORB extract+match frames/sec at 1/2/4/8 B200; per-frame p50 latency ms"
 CONFIGS = {
-    "c1": dict(shape="euroc", clients=1, nf=1000, mode="window", queries=5000, th=1.0, map=0,
-               desc="c1: single synthetic 752x480 frame, 8 levels x1.2, 1000 ORB features, search local points vs 5k local-map points (GPU projection + windowed match)"),
-    "c2": dict(shape="euroc", clients=4, nf=1000, mode="window", queries=5000, th=1.0, map=0,
+    "c1": dict(shape="euroc", clients=1, nf=1000, mode="window", queries=5000, th=1.0, map=0, lf=600, lf_th=15.0,
+               desc="c1: single synthetic 752x480 frame, 8 levels x1.2, 1000 ORB features, frame-to-frame matching of 600 last-frame points + search local points vs 5k local-map points (GPU projection + windowed match)"),
+    "c2": dict(shape="euroc", clients=4, nf=1000, mode="window", queries=5000, th=1.0, map=0, lf=600, lf_th=15.0,
                desc="c2: EuRoC-shaped 752x480 mono stream, 4 concurrent clients per GPU, 1000 features/frame, "
-                    "search local points vs 5k local-map points per client (GPU projection + windowed match)"),
-    "c3": dict(shape="tum", clients=16, nf=1000, mode="window", queries=50000, th=3.0, map=0,
-               desc="c3: TUM-RGBD-shaped 640x480, 16 clients per GPU, 1000 features, search local points vs 50k local-map points (projection + windowed match)"),
+                    "frame-to-frame matching of 600 last-frame points + search local points vs 5k local-map points per client "
+                    "(GPU projection + windowed match)"),
+    "c3": dict(shape="tum", clients=16, nf=1000, mode="window", queries=50000, th=3.0, map=0, lf=600, lf_th=15.0,
+               desc="c3: TUM-RGBD-shaped 640x480, 16 clients per GPU, 1000 features, frame-to-frame matching of 600 last-frame points + search local points vs 50k local-map points (projection + windowed match)"),
     "c4": dict(shape="kitti", clients=8, stereo=True, nf=2000, mode="window", queries=10000, th=1.0, map=0,
+               lf=1200, lf_th=7.0,
                desc="c4: KITTI-shaped 1241x376 stereo pairs, 8 clients per GPU, 2000 features/image, "
-                    "ORB-SLAM stereo matching of every pair + search local points vs 10k local-map points "
+                    "ORB-SLAM stereo matching of every pair + frame-to-frame matching of 1200 last-frame points (stereo level gates) "
+                    "+ search local points vs 10k local-map points "
                     "(left image; projection + windowed match)"),
     "c5": dict(shape="euroc", clients=8, nf=1250, mode="brute", queries=0, th=0.0, map=200000,
                desc="c5: EuRoC-shaped clients (8 per GPU, 64 over 8xB200), 1250 features, brute-force Hamming "
@@ -74,6 +77,35 @@ def gather_to_owner(send, rank: int, world: int):
         return bufs
     dist.gather(send, None, dst=0)
     return None
+
+
+def window_inputs(p, kps, desc, counts, cfg, seed_lm, seed_lf, per_client):
+    """Search-local-points and frame-to-frame inputs of one tick (synth recipes):
+    a local map per client frame (left / mono images; O11 + O9) and the previous frame's
+    tracked points in the same camera (O13).  kps / desc / counts: every image of the tick.
+    Returns (cams [B], points, point_frame, qdesc, taken [B, cap], last_cams [B],
+    lf_offsets [B+1], lf_points, lf_desc)."""
+    B = kps.shape[0]
+    cap = p.kp_capacity
+    L = p.n_levels
+    w, h = p.width, p.height
+    sel = list(range(0, B, per_client))
+    npl = np.array(p.n_per_level[:L])
+    cm, pt, pf, qd, tk = synth.make_local_map(kps[sel], desc[sel], counts[sel], L, p.scale_factor, npl, w, h,
+                                              cfg["shape"], cfg["queries"], seed=seed_lm)
+    _, last, off, lp, ld = synth.make_last_frame(kps[sel], desc[sel], counts[sel], L, npl, w, h, cfg["shape"],
+                                                 cfg["lf"], seed=seed_lf, cams=cm,
+                                                 stereo_z=0.5 if per_client == 2 else 0.0)
+    cmf = np.zeros(B, synth.CAMERA_DTYPE)
+    cmf[sel] = cm
+    lastf = np.zeros(B, synth.CAMERA_DTYPE)
+    lastf[sel] = last
+    tkf = np.zeros((B, cap), np.uint8)
+    tkf[sel] = tk
+    n_lf = np.zeros(B, np.int64)
+    n_lf[sel] = np.diff(off)
+    offf = np.concatenate([[0], np.cumsum(n_lf)]).astype(np.int32)
+    return cmf, pt, (pf * per_client).astype(np.int32), qd, tkf, lastf, offf, lp, ld
 
 
 def _gen_frame(args):
@@ -177,7 +209,7 @@ FAST_OPS_PER_PX = 62.5
 # ALU pipe peak: 148 SMs x 4 SMSPs x 16 lanes x 1.965 GHz (B200_PROFILING / B300_MICROARCH:
 # alu pipe rt = 2 cycles per warp instruction per SMSP) = 18.6 Tops/s
 ALU_PEAK_TOPS = 148 * 64 * 1.965e9 / 1e12
-def kernel_work(name: str, p, B: int, cand_l: list, kps_l: list, nq: int, n_map: int) -> tuple[str, float]:
+def kernel_work(name: str, p, B: int, cand_l: list, kps_l: list, nq: int, n_map: int, nlf: int = 0) -> tuple[str, float]:
     """(bound, algorithmic bytes or work) per launch -- DESIGN.md §6 work model.
     cand_l / kps_l: candidates / kept keypoints per level summed over the batch."""
     W = [p.level_w[l] * p.level_h[l] for l in range(p.n_levels)]
@@ -197,6 +229,8 @@ def kernel_work(name: str, p, B: int, cand_l: list, kps_l: list, nq: int, n_map:
         return "hbm", float(nq * 64)
     if name == "stereo":  # per left keypoint: its record + descriptor, 11x11 + 11x21 SAD pixels
         return "hbm", float(sum(kps_l)) / 2 * (20 + 32 + 121 + 231)  # half of the images are left ones
+    if name == "lastframe":  # per last-frame point: 24 B point + 32 B descriptor read, 12 B written
+        return "hbm", float(nlf * 68)
     if name == "project":  # map point 32 B + frame index 4 B read, query 20 B written
         return "hbm", float(nq * 56)
     if name == "match_resolve":
@@ -238,7 +272,9 @@ def run_ours(args, cfg):
     cap = p.kp_capacity
     props = torch.cuda.get_device_properties(dev)
     l2 = getattr(props, "L2_cache_size", 126 * 2 ** 20)
-    slot_bytes = B * h * w + (Q * 68 + B * (cap + 96) if window else 0)
+    NLF = cfg.get("lf", 0) * len(clients)  # last-frame points per tick (O13)
+    MB = synth.STEREO_BASELINE.get(cfg["shape"], 0.0) if cfg.get("stereo") else 0.0
+    slot_bytes = B * h * w + (Q * 68 + B * (cap + 96) + NLF * 56 + B * 100 if window else 0)
     n_slots = int(min(256, max(4, math.ceil(2 * l2 / slot_bytes))))
     if args.ring:
         n_slots = args.ring
@@ -259,29 +295,31 @@ def run_ours(args, cfg):
         point_frame = torch.zeros((n_slots, Q), dtype=torch.int32, device=dev)
         qdesc = torch.zeros((n_slots, Q, 32), dtype=torch.uint8, device=dev)
         taken = torch.zeros((n_slots, B, cap), dtype=torch.uint8, device=dev)
+        # frame-to-frame matching inputs (O13): the previous frame's tracked points per client
+        lf_last = torch.zeros((n_slots, B, 96), dtype=torch.uint8, device=dev)
+        lf_off = torch.zeros((n_slots, B + 1), dtype=torch.int32, device=dev)
+        lf_pts = torch.zeros((n_slots, max(NLF, 1), 24), dtype=torch.uint8, device=dev)
+        lf_desc = torch.zeros((n_slots, max(NLF, 1), 32), dtype=torch.uint8, device=dev)
         q_host = []
         for s in range(n_slots):
             with torch.cuda.stream(stream):
                 pipe.extract(frames[s], stream=stream)
             stream.synchronize()
             kps, desc, counts = pipe.results(B)
-            sel = list(range(0, B, per_client))  # local maps of the left / mono images
-            cm, pt, pf, qd, tk = synth.make_local_map(kps[sel], desc[sel], counts[sel], L, p.scale_factor,
-                                                      np.array(p.n_per_level[:L]), w, h, cfg["shape"],
-                                                      cfg["queries"],
-                                                      seed=synth.frame_seed(CFG_ID[args.config], 1 << 16 | rank, s))
-            pf = pf * per_client
-            cm_full = np.zeros(B, synth.CAMERA_DTYPE)
-            cm_full[sel] = cm
-            tk_full = np.zeros((B, cap), np.uint8)
-            tk_full[sel] = tk
+            wi = window_inputs(p, kps, desc, counts, cfg, synth.frame_seed(CFG_ID[args.config], 1 << 16 | rank, s),
+                               synth.frame_seed(CFG_ID[args.config], 2 << 16 | rank, s), per_client)
+            cm_full, pt, pf, qd, tk_full, last_full, off_full, lp, ld = wi
             cams[s] = torch.from_numpy(cm_full.view(np.uint8).reshape(B, 96).copy()).to(dev)
             points[s] = torch.from_numpy(pt.view(np.uint8).reshape(Q, 32).copy()).to(dev)
             point_frame[s] = torch.from_numpy(pf).to(dev)
             qdesc[s] = torch.from_numpy(qd).to(dev)
             taken[s] = torch.from_numpy(tk_full).to(dev)
+            lf_last[s] = torch.from_numpy(last_full.view(np.uint8).reshape(B, 96).copy()).to(dev)
+            lf_off[s] = torch.from_numpy(off_full).to(dev)
+            lf_pts[s, :NLF] = torch.from_numpy(lp.view(np.uint8).reshape(NLF, 24).copy()).to(dev)
+            lf_desc[s, :NLF] = torch.from_numpy(ld).to(dev)
             if s < 16:
-                q_host.append((cm_full, pt, pf, qd, tk_full))
+                q_host.append(wi)
     else:
         # shared map: rank 0 builds it from its clients' first-slot keypoints, broadcast once
         with torch.cuda.stream(stream):
@@ -301,8 +339,8 @@ def run_ours(args, cfg):
     mode = ss.SS_MATCH_WINDOW if window else ss.SS_MATCH_BRUTE
     stereo = bool(cfg.get("stereo"))
     ek = ss.extract_kernels(L)
-    mk = (["stereo_prepare", "stereo", "stereo_outliers"] if stereo else []) + (["project"] if window else []) + \
-        ss.match_kernels(mode, True)
+    mk = (["stereo_prepare", "stereo", "stereo_outliers"] if stereo else []) + \
+        (["lastframe", "project"] if window else []) + ss.match_kernels(mode, True)
     BASE_M = synth.STEREO_BASELINE.get(cfg["shape"], 0.0)
     BF = float(np.float32(synth.INTRINSICS[cfg["shape"]][0] * BASE_M))
     base = ss.extract_events(L)
@@ -324,6 +362,9 @@ def run_ours(args, cfg):
         pp.set_distribution(dist_mode)
     outs = [out] + [torch.zeros_like(out) for _ in range(P - 1)]
     qbufs = [torch.zeros((max(Q, 1), 20), dtype=torch.uint8, device=dev) for _ in range(P)]  # projected queries
+    lf_out = [torch.zeros((max(NLF, 1), 3), dtype=torch.int32, device=dev) for _ in range(P)]
+    lf_n = [torch.zeros(B, dtype=torch.int32, device=dev) for _ in range(P)]
+    lf_mask = [torch.zeros((B, cap), dtype=torch.uint8, device=dev) for _ in range(P)]
     npairs = B // 2 if stereo else 0
     st_out = [(torch.zeros((max(npairs, 1), cap), dtype=torch.float32, device=dev),
                torch.zeros((max(npairs, 1), cap), dtype=torch.float32, device=dev)) for _ in range(P)]
@@ -342,9 +383,12 @@ def run_ours(args, cfg):
             pp.extract(frames[s], stream=st)
             if stereo:
                 pp.stereo(frames[s], BF, BASE_M, st_out[q][0], st_out[q][1], stream=st)
-            if window:
+            if window:  # ORB-Matching (O13), then search local points skipping its matches (O11 + O9)
+                pp.match_last_frame(B, cams[s], lf_off[s], lf_pts[s], lf_desc[s], lf_out[q], lf_n[q],
+                                    last_cams=lf_last[s] if MB > 0 else None, mb=MB, th=cfg["lf_th"],
+                                    min_matches=20, taken=taken[s], matched=lf_mask[q], stream=st)
                 pp.project(B, cams[s], points[s], point_frame[s], qbufs[q], th=cfg["th"], stream=st)
-                pp.match_window(B, qbufs[q], qdesc[s], ot, taken=taken[s], stream=st)
+                pp.match_window(B, qbufs[q], qdesc[s], ot, taken=lf_mask[q], stream=st)
             else:
                 pp.match_brute(B, map_desc, ot, stream=st)
         if prof:
@@ -364,7 +408,8 @@ def run_ours(args, cfg):
         gather_stream.wait_event(done_ev)
         with torch.cuda.stream(gather_stream):
             pp = pipes[q]
-            gather_to_owner(pack_results([pp.kps[:B], pp.desc[:B], pp.counts[:B], outs[q]]), rank, world)
+            parts = [pp.kps[:B], pp.desc[:B], pp.counts[:B], outs[q]] + ([lf_out[q], lf_n[q]] if window else [])
+            gather_to_owner(pack_results(parts), rank, world)
 
     W_, K = args.warmup, args.steps
     ev_start = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
@@ -454,8 +499,8 @@ def run_ours(args, cfg):
         per_func.setdefault(func_of.get(n_, n_), []).append(n_)
     dom_f = max(per_func, key=lambda f_: sum(avg_us[n_] for n_ in per_func[f_]))
     members = per_func[dom_f]
-    bound = kernel_work(members[0], p, B, cand_l, kps_l, Q, cfg["map"])[0]
-    work = sum(kernel_work(n_, p, B, cand_l, kps_l, Q, cfg["map"])[1] for n_ in members)
+    bound = kernel_work(members[0], p, B, cand_l, kps_l, Q, cfg["map"], NLF)[0]
+    work = sum(kernel_work(n_, p, B, cand_l, kps_l, Q, cfg["map"], NLF)[1] for n_ in members)
     dom_us = sum(avg_us[n_] for n_ in members)
     avg_us_dom = dom_us
     dom = dom_f if len(members) == 1 else f"{dom_f} ({' + '.join(members)})"
@@ -491,7 +536,7 @@ def run_ours(args, cfg):
 
     # --- e2e through the public API with host buffers (pinned), copies inside the timed region
     e2e = run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=cfg["th"],
-                  stereo=(BF, BASE_M, st_out) if stereo else None)
+                  stereo=(BF, BASE_M, st_out) if stereo else None, lf=(MB, cfg.get("lf_th", 15.0)))
 
     frames_per_step = B * world
     value = frames_per_step * K / (T_max / 1000.0)
@@ -533,7 +578,8 @@ def run_ours(args, cfg):
         print(json.dumps(res), flush=True)
 
 
-def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=1.0, stereo=None):
+def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=1.0, stereo=None,
+            lf=(0.0, 15.0)):
     """Same ticks end to end from pinned host buffers through ONE C-ABI call per tick
     (ss_track_tick: H2D of the tick's frames and local maps, extract, stereo, projection +
     match or brute match, D2H of every output), all inside the timed region; ticks
@@ -561,6 +607,10 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
              "desc": torch.empty(B * cap * 32, dtype=torch.uint8).pin_memory(),
              "counts": torch.empty(B * (L + 1), dtype=torch.int32).pin_memory(),
              "matches": torch.empty(rows * 3, dtype=torch.int32).pin_memory()}
+        if window:
+            nlf = int(q_host[0][6][-1])
+            o["lf_matches"] = torch.empty(max(nlf, 1) * 3, dtype=torch.int32).pin_memory()
+            o["lf_n"] = torch.empty(B, dtype=torch.int32).pin_memory()
         if stereo:
             o["uright"] = torch.empty((B // 2) * cap, dtype=torch.float32).pin_memory()
             o["depth"] = torch.empty((B // 2) * cap, dtype=torch.float32).pin_memory()
@@ -575,9 +625,12 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
             if stereo:
                 io.bf, io.baseline = stereo[0], stereo[1]
             if window:
-                cm, pt, pf, qd, tk = hin[i]
+                cm, pt, pf, qd, tk, last, off, lp, ld = hin[i]
                 io.cams, io.n_points, io.points, io.point_frame = cm.data_ptr(), Q, pt.data_ptr(), pf.data_ptr()
                 io.point_desc, io.taken, io.th = qd.data_ptr(), tk.data_ptr(), th
+                io.lf_offsets, io.lf_points, io.lf_desc = off.data_ptr(), lp.data_ptr(), ld.data_ptr()
+                io.last_cams, io.mb, io.lf_th, io.lf_min_matches = last.data_ptr(), lf[0], lf[1], 20
+                io.lf_matches, io.lf_n_matches = o["lf_matches"].data_ptr(), o["lf_n"].data_ptr()
             else:
                 io.d_map_desc, io.n_map = map_desc.data_ptr(), map_desc.shape[0]
             o = host_out[q]
@@ -587,7 +640,8 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
                 io.uright, io.depth = o["uright"].data_ptr(), o["depth"].data_ptr()
             row.append(io)
         ios.append(row)
-    h2d = fr[0].numel() + (sum(a.numel() for a in hin[0]) if window else 0)
+    # bytes actually copied per tick (the last cameras only in stereo, when mb > 0)
+    h2d = fr[0].numel() + (sum(a.numel() for j, a in enumerate(hin[0]) if j != 5 or lf[0] > 0) if window else 0)
     d2h = sum(t.numel() * t.element_size() for t in host_out[0].values())
     handles = [st.cuda_stream for st in streams]
 
@@ -615,7 +669,8 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
             "d2h_bytes_per_step": int(d2h), "steps": K, "ms_per_step": ms / K, "ticks_in_flight": P,
             "path": "pinned host -> ss_track_tick (one C-ABI call per tick: H2D, ss_orb_extract, " +
                     ("ss_stereo_match, " if stereo else "") +
-                    ("ss_project_points, ss_match_projection WINDOW" if window else "ss_match_projection BRUTE") +
+                    ("ss_match_last_frame, ss_project_points, ss_match_projection WINDOW" if window
+                     else "ss_match_projection BRUTE") +
                     ", D2H of all outputs; no graphs)"}
 
 
@@ -633,8 +688,13 @@ def _oracle_job(job):
         base = synth.STEREO_BASELINE["kitti"]
         bf = float(np.float32(synth.INTRINSICS["kitti"][0] * base))
         oracle.stereo_match(p, frame, right, kps, desc, counts, kr, dr, cr, bf, base)
-    if mode == "window" and lm is not None:
-        cm, pt, qd, tk = lm
+    if mode == "window" and lm is not None:  # O13, then O11 + O9 skipping O13's matches
+        cm, pt, qd, tk, last, lp, ld, mb, lf_th = lm
+        off = np.array([0, len(lp)], np.int32)
+        lfm, _ = oracle.match_last_frame(p, cm[None], last[None], mb, kps[None], desc[None], counts[None], tk[None],
+                                         off, lp, ld, th=lf_th, min_matches=20)
+        tk = tk.copy()
+        tk[lfm["idx"][lfm["idx"] >= 0]] = 1
         q = oracle.project_points(p, cm[None], pt, np.zeros(len(pt), np.int32), th)
         oracle.match_window(p, kps[None], desc[None], counts[None], tk[None], q, qd)
     elif mode == "brute" and mp is not None:
@@ -653,9 +713,11 @@ def _jobs_for(cfg, frames_h, q_host, n, w, h, mp=None):
         s, b = (i // Bimg) % S, i % Bimg
         lm = None
         if cfg["mode"] == "window" and q_host and b % per_client == 0:
-            cm, pt, pf, qd, tk = q_host[s % len(q_host)]
+            cm, pt, pf, qd, tk, last, off, lp, ld = q_host[s % len(q_host)]
             sel = pf == b
-            lm = (cm[b], pt[sel], qd[sel], tk[b])
+            mb = synth.STEREO_BASELINE.get(cfg["shape"], 0.0) if per_client == 2 else 0.0
+            lm = (cm[b], pt[sel], qd[sel], tk[b], last[b], lp[off[b]:off[b + 1]], ld[off[b]:off[b + 1]], mb,
+                  cfg["lf_th"])
         if per_client == 2:  # stereo: the left image's job covers the pair
             left = b % 2 == 0
             jobs.append((w, h, cfg["nf"], frames_h[s, b] if left else None, lm, cfg["mode"], mp, cfg["th"],
@@ -683,7 +745,8 @@ def cpu_baseline(args, cfg, frames_h, q_host, budget_s=15.0, mp=None):
     return {"value": len(jobs) / wall, "unit": "frames/s", "cores": cores, "kind": "oracle",
             "sample": f"{len(jobs)} frames of the {args.config} workload (extract + " +
                       ("stereo matching of each pair + " if cfg.get("stereo") else "") +
-                      (f"its {cfg['queries']}-point local map projected and window-matched" if cfg["mode"] == "window"
+                      (f"its {cfg.get('lf', 0)} last-frame points matched (O13), its {cfg['queries']}-point local map projected "
+                       "and window-matched" if cfg["mode"] == "window"
                        else "4 keypoints brute-matched against the map") +
                       " each), one single-threaded oracle process per core",
             "median_frame_s_single_core": float(np.median(per)),
@@ -721,16 +784,9 @@ def run_reference(args, cfg):
         per_client = 2 if cfg.get("stereo") else 1
         B = frames_h.shape[1]
         for s in range(frames_h.shape[0]):
-            kps, desc, counts = oracle.orb_extract_batch(p, frames_h[s][::per_client])
-            cm, pt, pf, qd, tk = synth.make_local_map(kps, desc, counts, 8, p.scale_factor,
-                                                      np.array(p.n_per_level[:8]), w, h, cfg["shape"],
-                                                      cfg["queries"], seed=synth.frame_seed(CFG_ID[args.config],
-                                                                                            1 << 16, s))
-            cmf = np.zeros(B, synth.CAMERA_DTYPE)
-            cmf[::per_client] = cm
-            tkf = np.zeros((B, p.kp_capacity), np.uint8)
-            tkf[::per_client] = tk
-            q_host.append((cmf, pt, pf * per_client, qd, tkf))
+            kps, desc, counts = oracle.orb_extract_batch(p, frames_h[s])
+            q_host.append(window_inputs(p, kps, desc, counts, cfg, synth.frame_seed(CFG_ID[args.config], 1 << 16, s),
+                                        synth.frame_seed(CFG_ID[args.config], 2 << 16, s), per_client))
     else:
         p = oracle.params(w, h, cfg["nf"])
         kps, desc, counts = oracle.orb_extract_batch(p, frames_h[0])
@@ -760,7 +816,8 @@ def run_reference(args, cfg):
                       "parallelism": "CPU oracle, one single-threaded process per core"},
            "cpu_baseline": {"value": value, "unit": "frames/s", "cores": min(cores, n_frames), "kind": "oracle",
                             "sample": f"{n_frames} of the tick's {B} frames per step (extract + " +
-                                      (f"{cfg['queries']}-point local map projected + window-matched"
+                                      (f"{cfg.get('lf', 0)} last-frame points matched + {cfg['queries']}-point "
+                                       "local map projected + window-matched"
                                        if cfg["mode"] == "window" else "4 keypoints brute-matched") + " each)",
                             "cpu": _cpu_model()},
            "e2e": {"value": value, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}

@@ -229,6 +229,10 @@ typedef struct {
  *   d_out [off[n_frames]]    per point: idx = keypoint index in its frame or -1; dist / dist2 =
  *                            best / second Hamming distance over its candidates (256 = none)
  *   d_n_matches [n_frames]   kept matches per frame, or NULL
+ *   d_kp_matched             [n_frames][kp_capacity] u8 or NULL: 1 where d_kp_taken is non-zero
+ *                            or a kept match claims the keypoint, else 0 -- the d_kp_taken of
+ *                            the following search-local-points ss_match_projection (ORB-SLAM's
+ *                            SearchLocalPoints skips keypoints the motion model already matched)
  * Per point: Pc = R*Pw + t, skip if Pc.z < 0, u = fx*X/Z + cx, v = fy*Y/Z + cy inside the
  * bounds; window r = th * scale[octave] (|x-u| < r and |y-v| < r, f32); levels [o-1, o+1], or,
  * when mb > 0 (stereo baseline) and the current camera centre seen from the last camera has
@@ -247,7 +251,7 @@ ss_status ss_match_last_frame(ss_ctx* ctx, int32_t n_frames, const ss_camera* d_
                               const uint8_t* d_kp_taken, const int32_t* d_point_offsets,
                               const ss_frame_point* d_points, const uint8_t* d_point_desc, float th,
                               int32_t th_high, int32_t check_orientation, int32_t min_matches, ss_match* d_out,
-                              int32_t* d_n_matches, ss_stream_t stream);
+                              int32_t* d_n_matches, uint8_t* d_kp_matched, ss_stream_t stream);
 
 /* Keypoint distribution of the following ss_orb_extract calls on ctx (default quadtree):
  * SS_DIST_QUADTREE = ORB-SLAM's DistributeOctTree reading (O4); SS_DIST_GRID_TOPN = grid
@@ -290,13 +294,28 @@ typedef struct {
   ss_match* matches;
   float* uright;
   float* depth;
+  /* O13 frame-to-frame matching (ss_match_last_frame), run before the WINDOW match when
+   * lf_offsets != NULL: lf_offsets [n_frames+1], lf_points / lf_desc [lf_offsets[n_frames]]
+   * (<= max_queries), current cameras = cams, last_cams [n_frames] (read when mb > 0);
+   * outputs lf_matches [lf_offsets[n_frames]], lf_n_matches [n_frames] (may be NULL).  The
+   * WINDOW match then skips keypoints that are taken OR kept by O13 (ORB-SLAM's
+   * SearchLocalPoints skips the motion model's matches). */
+  const int32_t* lf_offsets;
+  const ss_frame_point* lf_points;
+  const uint8_t* lf_desc;
+  const ss_camera* last_cams;
+  float mb, lf_th;
+  int32_t lf_min_matches;
+  ss_match* lf_matches;
+  int32_t* lf_n_matches;
 } ss_tick_io;
 
 /* One tick of the hot path for a batch of client frames, enqueued on `stream` from a single
  * call: host -> device copies into ctx-owned staging buffers (sized at ss_create: max_frames
  * frames, max_queries points), ss_orb_extract, ss_stereo_match (if io->bf > 0),
- * ss_project_points + ss_match_projection WINDOW (cfg->mode == SS_MATCH_WINDOW, n_points > 0)
- * or ss_match_projection BRUTE (cfg->mode == SS_MATCH_BRUTE), device -> host copies of the
+ * ss_match_last_frame (if io->lf_offsets, WINDOW only), ss_project_points +
+ * ss_match_projection WINDOW (cfg->mode == SS_MATCH_WINDOW, n_points > 0) or
+ * ss_match_projection BRUTE (cfg->mode == SS_MATCH_BRUTE), device -> host copies of the
  * outputs.  Asynchronous: outputs are valid once the stream reaches the end of the call; the
  * caller must not reuse the ctx for another tick before then.  Same results and errors as
  * the individual calls (SS_ECAPACITY when n_frames > max_frames or n_points > max_queries). */

@@ -67,6 +67,7 @@ struct LfArgs {
   int th_high, check_orientation, min_matches;
   ss_match* out;
   int32_t* n_matches;
+  uint8_t* matched;
   unsigned long long* claim;
   uint16_t* rowidx;
   int rows_per_frame;
@@ -93,9 +94,11 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
   const int32_t* cnt = a.counts + f * (L + 1);
   uint16_t* fri = a.rowidx + (int64_t)f * a.rows_per_frame;
   unsigned long long* fclaim = a.claim + (int64_t)f * cap;
+  uint8_t* fmask = a.matched ? a.matched + (int64_t)f * cap : nullptr;
   for (int k = ct; k < cap; k += nct) {  // P0
     rowidx_fill(g, fk, cnt, fri, k);
     fclaim[k] = ~0ull;
+    if (fmask) fmask[k] = (a.taken && a.taken[(int64_t)f * cap + k]) ? 1 : 0;
   }
   cluster.sync();
 
@@ -229,6 +232,11 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
     if (a.min_matches <= 0 || kept >= a.min_matches) break;  // uniform over the cluster
   }
   if (a.n_matches && rank == 0 && threadIdx.x == 0) a.n_matches[f] = kept;
+  if (fmask)  // kept matches are unique per keypoint (dedup), so these stores never collide
+    for (int i = i0 + ct; i < i1; i += nct) {
+      const int idx = a.out[i].idx;
+      if (idx >= 0) fmask[idx] = 1;
+    }
   cluster.sync();  // the leader's shared memory must outlive every remote access
 }
 
@@ -238,11 +246,11 @@ cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams,
                              const ss_keypoint* kps, const uint8_t* desc, const int32_t* counts, const uint8_t* taken,
                              const int32_t* pt_off, const ss_frame_point* pts, const uint8_t* pdesc, float th,
                              int th_high, int check_orientation, int min_matches, ss_match* out, int32_t* n_matches,
-                             unsigned long long* claim, uint16_t* rowidx, cudaStream_t s) {
+                             uint8_t* matched, unsigned long long* claim, uint16_t* rowidx, cudaStream_t s) {
   if (n_frames <= 0) return cudaSuccess;
   LfArgs a{g,     n_frames, cams,    last_cams,         mb,          kps, desc, counts,
            taken, pt_off,   pts,     pdesc,             th,          th_high, check_orientation,
-           min_matches, out, n_matches, claim, rowidx, match_rows_per_frame(g)};
+           min_matches, out, n_matches, matched, claim, rowidx, match_rows_per_frame(g)};
   cudaError_t e = launch_pdl(lastframe_kernel, dim3(n_frames * kCluster), dim3(kThreads), 0, s, a);
   return e != cudaSuccess ? e : cudaGetLastError();
 }

@@ -161,6 +161,13 @@ struct ss_ctx {
   ss_match* io_matches = nullptr;
   float* io_uright = nullptr;
   float* io_depth = nullptr;
+  int32_t* io_lf_off = nullptr;  // O13 staging
+  ss_frame_point* io_lf_pts = nullptr;
+  uint8_t* io_lf_desc = nullptr;
+  ss_camera* io_last_cams = nullptr;
+  ss_match* io_lf_matches = nullptr;
+  int32_t* io_lf_n = nullptr;
+  uint8_t* io_lf_mask = nullptr;
   int8_t* brute_qexp = nullptr;  // BRUTE: keypoint descriptors expanded to s8 +-1 (k_brute_tc.cu)
   int8_t* brute_mexp = nullptr;  // BRUTE: map descriptors expanded to s8 +-1
   int n_sm = 148;
@@ -202,7 +209,8 @@ void free_ctx(ss_ctx* c) {
                   c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->rowidx, c->phase_ts,
                   c->brute_qexp, c->brute_mexp, c->stereo_sad, c->io_frames, c->io_kps, c->io_desc, c->io_counts,
                   c->io_cams, c->io_points, c->io_pf, c->io_pdesc, c->io_taken, c->io_queries, c->io_matches,
-                  c->io_uright, c->io_depth};
+                  c->io_uright, c->io_depth, c->io_lf_off, c->io_lf_pts, c->io_lf_desc, c->io_last_cams,
+                  c->io_lf_matches, c->io_lf_n, c->io_lf_mask};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
@@ -473,6 +481,13 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     ALLOC(c->io_matches, sizeof(ss_match) * std::max<int64_t>(Qm, F * g.kp_capacity));
     ALLOC(c->io_uright, sizeof(float) * ((F + 1) / 2) * g.kp_capacity);
     ALLOC(c->io_depth, sizeof(float) * ((F + 1) / 2) * g.kp_capacity);
+    ALLOC(c->io_lf_off, sizeof(int32_t) * (F + 1));
+    ALLOC(c->io_lf_pts, sizeof(ss_frame_point) * Qm);
+    ALLOC(c->io_lf_desc, (size_t)Qm * SS_DESC_BYTES);
+    ALLOC(c->io_last_cams, sizeof(ss_camera) * F);
+    ALLOC(c->io_lf_matches, sizeof(ss_match) * Qm);
+    ALLOC(c->io_lf_n, sizeof(int32_t) * F);
+    ALLOC(c->io_lf_mask, (size_t)F * g.kp_capacity);
   }
   if (max_map > 0) {
     ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
@@ -680,7 +695,7 @@ ss_status ss_match_last_frame(ss_ctx* c, int32_t n_frames, const ss_camera* d_ca
                               const uint8_t* d_kp_taken, const int32_t* d_point_offsets,
                               const ss_frame_point* d_points, const uint8_t* d_point_desc, float th,
                               int32_t th_high, int32_t check_orientation, int32_t min_matches, ss_match* d_out,
-                              int32_t* d_n_matches, ss_stream_t stream) {
+                              int32_t* d_n_matches, uint8_t* d_kp_matched, ss_stream_t stream) {
   if (!c) return fail(SS_EINVAL, "NULL ctx");
   if (n_frames < 0) return fail(SS_EINVAL, "negative size");
   if (n_frames > c->max_frames) return fail(SS_ECAPACITY, "n_frames exceeds the ctx's max_frames");
@@ -694,7 +709,7 @@ ss_status ss_match_last_frame(ss_ctx* c, int32_t n_frames, const ss_camera* d_ca
   prof_mark(c, s);
   SS_CUDA_TRY(launch_lastframe(c->g, n_frames, d_cams, mb > 0.0f ? d_last_cams : nullptr, mb, d_kps, d_desc, d_counts,
                                d_kp_taken, d_point_offsets, d_points, d_point_desc, th, th_high, check_orientation,
-                               min_matches, d_out, d_n_matches, c->claim, c->rowidx, s));
+                               min_matches, d_out, d_n_matches, d_kp_matched, c->claim, c->rowidx, s));
   prof_mark(c, s);
   return SS_OK;
 }
@@ -723,6 +738,18 @@ ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, co
     if (io->n_points > c->max_queries) return fail(SS_ECAPACITY, "n_points exceeds the ctx's max_queries");
     if (!io->cams || !io->points || !io->point_frame || !io->point_desc) return fail(SS_EINVAL, "NULL window input");
   }
+  const bool lastf = window && io->lf_offsets;
+  int64_t n_lf = 0;
+  if (lastf) {
+    for (int f = 0; f < n_frames; f++)
+      if (io->lf_offsets[f + 1] < io->lf_offsets[f]) return fail(SS_EINVAL, "lf_offsets must be non-decreasing");
+    if (io->lf_offsets[0] != 0) return fail(SS_EINVAL, "lf_offsets[0] must be 0");
+    n_lf = io->lf_offsets[n_frames];
+    if (n_lf > c->max_queries) return fail(SS_ECAPACITY, "last-frame points exceed the ctx's max_queries");
+    if (n_lf > 0 && (!io->lf_points || !io->lf_desc)) return fail(SS_EINVAL, "NULL last-frame input");
+    if (io->mb > 0.0f && !io->last_cams) return fail(SS_EINVAL, "mb > 0 needs last_cams");
+    if (!(io->lf_th > 0.0f)) return fail(SS_EINVAL, "lf_th must be > 0");
+  }
   SS_CUDA_TRY(cudaSetDevice(c->device));
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   const int cap = g.kp_capacity, L = g.L;
@@ -749,6 +776,15 @@ ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, co
     if (io->taken)
       SS_CUDA_TRY(cudaMemcpyAsync(c->io_taken, io->taken, (size_t)n_frames * cap, cudaMemcpyHostToDevice, s));
   }
+  if (lastf) {
+    SS_CUDA_TRY(cudaMemcpyAsync(c->io_lf_off, io->lf_offsets, sizeof(int32_t) * (n_frames + 1), cudaMemcpyHostToDevice, s));
+    if (n_lf > 0) {
+      SS_CUDA_TRY(cudaMemcpyAsync(c->io_lf_pts, io->lf_points, sizeof(ss_frame_point) * n_lf, cudaMemcpyHostToDevice, s));
+      SS_CUDA_TRY(cudaMemcpyAsync(c->io_lf_desc, io->lf_desc, (size_t)n_lf * SS_DESC_BYTES, cudaMemcpyHostToDevice, s));
+    }
+    if (io->mb > 0.0f)
+      SS_CUDA_TRY(cudaMemcpyAsync(c->io_last_cams, io->last_cams, sizeof(ss_camera) * n_frames, cudaMemcpyHostToDevice, s));
+  }
   // the hot path
   ss_status st = ss_orb_extract(c, n_frames, c->io_frames, fstride, P, c->io_kps, c->io_desc, c->io_counts, stream);
   if (st != SS_OK) return st;
@@ -758,12 +794,20 @@ ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, co
     if (st != SS_OK) return st;
   }
   int64_t n_matches = 0;
+  const uint8_t* win_taken = io->taken ? c->io_taken : nullptr;
+  if (lastf) {
+    st = ss_match_last_frame(c, n_frames, c->io_cams, io->mb > 0.0f ? c->io_last_cams : nullptr, io->mb, c->io_kps,
+                             c->io_desc, c->io_counts, win_taken, c->io_lf_off, c->io_lf_pts, c->io_lf_desc,
+                             io->lf_th, 100, 1, io->lf_min_matches, c->io_lf_matches, c->io_lf_n, c->io_lf_mask,
+                             stream);
+    if (st != SS_OK) return st;
+    win_taken = c->io_lf_mask;
+  }
   if (window) {
     st = ss_project_points(c, n_frames, c->io_cams, io->n_points, c->io_points, c->io_pf, io->th, c->io_queries,
                            stream);
     if (st != SS_OK) return st;
-    st = ss_match_projection(c, n_frames, c->io_kps, c->io_desc, c->io_counts, io->taken ? c->io_taken : nullptr,
-                             io->n_points, c->io_queries, c->io_pdesc, 0, cfg, c->io_matches, stream);
+    st = ss_match_projection(c, n_frames, c->io_kps, c->io_desc, c->io_counts, win_taken, io->n_points, c->io_queries, c->io_pdesc, 0, cfg, c->io_matches, stream);
     if (st != SS_OK) return st;
     n_matches = io->n_points;
   } else if (cfg->mode == SS_MATCH_BRUTE) {
@@ -781,6 +825,10 @@ ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, co
     SS_CUDA_TRY(cudaMemcpyAsync(io->counts, c->io_counts, sizeof(int32_t) * n_frames * (L + 1), cudaMemcpyDeviceToHost, s));
   if (io->matches && n_matches > 0)
     SS_CUDA_TRY(cudaMemcpyAsync(io->matches, c->io_matches, sizeof(ss_match) * n_matches, cudaMemcpyDeviceToHost, s));
+  if (lastf && io->lf_matches && n_lf > 0)
+    SS_CUDA_TRY(cudaMemcpyAsync(io->lf_matches, c->io_lf_matches, sizeof(ss_match) * n_lf, cudaMemcpyDeviceToHost, s));
+  if (lastf && io->lf_n_matches)
+    SS_CUDA_TRY(cudaMemcpyAsync(io->lf_n_matches, c->io_lf_n, sizeof(int32_t) * n_frames, cudaMemcpyDeviceToHost, s));
   if (stereo && io->uright)
     SS_CUDA_TRY(cudaMemcpyAsync(io->uright, c->io_uright, sizeof(float) * (n_frames / 2) * cap, cudaMemcpyDeviceToHost, s));
   if (stereo && io->depth)

@@ -92,14 +92,14 @@ class OrbPipeline:
                          pdesc: torch.Tensor, out: torch.Tensor, n_matches: torch.Tensor | None = None,
                          last_cams: torch.Tensor | None = None, mb: float = 0.0, th: float = 15.0, th_high: int = 100,
                          check_orientation: bool = True, min_matches: int = 20, taken: torch.Tensor | None = None,
-                         stream: torch.cuda.Stream | None = None):
+                         matched: torch.Tensor | None = None, stream: torch.cuda.Stream | None = None):
         """O13 after extract(): cams / last_cams uint8 [n_frames, 96] (ss_camera), point_offsets int32
         [n_frames+1], points uint8 [n, 24] (ss_frame_point), pdesc uint8 [n, 32] -> out int32 [n, 3]
-        (ss_match), n_matches int32 [n_frames]."""
+        (ss_match), n_matches int32 [n_frames], matched uint8 [n_frames, cap] (taken | kept matches)."""
         stream = stream or torch.cuda.current_stream(self.device)
         ss.ss_match_last_frame(self.ctx, n_frames, cams, last_cams, mb, self.kps, self.desc, self.counts, taken,
                                point_offsets, points, pdesc, th, th_high, int(check_orientation), min_matches, out,
-                               n_matches, stream)
+                               n_matches, matched, stream)
 
     # -- host views (synchronising; tests / examples) -------------------------------
     def results(self, n_frames: int):

@@ -61,7 +61,10 @@ class ss_tick_io(C.Structure):
                 ("point_frame", C.c_void_p), ("point_desc", C.c_void_p), ("taken", C.c_void_p),
                 ("th", C.c_float), ("d_map_desc", C.c_void_p), ("n_map", C.c_int32),
                 ("kps", C.c_void_p), ("desc", C.c_void_p), ("counts", C.c_void_p), ("matches", C.c_void_p),
-                ("uright", C.c_void_p), ("depth", C.c_void_p)]
+                ("uright", C.c_void_p), ("depth", C.c_void_p),
+                ("lf_offsets", C.c_void_p), ("lf_points", C.c_void_p), ("lf_desc", C.c_void_p),
+                ("last_cams", C.c_void_p), ("mb", C.c_float), ("lf_th", C.c_float), ("lf_min_matches", C.c_int32),
+                ("lf_matches", C.c_void_p), ("lf_n_matches", C.c_void_p)]
 
 
 # numpy views of the 20-/20-/12-byte records of ss.h
@@ -102,7 +105,7 @@ def lib():
         L.ss_project_points.argtypes = [P, i32, P, i32, P, P, C.c_float, P, P]
         L.ss_stereo_match.argtypes = [P, i32, P, i64, i32, P, P, P, C.c_float, C.c_float, P, P, P]
         L.ss_match_last_frame.argtypes = [P, i32, P, P, C.c_float, P, P, P, P, P, P, P, C.c_float, i32, i32, i32,
-                                          P, P, P]
+                                          P, P, P, P]
         L.ss_set_distribution.argtypes = [P, i32]
         L.ss_track_tick.argtypes = [P, i32, C.POINTER(ss_match_cfg), C.POINTER(ss_tick_io), P]
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
@@ -206,12 +209,12 @@ def ss_project_points(ctx, n_frames, d_cams, n_points, d_points, d_point_frame, 
 
 def ss_match_last_frame(ctx, n_frames, d_cams, d_last_cams, mb, d_kps, d_desc, d_counts, d_kp_taken, d_point_offsets,
                         d_points, d_point_desc, th, th_high, check_orientation, min_matches, d_out, d_n_matches=None,
-                        stream=None):
+                        d_kp_matched=None, stream=None):
     _check(lib().ss_match_last_frame(ctx, n_frames, _ptr(d_cams), _ptr(d_last_cams), float(mb), _ptr(d_kps),
                                      _ptr(d_desc), _ptr(d_counts), _ptr(d_kp_taken), _ptr(d_point_offsets),
                                      _ptr(d_points), _ptr(d_point_desc), float(th), int(th_high),
                                      int(check_orientation), int(min_matches), _ptr(d_out), _ptr(d_n_matches),
-                                     _stream(stream)), ctx)
+                                     _ptr(d_kp_matched), _stream(stream)), ctx)
 
 
 def ss_profile_events(ctx, events) -> None:

@@ -282,11 +282,12 @@ def _camera(c, R, t, shape, width, height):
 
 def make_last_frame(kps: np.ndarray, desc: np.ndarray, counts: np.ndarray, n_levels: int, n_per_level: np.ndarray,
                     width: int, height: int, shape: str, n_points_per_frame: int, seed: int, true_frac=0.70,
-                    pos_sigma=1.5, stereo_z=0.0):
+                    pos_sigma=1.5, stereo_z=0.0, cams=None):
     """The previous frame's tracked map points for frame-to-frame matching (O13, ORB-SLAM
     TrackWithMotionModel), per frame:
 
-    * the current camera: a random pose and the dataset's intrinsics, bounds [0, W] x [0, H];
+    * the current camera: a random pose (or the given `cams`, e.g. the local map's) and the
+      dataset's intrinsics, bounds [0, W] x [0, H];
       the last camera: the current one moved by stereo_z * U(-2, 2) along its optical axis
       (0 = the same pose; the stereo forward / backward gate needs |motion| > baseline);
     * true points (70 % of Q, at most the keypoint count): a keypoint's position +
@@ -302,6 +303,7 @@ def make_last_frame(kps: np.ndarray, desc: np.ndarray, counts: np.ndarray, n_lev
     F, cap = kps.shape
     Q = n_points_per_frame
     fx, fy, cx, cy = INTRINSICS[shape]
+    given = cams
     cams = np.zeros(F, CAMERA_DTYPE)
     last = np.zeros(F, CAMERA_DTYPE)
     pts = np.zeros(F * Q, FRAME_POINT_DTYPE)
@@ -309,8 +311,14 @@ def make_last_frame(kps: np.ndarray, desc: np.ndarray, counts: np.ndarray, n_lev
     pl = np.asarray(n_per_level, np.float64)
     pl = pl / pl.sum()
     for f in range(F):
-        R, t = _rotation(rng), rng.normal(0, 3.0, 3)
-        _camera(cams[f], R, t, shape, width, height)
+        if given is None:
+            R, t = _rotation(rng), rng.normal(0, 3.0, 3)
+        else:
+            R, t = given[f]["R"].reshape(3, 3).astype(np.float64), given[f]["t"].astype(np.float64)
+        if given is None:
+            _camera(cams[f], R, t, shape, width, height)
+        else:
+            cams[f] = given[f]
         tl = t + np.array([0.0, 0.0, stereo_z * rng.uniform(-2.0, 2.0)])
         _camera(last[f], R, tl, shape, width, height)
         n = int(counts[f, n_levels])

@@ -60,11 +60,18 @@ def _gpu_match(torch, p, kps, desc, counts, cams, last, pt_off, pts, pdesc, mb, 
     out = torch.full((max(n, 1), 3), 7, dtype=torch.int32, device=dev)
     nm = torch.full((F,), -5, dtype=torch.int32, device=dev)
     d_taken = tk(taken) if taken is not None else None
+    mask = torch.full((F, p.kp_capacity), 9, dtype=torch.uint8, device=dev)
     ss.ss_match_last_frame(pipe.ctx, F, d_cams, d_last, mb, d_kps, d_desc, d_counts, d_taken, d_off, d_pts, d_pd, th,
-                           100, check, min_matches, out, nm, torch.cuda.current_stream())
+                           100, check, min_matches, out, nm, mask, torch.cuda.current_stream())
     torch.cuda.synchronize()
     got = match_records(out)[:n]
     pipe.close()
+    # matched mask = taken | kept matches
+    want_mask = np.zeros((F, p.kp_capacity), np.uint8) if taken is None else (taken != 0).astype(np.uint8)
+    for f in range(F):
+        o = got[pt_off[f]:pt_off[f + 1]]
+        want_mask[f, o["idx"][o["idx"] >= 0]] = 1
+    assert (mask.cpu().numpy() == want_mask).all()
     return got, nm.cpu().numpy()
 
 
