@@ -7,8 +7,8 @@
 // has three frame-wide dependencies (the dedup of keypoints claimed by several points, the
 // rotation histogram's three maxima, and the "fewer than min_matches -> redo with 2*th"
 // retry), which are cluster barriers here instead of kernel boundaries:
-//   P0  the frame's keypoint row index (first keypoint per (level, row), the matcher's
-//       index) built by the cluster into global scratch;                       | cluster.sync
+//   P0  every CTA stages the frame's keypoint positions and builds its row index (first
+//       keypoint per (level, row)) in shared memory; claims reset;             | cluster.sync
 //   P1  eight lanes per point: pose transform + pinhole projection + bounds (single-rounded
 //       f32 ops in the oracle's order), octave-scaled window, level gate, exact |x-u| < r,
 //       |y-v| < r, 8 x POPC Hamming over the candidate runs of the row index, shuffle merge
@@ -32,9 +32,10 @@ namespace ss {
 namespace {
 
 constexpr int kCluster = 8;    // CTAs per frame (portable cluster size)
-constexpr int kThreads = 256;  // per CTA
+constexpr int kThreads = 512;   // per CTA (16 warps)
 constexpr int kLanes = 8;      // lanes per point in P1
 constexpr int kHisto = 30;     // ORB-SLAM HISTO_LENGTH
+constexpr size_t kLfSmemMax = 200 * 1024;
 
 __device__ __forceinline__ float dot3r(const float* a, float b0, float b1, float b2) {
   float s = __fmul_rn(a[0], b0);
@@ -77,6 +78,7 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
   __shared__ int s_hist[2][32];
   __shared__ int s_count[2];
   __shared__ int s_keep[3];
+  __shared__ int s_roff[kMaxLevels];
   cg::cluster_group cluster = cg::this_cluster();
   const int rank = (int)cluster.block_rank();
   const int f = blockIdx.x / kCluster;
@@ -85,6 +87,7 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
   const int L = g.L, cap = g.kp_capacity;
   if (threadIdx.x < 64) (&s_hist[0][0])[threadIdx.x] = 0;
   if (threadIdx.x < 2) s_count[threadIdx.x] = 0;
+  if (threadIdx.x < kMaxLevels) s_roff[threadIdx.x] = threadIdx.x < a.g.L ? row_off(a.g, threadIdx.x) : 0;
   pdl_wait();
   pdl_trigger();
   int* lead_hist = cluster.map_shared_rank(&s_hist[0][0], 0);
@@ -92,11 +95,18 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
 
   const ss_keypoint* fk = a.kps + (int64_t)f * cap;
   const int32_t* cnt = a.counts + f * (L + 1);
-  uint16_t* fri = a.rowidx + (int64_t)f * a.rows_per_frame;
+  // every CTA keeps its own copy of the frame's keypoint positions and row index in shared
+  // memory, so the window walk of P1 touches global memory only for descriptors
+  extern __shared__ float2 s_xy[];                                        // [cap]
+  uint16_t* fri = reinterpret_cast<uint16_t*>(s_xy + cap);                // [rows_per_frame]
   unsigned long long* fclaim = a.claim + (int64_t)f * cap;
   uint8_t* fmask = a.matched ? a.matched + (int64_t)f * cap : nullptr;
-  for (int k = ct; k < cap; k += nct) {  // P0
+  const int nk = cnt[L];
+  for (int k = threadIdx.x; k < cap; k += kThreads) {  // P0
     rowidx_fill(g, fk, cnt, fri, k);
+    if (k < nk) s_xy[k] = make_float2(fk[k].x, fk[k].y);
+  }
+  for (int k = ct; k < cap; k += nct) {
     fclaim[k] = ~0ull;
     if (fmask) fmask[k] = (a.taken && a.taken[(int64_t)f * cap + k]) ? 1 : 0;
   }
@@ -139,10 +149,11 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
           for (int l = l0; l <= l1; l++) {
             int rlo, rhi;
             window_rows(g, l, v, r, &rlo, &rhi);
-            const uint16_t* ri = fri + row_off(g, l);
+            const uint16_t* ri = fri + s_roff[l];
             const int kb = ri[rlo], ke = ri[rhi];
             for (int k = kb + sub; k < ke; k += kLanes) {
-              const float dx = __fsub_rn(fk[k].x, u), dy = __fsub_rn(fk[k].y, v);
+              const float2 xy = s_xy[k];
+              const float dx = __fsub_rn(xy.x, u), dy = __fsub_rn(xy.y, v);
               if (!(fabsf(dx) < r && fabsf(dy) < r)) continue;
               if (ft && ft[k]) continue;
               const int d = hamming256(qa, qb, fd[2 * k], fd[2 * k + 1]);
@@ -242,6 +253,14 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
 
 }  // namespace
 
+cudaError_t lastframe_init() {  // at ss_create (never inside a stream capture)
+  return cudaFuncSetAttribute(lastframe_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kLfSmemMax);
+}
+
+size_t lastframe_smem_bytes(const Geom& g) {
+  return sizeof(float2) * (size_t)g.kp_capacity + sizeof(uint16_t) * (size_t)match_rows_per_frame(g);
+}
+
 cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams, const ss_camera* last_cams, float mb,
                              const ss_keypoint* kps, const uint8_t* desc, const int32_t* counts, const uint8_t* taken,
                              const int32_t* pt_off, const ss_frame_point* pts, const uint8_t* pdesc, float th,
@@ -251,7 +270,9 @@ cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams,
   LfArgs a{g,     n_frames, cams,    last_cams,         mb,          kps, desc, counts,
            taken, pt_off,   pts,     pdesc,             th,          th_high, check_orientation,
            min_matches, out, n_matches, matched, claim, rowidx, match_rows_per_frame(g)};
-  cudaError_t e = launch_pdl(lastframe_kernel, dim3(n_frames * kCluster), dim3(kThreads), 0, s, a);
+  const size_t smem = lastframe_smem_bytes(g);
+  if (smem > kLfSmemMax) return cudaErrorInvalidValue;
+  cudaError_t e = launch_pdl(lastframe_kernel, dim3(n_frames * kCluster), dim3(kThreads), smem, s, a);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 

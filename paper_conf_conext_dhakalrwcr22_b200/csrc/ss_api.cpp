@@ -495,6 +495,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     ALLOC(c->brute_mexp, brute_tc_map_bytes(max_map));
   }
 #undef ALLOC
+  if (e == cudaSuccess) e = lastframe_init();
   if (e == cudaSuccess) e = cudaMemcpy(c->cells, c->cells_h.data(), sizeof(CellInfo) * c->cells_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->bands, c->bands_h.data(), sizeof(BandInfo) * c->bands_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess && !tab.empty()) e = cudaMemcpy(c->xytab, tab.data(), sizeof(uint32_t) * tab.size(), cudaMemcpyHostToDevice);
@@ -700,6 +701,8 @@ ss_status ss_match_last_frame(ss_ctx* c, int32_t n_frames, const ss_camera* d_ca
   if (n_frames < 0) return fail(SS_EINVAL, "negative size");
   if (n_frames > c->max_frames) return fail(SS_ECAPACITY, "n_frames exceeds the ctx's max_frames");
   if (!(th > 0.0f)) return fail(SS_EINVAL, "th must be > 0");
+  if (lastframe_smem_bytes(c->g) > 200 * 1024)
+    return fail(SS_EUNSUPPORTED, "kp_capacity too large for the frame-to-frame matcher's shared memory");
   if (n_frames == 0) return SS_OK;
   if (!d_cams || !d_kps || !d_desc || !d_counts || !d_point_offsets || !d_points || !d_point_desc || !d_out)
     return fail(SS_EINVAL, "NULL buffer");

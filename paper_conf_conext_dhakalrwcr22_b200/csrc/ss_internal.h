@@ -192,7 +192,10 @@ cudaError_t launch_stereo(const Geom& g, int n_pairs, FrameSrc src, const ss_key
 cudaError_t launch_stereo_outliers(const Geom& g, int n_pairs, const int32_t* counts, const int32_t* sad,
                                    float* uright, float* depth, cudaStream_t s);
 
-// O13 frame-to-frame projection matching (k_lastframe.cu): one cluster of CTAs per frame.
+// O13 frame-to-frame projection matching (k_lastframe.cu): one cluster of CTAs per frame;
+// dynamic shared memory per CTA (keypoint positions + row index), at most 200 KB.
+size_t lastframe_smem_bytes(const Geom& g);
+cudaError_t lastframe_init();  // kernel attributes (ss_create)
 cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams, const ss_camera* last_cams, float mb,
                              const ss_keypoint* kps, const uint8_t* desc, const int32_t* counts, const uint8_t* taken,
                              const int32_t* pt_off, const ss_frame_point* pts, const uint8_t* pdesc, float th,
