@@ -108,6 +108,32 @@ def window_inputs(p, kps, desc, counts, cfg, seed_lm, seed_lf, per_client):
     return cmf, pt, (pf * per_client).astype(np.int32), qd, tkf, lastf, offf, lp, ld
 
 
+def shard_range(n_map: int, rank: int, world: int) -> tuple[int, int]:
+    """Map-sharded brute force (F4): rank r holds global map rows [lo, hi) (contiguous, covering)."""
+    return n_map * rank // world, n_map * (rank + 1) // world
+
+
+def allgather_queries(desc, counts, world: int):
+    """Every rank's keypoint descriptors / counts of this tick, rank-major ([world*B, ...])."""
+    import torch
+    import torch.distributed as dist
+    ad = torch.empty((world * desc.shape[0],) + tuple(desc.shape[1:]), dtype=desc.dtype, device=desc.device)
+    ac = torch.empty((world * counts.shape[0],) + tuple(counts.shape[1:]), dtype=counts.dtype, device=counts.device)
+    dist.all_gather_into_tensor(ad, desc.contiguous())
+    dist.all_gather_into_tensor(ac, counts.contiguous())
+    return ad, ac
+
+
+def exchange_partials(top2_all, world: int):
+    """top2_all [world*B, cap, 2] (this rank's shard top-2 for every rank's frames, rank-major)
+    -> [world, B, cap, 2]: every shard's top-2 for THIS rank's frames (all-to-all)."""
+    import torch
+    import torch.distributed as dist
+    recv = torch.empty_like(top2_all)
+    dist.all_to_all_single(recv, top2_all.contiguous())
+    return recv.reshape((world, top2_all.shape[0] // world) + tuple(top2_all.shape[1:]))
+
+
 def _gen_frame(args):
     w, h, seed, stereo = args
     if stereo:
@@ -265,7 +291,8 @@ def run_ours(args, cfg):
     L = 8
     Q = cfg["queries"] * len(clients)
     window = cfg["mode"] == "window"
-    pipe = OrbPipeline(w, h, cfg["nf"], L, max_frames=B, max_queries=max(Q, 1), max_map=cfg["map"], device=local)
+    pipe = OrbPipeline(w, h, cfg["nf"], L, max_frames=B * (world if args.map_shard else 1), max_queries=max(Q, 1),
+                       max_map=cfg["map"], device=local)
     dist_mode = ss.SS_DIST_GRID_TOPN if args.dist == "grid" else ss.SS_DIST_QUADTREE
     pipe.set_distribution(dist_mode)
     p = pipe.params
@@ -331,6 +358,9 @@ def run_ours(args, cfg):
         map_desc = torch.from_numpy(mp).to(dev)
         if world > 1:
             dist.broadcast(map_desc, src=0)
+        if args.map_shard:  # F4: keep only this rank's rows (global index offset lo)
+            shard_lo, shard_hi = shard_range(cfg["map"], rank, world)
+            map_desc = map_desc[shard_lo:shard_hi].contiguous()
         q_host = None
     torch.cuda.synchronize(dev)
 
@@ -339,8 +369,14 @@ def run_ours(args, cfg):
     mode = ss.SS_MATCH_WINDOW if window else ss.SS_MATCH_BRUTE
     stereo = bool(cfg.get("stereo"))
     ek = ss.extract_kernels(L)
+    shard = bool(args.map_shard) and not window
+    eager_tail = shard and world > 1  # the sharded exchange runs eagerly after the graph (NCCL)
     mk = (["stereo_prepare", "stereo", "stereo_outliers"] if stereo else []) + \
-        (["lastframe", "project"] if window else []) + ss.match_kernels(mode, True)
+        (["lastframe", "project"] if window else []) + \
+        (["brute_expand", "brute_tc", "brute_shard_top2", "brute_parts_merge"] if shard
+         else ss.match_kernels(mode, True))
+    if eager_tail:
+        mk = []
     BASE_M = synth.STEREO_BASELINE.get(cfg["shape"], 0.0)
     BF = float(np.float32(synth.INTRINSICS[cfg["shape"]][0] * BASE_M))
     base = ss.extract_events(L)
@@ -356,8 +392,8 @@ def run_ours(args, cfg):
     # ticks in flight: P independent contexts (scratch + outputs) on P streams, so consecutive
     # ticks overlap on the GPU the way the paper's clients share it; P = 1 serialises
     P = max(1, args.inflight)
-    pipes = [pipe] + [OrbPipeline(w, h, cfg["nf"], L, max_frames=B, max_queries=max(Q, 1), max_map=cfg["map"],
-                                  device=local) for _ in range(P - 1)]
+    pipes = [pipe] + [OrbPipeline(w, h, cfg["nf"], L, max_frames=B * (world if shard else 1), max_queries=max(Q, 1),
+                                  max_map=cfg["map"], device=local) for _ in range(P - 1)]
     for pp in pipes:
         pp.set_distribution(dist_mode)
     outs = [out] + [torch.zeros_like(out) for _ in range(P - 1)]
@@ -365,6 +401,22 @@ def run_ours(args, cfg):
     lf_out = [torch.zeros((max(NLF, 1), 3), dtype=torch.int32, device=dev) for _ in range(P)]
     lf_n = [torch.zeros(B, dtype=torch.int32, device=dev) for _ in range(P)]
     lf_mask = [torch.zeros((B, cap), dtype=torch.uint8, device=dev) for _ in range(P)]
+    # F4 map-sharded brute force: shard top-2 for every rank's frames, exchanged, merged
+    top2_all = [torch.zeros((B * world, cap, 2), dtype=torch.int64, device=dev) for _ in range(P)] if shard else None
+    bcfg = ss.brute_cfg()
+
+    def sharded_tail(q, st):
+        pp = pipes[q]
+        with torch.cuda.stream(st):
+            if world > 1:
+                qd, qc = allgather_queries(pp.desc[:B], pp.counts[:B], world)
+            else:
+                qd, qc = pp.desc[:B], pp.counts[:B]
+            ss.ss_match_brute_partial(pp.ctx, B * world, qd, qc, map_desc, map_desc.shape[0], shard_lo, top2_all[q],
+                                      st)
+            parts = exchange_partials(top2_all[q], world) if world > 1 else top2_all[q]
+            ss.ss_match_brute_merge(pp.ctx, B, pp.counts[:B], world, parts, bcfg, outs[q], st)
+
     npairs = B // 2 if stereo else 0
     st_out = [(torch.zeros((max(npairs, 1), cap), dtype=torch.float32, device=dev),
                torch.zeros((max(npairs, 1), cap), dtype=torch.float32, device=dev)) for _ in range(P)]
@@ -389,6 +441,9 @@ def run_ours(args, cfg):
                                     min_matches=20, taken=taken[s], matched=lf_mask[q], stream=st)
                 pp.project(B, cams[s], points[s], point_frame[s], qbufs[q], th=cfg["th"], stream=st)
                 pp.match_window(B, qbufs[q], qdesc[s], ot, taken=lf_mask[q], stream=st)
+            elif shard:
+                if not eager_tail:
+                    sharded_tail(q, st)
             else:
                 pp.match_brute(B, map_desc, ot, stream=st)
         if prof:
@@ -423,6 +478,8 @@ def run_ours(args, cfg):
                 if marks is not None:
                     marks[0][i].record(streams[q])
                 graphs[q][s].replay()
+                if eager_tail:
+                    sharded_tail(q, streams[q])
                 if marks is not None:
                     marks[1][i].record(streams[q])
             if world > 1:
@@ -535,8 +592,13 @@ def run_ours(args, cfg):
             pass
 
     # --- e2e through the public API with host buffers (pinned), copies inside the timed region
-    e2e = run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=cfg["th"],
-                  stereo=(BF, BASE_M, st_out) if stereo else None, lf=(MB, cfg.get("lf_th", 15.0)))
+    if eager_tail:  # ss_track_tick has no cross-rank exchange: no end-to-end number for a sharded map
+        e2e = {"value": None, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0,
+               "note": "map-sharded brute force over N > 1 ranks needs the NCCL exchange between the partial and "
+                       "merge calls; ss_track_tick serves a replicated map only"}
+    else:
+        e2e = run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=cfg["th"],
+                      stereo=(BF, BASE_M, st_out) if stereo else None, lf=(MB, cfg.get("lf_th", 15.0)))
 
     frames_per_step = B * world
     value = frames_per_step * K / (T_max / 1000.0)
@@ -552,7 +614,9 @@ def run_ours(args, cfg):
                    "l2": f"inputs ring of {n_slots} distinct slots = {n_slots * slot_bytes / 2**20:.0f} MiB "
                          f"> L2 {l2 / 2**20:.0f} MiB (no flush)",
                    "cuda_graphs": True, "ticks_in_flight": P, "setup_s": round(setup_s, 1),
-                   "distribution": "grid top-N (O4g)" if args.dist == "grid" else "quadtree (O4)"},
+                   "distribution": "grid top-N (O4g)" if args.dist == "grid" else "quadtree (O4)",
+                   "map": ("sharded over ranks (F4: shard top-2 for all ranks' frames, all-to-all, merge)"
+                           if shard else ("replicated" if not window else None))},
         "latency_ms": {"p50": float(np.percentile(step_ms, 50)), "p99": float(np.percentile(step_ms, 99)),
                        "samples": len(step_ms),
                        "note": f"per-frame latency = its tick's device time from start to end on its stream "
@@ -835,6 +899,8 @@ def main(argv=None):
     ap.add_argument("--inflight", type=int, default=4, help="ticks in flight (contexts/streams)")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--map-shard", action="store_true",
+                    help="brute configs: partition the map over the ranks (F4: shard top-2, all-to-all, merge)")
     ap.add_argument("--dist", choices=["quadtree", "grid"], default="quadtree",
                     help="keypoint distribution: ORB-SLAM quadtree (O4) or grid top-N (O4g)")
     args = ap.parse_args(argv)

@@ -170,6 +170,26 @@ ss_status ss_match_projection(ss_ctx* ctx, int32_t n_frames, const ss_keypoint* 
                               const ss_mp_query* d_queries, const uint8_t* d_map_desc, int32_t n_map,
                               const ss_match_cfg* cfg, ss_match* d_out, ss_stream_t stream);
 
+/* Map-sharded brute force (DESIGN.md §3 item 15): O10 with the map
+ * partitioned across ranks.  Each rank runs ss_match_brute_partial for the frames to match
+ * (typically every rank's frames, all-gathered) against its shard, the partial results are
+ * exchanged (all-to-all), and the frames' owner runs ss_match_brute_merge over the parts.
+ * For shards that partition [0, M) (map_offset = the shard's first global index), the merge is
+ * bit-identical to ss_match_projection BRUTE over the whole map.  Device pointers:
+ *   ss_match_brute_partial: d_desc / d_counts as ss_orb_extract writes them; d_map_desc
+ *     [n_map][32] (the shard); d_top2 [n_frames][kp_capacity][2] u64: per keypoint the two
+ *     smallest (distance << 32 | (map_offset + m)) over the shard, UINT64_MAX = none (also for
+ *     slots >= the frame's count).  SS_ECAPACITY if n_frames > max_frames or n_map > max_map;
+ *     SS_EINVAL for negative sizes / offset, map_offset + n_map > 2^31 - 1 or NULL buffers.
+ *   ss_match_brute_merge: d_parts [n_parts][n_frames][kp_capacity][2] (the shards' d_top2,
+ *     any order), cfg as BRUTE (th, ratio); d_out [n_frames][kp_capacity] as
+ *     ss_match_projection BRUTE (idx = global map index or -1).  n_parts >= 1. */
+ss_status ss_match_brute_partial(ss_ctx* ctx, int32_t n_frames, const uint8_t* d_desc, const int32_t* d_counts,
+                                 const uint8_t* d_map_desc, int32_t n_map, int32_t map_offset, uint64_t* d_top2,
+                                 ss_stream_t stream);
+ss_status ss_match_brute_merge(ss_ctx* ctx, int32_t n_frames, const int32_t* d_counts, int32_t n_parts,
+                               const uint64_t* d_parts, const ss_match_cfg* cfg, ss_match* d_out, ss_stream_t stream);
+
 /* O11: the per-map-point half of "search local points" (ORB-SLAM3
  * Frame::isInFrustum + MapPoint::PredictScale + ORBmatcher::RadiusByViewingCos): map point
  * i is tested against the camera of frame d_point_frame[i] and written as WINDOW query i.
@@ -336,7 +356,8 @@ ss_status ss_track_tick(ss_ctx* ctx, int32_t n_frames, const ss_match_cfg* cfg, 
  * alone).  WINDOW match: a pair per kernel
  * (match_prepare, match_window[, match_resolve if dedup]); BRUTE: brute_expand, brute_tc,
  * brute_merge; ss_project_points: project; ss_stereo_match: stereo_prepare, stereo, stereo_outliers;
- * ss_match_last_frame: lastframe.
+ * ss_match_last_frame: lastframe; ss_match_brute_partial: brute_expand, brute_tc, brute_shard_top2;
+ * ss_match_brute_merge: brute_parts_merge.
  * Works under CUDA-graph stream capture (the records become graph event nodes).
  * *next_index (may be NULL) receives the index of the next event to be recorded. */
 ss_status ss_profile_events(ss_ctx* ctx, void* const* events, int32_t n_events);

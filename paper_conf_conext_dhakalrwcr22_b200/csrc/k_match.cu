@@ -155,7 +155,86 @@ __global__ void __launch_bounds__(256) match_brute_merge(Geom g, int F, const in
   out[gq] = m;
 }
 
+// Map-sharded brute force (F4): per slot, the per-split partial top-2 of one map shard reduced
+// to its two smallest (distance << 32 | (map_offset + m)); slots >= the frame's count get
+// (~0, ~0).  Global indices keep the (distance, index) order of the unsharded matcher.
+__global__ void __launch_bounds__(256) brute_shard_top2(Geom g, int F, const int32_t* __restrict__ counts, int splits,
+                                                        const unsigned long long* __restrict__ partial, int map_offset,
+                                                        unsigned long long* __restrict__ top2) {
+  pdl_wait();
+  pdl_trigger();
+  const int gq = blockIdx.x * blockDim.x + threadIdx.x;
+  const int cap = g.kp_capacity, L = g.L;
+  if (gq >= F * cap) return;
+  const int f = gq / cap, k = gq - f * cap;
+  unsigned long long b1 = ~0ull, b2 = ~0ull;
+  if (k < counts[f * (L + 1) + L]) {
+    for (int s = 0; s < splits * 2; s++) {
+      const unsigned long long key = partial[(int64_t)gq * splits * 2 + s];
+      if (key < b1) {
+        b2 = b1;
+        b1 = key;
+      } else if (key < b2) {
+        b2 = key;
+      }
+    }
+    if (b1 != ~0ull) b1 += (unsigned)map_offset;  // index field: m < 2^31 - offset (checked on the host)
+    if (b2 != ~0ull) b2 += (unsigned)map_offset;
+  }
+  top2[(int64_t)gq * 2] = b1;
+  top2[(int64_t)gq * 2 + 1] = b2;
+}
+
+// Merge of n_parts shard top-2 lists [part][slot][2] + the O10 accept rule.
+__global__ void __launch_bounds__(256) brute_parts_merge(Geom g, int F, const int32_t* __restrict__ counts,
+                                                         int n_parts, const unsigned long long* __restrict__ parts,
+                                                         ss_match_cfg cfg, ss_match* __restrict__ out) {
+  pdl_wait();
+  pdl_trigger();
+  const int gq = blockIdx.x * blockDim.x + threadIdx.x;
+  const int cap = g.kp_capacity, L = g.L;
+  const int64_t nslots = (int64_t)F * cap;
+  if (gq >= nslots) return;
+  const int f = gq / cap, k = gq - f * cap;
+  ss_match m;
+  m.idx = -1;
+  m.dist = 256;
+  m.dist2 = 256;
+  if (k < counts[f * (L + 1) + L]) {
+    unsigned long long b1 = ~0ull, b2 = ~0ull;
+    for (int r = 0; r < n_parts; r++) {
+      const unsigned long long* pr = parts + ((int64_t)r * nslots + gq) * 2;
+      merge_top2(b1, b2, pr[0], pr[1]);
+    }
+    const int d1 = b1 == ~0ull ? 256 : (int)(b1 >> 32);
+    const int d2 = b2 == ~0ull ? 256 : (int)(b2 >> 32);
+    m.dist = d1;
+    m.dist2 = d2;
+    if (b1 != ~0ull && d1 <= cfg.th && cfg.ratio_den * d1 < cfg.ratio_num * d2) m.idx = (int)(b1 & 0xFFFFFFFFu);
+  }
+  out[gq] = m;
+}
+
 }  // namespace
+
+cudaError_t launch_brute_shard_top2(const Geom& g, int n_frames, const int32_t* counts, int splits,
+                                    const unsigned long long* partial, int map_offset, unsigned long long* top2,
+                                    cudaStream_t s) {
+  const int nslots = n_frames * g.kp_capacity;
+  if (nslots <= 0) return cudaSuccess;
+  cudaError_t e = launch_pdl(brute_shard_top2, dim3((nslots + 255) / 256), dim3(256), 0, s, g, n_frames, counts, splits,
+                             partial, map_offset, top2);
+  return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+cudaError_t launch_brute_parts_merge(const Geom& g, int n_frames, const int32_t* counts, int n_parts,
+                                     const unsigned long long* parts, ss_match_cfg cfg, ss_match* out, cudaStream_t s) {
+  const int nslots = n_frames * g.kp_capacity;
+  if (nslots <= 0) return cudaSuccess;
+  cudaError_t e = launch_pdl(brute_parts_merge, dim3((nslots + 255) / 256), dim3(256), 0, s, g, n_frames, counts,
+                             n_parts, parts, cfg, out);
+  return e != cudaSuccess ? e : cudaGetLastError();
+}
 
 int match_rows_per_frame(const Geom& g) { return row_off(g, g.L); }
 

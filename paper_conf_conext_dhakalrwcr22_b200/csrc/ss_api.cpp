@@ -1,6 +1,7 @@
 // ss_api.cpp -- host side of libss: parameter derivation, validation, scratch ownership and
 // the launch sequence of each C-ABI entry point (include/ss.h).  No per-call allocation,
 // no host synchronisation on the hot path; every entry point returns a status.
+#include <climits>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -645,6 +646,56 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
     return SS_OK;
   }
   return fail(SS_EINVAL, "unknown match mode");
+}
+
+ss_status ss_match_brute_partial(ss_ctx* c, int32_t n_frames, const uint8_t* d_desc, const int32_t* d_counts,
+                                 const uint8_t* d_map_desc, int32_t n_map, int32_t map_offset, uint64_t* d_top2,
+                                 ss_stream_t stream) {
+  if (!c) return fail(SS_EINVAL, "NULL ctx");
+  if (n_frames < 0 || n_map < 0 || map_offset < 0) return fail(SS_EINVAL, "negative size / offset");
+  if (n_frames > c->max_frames) return fail(SS_ECAPACITY, "n_frames exceeds the ctx's max_frames");
+  if (n_map > c->max_map) return fail(SS_ECAPACITY, "n_map exceeds the ctx's max_map");
+  if ((int64_t)map_offset + n_map > INT32_MAX) return fail(SS_EINVAL, "map_offset + n_map exceeds 2^31 - 1");
+  if (n_frames == 0) return SS_OK;
+  if (!d_desc || !d_counts || !d_top2 || (n_map > 0 && !d_map_desc)) return fail(SS_EINVAL, "NULL buffer");
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  SS_CUDA_TRY(check_stream(s));
+  const int n_slots = n_frames * c->g.kp_capacity;
+  unsigned long long* top2 = reinterpret_cast<unsigned long long*>(d_top2);
+  if (n_map == 0) {  // an empty shard contributes nothing
+    SS_CUDA_TRY(cudaMemsetAsync(top2, 0xFF, sizeof(unsigned long long) * 2 * n_slots, s));
+    return SS_OK;
+  }
+  const int splits = brute_tc_splits(n_slots, n_map, c->max_splits, c->n_sm);
+  prof_mark(c, s);
+  SS_CUDA_TRY(launch_brute_expand(n_slots, d_desc, n_map, d_map_desc, c->brute_qexp, c->brute_mexp, s));
+  prof_mark(c, s);
+  prof_mark(c, s);
+  SS_CUDA_TRY(launch_brute_tc(n_slots, n_map, c->brute_qexp, c->brute_mexp, splits, c->partial, s));
+  prof_mark(c, s);
+  prof_mark(c, s);
+  SS_CUDA_TRY(launch_brute_shard_top2(c->g, n_frames, d_counts, splits, c->partial, map_offset, top2, s));
+  prof_mark(c, s);
+  return SS_OK;
+}
+
+ss_status ss_match_brute_merge(ss_ctx* c, int32_t n_frames, const int32_t* d_counts, int32_t n_parts,
+                               const uint64_t* d_parts, const ss_match_cfg* cfg, ss_match* d_out, ss_stream_t stream) {
+  if (!c || !cfg) return fail(SS_EINVAL, "NULL ctx/cfg");
+  if (n_frames < 0 || n_parts < 1) return fail(SS_EINVAL, "n_frames < 0 or n_parts < 1");
+  if (n_frames > c->max_frames) return fail(SS_ECAPACITY, "n_frames exceeds the ctx's max_frames");
+  if (cfg->ratio_den <= 0 || cfg->ratio_num < 0) return fail(SS_EINVAL, "bad ratio");
+  if (n_frames == 0) return SS_OK;
+  if (!d_counts || !d_parts || !d_out) return fail(SS_EINVAL, "NULL buffer");
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  SS_CUDA_TRY(check_stream(s));
+  prof_mark(c, s);
+  SS_CUDA_TRY(launch_brute_parts_merge(c->g, n_frames, d_counts, n_parts,
+                                       reinterpret_cast<const unsigned long long*>(d_parts), *cfg, d_out, s));
+  prof_mark(c, s);
+  return SS_OK;
 }
 
 ss_status ss_stereo_match(ss_ctx* c, int32_t n_pairs, const uint8_t* d_frames, int64_t frame_stride, int32_t pitch,

@@ -165,6 +165,13 @@ cudaError_t launch_match_resolve(const Geom& g, int n_queries, const ss_mp_query
 cudaError_t launch_brute_merge(const Geom& g, int n_frames, const int32_t* counts, int splits,
                                const unsigned long long* partial, ss_match_cfg cfg, ss_match* out,
                                cudaStream_t s);
+// Map-sharded brute force (F4): one shard's top-2 with global indices, and the merge of the
+// shards' top-2 lists + the accept rule.
+cudaError_t launch_brute_shard_top2(const Geom& g, int n_frames, const int32_t* counts, int splits,
+                                    const unsigned long long* partial, int map_offset, unsigned long long* top2,
+                                    cudaStream_t s);
+cudaError_t launch_brute_parts_merge(const Geom& g, int n_frames, const int32_t* counts, int n_parts,
+                                     const unsigned long long* parts, ss_match_cfg cfg, ss_match* out, cudaStream_t s);
 // Tensor-core brute matcher (k_brute_tc.cu): expanded-operand scratch sizes, the map split
 // count (whole waves of one CTA per SM), and expand + tcgen05 partial top-2 (per-split partial
 // top-2, reduced by launch_brute_merge).

@@ -106,6 +106,8 @@ def lib():
         L.ss_stereo_match.argtypes = [P, i32, P, i64, i32, P, P, P, C.c_float, C.c_float, P, P, P]
         L.ss_match_last_frame.argtypes = [P, i32, P, P, C.c_float, P, P, P, P, P, P, P, C.c_float, i32, i32, i32,
                                           P, P, P, P]
+        L.ss_match_brute_partial.argtypes = [P, i32, P, P, P, i32, i32, P, P]
+        L.ss_match_brute_merge.argtypes = [P, i32, P, i32, P, C.POINTER(ss_match_cfg), P, P]
         L.ss_set_distribution.argtypes = [P, i32]
         L.ss_track_tick.argtypes = [P, i32, C.POINTER(ss_match_cfg), C.POINTER(ss_tick_io), P]
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
@@ -116,7 +118,7 @@ def lib():
         L.ss_profile_next.argtypes = [P, C.POINTER(i32)]
         for fn in ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_orb_extract", "ss_match_projection",
                    "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_set_distribution",
-                   "ss_match_last_frame", "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
+                   "ss_match_last_frame", "ss_match_brute_partial", "ss_match_brute_merge", "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
                    "ss_profile_next", "ss_debug_phase_times"):
             getattr(L, fn).restype = C.c_int
         _lib = L
@@ -125,7 +127,7 @@ def lib():
 
 EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "ss_orb_extract",
             "ss_match_projection", "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_set_distribution",
-            "ss_match_last_frame", "ss_profile_events", "ss_profile_next", "ss_debug_level",
+            "ss_match_last_frame", "ss_match_brute_partial", "ss_match_brute_merge", "ss_profile_events", "ss_profile_next", "ss_debug_level",
             "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times")
 
 
@@ -215,6 +217,16 @@ def ss_match_last_frame(ctx, n_frames, d_cams, d_last_cams, mb, d_kps, d_desc, d
                                      _ptr(d_points), _ptr(d_point_desc), float(th), int(th_high),
                                      int(check_orientation), int(min_matches), _ptr(d_out), _ptr(d_n_matches),
                                      _ptr(d_kp_matched), _stream(stream)), ctx)
+
+
+def ss_match_brute_partial(ctx, n_frames, d_desc, d_counts, d_map_desc, n_map, map_offset, d_top2, stream=None):
+    _check(lib().ss_match_brute_partial(ctx, n_frames, _ptr(d_desc), _ptr(d_counts), _ptr(d_map_desc), n_map,
+                                        map_offset, _ptr(d_top2), _stream(stream)), ctx)
+
+
+def ss_match_brute_merge(ctx, n_frames, d_counts, n_parts, d_parts, cfg: "ss_match_cfg", d_out, stream=None):
+    _check(lib().ss_match_brute_merge(ctx, n_frames, _ptr(d_counts), n_parts, _ptr(d_parts), C.byref(cfg),
+                                      _ptr(d_out), _stream(stream)), ctx)
 
 
 def ss_profile_events(ctx, events) -> None:
