@@ -598,7 +598,8 @@ def run_ours(args, cfg):
                        "merge calls; ss_track_tick serves a replicated map only"}
     else:
         e2e = run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=cfg["th"],
-                      stereo=(BF, BASE_M, st_out) if stereo else None, lf=(MB, cfg.get("lf_th", 15.0)))
+                      stereo=(BF, BASE_M, st_out) if stereo else None, lf=(MB, cfg.get("lf_th", 15.0)),
+                      dev_map=(points, point_frame, qdesc, taken, lf_pts, lf_desc, lf_last) if window else None)
 
     frames_per_step = B * world
     value = frames_per_step * K / (T_max / 1000.0)
@@ -643,7 +644,7 @@ def run_ours(args, cfg):
 
 
 def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=1.0, stereo=None,
-            lf=(0.0, 15.0)):
+            lf=(0.0, 15.0), dev_map=None):
     """Same ticks end to end from pinned host buffers through ONE C-ABI call per tick
     (ss_track_tick: H2D of the tick's frames and local maps, extract, stereo, projection +
     match or brute match, D2H of every output), all inside the timed region; ticks
@@ -680,62 +681,86 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
             o["depth"] = torch.empty((B // 2) * cap, dtype=torch.float32).pin_memory()
         host_out.append(o)
     cfg = ss.window_cfg() if window else ss.brute_cfg()
-    ios = []
-    for q in range(P):
-        row = []
-        for i in range(n_host):
-            io = ss.ss_tick_io()
-            io.frames, io.frame_stride, io.pitch = fr[i].data_ptr(), H * W, W
-            if stereo:
-                io.bf, io.baseline = stereo[0], stereo[1]
-            if window:
-                cm, pt, pf, qd, tk, last, off, lp, ld = hin[i]
-                io.cams, io.n_points, io.points, io.point_frame = cm.data_ptr(), Q, pt.data_ptr(), pf.data_ptr()
-                io.point_desc, io.taken, io.th = qd.data_ptr(), tk.data_ptr(), th
-                io.lf_offsets, io.lf_points, io.lf_desc = off.data_ptr(), lp.data_ptr(), ld.data_ptr()
-                io.last_cams, io.mb, io.lf_th, io.lf_min_matches = last.data_ptr(), lf[0], lf[1], 20
-                io.lf_matches, io.lf_n_matches = o["lf_matches"].data_ptr(), o["lf_n"].data_ptr()
-            else:
-                io.d_map_desc, io.n_map = map_desc.data_ptr(), map_desc.shape[0]
-            o = host_out[q]
-            io.kps, io.desc, io.counts = o["kps"].data_ptr(), o["desc"].data_ptr(), o["counts"].data_ptr()
-            io.matches = o["matches"].data_ptr()
-            if stereo:
-                io.uright, io.depth = o["uright"].data_ptr(), o["depth"].data_ptr()
-            row.append(io)
-        ios.append(row)
-    # bytes actually copied per tick (the last cameras only in stereo, when mb > 0)
-    h2d = fr[0].numel() + (sum(a.numel() for j, a in enumerate(hin[0]) if j != 5 or lf[0] > 0) if window else 0)
-    d2h = sum(t.numel() * t.element_size() for t in host_out[0].values())
     handles = [st.cuda_stream for st in streams]
-
-    def step(s):
-        i, q = s % n_host, s % P
-        ss.ss_track_tick(pipes[q].ctx, B, cfg, ios[q][i], handles[q])
-
-    K = max(1, min(args.steps, 200))
-    for s in range(3):
-        step(s)
-    torch.cuda.synchronize(dev)
-    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    t0.record(streams[0])
-    for q in range(1, P):
-        streams[q].wait_event(t0)
-    for s in range(K):
-        step(s)
-    for q in range(1, P):
-        streams[0].wait_stream(streams[q])
-    t1.record(streams[0])
-    torch.cuda.synchronize(dev)
-    ms = t0.elapsed_time(t1)
     world = int(os.environ.get("WORLD_SIZE", 1))
-    return {"value": B * world * K / (ms / 1000.0), "unit": "frames/s", "h2d_bytes_per_step": int(h2d),
-            "d2h_bytes_per_step": int(d2h), "steps": K, "ms_per_step": ms / K, "ticks_in_flight": P,
-            "path": "pinned host -> ss_track_tick (one C-ABI call per tick: H2D, ss_orb_extract, " +
-                    ("ss_stereo_match, " if stereo else "") +
-                    ("ss_match_last_frame, ss_project_points, ss_match_projection WINDOW" if window
-                     else "ss_match_projection BRUTE") +
-                    ", D2H of all outputs; no graphs)"}
+    d2h = sum(t.numel() * t.element_size() for t in host_out[0].values())
+
+    def measure(resident: bool):
+        """resident: the map state (local-map points, last-frame points, masks) is the server's,
+        kept in HBM across ticks (dev_map, slot i); per tick only frames, camera predictions and
+        the last-frame offsets come from the host."""
+        ios = []
+        for q in range(P):
+            row = []
+            o = host_out[q]
+            for i in range(n_host):
+                io = ss.ss_tick_io()
+                io.frames, io.frame_stride, io.pitch = fr[i].data_ptr(), H * W, W
+                if stereo:
+                    io.bf, io.baseline = stereo[0], stereo[1]
+                if window:
+                    cm, pt, pf, qd, tk, last, off, lp, ld = hin[i]
+                    if resident:
+                        pt, pf, qd, tk, lp, ld, last = (t_[i] for t_ in dev_map)
+                    io.map_resident = int(resident)
+                    io.cams, io.n_points, io.points, io.point_frame = cm.data_ptr(), Q, pt.data_ptr(), pf.data_ptr()
+                    io.point_desc, io.taken, io.th = qd.data_ptr(), tk.data_ptr(), th
+                    io.lf_offsets, io.lf_points, io.lf_desc = off.data_ptr(), lp.data_ptr(), ld.data_ptr()
+                    io.last_cams, io.mb, io.lf_th, io.lf_min_matches = last.data_ptr(), lf[0], lf[1], 20
+                    io.lf_matches, io.lf_n_matches = o["lf_matches"].data_ptr(), o["lf_n"].data_ptr()
+                else:
+                    io.d_map_desc, io.n_map = map_desc.data_ptr(), map_desc.shape[0]
+                io.kps, io.desc, io.counts = o["kps"].data_ptr(), o["desc"].data_ptr(), o["counts"].data_ptr()
+                io.matches = o["matches"].data_ptr()
+                if stereo:
+                    io.uright, io.depth = o["uright"].data_ptr(), o["depth"].data_ptr()
+                row.append(io)
+            ios.append(row)
+        # bytes actually copied per tick (hin: cams, points, point_frame, qdesc, taken, last_cams,
+        # lf_offsets, lf_points, lf_desc; the last cameras only in stereo, when mb > 0)
+        if not window:
+            h2d = fr[0].numel()
+        elif resident:
+            h2d = fr[0].numel() + hin[0][0].numel() + hin[0][6].numel()
+        else:
+            h2d = fr[0].numel() + sum(a.numel() for j, a in enumerate(hin[0]) if j != 5 or lf[0] > 0)
+
+        def step(s):
+            i, q = s % n_host, s % P
+            ss.ss_track_tick(pipes[q].ctx, B, cfg, ios[q][i], handles[q])
+
+        K = max(1, min(args.steps, 200))
+        for s in range(3):
+            step(s)
+        torch.cuda.synchronize(dev)
+        t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        t0.record(streams[0])
+        for q in range(1, P):
+            streams[q].wait_event(t0)
+        for s in range(K):
+            step(s)
+        for q in range(1, P):
+            streams[0].wait_stream(streams[q])
+        t1.record(streams[0])
+        torch.cuda.synchronize(dev)
+        ms = t0.elapsed_time(t1)
+        return {"value": B * world * K / (ms / 1000.0), "unit": "frames/s", "h2d_bytes_per_step": int(h2d),
+                "d2h_bytes_per_step": int(d2h), "steps": K, "ms_per_step": ms / K, "ticks_in_flight": P}
+
+    path = ("one C-ABI call per tick: H2D, ss_orb_extract, " + ("ss_stereo_match, " if stereo else "") +
+            ("ss_match_last_frame, ss_project_points, ss_match_projection WINDOW" if window
+             else "ss_match_projection BRUTE") + ", D2H of all outputs; no graphs")
+    if not window or dev_map is None:
+        r = measure(False)
+        r["path"] = "pinned host -> ss_track_tick (" + path + ")" + \
+            ("; the shared map is device-resident server state" if not window else "")
+        return r
+    r = measure(True)
+    r["path"] = ("pinned host frames + camera predictions -> ss_track_tick (" + path + "); the map state (each "
+                 "client's local-map points, last-frame points, masks) is server state resident in HBM, "
+                 "as the SLAM-Share server keeps the maps and clients upload only frames (P:L64, P:L68); host_map = the same with it copied too")
+    r["host_map"] = measure(False)
+    return r
 
 
 # ----------------------------------------------------------------------------- oracle (CPU) legs

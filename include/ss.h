@@ -328,6 +328,10 @@ typedef struct {
   int32_t lf_min_matches;
   ss_match* lf_matches;
   int32_t* lf_n_matches;
+  /* 1 = the map state is DEVICE-resident (the server's map, kept in HBM across ticks):
+   * points, point_frame, point_desc, taken, lf_points, lf_desc and last_cams are device
+   * pointers and are not copied; frames, cams and lf_offsets stay host inputs. */
+  int32_t map_resident;
 } ss_tick_io;
 
 /* One tick of the hot path for a batch of client frames, enqueued on `stream` from a single

@@ -821,22 +821,33 @@ ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, co
       SS_CUDA_TRY(cudaMemcpy2DAsync(c->io_frames + f * fstride, P, io->frames + f * io->frame_stride, io->pitch, g.W,
                                     g.H, cudaMemcpyHostToDevice, s));
   }
+  // map state: host copies staged into the ctx, or (map_resident) the caller's device buffers
+  const bool res = io->map_resident != 0;
+  const ss_map_point* d_points = res ? io->points : c->io_points;
+  const int32_t* d_pf = res ? io->point_frame : c->io_pf;
+  const uint8_t* d_pdesc = res ? io->point_desc : c->io_pdesc;
+  const uint8_t* d_taken = io->taken ? (res ? io->taken : c->io_taken) : nullptr;
+  const ss_frame_point* d_lf_pts = res ? io->lf_points : c->io_lf_pts;
+  const uint8_t* d_lf_desc = res ? io->lf_desc : c->io_lf_desc;
+  const ss_camera* d_last = res ? io->last_cams : c->io_last_cams;
   if (window) {
     const int64_t n = io->n_points;
     SS_CUDA_TRY(cudaMemcpyAsync(c->io_cams, io->cams, sizeof(ss_camera) * n_frames, cudaMemcpyHostToDevice, s));
-    SS_CUDA_TRY(cudaMemcpyAsync(c->io_points, io->points, sizeof(ss_map_point) * n, cudaMemcpyHostToDevice, s));
-    SS_CUDA_TRY(cudaMemcpyAsync(c->io_pf, io->point_frame, sizeof(int32_t) * n, cudaMemcpyHostToDevice, s));
-    SS_CUDA_TRY(cudaMemcpyAsync(c->io_pdesc, io->point_desc, (size_t)n * SS_DESC_BYTES, cudaMemcpyHostToDevice, s));
-    if (io->taken)
-      SS_CUDA_TRY(cudaMemcpyAsync(c->io_taken, io->taken, (size_t)n_frames * cap, cudaMemcpyHostToDevice, s));
+    if (!res) {
+      SS_CUDA_TRY(cudaMemcpyAsync(c->io_points, io->points, sizeof(ss_map_point) * n, cudaMemcpyHostToDevice, s));
+      SS_CUDA_TRY(cudaMemcpyAsync(c->io_pf, io->point_frame, sizeof(int32_t) * n, cudaMemcpyHostToDevice, s));
+      SS_CUDA_TRY(cudaMemcpyAsync(c->io_pdesc, io->point_desc, (size_t)n * SS_DESC_BYTES, cudaMemcpyHostToDevice, s));
+      if (io->taken)
+        SS_CUDA_TRY(cudaMemcpyAsync(c->io_taken, io->taken, (size_t)n_frames * cap, cudaMemcpyHostToDevice, s));
+    }
   }
   if (lastf) {
     SS_CUDA_TRY(cudaMemcpyAsync(c->io_lf_off, io->lf_offsets, sizeof(int32_t) * (n_frames + 1), cudaMemcpyHostToDevice, s));
-    if (n_lf > 0) {
+    if (n_lf > 0 && !res) {
       SS_CUDA_TRY(cudaMemcpyAsync(c->io_lf_pts, io->lf_points, sizeof(ss_frame_point) * n_lf, cudaMemcpyHostToDevice, s));
       SS_CUDA_TRY(cudaMemcpyAsync(c->io_lf_desc, io->lf_desc, (size_t)n_lf * SS_DESC_BYTES, cudaMemcpyHostToDevice, s));
     }
-    if (io->mb > 0.0f)
+    if (io->mb > 0.0f && !res)
       SS_CUDA_TRY(cudaMemcpyAsync(c->io_last_cams, io->last_cams, sizeof(ss_camera) * n_frames, cudaMemcpyHostToDevice, s));
   }
   // the hot path
@@ -848,20 +859,20 @@ ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, co
     if (st != SS_OK) return st;
   }
   int64_t n_matches = 0;
-  const uint8_t* win_taken = io->taken ? c->io_taken : nullptr;
+  const uint8_t* win_taken = d_taken;
   if (lastf) {
-    st = ss_match_last_frame(c, n_frames, c->io_cams, io->mb > 0.0f ? c->io_last_cams : nullptr, io->mb, c->io_kps,
-                             c->io_desc, c->io_counts, win_taken, c->io_lf_off, c->io_lf_pts, c->io_lf_desc,
+    st = ss_match_last_frame(c, n_frames, c->io_cams, io->mb > 0.0f ? d_last : nullptr, io->mb, c->io_kps,
+                             c->io_desc, c->io_counts, win_taken, c->io_lf_off, d_lf_pts, d_lf_desc,
                              io->lf_th, 100, 1, io->lf_min_matches, c->io_lf_matches, c->io_lf_n, c->io_lf_mask,
                              stream);
     if (st != SS_OK) return st;
     win_taken = c->io_lf_mask;
   }
   if (window) {
-    st = ss_project_points(c, n_frames, c->io_cams, io->n_points, c->io_points, c->io_pf, io->th, c->io_queries,
-                           stream);
+    st = ss_project_points(c, n_frames, c->io_cams, io->n_points, d_points, d_pf, io->th, c->io_queries, stream);
     if (st != SS_OK) return st;
-    st = ss_match_projection(c, n_frames, c->io_kps, c->io_desc, c->io_counts, win_taken, io->n_points, c->io_queries, c->io_pdesc, 0, cfg, c->io_matches, stream);
+    st = ss_match_projection(c, n_frames, c->io_kps, c->io_desc, c->io_counts, win_taken, io->n_points, c->io_queries,
+                             d_pdesc, 0, cfg, c->io_matches, stream);
     if (st != SS_OK) return st;
     n_matches = io->n_points;
   } else if (cfg->mode == SS_MATCH_BRUTE) {

@@ -117,7 +117,8 @@ def test_track_tick_brute(torch_cuda, ref):
     pipe.close()
 
 
-def test_track_tick_lastframe_window(torch_cuda, ref):
+@pytest.mark.parametrize("resident", [0, 1])
+def test_track_tick_lastframe_window(torch_cuda, ref, resident):
     """Mono tick with frame-to-frame matching (O13) before search local points: the window
     match skips keypoints that are taken or kept by O13.  Oracle chain: extract -> O13 ->
     taken | kept -> O11 -> O9."""
@@ -145,6 +146,10 @@ def test_track_tick_lastframe_window(torch_cuda, ref):
     io.point_desc, io.taken, io.th = hqd.data_ptr(), htk.data_ptr(), 1.0
     io.lf_offsets, io.lf_points, io.lf_desc = hoff.data_ptr(), hlp.data_ptr(), hld.data_ptr()
     io.lf_th, io.lf_min_matches = 15.0, 20
+    if resident:  # the map state lives in HBM (server state): device pointers, not copied
+        dev = [t.cuda() for t in (hp, hpf, hqd, htk, hlp, hld)]
+        io.map_resident = 1
+        io.points, io.point_frame, io.point_desc, io.taken, io.lf_points, io.lf_desc = (t.data_ptr() for t in dev)
     for k in o:
         setattr(io, k, o[k].data_ptr())
     pipe = OrbPipeline(w, h, nf, 8, max_frames=B, max_queries=B * Qm)
