@@ -1,6 +1,7 @@
 """Small runs of every kernel for compute-sanitizer (memcheck / racecheck / synccheck): extract
-(quadtree and grid top-N), window match, projection, stereo, brute force (tensor cores;
-skipped when SANITIZE_BRUTE=0) and one ss_track_tick.
+(quadtree and grid top-N), window match, projection, frame-to-frame matching (cluster kernel,
+with its 2*th retry), stereo, brute force (tensor cores, replicated and map-sharded; skipped
+when SANITIZE_BRUTE=0) and one ss_track_tick.
 
 usage: compute-sanitizer --tool racecheck python scripts/sanitize_extract.py
 """
@@ -49,6 +50,18 @@ def main():
     pipe.project(B, torch.from_numpy(cams.view(np.uint8).reshape(B, -1).copy()).cuda(),
                  torch.from_numpy(pts.view(np.uint8).reshape(512, -1).copy()).cuda(), torch.from_numpy(pf).cuda(), qb)
     pipe.match_window(B, qb, torch.from_numpy(qd).cuda(), out)
+    # frame-to-frame matching (O13): every frame retried (min_matches huge), stereo gates on
+    kk, dd, cc = pipe.results(B)
+    lcams, llast, loff, lp, ld = synth.make_last_frame(kk, dd, cc, 4, np.array([100, 80, 70, 50]), w, h, "euroc", 200,
+                                                       3, stereo_z=1.0)
+    lo = match_out(len(lp), "cuda")
+    ln = torch.zeros(B, dtype=torch.int32, device="cuda")
+    lm = torch.zeros((B, pipe.cap), dtype=torch.uint8, device="cuda")
+    for mm, mb in ((20, 0.0), (10 ** 6, 0.3)):
+        pipe.match_last_frame(B, to_device_records(lcams, "cuda"), torch.from_numpy(loff).cuda(),
+                              to_device_records(lp, "cuda"), torch.from_numpy(ld).cuda(), lo, ln,
+                              last_cams=to_device_records(llast, "cuda"), mb=mb, min_matches=mm, matched=lm)
+    torch.cuda.synchronize()
     # stereo on the (frame 0, frame 1) pair
     d_frames = torch.from_numpy(frames).cuda()
     ur = torch.zeros((1, pipe.cap), dtype=torch.float32, device="cuda")
@@ -65,6 +78,11 @@ def main():
         bp.extract(d_frames)
         bo = torch.zeros((B * bp.cap, 3), dtype=torch.int32, device="cuda")
         bp.match_brute(B, torch.from_numpy(mp).cuda(), bo)
+        parts = torch.zeros((2, B, bp.cap, 2), dtype=torch.int64, device="cuda")  # F4: two shards + merge
+        dm = torch.from_numpy(mp).cuda()
+        for r, (a, b) in enumerate(((0, 130), (130, 300))):
+            ss.ss_match_brute_partial(bp.ctx, B, bp.desc, bp.counts, dm[a:b], b - a, a, parts[r])
+        ss.ss_match_brute_merge(bp.ctx, B, bp.counts, 2, parts, ss.brute_cfg(), bo)
         torch.cuda.synchronize()
         bp.close()
     # one tick from host memory
