@@ -592,14 +592,33 @@ def run_ours(args, cfg):
             pass
 
     # --- e2e through the public API with host buffers (pinned), copies inside the timed region
+    # release the ring's CUDA graphs (hundreds of executable graphs make every later graph launch
+    # slower, e.g. the end-to-end path's per-tick graphs)
+    for row in graphs:
+        for g_ in row:
+            g_.reset()
+    for g_ in graphs_prof:
+        g_.reset()
+    graphs = graphs_prof = None
+    torch.cuda.synchronize(dev)
     if eager_tail:  # ss_track_tick has no cross-rank exchange: no end-to-end number for a sharded map
         e2e = {"value": None, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0,
                "note": "map-sharded brute force over N > 1 ranks needs the NCCL exchange between the partial and "
                        "merge calls; ss_track_tick serves a replicated map only"}
     else:
-        e2e = run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, streams, th=cfg["th"],
-                      stereo=(BF, BASE_M, st_out) if stereo else None, lf=(MB, cfg.get("lf_th", 15.0)),
+        # the end-to-end path keeps more ticks in flight: a tick's frames must cross PCIe before its
+        # kernels start, so with only P contexts part of the GPU idles behind the copies
+        Pe = max(P, args.e2e_inflight)
+        e2e_pipes = [OrbPipeline(w, h, cfg["nf"], L, max_frames=B, max_queries=max(Q, 1), max_map=cfg["map"],
+                                 device=local) for _ in range(Pe)]
+        for pp in e2e_pipes:
+            pp.set_distribution(dist_mode)
+        e2e_streams = [torch.cuda.Stream(dev) for _ in range(Pe)]
+        e2e = run_e2e(args, e2e_pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, e2e_streams,
+                      th=cfg["th"], stereo=(BF, BASE_M, st_out) if stereo else None, lf=(MB, cfg.get("lf_th", 15.0)),
                       dev_map=(points, point_frame, qdesc, taken, lf_pts, lf_desc, lf_last) if window else None)
+        for pp in e2e_pipes:
+            pp.close()
 
     frames_per_step = B * world
     value = frames_per_step * K / (T_max / 1000.0)
@@ -685,7 +704,7 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
     world = int(os.environ.get("WORLD_SIZE", 1))
     d2h = sum(t.numel() * t.element_size() for t in host_out[0].values())
 
-    def measure(resident: bool):
+    def measure(resident: bool, reuse: bool = False):
         """resident: the map state (local-map points, last-frame points, masks) is the server's,
         kept in HBM across ticks (dev_map, slot i); per tick only frames, camera predictions and
         the last-frame offsets come from the host."""
@@ -696,6 +715,7 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
             for i in range(n_host):
                 io = ss.ss_tick_io()
                 io.frames, io.frame_stride, io.pitch = fr[i].data_ptr(), H * W, W
+                io.reuse_graph = int(reuse)
                 if stereo:
                     io.bf, io.baseline = stereo[0], stereo[1]
                 if window:
@@ -729,37 +749,58 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
             i, q = s % n_host, s % P
             ss.ss_track_tick(pipes[q].ctx, B, cfg, ios[q][i], handles[q])
 
-        K = max(1, min(args.steps, 200))
-        for s in range(3):
+        K = 1000  # ~60-100 ms of ticks: long enough that one host hiccup does not move the rate
+        for s in range(3 * n_host if reuse else 3):  # reuse: every (ctx, slot) graph captured before timing
             step(s)
         torch.cuda.synchronize(dev)
         t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         t0.record(streams[0])
         for q in range(1, P):
             streams[q].wait_event(t0)
+        h0 = time.perf_counter()
         for s in range(K):
             step(s)
+        h1 = time.perf_counter()
         for q in range(1, P):
             streams[0].wait_stream(streams[q])
         t1.record(streams[0])
         torch.cuda.synchronize(dev)
         ms = t0.elapsed_time(t1)
         return {"value": B * world * K / (ms / 1000.0), "unit": "frames/s", "h2d_bytes_per_step": int(h2d),
-                "d2h_bytes_per_step": int(d2h), "steps": K, "ms_per_step": ms / K, "ticks_in_flight": P}
+                "d2h_bytes_per_step": int(d2h), "steps": K, "ms_per_step": ms / K, "ticks_in_flight": P,
+                "host_us_per_call": 1e6 * (h1 - h0) / K}
 
     path = ("one C-ABI call per tick: H2D, ss_orb_extract, " + ("ss_stereo_match, " if stereo else "") +
             ("ss_match_last_frame, ss_project_points, ss_match_projection WINDOW" if window
              else "ss_match_projection BRUTE") + ", D2H of all outputs; no graphs")
+    # raw pinned H2D bandwidth of one tick's frames, as seen by this process (diagnostic)
+    _dbuf = torch.empty(fr[0].numel(), dtype=torch.uint8, device=dev)
+    torch.cuda.synchronize(dev)
+    _t0, _t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    _t0.record()
+    for _ in range(50):
+        _dbuf.copy_(fr[0], non_blocking=True)
+    _t1.record()
+    torch.cuda.synchronize(dev)
+    h2d_gbs = fr[0].numel() * 50 / (_t0.elapsed_time(_t1) * 1e-3) / 1e9
+    del _dbuf
+    graph_note = ("; io.reuse_graph = 1: each (ctx, input-ring slot) tick is a cached CUDA graph replayed by "
+                  "ss_track_tick (one launch per tick); direct = the same calls without graph reuse")
     if not window or dev_map is None:
-        r = measure(False)
+        r = measure(False, True)
         r["path"] = "pinned host -> ss_track_tick (" + path + ")" + \
-            ("; the shared map is device-resident server state" if not window else "")
+            ("; the shared map is device-resident server state" if not window else "") + graph_note
+        r["direct"] = measure(False, False)
+        r["h2d_gbs_raw"] = h2d_gbs
         return r
-    r = measure(True)
+    r = measure(True, True)
     r["path"] = ("pinned host frames + camera predictions -> ss_track_tick (" + path + "); the map state (each "
                  "client's local-map points, last-frame points, masks) is server state resident in HBM, "
-                 "as the SLAM-Share server keeps the maps and clients upload only frames (P:L64, P:L68); host_map = the same with it copied too")
-    r["host_map"] = measure(False)
+                 "as the SLAM-Share server keeps the maps and clients upload only frames (P:L64, P:L68); "
+                 "host_map = the same with the map state copied from the host too" + graph_note)
+    r["direct"] = measure(True, False)
+    r["host_map"] = measure(False, True)
+    r["h2d_gbs_raw"] = h2d_gbs
     return r
 
 
@@ -922,6 +963,7 @@ def main(argv=None):
     ap.add_argument("--config", choices=sorted(CONFIGS), default="c2")
     ap.add_argument("--ring", type=int, default=0, help="override the number of input ring slots")
     ap.add_argument("--inflight", type=int, default=4, help="ticks in flight (contexts/streams)")
+    ap.add_argument("--e2e-inflight", type=int, default=8, help="ticks in flight on the end-to-end (host memory) path")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--map-shard", action="store_true",

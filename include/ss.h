@@ -332,6 +332,14 @@ typedef struct {
    * points, point_frame, point_desc, taken, lf_points, lf_desc and last_cams are device
    * pointers and are not copied; frames, cams and lf_offsets stay host inputs. */
   int32_t map_resident;
+  /* 1 = replay from a CUDA graph: the ctx caches (LRU, 16 entries) an instantiated graph of
+   * the tick per distinct argument set (every pointer and size in io, cfg, n_frames and
+   * lf_offsets[n_frames]); the second call with the same arguments captures it, later ones
+   * launch it (one launch instead of ~30 API calls).  Requires every HOST buffer of io to be
+   * page-locked and to stay allocated while the ctx lives (a ring of pinned buffers).  The
+   * buffers' CONTENTS may change freely between calls.  Ignored while profiling events are
+   * installed or when the stream is already capturing. */
+  int32_t reuse_graph;
 } ss_tick_io;
 
 /* One tick of the hot path for a batch of client frames, enqueued on `stream` from a single

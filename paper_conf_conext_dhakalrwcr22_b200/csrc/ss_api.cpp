@@ -169,6 +169,15 @@ struct ss_ctx {
   ss_match* io_lf_matches = nullptr;
   int32_t* io_lf_n = nullptr;
   uint8_t* io_lf_mask = nullptr;
+  // ss_track_tick graph cache (io->reuse_graph): LRU of instantiated tick graphs by argument key
+  struct TickGraph {
+    std::vector<unsigned char> key;
+    cudaGraphExec_t exec;
+    uint64_t last_use;
+  };
+  static constexpr size_t kTickGraphs = 16;
+  std::vector<TickGraph> tick_graphs;
+  uint64_t tick_clock = 0;
   int8_t* brute_qexp = nullptr;  // BRUTE: keypoint descriptors expanded to s8 +-1 (k_brute_tc.cu)
   int8_t* brute_mexp = nullptr;  // BRUTE: map descriptors expanded to s8 +-1
   int n_sm = 148;
@@ -214,6 +223,8 @@ void free_ctx(ss_ctx* c) {
                   c->io_lf_matches, c->io_lf_n, c->io_lf_mask};
   for (void* q : ptrs)
     if (q) cudaFree(q);
+  for (ss_ctx::TickGraph& tg : c->tick_graphs)
+    if (tg.exec) cudaGraphExecDestroy(tg.exec);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   for (cudaEvent_t e : c->ev_level)
     if (e) cudaEventDestroy(e);
@@ -775,37 +786,14 @@ ss_status ss_set_distribution(ss_ctx* c, int32_t mode) {
   return SS_OK;
 }
 
-ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, const ss_tick_io* io,
-                        ss_stream_t stream) {
-  if (!c || !cfg || !io) return fail(SS_EINVAL, "NULL ctx/cfg/io");
-  if (n_frames < 0 || io->n_points < 0 || io->n_map < 0) return fail(SS_EINVAL, "negative size");
-  if (n_frames > c->max_frames) return fail(SS_ECAPACITY, "n_frames exceeds the ctx's max_frames");
-  if (n_frames == 0) return SS_OK;
-  if (!io->frames) return fail(SS_EINVAL, "NULL frames");
+namespace {
+
+// Everything one tick enqueues on s (ss_track_tick after validation): copies in, the hot path,
+// copies out.  Captured into a CUDA graph when io->reuse_graph is set (see ss_track_tick).
+ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, const ss_tick_io* io, cudaStream_t s,
+                       bool stereo, bool window, bool lastf, int64_t n_lf) {
   const Geom& g = c->g;
-  if (io->pitch < g.W || (n_frames > 1 && io->frame_stride < (int64_t)io->pitch * g.H))
-    return fail(SS_EINVAL, "bad pitch / frame stride");
-  const bool stereo = io->bf > 0.0f;
-  if (stereo && (n_frames & 1)) return fail(SS_EINVAL, "stereo needs an even frame count");
-  const bool window = cfg->mode == SS_MATCH_WINDOW && io->n_points > 0;
-  if (window) {
-    if (io->n_points > c->max_queries) return fail(SS_ECAPACITY, "n_points exceeds the ctx's max_queries");
-    if (!io->cams || !io->points || !io->point_frame || !io->point_desc) return fail(SS_EINVAL, "NULL window input");
-  }
-  const bool lastf = window && io->lf_offsets;
-  int64_t n_lf = 0;
-  if (lastf) {
-    for (int f = 0; f < n_frames; f++)
-      if (io->lf_offsets[f + 1] < io->lf_offsets[f]) return fail(SS_EINVAL, "lf_offsets must be non-decreasing");
-    if (io->lf_offsets[0] != 0) return fail(SS_EINVAL, "lf_offsets[0] must be 0");
-    n_lf = io->lf_offsets[n_frames];
-    if (n_lf > c->max_queries) return fail(SS_ECAPACITY, "last-frame points exceed the ctx's max_queries");
-    if (n_lf > 0 && (!io->lf_points || !io->lf_desc)) return fail(SS_EINVAL, "NULL last-frame input");
-    if (io->mb > 0.0f && !io->last_cams) return fail(SS_EINVAL, "mb > 0 needs last_cams");
-    if (!(io->lf_th > 0.0f)) return fail(SS_EINVAL, "lf_th must be > 0");
-  }
-  SS_CUDA_TRY(cudaSetDevice(c->device));
-  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  ss_stream_t stream = reinterpret_cast<ss_stream_t>(s);
   const int cap = g.kp_capacity, L = g.L;
   // host -> device.  Frames stored densely (pitch <= the staging pitch, frame_stride = H *
   // pitch) go in ONE linear copy and keep their pitch; anything else is repacked by 2-D
@@ -899,6 +887,105 @@ ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, co
   if (stereo && io->depth)
     SS_CUDA_TRY(cudaMemcpyAsync(io->depth, c->io_depth, sizeof(float) * (n_frames / 2) * cap, cudaMemcpyDeviceToHost, s));
   return SS_OK;
+}
+
+
+// Graph-cache key of a tick: every argument the enqueued work depends on (host pointers and
+// sizes of io, the match cfg, the last-frame point count read from the host offsets).
+std::vector<unsigned char> tick_key(int32_t n_frames, const ss_match_cfg* cfg, const ss_tick_io* io, int64_t n_lf) {
+  std::vector<unsigned char> k;
+  auto put = [&k](const void* p, size_t n) {
+    const unsigned char* b = static_cast<const unsigned char*>(p);
+    k.insert(k.end(), b, b + n);
+  };
+  auto ptr = [&put](const void* p) { put(&p, sizeof(p)); };
+  put(&n_frames, 4);
+  put(&cfg->mode, 4); put(&cfg->th, 4); put(&cfg->ratio_num, 4); put(&cfg->ratio_den, 4); put(&cfg->dedup, 4);
+  ptr(io->frames); put(&io->frame_stride, 8); put(&io->pitch, 4); put(&io->bf, 4); put(&io->baseline, 4);
+  ptr(io->cams); put(&io->n_points, 4); ptr(io->points); ptr(io->point_frame); ptr(io->point_desc); ptr(io->taken);
+  put(&io->th, 4); ptr(io->d_map_desc); put(&io->n_map, 4);
+  ptr(io->kps); ptr(io->desc); ptr(io->counts); ptr(io->matches); ptr(io->uright); ptr(io->depth);
+  ptr(io->lf_offsets); ptr(io->lf_points); ptr(io->lf_desc); ptr(io->last_cams); put(&io->mb, 4); put(&io->lf_th, 4);
+  put(&io->lf_min_matches, 4); ptr(io->lf_matches); ptr(io->lf_n_matches); put(&io->map_resident, 4);
+  put(&n_lf, 8);
+  return k;
+}
+
+}  // namespace
+
+ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, const ss_tick_io* io,
+                        ss_stream_t stream) {
+  if (!c || !cfg || !io) return fail(SS_EINVAL, "NULL ctx/cfg/io");
+  if (n_frames < 0 || io->n_points < 0 || io->n_map < 0) return fail(SS_EINVAL, "negative size");
+  if (n_frames > c->max_frames) return fail(SS_ECAPACITY, "n_frames exceeds the ctx's max_frames");
+  if (n_frames == 0) return SS_OK;
+  if (!io->frames) return fail(SS_EINVAL, "NULL frames");
+  const Geom& g = c->g;
+  if (io->pitch < g.W || (n_frames > 1 && io->frame_stride < (int64_t)io->pitch * g.H))
+    return fail(SS_EINVAL, "bad pitch / frame stride");
+  const bool stereo = io->bf > 0.0f;
+  if (stereo && (n_frames & 1)) return fail(SS_EINVAL, "stereo needs an even frame count");
+  const bool window = cfg->mode == SS_MATCH_WINDOW && io->n_points > 0;
+  if (window) {
+    if (io->n_points > c->max_queries) return fail(SS_ECAPACITY, "n_points exceeds the ctx's max_queries");
+    if (!io->cams || !io->points || !io->point_frame || !io->point_desc) return fail(SS_EINVAL, "NULL window input");
+  }
+  const bool lastf = window && io->lf_offsets;
+  int64_t n_lf = 0;
+  if (lastf) {
+    for (int f = 0; f < n_frames; f++)
+      if (io->lf_offsets[f + 1] < io->lf_offsets[f]) return fail(SS_EINVAL, "lf_offsets must be non-decreasing");
+    if (io->lf_offsets[0] != 0) return fail(SS_EINVAL, "lf_offsets[0] must be 0");
+    n_lf = io->lf_offsets[n_frames];
+    if (n_lf > c->max_queries) return fail(SS_ECAPACITY, "last-frame points exceed the ctx's max_queries");
+    if (n_lf > 0 && (!io->lf_points || !io->lf_desc)) return fail(SS_EINVAL, "NULL last-frame input");
+    if (io->mb > 0.0f && !io->last_cams) return fail(SS_EINVAL, "mb > 0 needs last_cams");
+    if (!(io->lf_th > 0.0f)) return fail(SS_EINVAL, "lf_th must be > 0");
+  }
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  SS_CUDA_TRY(cudaStreamIsCapturing(s, &cs));
+  // (the legacy default stream cannot be captured: such ticks always run directly)
+  if (!io->reuse_graph || !c->prof.empty() || cs != cudaStreamCaptureStatusNone || s == nullptr ||
+      s == cudaStreamLegacy)
+    return tick_enqueue(c, n_frames, cfg, io, s, stereo, window, lastf, n_lf);
+  // graph reuse: a tick seen before with identical arguments is replayed from a CUDA graph
+  // (one launch instead of ~30 API calls); the second occurrence of a key is captured (the
+  // first runs directly, so lazily-set kernel attributes are never set under capture)
+  std::vector<unsigned char> key = tick_key(n_frames, cfg, io, n_lf);
+  c->tick_clock++;
+  for (ss_ctx::TickGraph& tg : c->tick_graphs) {
+    if (tg.key != key) continue;
+    tg.last_use = c->tick_clock;
+    if (tg.exec) {
+      SS_CUDA_TRY(cudaGraphLaunch(tg.exec, s));
+      return SS_OK;
+    }
+    cudaGraph_t graph = nullptr;
+    SS_CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+    ss_status st = tick_enqueue(c, n_frames, cfg, io, s, stereo, window, lastf, n_lf);
+    cudaError_t e = cudaStreamEndCapture(s, &graph);
+    if (st != SS_OK) {
+      if (graph) cudaGraphDestroy(graph);
+      return st;
+    }
+    SS_CUDA_TRY(e);
+    e = cudaGraphInstantiate(&tg.exec, graph, 0);
+    cudaGraphDestroy(graph);
+    SS_CUDA_TRY(e);
+    SS_CUDA_TRY(cudaGraphLaunch(tg.exec, s));
+    return SS_OK;
+  }
+  if (c->tick_graphs.size() >= ss_ctx::kTickGraphs) {  // evict the least recently used
+    size_t lru = 0;
+    for (size_t i = 1; i < c->tick_graphs.size(); i++)
+      if (c->tick_graphs[i].last_use < c->tick_graphs[lru].last_use) lru = i;
+    if (c->tick_graphs[lru].exec) cudaGraphExecDestroy(c->tick_graphs[lru].exec);
+    c->tick_graphs.erase(c->tick_graphs.begin() + lru);
+  }
+  c->tick_graphs.push_back({key, nullptr, c->tick_clock});
+  return tick_enqueue(c, n_frames, cfg, io, s, stereo, window, lastf, n_lf);
 }
 
 ss_status ss_profile_events(ss_ctx* c, void* const* events, int32_t n_events) {

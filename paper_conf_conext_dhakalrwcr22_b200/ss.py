@@ -64,7 +64,8 @@ class ss_tick_io(C.Structure):
                 ("uright", C.c_void_p), ("depth", C.c_void_p),
                 ("lf_offsets", C.c_void_p), ("lf_points", C.c_void_p), ("lf_desc", C.c_void_p),
                 ("last_cams", C.c_void_p), ("mb", C.c_float), ("lf_th", C.c_float), ("lf_min_matches", C.c_int32),
-                ("lf_matches", C.c_void_p), ("lf_n_matches", C.c_void_p), ("map_resident", C.c_int32)]
+                ("lf_matches", C.c_void_p), ("lf_n_matches", C.c_void_p), ("map_resident", C.c_int32),
+                ("reuse_graph", C.c_int32)]
 
 
 # numpy views of the 20-/20-/12-byte records of ss.h

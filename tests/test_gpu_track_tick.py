@@ -176,3 +176,49 @@ def test_track_tick_lastframe_window(torch_cuda, ref, resident):
     np.testing.assert_array_equal(got, want)
     assert (got["idx"] >= 0).sum() > 100
     pipe.close()
+
+
+def test_track_tick_graph_reuse(torch_cuda, ref):
+    """io.reuse_graph = 1: the same io (pinned buffers) replayed from the ctx's cached CUDA graph
+    follows changes of the buffers' CONTENTS (new frames, new local maps) exactly like direct
+    calls -- checked against the oracle on every call."""
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import OrbPipeline
+    w, h = synth.SHAPES["euroc"]
+    B, Q, nf = 2, 800, 1000
+    p = ref.params(w, h, nf)
+    cap = p.kp_capacity
+    hf = torch.zeros(B * h * w, dtype=torch.uint8).pin_memory()
+    hc = torch.zeros(B * 96, dtype=torch.uint8).pin_memory()
+    hp = torch.zeros(B * Q * 32, dtype=torch.uint8).pin_memory()
+    hpf = torch.zeros(B * Q * 4, dtype=torch.uint8).pin_memory()
+    hqd = torch.zeros(B * Q * 32, dtype=torch.uint8).pin_memory()
+    o = {k: torch.zeros(n, dtype=torch.uint8).pin_memory()
+         for k, n in (("kps", B * cap * 20), ("desc", B * cap * 32), ("counts", B * 9 * 4), ("matches", B * Q * 12))}
+    io = ss.ss_tick_io()
+    io.frames, io.frame_stride, io.pitch, io.reuse_graph = hf.data_ptr(), h * w, w, 1
+    io.cams, io.n_points, io.points, io.point_frame = hc.data_ptr(), B * Q, hp.data_ptr(), hpf.data_ptr()
+    io.point_desc, io.th = hqd.data_ptr(), 1.0
+    for k in o:
+        setattr(io, k, o[k].data_ptr())
+    pipe = OrbPipeline(w, h, nf, 8, max_frames=B, max_queries=B * Q)
+    st = torch.cuda.Stream()  # a capturable stream (the legacy NULL stream always runs directly)
+    for it in range(4):  # call 0 direct, call 1 captures, calls 2, 3 replay
+        frames = synth.make_frames(w, h, B, cfg=50 + it)
+        rk, rd, rc = ref.orb_extract_batch(p, frames)
+        cm, pt, pf, qd, _ = synth.make_local_map(rk, rd, rc, 8, p.scale_factor, np.array(p.n_per_level[:8]), w, h,
+                                                 "euroc", Q, seed=60 + it)
+        for dst, a in ((hf, frames), (hc, cm), (hp, pt), (hpf, pf), (hqd, qd)):
+            dst.copy_(torch.from_numpy(np.ascontiguousarray(a).view(np.uint8).reshape(-1)))
+        ss.ss_track_tick(pipe.ctx, B, ss.window_cfg(), io, st)
+        torch.cuda.synchronize()
+        counts = o["counts"].numpy().view(np.int32).reshape(B, 9)
+        np.testing.assert_array_equal(counts, rc)
+        desc = o["desc"].numpy().reshape(B, cap, 32)
+        for f in range(B):
+            np.testing.assert_array_equal(desc[f, :rc[f, -1]], rd[f, :rc[f, -1]])
+        q = ref.project_points(p, cm, pt, pf, 1.0)
+        want = ref.match_window(p, rk, rd, rc, None, q, qd)
+        np.testing.assert_array_equal(o["matches"].numpy().view(ref.MATCH_DTYPE).reshape(-1), want)
+    pipe.close()
