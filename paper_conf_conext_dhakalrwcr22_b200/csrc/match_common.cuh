@@ -11,9 +11,7 @@ __device__ __forceinline__ int hamming256(const uint4 a0, const uint4 a1, const 
 }
 
 __host__ __device__ __forceinline__ int row_off(const Geom& g, int l) {  // start of level l in a frame's row index
-  int o = 0;
-  for (int i = 0; i < l; i++) o += g.h[i] + 1;
-  return o;
+  return l < g.L ? g.row_off[l] : g.row_off[g.L - 1] + g.h[g.L - 1] + 1;
 }
 
 // Row-index entries owned by slot k of one frame (keypoints in canonical (level, ly, lx)
@@ -38,12 +36,14 @@ __device__ __forceinline__ void rowidx_fill(const Geom& g, const ss_keypoint* __
 }
 
 // Rows [rlo, rhi) of level l (clamped to [0, h_l]) that can hold |y - v| < r, widened by one
-// row each side for f32 rounding; the exact test on each keypoint decides.
+// row each side; the exact test on each keypoint decides, so the bounds only need to be a
+// superset: (v -+ r) * f32(1/scale) is within 1e-3 rows of the real quotient (rows < 2048),
+// far inside the one-row margin that also covers y = f32(ly * scale) rounding.
 __device__ __forceinline__ void window_rows(const Geom& g, int l, float v, float r, int* rlo, int* rhi) {
-  const float s_l = g.scale[l];
+  const float is_l = g.inv_scale[l];
   const int hl = g.h[l];
-  *rlo = max(0, min(hl, (int)floorf(__fdiv_rn(__fsub_rn(v, r), s_l)) - 1));
-  *rhi = max(0, min(hl, (int)ceilf(__fdiv_rn(__fadd_rn(v, r), s_l)) + 2));
+  *rlo = max(0, min(hl, (int)floorf(__fsub_rn(v, r) * is_l) - 1));
+  *rhi = max(0, min(hl, (int)ceilf(__fadd_rn(v, r) * is_l) + 2));
 }
 
 // top-2 of two packed (distance << 32 | index) pairs

@@ -287,6 +287,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     g.h[l] = q.level_h[l];
     g.scale[l] = q.scale[l];
     g.inv_scale[l] = q.inv_scale[l];
+    g.row_off[l] = l == 0 ? 0 : g.row_off[l - 1] + g.h[l - 1] + 1;
     g.pitch[l] = (g.w[l] + 15) & ~15;
     g.lvl_off[l] = 0;
     if (l >= 1) {

@@ -47,6 +47,7 @@ struct Geom {
   int64_t pyr_frame_bytes;
   float scale[kMaxLevels];
   float inv_scale[kMaxLevels];      // f32(1 / scale[l]) (O0)
+  int32_t row_off[kMaxLevels];      // start of level l in a frame's keypoint row index (sum of h + 1)
   int32_t cell_first[kMaxLevels];   // first active cell of level l in the cell table
   int32_t ncells[kMaxLevels];       // active cells of level l (row-major, skipped cells removed)
   int32_t total_cells;              // per frame
