@@ -9,7 +9,7 @@
 // retry), which are cluster barriers here instead of kernel boundaries:
 //   P0  every CTA stages the frame's keypoint positions and builds its row index (first
 //       keypoint per (level, row)) in shared memory; claims reset;             | cluster.sync
-//   P1  eight lanes per point: pose transform + pinhole projection + bounds (single-rounded
+//   P1  four lanes per point: pose transform + pinhole projection + bounds (single-rounded
 //       f32 ops in the oracle's order), octave-scaled window, level gate, exact |x-u| < r,
 //       |y-v| < r, 8 x POPC Hamming over the candidate runs of the row index, shuffle merge
 //       of packed (d << 32 | k) top-2; accepted -> atomicMin claim (pass tag | d | point);
@@ -33,7 +33,7 @@ namespace {
 
 constexpr int kCluster = 8;    // CTAs per frame (portable cluster size)
 constexpr int kThreads = 512;   // per CTA (16 warps)
-constexpr int kLanes = 8;      // lanes per point in P1
+constexpr int kLanes = 4;      // lanes per point in P1
 constexpr int kHisto = 30;     // ORB-SLAM HISTO_LENGTH
 constexpr size_t kLfSmemMax = 200 * 1024;
 
@@ -123,7 +123,7 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
   const uint4* fd = reinterpret_cast<const uint4*>(a.desc + (int64_t)f * cap * SS_DESC_BYTES);
   const uint8_t* ft = a.taken ? a.taken + (int64_t)f * cap : nullptr;
   const int sub = threadIdx.x % kLanes;
-  const unsigned gmask = 0xFFu << ((threadIdx.x & 31) & ~(kLanes - 1));
+  const unsigned gmask = ((1u << kLanes) - 1u) << ((threadIdx.x & 31) & ~(kLanes - 1));
   int kept = 0;
 
   for (int pass = 0; pass < 2; pass++) {

@@ -1,11 +1,11 @@
 // k_match.cu -- S9 windowed matcher ("search local points") and S10
 // brute-force matcher (DESIGN.md §3 O9, O10).
 //
-// WINDOW: eight lanes per map-point query.  Keypoints are in canonical (level, ly, lx)
+// WINDOW: 1-8 lanes per map-point query (fewer when there are many queries).  Keypoints are in canonical (level, ly, lx)
 // order, so on each level of the gate [l-1, l] the rows with |y - v| < r (f32) form one
 // contiguous run found by two binary searches on the exact predicate; the run is scanned
 // with the exact |x - u| < r test, the taken mask, and a 256-bit Hamming distance
-// (8 x POPC over 2 x 16-byte loads); the eight lanes split the run and merge their packed
+// (8 x POPC over 2 x 16-byte loads); the lanes split the run and merge their packed
 // (distance << 32 | index) top-2 by shuffles, i.e. top-2 by (distance, index); ORB-SLAM's
 // accept rule; a keypoint claimed by several accepted
 // queries keeps the min (distance, query) (atomicMin on packed u64, then a resolve pass).
@@ -17,7 +17,6 @@ namespace ss {
 
 namespace {
 
-constexpr int WG = 8;  // lanes cooperating on one query
 
 // Per frame and level: rowidx[r] = index of the first keypoint with ly >= r (r in [0, h_l]),
 // from the canonical (level, ly, lx) order; plus the dedup claim table reset.
@@ -35,6 +34,7 @@ __global__ void __launch_bounds__(256) match_prepare(Geom g, int F, const ss_key
   rowidx_fill(g, kps + (int64_t)f * cap, counts + f * (L + 1), rowidx + (int64_t)f * rows_per_frame, k);
 }
 
+template <int WG>  // lanes cooperating on one query
 __global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const ss_keypoint* __restrict__ kps,
                                                            const uint8_t* __restrict__ desc,
                                                            const int32_t* __restrict__ counts,
@@ -48,7 +48,7 @@ __global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const 
   pdl_trigger();
   const int gt = blockIdx.x * blockDim.x + threadIdx.x;
   const int qi = gt / WG, sub = gt % WG;
-  const unsigned gmask = 0xFFu << ((threadIdx.x & 31) & ~(WG - 1));
+  const unsigned gmask = ((1u << WG) - 1u) << ((threadIdx.x & 31) & ~(WG - 1));
   if (qi >= nq) return;  // whole groups exit together (WG divides 32)
   const ss_mp_query Q = q[qi];
   const int L = g.L, cap = g.kp_capacity;
@@ -252,10 +252,18 @@ cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* 
                                 const uint8_t* qdesc, ss_match_cfg cfg, unsigned long long* claim, ss_match* out,
                                 const uint16_t* rowidx, cudaStream_t s) {
   if (n_queries <= 0) return cudaSuccess;
-  const int64_t threads = (int64_t)n_queries * WG;
-  cudaError_t e = launch_pdl(match_window_kernel, dim3((unsigned)((threads + 255) / 256)), dim3(256), 0, s, g, n_frames,
-                             kps, desc, counts, taken, n_queries, q, qdesc, cfg, claim, out, rowidx,
-                             match_rows_per_frame(g));
+  // lanes per query: enough groups to fill ~2 waves of the GPU (148 SMs x 2048 threads); a
+  // query's window holds a handful of candidates, so with many queries fewer lanes per query
+  // (less redundant per-query work) win: c3 (800 k queries) 1-2 lanes, c2 (20 k) 8
+  // (measured c3: 8 lanes 130 us, 4: 97, 2: 83, 1: 64)
+  int wg = 8;
+  const int64_t want = 2LL * 148 * 2048;
+  while (wg > 1 && (int64_t)n_queries * (wg / 2) >= want) wg /= 2;
+  auto kern = wg == 1 ? match_window_kernel<1> : wg == 2 ? match_window_kernel<2> : wg == 4 ? match_window_kernel<4>
+                                                                                            : match_window_kernel<8>;
+  const int64_t threads = (int64_t)n_queries * wg;
+  cudaError_t e = launch_pdl(kern, dim3((unsigned)((threads + 255) / 256)), dim3(256), 0, s, g, n_frames, kps, desc,
+                             counts, taken, n_queries, q, qdesc, cfg, claim, out, rowidx, match_rows_per_frame(g));
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 
