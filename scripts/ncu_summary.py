@@ -18,7 +18,10 @@ METRICS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.
 SHORT = {"fast_bands_kernel": "fast", "distribute_kernel": "distribute", "pyramid_fused_kernel": "pyramid",
          "describe_kernel": "describe", "match_prepare": "match_prepare", "match_window_kernel": "match_window",
          "match_window_resolve": "match_resolve", "brute_tc_kernel": "brute_tc", "brute_expand_kernel": "brute_expand",
-         "match_brute_merge": "brute_merge"}
+         "match_brute_merge": "brute_merge", "lastframe_kernel": "lastframe", "project_kernel": "project",
+         "brute_shard_top2": "brute_shard_top2", "brute_parts_merge": "brute_parts_merge",
+         "stereo_match_kernel": "stereo", "stereo_outlier_kernel": "stereo_outliers",
+         "distribute_grid_kernel": "distribute_grid"}
 
 
 def main():
