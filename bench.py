@@ -421,6 +421,7 @@ def run_ours(args, cfg):
     st_out = [(torch.zeros((max(npairs, 1), cap), dtype=torch.float32, device=dev),
                torch.zeros((max(npairs, 1), cap), dtype=torch.float32, device=dev)) for _ in range(P)]
     streams = [stream] + [torch.cuda.Stream(dev) for _ in range(P - 1)]
+    aux_streams = [torch.cuda.Stream(dev) for _ in range(P)]
     for q in range(1, P):  # first call outside capture (kernel attributes)
         with torch.cuda.stream(streams[q]):
             pipes[q].extract(frames[0], stream=streams[q])
@@ -431,7 +432,18 @@ def run_ours(args, cfg):
         pp, st, ot = pipes[q], streams[q], outs[q]
         if prof:
             ss.ss_profile_events(pp.ctx, events[s])
+        # the local-map projection (cameras + map points only) could run on a forked branch
+        # concurrently with the extraction; measured on c2 with 4 ticks in flight that cost 7 %
+        # of throughput (63.0k -> 58.9k frames/s), so the ring graphs keep it serial (the
+        # per-tick executor ss_track_tick forks it: +1-2 % there)
+        fork = False
         with torch.cuda.graph(g, stream=st):
+            if fork:
+                ev0, ev1 = torch.cuda.Event(), torch.cuda.Event()
+                ev0.record(st)
+                aux_streams[q].wait_event(ev0)
+                pp.project(B, cams[s], points[s], point_frame[s], qbufs[q], th=cfg["th"], stream=aux_streams[q])
+                ev1.record(aux_streams[q])
             pp.extract(frames[s], stream=st)
             if stereo:
                 pp.stereo(frames[s], BF, BASE_M, st_out[q][0], st_out[q][1], stream=st)
@@ -439,7 +451,10 @@ def run_ours(args, cfg):
                 pp.match_last_frame(B, cams[s], lf_off[s], lf_pts[s], lf_desc[s], lf_out[q], lf_n[q],
                                     last_cams=lf_last[s] if MB > 0 else None, mb=MB, th=cfg["lf_th"],
                                     min_matches=20, taken=taken[s], matched=lf_mask[q], stream=st)
-                pp.project(B, cams[s], points[s], point_frame[s], qbufs[q], th=cfg["th"], stream=st)
+                if fork:
+                    st.wait_event(ev1)
+                else:
+                    pp.project(B, cams[s], points[s], point_frame[s], qbufs[q], th=cfg["th"], stream=st)
                 pp.match_window(B, qbufs[q], qdesc[s], ot, taken=lf_mask[q], stream=st)
             elif shard:
                 if not eager_tail:

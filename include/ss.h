@@ -265,7 +265,9 @@ typedef struct {
  * with an octave outside [0, L-1] get {-1, 256, 256}.  Bit-exact with the oracle.
  * SS_EINVAL for negative sizes, NULL buffers, th <= 0; SS_ECAPACITY if n_frames > max_frames.
  * Uses the ctx's matcher scratch (row index, claims): not concurrently with another match
- * call on the same ctx. */
+ * call on the same ctx.  It also prepares the WINDOW matcher's row index and claims for these
+ * keypoints, so a following ss_match_projection WINDOW on the same d_kps / d_counts (no
+ * ss_orb_extract or ss_stereo_match in between) skips its match_prepare kernel. */
 ss_status ss_match_last_frame(ss_ctx* ctx, int32_t n_frames, const ss_camera* d_cams, const ss_camera* d_last_cams,
                               float mb, const ss_keypoint* d_kps, const uint8_t* d_desc, const int32_t* d_counts,
                               const uint8_t* d_kp_taken, const int32_t* d_point_offsets,
@@ -366,7 +368,8 @@ ss_status ss_track_tick(ss_ctx* ctx, int32_t n_frames, const ss_match_cfg* cfg, 
  * distribute(levels >= 1), describe -- 13 events (while events are installed the level-0
  * branch runs in line on `stream` instead of on its side stream, so each kernel is timed
  * alone).  WINDOW match: a pair per kernel
- * (match_prepare, match_window[, match_resolve if dedup]); BRUTE: brute_expand, brute_tc,
+ * (match_prepare, match_window[, match_resolve if dedup]; the match_prepare pair encloses
+ * no work when ss_match_last_frame already prepared the index); BRUTE: brute_expand, brute_tc,
  * brute_merge; ss_project_points: project; ss_stereo_match: stereo_prepare, stereo, stereo_outliers;
  * ss_match_last_frame: lastframe; ss_match_brute_partial: brute_expand, brute_tc, brute_shard_top2;
  * ss_match_brute_merge: brute_parts_merge.

@@ -8,7 +8,9 @@
 // rotation histogram's three maxima, and the "fewer than min_matches -> redo with 2*th"
 // retry), which are cluster barriers here instead of kernel boundaries:
 //   P0  every CTA stages the frame's keypoint positions and builds its row index (first
-//       keypoint per (level, row)) in shared memory; claims reset;             | cluster.sync
+//       keypoint per (level, row)) in shared memory; claims reset; the cluster also writes
+//       the window matcher's global row index and resets its claims (match_prepare's work,
+//       so the following search-local-points match skips that launch); | cluster.sync
 //   P1  four lanes per point: pose transform + pinhole projection + bounds (single-rounded
 //       f32 ops in the oracle's order), octave-scaled window, level gate, exact |x-u| < r,
 //       |y-v| < r, 8 x POPC Hamming over the candidate runs of the row index, shuffle merge
@@ -69,8 +71,9 @@ struct LfArgs {
   ss_match* out;
   int32_t* n_matches;
   uint8_t* matched;
-  unsigned long long* claim;
-  uint16_t* rowidx;
+  unsigned long long* claim;       // this matcher's dedup claims [F][cap]
+  uint16_t* rowidx;                // if set: the window matcher's global row index, built here too
+  unsigned long long* win_claim;   // ... and its dedup claims, reset here (match_prepare's work)
   int rows_per_frame;
 };
 
@@ -109,6 +112,10 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
   for (int k = ct; k < cap; k += nct) {
     fclaim[k] = ~0ull;
     if (fmask) fmask[k] = (a.taken && a.taken[(int64_t)f * cap + k]) ? 1 : 0;
+    if (a.rowidx) {  // the following search-local-points match reuses this index (no match_prepare)
+      rowidx_fill(g, fk, cnt, a.rowidx + (int64_t)f * a.rows_per_frame, k);
+      a.win_claim[(int64_t)f * cap + k] = ~0ull;
+    }
   }
   cluster.sync();
 
@@ -265,11 +272,12 @@ cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams,
                              const ss_keypoint* kps, const uint8_t* desc, const int32_t* counts, const uint8_t* taken,
                              const int32_t* pt_off, const ss_frame_point* pts, const uint8_t* pdesc, float th,
                              int th_high, int check_orientation, int min_matches, ss_match* out, int32_t* n_matches,
-                             uint8_t* matched, unsigned long long* claim, uint16_t* rowidx, cudaStream_t s) {
+                             uint8_t* matched, unsigned long long* claim, uint16_t* rowidx,
+                             unsigned long long* win_claim, cudaStream_t s) {
   if (n_frames <= 0) return cudaSuccess;
   LfArgs a{g,     n_frames, cams,    last_cams,         mb,          kps, desc, counts,
            taken, pt_off,   pts,     pdesc,             th,          th_high, check_orientation,
-           min_matches, out, n_matches, matched, claim, rowidx, match_rows_per_frame(g)};
+           min_matches, out, n_matches, matched, claim, rowidx, win_claim, match_rows_per_frame(g)};
   const size_t smem = lastframe_smem_bytes(g);
   if (smem > kLfSmemMax) return cudaErrorInvalidValue;
   cudaError_t e = launch_pdl(lastframe_kernel, dim3(n_frames * kCluster), dim3(kThreads), smem, s, a);

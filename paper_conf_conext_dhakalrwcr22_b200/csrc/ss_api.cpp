@@ -142,7 +142,14 @@ struct ss_ctx {
   int32_t* ovf_counter = nullptr;  // [0] overflowed levels, [1] capacity violations
   int8_t* pattern = nullptr;
   unsigned long long* claim = nullptr;
+  unsigned long long* claim_lf = nullptr;  // O13's own dedup claims
   uint16_t* rowidx = nullptr;  // WINDOW matcher: first keypoint per (frame, level, row)
+  // rowidx + claim already prepared (by ss_match_last_frame) for these keypoints: the next
+  // WINDOW match skips match_prepare.  Cleared by every ss_orb_extract.
+  bool win_ready = false;
+  const ss_keypoint* win_kps = nullptr;
+  const int32_t* win_counts = nullptr;
+  int win_nf = 0;
   uint64_t* phase_ts = nullptr;  // distribution phase timestamps [max_frames][L][16] (debug hook)
   unsigned long long* partial = nullptr;
   int dist_mode = SS_DIST_QUADTREE;  // ss_set_distribution
@@ -186,6 +193,9 @@ struct ss_ctx {
   static constexpr int kSide = 4, kSideLevel = 3;
   cudaStream_t side[kSide] = {};
   cudaEvent_t ev_fork = nullptr, ev_level[kMaxLevels] = {}, ev_join[kSide] = {};
+  // ss_track_tick: the local-map projection runs on its own branch, concurrently with extraction
+  cudaStream_t aux = nullptr;
+  cudaEvent_t ev_aux0 = nullptr, ev_aux1 = nullptr;
   // profiling hook
   std::vector<cudaEvent_t> prof;
   size_t prof_next = 0;
@@ -216,7 +226,7 @@ void free_ctx(ss_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->device);
   void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr_plan, c->pyr_gtab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
-                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->partial, c->rowidx, c->phase_ts,
+                  c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->claim_lf, c->partial, c->rowidx, c->phase_ts,
                   c->brute_qexp, c->brute_mexp, c->stereo_sad, c->io_frames, c->io_kps, c->io_desc, c->io_counts,
                   c->io_cams, c->io_points, c->io_pf, c->io_pdesc, c->io_taken, c->io_queries, c->io_matches,
                   c->io_uright, c->io_depth, c->io_lf_off, c->io_lf_pts, c->io_lf_desc, c->io_last_cams,
@@ -226,6 +236,9 @@ void free_ctx(ss_ctx* c) {
   for (ss_ctx::TickGraph& tg : c->tick_graphs)
     if (tg.exec) cudaGraphExecDestroy(tg.exec);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_aux0) cudaEventDestroy(c->ev_aux0);
+  if (c->ev_aux1) cudaEventDestroy(c->ev_aux1);
+  if (c->aux) cudaStreamDestroy(c->aux);
   for (cudaEvent_t e : c->ev_level)
     if (e) cudaEventDestroy(e);
   for (cudaEvent_t e : c->ev_join)
@@ -475,6 +488,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->ovf_counter, sizeof(int32_t) * 2);
   ALLOC(c->pattern, 1024);
   ALLOC(c->claim, sizeof(unsigned long long) * F * g.kp_capacity);
+  ALLOC(c->claim_lf, sizeof(unsigned long long) * F * g.kp_capacity);
   ALLOC(c->rowidx, sizeof(uint16_t) * F * match_rows_per_frame(g));
   ALLOC(c->phase_ts, sizeof(uint64_t) * F * L * 16);
   ALLOC(c->stereo_sad, sizeof(int32_t) * ((F + 1) / 2) * g.kp_capacity);
@@ -526,6 +540,9 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   for (int l = 0; l < kMaxLevels && e == cudaSuccess; l++)
     e = cudaEventCreateWithFlags(&c->ev_level[l], cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_aux0, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_aux1, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaMemset(c->sel_counts, 0, sizeof(int32_t) * F * L);
   if (e != cudaSuccess) {
     std::string m = std::string("ss_create: ") + cudaGetErrorString(e);
@@ -551,6 +568,7 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   if (!d_frames || !d_kps || !d_desc || !d_counts) return fail(SS_EINVAL, "NULL buffer");
   if (pitch < c->g.W) return fail(SS_EINVAL, "pitch < width");
   if (n_frames > 1 && frame_stride < (int64_t)pitch * c->g.H) return fail(SS_EINVAL, "frame_stride < height*pitch");
+  c->win_ready = false;  // new keypoints: any prepared window index is stale
   SS_CUDA_TRY(cudaSetDevice(c->device));
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   SS_CUDA_TRY(check_stream(s));
@@ -626,7 +644,9 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
     if (n_queries > 0 && (!d_queries || !d_map_desc)) return fail(SS_EINVAL, "NULL queries");
     if (n_queries == 0) return SS_OK;
     prof_mark(c, s);
-    SS_CUDA_TRY(launch_match_prepare(c->g, n_frames, d_kps, d_counts, c->rowidx, c->claim, cfg->dedup, s));
+    if (!(c->win_ready && d_kps == c->win_kps && d_counts == c->win_counts && n_frames <= c->win_nf))
+      SS_CUDA_TRY(launch_match_prepare(c->g, n_frames, d_kps, d_counts, c->rowidx, c->claim, cfg->dedup, s));
+    c->win_ready = false;  // the claims are consumed by this match
     prof_mark(c, s);
     prof_mark(c, s);
     SS_CUDA_TRY(launch_match_window(c->g, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_queries, d_queries,
@@ -724,6 +744,7 @@ ss_status ss_stereo_match(ss_ctx* c, int32_t n_pairs, const uint8_t* d_frames, i
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   SS_CUDA_TRY(check_stream(s));
   const float maxD = bf / baseline;  // ORB-SLAM: maxD = mbf / minZ, minZ = mb
+  c->win_ready = false;               // its prepare rewrites the shared row index
   FrameSrc src{d_frames, frame_stride, pitch, c->pyr};
   prof_mark(c, s);
   SS_CUDA_TRY(launch_match_prepare(c->g, 2 * n_pairs, d_kps, d_counts, c->rowidx, c->claim, 0, s));
@@ -775,8 +796,12 @@ ss_status ss_match_last_frame(ss_ctx* c, int32_t n_frames, const ss_camera* d_ca
   prof_mark(c, s);
   SS_CUDA_TRY(launch_lastframe(c->g, n_frames, d_cams, mb > 0.0f ? d_last_cams : nullptr, mb, d_kps, d_desc, d_counts,
                                d_kp_taken, d_point_offsets, d_points, d_point_desc, th, th_high, check_orientation,
-                               min_matches, d_out, d_n_matches, d_kp_matched, c->claim, c->rowidx, s));
+                               min_matches, d_out, d_n_matches, d_kp_matched, c->claim_lf, c->rowidx, c->claim, s));
   prof_mark(c, s);
+  c->win_ready = true;
+  c->win_kps = d_kps;
+  c->win_counts = d_counts;
+  c->win_nf = n_frames;
   return SS_OK;
 }
 
@@ -839,8 +864,20 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
     if (io->mb > 0.0f && !res)
       SS_CUDA_TRY(cudaMemcpyAsync(c->io_last_cams, io->last_cams, sizeof(ss_camera) * n_frames, cudaMemcpyHostToDevice, s));
   }
-  // the hot path
-  ss_status st = ss_orb_extract(c, n_frames, c->io_frames, fstride, P, c->io_kps, c->io_desc, c->io_counts, stream);
+  // the hot path.  The local-map projection needs only the cameras and map points, so (unless
+  // profiling events are installed, which time every kernel alone on `stream`) it forks onto
+  // the ctx's aux stream and overlaps the extraction; the WINDOW match joins it.
+  ss_status st;
+  const bool fork_project = window && c->prof.empty();
+  if (fork_project) {
+    SS_CUDA_TRY(cudaEventRecord(c->ev_aux0, s));
+    SS_CUDA_TRY(cudaStreamWaitEvent(c->aux, c->ev_aux0, 0));
+    st = ss_project_points(c, n_frames, c->io_cams, io->n_points, d_points, d_pf, io->th, c->io_queries,
+                           reinterpret_cast<ss_stream_t>(c->aux));
+    if (st != SS_OK) return st;
+    SS_CUDA_TRY(cudaEventRecord(c->ev_aux1, c->aux));
+  }
+  st = ss_orb_extract(c, n_frames, c->io_frames, fstride, P, c->io_kps, c->io_desc, c->io_counts, stream);
   if (st != SS_OK) return st;
   if (stereo) {
     st = ss_stereo_match(c, n_frames / 2, c->io_frames, fstride, P, c->io_kps, c->io_desc, c->io_counts, io->bf,
@@ -858,8 +895,12 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
     win_taken = c->io_lf_mask;
   }
   if (window) {
-    st = ss_project_points(c, n_frames, c->io_cams, io->n_points, d_points, d_pf, io->th, c->io_queries, stream);
-    if (st != SS_OK) return st;
+    if (fork_project) {
+      SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_aux1, 0));
+    } else {
+      st = ss_project_points(c, n_frames, c->io_cams, io->n_points, d_points, d_pf, io->th, c->io_queries, stream);
+      if (st != SS_OK) return st;
+    }
     st = ss_match_projection(c, n_frames, c->io_kps, c->io_desc, c->io_counts, win_taken, io->n_points, c->io_queries,
                              d_pdesc, 0, cfg, c->io_matches, stream);
     if (st != SS_OK) return st;

@@ -208,7 +208,8 @@ cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams,
                              const ss_keypoint* kps, const uint8_t* desc, const int32_t* counts, const uint8_t* taken,
                              const int32_t* pt_off, const ss_frame_point* pts, const uint8_t* pdesc, float th,
                              int th_high, int check_orientation, int min_matches, ss_match* out, int32_t* n_matches,
-                             uint8_t* matched, unsigned long long* claim, uint16_t* rowidx, cudaStream_t s);
+                             uint8_t* matched, unsigned long long* claim, uint16_t* rowidx,
+                             unsigned long long* win_claim, cudaStream_t s);
 
 // Overflow scratch bytes the distribution needs for a level with `slots` candidate slots.
 int64_t distribute_ovf_bytes(int64_t slots);
