@@ -132,8 +132,9 @@ ss_status ss_orb_params_init(int32_t width, int32_t height, int32_t n_features, 
  * max_frames bounds n_frames per call, max_queries the WINDOW query count and max_map the
  * BRUTE map size (0 = that mode unused).  Allocates all scratch here (none per call).
  * SS_EUNSUPPORTED when this build's kernels cannot serve p: scale_factor above 4/3 (the
- * pyramid kernel's source window), kp_capacity above 65535, or a FAST band / pyramid block
- * that does not fit in shared memory. */
+ * pyramid kernel's source window), kp_capacity above 65535, a FAST band / pyramid block
+ * that does not fit in shared memory, or max_map >= 2^23 (larger maps: shard them, see
+ * ss_match_brute_partial). */
 ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, int32_t max_queries,
                     int32_t max_map, ss_ctx** out);
 ss_status ss_destroy(ss_ctx* ctx);

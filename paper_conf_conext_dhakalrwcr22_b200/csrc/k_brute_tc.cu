@@ -99,24 +99,25 @@ __device__ __forceinline__ void tc_commit(uint32_t bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
 }
 
-#define TC_LD32(addr, r)                                                                                          \
+// 32 accumulator columns of this warp's 32 lanes, the low 16 bits of adjacent columns (2i,
+// 2i+1) packed into register i (tcgen05.ld .pack::16b): half the TMEM-to-register traffic
+#define TC_LD16P(addr, r)                                                                                         \
   asm volatile(                                                                                                   \
-      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18," \
-      "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"                                              \
+      "tcgen05.ld.sync.aligned.32x32b.x16.pack::16b.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15},"  \
+      " [%16];"                                                                                                   \
       : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),           \
-        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),     \
-        "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),   \
-        "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])    \
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])      \
       : "r"(addr))
+// wait for this thread's outstanding tcgen05.ld, then pin the 16 registers after the wait (an
+// empty asm that "rewrites" them, so no use of them can be scheduled above the wait)
+#define TC_WAIT16(r)                                                                                               \
+  do {                                                                                                             \
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");                                                \
+    asm volatile("" : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]), "+r"(r[6]),         \
+                 "+r"(r[7]), "+r"(r[8]), "+r"(r[9]), "+r"(r[10]), "+r"(r[11]), "+r"(r[12]), "+r"(r[13]),          \
+                 "+r"(r[14]), "+r"(r[15]));                                                                        \
+  } while (0)
 
-__device__ __forceinline__ void top2_insert(unsigned long long k, unsigned long long& b1, unsigned long long& b2) {
-  if (k < b1) {
-    b2 = b1;
-    b1 = k;
-  } else if (k < b2) {
-    b2 = k;
-  }
-}
 
 // Expand packed descriptors (32 B per row) into s8 {+1 (bit 0), -1 (bit 1)} in the canonical
 // layout above.  Output byte 16*i.. of a segment is chunk c = (i >> 3) & 15 (descriptor bits
@@ -143,7 +144,9 @@ __global__ void __launch_bounds__(256) brute_expand_kernel(const uint8_t* __rest
       for (int j = 0; j < 4; j++) {
         const uint32_t nib = (v >> (4 * j)) & 0xFu;
         const uint32_t t = (nib * 0x00204081u) & 0x01010101u;  // bit i of nib -> bit 8i
-        w[j] = t * 0xFEu + 0x01010101u;                          // byte 0 -> 0x01 (+1), 1 -> 0xFF (-1)
+        // keypoints: bit 0 -> +1 (0x01), 1 -> -1 (0xFF); map rows: bit 0 -> -64 (0xC0), 1 -> +64
+        // (0x40), so the accumulator is -64 * (256 - 2 * Hamming), a 16-bit value
+        w[j] = isq ? t * 0xFEu + 0x01010101u : 0xC0C0C0C0u ^ (t << 7);
       }
       o = make_uint4(w[0], w[1], w[2], w[3]);
     }
@@ -151,25 +154,30 @@ __global__ void __launch_bounds__(256) brute_expand_kernel(const uint8_t* __rest
   }
 }
 
-// Packed 16-bit key of one column: 128 * distance + column-within-half (distance <= 256,
-// column < 64 => key <= 32831; 0xFFFF = "none").  From the s32 dot: 128*d + j =
-// 16384 + j - 64*dot.  Two columns (j, j + 64) share one register (low / high halves);
-// the low half never borrows from the high one (16384 + j - 64*dot >= 0).
+// Packed keys of 32 columns (j0 + 2i, j0 + 2i + 1 in the low / high half of v[i]): the
+// accumulator half is -64 * dot = 64 * (2d - 256) (16-bit two's complement), so
+// 16384 + j + acc = 128 * d + j (<= 32895) comes from ONE lane-wise add (VIADD.16x2).
+// Two registers at a time, the running sorted (b1, b2) of {b1, b2, ka, kb} (distinct keys) in
+// five VIMNMX: m, M = min / max(ka, kb); b1' = min3(b1, ka, kb); b2' = min3(b2, max(b1, m), M).
 template <bool kMasked>
-__device__ __forceinline__ void top2_columns(const uint32_t* lo, const uint32_t* hi, int j0, int valid, uint32_t& b1,
-                                             uint32_t& b2) {
+__device__ __forceinline__ void top2_packed(const uint32_t* v, int j0, int valid, uint32_t& b1, uint32_t& b2) {
+  uint32_t k[16];
 #pragma unroll
-  for (int i = 0; i < 32; i++) {
-    const int j = j0 + i;
-    const uint32_t c = (uint32_t)(16384 + j) * 0x10001u;
-    uint32_t k = c - (lo[i] << 6) - (hi[i] << 22);
+  for (int i = 0; i < 16; i++) {
+    const int j = j0 + 2 * i;
+    const uint32_t c = (uint32_t)(16384 + j) | ((uint32_t)(16384 + j + 1) << 16);
+    k[i] = __vadd2(c, v[i]);
     if (kMasked) {
-      if (j >= valid) k |= 0xFFFFu;
-      if (j + 64 >= valid) k |= 0xFFFF0000u;
+      if (j >= valid) k[i] |= 0xFFFFu;
+      if (j + 1 >= valid) k[i] |= 0xFFFF0000u;
     }
-    const uint32_t t = __vmaxu2(b1, k);
-    b1 = __vminu2(b1, k);
-    b2 = __vminu2(b2, t);
+  }
+#pragma unroll
+  for (int i = 0; i < 16; i += 2) {
+    const uint32_t m = __vminu2(k[i], k[i + 1]), M = __vmaxu2(k[i], k[i + 1]);
+    const uint32_t x = __vmaxu2(b1, m);
+    b1 = __vimin3_u16x2(b1, k[i], k[i + 1]);
+    b2 = __vimin3_u16x2(b2, x, M);
   }
 }
 
@@ -260,7 +268,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1) brute_tc_kernel(const int8_t* _
   } else if (warp >= 4) {
     const int acc = (warp - 4) >> 2, quarter = warp & 3;
     const int row = acc * TC_M + quarter * 32 + lane;
-    unsigned long long g1 = ~0ull, g2 = ~0ull;
+    // running top-2 as 32-bit keys (distance << 23 | map index): map indices < 2^23 (ss_create)
+    uint32_t g1 = 0xFFFFFFFFu, g2 = 0xFFFFFFFFu;
     for (int t = 0; t < nt; t++) {
       const int b = t & 1;
       const uint32_t bph = (uint32_t)(t >> 1) & 1u;
@@ -270,34 +279,47 @@ __global__ void __launch_bounds__(TC_THREADS, 1) brute_tc_kernel(const int8_t* _
       const int base = (t0 + t) * TC_N;
       const int valid = min(TC_N, n_map - base);
       uint32_t b1 = 0xFFFFFFFFu, b2 = 0xFFFFFFFFu;
-#pragma unroll
-      for (int h = 0; h < 2; h++) {
-        uint32_t lo[32], hi[32];
-        TC_LD32(taddr + 32 * h, lo);
-        TC_LD32(taddr + 64 + 32 * h, hi);
-        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-        if (valid == TC_N)
-          top2_columns<false>(lo, hi, 32 * h, valid, b1, b2);
-        else
-          top2_columns<true>(lo, hi, 32 * h, valid, b1, b2);
+      {
+        // four 32-column chunks, software-pipelined: chunk c + 1 is read out of TMEM while the
+        // ALU reduces chunk c (TMEM reads and the top-2 otherwise serialise per tile); the
+        // buffer is released to the MMA warp as soon as its last chunk has landed
+        uint32_t va[16], vb[16];
+        TC_LD16P(taddr, va);
+        TC_WAIT16(va);
+        TC_LD16P(taddr + 32, vb);
+        if (valid == TC_N) top2_packed<false>(va, 0, valid, b1, b2); else top2_packed<true>(va, 0, valid, b1, b2);
+        TC_WAIT16(vb);
+        TC_LD16P(taddr + 64, va);
+        if (valid == TC_N) top2_packed<false>(vb, 32, valid, b1, b2); else top2_packed<true>(vb, 32, valid, b1, b2);
+        TC_WAIT16(va);
+        TC_LD16P(taddr + 96, vb);
+        if (valid == TC_N) top2_packed<false>(va, 64, valid, b1, b2); else top2_packed<true>(va, 64, valid, b1, b2);
+        TC_WAIT16(vb);
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(tempty(b));
+        if (valid == TC_N) top2_packed<false>(vb, 96, valid, b1, b2); else top2_packed<true>(vb, 96, valid, b1, b2);
       }
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(tempty(b));
-      // per-half top-2 -> the running 64-bit top-2 (distance << 32 | map index)
+      // per-lane-half top-2 (16-bit 128 d + j) -> the running 32-bit top-2, branch-free
+      // (keys of different columns are distinct; "none" maps to 0xFFFFFFFF)
+      auto to32 = [base](uint32_t k) {
+        return k == 0xFFFFu ? 0xFFFFFFFFu : (((k & 0xFF80u) << 16) | (k & 127u)) + (uint32_t)base;
+      };
+      const uint32_t c[4] = {to32(b1 & 0xFFFFu), to32(b2 & 0xFFFFu), to32(b1 >> 16), to32(b2 >> 16)};
 #pragma unroll
-      for (int half = 0; half < 2; half++) {
-        const uint32_t k1 = (b1 >> (16 * half)) & 0xFFFFu, k2 = (b2 >> (16 * half)) & 0xFFFFu;
-        if (k1 != 0xFFFFu)
-          top2_insert(((unsigned long long)(k1 >> 7) << 32) | (unsigned)(base + 64 * half + (k1 & 127)), g1, g2);
-        if (k2 != 0xFFFFu)
-          top2_insert(((unsigned long long)(k2 >> 7) << 32) | (unsigned)(base + 64 * half + (k2 & 127)), g1, g2);
+      for (int i = 0; i < 4; i++) {
+        const uint32_t t = max(g1, c[i]);
+        g1 = min(g1, c[i]);
+        g2 = min(g2, t);
       }
     }
     const int gq = pair * TC_ROWS + row;
-    if (gq < n_slots) {
-      partial[((int64_t)gq * splits + split) * 2] = g1;
-      partial[((int64_t)gq * splits + split) * 2 + 1] = g2;
+    if (gq < n_slots) {  // back to the (distance << 32 | map index) partial layout of the merge
+      auto to64 = [](uint32_t g) {
+        return g == 0xFFFFFFFFu ? ~0ull : ((unsigned long long)(g >> 23) << 32) | (g & 0x7FFFFFu);
+      };
+      partial[((int64_t)gq * splits + split) * 2] = to64(g1);
+      partial[((int64_t)gq * splits + split) * 2 + 1] = to64(g2);
     }
   }
   tc_fence_before();

@@ -270,6 +270,8 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (!p || !out) return fail(SS_EINVAL, "NULL argument");
   *out = nullptr;
   if (max_frames < 1 || max_queries < 0 || max_map < 0) return fail(SS_EINVAL, "bad capacities");
+  if (max_map >= (1 << 23))  // the brute kernel's running top-2 packs (distance << 23 | map row)
+    return fail(SS_EUNSUPPORTED, "max_map must be below 2^23 (8388608) map descriptors per ctx / shard");
   ss_orb_params q;
   ss_status st = params_init(p->width, p->height, p->n_features, p->n_levels, p->scale_factor, p->ini_th_fast,
                              p->min_th_fast, &q);
