@@ -32,14 +32,15 @@ namespace ss {
 
 namespace {
 
-constexpr int TC_M = 128;                    // keypoint rows per accumulator (TMEM lanes)
-constexpr int TC_N = 128;                    // map rows per tile (TMEM columns per accumulator)
+constexpr int TC_M = 128;                    // keypoint rows per CTA (TMEM lanes)
+constexpr int TC_N = 128;                    // map rows per CTA per tile; columns per epilogue warp
+constexpr int TC_NT = 256;                   // map rows per tile = MMA N (cta_group::2 pair)
 constexpr int TC_K = 256;                    // descriptor bits
-constexpr int TC_ROWS = 2 * TC_M;            // keypoint rows per CTA (two accumulators)
+constexpr int TC_ROWS = 2 * TC_M;            // keypoint rows per CTA pair (MMA M = 256)
 constexpr int BLK_BYTES = TC_M * TC_K;       // one expanded 128-row block: 32 KB
 constexpr int STAGES = 4;
 constexpr int TC_THREADS = 384;
-constexpr int SMEM_A = 2 * BLK_BYTES;
+constexpr int SMEM_A = BLK_BYTES;
 constexpr int SMEM_B = STAGES * BLK_BYTES;
 constexpr int SMEM_BAR = 256;
 constexpr int TC_SMEM = SMEM_A + SMEM_B + SMEM_BAR;
@@ -47,8 +48,8 @@ constexpr uint32_t TMEM_COLS = 512;
 
 // instruction descriptor: D s32 (bits 4-5 = 2), A/B signed 8-bit (bits 7-9, 10-12 = 1),
 // both K-major, N >> 3 at bits 17-22, M >> 4 at bits 24-28
-constexpr uint32_t IDESC = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(TC_N >> 3) << 17) |
-                           ((uint32_t)(TC_M >> 4) << 24);
+constexpr uint32_t IDESC = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(TC_NT >> 3) << 17) |
+                           ((uint32_t)(TC_ROWS >> 4) << 24);  // M = 256, N = 256 (cta_group::2)
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -87,16 +88,45 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t
 }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
-__device__ __forceinline__ void tc_mma_i8(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accumulate) {
+__device__ __forceinline__ void tc_mma2_i8(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accumulate) {
   asm volatile(
       "{\n\t.reg .pred p;\n\t"
       "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n}" ::"r"(tmem_d),
+      "tcgen05.mma.cta_group::2.kind::i8 [%0], %1, %2, %3, p;\n}" ::"r"(tmem_d),
       "l"(adesc), "l"(bdesc), "r"(IDESC), "r"(accumulate)
       : "memory");
 }
-__device__ __forceinline__ void tc_commit(uint32_t bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+// completion of the leader's MMAs, signalled on the barrier at this offset in BOTH CTAs
+__device__ __forceinline__ void tc_commit2_mc(uint32_t bar) {
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(bar),
+      "h"((uint16_t)3)
+      : "memory");
+}
+__device__ __forceinline__ uint32_t mapa_shared(uint32_t addr, uint32_t cta) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(cta));
+  return r;
+}
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+// arrival without a memory fence: the epilogue only reports that its TMEM reads are done
+// (ordered by tcgen05.fence::before_thread_sync), no data it wrote needs publishing
+__device__ __forceinline__ void mbar_arrive_remote_relaxed(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_cluster(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n"
+      "WAITC_%=:\n\t"
+      "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@!P1 bra WAITC_%=;\n}" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void cluster_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
 // 32 accumulator columns of this warp's 32 lanes, the low 16 bits of adjacent columns (2i,
@@ -181,108 +211,120 @@ __device__ __forceinline__ void top2_packed(const uint32_t* v, int j0, int valid
   }
 }
 
-// grid: (pairs = ceil(n_slots / 256), splits).  Split s covers map tiles
-// [s*T/S, (s+1)*T/S) of T = ceil(n_map / 128); CTAs of one split run side by side, so its
-// map tiles are read from L2 by every pair.
-__global__ void __launch_bounds__(TC_THREADS, 1) brute_tc_kernel(const int8_t* __restrict__ qexp,
-                                                                  const int8_t* __restrict__ mexp, int n_slots,
-                                                                  int n_map, int n_tiles, int splits,
-                                                                  unsigned long long* __restrict__ partial) {
+// grid: (2 * pairs, splits), clusters of 2 CTAs = one SM pair per (256-keypoint pair-block,
+// map split).  CTA rank r holds keypoint rows [256 pair + 128 r, +128) in its shared memory
+// and, per map tile of 256 rows, the 128 rows [256 t + 128 r, +128): the leader (rank 0) issues
+// tcgen05.mma.cta_group::2 M=256 N=256 K=32, which reads A and B halves from both SMs and
+// writes each CTA's 128 x 256 s32 block into its own TMEM (two buffers of 256 columns).  Each
+// SM thus reads 8 KB of operands per 128-cycle MMA (half the shared-memory traffic per MAC of
+// the 1-SM M=128 N=128 form).  Split s covers tiles [s*T/S, (s+1)*T/S) of T = ceil(n_map/256).
+// Cross-CTA protocol: the peer's relay thread (warp 1) forwards the completion of its own
+// operand copies to the leader's full / afull barriers; the leader's commits multicast to both
+// CTAs' empty / tfull barriers; the peer's epilogue warps arrive remotely on the leader's tempty.
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(TC_THREADS, 1)
+    brute_tc_kernel(const int8_t* __restrict__ qexp, const int8_t* __restrict__ mexp, int n_slots, int n_map,
+                    int n_tiles, int splits, unsigned long long* __restrict__ partial) {
   extern __shared__ __align__(1024) uint8_t smem[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int pair = blockIdx.x, split = blockIdx.y;
+  uint32_t rank;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+  const int pair = blockIdx.x >> 1, split = blockIdx.y;
   const int t0 = (int)((int64_t)split * n_tiles / splits), t1 = (int)((int64_t)(split + 1) * n_tiles / splits);
   const int nt = t1 - t0;
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SMEM_A + SMEM_B);
   const uint32_t sa = smem_u32(smem), sb = sa + SMEM_A;
   const uint32_t bar0 = smem_u32(bars);
-  // barrier k at bar0 + 8k: full[0..3], empty[4..7], tfull[8..9], tempty[10..11], a_full[12]
+  // barrier k at bar0 + 8k: full[0..S), empty[S..2S), tfull[2S, 2S+1], tempty[2S+2, 2S+3], afull
   auto full = [&](int s) { return bar0 + 8u * s; };
   auto empty = [&](int s) { return bar0 + 8u * (STAGES + s); };
   auto tfull = [&](int b) { return bar0 + 8u * (2 * STAGES + b); };
   auto tempty = [&](int b) { return bar0 + 8u * (2 * STAGES + 2 + b); };
   const uint32_t afull = bar0 + 8u * (2 * STAGES + 4);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 5);
+  const bool leader = rank == 0;
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < STAGES; s++) {
-      mbar_init(full(s), 1);
+      mbar_init(full(s), leader ? 2 : 1);  // leader: own copy + the peer's relayed copy
       mbar_init(empty(s), 1);
     }
     for (int b = 0; b < 2; b++) {
       mbar_init(tfull(b), 1);
-      mbar_init(tempty(b), 8);  // one arrive per epilogue warp
+      mbar_init(tempty(b), 16);  // leader's: 8 local + 8 peer epilogue warps
     }
-    mbar_init(afull, 1);
+    mbar_init(afull, leader ? 2 : 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 2) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
                  "r"(TMEM_COLS)
                  : "memory");
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
   }
   tc_fence_before();
-  __syncthreads();
+  cluster_sync();  // barriers of both CTAs initialised, TMEM of both allocated
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
   pdl_wait();  // the expanded operands come from the previous kernel
 
   if (warp == 0) {
-    if (lane == 0) {
-      mbar_expect_tx(afull, SMEM_A);
-      const int8_t* a = qexp + (int64_t)pair * SMEM_A;
-      bulk_g2s(sa, a, BLK_BYTES, afull);
-      bulk_g2s(sa + BLK_BYTES, a + BLK_BYTES, BLK_BYTES, afull);
+    if (lane == 0) {  // producer (both CTAs): own A block once, own half of every map tile
+      mbar_expect_tx(afull, BLK_BYTES);
+      bulk_g2s(sa, qexp + ((int64_t)pair * 2 + rank) * BLK_BYTES, BLK_BYTES, afull);
       for (int t = 0; t < nt; t++) {
         const int s = t % STAGES;
         const uint32_t ph = (uint32_t)(t / STAGES) & 1u;
         mbar_wait(empty(s), ph ^ 1u);
         mbar_expect_tx(full(s), BLK_BYTES);
-        bulk_g2s(sb + s * BLK_BYTES, mexp + (int64_t)(t0 + t) * BLK_BYTES, BLK_BYTES, full(s));
+        bulk_g2s(sb + s * BLK_BYTES, mexp + ((int64_t)(t0 + t) * 2 + rank) * BLK_BYTES, BLK_BYTES, full(s));
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
-      mbar_wait(afull, 0);
+    if (lane == 0 && leader) {  // MMA issuer
+      mbar_wait_cluster(afull, 0);
       tc_fence_after();
       for (int t = 0; t < nt; t++) {
         const int s = t % STAGES;
         const uint32_t ph = (uint32_t)(t / STAGES) & 1u;
         const int b = t & 1;
         const uint32_t bph = (uint32_t)(t >> 1) & 1u;
-        mbar_wait(tempty(b), bph ^ 1u);
-        mbar_wait(full(s), ph);
+        mbar_wait_cluster(tempty(b), bph ^ 1u);
+        mbar_wait_cluster(full(s), ph);
         tc_fence_after();
+        const uint32_t d = tmem + (uint32_t)(b * TC_NT);
 #pragma unroll
-        for (int acc = 0; acc < 2; acc++) {
-          const uint32_t d = tmem + (uint32_t)(b * 2 * TC_N + acc * TC_N);
-#pragma unroll
-          for (int k = 0; k < TC_K / 32; k++)
-            tc_mma_i8(d, umma_desc(sa + acc * BLK_BYTES + k * 256), umma_desc(sb + s * BLK_BYTES + k * 256), k > 0);
-        }
-        tc_commit(empty(s));
-        tc_commit(tfull(b));
+        for (int k = 0; k < TC_K / 32; k++)
+          tc_mma2_i8(d, umma_desc(sa + k * 256), umma_desc(sb + s * BLK_BYTES + k * 256), k > 0);
+        tc_commit2_mc(empty(s));
+        tc_commit2_mc(tfull(b));
+      }
+    } else if (lane == 0) {  // peer relay: own copies landed -> the leader's barriers
+      mbar_wait(afull, 0);
+      mbar_arrive_remote(mapa_shared(afull, 0));
+      for (int t = 0; t < nt; t++) {
+        const int s = t % STAGES;
+        mbar_wait(full(s), (uint32_t)(t / STAGES) & 1u);
+        mbar_arrive_remote(mapa_shared(full(s), 0));
       }
     }
   } else if (warp >= 4) {
-    const int acc = (warp - 4) >> 2, quarter = warp & 3;
-    const int row = acc * TC_M + quarter * 32 + lane;
+    const int hc = (warp - 4) >> 2, quarter = warp & 3;  // column half, TMEM lane quarter
+    const int row = quarter * 32 + lane;
     // running top-2 as 32-bit keys (distance << 23 | map index): map indices < 2^23 (ss_create)
     uint32_t g1 = 0xFFFFFFFFu, g2 = 0xFFFFFFFFu;
+    const uint32_t tempty_leader0 = mapa_shared(tempty(0), 0), tempty_leader1 = mapa_shared(tempty(1), 0);
     for (int t = 0; t < nt; t++) {
       const int b = t & 1;
       const uint32_t bph = (uint32_t)(t >> 1) & 1u;
       mbar_wait(tfull(b), bph);
       tc_fence_after();
-      const uint32_t taddr = tmem + ((uint32_t)(quarter * 32) << 16) + (uint32_t)(b * 2 * TC_N + acc * TC_N);
-      const int base = (t0 + t) * TC_N;
+      const uint32_t taddr = tmem + ((uint32_t)(quarter * 32) << 16) + (uint32_t)(b * TC_NT + hc * TC_N);
+      const int base = (t0 + t) * TC_NT + hc * TC_N;
       const int valid = min(TC_N, n_map - base);
       uint32_t b1 = 0xFFFFFFFFu, b2 = 0xFFFFFFFFu;
       {
         // four 32-column chunks, software-pipelined: chunk c + 1 is read out of TMEM while the
-        // ALU reduces chunk c (TMEM reads and the top-2 otherwise serialise per tile); the
-        // buffer is released to the MMA warp as soon as its last chunk has landed
+        // ALU reduces chunk c; the buffer is released as soon as its last chunk has landed
         uint32_t va[16], vb[16];
         TC_LD16P(taddr, va);
         TC_WAIT16(va);
@@ -297,7 +339,12 @@ __global__ void __launch_bounds__(TC_THREADS, 1) brute_tc_kernel(const int8_t* _
         TC_WAIT16(vb);
         tc_fence_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(tempty(b));
+        if (lane == 0) {
+          if (leader)
+            mbar_arrive(tempty(b));
+          else
+            mbar_arrive_remote_relaxed(b ? tempty_leader1 : tempty_leader0);
+        }
         if (valid == TC_N) top2_packed<false>(vb, 96, valid, b1, b2); else top2_packed<true>(vb, 96, valid, b1, b2);
       }
       // per-lane-half top-2 (16-bit 128 d + j) -> the running 32-bit top-2, branch-free
@@ -308,44 +355,46 @@ __global__ void __launch_bounds__(TC_THREADS, 1) brute_tc_kernel(const int8_t* _
       const uint32_t c[4] = {to32(b1 & 0xFFFFu), to32(b2 & 0xFFFFu), to32(b1 >> 16), to32(b2 >> 16)};
 #pragma unroll
       for (int i = 0; i < 4; i++) {
-        const uint32_t t = max(g1, c[i]);
+        const uint32_t tt = max(g1, c[i]);
         g1 = min(g1, c[i]);
-        g2 = min(g2, t);
+        g2 = min(g2, tt);
       }
     }
-    const int gq = pair * TC_ROWS + row;
-    if (gq < n_slots) {  // back to the (distance << 32 | map index) partial layout of the merge
+    const int gq = pair * TC_ROWS + (int)rank * TC_M + row;
+    if (gq < n_slots) {  // one partial per (split, column half): the merges see 2 * splits parts
       auto to64 = [](uint32_t g) {
         return g == 0xFFFFFFFFu ? ~0ull : ((unsigned long long)(g >> 23) << 32) | (g & 0x7FFFFFu);
       };
-      partial[((int64_t)gq * splits + split) * 2] = to64(g1);
-      partial[((int64_t)gq * splits + split) * 2 + 1] = to64(g2);
+      unsigned long long* o = partial + ((int64_t)gq * 2 * splits + 2 * split + hc) * 2;
+      o[0] = to64(g1);
+      o[1] = to64(g2);
     }
   }
   tc_fence_before();
   __syncthreads();
+  cluster_sync();  // the peer's last MMA and remote arrivals are done before either CTA leaves
   pdl_trigger();
   if (warp == 2) {
     tc_fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS) : "memory");
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS) : "memory");
   }
 }
 
 }  // namespace
 
-int64_t brute_tc_query_bytes(int64_t n_slots) { return (n_slots + TC_ROWS - 1) / TC_ROWS * (int64_t)SMEM_A; }
-int64_t brute_tc_map_bytes(int64_t n_map) { return (n_map + TC_N - 1) / TC_N * (int64_t)BLK_BYTES; }
+int64_t brute_tc_query_bytes(int64_t n_slots) { return (n_slots + TC_ROWS - 1) / TC_ROWS * 2LL * BLK_BYTES; }
+int64_t brute_tc_map_bytes(int64_t n_map) { return (n_map + TC_NT - 1) / TC_NT * 2LL * BLK_BYTES; }
 
 int brute_tc_splits(int n_slots, int n_map, int max_splits, int n_sm) {
   const int pairs = (n_slots + TC_ROWS - 1) / TC_ROWS;
-  const int tiles = (n_map + TC_N - 1) / TC_N;
+  const int tiles = (n_map + TC_NT - 1) / TC_NT;
   if (pairs <= 0 || tiles <= 0) return 1;
-  // fill whole waves of one CTA per SM; the first wave count whose fill is >= 90 % wins
+  // fill whole waves of one CTA per SM (two per pair-block); the first >= 90 % fill wins
   int best = 1;
   double best_eff = -1.0;
   for (int w = 1; w <= 8; w++) {
-    const int s = std::max(1, std::min(std::min(w * n_sm / pairs, tiles), max_splits));
-    const int ctas = pairs * s;
+    const int s = std::max(1, std::min(std::min(w * n_sm / (2 * pairs), tiles), max_splits));
+    const int ctas = 2 * pairs * s;
     const double eff = (double)ctas / ((double)n_sm * ((ctas + n_sm - 1) / n_sm));
     if (eff > best_eff + 1e-9) {
       best_eff = eff;
@@ -360,8 +409,8 @@ cudaError_t launch_brute_expand(int n_slots, const uint8_t* desc, int n_map, con
                                 int8_t* mexp, cudaStream_t s) {
   if (n_slots <= 0 || n_map <= 0) return cudaSuccess;
   const int pairs = (n_slots + TC_ROWS - 1) / TC_ROWS;
-  const int tiles = (n_map + TC_N - 1) / TC_N;
-  const int64_t q_units = (int64_t)pairs * TC_ROWS * 16, m_units = (int64_t)tiles * TC_N * 16;
+  const int tiles = (n_map + TC_NT - 1) / TC_NT;
+  const int64_t q_units = (int64_t)pairs * TC_ROWS * 16, m_units = (int64_t)tiles * TC_NT * 16;
   const int64_t units = q_units + m_units;
   const int blocks = (int)std::min<int64_t>((units + 255) / 256, 148 * 16);
   cudaError_t e = launch_pdl(brute_expand_kernel, dim3(blocks), dim3(256), 0, s, desc, n_slots, q_units, qexp,
@@ -373,10 +422,10 @@ cudaError_t launch_brute_tc(int n_slots, int n_map, const int8_t* qexp, const in
                             unsigned long long* partial, cudaStream_t s) {
   if (n_slots <= 0 || n_map <= 0) return cudaSuccess;
   const int pairs = (n_slots + TC_ROWS - 1) / TC_ROWS;
-  const int tiles = (n_map + TC_N - 1) / TC_N;
+  const int tiles = (n_map + TC_NT - 1) / TC_NT;
   cudaError_t e = cudaFuncSetAttribute(brute_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM);
   if (e != cudaSuccess) return e;
-  e = launch_pdl(brute_tc_kernel, dim3(pairs, splits), dim3(TC_THREADS), TC_SMEM, s, qexp, mexp, n_slots, n_map,
+  e = launch_pdl(brute_tc_kernel, dim3(2 * pairs, splits), dim3(TC_THREADS), TC_SMEM, s, qexp, mexp, n_slots, n_map,
                  tiles, splits, partial);
   return e != cudaSuccess ? e : cudaGetLastError();
 }

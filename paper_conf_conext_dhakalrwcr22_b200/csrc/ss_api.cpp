@@ -519,7 +519,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     ALLOC(c->io_lf_mask, (size_t)F * g.kp_capacity);
   }
   if (max_map > 0) {
-    ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 2);
+    ALLOC(c->partial, sizeof(unsigned long long) * F * g.kp_capacity * c->max_splits * 4);  // [slot][2 splits][2]
     ALLOC(c->brute_qexp, brute_tc_query_bytes(F * g.kp_capacity));
     ALLOC(c->brute_mexp, brute_tc_map_bytes(max_map));
   }
@@ -675,7 +675,8 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
     SS_CUDA_TRY(launch_brute_tc(n_slots, n_map, c->brute_qexp, c->brute_mexp, splits, c->partial, s));
     prof_mark(c, s);
     prof_mark(c, s);
-    SS_CUDA_TRY(launch_brute_merge(c->g, n_frames, d_counts, splits, c->partial, *cfg, d_out, s));
+    // brute_tc writes one partial top-2 per (split, column half of the pair's 256-row tiles)
+    SS_CUDA_TRY(launch_brute_merge(c->g, n_frames, d_counts, 2 * splits, c->partial, *cfg, d_out, s));
     prof_mark(c, s);
     return SS_OK;
   }
@@ -709,7 +710,7 @@ ss_status ss_match_brute_partial(ss_ctx* c, int32_t n_frames, const uint8_t* d_d
   SS_CUDA_TRY(launch_brute_tc(n_slots, n_map, c->brute_qexp, c->brute_mexp, splits, c->partial, s));
   prof_mark(c, s);
   prof_mark(c, s);
-  SS_CUDA_TRY(launch_brute_shard_top2(c->g, n_frames, d_counts, splits, c->partial, map_offset, top2, s));
+  SS_CUDA_TRY(launch_brute_shard_top2(c->g, n_frames, d_counts, 2 * splits, c->partial, map_offset, top2, s));
   prof_mark(c, s);
   return SS_OK;
 }
