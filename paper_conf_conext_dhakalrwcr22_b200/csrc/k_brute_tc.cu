@@ -255,6 +255,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(TC_THREADS, 1)
     mbar_init(afull, leader ? 2 : 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  // the pair's cta_group::2 allocation is collective: warp 2 of BOTH CTAs issues it (the
+  // leader alone hangs); both receive the same column base in their own slot
   if (warp == 2) {
     asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
                  "r"(TMEM_COLS)
