@@ -60,23 +60,25 @@ __device__ __forceinline__ int rhe_rot(int a, int b, float ca, float cb, int ma,
   return rhe_exact((long long)a * ma + (long long)b * mb, r2, k);
 }
 
-__global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, FrameSrc src,
+__global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, FrameSrc src,
                                                                    const uint32_t* __restrict__ selected,
                                                                    const int32_t* __restrict__ sel_counts,
                                                                    const int8_t* __restrict__ pattern,
                                                                    ss_keypoint* __restrict__ kps,
                                                                    uint8_t* __restrict__ desc,
                                                                    int32_t* __restrict__ counts) {
-  pdl_wait();
   pdl_trigger();
   extern __shared__ __align__(16) uint8_t sm[];  // DESC_WARPS * PER_WARP
-  __shared__ int8_t pat[1024];
   __shared__ int off[kMaxLevels + 1];
   __shared__ __align__(16) uint32_t s_wmask[16 * 8], s_wu[16 * 8];  // per |v|: 32 byte weights
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int f = blockIdx.y;
   const int L = g.L;
-  for (int i = threadIdx.x; i < 1024; i += blockDim.x) pat[i] = pattern[i];
+  // Constant inputs (set at ss_create) are read before the dependency wait, overlapping the
+  // predecessor kernel's tail.  Lane = output byte: its 8 pairs are the 32 pattern bytes
+  // 32 * lane .. 32 * lane + 31, one word (px0, py0, px1, py1) per bit, held in registers.
+  const uint4 pa = __ldg(reinterpret_cast<const uint4*>(pattern) + 2 * lane);
+  const uint4 pb = __ldg(reinterpret_cast<const uint4*>(pattern) + 2 * lane + 1);
   if (threadIdx.x < 256) {  // byte j = u + 15 of row |v|: inside the disk -> (1, u + 15), else 0
     const int t = threadIdx.x >> 7, av = (threadIdx.x >> 3) & 15, k = threadIdx.x & 7;
     uint32_t word = 0;
@@ -86,13 +88,16 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
     }
     (t ? s_wu : s_wmask)[(threadIdx.x & 127)] = word;
   }
-  if (threadIdx.x == 0) {
-    int s = 0;
-    off[0] = 0;
-    for (int l = 0; l < L; l++) {
-      s += sel_counts[f * L + l];
-      off[l + 1] = s;
+  pdl_wait();
+  if (warp == 0) {  // level offsets: the L counts loaded at once, inclusive warp scan
+    int s = lane < L ? sel_counts[f * L + lane] : 0;
+#pragma unroll
+    for (int o = 1; o < kMaxLevels; o <<= 1) {
+      const int v = __shfl_up_sync(0xFFFFFFFFu, s, o);
+      if (lane >= o) s += v;
     }
+    if (lane < L) off[lane + 1] = s;
+    if (lane == 0) off[0] = 0;
   }
   __syncthreads();
   if (blockIdx.x == 0 && threadIdx.x <= L) counts[f * (L + 1) + threadIdx.x] = off[threadIdx.x];
@@ -117,19 +122,48 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
   const uint8_t* p0 = img + (int64_t)(ly - 21) * ip + (lx - 21);
   const int sh = (int)(reinterpret_cast<uintptr_t>(p0) & 15);
   const uint8_t* P;  // P[r * PP + c] = raw patch pixel (ly - 21 + r, lx - 21 + c)
-  if ((ip & 15) == 0 && lx >= 21 && lx + 21 < w && ly >= 21 && ly + 21 < h && lx - 21 - sh + 64 <= ip) {
-    // interior: 43 rows x four aligned 16-B chunks, all loads in flight at once
-    const uint4* base = reinterpret_cast<const uint4*>(p0 - sh);
-    for (int i = lane; i < PR * 4; i += 32) {
-      const int r = i >> 2, c = i & 3;
-      *reinterpret_cast<uint4*>(Pw + r * PP + 16 * c) = __ldg(base + (int64_t)r * (ip >> 4) + c);
+  if ((ip & 15) == 0 && lx >= 21 && lx + 21 < w && lx - 21 - sh + 64 <= ip) {
+    // columns inside the level: 43 rows x four aligned 16-B chunks, rows mapped by REFLECT_101
+    // (identity away from the top/bottom border); all six loads of a lane are issued before
+    // the first store (one global latency, not six)
+    const uint8_t* cb = img + (lx - 21 - sh);
+    const bool rows_in = ly >= 21 && ly + 21 < h;
+    constexpr int NCH = (PR * 4 + 31) / 32;
+    uint4 chunk[NCH];
+#pragma unroll
+    for (int k = 0; k < NCH; k++) {
+      const int i = lane + 32 * k;
+      if (i < PR * 4) {
+        const int r = i >> 2, sr = rows_in ? ly - 21 + r : reflect101(ly - 21 + r, h);
+        chunk[k] = __ldg(reinterpret_cast<const uint4*>(cb + (int64_t)sr * ip) + (i & 3));
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < NCH; k++) {
+      const int i = lane + 32 * k;
+      if (i < PR * 4) *reinterpret_cast<uint4*>(Pw + (i >> 2) * PP + 16 * (i & 3)) = chunk[k];
     }
     P = Pw + sh;
   } else {
-    // near the level border: REFLECT_101 (the blur's border rule), byte loads
-    for (int i = lane; i < PR * PR; i += 32) {
-      const int r = i / PR, c = i - r * PR;
-      Pw[r * PP + c] = __ldg(img + (int64_t)reflect101(ly - 21 + r, h) * ip + reflect101(lx - 21 + c, w));
+    // near the left/right level border: REFLECT_101 (the blur's border rule) byte loads, 8 per
+    // lane in flight per batch
+    constexpr int BB = 8;
+#pragma unroll 1
+    for (int i0 = 0; i0 < PR * PR; i0 += 32 * BB) {
+      uint32_t v[BB];
+#pragma unroll
+      for (int k = 0; k < BB; k++) {
+        const int i = i0 + lane + 32 * k;
+        if (i < PR * PR) {
+          const int r = i / PR, c = i - r * PR;
+          v[k] = __ldg(img + (int64_t)reflect101(ly - 21 + r, h) * ip + reflect101(lx - 21 + c, w));
+        }
+      }
+#pragma unroll
+      for (int k = 0; k < BB; k++) {
+        const int i = i0 + lane + 32 * k;
+        if (i < PR * PR) Pw[(i / PR) * PP + (i % PR)] = (uint8_t)v[k];
+      }
     }
     P = Pw;
   }
@@ -183,8 +217,8 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
     };
     uint32_t q0 = ld2(0), q1 = ld2(1), q2 = ld2(2), q3 = ld2(3), q4 = ld2(4), q5 = ld2(5);
     uint32_t* V32 = reinterpret_cast<uint32_t*>(V) + lane;
-#pragma unroll 4
-    for (int r = 0; r < BR; r++) {
+#pragma unroll
+    for (int r = 0; r < BR; r++) {  // fully unrolled: the window shift is register renaming
       const uint32_t q6 = ld2(r + 6);
       V32[r * (VP / 2)] = 18u * (q0 + q6) + 34u * (q1 + q5) + 48u * (q2 + q4) + 56u * q3;
       q0 = q1; q1 = q2; q2 = q3; q3 = q4; q4 = q5; q5 = q6;
@@ -195,26 +229,64 @@ __global__ void __launch_bounds__(DESC_WARPS * 32) describe_kernel(Geom g, Frame
   // The blurred value is needed only at the 512 sample points, so the horizontal pass runs
   // there alone: B(oy, ox) = (sum_j k_j V[18 + oy][18 + ox + j] + 2^15) >> 16.
   const long long r2 = (long long)m10 * m10 + (long long)m01 * m01;
-  const float inv_r = r2 ? (float)(1.0 / sqrt((double)r2)) : 0.f;
-  const float cs = (float)m10 * inv_r, sn = (float)m01 * inv_r;  // |m| < 2^24: exact conversions
+  // 1/r in f32: r2 < 2^49 converts with relative error <= 2^-24 and rsqrtf is within 2 ulp,
+  // so cs, sn carry < 4e-7 relative error and |t| <= 19 stays within 1e-5 of the exact
+  // quotient -- far inside the 1e-4 band that sends a near-tie to the exact integer test
+  const float inv_r = r2 ? rsqrtf((float)r2) : 0.f;
+  // r2 == 0 (no rotation): (cs, sn) = (1, 0) gives t = px, py exactly, never near a tie
+  const float cs = r2 ? (float)m10 * inv_r : 1.f, sn = r2 ? (float)m01 * inv_r : 0.f;  // |m| < 2^24: exact
+  const uint32_t pw[8] = {pa.x, pa.y, pa.z, pa.w, pb.x, pb.y, pb.z, pb.w};
+  // horizontal pass at one sample: the 7 V values v0..v6 from the 4 words covering them
+  // (funnel shift by 16 when they start at an odd u16; V is word aligned, the 4th word may be
+  // the padding after V), weighted by dp2a on 16-bit pairs (v <= 65280, weights < 256)
+  const uint32_t* V32 = reinterpret_cast<const uint32_t*>(V);
+  auto blurred = [&](int ox, int oy) -> int {
+    const int idx = (18 + oy) * VP + 18 + ox + podd;
+    const uint32_t* wv = V32 + (idx >> 1);
+    const uint32_t s = 16u * (uint32_t)(idx & 1);
+    const uint32_t w0 = wv[0], w1 = wv[1], w2 = wv[2], w3 = wv[3];
+    uint32_t sum = __dp2a_lo(__funnelshift_r(w0, w1, s), 18u | 34u << 8, 1u << 15);  // 18 v0 + 34 v1
+    sum = __dp2a_lo(__funnelshift_r(w1, w2, s), 48u | 56u << 8, sum);               // 48 v2 + 56 v3
+    sum = __dp2a_lo(__funnelshift_r(w2, w3, s), 48u | 34u << 8, sum);               // 48 v4 + 34 v5
+    sum = __dp2a_lo(__funnelshift_r(w3, w3, s), 18u, sum);                          // 18 v6
+    return (int)(sum >> 16);
+  };
+  // fast pass, branch-free: every offset from the f32 estimate rounded half-to-even with the
+  // 1.5 * 2^23 trick; an estimate within 1e-4 of a half-integer only raises `near`
   uint32_t byte = 0;
-#pragma unroll 2
+  bool near = false;
+#pragma unroll
   for (int t = 0; t < 8; t++) {
-    const int b = lane * 8 + t;
     int v[2];
 #pragma unroll
     for (int e = 0; e < 2; e++) {
-      const int px = pat[4 * b + 2 * e], py = pat[4 * b + 2 * e + 1];
-      int ox = px, oy = py;
-      if (r2) {
-        ox = rhe_rot(px, -py, cs, sn, m10, m01, r2);  // (px m10 - py m01) / r
-        oy = rhe_rot(px, py, sn, cs, m01, m10, r2);   // (px m01 + py m10) / r
-      }
-      const uint16_t* vr = V + (18 + oy) * VP + 18 + ox + podd;
-      const int sum = 18 * (vr[0] + vr[6]) + 34 * (vr[1] + vr[5]) + 48 * (vr[2] + vr[4]) + 56 * vr[3];
-      v[e] = (sum + (1 << 15)) >> 16;
+      // signed bytes 2e (x) and 2e + 1 (y) of the pair's word
+      const int px = (int)(pw[t] << (24 - 16 * e)) >> 24, py = (int)(pw[t] << (16 - 16 * e)) >> 24;
+      const float tx = __fmaf_rn((float)px, cs, __fmul_rn((float)-py, sn));  // (px m10 - py m01) / r
+      const float ty = __fmaf_rn((float)px, sn, __fmul_rn((float)py, cs));   // (px m01 + py m10) / r
+      const float bx = __fadd_rn(tx, 12582912.0f), by = __fadd_rn(ty, 12582912.0f);
+      const float dx = __fsub_rn(tx, __fsub_rn(bx, 12582912.0f)), dy = __fsub_rn(ty, __fsub_rn(by, 12582912.0f));
+      near |= (fabsf(fabsf(dx) - 0.5f) <= 1e-4f) | (fabsf(fabsf(dy) - 0.5f) <= 1e-4f);
+      v[e] = blurred(__float_as_int(bx) - 0x4B400000, __float_as_int(by) - 0x4B400000);
     }
     byte |= (uint32_t)(v[0] < v[1]) << t;
+  }
+  if (__any_sync(0xFFFFFFFFu, near)) {  // rare: redo the byte with the exact tie test
+    byte = 0;
+    for (int t = 0; t < 8; t++) {
+      int v[2];
+      for (int e = 0; e < 2; e++) {
+        const uint32_t wd = __ldg(reinterpret_cast<const uint32_t*>(pattern) + 8 * lane + t);
+        const int px = (int)(wd << (24 - 16 * e)) >> 24, py = (int)(wd << (16 - 16 * e)) >> 24;
+        int ox = px, oy = py;
+        if (r2) {
+          ox = rhe_rot(px, -py, cs, sn, m10, m01, r2);
+          oy = rhe_rot(px, py, sn, cs, m01, m10, r2);
+        }
+        v[e] = blurred(ox, oy);
+      }
+      byte |= (uint32_t)(v[0] < v[1]) << t;
+    }
   }
   const int64_t o = (int64_t)f * g.kp_capacity + i;
   desc[o * SS_DESC_BYTES + lane] = (uint8_t)byte;
