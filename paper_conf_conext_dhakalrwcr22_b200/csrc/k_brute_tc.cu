@@ -280,6 +280,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(TC_THREADS, 1)
         mbar_expect_tx(full(s), BLK_BYTES);
         bulk_g2s(sb + s * BLK_BYTES, mexp + ((int64_t)(t0 + t) * 2 + rank) * BLK_BYTES, BLK_BYTES, full(s));
       }
+      // drain: the leader's multicast commits of the last STAGES tiles arrive on this CTA's
+      // empty barriers asynchronously; wait for them so no arrival can land in this shared
+      // memory after the CTA has exited (where the next CTA on the SM keeps its barriers)
+      for (int t = nt > STAGES ? nt - STAGES : 0; t < nt; t++) mbar_wait(empty(t % STAGES), (uint32_t)(t / STAGES) & 1u);
     }
   } else if (warp == 1) {
     if (lane == 0 && leader) {  // MMA issuer
