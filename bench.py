@@ -802,20 +802,33 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
     h2d_gbs = fr[0].numel() * 50 / (_t0.elapsed_time(_t1) * 1e-3) / 1e9
     del _dbuf
     graph_note = ("; io.reuse_graph = 1: each (ctx, input-ring slot) tick is a cached CUDA graph replayed by "
-                  "ss_track_tick (one launch per tick); direct = the same calls without graph reuse")
-    if not window or dev_map is None:
-        r = measure(False, True)
+                  "ss_track_tick (one launch per tick); direct = the same calls without graph reuse; both modes "
+                  "are trial-measured, the faster one (`mode`) is measured again for `value`")
+    resident = bool(window and dev_map is not None)
+
+    def pick(res: bool):
+        """Both API modes (io.reuse_graph 1 / 0) are trial-measured; the faster one is measured
+        AGAIN and that fresh run is the reported value (the selection never reuses its own sample)."""
+        trial_reuse, trial_direct = measure(res, True), measure(res, False)
+        reuse = trial_reuse["value"] >= trial_direct["value"]
+        r_ = measure(res, reuse)
+        r_["mode"] = "reuse_graph" if reuse else "direct"
+        r_["trials"] = {"reuse_graph": trial_reuse["value"], "direct": trial_direct["value"]}
+        return r_, trial_reuse, trial_direct
+
+    if not resident:
+        r, tr, td = pick(False)
         r["path"] = "pinned host -> ss_track_tick (" + path + ")" + \
             ("; the shared map is device-resident server state" if not window else "") + graph_note
-        r["direct"] = measure(False, False)
+        r["reuse_graph"], r["direct"] = tr, td
         r["h2d_gbs_raw"] = h2d_gbs
         return r
-    r = measure(True, True)
+    r, tr, td = pick(True)
     r["path"] = ("pinned host frames + camera predictions -> ss_track_tick (" + path + "); the map state (each "
                  "client's local-map points, last-frame points, masks) is server state resident in HBM, "
                  "as the SLAM-Share server keeps the maps and clients upload only frames (P:L64, P:L68); "
                  "host_map = the same with the map state copied from the host too" + graph_note)
-    r["direct"] = measure(True, False)
+    r["reuse_graph"], r["direct"] = tr, td
     r["host_map"] = measure(False, True)
     r["h2d_gbs_raw"] = h2d_gbs
     return r
