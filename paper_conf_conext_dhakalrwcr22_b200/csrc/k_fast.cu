@@ -185,6 +185,47 @@ __global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(const __grid_
     const CellInfo c = cells[ci];
     const int cx0 = c.x0 - xa, cw = c.x1 - c.x0;  // staged columns [cx0, cx0 + cw), cw < 64
     unsigned long long kmin[2] = {0ull, 0ull}, kini[2] = {0ull, 0ull};
+    if (Dh <= 32) {
+      // one pass, lane = row: only the row's own words are read; the neighbour rows' 3-wide
+      // maxima come from lanes y - 1 and y + 1 by shuffles (rows -1 and Dh are the zero rows
+      // of the score map, hence the lane masks); lanes >= Dh read the zero row below the band
+      const int base = cx0 - 4, a0 = base & ~3;
+      const uint32_t sh = 8u * (uint32_t)(base & 3);
+      const uint32_t* pr = reinterpret_cast<const uint32_t*>(Mb + ((lane < Dh ? lane : Dh) + 1) * mbw + a0);
+      auto aword = [&](int j) -> uint32_t {
+        const int valid = cw - (4 * j - 4);
+        const uint32_t v = __funnelshift_r(pr[j], pr[j + 1], sh);
+        return valid >= 4 ? v : (valid <= 0 ? 0u : v & (0xFFFFFFFFu >> (8 * (4 - valid))));
+      };
+      const uint32_t upm = lane > 0 ? 0xFFFFFFFFu : 0u, dnm = lane + 1 < Dh ? 0xFFFFFFFFu : 0u;
+      const uint32_t tmin1 = (uint32_t)(tmin + 1) * 0x10001u, tini1 = (uint32_t)(tini + 1) * 0x10001u;
+      uint32_t pw = 0u, cwd = aword(1);
+      const int nk = (cw + 3) >> 2;
+      for (int k = 0; k < nk; k++) {
+        const uint32_t nw = aword(k + 2);
+        const uint32_t Lw = __byte_perm(pw, cwd, 0x6543), Rw = __byte_perm(cwd, nw, 0x4321);
+        uint32_t bmin = 0u, bini = 0u;
+#pragma unroll
+        for (int half = 0; half < 2; half++) {  // lanes: pixels (0, 2), then (1, 3)
+          const uint32_t sel = half ? 0x7371u : 0x7270u;
+          const uint32_t Ch = __byte_perm(cwd, 0, sel), Lh = __byte_perm(Lw, 0, sel), Rh = __byte_perm(Rw, 0, sel);
+          const uint32_t hlr = __vimax3_u16x2(Lh, Rh, Lh), hf = __vimax3_u16x2(Lh, Rh, Ch);
+          const uint32_t up = __shfl_up_sync(0xFFFFFFFFu, hf, 1) & upm;
+          const uint32_t dn = __shfl_down_sync(0xFFFFFFFFu, hf, 1) & dnm;
+          const uint32_t nb = __vimax3_u16x2(hlr, up, dn);
+          const uint32_t C = Ch | 0x80008000u;
+          const uint32_t ok = (C - nb - 0x00010001u) & (C - tmin1) & 0x80008000u;  // > neighbours, > minTh
+          const uint32_t oi = ok & (C - tini1);                                       // and > iniTh
+          bmin |= ((ok >> 15) & 1u) << half | ((ok >> 31) & 1u) << (2 + half);
+          bini |= ((oi >> 15) & 1u) << half | ((oi >> 31) & 1u) << (2 + half);
+        }
+        kmin[0] |= (unsigned long long)bmin << (4 * k);
+        kini[0] |= (unsigned long long)bini << (4 * k);
+        pw = cwd;
+        cwd = nw;
+      }
+      if (lane >= Dh) kmin[0] = kini[0] = 0ull;
+    } else
 #pragma unroll
     for (int hh = 0; hh < 2; hh++) {
       const int y = lane + 32 * hh;
