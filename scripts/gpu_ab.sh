@@ -10,7 +10,7 @@ for rep in 1 2; do for V in "$@"; do
   timeout 600 python bench.py --no-cpu-baseline > $OUT/ab_${TAG}_${V}_$rep.json 2>/dev/null
   python -c "import json,sys; d=json.loads(open('$OUT/ab_${TAG}_${V}_$rep.json').read().strip().splitlines()[-1]); print('$V', $rep, round(d['value']), round(d['kernels_us']['describe'],2), round(d['e2e']['value']))"
 done; done
-for P in 3 6 8; do
+for P in ${SWEEP:-}; do
   timeout 600 python bench.py --no-cpu-baseline --inflight $P > $OUT/ab_${TAG}_inflight$P.json 2>/dev/null
   python -c "import json; d=json.loads(open('$OUT/ab_${TAG}_inflight$P.json').read().strip().splitlines()[-1]); print('inflight $P', round(d['value']), d['latency_ms']['p50'])"
 done
