@@ -569,32 +569,42 @@ def run_ours(args, cfg):
     per_func = {}
     for n_, t_ in avg_us.items():
         per_func.setdefault(func_of.get(n_, n_), []).append(n_)
-    dom_f = max(per_func, key=lambda f_: sum(avg_us[n_] for n_ in per_func[f_]))
-    members = per_func[dom_f]
-    bound = kernel_work(members[0], p, B, cand_l, kps_l, Q, cfg["map"], NLF)[0]
-    work = sum(kernel_work(n_, p, B, cand_l, kps_l, Q, cfg["map"], NLF)[1] for n_ in members)
-    dom_us = sum(avg_us[n_] for n_ in members)
-    avg_us_dom = dom_us
-    dom = dom_f if len(members) == 1 else f"{dom_f} ({' + '.join(members)})"
     peaks = measured_peaks()
-    step_share = dom_us / (1000.0 * float(np.mean(prof_step_ms)))
-    if bound == "hbm":
-        achieved = work / (avg_us_dom * 1e-6) / 1e9
-        roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                "frac": achieved / peaks["hbm_gbs"], "traffic": None, "kernel": dom, "peak_src": peaks["src"],
-                "share_of_step": step_share}
-    elif bound == "alu":
-        achieved = work / (avg_us_dom * 1e-6) / 1e12
-        roof = {"bound": "alu", "achieved": achieved, "peak": ALU_PEAK_TOPS, "unit": "Tops/s",
-                "frac": achieved / ALU_PEAK_TOPS, "traffic": None, "kernel": dom,
-                "peak_src": "derived: 148 SM x 64 ALU lanes/clk x 1.965 GHz (DESIGN.md §6)",
-                "work": f"{FAST_OPS_PER_PX} ops per detect pixel", "share_of_step": step_share}
-    else:  # tensor: int8 dense peak = measured bf16 dense x 2 (the guide's nominal i8 : bf16 ratio)
-        achieved = work / (avg_us_dom * 1e-6) / 1e12
-        roof = {"bound": "tensor", "achieved": achieved, "peak": peaks["i8_tops"], "unit": "TOPS",
-                "frac": achieved / peaks["i8_tops"], "traffic": None, "kernel": dom, "peak_src": peaks["tc_src"],
-                "work": "512 int8 ops per keypoint x map distance (256-long +-1 dot product)",
-                "share_of_step": step_share}
+    prof_step_us = 1000.0 * float(np.mean(prof_step_ms))
+
+    def roof_of(func):
+        members = per_func[func]
+        bound = kernel_work(members[0], p, B, cand_l, kps_l, Q, cfg["map"], NLF)[0]
+        work = sum(kernel_work(n_, p, B, cand_l, kps_l, Q, cfg["map"], NLF)[1] for n_ in members)
+        us = sum(avg_us[n_] for n_ in members)
+        name = func if len(members) == 1 else f"{func} ({' + '.join(members)})"
+        share = us / prof_step_us
+        if bound == "hbm":
+            achieved = work / (us * 1e-6) / 1e9
+            return members, {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                             "frac": achieved / peaks["hbm_gbs"], "traffic": None, "kernel": name,
+                             "peak_src": peaks["src"], "share_of_step": share}
+        if bound == "alu":
+            achieved = work / (us * 1e-6) / 1e12
+            return members, {"bound": "alu", "achieved": achieved, "peak": ALU_PEAK_TOPS, "unit": "Tops/s",
+                             "frac": achieved / ALU_PEAK_TOPS, "traffic": None, "kernel": name,
+                             "peak_src": "derived: 148 SM x 64 ALU lanes/clk x 1.965 GHz (DESIGN.md §6)",
+                             "work": f"{FAST_OPS_PER_PX} ops per detect pixel", "share_of_step": share}
+        # tensor: int8 dense peak = measured bf16 dense x 2 (the guide's nominal i8 : bf16 ratio)
+        achieved = work / (us * 1e-6) / 1e12
+        return members, {"bound": "tensor", "achieved": achieved, "peak": peaks["i8_tops"], "unit": "TOPS",
+                         "frac": achieved / peaks["i8_tops"], "traffic": None, "kernel": name,
+                         "peak_src": peaks["tc_src"],
+                         "work": "512 int8 ops per keypoint x map distance (256-long +-1 dot product)",
+                         "share_of_step": share}
+
+    dom_f = max(per_func, key=lambda f_: sum(avg_us[n_] for n_ in per_func[f_]))
+    members, roof = roof_of(dom_f)
+    # every kernel function's roofline, largest device time first (the dominant one is `roofline`)
+    rooflines = []
+    for f_ in sorted(per_func, key=lambda f_: -sum(avg_us[n_] for n_ in per_func[f_])):
+        r_ = roof_of(f_)[1]
+        rooflines.append({k_: r_[k_] for k_ in ("kernel", "bound", "achieved", "unit", "frac", "share_of_step")})
     traffic_file = os.path.join(ROOT, "profiles", "dram_traffic_r01.json")
     if os.path.exists(traffic_file):
         try:
@@ -664,6 +674,7 @@ def run_ours(args, cfg):
                         "profiling events inside instrumented twin graphs replaying the same "
                         f"{K} ticks one at a time (instrumented tick {float(np.mean(prof_step_ms)):.4f} ms)",
         "roofline": roof,
+        "rooflines": rooflines,
         "e2e": e2e,
         "gpu_launches": launches_per_step * K * world,
         "clocks": sampler.summary(),
