@@ -64,6 +64,7 @@ struct Shared {
   BScan::TempStorage scan;
   int sh[8];
   int H[16], G[17], S[15], E[15];
+  int W[DT / 32][8];  // dense path: per-warp packed (non-empty, multi-key) bin counts per depth
 };
 
 __device__ __forceinline__ void root_geom(const Geom& g, int l, int ri, int& ulx, int& urx) {
@@ -445,7 +446,9 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
       }
     }
     __syncthreads();
-    for (int r = r_lo - 1; r >= 0; r--) {
+#pragma unroll
+    for (int r = 2; r >= 0; r--) {  // r < r_lo <= 3; compile-time r keeps nz / mu in registers
+      if (r >= r_lo) continue;
       const int sz = nini << (2 * r);
       for (int b = tid; b < sz; b += DT) {
         const uint32_t* ch = cnt + off(r + 1) + 4 * b;
@@ -465,10 +468,18 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
         a += __shfl_xor_sync(0xFFFFFFFFu, a, o);
         m += __shfl_xor_sync(0xFFFFFFFFu, m, o);
       }
-      if (lane == 0) {
-        if (a) atomicAdd(&S_.H[r], a);
-        if (m) atomicAdd(&S_.G[r], m);
-      }
+      if (lane == 0) S_.W[tid >> 5][r] = a | (m << 16);  // per-warp partials (a, m <= 8192)
+    }
+  }
+  __syncthreads();
+  // warp r sums depth r's 32 warp partials (no same-address shared atomics across 32 warps)
+  if ((tid >> 5) <= R) {
+    int s = S_.W[lane][tid >> 5];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xFFFFFFFFu, s, o);
+    if (lane == 0) {
+      S_.H[tid >> 5] = s & 0xFFFF;
+      S_.G[tid >> 5] = s >> 16;
     }
   }
   __syncthreads();
