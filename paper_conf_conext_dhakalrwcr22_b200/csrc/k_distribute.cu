@@ -627,12 +627,14 @@ __global__ void __launch_bounds__(DT, 1)
   // ---- 1. candidate offsets per cell (rank order = cells row-major, then raster) ----
   {
     const int cpt = (ncells + DT - 1) / DT;  // <= 5 (MAX_CELLS)
-    int cnt[5];
+    int cnt[5], slot[5];
     int s = 0;
 #pragma unroll
-    for (int j = 0; j < 5; j++) {
+    for (int j = 0; j < 5; j++) {  // both loads issued before the scan (one global round trip)
       const int c = tid * cpt + j;
-      cnt[j] = (j < cpt && c < ncells) ? cc[c] : 0;
+      const bool in = j < cpt && c < ncells;
+      cnt[j] = in ? cc[c] : 0;
+      slot[j] = in ? cells[c0 + c].slot_off : 0;
       s += cnt[j];
     }
     int ex, tot;
@@ -642,7 +644,7 @@ __global__ void __launch_bounds__(DT, 1)
       const int c = tid * cpt + j;
       if (j < cpt && c < ncells) {
         cell_off[c] = ex;
-        cell_slot[c] = cells[c0 + c].slot_off;
+        cell_slot[c] = slot[j];
         ex += cnt[j];
       }
     }
@@ -666,13 +668,20 @@ __global__ void __launch_bounds__(DT, 1)
     uint32_t* key = cand + DCAP;
     {  // gather candidates into rank order (cells row-major, raster inside a cell)
       const uint32_t* fs = slots + (int64_t)f * g.slots_per_frame;
-      for (int i = tid; i < n; i += DT) {
-        int lo = 0, hi = ncells - 1;  // last cell with cell_off[c] <= i
+      auto src = [&](int i) {  // slot of rank i: last cell with cell_off[c] <= i
+        int lo = 0, hi = ncells - 1;
         while (lo < hi) {
           const int mid = (lo + hi + 1) >> 1;
           if (cell_off[mid] <= i) lo = mid; else hi = mid - 1;
         }
-        cand[i] = fs[cell_slot[lo] + (i - cell_off[lo])];
+        return cell_slot[lo] + (i - cell_off[lo]);
+      };
+      for (int i = tid; i < n; i += 2 * DT) {  // two independent global loads in flight per thread
+        const int i1 = i + DT;
+        const uint32_t v0 = fs[src(i)];
+        const uint32_t v1 = i1 < n ? fs[src(i1)] : 0u;
+        cand[i] = v0;
+        if (i1 < n) cand[i1] = v1;
       }
       __syncthreads();
     }
