@@ -591,11 +591,17 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
   const int nk_w = min(nk, g.cap[l]);
   SS_PHASE(8);
   uint32_t* sel_out = selected + (int64_t)f * g.kp_capacity + g.cap_off[l];
-  for (int t = tid; t < nk; t += DT) {
-    const uint32_t k = kept[t] >> 8;
+  // rank of each kept key = #smaller keys; 4 lanes per key each count a quarter of the list
+  for (int t0 = 0; t0 < nk; t0 += DT / 4) {
+    const int t = t0 + (tid >> 2), part = tid & 3;
+    const bool act = t < nk;
+    const uint32_t k = act ? kept[t] >> 8 : 0u;
     int pos = 0;
-    for (int u = 0; u < nk; u++) pos += (kept[u] >> 8) < k;
-    if (pos < nk_w) sel_out[pos] = kept[t];
+    if (act)
+      for (int u = part; u < nk; u += 4) pos += (kept[u] >> 8) < k;
+    pos += __shfl_xor_sync(0xFFFFFFFFu, pos, 1);
+    pos += __shfl_xor_sync(0xFFFFFFFFu, pos, 2);
+    if (act && part == 0 && pos < nk_w) sel_out[pos] = kept[t];
   }
   if (tid == 0) {
     sel_counts[f * g.L + l] = nk_w;
