@@ -402,6 +402,26 @@ ss_status ss_debug_phase_times(ss_ctx* ctx, int32_t frame, int32_t level, int64_
  * in-shared-memory capacity and took the global-memory path (for tests/benchmarks). */
 ss_status ss_debug_overflow_count(ss_ctx* ctx, int32_t* n);
 
+/* Which quadtree paths the (frame, level) distributions of the last ss_orb_extract took
+ * (DESIGN.md §5 distribute_kernel): *n_sort_smem = how many fell back from the dense-histogram
+ * fast path to the in-shared-memory sort path (the stop rules needed a depth beyond the dense
+ * tables), *n_global = how many ran on global scratch (> 8192 candidates).  Either may be NULL. */
+ss_status ss_debug_distribution_paths(ss_ctx* ctx, int32_t* n_sort_smem, int32_t* n_global);
+
+/* Lanes per query of the following WINDOW matches on ctx (1, 2, 4 or 8; 0 = chosen per launch
+ * from the query count, the default).  Results are identical for every value; tests use this
+ * to cover each kernel instance.  SS_EINVAL for other values.  Host only. */
+ss_status ss_debug_match_lanes(ss_ctx* ctx, int32_t lanes);
+
+/* Blurred-sample capture (S6 blur parity): while d_samples != NULL, every following
+ * ss_orb_extract also writes, per output keypoint slot, the 512 blurred values (u8) its 256
+ * comparisons read -- d_samples[f][slot][2b + e] = B_level(ly + oy, lx + ox) at point e of
+ * comparison b, (ox, oy) the rotated pattern offset (O6, O7) -- into the caller's DEVICE buffer
+ * of n_frames * kp_capacity * 512 bytes (slots >= the frame's count untouched).  The capture
+ * runs a second instance of the descriptor kernel; NULL (the default) restores the product
+ * kernel.  Host only (the pointer is stored, nothing is enqueued). */
+ss_status ss_debug_capture_samples(ss_ctx* ctx, uint8_t* d_samples);
+
 #ifdef __cplusplus
 }
 #endif

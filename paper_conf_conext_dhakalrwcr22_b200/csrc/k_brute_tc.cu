@@ -424,14 +424,16 @@ cudaError_t launch_brute_expand(int n_slots, const uint8_t* desc, int n_map, con
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 
+cudaError_t brute_tc_init() {  // ss_create, per device
+  return cudaFuncSetAttribute(brute_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM);
+}
+
 cudaError_t launch_brute_tc(int n_slots, int n_map, const int8_t* qexp, const int8_t* mexp, int splits,
                             unsigned long long* partial, cudaStream_t s) {
   if (n_slots <= 0 || n_map <= 0) return cudaSuccess;
   const int pairs = (n_slots + TC_ROWS - 1) / TC_ROWS;
   const int tiles = (n_map + TC_NT - 1) / TC_NT;
-  cudaError_t e = cudaFuncSetAttribute(brute_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM);
-  if (e != cudaSuccess) return e;
-  e = launch_pdl(brute_tc_kernel, dim3(2 * pairs, splits), dim3(TC_THREADS), TC_SMEM, s, qexp, mexp, n_slots, n_map,
+  cudaError_t e = launch_pdl(brute_tc_kernel, dim3(2 * pairs, splits), dim3(TC_THREADS), TC_SMEM, s, qexp, mexp, n_slots, n_map,
                  tiles, splits, partial);
   return e != cudaSuccess ? e : cudaGetLastError();
 }

@@ -60,13 +60,17 @@ __device__ __forceinline__ int rhe_rot(int a, int b, float ca, float cb, int ma,
   return rhe_exact((long long)a * ma + (long long)b * mb, r2, k);
 }
 
+// SAMPLES (test hook, ss_debug_capture_samples): also write the blurred value of every sample
+// point the comparisons read, samples[slot][b][e] for bit b = 8 * lane + t, point e
+template <bool SAMPLES>
 __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, FrameSrc src,
                                                                    const uint32_t* __restrict__ selected,
                                                                    const int32_t* __restrict__ sel_counts,
                                                                    const int8_t* __restrict__ pattern,
                                                                    ss_keypoint* __restrict__ kps,
                                                                    uint8_t* __restrict__ desc,
-                                                                   int32_t* __restrict__ counts) {
+                                                                   int32_t* __restrict__ counts,
+                                                                   uint8_t* __restrict__ samples) {
   pdl_trigger();
   extern __shared__ __align__(16) uint8_t sm[];  // DESC_WARPS * PER_WARP
   __shared__ int off[kMaxLevels + 1];
@@ -253,6 +257,8 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
   };
   // fast pass, branch-free: every offset from the f32 estimate rounded half-to-even with the
   // 1.5 * 2^23 trick; an estimate within 1e-4 of a half-integer only raises `near`
+  const int64_t o = (int64_t)f * g.kp_capacity + i;
+  uint8_t* smp = SAMPLES ? samples + o * 512 + 16 * lane : nullptr;
   uint32_t byte = 0;
   bool near = false;
 #pragma unroll
@@ -268,6 +274,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
       const float dx = __fsub_rn(tx, __fsub_rn(bx, 12582912.0f)), dy = __fsub_rn(ty, __fsub_rn(by, 12582912.0f));
       near |= (fabsf(fabsf(dx) - 0.5f) <= 1e-4f) | (fabsf(fabsf(dy) - 0.5f) <= 1e-4f);
       v[e] = blurred(__float_as_int(bx) - 0x4B400000, __float_as_int(by) - 0x4B400000);
+      if (SAMPLES) smp[2 * t + e] = (uint8_t)v[e];
     }
     byte |= (uint32_t)(v[0] < v[1]) << t;
   }
@@ -284,11 +291,11 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
           oy = rhe_rot(px, py, sn, cs, m01, m10, r2);
         }
         v[e] = blurred(ox, oy);
+        if (SAMPLES) smp[2 * t + e] = (uint8_t)v[e];
       }
       byte |= (uint32_t)(v[0] < v[1]) << t;
     }
   }
-  const int64_t o = (int64_t)f * g.kp_capacity + i;
   desc[o * SS_DESC_BYTES + lane] = (uint8_t)byte;
   if (lane == 0) {
     float ang = 0.f;
@@ -315,19 +322,23 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
 
 const int* brief_pattern_host() { return SS_BRIEF_PATTERN_HOST; }
 
+cudaError_t describe_init() {  // ss_create, per device (never under stream capture)
+  cudaError_t e = cudaFuncSetAttribute(describe_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)(DESC_WARPS * PER_WARP));
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(describe_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              (int)(DESC_WARPS * PER_WARP));
+}
+
 cudaError_t launch_describe(const Geom& g, int n_frames, FrameSrc src, const uint32_t* selected,
                             const int32_t* sel_counts, const int8_t* pattern, ss_keypoint* kps, uint8_t* desc,
-                            int32_t* counts, cudaStream_t s) {
+                            int32_t* counts, uint8_t* samples, cudaStream_t s) {
   const size_t smem = (size_t)DESC_WARPS * PER_WARP;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(describe_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
   dim3 grid((g.kp_capacity + DESC_WARPS - 1) / DESC_WARPS, n_frames);
-  cudaError_t e = launch_pdl(describe_kernel, grid, dim3(DESC_WARPS * 32), smem, s, g, src, selected, sel_counts,
-                             pattern, kps, desc, counts);
+  cudaError_t e = samples ? launch_pdl(describe_kernel<true>, grid, dim3(DESC_WARPS * 32), smem, s, g, src, selected,
+                                       sel_counts, pattern, kps, desc, counts, samples)
+                          : launch_pdl(describe_kernel<false>, grid, dim3(DESC_WARPS * 32), smem, s, g, src, selected,
+                                       sel_counts, pattern, kps, desc, counts, samples);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 

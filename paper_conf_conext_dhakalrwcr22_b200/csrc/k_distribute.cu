@@ -695,6 +695,7 @@ __global__ void __launch_bounds__(DT, 1)
     if (dense_body(g, l, f, n, cand, key, reinterpret_cast<uint8_t*>(key + DCAP), S_, selected, sel_counts,
                    ovf_counter, phase_ts))
       return;
+    if (tid == 0) atomicAdd(ovf_counter + 2, 1);  // counted for the tests (ss_debug_distribution_paths)
     __syncthreads();
     if (tid < 16) S_.H[tid] = 0;
     if (tid < 17) S_.G[tid] = 0;
@@ -720,17 +721,15 @@ int64_t distribute_ovf_bytes(int64_t slots) {
   return (b + 255) & ~(int64_t)255;
 }
 
+cudaError_t distribute_init() {  // ss_create, per device
+  return cudaFuncSetAttribute(distribute_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemTotal);
+}
+
 cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_levels, const CellInfo* cells,
                               const uint32_t* slots, const int32_t* cell_counts, uint32_t* selected, int32_t* sel_counts,
                               uint8_t* ovf, int64_t ovf_frame_bytes, const int64_t* ovf_level_off, int32_t* ovf_counter,
                               uint64_t* phase_ts, cudaStream_t s) {
   if (n_levels <= 0) return cudaSuccess;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(distribute_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemTotal);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
   dim3 grid(n_levels, n_frames);
   cudaError_t e = launch_pdl(distribute_kernel, grid, dim3(DT), kSmemTotal, s, g, cells, slots, cell_counts, selected,
                              sel_counts, ovf, ovf_frame_bytes, ovf_level_off, ovf_counter, level0, phase_ts);

@@ -315,17 +315,15 @@ size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int*
   return (size_t)*region_bytes + *mband_bytes;
 }
 
+cudaError_t fast_init() {  // ss_create, per device; ss_create rejects bands above 227 KB
+  return cudaFuncSetAttribute(fast_bands_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+}
+
 cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands, int n_bands,
                               const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s) {
   if (n_bands <= 0) return cudaSuccess;
   int rp, mbw, rb, mb, nb;
   const size_t smem = fast_smem_bytes(g, &rp, &mbw, &rb, &mb, &nb);
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(fast_bands_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 224 * 1024);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
   dim3 grid(n_bands, n_frames);
   cudaError_t e = launch_pdl(fast_bands_kernel, grid, dim3(FB_THREADS), smem, s, g, src, bands, cells, slots,
                              cell_counts, rp, mbw, rb);

@@ -169,16 +169,22 @@ __global__ void __launch_bounds__(GT, 1)
 
 }  // namespace
 
+size_t grid_smem_bytes(const Geom& g) {
+  int capmax = 0;
+  for (int l = 0; l < g.L; l++) capmax = capmax > g.N[l] ? capmax : g.N[l];
+  return (size_t)(2 * GMAX_CELLS + 1) * 4 + (size_t)capmax * 4 + 16;
+}
+
+cudaError_t grid_init() {  // ss_create, per device (ss_set_distribution checks grid_smem_bytes)
+  return cudaFuncSetAttribute(distribute_grid_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+}
+
 cudaError_t launch_distribute_grid(const Geom& g, int n_frames, int level0, int n_levels, const CellInfo* cells,
                                    const uint32_t* slots, const int32_t* cell_counts, uint32_t* selected,
                                    int32_t* sel_counts, cudaStream_t s) {
   if (n_levels <= 0) return cudaSuccess;
-  int capmax = 0;
-  for (int l = 0; l < g.L; l++) capmax = capmax > g.N[l] ? capmax : g.N[l];
-  const size_t smem = (size_t)(2 * GMAX_CELLS + 1) * 4 + (size_t)capmax * 4 + 16;
-  cudaError_t e = cudaFuncSetAttribute(distribute_grid_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  e = launch_pdl(distribute_grid_kernel, dim3(n_levels, n_frames), dim3(GT), smem, s, g, cells, slots, cell_counts,
+  const size_t smem = grid_smem_bytes(g);
+  cudaError_t e = launch_pdl(distribute_grid_kernel, dim3(n_levels, n_frames), dim3(GT), smem, s, g, cells, slots, cell_counts,
                  selected, sel_counts, level0);
   return e != cudaSuccess ? e : cudaGetLastError();
 }

@@ -250,7 +250,7 @@ cudaError_t launch_match_prepare(const Geom& g, int n_frames, const ss_keypoint*
 cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* kps, const uint8_t* desc,
                                 const int32_t* counts, const uint8_t* taken, int n_queries, const ss_mp_query* q,
                                 const uint8_t* qdesc, ss_match_cfg cfg, unsigned long long* claim, ss_match* out,
-                                const uint16_t* rowidx, cudaStream_t s) {
+                                const uint16_t* rowidx, int lanes, cudaStream_t s) {
   if (n_queries <= 0) return cudaSuccess;
   // lanes per query: enough groups to fill ~2 waves of the GPU (148 SMs x 2048 threads); a
   // query's window holds a handful of candidates, so with many queries fewer lanes per query
@@ -259,6 +259,7 @@ cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* 
   int wg = 8;
   const int64_t want = 2LL * 148 * 2048;
   while (wg > 1 && (int64_t)n_queries * (wg / 2) >= want) wg /= 2;
+  if (lanes == 1 || lanes == 2 || lanes == 4 || lanes == 8) wg = lanes;  // test hook override
   auto kern = wg == 1 ? match_window_kernel<1> : wg == 2 ? match_window_kernel<2> : wg == 4 ? match_window_kernel<4>
                                                                                             : match_window_kernel<8>;
   const int64_t threads = (int64_t)n_queries * wg;

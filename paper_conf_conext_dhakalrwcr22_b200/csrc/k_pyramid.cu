@@ -289,14 +289,12 @@ bool pyramid_plan(const Geom& g, const uint32_t* tab, const int64_t* xoff, const
   return *smem <= kPyrSmemMax && max_g < 16384 && max_y < 65536;
 }
 
+cudaError_t pyramid_init() {  // ss_create, per device; pyramid_plan keeps every plan within kPyrSmemMax
+  return cudaFuncSetAttribute(pyramid_fused_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kPyrSmemMax);
+}
+
 cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const uint4* gtab, const uint32_t* ytab,
                            const PyrLvl* plan, int n_blocks, int buf0, int buf1, int smem, cudaStream_t s) {
-  static bool attr_set = false;
-  if (!attr_set) {  // pyramid_plan keeps every plan within kPyrSmemMax
-    cudaError_t e = cudaFuncSetAttribute(pyramid_fused_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kPyrSmemMax);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
   dim3 grid(n_blocks, n_frames);
   cudaError_t e = launch_pdl(pyramid_fused_kernel, grid, dim3(PT), (size_t)smem, s, g, src, gtab, ytab, plan, buf0, buf1);
   return e != cudaSuccess ? e : cudaGetLastError();

@@ -139,7 +139,7 @@ struct ss_ctx {
   uint8_t* ovf = nullptr;
   int64_t ovf_frame_bytes = 0;
   int64_t* ovf_level_off = nullptr;
-  int32_t* ovf_counter = nullptr;  // [0] overflowed levels, [1] capacity violations
+  int32_t* ovf_counter = nullptr;  // [0] overflowed levels, [1] capacity violations, [2] sort fallbacks
   int8_t* pattern = nullptr;
   unsigned long long* claim = nullptr;
   unsigned long long* claim_lf = nullptr;  // O13's own dedup claims
@@ -153,9 +153,13 @@ struct ss_ctx {
   uint64_t* phase_ts = nullptr;  // distribution phase timestamps [max_frames][L][16] (debug hook)
   unsigned long long* partial = nullptr;
   int dist_mode = SS_DIST_QUADTREE;  // ss_set_distribution
+  // test hooks: lanes per WINDOW query (0 = chosen per launch), blurred-sample capture buffer
+  int win_lanes = 0;
+  uint8_t* dbg_samples = nullptr;
   int32_t* stereo_sad = nullptr;  // O12: accepted SAD per left keypoint [max_frames/2][cap]
   // ss_track_tick staging (device copies of the host inputs / outputs of a tick)
   uint8_t* io_frames = nullptr;   // [max_frames][H][io_pitch]
+  uint8_t* io_frames_lin = nullptr;  // [max_frames][H][W]: dense frames with an unaligned pitch land here first
   int32_t io_pitch = 0;
   ss_keypoint* io_kps = nullptr;
   uint8_t* io_desc = nullptr;
@@ -227,7 +231,7 @@ void free_ctx(ss_ctx* c) {
   cudaSetDevice(c->device);
   void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr_plan, c->pyr_gtab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
                   c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->claim_lf, c->partial, c->rowidx, c->phase_ts,
-                  c->brute_qexp, c->brute_mexp, c->stereo_sad, c->io_frames, c->io_kps, c->io_desc, c->io_counts,
+                  c->brute_qexp, c->brute_mexp, c->stereo_sad, c->io_frames, c->io_frames_lin, c->io_kps, c->io_desc, c->io_counts,
                   c->io_cams, c->io_points, c->io_pf, c->io_pdesc, c->io_taken, c->io_queries, c->io_matches,
                   c->io_uright, c->io_depth, c->io_lf_off, c->io_lf_pts, c->io_lf_desc, c->io_last_cams,
                   c->io_lf_matches, c->io_lf_n, c->io_lf_mask};
@@ -487,7 +491,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->sel_counts, sizeof(int32_t) * F * L);
   ALLOC(c->ovf, F * c->ovf_frame_bytes);
   ALLOC(c->ovf_level_off, sizeof(int64_t) * L);
-  ALLOC(c->ovf_counter, sizeof(int32_t) * 2);
+  ALLOC(c->ovf_counter, sizeof(int32_t) * 4);
   ALLOC(c->pattern, 1024);
   ALLOC(c->claim, sizeof(unsigned long long) * F * g.kp_capacity);
   ALLOC(c->claim_lf, sizeof(unsigned long long) * F * g.kp_capacity);
@@ -498,6 +502,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   {
     const int64_t Qm = std::max<int64_t>(max_queries, 1);
     ALLOC(c->io_frames, (size_t)F * g.H * c->io_pitch);
+    ALLOC(c->io_frames_lin, (size_t)F * g.H * c->io_pitch);
     ALLOC(c->io_kps, sizeof(ss_keypoint) * F * g.kp_capacity);
     ALLOC(c->io_desc, (size_t)F * g.kp_capacity * SS_DESC_BYTES);
     ALLOC(c->io_counts, sizeof(int32_t) * F * (L + 1));
@@ -525,6 +530,12 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   }
 #undef ALLOC
   if (e == cudaSuccess) e = lastframe_init();
+  if (e == cudaSuccess) e = fast_init();
+  if (e == cudaSuccess) e = distribute_init();
+  if (e == cudaSuccess) e = describe_init();
+  if (e == cudaSuccess) e = pyramid_init();
+  if (e == cudaSuccess) e = brute_tc_init();
+  if (e == cudaSuccess) e = grid_init();
   if (e == cudaSuccess) e = cudaMemcpy(c->cells, c->cells_h.data(), sizeof(CellInfo) * c->cells_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->bands, c->bands_h.data(), sizeof(BandInfo) * c->bands_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess && !tab.empty()) e = cudaMemcpy(c->xytab, tab.data(), sizeof(uint32_t) * tab.size(), cudaMemcpyHostToDevice);
@@ -534,7 +545,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     e = cudaMemcpy(c->pyr_gtab, gtab.data(), sizeof(uint4) * gtab.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->ovf_level_off, ovf_off.data(), sizeof(int64_t) * L, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->pattern, pat.data(), 1024, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMemset(c->ovf_counter, 0, sizeof(int32_t) * 2);
+  if (e == cudaSuccess) e = cudaMemset(c->ovf_counter, 0, sizeof(int32_t) * 4);
   for (int i = 0; i < ss_ctx::kSide && e == cudaSuccess; i++) {
     e = cudaStreamCreateWithFlags(&c->side[i], cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_join[i], cudaEventDisableTiming);
@@ -582,7 +593,7 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   // Profiling events: start, then a (before, after) pair around every launch in this order:
   // fast l0, distribute l0, pyramid (levels 1..L-1, one launch), fast l>=1, distribute l>=1, describe.
   prof_mark(c, s);
-  SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 2, s));
+  SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 4, s));
   SS_CUDA_TRY(cudaEventRecord(c->ev_fork, s));
   // with profiling events installed the level-0 branch runs in line on `stream`, so every
   // kernel is timed alone (the fork/join only changes overlap, not any kernel's work)
@@ -620,7 +631,8 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   prof_mark(c, s);
   if (q != s) SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[0], 0));
   prof_mark(c, s);
-  SS_CUDA_TRY(launch_describe(g, n_frames, src, c->selected, c->sel_counts, c->pattern, d_kps, d_desc, d_counts, s));
+  SS_CUDA_TRY(launch_describe(g, n_frames, src, c->selected, c->sel_counts, c->pattern, d_kps, d_desc, d_counts,
+                              c->dbg_samples, s));
   prof_mark(c, s);
   c->last_frames = d_frames;
   c->last_stride = frame_stride;
@@ -652,7 +664,7 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
     prof_mark(c, s);
     prof_mark(c, s);
     SS_CUDA_TRY(launch_match_window(c->g, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_queries, d_queries,
-                                    d_map_desc, *cfg, c->claim, d_out, c->rowidx, s));
+                                    d_map_desc, *cfg, c->claim, d_out, c->rowidx, c->win_lanes, s));
     prof_mark(c, s);
     if (cfg->dedup) {
       prof_mark(c, s);
@@ -667,6 +679,15 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
     if (n_map > 0 && !d_map_desc) return fail(SS_EINVAL, "NULL map");
     if (n_frames == 0) return SS_OK;
     const int n_slots = n_frames * c->g.kp_capacity;
+    if (n_map == 0) {
+      // an empty map (e.g. at session start): no candidates, every slot gets {-1, 256, 256}
+      // (the merge with zero partials; c->partial may not even exist when max_map == 0)
+      for (int i = 0; i < 4; i++) prof_mark(c, s);
+      prof_mark(c, s);
+      SS_CUDA_TRY(launch_brute_merge(c->g, n_frames, d_counts, 0, nullptr, *cfg, d_out, s));
+      prof_mark(c, s);
+      return SS_OK;
+    }
     const int splits = brute_tc_splits(n_slots, n_map, c->max_splits, c->n_sm);
     prof_mark(c, s);
     SS_CUDA_TRY(launch_brute_expand(n_slots, d_desc, n_map, d_map_desc, c->brute_qexp, c->brute_mexp, s));
@@ -811,6 +832,15 @@ ss_status ss_match_last_frame(ss_ctx* c, int32_t n_frames, const ss_camera* d_ca
 ss_status ss_set_distribution(ss_ctx* c, int32_t mode) {
   if (!c) return fail(SS_EINVAL, "NULL ctx");
   if (mode != SS_DIST_QUADTREE && mode != SS_DIST_GRID_TOPN) return fail(SS_EINVAL, "unknown distribution mode");
+  if (mode == SS_DIST_GRID_TOPN && grid_smem_bytes(c->g) > 227 * 1024)
+    return fail(SS_EUNSUPPORTED, "n_per_level too large for the grid top-N kernel's shared memory");
+  if (mode != c->dist_mode) {
+    // cached tick graphs were captured with the other distribution's kernels
+    cudaSetDevice(c->device);
+    for (ss_ctx::TickGraph& tg : c->tick_graphs)
+      if (tg.exec) cudaGraphExecDestroy(tg.exec);
+    c->tick_graphs.clear();
+  }
   c->dist_mode = mode;
   return SS_OK;
 }
@@ -829,10 +859,19 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
   // copies (a 2-D copy moves row by row, several times slower for 0.3-0.5 MB frames).
   int P = c->io_pitch;
   int64_t fstride = (int64_t)g.H * P;
-  if (io->pitch <= c->io_pitch && (n_frames == 1 || io->frame_stride == (int64_t)io->pitch * g.H)) {
+  const bool dense = io->pitch <= c->io_pitch && (n_frames == 1 || io->frame_stride == (int64_t)io->pitch * g.H);
+  if (dense && io->pitch % 16 == 0) {
     P = io->pitch;
     fstride = (int64_t)g.H * P;
     SS_CUDA_TRY(cudaMemcpyAsync(c->io_frames, io->frames, (size_t)fstride * n_frames, cudaMemcpyHostToDevice, s));
+  } else if (dense) {
+    // a pitch that is not a multiple of 16 B (e.g. KITTI's 1241) would send FAST's band staging
+    // and describe's patch loads down their per-byte paths: one linear H2D into the lead-in
+    // staging buffer, then one device-side 2-D copy to the 16-B aligned staging pitch
+    const int64_t lin = (int64_t)g.H * io->pitch * n_frames;
+    SS_CUDA_TRY(cudaMemcpyAsync(c->io_frames_lin, io->frames, (size_t)lin, cudaMemcpyHostToDevice, s));
+    SS_CUDA_TRY(cudaMemcpy2DAsync(c->io_frames, P, c->io_frames_lin, io->pitch, g.W, (size_t)g.H * n_frames,
+                                  cudaMemcpyDeviceToDevice, s));
   } else {
     for (int f = 0; f < n_frames; f++)
       SS_CUDA_TRY(cudaMemcpy2DAsync(c->io_frames + f * fstride, P, io->frames + f * io->frame_stride, io->pitch, g.W,
@@ -1107,6 +1146,30 @@ ss_status ss_debug_overflow_count(ss_ctx* c, int32_t* n) {
   SS_CUDA_TRY(cudaMemcpy(v, c->ovf_counter, sizeof(v), cudaMemcpyDeviceToHost));
   *n = v[0];
   if (v[1] != 0) return fail(SS_ECAPACITY, "a level kept more keypoints than its level_cap (bug)");
+  return SS_OK;
+}
+
+ss_status ss_debug_distribution_paths(ss_ctx* c, int32_t* n_sort_smem, int32_t* n_global) {
+  if (!c) return fail(SS_EINVAL, "NULL argument");
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  SS_CUDA_TRY(cudaDeviceSynchronize());
+  int32_t v[3];
+  SS_CUDA_TRY(cudaMemcpy(v, c->ovf_counter, sizeof(v), cudaMemcpyDeviceToHost));
+  if (n_global) *n_global = v[0];
+  if (n_sort_smem) *n_sort_smem = v[2];
+  return SS_OK;
+}
+
+ss_status ss_debug_match_lanes(ss_ctx* c, int32_t lanes) {
+  if (!c) return fail(SS_EINVAL, "NULL ctx");
+  if (lanes != 0 && lanes != 1 && lanes != 2 && lanes != 4 && lanes != 8) return fail(SS_EINVAL, "lanes must be 0, 1, 2, 4 or 8");
+  c->win_lanes = lanes;
+  return SS_OK;
+}
+
+ss_status ss_debug_capture_samples(ss_ctx* c, uint8_t* d_samples) {
+  if (!c) return fail(SS_EINVAL, "NULL ctx");
+  c->dbg_samples = d_samples;
   return SS_OK;
 }
 

@@ -149,7 +149,7 @@ cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_lev
                               cudaStream_t s);
 cudaError_t launch_describe(const Geom& g, int n_frames, FrameSrc src, const uint32_t* selected,
                             const int32_t* sel_counts, const int8_t* pattern, ss_keypoint* kps, uint8_t* desc,
-                            int32_t* counts, cudaStream_t s);
+                            int32_t* counts, uint8_t* samples, cudaStream_t s);  // samples: test hook or NULL
 // The rotated-BRIEF pattern (1024 ints: 256 pairs x 2 points x (x, y)), host copy.
 const int* brief_pattern_host();
 // Row index of the keypoints (first keypoint per (frame, level, row)) + dedup claim reset.
@@ -160,7 +160,7 @@ cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* 
                                 const int32_t* counts, const uint8_t* taken, int n_queries,
                                 const ss_mp_query* q, const uint8_t* qdesc, ss_match_cfg cfg,
                                 unsigned long long* claim, ss_match* out, const uint16_t* rowidx,
-                                cudaStream_t s);
+                                int lanes, cudaStream_t s);  // lanes per query: 0 = chosen per launch
 cudaError_t launch_match_resolve(const Geom& g, int n_queries, const ss_mp_query* q,
                                  const unsigned long long* claim, ss_match* out, cudaStream_t s);
 cudaError_t launch_brute_merge(const Geom& g, int n_frames, const int32_t* counts, int splits,
@@ -204,6 +204,15 @@ cudaError_t launch_stereo_outliers(const Geom& g, int n_pairs, const int32_t* co
 // dynamic shared memory per CTA (keypoint positions + row index), at most 200 KB.
 size_t lastframe_smem_bytes(const Geom& g);
 cudaError_t lastframe_init();  // kernel attributes (ss_create)
+// Kernel attributes (the >48 KB dynamic shared-memory opt-in) of the other kernels.  Attributes
+// are per device, so ss_create sets them on its device every time (cheap; never under capture).
+cudaError_t fast_init();
+cudaError_t distribute_init();
+cudaError_t describe_init();
+cudaError_t pyramid_init();
+cudaError_t brute_tc_init();
+cudaError_t grid_init();
+size_t grid_smem_bytes(const Geom& g);  // dynamic shared memory of the grid top-N kernel
 cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams, const ss_camera* last_cams, float mb,
                              const ss_keypoint* kps, const uint8_t* desc, const int32_t* counts, const uint8_t* taken,
                              const int32_t* pt_off, const ss_frame_point* pts, const uint8_t* pdesc, float th,

@@ -114,13 +114,17 @@ def lib():
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
         L.ss_debug_candidates.argtypes = [P, i32, i32, P, P, P, i32, C.POINTER(i32)]
         L.ss_debug_overflow_count.argtypes = [P, C.POINTER(i32)]
+        L.ss_debug_distribution_paths.argtypes = [P, C.POINTER(i32), C.POINTER(i32)]
+        L.ss_debug_match_lanes.argtypes = [P, i32]
+        L.ss_debug_capture_samples.argtypes = [P, P]
         L.ss_profile_events.argtypes = [P, C.POINTER(P), i32]
         L.ss_debug_phase_times.argtypes = [P, i32, i32, P, i32]
         L.ss_profile_next.argtypes = [P, C.POINTER(i32)]
         for fn in ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_orb_extract", "ss_match_projection",
                    "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_set_distribution",
                    "ss_match_last_frame", "ss_match_brute_partial", "ss_match_brute_merge", "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
-                   "ss_profile_next", "ss_debug_phase_times"):
+                   "ss_profile_next", "ss_debug_phase_times", "ss_debug_distribution_paths", "ss_debug_match_lanes",
+                   "ss_debug_capture_samples"):
             getattr(L, fn).restype = C.c_int
         _lib = L
     return _lib
@@ -129,7 +133,8 @@ def lib():
 EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "ss_orb_extract",
             "ss_match_projection", "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_set_distribution",
             "ss_match_last_frame", "ss_match_brute_partial", "ss_match_brute_merge", "ss_profile_events", "ss_profile_next", "ss_debug_level",
-            "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times")
+            "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times", "ss_debug_distribution_paths",
+            "ss_debug_match_lanes", "ss_debug_capture_samples")
 
 
 def _check(status: int, ctx=None):
@@ -288,6 +293,22 @@ def ss_debug_overflow_count(ctx) -> int:
     n = C.c_int32()
     _check(lib().ss_debug_overflow_count(ctx, C.byref(n)), ctx)
     return n.value
+
+
+def ss_debug_distribution_paths(ctx) -> tuple[int, int]:
+    """(sort fallbacks, global-memory distributions) of the last extract."""
+    a, b = C.c_int32(), C.c_int32()
+    _check(lib().ss_debug_distribution_paths(ctx, C.byref(a), C.byref(b)), ctx)
+    return a.value, b.value
+
+
+def ss_debug_match_lanes(ctx, lanes: int) -> None:
+    _check(lib().ss_debug_match_lanes(ctx, lanes), ctx)
+
+
+def ss_debug_capture_samples(ctx, d_samples) -> None:
+    """d_samples: uint8 CUDA tensor of n_frames * kp_capacity * 512 bytes, or None to stop."""
+    _check(lib().ss_debug_capture_samples(ctx, _ptr(d_samples)), ctx)
 
 
 def window_cfg(th=100, ratio_num=4, ratio_den=5, dedup=1) -> ss_match_cfg:

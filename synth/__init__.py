@@ -7,4 +7,4 @@ and statistics of the paper's workloads (recipe: SURVEY.md §8(d), restated in D
 """
 from .gen import (SHAPES, frame_seed, make_frame, make_frames, make_stereo_pair, make_queries,
                   make_brute_map, flip_bits, make_local_map, INTRINSICS, STEREO_BASELINE, CAMERA_DTYPE,
-                  MAP_POINT_DTYPE, FRAME_POINT_DTYPE, make_last_frame)  # noqa: F401
+                  MAP_POINT_DTYPE, FRAME_POINT_DTYPE, make_last_frame, make_dotted_frame)  # noqa: F401

@@ -353,3 +353,23 @@ def make_last_frame(kps: np.ndarray, desc: np.ndarray, counts: np.ndarray, n_lev
         pdesc[f * Q:(f + 1) * Q] = pd[perm]
     pt_off = (np.arange(F + 1) * Q).astype(np.int32)
     return cams, last, pt_off, pts, pdesc
+
+
+def make_dotted_frame(width: int, height: int, seed: int, n_clusters: int = 12) -> np.ndarray:
+    """Adversarial frame for the quadtree's deep-split path: a flat gray background with
+    isolated bright pixels (each one FAST corner) arranged in clusters whose members sit at
+    distances 3, 5, 9, ..., 129 px from the cluster centre, so the node count keeps growing
+    at every quadtree depth (the kernel's dense-histogram tables stop at depth ~5, and the
+    stop rules then need the sort fallback).  No method arithmetic: only pixel placement."""
+    rng = _rng(seed)
+    img = np.full((height, width), 60, np.uint8)
+    for _ in range(n_clusters):
+        cx, cy = int(rng.integers(40, width - 40)), int(rng.integers(40, height - 40))
+        img[cy, cx] = 200
+        for k in range(1, 8):
+            a = rng.uniform(0, 2 * np.pi)
+            d = 2 ** k + 1
+            x, y = int(cx + d * np.cos(a)), int(cy + d * np.sin(a))
+            if 20 <= x < width - 20 and 20 <= y < height - 20:
+                img[y, x] = 200
+    return img

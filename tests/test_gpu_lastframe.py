@@ -145,6 +145,14 @@ def test_lastframe_chained_gpu_extract(env):
     got = match_records(out)
     pipe.close()
     assert (gc == counts).all() and (gd == desc).all()
+    # exact: the oracle's O13 on the GPU keypoints (GPU angles, <= 1e-4 rad from the oracle's)
+    # takes every rotation-bin decision on the same values as the kernel
+    want_g, wn_g = ref.match_last_frame(p, cams, None, 0.0, gk, desc, counts, None, pt_off, pts, pdesc, th=15.0,
+                                        min_matches=20)
+    assert (got == want_g).all()
+    np.testing.assert_array_equal(nm.cpu().numpy(), wn_g)
+    # and against the oracle's own extraction: identical except where a rotation bin sits within
+    # the angle tolerance of a bin edge
     edge = np.zeros(len(pts), bool)
     for f in range(F):
         for i in range(pt_off[f], pt_off[f + 1]):

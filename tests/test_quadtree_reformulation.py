@@ -279,3 +279,22 @@ def test_dense_fast_path_taken_on_frames(ref):
         got = dense_model(*[a.tolist() if hasattr(a, "tolist") else a for a in args])
         assert got is not None, l  # synthetic frames never need the sort fallback
         assert got == ref.distribute(*args).tolist()
+
+
+def test_dotted_frame_needs_sort_fallback(ref):
+    """The adversarial frame the GPU test uses to drive distribute_kernel into its sort path
+    (tests/test_gpu_coverage.py): its level candidates need quadtree depths beyond the dense
+    tables on several levels, and the sort-path model still equals the oracle there."""
+    p = ref.params(752, 480, 1000)
+    img = synth.make_dotted_frame(752, 480, seed=0)
+    levs = ref.pyramid(p, img)
+    fell = 0
+    for l in range(8):
+        lx, ly, sc = ref.cell_candidates(p, l, ref.fast_M(levs[l]))
+        args = (lx - 16, ly - 16, sc, p.level_w[l] - 32, p.level_h[l] - 32, p.n_per_level[l])
+        lists = [a.tolist() if hasattr(a, "tolist") else a for a in args]
+        want = ref.distribute(*args).tolist()
+        if dense_model(*lists) is None:
+            fell += 1
+        assert gpu_model(*lists) == want, l
+    assert fell >= 3
