@@ -316,7 +316,7 @@ size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int*
 }
 
 cudaError_t fast_init() {  // ss_create, per device; ss_create rejects bands above 227 KB
-  return cudaFuncSetAttribute(fast_bands_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+  return set_max_dynamic_smem(fast_bands_kernel);
 }
 
 cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands, int n_bands,

@@ -175,8 +175,8 @@ size_t grid_smem_bytes(const Geom& g) {
   return (size_t)(2 * GMAX_CELLS + 1) * 4 + (size_t)capmax * 4 + 16;
 }
 
-cudaError_t grid_init() {  // ss_create, per device (ss_set_distribution checks grid_smem_bytes)
-  return cudaFuncSetAttribute(distribute_grid_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+cudaError_t grid_init() {  // ss_create, per device (ss_set_distribution checks grid_smem_bytes vs 200 KB)
+  return set_max_dynamic_smem(distribute_grid_kernel);
 }
 
 cudaError_t launch_distribute_grid(const Geom& g, int n_frames, int level0, int n_levels, const CellInfo* cells,

@@ -832,7 +832,7 @@ ss_status ss_match_last_frame(ss_ctx* c, int32_t n_frames, const ss_camera* d_ca
 ss_status ss_set_distribution(ss_ctx* c, int32_t mode) {
   if (!c) return fail(SS_EINVAL, "NULL ctx");
   if (mode != SS_DIST_QUADTREE && mode != SS_DIST_GRID_TOPN) return fail(SS_EINVAL, "unknown distribution mode");
-  if (mode == SS_DIST_GRID_TOPN && grid_smem_bytes(c->g) > 227 * 1024)
+  if (mode == SS_DIST_GRID_TOPN && grid_smem_bytes(c->g) > 200 * 1024)
     return fail(SS_EUNSUPPORTED, "n_per_level too large for the grid top-N kernel's shared memory");
   if (mode != c->dist_mode) {
     // cached tick graphs were captured with the other distribution's kernels

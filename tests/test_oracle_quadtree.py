@@ -23,6 +23,13 @@ GOLD = os.path.join(os.path.dirname(__file__), "golden")
 #   (10,10),(12,12) together in TL; root 1 sends (60,40)->BL, (70,5)->TL, (90,45)->BR. 4 >= 3:
 #   stop; the 2-key node keeps its max (12,12,9).
 # ex2 (100x100, N=5): both keys land in TL of the single root -> node count 1 == prev: stop.
+# ex3 (64x64, 9 keys in 4 tight clusters of 3/2/2/2, N = 5, 6, 7): nIni = 1; round 1 puts one
+#   cluster in each 32x32 quadrant -> 4 nodes (< N, 4 + 3*4 = 16 > N) -> phase 2.  Its first round
+#   splits each 32x32 node at 16 px, but every cluster lies inside one 16x16 child (TL keys
+#   x,y < 16; TR x in [32,48), y < 16; BL x < 16, y in [32,48); BR x,y >= 48), so each split
+#   yields ONE child: node count 4 == prev -> no-progress stop with 4 outputs for every N.
+#   Kept = each cluster's max score: TL (5,6,9) and (7,5,9) tie -> the smaller rank (5,6);
+#   TR (42,2,7); BL (10,40,6); BR (52,53,8).
 # ex4 (64x64): round 1 gives four 2-key nodes (4 < N, 4+12 > N) -> phase 2 in order
 #   TL (UL 0,0), TR (UL 32,0), BL (UL 0,32), BR (UL 32,32), each split separating its pair.
 def test_hand_worked_cases(ref):

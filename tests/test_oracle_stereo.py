@@ -38,6 +38,36 @@ def test_integer_shift_recovers_disparity(ref, d):
     np.testing.assert_allclose(dp[:n0][good], BF / (uL[good] - ur[:n0][good]), rtol=1e-6)
 
 
+@pytest.mark.parametrize("d", [7, 23, 36])
+def test_integer_shift_on_every_octave(ref, d):
+    """O12 on octaves >= 1: the refinement runs on octave o's level at round(uR0 * invScale)
+    and maps back with scale[o], so a matched level-o keypoint lands within half a level-o
+    pixel (0.5 * scale[o] level-0 px) of uL - d.  Level o of the shifted frame is only
+    approximately shifted (resampling), so the pin asks for >= 90 % of all octave >= 1 matches
+    and >= 80 % on every octave with >= 20 matches; a refinement on the wrong level or with
+    the wrong scale misses by several pixels."""
+    w, h = 752, 480
+    p = ref.params(w, h, 1500)
+    L, R = _pair_shift(w, h, d, seed=100 + d)
+    kl, dl, cl = ref.orb_extract(p, L)
+    kr, dr, cr = ref.orb_extract(p, R)
+    ur, dp, sad = ref.stereo_match(p, L, R, kl, dl, cl, kr, dr, cr, BF, BASE)
+    ok_all = n_all = 0
+    for o in range(1, p.n_levels):
+        a, b = int(cl[o]), int(cl[o + 1])
+        got = ur[a:b] >= 0
+        if not got.any():
+            continue
+        err = np.abs(ur[a:b][got] - (kl["x"][a:b][got] - d))
+        good = err < 0.5 * p.scale[o]
+        ok_all += int(good.sum())
+        n_all += int(got.sum())
+        if got.sum() >= 20:
+            assert good.mean() >= 0.8, (o, good.mean())
+        np.testing.assert_allclose(dp[a:b][got], BF / (kl["x"][a:b][got] - ur[a:b][got]), rtol=1e-6)
+    assert n_all >= 300 and ok_all >= 0.9 * n_all, (ok_all, n_all)
+
+
 def test_invariants_on_warped_pairs(ref):
     w, h = synth.SHAPES["kitti"]
     p = ref.params(w, h, 2000)
