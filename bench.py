@@ -79,6 +79,65 @@ def gather_to_owner(send, rank: int, world: int):
     return None
 
 
+class HostStagedGather:
+    """NCCL-free per-tick result gather (``--backend gloo``): the packed send slot is copied to
+    a pinned host buffer on the gather stream (gated by the tick's completion event), and a
+    host thread runs the gloo gather to rank 0 once that copy has landed -- still off the
+    per-frame critical path.  Lets N > 1 ranks share ONE GPU (NCCL refuses two ranks on a
+    device), so the multi-rank path runs on a 1-GPU box; rank 0 keeps the last gathered slots."""
+
+    def __init__(self, rank: int, world: int, slot_bytes: int, depth: int = 8):
+        import queue
+
+        import torch
+        self.rank, self.world = rank, world
+        self.bufs = [torch.empty(slot_bytes, dtype=torch.uint8).pin_memory() for _ in range(depth)]
+        self.recv = [[torch.empty(slot_bytes, dtype=torch.uint8) for _ in range(world)] for _ in range(depth)]
+        self.events = [torch.cuda.Event() for _ in range(depth)]
+        self.i = 0
+        self.q = queue.Queue(maxsize=depth - 1)
+        self.last = None
+        self.err = None
+        self.t = threading.Thread(target=self._run, daemon=True)
+        self.t.start()
+
+    def _run(self):
+        import torch.distributed as dist
+        while True:
+            item = self.q.get()
+            if item is None:
+                return
+            try:
+                k = item
+                self.events[k].synchronize()
+                if self.rank == 0:
+                    dist.gather(self.bufs[k], self.recv[k], dst=0)
+                    self.last = [r.clone() for r in self.recv[k]]
+                else:
+                    dist.gather(self.bufs[k], None, dst=0)
+            except Exception as e:  # pragma: no cover - surfaced by drain()
+                self.err = e
+
+    def submit(self, send, stream):
+        """Enqueue the D2H copy of `send` on `stream` (already waiting for the tick)."""
+        import torch
+        k = self.i % len(self.bufs)
+        self.i += 1
+        with torch.cuda.stream(stream):
+            self.bufs[k].copy_(send, non_blocking=True)
+            self.events[k].record(stream)
+        self.q.put(k)  # blocks when `depth - 1` gathers are outstanding (buffer reuse)
+
+    def drain(self):
+        import time as _t
+        while not self.q.empty():
+            _t.sleep(0.0005)
+        self.q.put(None)
+        self.t.join()
+        if self.err:
+            raise self.err
+
+
 def window_inputs(p, kps, desc, counts, cfg, seed_lm, seed_lf, per_client):
     """Search-local-points and frame-to-frame inputs of one tick (synth recipes):
     a local map per client frame (left / mono images; O11 + O9) and the previous frame's
@@ -228,13 +287,52 @@ def measured_peaks() -> dict:
 
 
 # ----------------------------------------------------------------------------- algorithmic work
-# Exact FAST-9 score, packed 16x2 formulation: per 4 pixels 14 byte permutes
-# (ring words) + 32 unpacks + 34 biased differences + 2 pairs x 2 polarities x 41 three-way
-# min/max (16 windows of 3, 16 of 9, a 16-way reduction) + 6 to combine = 250 ops -> 62.5/px.
-FAST_OPS_PER_PX = 62.5
-# ALU pipe peak: 148 SMs x 4 SMSPs x 16 lanes x 1.965 GHz (B200_PROFILING / B300_MICROARCH:
-# alu pipe rt = 2 cycles per warp instruction per SMSP) = 18.6 Tops/s
-ALU_PEAK_TOPS = 148 * 64 * 1.965e9 / 1e12
+# FAST-9 work model of SURVEY.md §8(d) (N2+N3 row): >= 32 compares per detect pixel (16 ring
+# pixels x 2 polarities) + the contiguity test ~= 40 integer ops per detect pixel.  (The
+# kernel's own exact-score formulation issues ~52 ALU-pipe ops per pixel: DESIGN.md §5.)
+FAST_OPS_PER_PX = 40.0
+FAST_KERNEL_OPS_PER_PX = 51.5
+# Hamming distance of two 256-bit descriptors: 8 POPC (XU pipe) per candidate (O9 / O13)
+POPC_PER_DISTANCE = 8
+
+
+def int_peaks() -> dict:
+    """Measured issue rates per SM per clock (profiles/peaks_int_r02.json, scripts/micro/int_peaks.cu)."""
+    path = os.path.join(ROOT, "profiles", "peaks_int_r02.json")
+    try:
+        with open(path) as f:
+            pk = json.load(f)["peaks"]
+        return {"alu": float(pk["alu_pipe_thread_ops_per_clk_per_sm"]),
+                "popc": float(pk["xu_popc_thread_ops_per_clk_per_sm"]),
+                "src": "measured: profiles/peaks_int_r02.json (scripts/micro/int_peaks.cu on a B200)"}
+    except Exception:
+        return {"alu": 64.0, "popc": 16.0, "src": "fallback: CUDA guide rates (profiles/peaks_int_r02.json missing)"}
+
+
+def window_candidates(kps, counts, taken, queries, n_levels: int, max_q: int = 20000) -> tuple[int, int]:
+    """(candidate distances evaluated, queries sampled) of O9 for the first max_q queries: keypoints of
+    the query's frame on levels [pl-1, pl] with |x-u| < r and |y-v| < r (f32) that are not taken --
+    exactly the pairs whose Hamming distance the matcher computes (8 POPC each)."""
+    q = queries[:max_q]
+    total = 0
+    for f in np.unique(q["frame"]):
+        if f < 0 or f >= kps.shape[0]:
+            continue
+        qq = q[q["frame"] == f]
+        n = int(counts[f][-1])
+        k = kps[f][:n]
+        ok = taken[f][:n] == 0 if taken is not None else np.ones(n, bool)
+        x, y, lev = k["x"][ok], k["y"][ok], k["level"][ok].astype(np.int32)
+        for i0 in range(0, len(qq), 2048):
+            b = qq[i0:i0 + 2048]
+            r = b["radius"][:, None]
+            dx = np.abs(np.float32(x)[None, :] - b["u"][:, None])
+            dy = np.abs(np.float32(y)[None, :] - b["v"][:, None])
+            gate = (lev[None, :] >= (b["pred_level"][:, None] - 1)) & (lev[None, :] <= b["pred_level"][:, None])
+            total += int(((dx < r) & (dy < r) & gate).sum())
+    return total, len(q)
+
+
 def kernel_work(name: str, p, B: int, cand_l: list, kps_l: list, nq: int, n_map: int, nlf: int = 0) -> tuple[str, float]:
     """(bound, algorithmic bytes or work) per launch -- DESIGN.md §6 work model.
     cand_l / kps_l: candidates / kept keypoints per level summed over the batch."""
@@ -263,9 +361,9 @@ def kernel_work(name: str, p, B: int, cand_l: list, kps_l: list, nq: int, n_map:
         return "hbm", float(nq * 12)
     if name == "brute_tc":  # s8 +-1 dot products on tcgen05: 2 x 256 ops per distance
         return "tensor", float(sum(kps_l)) * n_map * 512.0
-    if name == "brute_expand":  # packed descriptors read (32 B/row), expanded s8 rows written (256 B/row)
+    if name == "brute_expand":  # the tick's keypoints only (the map was prepared once): 32 B read, 256 B written
         slots = B * p.kp_capacity
-        return "hbm", float((slots + n_map) * (32 + 256))
+        return "hbm", float(slots * (32 + 256))
     return "hbm", 0.0
 
 
@@ -279,11 +377,17 @@ def run_ours(args, cfg):
 
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
-    local = int(os.environ.get("LOCAL_RANK", 0))
+    local = 0 if args.same_device else int(os.environ.get("LOCAL_RANK", 0))
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    backend = args.backend
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
+    if args.clients:
+        cfg = dict(cfg, clients=args.clients)
     w, h = synth.SHAPES[cfg["shape"]]
     clients = client_ids(rank, world, cfg["clients"])
     per_client = 2 if cfg.get("stereo") else 1
@@ -357,10 +461,18 @@ def run_ours(args, cfg):
                                   n_from_kps=int(0.4 * cfg["map"]))
         map_desc = torch.from_numpy(mp).to(dev)
         if world > 1:
-            dist.broadcast(map_desc, src=0)
+            if backend == "nccl":
+                dist.broadcast(map_desc, src=0)
+            else:
+                mh = map_desc.cpu()
+                dist.broadcast(mh, src=0)
+                map_desc = mh.to(dev)
         if args.map_shard:  # F4: keep only this rank's rows (global index offset lo)
             shard_lo, shard_hi = shard_range(cfg["map"], rank, world)
             map_desc = map_desc[shard_lo:shard_hi].contiguous()
+        # the shared map is server state: expanded into each context's tensor-core operand
+        # layout once (ss_brute_map_prepare); every tick then expands only its keypoints
+        pipe.prepare_map(map_desc, stream=stream)
         q_host = None
     torch.cuda.synchronize(dev)
 
@@ -396,6 +508,8 @@ def run_ours(args, cfg):
                                   max_map=cfg["map"], device=local) for _ in range(P - 1)]
     for pp in pipes:
         pp.set_distribution(dist_mode)
+        if not window and pp is not pipe:
+            pp.prepare_map(map_desc)
     outs = [out] + [torch.zeros_like(out) for _ in range(P - 1)]
     qbufs = [torch.zeros((max(Q, 1), 20), dtype=torch.uint8, device=dev) for _ in range(P)]  # projected queries
     lf_out = [torch.zeros((max(NLF, 1), 3), dtype=torch.int32, device=dev) for _ in range(P)]
@@ -412,8 +526,8 @@ def run_ours(args, cfg):
                 qd, qc = allgather_queries(pp.desc[:B], pp.counts[:B], world)
             else:
                 qd, qc = pp.desc[:B], pp.counts[:B]
-            ss.ss_match_brute_partial(pp.ctx, B * world, qd, qc, map_desc, map_desc.shape[0], shard_lo, top2_all[q],
-                                      st)
+            ss.ss_match_brute_partial(pp.ctx, B * world, qd, qc, None, map_desc.shape[0], shard_lo, top2_all[q],
+                                      st)  # the prepared shard
             parts = exchange_partials(top2_all[q], world) if world > 1 else top2_all[q]
             ss.ss_match_brute_merge(pp.ctx, B, pp.counts[:B], world, parts, bcfg, outs[q], st)
 
@@ -460,7 +574,7 @@ def run_ours(args, cfg):
                 if not eager_tail:
                     sharded_tail(q, st)
             else:
-                pp.match_brute(B, map_desc, ot, stream=st)
+                pp.match_brute(B, None, ot, stream=st)  # the prepared shared map
         if prof:
             assert ss.ss_profile_next(pp.ctx) == n_ev, (ss.ss_profile_next(pp.ctx), n_ev)
             ss.ss_profile_events(pp.ctx, [])
@@ -472,14 +586,26 @@ def run_ours(args, cfg):
 
     # --- optional gather of per-frame results to rank 0 (map owner), off the critical path
     gather_stream = torch.cuda.Stream(dev) if world > 1 else None
+    if eager_tail and backend != "nccl":
+        raise SystemExit("--map-shard over N > 1 ranks needs --backend nccl")
+
+    def tick_parts(q):
+        pp = pipes[q]
+        return [pp.kps[:B], pp.desc[:B], pp.counts[:B], outs[q]] + ([lf_out[q], lf_n[q]] if window else [])
+
+    staged = None
+    if world > 1 and backend != "nccl":
+        staged = HostStagedGather(rank, world, sum(t.numel() * t.element_size() for t in tick_parts(0)))
 
     def gather_step(done_ev, q):
         # side stream: waits for the tick, packs its results and gathers them to rank 0
         gather_stream.wait_event(done_ev)
         with torch.cuda.stream(gather_stream):
-            pp = pipes[q]
-            parts = [pp.kps[:B], pp.desc[:B], pp.counts[:B], outs[q]] + ([lf_out[q], lf_n[q]] if window else [])
-            gather_to_owner(pack_results(parts), rank, world)
+            send = pack_results(tick_parts(q))
+            if staged is not None:
+                staged.submit(send, gather_stream)
+            else:
+                gather_to_owner(send, rank, world)
 
     W_, K = args.warmup, args.steps
     ev_start = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
@@ -520,13 +646,31 @@ def run_ours(args, cfg):
         torch.cuda.synchronize(dev)
         if gather_stream is not None:
             gather_stream.synchronize()
+    if staged is None and args.dump_gather:  # single rank: its own last slot
+        np.save(f"{args.dump_gather}.rank{rank}.npy", pack_results(tick_parts((W_ + K - 1) % P)).cpu().numpy())
+    if staged is not None:
+        staged.drain()
+        if args.dump_gather:  # the last tick's slots: rank 0 gathered, every rank its own
+            last_q = (W_ + K - 1) % P
+            own = pack_results(tick_parts(last_q)).cpu().numpy()
+            np.save(f"{args.dump_gather}.rank{rank}.npy", own)
+            if rank == 0:
+                np.save(f"{args.dump_gather}.gathered.npy", np.stack([t_.numpy() for t_ in staged.last]))
     if world > 1:
         dist.barrier()
     T_ms = t0.elapsed_time(t1)
     step_ms = [ev_start[i].elapsed_time(ev_end[i]) for i in range(K)]
+    # steady state: ticks completed between the end of step P and the end of step K (the
+    # pipeline is full; excludes the ramp-up of the first P ticks in flight)
+    steady = None
+    if K > P + 1:
+        sw = ev_end[P - 1].elapsed_time(ev_end[K - 1])
+        if sw > 0:
+            steady = {"value": B * world * (K - P) / (sw / 1000.0), "unit": "frames/s",
+                      "window": f"end of step {P} to end of step {K} ({K - P} ticks, {P} in flight)"}
     T_max = T_ms
     if world > 1:
-        tt = torch.tensor([T_ms], device=dev)
+        tt = torch.tensor([T_ms], device=dev if backend == "nccl" else "cpu")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         T_max = float(tt.item())
 
@@ -558,6 +702,18 @@ def run_ours(args, cfg):
     avg_us = {n: 1000.0 * float(np.mean(v)) for n, v in per_kernel.items()}
 
     # --- work model for the roofline of the dominant kernel
+    win_sample = None
+    if window:  # one tick (ring slot 0) run eagerly to read back what the matcher sees
+        with torch.cuda.stream(stream):
+            pipe.extract(frames[0], stream=stream)
+            pipe.match_last_frame(B, cams[0], lf_off[0], lf_pts[0], lf_desc[0], lf_out[0], lf_n[0],
+                                  last_cams=lf_last[0] if MB > 0 else None, mb=MB, th=cfg["lf_th"], min_matches=20,
+                                  taken=taken[0], matched=lf_mask[0], stream=stream)
+            pipe.project(B, cams[0], points[0], point_frame[0], qbufs[0], th=cfg["th"], stream=stream)
+        stream.synchronize()
+        k0, _, c0 = pipe.results(B)
+        qrec = qbufs[0].cpu().numpy().reshape(-1).view(ss.QUERY_DTYPE)
+        win_sample = (k0, c0, lf_mask[0].cpu().numpy(), qrec)
     kps_h, desc_h, counts_h = pipe.results(B)  # last step's outputs
     kps_l = [int((counts_h[:, l + 1] - counts_h[:, l]).sum()) for l in range(L)]
     cand_l = [sum(len(ss.ss_debug_candidates(pipe.ctx, b, l)[0]) for b in range(B)) for l in range(L)]
@@ -571,6 +727,12 @@ def run_ours(args, cfg):
         per_func.setdefault(func_of.get(n_, n_), []).append(n_)
     peaks = measured_peaks()
     prof_step_us = 1000.0 * float(np.mean(prof_step_ms))
+    ipk = int_peaks()
+    n_sm = props.multi_processor_count
+    clk = sampler.summary()
+    clk_mhz = float(clk.get("sm_mhz") or clk.get("sm_max_mhz") or 1965.0)
+    alu_peak_tops = ipk["alu"] * n_sm * clk_mhz * 1e6 / 1e12
+    popc_peak_tops = ipk["popc"] * n_sm * clk_mhz * 1e6 / 1e12
 
     def roof_of(func):
         members = per_func[func]
@@ -586,10 +748,12 @@ def run_ours(args, cfg):
                              "peak_src": peaks["src"], "share_of_step": share}
         if bound == "alu":
             achieved = work / (us * 1e-6) / 1e12
-            return members, {"bound": "alu", "achieved": achieved, "peak": ALU_PEAK_TOPS, "unit": "Tops/s",
-                             "frac": achieved / ALU_PEAK_TOPS, "traffic": None, "kernel": name,
-                             "peak_src": "derived: 148 SM x 64 ALU lanes/clk x 1.965 GHz (DESIGN.md §6)",
-                             "work": f"{FAST_OPS_PER_PX} ops per detect pixel", "share_of_step": share}
+            return members, {"bound": "alu", "achieved": achieved, "peak": alu_peak_tops, "unit": "Tops/s",
+                             "frac": achieved / alu_peak_tops, "traffic": None, "kernel": name,
+                             "peak_src": f"{ipk['src']}: {ipk['alu']:.0f} ALU-pipe ops/clk/SM x {n_sm} SMs x "
+                                         f"{clk_mhz:.0f} MHz (SM clock under load in this run)",
+                             "work": f"{FAST_OPS_PER_PX:g} int ops per detect pixel (SURVEY.md §8(d)); the kernel "
+                                     f"issues ~{FAST_KERNEL_OPS_PER_PX:g}", "share_of_step": share}
         # tensor: int8 dense peak = measured bf16 dense x 2 (the guide's nominal i8 : bf16 ratio)
         achieved = work / (us * 1e-6) / 1e12
         return members, {"bound": "tensor", "achieved": achieved, "peak": peaks["i8_tops"], "unit": "TOPS",
@@ -605,6 +769,20 @@ def run_ours(args, cfg):
     for f_ in sorted(per_func, key=lambda f_: -sum(avg_us[n_] for n_ in per_func[f_])):
         r_ = roof_of(f_)[1]
         rooflines.append({k_: r_[k_] for k_ in ("kernel", "bound", "achieved", "unit", "frac", "share_of_step")})
+    # integer-pipe (POPC) utilisation of the Hamming matcher (north_star): 8 POPC per candidate
+    # distance it evaluates, counted exactly on a tick's inputs (a sample of its queries)
+    if window and "match_window" in avg_us:
+        pairs, nsamp = window_candidates(*win_sample, L)
+        ops = POPC_PER_DISTANCE * pairs * (Q / max(nsamp, 1))
+        ach = ops / (avg_us["match_window"] * 1e-6) / 1e12
+        popc = {"kernel": "match_window", "bound": "popc (XU pipe)", "achieved": ach, "peak": popc_peak_tops,
+                "unit": "Tops/s", "frac": ach / popc_peak_tops,
+                "work": f"{POPC_PER_DISTANCE} POPC per candidate distance; {pairs} candidates in {nsamp} sampled "
+                        f"queries of {Q} ({pairs / max(nsamp, 1):.2f} per query)",
+                "peak_src": f"{ipk['src']}: {ipk['popc']:.0f} POPC/clk/SM x {n_sm} SMs x {clk_mhz:.0f} MHz"}
+        for r_ in rooflines:
+            if r_["kernel"] == "match_window":
+                r_["popc"] = popc
     traffic_file = os.path.join(ROOT, "profiles", "dram_traffic_r01.json")
     if os.path.exists(traffic_file):
         try:
@@ -638,6 +816,8 @@ def run_ours(args, cfg):
                                  device=local) for _ in range(Pe)]
         for pp in e2e_pipes:
             pp.set_distribution(dist_mode)
+            if not window:
+                pp.prepare_map(map_desc)
         e2e_streams = [torch.cuda.Stream(dev) for _ in range(Pe)]
         e2e = run_e2e(args, e2e_pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, e2e_streams,
                       th=cfg["th"], stereo=(BF, BASE_M, st_out) if stereo else None, lf=(MB, cfg.get("lf_th", 15.0)),
@@ -657,13 +837,16 @@ def run_ours(args, cfg):
         "config": {"workload": cfg["desc"], "config": args.config, "frames_per_step": frames_per_step,
                    "images_per_step_per_gpu": B, "features_per_image": cfg["nf"],
                    "map_points_per_step_per_gpu": Q if window else 0, "map_size": cfg["map"],
-                   "parallelism": f"dp{world} (clients sharded over GPUs)",
+                   "parallelism": f"dp{world} (clients sharded over GPUs)" +
+                                  (f"; result gather over {backend}" if world > 1 else "") +
+                                  ("; all ranks on one GPU (--same-device)" if args.same_device and world > 1 else ""),
                    "l2": f"inputs ring of {n_slots} distinct slots = {n_slots * slot_bytes / 2**20:.0f} MiB "
                          f"> L2 {l2 / 2**20:.0f} MiB (no flush)",
                    "cuda_graphs": True, "ticks_in_flight": P, "setup_s": round(setup_s, 1),
                    "distribution": "grid top-N (O4g)" if args.dist == "grid" else "quadtree (O4)",
                    "map": ("sharded over ranks (F4: shard top-2 for all ranks' frames, all-to-all, merge)"
                            if shard else ("replicated" if not window else None))},
+        "steady_state": steady,
         "latency_ms": {"p50": float(np.percentile(step_ms, 50)), "p99": float(np.percentile(step_ms, 99)),
                        "samples": len(step_ms),
                        "note": f"per-frame latency = its tick's device time from start to end on its stream "
@@ -756,8 +939,8 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
                     io.lf_offsets, io.lf_points, io.lf_desc = off.data_ptr(), lp.data_ptr(), ld.data_ptr()
                     io.last_cams, io.mb, io.lf_th, io.lf_min_matches = last.data_ptr(), lf[0], lf[1], 20
                     io.lf_matches, io.lf_n_matches = o["lf_matches"].data_ptr(), o["lf_n"].data_ptr()
-                else:
-                    io.d_map_desc, io.n_map = map_desc.data_ptr(), map_desc.shape[0]
+                else:  # the map prepared on each context (ss_brute_map_prepare): io.d_map_desc = NULL
+                    io.d_map_desc, io.n_map = None, map_desc.shape[0]
                 io.kps, io.desc, io.counts = o["kps"].data_ptr(), o["desc"].data_ptr(), o["counts"].data_ptr()
                 io.matches = o["matches"].data_ptr()
                 if stereo:
@@ -1009,6 +1192,11 @@ def main(argv=None):
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--map-shard", action="store_true",
                     help="brute configs: partition the map over the ranks (F4: shard top-2, all-to-all, merge)")
+    ap.add_argument("--backend", choices=["nccl", "gloo"], default="nccl",
+                    help="N > 1: NCCL gather on a side stream, or gloo with host-staged slots (ranks may share a GPU)")
+    ap.add_argument("--same-device", action="store_true", help="every rank on cuda:0 (multi-rank test on one GPU)")
+    ap.add_argument("--clients", type=int, default=0, help="override the config's clients per rank")
+    ap.add_argument("--dump-gather", default="", help="write the last tick's gathered / own slots to PATH.*.npy")
     ap.add_argument("--dist", choices=["quadtree", "grid"], default="quadtree",
                     help="keypoint distribution: ORB-SLAM quadtree (O4) or grid top-N (O4g)")
     args = ap.parse_args(argv)

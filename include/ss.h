@@ -162,9 +162,12 @@ ss_status ss_orb_extract(ss_ctx* ctx, int32_t n_frames, const uint8_t* d_frames,
  *   [pred_level-1, pred_level], |x-u| < r and |y-v| < r (f32), not taken; top-2 by
  *   (distance, index); accepted as in ss_match_cfg; queries with an out-of-range frame
  *   get {-1, 256, 256}.
- * BRUTE: d_kp_taken and d_queries ignored (n_queries must be 0); d_map_desc [n_map][32];
- *   d_out [n_frames][kp_capacity]: per keypoint, top-2 over the map by (distance, index);
- *   slots >= the frame's count get {-1, 256, 256}. */
+ * BRUTE: d_kp_taken and d_queries ignored (n_queries must be 0); d_map_desc [n_map][32], or
+ *   NULL to use the map prepared by ss_brute_map_prepare (its n_map must equal the prepared
+ *   row count, else SS_EINVAL); d_out [n_frames][kp_capacity]: per keypoint, top-2 over the
+ *   map by (distance, index); slots >= the frame's count get {-1, 256, 256}; n_map = 0 (an
+ *   empty map) gives {-1, 256, 256} everywhere.  A non-NULL d_map_desc overwrites (forgets)
+ *   the prepared map. */
 ss_status ss_match_projection(ss_ctx* ctx, int32_t n_frames, const ss_keypoint* d_kps,
                               const uint8_t* d_desc, const int32_t* d_counts,
                               const uint8_t* d_kp_taken, int32_t n_queries,
@@ -190,6 +193,16 @@ ss_status ss_match_brute_partial(ss_ctx* ctx, int32_t n_frames, const uint8_t* d
                                  ss_stream_t stream);
 ss_status ss_match_brute_merge(ss_ctx* ctx, int32_t n_frames, const int32_t* d_counts, int32_t n_parts,
                                const uint64_t* d_parts, const ss_match_cfg* cfg, ss_match* d_out, ss_stream_t stream);
+
+/* BRUTE map preparation (O10; the shared map of C5 is server state that changes rarely):
+ * enqueues on `stream` the one-time expansion of d_map_desc [n_map][32] (DEVICE) into the
+ * ctx's tensor-core operand scratch (s8 +-1 rows in the UMMA K-major layout, 256 B per row),
+ * so BRUTE calls with d_map_desc = NULL and the same n_map (ss_match_projection,
+ * ss_match_brute_partial, ss_track_tick's io->d_map_desc) expand only their keypoints.  The
+ * prepared copy is a snapshot: after changing the map's contents, call again.  Any BRUTE call
+ * with a non-NULL map replaces the scratch and forgets the preparation.  SS_EINVAL for
+ * n_map < 1 or a NULL map, SS_ECAPACITY for n_map > max_map. */
+ss_status ss_brute_map_prepare(ss_ctx* ctx, const uint8_t* d_map_desc, int32_t n_map, ss_stream_t stream);
 
 /* O11: the per-map-point half of "search local points" (ORB-SLAM3
  * Frame::isInFrustum + MapPoint::PredictScale + ORBmatcher::RadiusByViewingCos): map point
@@ -305,7 +318,8 @@ typedef struct {
   const uint8_t* point_desc;
   const uint8_t* taken;
   float th;
-  /* BRUTE (O10): a DEVICE-resident map [n_map][32] (a shared map is uploaded once) */
+  /* BRUTE (O10): a DEVICE-resident map [n_map][32] (a shared map is uploaded once), or NULL
+   * for the map prepared on this ctx by ss_brute_map_prepare */
   const uint8_t* d_map_desc;
   int32_t n_map;
   /* outputs: kps [n_frames][kp_capacity], desc [n_frames][kp_capacity][32], counts

@@ -413,9 +413,12 @@ int brute_tc_splits(int n_slots, int n_map, int max_splits, int n_sm) {
 
 cudaError_t launch_brute_expand(int n_slots, const uint8_t* desc, int n_map, const uint8_t* map_desc, int8_t* qexp,
                                 int8_t* mexp, cudaStream_t s) {
-  if (n_slots <= 0 || n_map <= 0) return cudaSuccess;
-  const int pairs = (n_slots + TC_ROWS - 1) / TC_ROWS;
-  const int tiles = (n_map + TC_NT - 1) / TC_NT;
+  // either part may be skipped: desc == NULL (map only: ss_brute_map_prepare) or map_desc ==
+  // NULL (keypoints only: the map was prepared once)
+  const bool doq = desc != nullptr && n_slots > 0, dom = map_desc != nullptr && n_map > 0;
+  if (!doq && !dom) return cudaSuccess;
+  const int pairs = doq ? (n_slots + TC_ROWS - 1) / TC_ROWS : 0;
+  const int tiles = dom ? (n_map + TC_NT - 1) / TC_NT : 0;
   const int64_t q_units = (int64_t)pairs * TC_ROWS * 16, m_units = (int64_t)tiles * TC_NT * 16;
   const int64_t units = q_units + m_units;
   const int blocks = (int)std::min<int64_t>((units + 255) / 256, 148 * 16);

@@ -6,11 +6,13 @@
 // of one frame (the cells of a row share their detect rows and their detect windows tile
 // [x0, x1) without gaps):
 //  1. stage the band + ring halo in shared memory with 16-byte coalesced loads;
-//  2. the score M of EVERY band pixel, four horizontally adjacent pixels per thread: the 16
-//     ring values of the 4 pixels are 16 byte-permutes of a sliding 7-row x 3-word register
-//     window (3 shared loads per row step), unpacked into two 16x2 lanes, and the cyclic
-//     min/max over the 16 arcs of 9 runs on DPX three-way min/max (VIMNMX3.U16x2) -- no
-//     pre-test, no divergence, one 32-bit store of 4 scores;
+//  2. the score M of EVERY band pixel, four horizontally adjacent pixels per thread: the band
+//     is staged as I - 128 (bytes XOR 0x80); each ring value PAIR of pixels (0, 2) or (1, 3)
+//     is one sign-replicating byte permute of a sliding 7-row x 3-word register window (3
+//     shared loads per row step) into two signed 16-bit lanes, and the cyclic min / max over
+//     the 16 arcs of 9 of the RAW ring values runs on DPX three-way min/max (VIMNMX3.S16x2);
+//     the centre enters only at the end (min_k (c - r_k) = c - max_k r_k) -- no pre-test, no
+//     divergence, one 32-bit store of 4 scores;
 //  3. one warp per cell, one lane per cell row: strict 8-neighbour maxima inside the cell's
 //     window (neighbours in the next cell are ignored: per-cell ROI semantics), four columns
 //     per step as 16x2 three-way max trees over cell-masked neighbour words, as 64-bit row
@@ -18,6 +20,7 @@
 //     survivors written in raster order (warp prefix sum of the row counts).
 //
 //   M(p) = max_s max( min_{k<9} d_{s+k}, min_{k<9} -d_{s+k} ),  d_k = I(p) - I(p + R_k)
+//        = max( I(p) - min_s max_{k<9} I(p + R_{s+k}),  max_s min_{k<9} I(p + R_{s+k}) - I(p) )
 //   corner at t <=> M > t (stored clamped to >= 0; scores <= minTh can neither be candidates
 //   nor suppress one, so no thresholding is needed before the NMS).
 #include "ss_internal.h"
@@ -30,67 +33,98 @@ constexpr int FB_WARPS = 8;
 constexpr int FB_THREADS = FB_WARPS * 32;
 constexpr int ROWS_PER_TASK = 8;
 
-__device__ __forceinline__ uint32_t lo_pair(uint32_t w) { return __byte_perm(w, 0, 0x7270); }  // bytes 0, 2
-__device__ __forceinline__ uint32_t hi_pair(uint32_t w) { return __byte_perm(w, 0, 0x7371); }  // bytes 1, 3
-
-// Cyclic arc min/max of one 16x2 pair of pixels.  d[k] = c - r_k + 256 (both lanes).
-// Returns max(max_s min9 d, 512 - min_s max9 d) clamped to >= 256, i.e. M + 256 >= 256.
-__device__ __forceinline__ uint32_t arc_score2(const uint32_t (&d)[16]) {
+// The band is staged with every byte XOR 0x80, so a byte read as a signed char is I - 128
+// (order preserving).  A PRMT whose selector nibbles set the sign-replicate bit turns two
+// bytes of a 64-bit window straight into two signed 16-bit lanes, so every ring value of a
+// pixel pair is ONE byte permute of the row's words (no separate unpack and no subtraction).
+//
+// For a pair of pixels (16x2 lanes, values v = I - 128) with ring values r[0..15] and
+// centre c, using min_k (c - r_k) = c - max_k r_k and min_k (r_k - c) = min_k r_k - c:
+//   M = max( max_s min9(r)[s] - c,  c - min_s max9(r)[s],  0 ).
+// Returns M + 256 in both lanes (the low byte of each lane is M).
+__device__ __forceinline__ uint32_t arc_score2(const uint32_t (&r)[16], uint32_t c) {
   uint32_t mn3[16], mx3[16];
 #pragma unroll
   for (int k = 0; k < 16; k++) {
-    mn3[k] = __vimin3_u16x2(d[k], d[(k + 1) & 15], d[(k + 2) & 15]);
-    mx3[k] = __vimax3_u16x2(d[k], d[(k + 1) & 15], d[(k + 2) & 15]);
+    mn3[k] = __vimin3_s16x2(r[k], r[(k + 1) & 15], r[(k + 2) & 15]);
+    mx3[k] = __vimax3_s16x2(r[k], r[(k + 1) & 15], r[(k + 2) & 15]);
   }
   uint32_t mn9[16], mx9[16];
 #pragma unroll
   for (int s = 0; s < 16; s++) {
-    mn9[s] = __vimin3_u16x2(mn3[s], mn3[(s + 3) & 15], mn3[(s + 6) & 15]);
-    mx9[s] = __vimax3_u16x2(mx3[s], mx3[(s + 3) & 15], mx3[(s + 6) & 15]);
+    mn9[s] = __vimin3_s16x2(mn3[s], mn3[(s + 3) & 15], mn3[(s + 6) & 15]);
+    mx9[s] = __vimax3_s16x2(mx3[s], mx3[(s + 3) & 15], mx3[(s + 6) & 15]);
   }
-  const uint32_t a1 = __vimax3_u16x2(__vimax3_u16x2(mn9[0], mn9[1], mn9[2]), __vimax3_u16x2(mn9[3], mn9[4], mn9[5]),
-                                     __vimax3_u16x2(mn9[6], mn9[7], mn9[8]));
-  const uint32_t a2 = __vimax3_u16x2(__vimax3_u16x2(mn9[9], mn9[10], mn9[11]),
-                                     __vimax3_u16x2(mn9[12], mn9[13], mn9[14]), mn9[15]);
-  const uint32_t z1 = __vimin3_u16x2(__vimin3_u16x2(mx9[0], mx9[1], mx9[2]), __vimin3_u16x2(mx9[3], mx9[4], mx9[5]),
-                                     __vimin3_u16x2(mx9[6], mx9[7], mx9[8]));
-  const uint32_t z2 = __vimin3_u16x2(__vimin3_u16x2(mx9[9], mx9[10], mx9[11]),
-                                     __vimin3_u16x2(mx9[12], mx9[13], mx9[14]), mx9[15]);
-  const uint32_t maxmin = __vimax3_u16x2(a1, a2, a2);                 // max_s min9(d) + 256 (dark ring)
-  const uint32_t minmax = __vimin3_u16x2(z1, z2, z2);                 // min_s max9(d) + 256 (bright ring)
-  return __vimax3_u16x2(maxmin, 0x02000200u - minmax, 0x01000100u);  // max(.., 256 + max(0, ..))
+  const uint32_t a1 = __vimax3_s16x2(__vimax3_s16x2(mn9[0], mn9[1], mn9[2]), __vimax3_s16x2(mn9[3], mn9[4], mn9[5]),
+                                     __vimax3_s16x2(mn9[6], mn9[7], mn9[8]));
+  const uint32_t a2 = __vimax3_s16x2(__vimax3_s16x2(mn9[9], mn9[10], mn9[11]),
+                                     __vimax3_s16x2(mn9[12], mn9[13], mn9[14]), mn9[15]);
+  const uint32_t z1 = __vimin3_s16x2(__vimin3_s16x2(mx9[0], mx9[1], mx9[2]), __vimin3_s16x2(mx9[3], mx9[4], mx9[5]),
+                                     __vimin3_s16x2(mx9[6], mx9[7], mx9[8]));
+  const uint32_t z2 = __vimin3_s16x2(__vimin3_s16x2(mx9[9], mx9[10], mx9[11]),
+                                     __vimin3_s16x2(mx9[12], mx9[13], mx9[14]), mx9[15]);
+  // to offset-binary (s16 + 32768, order preserving) so the differences below are lane-local:
+  // (x + 32768) + 256 - (y + 32768) = x - y + 256 in [1, 511], never borrowing across lanes
+  const uint32_t maxmin = __vimax3_s16x2(a1, a2, a2) ^ 0x80008000u;  // max_s min9(r)
+  const uint32_t minmax = __vimin3_s16x2(z1, z2, z2) ^ 0x80008000u;  // min_s max9(r)
+  const uint32_t cb = c ^ 0x80008000u;
+  const uint32_t bright = maxmin + 0x01000100u - cb;                 // 256 + max_s min9(r) - c
+  const uint32_t dark = cb + 0x01000100u - minmax;                   // 256 + c - min_s max9(r)
+  return __vimax3_u16x2(bright, dark, 0x01000100u);
+}
+
+// Sign-replicating byte-permute selector: lanes = bytes (i, j) of the 8-byte window {b:a},
+// each sign-extended to 16 bits.
+__host__ __device__ constexpr uint32_t sx_sel(int i, int j) {
+  return (uint32_t)i | (uint32_t)(i | 8) << 4 | (uint32_t)j << 8 | (uint32_t)(j | 8) << 12;
+}
+// PTX prmt: a selector nibble with bit 3 set replicates the sign of the selected byte (the
+// __byte_perm intrinsic masks bit 3 away, so this is inline PTX)
+template <uint32_t SEL>
+__device__ __forceinline__ uint32_t prmt_sx(uint32_t a, uint32_t b) {
+  uint32_t r;
+  asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "n"(SEL));
+  return r;
+}
+
+// Ring value pair of ring offset dx for pixels (q, q + 2) (q = 0: pixels 0, 2; q = 1: 1, 3)
+// from one row's words w0..w2 (bytes 0..11 <-> columns gx-4 .. gx+7): bytes 4+q+dx, 6+q+dx.
+template <int Q, int DX>
+__device__ __forceinline__ uint32_t ring_pair(uint32_t w0, uint32_t w1, uint32_t w2) {
+  constexpr int b = 4 + Q + DX;  // first byte, 1..8
+  if constexpr (b <= 3) return prmt_sx<sx_sel(b, b + 2)>(w0, w1);
+  else if constexpr (b <= 7) return prmt_sx<sx_sel(b - 4, b - 2)>(w1, w2);
+  else return prmt_sx<sx_sel(b - 8, b - 6)>(w2, w2);
 }
 
 // M of 4 horizontally adjacent pixels from the 7-row window W[dy + 3][0..2] (columns
-// gx-4 .. gx+7 of rows y-3 .. y+3), packed as 4 bytes (pixel i in byte i).
+// gx-4 .. gx+7 of rows y-3 .. y+3, bytes XOR 0x80), packed as 4 bytes (pixel i in byte i).
+template <int Q>
+__device__ __forceinline__ uint32_t fast_M2(const uint32_t (&W)[7][3]) {
+  uint32_t r[16];
+  // OpenCV offsets16 order: (dx, dy)
+  r[0] = ring_pair<Q, 0>(W[6][0], W[6][1], W[6][2]);    // ( 0, 3)
+  r[1] = ring_pair<Q, 1>(W[6][0], W[6][1], W[6][2]);    // ( 1, 3)
+  r[2] = ring_pair<Q, 2>(W[5][0], W[5][1], W[5][2]);    // ( 2, 2)
+  r[3] = ring_pair<Q, 3>(W[4][0], W[4][1], W[4][2]);    // ( 3, 1)
+  r[4] = ring_pair<Q, 3>(W[3][0], W[3][1], W[3][2]);    // ( 3, 0)
+  r[5] = ring_pair<Q, 3>(W[2][0], W[2][1], W[2][2]);    // ( 3,-1)
+  r[6] = ring_pair<Q, 2>(W[1][0], W[1][1], W[1][2]);    // ( 2,-2)
+  r[7] = ring_pair<Q, 1>(W[0][0], W[0][1], W[0][2]);    // ( 1,-3)
+  r[8] = ring_pair<Q, 0>(W[0][0], W[0][1], W[0][2]);    // ( 0,-3)
+  r[9] = ring_pair<Q, -1>(W[0][0], W[0][1], W[0][2]);   // (-1,-3)
+  r[10] = ring_pair<Q, -2>(W[1][0], W[1][1], W[1][2]);  // (-2,-2)
+  r[11] = ring_pair<Q, -3>(W[2][0], W[2][1], W[2][2]);  // (-3,-1)
+  r[12] = ring_pair<Q, -3>(W[3][0], W[3][1], W[3][2]);  // (-3, 0)
+  r[13] = ring_pair<Q, -3>(W[4][0], W[4][1], W[4][2]);  // (-3, 1)
+  r[14] = ring_pair<Q, -2>(W[5][0], W[5][1], W[5][2]);  // (-2, 2)
+  r[15] = ring_pair<Q, -1>(W[6][0], W[6][1], W[6][2]);  // (-1, 3)
+  return arc_score2(r, ring_pair<Q, 0>(W[3][0], W[3][1], W[3][2]));
+}
+
 __device__ __forceinline__ uint32_t fast_M4(const uint32_t (&W)[7][3]) {
-  uint32_t R[16];
-  R[0] = W[6][1];                              // ( 0, 3)
-  R[1] = __byte_perm(W[6][1], W[6][2], 0x4321);  // ( 1, 3)
-  R[2] = __byte_perm(W[5][1], W[5][2], 0x5432);  // ( 2, 2)
-  R[3] = __byte_perm(W[4][1], W[4][2], 0x6543);  // ( 3, 1)
-  R[4] = __byte_perm(W[3][1], W[3][2], 0x6543);  // ( 3, 0)
-  R[5] = __byte_perm(W[2][1], W[2][2], 0x6543);  // ( 3,-1)
-  R[6] = __byte_perm(W[1][1], W[1][2], 0x5432);  // ( 2,-2)
-  R[7] = __byte_perm(W[0][1], W[0][2], 0x4321);  // ( 1,-3)
-  R[8] = W[0][1];                              // ( 0,-3)
-  R[9] = __byte_perm(W[0][0], W[0][1], 0x6543);  // (-1,-3)
-  R[10] = __byte_perm(W[1][0], W[1][1], 0x5432); // (-2,-2)
-  R[11] = __byte_perm(W[2][0], W[2][1], 0x4321); // (-3,-1)
-  R[12] = __byte_perm(W[3][0], W[3][1], 0x4321); // (-3, 0)
-  R[13] = __byte_perm(W[4][0], W[4][1], 0x4321); // (-3, 1)
-  R[14] = __byte_perm(W[5][0], W[5][1], 0x5432); // (-2, 2)
-  R[15] = __byte_perm(W[6][0], W[6][1], 0x6543); // (-1, 3)
-  const uint32_t C = W[3][1];
-  uint32_t d[16];
-  const uint32_t clo = lo_pair(C) + 0x01000100u;
-#pragma unroll
-  for (int k = 0; k < 16; k++) d[k] = clo - lo_pair(R[k]);
-  const uint32_t slo = arc_score2(d) - 0x01000100u;  // pixels 0, 2
-  const uint32_t chi = hi_pair(C) + 0x01000100u;
-#pragma unroll
-  for (int k = 0; k < 16; k++) d[k] = chi - hi_pair(R[k]);
-  const uint32_t shi = arc_score2(d) - 0x01000100u;  // pixels 1, 3
+  const uint32_t slo = fast_M2<0>(W);  // pixels 0, 2 (M + 256 per lane)
+  const uint32_t shi = fast_M2<1>(W);  // pixels 1, 3
   return __byte_perm(slo, shi, 0x6240);
 }
 
@@ -129,13 +163,14 @@ __global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(const __grid_
   if ((ip & 15) == 0 && (reinterpret_cast<uintptr_t>(img) & 15) == 0) {
     for (int i = threadIdx.x; i < (Dh + 6) * nchunk; i += FB_THREADS) {
       const int r = i / nchunk, c = i - r * nchunk;
-      *reinterpret_cast<uint4*>(reg + r * rp + 16 * c) =
-          __ldg(reinterpret_cast<const uint4*>(row0 + (int64_t)r * ip) + c);
+      uint4 v = __ldg(reinterpret_cast<const uint4*>(row0 + (int64_t)r * ip) + c);
+      v.x ^= 0x80808080u, v.y ^= 0x80808080u, v.z ^= 0x80808080u, v.w ^= 0x80808080u;  // bytes as I - 128
+      *reinterpret_cast<uint4*>(reg + r * rp + 16 * c) = v;
     }
   } else {
     for (int i = threadIdx.x; i < (Dh + 6) * sw; i += FB_THREADS) {
       const int r = i / sw, c = i - r * sw;
-      reg[r * rp + c] = __ldg(row0 + (int64_t)r * ip + c);
+      reg[r * rp + c] = __ldg(row0 + (int64_t)r * ip + c) ^ 0x80;
     }
   }
   // zero border rows of the score map

@@ -24,11 +24,13 @@ constexpr int PT = 1024;
 
 // Four destination pixels of one row.  Per thread the four columns are fixed: their source
 // bytes x0_q, x1_q lie in [x0_0, x0_0 + 6) (x1_3 - x0_0 <= 5 for scale <= 4/3), read as three
-// aligned words from a = x0_0 & ~3 and funnel-shifted by sh = 8 * (x0_0 & 3); sel0 / sel1
-// then gather s[x0_q] / s[x1_q] with one byte permute each.  Vertical first, two pixels per
-// register (16-bit lanes: wy * byte <= 65280 never carries into the next lane), then
-// horizontal per pixel; the bilinear sum is exact integer arithmetic, so the order does not
-// change the result.
+// aligned words from a = x0_0 & ~3 and funnel-shifted by sh = 8 * (x0_0 & 3).  Horizontal
+// first: one byte permute gathers (s[x0_q], s[x1_q]) of two pixels into the bytes of one
+// register and one IDP.2A per pixel forms h_q = wx0_q * s[x0_q] + wx1_q * s[x1_q] (weights as a
+// 16x2 pair, wx0 + wx1 = 256, h <= 65280); then vertical per pixel with two IMADs,
+// acc = wy0 * h(y0) + wy1 * h(y1) + 2^15 < 2^24, whose byte 2 is the output (>> 16), picked by
+// byte permutes.  Exact integer arithmetic: the order of the two passes does not change the
+// result (INTER_LINEAR_EXACT, DESIGN.md §3 O1).
 __device__ __forceinline__ void window8(const uint8_t* row, uint32_t sh, uint32_t* lo, uint32_t* hi) {
   const uint32_t* w = reinterpret_cast<const uint32_t*>(row);
   const uint32_t w0 = w[0], w1 = w[1], w2 = w[2];
@@ -36,28 +38,29 @@ __device__ __forceinline__ void window8(const uint8_t* row, uint32_t sh, uint32_
   *hi = __funnelshift_r(w1, w2, sh);
 }
 
-__device__ __forceinline__ uint32_t lerp4(const uint8_t* r0, const uint8_t* r1, uint32_t sh, uint32_t sel0,
-                                          uint32_t sel1, const uint32_t (&wx1)[4], uint32_t wy1) {
-  uint32_t p0x, p0y, p1x, p1y;
-  window8(r0, sh, &p0x, &p0y);
-  window8(r1, sh, &p1x, &p1y);
-  const uint32_t a0 = __byte_perm(p0x, p0y, sel0), a1 = __byte_perm(p0x, p0y, sel1);
-  const uint32_t b0 = __byte_perm(p1x, p1y, sel0), b1 = __byte_perm(p1x, p1y, sel1);
+// h_q of one source row (sel: byte gathers (x0_0, x1_0, x0_1, x1_1) | (x0_2, x1_2, x0_3, x1_3) << 16)
+__device__ __forceinline__ void hrow4(const uint8_t* row, uint32_t sh, uint32_t sel, const uint32_t (&W)[4],
+                                      uint32_t (&h)[4]) {
+  uint32_t lo, hi;
+  window8(row, sh, &lo, &hi);
+  const uint32_t g01 = __byte_perm(lo, hi, sel & 0xFFFF), g23 = __byte_perm(lo, hi, sel >> 16);
+  h[0] = __dp2a_lo(W[0], g01, 0u);
+  h[1] = __dp2a_hi(W[1], g01, 0u);
+  h[2] = __dp2a_lo(W[2], g23, 0u);
+  h[3] = __dp2a_hi(W[3], g23, 0u);
+}
+
+__device__ __forceinline__ uint32_t lerp4(const uint8_t* r0, const uint8_t* r1, uint32_t sh, uint32_t sel,
+                                          const uint32_t (&W)[4], uint32_t wy1) {
+  uint32_t h0[4], h1[4];
+  hrow4(r0, sh, sel, W, h0);
+  hrow4(r1, sh, sel, W, h1);
   const uint32_t wy0 = 256 - wy1;
-  // lanes (px0, px1) and (px2, px3)
-  const uint32_t v0l = __byte_perm(a0, 0, 0x5150) * wy0 + __byte_perm(b0, 0, 0x5150) * wy1;
-  const uint32_t v0h = __byte_perm(a0, 0, 0x5352) * wy0 + __byte_perm(b0, 0, 0x5352) * wy1;
-  const uint32_t v1l = __byte_perm(a1, 0, 0x5150) * wy0 + __byte_perm(b1, 0, 0x5150) * wy1;
-  const uint32_t v1h = __byte_perm(a1, 0, 0x5352) * wy0 + __byte_perm(b1, 0, 0x5352) * wy1;
-  uint32_t packed = 0;
+  uint32_t a[4];
 #pragma unroll
-  for (int q = 0; q < 4; q++) {
-    const uint32_t v0 = ((q < 2 ? v0l : v0h) >> (16 * (q & 1))) & 0xFFFF;
-    const uint32_t v1 = ((q < 2 ? v1l : v1h) >> (16 * (q & 1))) & 0xFFFF;
-    const uint32_t o = ((256 - wx1[q]) * v0 + wx1[q] * v1 + (1u << 15)) >> 16;  // wx1 in [0, 256]
-    packed |= o << (8 * q);
-  }
-  return packed;
+  for (int q = 0; q < 4; q++) a[q] = h0[q] * wy0 + (h1[q] * wy1 + (1u << 15));  // < 2^24
+  // byte 2 of each accumulator = (acc >> 16)
+  return __byte_perm(__byte_perm(a[0], a[1], 0x0062), __byte_perm(a[2], a[3], 0x0062), 0x5410);
 }
 
 __global__ void __launch_bounds__(PT, 1) pyramid_fused_kernel(const __grid_constant__ Geom g, FrameSrc src,
@@ -132,8 +135,10 @@ __global__ void __launch_bounds__(PT, 1) pyramid_fused_kernel(const __grid_const
     const int spitch = C.z, dpitch = C.w;
     // this thread's four columns (host-built: source window, gather selectors, weights)
     const uint4 gq = s_g[(D.y & 0xFFFF) + cx];
-    const uint32_t sh = gq.x >> 16, sel0 = gq.y & 0xFFFF, sel1 = gq.y >> 16;
-    const uint32_t wx1[4] = {gq.z & 0xFFFF, gq.z >> 16, gq.w & 0xFFFF, gq.w >> 16};
+    const uint32_t sh = gq.x >> 16, sel = gq.y;
+    // (wx0, wx1) = (256 - wx1, wx1) as a 16x2 pair: wx1 * 65535 + 256
+    const uint32_t W[4] = {(gq.z & 0xFFFF) * 0xFFFFu + 256u, (gq.z >> 16) * 0xFFFFu + 256u,
+                           (gq.w & 0xFFFF) * 0xFFFFu + 256u, (gq.w >> 16) * 0xFFFFu + 256u};
     const uint8_t* const sa = sb + (int)(gq.x & 0xFFFF) - C.x;
     uint8_t* const da = db + 4 * cx;
     // owned columns come in whole groups of 4 (cuts are multiples of 4); only the level's
@@ -147,7 +152,7 @@ __global__ void __launch_bounds__(PT, 1) pyramid_fused_kernel(const __grid_const
     for (int r = ry; r < rows; r += (D.x >> 21)) {
       const uint32_t cy = yc[r];
       const int y0 = (int)(cy & 0xFFFF) - C.y, y1 = y0 + (int)(cy >> 25);
-      const uint32_t packed = lerp4(sa + y0 * spitch, sa + y1 * spitch, sh, sel0, sel1, wx1, (cy >> 16) & 0x1FF);
+      const uint32_t packed = lerp4(sa + y0 * spitch, sa + y1 * spitch, sh, sel, W, (cy >> 16) & 0x1FF);
       *reinterpret_cast<uint32_t*>(da + r * dpitch) = packed;
       const int y = ny0 + r;
       if (own_x && y >= B.z && y < B.w) {
@@ -184,16 +189,15 @@ bool pyramid_groups(const Geom& g, const uint32_t* tab, const int64_t* xoff, std
       uint32_t c[4];
       for (int q = 0; q < 4; q++) c[q] = xt[x + q < g.w[l] ? x + q : g.w[l] - 1];
       const uint32_t x00 = c[0] & 0xFFFF;
-      uint32_t sel0 = 0, sel1 = 0;
+      uint32_t sel = 0;  // byte gathers: (x0_q, x1_q) of pixel q in bytes 2(q%2), 2(q%2)+1 of word q/2
       for (int q = 0; q < 4; q++) {
         const uint32_t k = (c[q] & 0xFFFF) - x00;
         if (k + (c[q] >> 25) > 5) return false;  // the kernel's 6-byte window (scale <= 4/3)
-        sel0 |= k << (4 * q);
-        sel1 |= (k + (c[q] >> 25)) << (4 * q);
+        sel |= (k | (k + (c[q] >> 25)) << 4) << (8 * q);
       }
       uint4 e;
       e.x = (x00 & ~3u) | ((8u * (x00 & 3)) << 16);
-      e.y = sel0 | (sel1 << 16);
+      e.y = sel;
       e.z = ((c[0] >> 16) & 0x1FF) | (((c[1] >> 16) & 0x1FF) << 16);
       e.w = ((c[2] >> 16) & 0x1FF) | (((c[3] >> 16) & 0x1FF) << 16);
       gtab->push_back(e);

@@ -191,6 +191,7 @@ struct ss_ctx {
   uint64_t tick_clock = 0;
   int8_t* brute_qexp = nullptr;  // BRUTE: keypoint descriptors expanded to s8 +-1 (k_brute_tc.cu)
   int8_t* brute_mexp = nullptr;  // BRUTE: map descriptors expanded to s8 +-1
+  int prepared_map = -1;         // rows of the map brute_mexp holds from ss_brute_map_prepare (-1: none)
   int n_sm = 148;
   // per-extract DAG: level 0's FAST + distribution on side stream 0 right away; level l >= 1's
   // on side stream 1 + (l % kSideLevel) as soon as the pyramid (caller's stream) has level l
@@ -676,7 +677,9 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
   if (cfg->mode == SS_MATCH_BRUTE) {
     if (n_queries != 0) return fail(SS_EINVAL, "BRUTE mode takes no queries");
     if (n_map > c->max_map) return fail(SS_ECAPACITY, "n_map exceeds the ctx's max_map");
-    if (n_map > 0 && !d_map_desc) return fail(SS_EINVAL, "NULL map");
+    const bool prepared = n_map > 0 && !d_map_desc;
+    if (prepared && c->prepared_map != n_map)
+      return fail(SS_EINVAL, "NULL map and no map of n_map rows prepared by ss_brute_map_prepare");
     if (n_frames == 0) return SS_OK;
     const int n_slots = n_frames * c->g.kp_capacity;
     if (n_map == 0) {
@@ -689,8 +692,10 @@ ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_
       return SS_OK;
     }
     const int splits = brute_tc_splits(n_slots, n_map, c->max_splits, c->n_sm);
+    if (!prepared) c->prepared_map = -1;  // the expansion below overwrites the prepared map
     prof_mark(c, s);
-    SS_CUDA_TRY(launch_brute_expand(n_slots, d_desc, n_map, d_map_desc, c->brute_qexp, c->brute_mexp, s));
+    SS_CUDA_TRY(launch_brute_expand(n_slots, d_desc, n_map, prepared ? nullptr : d_map_desc, c->brute_qexp,
+                                    c->brute_mexp, s));
     prof_mark(c, s);
     prof_mark(c, s);
     SS_CUDA_TRY(launch_brute_tc(n_slots, n_map, c->brute_qexp, c->brute_mexp, splits, c->partial, s));
@@ -713,7 +718,10 @@ ss_status ss_match_brute_partial(ss_ctx* c, int32_t n_frames, const uint8_t* d_d
   if (n_map > c->max_map) return fail(SS_ECAPACITY, "n_map exceeds the ctx's max_map");
   if ((int64_t)map_offset + n_map > INT32_MAX) return fail(SS_EINVAL, "map_offset + n_map exceeds 2^31 - 1");
   if (n_frames == 0) return SS_OK;
-  if (!d_desc || !d_counts || !d_top2 || (n_map > 0 && !d_map_desc)) return fail(SS_EINVAL, "NULL buffer");
+  if (!d_desc || !d_counts || !d_top2) return fail(SS_EINVAL, "NULL buffer");
+  const bool prepared = n_map > 0 && !d_map_desc;
+  if (prepared && c->prepared_map != n_map)
+    return fail(SS_EINVAL, "NULL map and no map of n_map rows prepared by ss_brute_map_prepare");
   SS_CUDA_TRY(cudaSetDevice(c->device));
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   SS_CUDA_TRY(check_stream(s));
@@ -724,8 +732,10 @@ ss_status ss_match_brute_partial(ss_ctx* c, int32_t n_frames, const uint8_t* d_d
     return SS_OK;
   }
   const int splits = brute_tc_splits(n_slots, n_map, c->max_splits, c->n_sm);
+  if (!prepared) c->prepared_map = -1;
   prof_mark(c, s);
-  SS_CUDA_TRY(launch_brute_expand(n_slots, d_desc, n_map, d_map_desc, c->brute_qexp, c->brute_mexp, s));
+  SS_CUDA_TRY(launch_brute_expand(n_slots, d_desc, n_map, prepared ? nullptr : d_map_desc, c->brute_qexp,
+                                  c->brute_mexp, s));
   prof_mark(c, s);
   prof_mark(c, s);
   SS_CUDA_TRY(launch_brute_tc(n_slots, n_map, c->brute_qexp, c->brute_mexp, splits, c->partial, s));
@@ -733,6 +743,18 @@ ss_status ss_match_brute_partial(ss_ctx* c, int32_t n_frames, const uint8_t* d_d
   prof_mark(c, s);
   SS_CUDA_TRY(launch_brute_shard_top2(c->g, n_frames, d_counts, 2 * splits, c->partial, map_offset, top2, s));
   prof_mark(c, s);
+  return SS_OK;
+}
+
+ss_status ss_brute_map_prepare(ss_ctx* c, const uint8_t* d_map_desc, int32_t n_map, ss_stream_t stream) {
+  if (!c) return fail(SS_EINVAL, "NULL ctx");
+  if (n_map < 1 || !d_map_desc) return fail(SS_EINVAL, "n_map < 1 or NULL map");
+  if (n_map > c->max_map) return fail(SS_ECAPACITY, "n_map exceeds the ctx's max_map");
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  SS_CUDA_TRY(check_stream(s));
+  SS_CUDA_TRY(launch_brute_expand(0, nullptr, n_map, d_map_desc, c->brute_qexp, c->brute_mexp, s));
+  c->prepared_map = n_map;
   return SS_OK;
 }
 

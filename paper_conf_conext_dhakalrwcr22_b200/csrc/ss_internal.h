@@ -192,6 +192,7 @@ cudaError_t launch_brute_parts_merge(const Geom& g, int n_frames, const int32_t*
 int64_t brute_tc_query_bytes(int64_t n_slots);
 int64_t brute_tc_map_bytes(int64_t n_map);
 int brute_tc_splits(int n_slots, int n_map, int max_splits, int n_sm);
+// desc == NULL: map rows only; map_desc == NULL: keypoint rows only (prepared map)
 cudaError_t launch_brute_expand(int n_slots, const uint8_t* desc, int n_map, const uint8_t* map_desc, int8_t* qexp,
                                 int8_t* mexp, cudaStream_t s);
 cudaError_t launch_brute_tc(int n_slots, int n_map, const int8_t* qexp, const int8_t* mexp, int splits,

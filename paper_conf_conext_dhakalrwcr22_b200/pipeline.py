@@ -30,6 +30,7 @@ class OrbPipeline:
         self.kps = torch.zeros((max_frames, self.cap, 20), dtype=torch.uint8, device=self.device)
         self.desc = torch.zeros((max_frames, self.cap, ss.DESC_BYTES), dtype=torch.uint8, device=self.device)
         self.counts = torch.zeros((max_frames, n_levels + 1), dtype=torch.int32, device=self.device)
+        self.prepared_rows = 0
 
     def set_distribution(self, mode: int):
         """ss.SS_DIST_QUADTREE (default) or ss.SS_DIST_GRID_TOPN for the following extracts."""
@@ -65,12 +66,21 @@ class OrbPipeline:
         ss.ss_match_projection(self.ctx, n_frames, self.kps, self.desc, self.counts, taken, nq, queries, qdesc,
                                0, cfg, out, stream)
 
-    def match_brute(self, n_frames: int, map_desc: torch.Tensor, out: torch.Tensor,
+    def prepare_map(self, map_desc: torch.Tensor, stream: torch.cuda.Stream | None = None):
+        """ss_brute_map_prepare: expand a (static) shared map once; match_brute(n, None, out)
+        then uses it."""
+        stream = stream or torch.cuda.current_stream(self.device)
+        ss.ss_brute_map_prepare(self.ctx, map_desc, map_desc.shape[0], stream)
+        self.prepared_rows = map_desc.shape[0]
+
+    def match_brute(self, n_frames: int, map_desc: torch.Tensor | None, out: torch.Tensor,
                     cfg: ss.ss_match_cfg | None = None, stream: torch.cuda.Stream | None = None):
+        """map_desc [n_map, 32] uint8 CUDA tensor, or None for the prepared map (prepare_map)."""
         cfg = cfg or ss.brute_cfg()
         stream = stream or torch.cuda.current_stream(self.device)
+        n_map = self.prepared_rows if map_desc is None else map_desc.shape[0]
         ss.ss_match_projection(self.ctx, n_frames, self.kps, self.desc, self.counts, None, 0, None, map_desc,
-                               map_desc.shape[0], cfg, out, stream)
+                               n_map, cfg, out, stream)
 
     def project(self, n_frames: int, cams: torch.Tensor, points: torch.Tensor, point_frame: torch.Tensor,
                 out: torch.Tensor, th: float = 1.0, stream: torch.cuda.Stream | None = None):

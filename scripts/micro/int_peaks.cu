@@ -45,6 +45,11 @@ __device__ __forceinline__ unsigned smid() {
 #define OP_VMIN3 x[c] = __vimin3_u16x2(x[c], k, k2);
 #define OP_VMAX3 x[c] = __vimax3_u16x2(x[c], k, k2);
 #define OP_VMIN2 asm volatile("min.u16x2 %0, %0, %1;" : "+r"(x[c]) : "r"(x[(c + 1) % NCH]));
+#define OP_HMIN2 asm volatile("min.f16x2 %0, %0, %1;" : "+r"(x[c]) : "r"(x[(c + 1) % NCH]));
+#define OP_FMIN asm volatile("min.f32 %0, %0, %1;" : "+f"(fx[c]) : "f"(fx[(c + 1) % NCH]));
+#define OP_FMIN3 fx[c] = fminf(fminf(fx[c], fx[(c + 1) % NCH]), fx[(c + 2) % NCH]);
+#define OP_IMIN asm volatile("min.s32 %0, %0, %1;" : "+r"(x[c]) : "r"(x[(c + 1) % NCH]));
+#define OP_VADDMIN x[c] = __viaddmin_u16x2(x[c], k, x[(c + 1) % NCH]);
 #define OP_SHF asm volatile("shf.r.wrap.b32 %0, %0, %1, %2;" : "+r"(x[c]) : "r"(k), "r"(k2));
 
 #define KERNEL(NAME, OPSTMT)                                                                   \
@@ -52,7 +57,9 @@ __device__ __forceinline__ unsigned smid() {
                                                        unsigned long long* t0, unsigned long long* t1, \
                                                        unsigned* sm) {                          \
     uint32_t x[NCH];                                                                           \
+    float fx[NCH];                                                                             \
     _Pragma("unroll") for (int c = 0; c < NCH; c++) x[c] = threadIdx.x * 7 + c;                 \
+    _Pragma("unroll") for (int c = 0; c < NCH; c++) fx[c] = (float)(threadIdx.x * 7 + c);       \
     __syncthreads();                                                                           \
     unsigned long long a = clock64();                                                          \
     for (int it = 0; it < ITERS; it++) {                                                       \
@@ -61,7 +68,7 @@ __device__ __forceinline__ unsigned smid() {
     __syncthreads();                                                                           \
     unsigned long long b = clock64();                                                          \
     uint32_t s = 0;                                                                            \
-    _Pragma("unroll") for (int c = 0; c < NCH; c++) s ^= x[c];                                 \
+    _Pragma("unroll") for (int c = 0; c < NCH; c++) s ^= x[c] ^ __float_as_uint(fx[c]);        \
     if (s == 0xDEADBEEFu) sink[0] = s;                                                         \
     if (threadIdx.x == 0) {                                                                    \
       t0[blockIdx.x] = a;                                                                      \
@@ -80,6 +87,11 @@ KERNEL(imad, OP_IMAD)
 KERNEL(vimin3_u16x2, OP_VMIN3)
 KERNEL(vimax3_u16x2, OP_VMAX3)
 KERNEL(vminu2, OP_VMIN2)
+KERNEL(hmin2, OP_HMIN2)
+KERNEL(fmin, OP_FMIN)
+KERNEL(fmin3, OP_FMIN3)
+KERNEL(imin, OP_IMIN)
+KERNEL(viaddmin_u16x2, OP_VADDMIN)
 
 typedef void (*kfn)(uint32_t, uint32_t, uint32_t*, unsigned long long*, unsigned long long*, unsigned*);
 
@@ -105,7 +117,10 @@ int main() {
             {"prmt", "PRMT", k_prmt},             {"shf", "SHF", k_shf},
             {"popc", "POPC", k_popc},             {"dp4a", "IDP.4A", k_dp4a},
             {"imad", "IMAD", k_imad},             {"vimin3_u16x2", "VIMNMX3.U16x2", k_vimin3_u16x2},
-            {"vimax3_u16x2", "VIMNMX3.U16x2", k_vimax3_u16x2}, {"vminu2", "VIMNMX.U16x2", k_vminu2}};
+            {"vimax3_u16x2", "VIMNMX3.U16x2", k_vimax3_u16x2}, {"vminu2", "VIMNMX.U16x2", k_vminu2},
+            {"hmin2", "HMNMX2", k_hmin2},         {"fmin", "FMNMX", k_fmin},
+            {"fmin3", "FMNMX3", k_fmin3},         {"imin", "IMNMX", k_imin},
+            {"viaddmin_u16x2", "VIADDMNMX.U16x2", k_viaddmin_u16x2}};
   cudaEvent_t e0, e1;
   cudaEventCreate(&e0);
   cudaEventCreate(&e1);

@@ -272,3 +272,66 @@ def test_distribution_switch_with_graph_reuse(torch_cuda, ref):
             np.testing.assert_array_equal(gk["lx"], want[mode][0][b][:n]["lx"])
             np.testing.assert_array_equal(gk["ly"], want[mode][0][b][:n]["ly"])
     pipe.close()
+
+
+def test_brute_prepared_map(torch_cuda, ref):
+    """ss_brute_map_prepare: the map expanded once, then BRUTE calls with a NULL map (direct,
+    map-sharded partial and ss_track_tick) expand only their keypoints -- bit-exact with the
+    oracle; a call with an explicit map forgets the preparation; a NULL map without a matching
+    preparation is rejected."""
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import match_records
+    w, h = synth.SHAPES["euroc"]
+    B, nf, n_map = 3, 1250, 20000
+    p = ref.params(w, h, nf)
+    cap = p.kp_capacity
+    frames = synth.make_frames(w, h, B, cfg=29)
+    rk, rd, rc = ref.orb_extract_batch(p, frames)
+    mp = synth.make_brute_map([rd[b][: rc[b][-1]] for b in range(B)], n_map, seed=31, n_from_kps=3000)
+    want = ref.match_brute(p, rd, rc, mp, 50, 3, 4)
+    pipe = _extract(torch, p, frames, max_map=n_map)
+    d_map = torch.from_numpy(mp).cuda()
+    out = torch.zeros((B * cap, 3), dtype=torch.int32, device="cuda")
+    st = torch.cuda.current_stream()
+    with pytest.raises(ss.SSError):  # nothing prepared yet
+        ss.ss_match_projection(pipe.ctx, B, pipe.kps, pipe.desc, pipe.counts, None, 0, None, None, n_map,
+                               ss.brute_cfg(), out, st)
+    pipe.prepare_map(d_map)
+    d_map.zero_()  # the preparation is a snapshot: later changes of the source are not seen
+    pipe.match_brute(B, None, out)
+    got = match_records(out).reshape(B, cap)
+    for b in range(B):
+        n = int(rc[b][-1])
+        np.testing.assert_array_equal(got[b, :n], want[b, :n])
+    # sharded partial over the prepared map == top-2 of the direct result
+    top2 = torch.zeros((B, cap, 2), dtype=torch.int64, device="cuda")
+    ss.ss_match_brute_partial(pipe.ctx, B, pipe.desc, pipe.counts, None, n_map, 0, top2, torch.cuda.current_stream())
+    out2 = torch.zeros_like(out)
+    ss.ss_match_brute_merge(pipe.ctx, B, pipe.counts, 1, top2, ss.brute_cfg(), out2, torch.cuda.current_stream())
+    got2 = match_records(out2).reshape(B, cap)
+    for b in range(B):
+        n = int(rc[b][-1])
+        np.testing.assert_array_equal(got2[b, :n], want[b, :n])
+    # ss_track_tick with io.d_map_desc = NULL
+    hf = torch.from_numpy(frames.reshape(-1).copy()).pin_memory()
+    hm = torch.zeros(B * cap * 12, dtype=torch.uint8).pin_memory()
+    io = ss.ss_tick_io()
+    io.frames, io.frame_stride, io.pitch = hf.data_ptr(), h * w, w
+    io.d_map_desc, io.n_map, io.matches = None, n_map, hm.data_ptr()
+    ss.ss_track_tick(pipe.ctx, B, ss.brute_cfg(), io, torch.cuda.current_stream())
+    torch.cuda.synchronize()
+    got3 = hm.numpy().view(ref.MATCH_DTYPE).reshape(B, cap)
+    for b in range(B):
+        n = int(rc[b][-1])
+        np.testing.assert_array_equal(got3[b, :n], want[b, :n])
+    with pytest.raises(ss.SSError):
+        ss.ss_match_projection(pipe.ctx, B, pipe.kps, pipe.desc, pipe.counts, None, 0, None, None, n_map - 1,
+                               ss.brute_cfg(), out, torch.cuda.current_stream())  # row count differs
+    # an explicit map replaces the prepared one
+    d_map2 = torch.from_numpy(mp).cuda()
+    pipe.match_brute(B, d_map2, out)
+    with pytest.raises(ss.SSError):
+        ss.ss_match_projection(pipe.ctx, B, pipe.kps, pipe.desc, pipe.counts, None, 0, None, None, n_map,
+                               ss.brute_cfg(), out, st)
+    pipe.close()
