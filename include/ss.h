@@ -154,6 +154,17 @@ ss_status ss_orb_extract(ss_ctx* ctx, int32_t n_frames, const uint8_t* d_frames,
                          int32_t pitch, ss_keypoint* d_kps, uint8_t* d_desc, int32_t* d_counts,
                          ss_stream_t stream);
 
+/* ss_orb_extract for n_frames independently allocated client frames (SURVEY.md §8(b)'s
+ * d_frames[] / pitches[] form): d_frames = HOST array of n_frames DEVICE pointers, pitches =
+ * HOST array of their row pitches (>= width).  The frames are packed into the ctx's frame
+ * staging buffer by one device-side 2-D copy each (enqueued on `stream`), then extracted as
+ * one batch; outputs, results and errors as ss_orb_extract (plus SS_EINVAL for a NULL frame
+ * pointer or a pitch < width).  The staging buffer is shared with ss_track_tick: the two must
+ * not be in flight on one ctx at the same time.  Stereo pairs (ss_stereo_match reads level 0
+ * from the buffer it is given) use ss_orb_extract's single-buffer form or ss_track_tick. */
+ss_status ss_orb_extract_frames(ss_ctx* ctx, int32_t n_frames, const uint8_t* const* d_frames, const int32_t* pitches,
+                                ss_keypoint* d_kps, uint8_t* d_desc, int32_t* d_counts, ss_stream_t stream);
+
 /* O9 / O10 on the outputs of ss_orb_extract (same layouts).  Device pointers:
  * WINDOW ("search local points"):
  *   d_kp_taken [n_frames][kp_capacity] u8 (non-zero = keypoint already matched; may be NULL),

@@ -15,7 +15,7 @@ OBJ = os.path.join(PKG, "build")
 LIB = os.path.join(PKG, "libss.so")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC_FLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-ffp-contract=off,-O2",
-                     "-I", os.path.join(ROOT, "include"), "-Xptxas", "-v"]
+                     "-I", os.path.join(ROOT, "include"), "-Xptxas", "-v"] + os.environ.get("SS_NVCC_EXTRA", "").split()
 SOURCES = ["ss_api.cpp", "k_pyramid.cu", "k_fast.cu", "k_distribute.cu", "k_describe.cu", "k_match.cu", "k_brute_tc.cu", "k_project.cu", "k_stereo.cu", "k_grid.cu", "k_lastframe.cu"]
 HEADERS = ["ss_internal.h", "brief_pattern.inc", "match_common.cuh"]
 

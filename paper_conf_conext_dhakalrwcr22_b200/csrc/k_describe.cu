@@ -12,6 +12,8 @@
 // the samples read replaces a whole-level blur pass and its HBM round trip.  Output
 // position = the keypoint's canonical index, so the per-level counts of the distribution
 // become the prefix offsets written to d_counts.
+#include <cudaTypedefs.h>  // PFN_cuTensorMapEncodeTiled
+
 #include "brief_pattern.inc"
 #include "ss_internal.h"
 
@@ -60,6 +62,36 @@ __device__ __forceinline__ int rhe_rot(int a, int b, float ca, float cb, int ma,
   return rhe_exact((long long)a * ma + (long long)b * mb, r2, k);
 }
 
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+// A 43-row x 64-byte box (rows y.., columns x.., x a multiple of 16) of frame f's level by one
+// TMA tensor copy into the warp's buffer (lane 0 issues; the warp waits on its mbarrier).
+__device__ __forceinline__ void tma_patch(const CUtensorMap* map, uint8_t* dst, uint64_t* bar, int x, int y, int f,
+                                          int lane) {
+  const uint32_t b = smem_addr(bar);
+  if (lane == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(b));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(b), "r"(kPatchBoxW * kPatchBoxH)
+                 : "memory");
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], "
+        "[%5];" ::"r"(smem_addr(dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(f), "r"(b)
+        : "memory");
+  }
+  __syncwarp();
+  asm volatile(
+      "{\n\t.reg .pred P1;\n"
+      "TMA_WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], 0;\n\t"
+      "@!P1 bra TMA_WAIT_%=;\n}" ::"r"(b)
+      : "memory");
+}
+
 // SAMPLES (test hook, ss_debug_capture_samples): also write the blurred value of every sample
 // point the comparisons read, samples[slot][b][e] for bit b = 8 * lane + t, point e
 template <bool SAMPLES>
@@ -70,9 +102,13 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
                                                                    ss_keypoint* __restrict__ kps,
                                                                    uint8_t* __restrict__ desc,
                                                                    int32_t* __restrict__ counts,
-                                                                   uint8_t* __restrict__ samples) {
+                                                                   uint8_t* __restrict__ samples,
+                                                                   const __grid_constant__ PatchMaps maps) {
   pdl_trigger();
-  extern __shared__ __align__(16) uint8_t sm[];  // DESC_WARPS * PER_WARP
+  extern __shared__ __align__(128) uint8_t sm_raw[];  // DESC_WARPS * PER_WARP + 128
+  // 128-B aligned warp buffers (TMA destinations)
+  uint8_t* const sm = sm_raw + ((128 - (smem_addr(sm_raw) & 127)) & 127);
+  __shared__ __align__(8) uint64_t s_bar[DESC_WARPS];
   __shared__ int off[kMaxLevels + 1];
   __shared__ __align__(16) uint32_t s_wmask[16 * 8], s_wu[16 * 8];  // per |v|: 32 byte weights
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -126,7 +162,15 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
   const uint8_t* p0 = img + (int64_t)(ly - 21) * ip + (lx - 21);
   const int sh = (int)(reinterpret_cast<uintptr_t>(p0) & 15);
   const uint8_t* P;  // P[r * PP + c] = raw patch pixel (ly - 21 + r, lx - 21 + c)
-  if ((ip & 15) == 0 && lx >= 21 && lx + 21 < w && lx - 21 - sh + 64 <= ip) {
+  if (((maps.valid >> l) & 1u) && lx >= 21 && lx + 21 < w && ly >= 21 && ly + 21 < h) {
+    // the patch lies inside the level (no REFLECT_101 needed): one TMA tensor copy of 43 rows
+    // x 64 columns from the 16-B aligned column at or left of lx - 21 (a u8 tile's innermost
+    // coordinate must be 16-B aligned: measured, scripts/micro/tma_probe2.cu); columns past the
+    // level edge arrive as zeros and are never read
+    const int x0 = lx - 21;
+    tma_patch(&maps.level[l], Pw, &s_bar[warp], x0 & ~15, ly - 21, f, lane);
+    P = Pw + (x0 & 15);
+  } else if ((ip & 15) == 0 && lx >= 21 && lx + 21 < w && lx - 21 - sh + 64 <= ip) {
     // columns inside the level: 43 rows x four aligned 16-B chunks, rows mapped by REFLECT_101
     // (identity away from the top/bottom border); all six loads of a lane are issued before
     // the first store (one global latency, not six)
@@ -324,21 +368,45 @@ const int* brief_pattern_host() { return SS_BRIEF_PATTERN_HOST; }
 
 cudaError_t describe_init() {  // ss_create, per device (never under stream capture)
   cudaError_t e = cudaFuncSetAttribute(describe_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)(DESC_WARPS * PER_WARP));
+                                       (int)(DESC_WARPS * PER_WARP + 128));
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(describe_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              (int)(DESC_WARPS * PER_WARP));
+                              (int)(DESC_WARPS * PER_WARP + 128));
+}
+
+bool encode_patch_map(CUtensorMap* m, const void* base, int w, int h, int frames, int64_t pitch, int64_t fstride) {
+  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+  static bool tried = false;
+  if (!tried) {  // the driver entry point through the runtime (no -lcuda link)
+    tried = true;
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  }
+  if (!encode || !base || w < kPatchBoxW || h < kPatchBoxH || frames < 1) return false;
+  if ((reinterpret_cast<uintptr_t>(base) & 15) || (pitch & 15)) return false;
+  if (frames == 1) fstride = ((int64_t)pitch * h + 15) & ~(int64_t)15;  // unused dimension
+  if (fstride & 15) return false;
+  const cuuint64_t dims[3] = {(cuuint64_t)w, (cuuint64_t)h, (cuuint64_t)frames};
+  const cuuint64_t strides[2] = {(cuuint64_t)pitch, (cuuint64_t)fstride};
+  const cuuint32_t box[3] = {(cuuint32_t)kPatchBoxW, (cuuint32_t)kPatchBoxH, 1u};
+  const cuuint32_t estr[3] = {1u, 1u, 1u};
+  return encode(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 3, const_cast<void*>(base), dims, strides, box, estr,
+                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 cudaError_t launch_describe(const Geom& g, int n_frames, FrameSrc src, const uint32_t* selected,
                             const int32_t* sel_counts, const int8_t* pattern, ss_keypoint* kps, uint8_t* desc,
-                            int32_t* counts, uint8_t* samples, cudaStream_t s) {
-  const size_t smem = (size_t)DESC_WARPS * PER_WARP;
+                            int32_t* counts, uint8_t* samples, const PatchMaps& maps, cudaStream_t s) {
+  const size_t smem = (size_t)DESC_WARPS * PER_WARP + 128;
   dim3 grid((g.kp_capacity + DESC_WARPS - 1) / DESC_WARPS, n_frames);
   cudaError_t e = samples ? launch_pdl(describe_kernel<true>, grid, dim3(DESC_WARPS * 32), smem, s, g, src, selected,
-                                       sel_counts, pattern, kps, desc, counts, samples)
+                                       sel_counts, pattern, kps, desc, counts, samples, maps)
                           : launch_pdl(describe_kernel<false>, grid, dim3(DESC_WARPS * 32), smem, s, g, src, selected,
-                                       sel_counts, pattern, kps, desc, counts, samples);
+                                       sel_counts, pattern, kps, desc, counts, samples, maps);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 

@@ -128,6 +128,13 @@ __device__ __forceinline__ uint32_t fast_M4(const uint32_t (&W)[7][3]) {
   return __byte_perm(slo, shi, 0x6240);
 }
 
+// 4-bit column mask of one NMS step from the two 16x2 half results (bit 15 / 31 of h0 =
+// pixels 0 / 2, of h1 = pixels 1 / 3): bits 0..3 = pixels 0..3
+__device__ __forceinline__ uint32_t nibble4(uint32_t h0, uint32_t h1) {
+  const uint32_t t = (h0 >> 15) | (h1 >> 14);  // bits 0, 16 (pixels 0, 2) and 1, 17 (pixels 1, 3)
+  return (t | (t >> 14)) & 0xFu;
+}
+
 __global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(const __grid_constant__ Geom g, FrameSrc src,
                                                                 const BandInfo* __restrict__ bands,
                                                                 const CellInfo* __restrict__ cells,
@@ -220,6 +227,10 @@ __global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(const __grid_
     const CellInfo c = cells[ci];
     const int cx0 = c.x0 - xa, cw = c.x1 - c.x0;  // staged columns [cx0, cx0 + cw), cw < 64
     unsigned long long kmin[2] = {0ull, 0ull}, kini[2] = {0ull, 0ull};
+    // words A_j (cell columns [4j-4, 4j)) are whole for j < nk, partial at j = nk (lastmask),
+    // outside the cell beyond
+    const int nk = (cw + 3) >> 2;
+    const uint32_t lastmask = 0xFFFFFFFFu >> (8 * (4 * nk - cw));
     if (Dh <= 32) {
       // one pass, lane = row: only the row's own words are read; the neighbour rows' 3-wide
       // maxima come from lanes y - 1 and y + 1 by shuffles (rows -1 and Dh are the zero rows
@@ -228,18 +239,16 @@ __global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(const __grid_
       const uint32_t sh = 8u * (uint32_t)(base & 3);
       const uint32_t* pr = reinterpret_cast<const uint32_t*>(Mb + ((lane < Dh ? lane : Dh) + 1) * mbw + a0);
       auto aword = [&](int j) -> uint32_t {
-        const int valid = cw - (4 * j - 4);
         const uint32_t v = __funnelshift_r(pr[j], pr[j + 1], sh);
-        return valid >= 4 ? v : (valid <= 0 ? 0u : v & (0xFFFFFFFFu >> (8 * (4 - valid))));
+        return j < nk ? v : (j == nk ? v & lastmask : 0u);
       };
       const uint32_t upm = lane > 0 ? 0xFFFFFFFFu : 0u, dnm = lane + 1 < Dh ? 0xFFFFFFFFu : 0u;
       const uint32_t tmin1 = (uint32_t)(tmin + 1) * 0x10001u, tini1 = (uint32_t)(tini + 1) * 0x10001u;
       uint32_t pw = 0u, cwd = aword(1);
-      const int nk = (cw + 3) >> 2;
       for (int k = 0; k < nk; k++) {
         const uint32_t nw = aword(k + 2);
         const uint32_t Lw = __byte_perm(pw, cwd, 0x6543), Rw = __byte_perm(cwd, nw, 0x4321);
-        uint32_t bmin = 0u, bini = 0u;
+        uint32_t ok[2], oi[2];
 #pragma unroll
         for (int half = 0; half < 2; half++) {  // lanes: pixels (0, 2), then (1, 3)
           const uint32_t sel = half ? 0x7371u : 0x7270u;
@@ -249,13 +258,11 @@ __global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(const __grid_
           const uint32_t dn = __shfl_down_sync(0xFFFFFFFFu, hf, 1) & dnm;
           const uint32_t nb = __vimax3_u16x2(hlr, up, dn);
           const uint32_t C = Ch | 0x80008000u;
-          const uint32_t ok = (C - nb - 0x00010001u) & (C - tmin1) & 0x80008000u;  // > neighbours, > minTh
-          const uint32_t oi = ok & (C - tini1);                                       // and > iniTh
-          bmin |= ((ok >> 15) & 1u) << half | ((ok >> 31) & 1u) << (2 + half);
-          bini |= ((oi >> 15) & 1u) << half | ((oi >> 31) & 1u) << (2 + half);
+          ok[half] = (C - nb - 0x00010001u) & (C - tmin1) & 0x80008000u;  // > neighbours, > minTh
+          oi[half] = ok[half] & (C - tini1);                                // and > iniTh
         }
-        kmin[0] |= (unsigned long long)bmin << (4 * k);
-        kini[0] |= (unsigned long long)bini << (4 * k);
+        kmin[0] |= (unsigned long long)nibble4(ok[0], ok[1]) << (4 * k);
+        kini[0] |= (unsigned long long)nibble4(oi[0], oi[1]) << (4 * k);
         pw = cwd;
         cwd = nw;
       }
@@ -275,20 +282,18 @@ __global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(const __grid_
         const uint32_t* pr1 = reinterpret_cast<const uint32_t*>(Mb + (y + 1) * mbw + a0);
         const uint32_t* pr2 = reinterpret_cast<const uint32_t*>(Mb + (y + 2) * mbw + a0);
         auto aword = [&](const uint32_t* pr, int j) -> uint32_t {
-          const int valid = cw - (4 * j - 4);  // bytes of A_j inside the cell (j >= 1)
           const uint32_t v = __funnelshift_r(pr[j], pr[j + 1], sh);
-          return valid >= 4 ? v : (valid <= 0 ? 0u : v & (0xFFFFFFFFu >> (8 * (4 - valid))));
+          return j < nk ? v : (j == nk ? v & lastmask : 0u);
         };
         uint32_t p0 = 0u, p1 = 0u, p2 = 0u;  // A_k of rows y-1, y, y+1
         uint32_t c0w = aword(pr0, 1), c1w = aword(pr1, 1), c2w = aword(pr2, 1);  // A_{k+1}
         const uint32_t tmin1 = (uint32_t)(tmin + 1) * 0x10001u, tini1 = (uint32_t)(tini + 1) * 0x10001u;
-        const int nk = (cw + 3) >> 2;
         for (int k = 0; k < nk; k++) {
           const uint32_t n0 = aword(pr0, k + 2), n1 = aword(pr1, k + 2), n2 = aword(pr2, k + 2);
           const uint32_t L0 = __byte_perm(p0, c0w, 0x6543), R0 = __byte_perm(c0w, n0, 0x4321);
           const uint32_t L1 = __byte_perm(p1, c1w, 0x6543), R1 = __byte_perm(c1w, n1, 0x4321);
           const uint32_t L2 = __byte_perm(p2, c2w, 0x6543), R2 = __byte_perm(c2w, n2, 0x4321);
-          uint32_t bmin = 0u, bini = 0u;
+          uint32_t ok[2], oi[2];
 #pragma unroll
           for (int half = 0; half < 2; half++) {  // lanes: pixels (0, 2), then (1, 3)
             const uint32_t sel = half ? 0x7371u : 0x7270u;
@@ -297,13 +302,11 @@ __global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(const __grid_
                 __vimax3_u16x2(__vimax3_u16x2(__byte_perm(c0w, 0, sel), __byte_perm(L0, 0, sel), __byte_perm(R0, 0, sel)),
                                __vimax3_u16x2(__byte_perm(c2w, 0, sel), __byte_perm(L2, 0, sel), __byte_perm(R2, 0, sel)),
                                __vimax3_u16x2(__byte_perm(L1, 0, sel), __byte_perm(R1, 0, sel), 0u));
-            const uint32_t ok = (C - nb - 0x00010001u) & (C - tmin1) & 0x80008000u;  // > neighbours, > minTh
-            const uint32_t oi = ok & (C - tini1);                                       // and > iniTh
-            bmin |= ((ok >> 15) & 1u) << half | ((ok >> 31) & 1u) << (2 + half);
-            bini |= ((oi >> 15) & 1u) << half | ((oi >> 31) & 1u) << (2 + half);
+            ok[half] = (C - nb - 0x00010001u) & (C - tmin1) & 0x80008000u;  // > neighbours, > minTh
+            oi[half] = ok[half] & (C - tini1);                                // and > iniTh
           }
-          kmin[hh] |= (unsigned long long)bmin << (4 * k);
-          kini[hh] |= (unsigned long long)bini << (4 * k);
+          kmin[hh] |= (unsigned long long)nibble4(ok[0], ok[1]) << (4 * k);
+          kini[hh] |= (unsigned long long)nibble4(oi[0], oi[1]) << (4 * k);
           p0 = c0w, p1 = c1w, p2 = c2w;
           c0w = n0, c1w = n1, c2w = n2;
         }

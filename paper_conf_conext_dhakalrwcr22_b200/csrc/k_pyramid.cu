@@ -20,7 +20,10 @@ namespace ss {
 
 namespace {
 
-constexpr int PT = 1024;
+#ifndef SS_PYR_THREADS
+#define SS_PYR_THREADS 1024
+#endif
+constexpr int PT = SS_PYR_THREADS;  // threads per CTA (a block of every level per CTA)
 
 // Four destination pixels of one row.  Per thread the four columns are fixed: their source
 // bytes x0_q, x1_q lie in [x0_0, x0_0 + 6) (x1_3 - x0_0 <= 5 for scale <= 4/3), read as three
@@ -63,7 +66,7 @@ __device__ __forceinline__ uint32_t lerp4(const uint8_t* r0, const uint8_t* r1, 
   return __byte_perm(__byte_perm(a[0], a[1], 0x0062), __byte_perm(a[2], a[3], 0x0062), 0x5410);
 }
 
-__global__ void __launch_bounds__(PT, 1) pyramid_fused_kernel(const __grid_constant__ Geom g, FrameSrc src,
+__global__ void __launch_bounds__(PT, 2048 / PT > 1 ? 2048 / PT : 1) pyramid_fused_kernel(const __grid_constant__ Geom g, FrameSrc src,
                                                               const uint4* __restrict__ gtab,
                                                               const uint32_t* __restrict__ ytab,
                                                               const PyrLvl* __restrict__ plan, int buf0_bytes,

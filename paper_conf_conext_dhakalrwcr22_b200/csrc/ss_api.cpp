@@ -153,6 +153,7 @@ struct ss_ctx {
   uint64_t* phase_ts = nullptr;  // distribution phase timestamps [max_frames][L][16] (debug hook)
   unsigned long long* partial = nullptr;
   int dist_mode = SS_DIST_QUADTREE;  // ss_set_distribution
+  PatchMaps maps{};                  // TMA maps of the describe kernel (levels >= 1 at ss_create)
   // test hooks: lanes per WINDOW query (0 = chosen per launch), blurred-sample capture buffer
   int win_lanes = 0;
   uint8_t* dbg_samples = nullptr;
@@ -558,6 +559,13 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_aux0, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_aux1, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaMemset(c->sel_counts, 0, sizeof(int32_t) * F * L);
+  if (e == cudaSuccess) {
+    c->maps.valid = 0;
+    for (int l = 1; l < L; l++)
+      if (encode_patch_map(&c->maps.level[l], c->pyr + g.lvl_off[l], g.w[l], g.h[l], max_frames, g.pitch[l],
+                           g.pyr_frame_bytes))
+        c->maps.valid |= 1u << l;
+  }
   if (e != cudaSuccess) {
     std::string m = std::string("ss_create: ") + cudaGetErrorString(e);
     free_ctx(c);
@@ -632,14 +640,40 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   prof_mark(c, s);
   if (q != s) SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[0], 0));
   prof_mark(c, s);
+  // level 0: the caller's frames, encoded for this call (TMA when 16-B aligned, else LDG)
+  c->maps.valid &= ~1u;
+  if (encode_patch_map(&c->maps.level[0], d_frames, g.W, g.H, n_frames, pitch, frame_stride)) c->maps.valid |= 1u;
   SS_CUDA_TRY(launch_describe(g, n_frames, src, c->selected, c->sel_counts, c->pattern, d_kps, d_desc, d_counts,
-                              c->dbg_samples, s));
+                              c->dbg_samples, c->maps, s));
   prof_mark(c, s);
   c->last_frames = d_frames;
   c->last_stride = frame_stride;
   c->last_pitch = pitch;
   c->last_n = n_frames;
   return SS_OK;
+}
+
+ss_status ss_orb_extract_frames(ss_ctx* c, int32_t n_frames, const uint8_t* const* d_frames, const int32_t* pitches,
+                                ss_keypoint* d_kps, uint8_t* d_desc, int32_t* d_counts, ss_stream_t stream) {
+  if (!c) return fail(SS_EINVAL, "NULL ctx");
+  if (n_frames < 0) return fail(SS_EINVAL, "n_frames < 0");
+  if (n_frames > c->max_frames) return fail(SS_ECAPACITY, "n_frames exceeds the ctx's max_frames");
+  if (n_frames == 0) return SS_OK;
+  if (!d_frames || !pitches) return fail(SS_EINVAL, "NULL frame / pitch array");
+  for (int f = 0; f < n_frames; f++) {
+    if (!d_frames[f]) return fail(SS_EINVAL, "NULL frame pointer");
+    if (pitches[f] < c->g.W) return fail(SS_EINVAL, "pitch < width");
+  }
+  SS_CUDA_TRY(cudaSetDevice(c->device));
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  // independently allocated client frames are packed into the ctx's frame staging buffer (one
+  // device-side 2-D copy per frame, 16-B aligned pitch), then extracted as one batch
+  const int P = c->io_pitch;
+  const int64_t fstride = (int64_t)c->g.H * P;
+  for (int f = 0; f < n_frames; f++)
+    SS_CUDA_TRY(cudaMemcpy2DAsync(c->io_frames + f * fstride, P, d_frames[f], pitches[f], c->g.W, c->g.H,
+                                  cudaMemcpyDeviceToDevice, s));
+  return ss_orb_extract(c, n_frames, c->io_frames, fstride, P, d_kps, d_desc, d_counts, stream);
 }
 
 ss_status ss_match_projection(ss_ctx* c, int32_t n_frames, const ss_keypoint* d_kps, const uint8_t* d_desc,

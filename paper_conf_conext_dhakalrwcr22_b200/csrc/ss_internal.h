@@ -1,6 +1,7 @@
 // ss_internal.h -- product-internal types shared by the host layer (ss_api.cpp) and the
 // sm_100a kernels.  Nothing here is shared with oracle/ (the CPU checker).
 #pragma once
+#include <cuda.h>  // CUtensorMap (TMA descriptors; encoded through the runtime's driver entry point)
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -76,6 +77,19 @@ struct FrameSrc {
   int32_t pitch;
   uint8_t* pyr;  // pyramid scratch (levels >= 1)
 };
+
+// TMA tensor maps of the descriptor kernel's 43-row x 64-byte patch loads, one per pyramid
+// level: 3-D u8 [frames][h_l][w_l] with the level's row pitch and frame stride (level 0 = the
+// caller's frames, encoded per ss_orb_extract call; levels >= 1 = the pyramid scratch, encoded
+// at ss_create).  Bit l of `valid`: level l may be loaded by TMA (16-B aligned base / pitch /
+// stride), else the kernel uses its LDG path.
+constexpr int kPatchBoxW = 64, kPatchBoxH = 43;
+struct PatchMaps {
+  CUtensorMap level[kMaxLevels];
+  uint32_t valid;
+};
+// Encode one level's map; false if the layout is not TMA-addressable (alignment).
+bool encode_patch_map(CUtensorMap* m, const void* base, int w, int h, int frames, int64_t pitch, int64_t fstride);
 
 // Candidate / selected key: (ly << 19) | (lx << 8) | M  (lx, ly < 2048, M = FAST score + 1).
 __host__ __device__ inline uint32_t pack_key(int lx, int ly, int m) {
@@ -162,7 +176,8 @@ cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_lev
                               cudaStream_t s);
 cudaError_t launch_describe(const Geom& g, int n_frames, FrameSrc src, const uint32_t* selected,
                             const int32_t* sel_counts, const int8_t* pattern, ss_keypoint* kps, uint8_t* desc,
-                            int32_t* counts, uint8_t* samples, cudaStream_t s);  // samples: test hook or NULL
+                            int32_t* counts, uint8_t* samples, const PatchMaps& maps,
+                            cudaStream_t s);  // samples: test hook or NULL
 // The rotated-BRIEF pattern (1024 ints: 256 pairs x 2 points x (x, y)), host copy.
 const int* brief_pattern_host();
 // Row index of the keypoints (first keypoint per (frame, level, row)) + dedup claim reset.

@@ -110,6 +110,7 @@ def lib():
         L.ss_match_brute_partial.argtypes = [P, i32, P, P, P, i32, i32, P, P]
         L.ss_match_brute_merge.argtypes = [P, i32, P, i32, P, C.POINTER(ss_match_cfg), P, P]
         L.ss_brute_map_prepare.argtypes = [P, P, i32, P]
+        L.ss_orb_extract_frames.argtypes = [P, i32, C.POINTER(P), C.POINTER(i32), P, P, P, P]
         L.ss_set_distribution.argtypes = [P, i32]
         L.ss_track_tick.argtypes = [P, i32, C.POINTER(ss_match_cfg), C.POINTER(ss_tick_io), P]
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
@@ -125,7 +126,7 @@ def lib():
                    "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_set_distribution",
                    "ss_match_last_frame", "ss_match_brute_partial", "ss_match_brute_merge", "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
                    "ss_profile_next", "ss_debug_phase_times", "ss_debug_distribution_paths", "ss_debug_match_lanes",
-                   "ss_debug_capture_samples", "ss_brute_map_prepare"):
+                   "ss_debug_capture_samples", "ss_brute_map_prepare", "ss_orb_extract_frames"):
             getattr(L, fn).restype = C.c_int
         _lib = L
     return _lib
@@ -135,7 +136,7 @@ EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "s
             "ss_match_projection", "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_set_distribution",
             "ss_match_last_frame", "ss_match_brute_partial", "ss_match_brute_merge", "ss_profile_events", "ss_profile_next", "ss_debug_level",
             "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times", "ss_debug_distribution_paths",
-            "ss_debug_match_lanes", "ss_debug_capture_samples", "ss_brute_map_prepare")
+            "ss_debug_match_lanes", "ss_debug_capture_samples", "ss_brute_map_prepare", "ss_orb_extract_frames")
 
 
 def _check(status: int, ctx=None):
@@ -294,6 +295,15 @@ def ss_debug_overflow_count(ctx) -> int:
     n = C.c_int32()
     _check(lib().ss_debug_overflow_count(ctx, C.byref(n)), ctx)
     return n.value
+
+
+def ss_orb_extract_frames(ctx, frames, d_kps, d_desc, d_counts, stream=None):
+    """frames: list of uint8 CUDA tensors [H, pitch] (one per client, separately allocated)."""
+    n = len(frames)
+    ptrs = (C.c_void_p * max(n, 1))(*[f.data_ptr() for f in frames])
+    pitches = (C.c_int32 * max(n, 1))(*[f.stride(0) for f in frames])
+    _check(lib().ss_orb_extract_frames(ctx, n, ptrs, pitches, _ptr(d_kps), _ptr(d_desc), _ptr(d_counts),
+                                       _stream(stream)), ctx)
 
 
 def ss_brute_map_prepare(ctx, d_map_desc, n_map: int, stream=None) -> None:

@@ -1,7 +1,12 @@
-# c2 throughput vs ticks in flight
-mkdir -p gpurun_out
-python -c "from paper_conf_conext_dhakalrwcr22_b200 import build as b; b.build()"
-for P in 1 2 4 6 8 12; do
-  timeout 300 python bench.py --steps 200 --warmup 10 --no-cpu-baseline --inflight $P > gpurun_out/sweep_if$P.json 2>/dev/null
-  python -c "import json;d=json.loads([l for l in open('gpurun_out/sweep_if$P.json') if l.startswith('{')][-1]);print($P, round(d['value']), d['latency_ms']['p50'], round(d['e2e']['value']))"
+#!/bin/bash
+# Ticks-in-flight sweep of the c2 bench (one gpurun call).  Usage: bash scripts/sweep_inflight.sh [config]
+set -u
+OUT=gpurun_out; mkdir -p $OUT
+C=${1:-c2}
+python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
+for P in ${INFLIGHT:-3 4 5 6 8}; do
+  timeout 600 python bench.py --config $C --inflight $P --no-cpu-baseline > $OUT/sweep_${C}_p$P.json 2> $OUT/sweep_${C}_p$P.err
+  python -c "
+import json; d=json.loads(open('$OUT/sweep_${C}_p$P.json').read().strip().splitlines()[-1])
+print('P=$P', round(d['value']), 'steady', round(d['steady_state']['value']), 'p50', round(d['latency_ms']['p50'],4), 'iso', round(d['latency_ms']['isolated_tick_ms'],4))"
 done

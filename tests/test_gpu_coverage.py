@@ -335,3 +335,24 @@ def test_brute_prepared_map(torch_cuda, ref):
         ss.ss_match_projection(pipe.ctx, B, pipe.kps, pipe.desc, pipe.counts, None, 0, None, None, n_map,
                                ss.brute_cfg(), out, st)
     pipe.close()
+
+
+def test_extract_separately_allocated_frames(torch_cuda, ref):
+    """ss_orb_extract_frames (SURVEY §8(b)'s d_frames[] / pitches[] boundary): independently
+    allocated client frames with different pitches give the oracle's results bit for bit."""
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import OrbPipeline
+    w, h = synth.SHAPES["tum"]
+    p = ref.params(w, h, 1000)
+    frames = synth.make_frames(w, h, 3, cfg=33)
+    rk, rd, rc = ref.orb_extract_batch(p, frames)
+    bufs = []
+    for b, pitch in enumerate((w, w + 7, w + 64)):
+        t = torch.zeros((h, pitch), dtype=torch.uint8, device="cuda")
+        t[:, :w] = torch.from_numpy(frames[b]).cuda()
+        bufs.append(t)
+    pipe = OrbPipeline(w, h, 1000, 8, max_frames=3)
+    ss.ss_orb_extract_frames(pipe.ctx, bufs, pipe.kps, pipe.desc, pipe.counts, torch.cuda.current_stream())
+    _assert_same_extract(pipe, rk, rd, rc)
+    pipe.close()
