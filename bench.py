@@ -90,7 +90,11 @@ class HostStagedGather:
         import queue
 
         import torch
+        import torch.distributed as dist
         self.rank, self.world = rank, world
+        # a process group of its own: the worker thread's gathers must never interleave with
+        # the main thread's collectives (barriers, the timing all-reduce) on the default group
+        self.pg = dist.new_group(backend="gloo")
         self.bufs = [torch.empty(slot_bytes, dtype=torch.uint8).pin_memory() for _ in range(depth)]
         self.recv = [[torch.empty(slot_bytes, dtype=torch.uint8) for _ in range(world)] for _ in range(depth)]
         self.events = [torch.cuda.Event() for _ in range(depth)]
@@ -111,10 +115,10 @@ class HostStagedGather:
                 k = item
                 self.events[k].synchronize()
                 if self.rank == 0:
-                    dist.gather(self.bufs[k], self.recv[k], dst=0)
+                    dist.gather(self.bufs[k], self.recv[k], dst=0, group=self.pg)
                     self.last = [r.clone() for r in self.recv[k]]
                 else:
-                    dist.gather(self.bufs[k], None, dst=0)
+                    dist.gather(self.bufs[k], None, dst=0, group=self.pg)
             except Exception as e:  # pragma: no cover - surfaced by drain()
                 self.err = e
 
@@ -956,21 +960,18 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
         else:
             h2d = fr[0].numel() + sum(a.numel() for j, a in enumerate(hin[0]) if j != 5 or lf[0] > 0)
 
-        def step(s):
-            i, q = s % n_host, s % P
-            ss.ss_track_tick(pipes[q].ctx, B, cfg, ios[q][i], handles[q])
-
+        # the tick loop runs natively (ss_track_run: tick t = ss_track_tick on ctx t % P with
+        # io slot t % n_host), so the measurement is the library's, not the Python loop's
+        runner = ss.TrackRun([pp.ctx for pp in pipes], handles, B, cfg, ios)
         K = 1000  # ~60-100 ms of ticks: long enough that one host hiccup does not move the rate
-        for s in range(3 * n_host if reuse else 3):  # reuse: every (ctx, slot) graph captured before timing
-            step(s)
+        runner.run(3 * n_host if reuse else 3)  # reuse: every (ctx, slot) graph captured before timing
         torch.cuda.synchronize(dev)
         t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         t0.record(streams[0])
         for q in range(1, P):
             streams[q].wait_event(t0)
         h0 = time.perf_counter()
-        for s in range(K):
-            step(s)
+        runner.run(K)
         h1 = time.perf_counter()
         for q in range(1, P):
             streams[0].wait_stream(streams[q])
@@ -981,7 +982,8 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
                 "d2h_bytes_per_step": int(d2h), "steps": K, "ms_per_step": ms / K, "ticks_in_flight": P,
                 "host_us_per_call": 1e6 * (h1 - h0) / K}
 
-    path = ("one C-ABI call per tick: H2D, ss_orb_extract, " + ("ss_stereo_match, " if stereo else "") +
+    path = ("ss_track_run: one ss_track_tick per tick in native code: H2D, ss_orb_extract, " +
+            ("ss_stereo_match, " if stereo else "") +
             ("ss_match_last_frame, ss_project_points, ss_match_projection WINDOW" if window
              else "ss_match_projection BRUTE") + ", D2H of all outputs; no graphs")
     # raw pinned H2D bandwidth of one tick's frames, as seen by this process (diagnostic)

@@ -382,6 +382,14 @@ typedef struct {
 ss_status ss_track_tick(ss_ctx* ctx, int32_t n_frames, const ss_match_cfg* cfg, const ss_tick_io* io,
                         ss_stream_t stream);
 
+/* A server's tick loop in native code: n_ticks calls of ss_track_tick, tick t on ctxs[t %
+ * n_ctx] and streams[t % n_ctx] with ios[(t % n_ctx) * n_io + t % n_io] (HOST arrays; each
+ * ctx owns its own staging, so consecutive ticks on different ctxs / streams overlap: one
+ * tick's copies with another's kernels).  Same requirements, results and errors as the
+ * individual calls (stops at the first failing tick).  Asynchronous like ss_track_tick. */
+ss_status ss_track_run(ss_ctx* const* ctxs, int32_t n_ctx, const ss_stream_t* streams, int32_t n_frames,
+                       const ss_match_cfg* cfg, const ss_tick_io* ios, int32_t n_io, int32_t n_ticks);
+
 /* ---- profiling hook (bench.py; does not synchronise) ---- */
 
 /* When n_events > 0, every following ss_orb_extract / ss_match_projection records the

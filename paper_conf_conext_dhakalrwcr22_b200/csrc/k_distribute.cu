@@ -414,15 +414,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
   uint8_t* split = recch + DENSE_REC;                         // [DENSE_BINS / 4]
   // bins of depth r start at off(r) = nini (4^r - 1) / 3
   auto off = [&](int r) { return nini * (((1 << (2 * r)) - 1) / 3); };
-  {
-    const int o = off(R + 1);
-    for (int i = tid; i < o; i += DT) cnt[i] = 0u;
-    if (tid < 8) {
-      S_.H[tid] = 0;  // non-empty bins per depth
-      S_.G[tid] = 0;  // bins with >= 2 keys per depth
-    }
-  }
-  __syncthreads();  // bins zeroed before any increment
+  // the bins were zeroed (and S_.H / S_.G reset) at the kernel's start, before its first barrier
   SS_PHASE(3);
   // one pass over the keys in a scattered order (consecutive candidates share cells, hence
   // bins): key to depth R (+1 spare round), one increment per depth >= r_lo; the value an
@@ -446,18 +438,22 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
       }
     }
     __syncthreads();
+    // the few shallow bins (nini * (1 + 4 + 16)) by warp 0 alone, depth by depth with warp
+    // syncs instead of three block barriers; the barrier after the partials orders them
+    if (tid < 32) {
 #pragma unroll
-    for (int r = 2; r >= 0; r--) {  // r < r_lo <= 3; compile-time r keeps nz / mu in registers
-      if (r >= r_lo) continue;
-      const int sz = nini << (2 * r);
-      for (int b = tid; b < sz; b += DT) {
-        const uint32_t* ch = cnt + off(r + 1) + 4 * b;
-        const uint32_t c = ch[0] + ch[1] + ch[2] + ch[3];
-        cnt[off(r) + b] = c;
-        nz[r] += c > 0u;
-        mu[r] += c > 1u;
+      for (int r = 2; r >= 0; r--) {  // r < r_lo <= 3; compile-time r keeps nz / mu in registers
+        if (r >= r_lo) continue;
+        const int sz = nini << (2 * r);
+        for (int b = lane; b < sz; b += 32) {
+          const uint32_t* ch = cnt + off(r + 1) + 4 * b;
+          const uint32_t c = ch[0] + ch[1] + ch[2] + ch[3];
+          cnt[off(r) + b] = c;
+          nz[r] += c > 0u;
+          mu[r] += c > 1u;
+        }
+        __syncwarp();
       }
-      __syncthreads();
     }
 #pragma unroll
     for (int r = 0; r < 7; r++) {
@@ -661,6 +657,14 @@ __global__ void __launch_bounds__(DT, 1)
     }
     if (tid < 16) S_.H[tid] = 0;
     if (tid < 17) S_.G[tid] = 0;
+    {  // the dense path's per-depth bins, zeroed here so its first phase needs no barrier of
+       // its own (the region is past the candidate / key arrays; other paths overwrite it)
+      int R = 0;
+      while (R < 6 && g.nini[l] << (2 * (R + 1)) <= DENSE_BINS) R++;
+      uint32_t* bins = reinterpret_cast<uint32_t*>(sm + kSmemCells) + 2 * DCAP;
+      const int o = g.nini[l] * (((1 << (2 * (R + 1))) - 1) / 3);
+      for (int i = tid; i < o; i += DT) bins[i] = 0u;
+    }
     __syncthreads();
   }
   const int n = S_.sh[0];

@@ -1128,6 +1128,18 @@ ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, co
   return tick_enqueue(c, n_frames, cfg, io, s, stereo, window, lastf, n_lf);
 }
 
+ss_status ss_track_run(ss_ctx* const* ctxs, int32_t n_ctx, const ss_stream_t* streams, int32_t n_frames,
+                       const ss_match_cfg* cfg, const ss_tick_io* ios, int32_t n_io, int32_t n_ticks) {
+  if (!ctxs || !streams || !cfg || !ios || n_ctx < 1 || n_io < 1 || n_ticks < 0)
+    return fail(SS_EINVAL, "bad ss_track_run arguments");
+  for (int32_t t = 0; t < n_ticks; t++) {
+    const int q = t % n_ctx, i = t % n_io;
+    const ss_status st = ss_track_tick(ctxs[q], n_frames, cfg, &ios[(int64_t)q * n_io + i], streams[q]);
+    if (st != SS_OK) return st;
+  }
+  return SS_OK;
+}
+
 ss_status ss_profile_events(ss_ctx* c, void* const* events, int32_t n_events) {
   if (!c || n_events < 0 || (n_events > 0 && !events)) return fail(SS_EINVAL, "bad profiling events");
   for (int i = 0; i < n_events; i++)

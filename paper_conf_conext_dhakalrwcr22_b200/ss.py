@@ -111,6 +111,8 @@ def lib():
         L.ss_match_brute_merge.argtypes = [P, i32, P, i32, P, C.POINTER(ss_match_cfg), P, P]
         L.ss_brute_map_prepare.argtypes = [P, P, i32, P]
         L.ss_orb_extract_frames.argtypes = [P, i32, C.POINTER(P), C.POINTER(i32), P, P, P, P]
+        L.ss_track_run.argtypes = [C.POINTER(P), i32, C.POINTER(P), i32, C.POINTER(ss_match_cfg),
+                                   C.POINTER(ss_tick_io), i32, i32]
         L.ss_set_distribution.argtypes = [P, i32]
         L.ss_track_tick.argtypes = [P, i32, C.POINTER(ss_match_cfg), C.POINTER(ss_tick_io), P]
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
@@ -126,7 +128,7 @@ def lib():
                    "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_set_distribution",
                    "ss_match_last_frame", "ss_match_brute_partial", "ss_match_brute_merge", "ss_debug_level", "ss_debug_candidates", "ss_debug_overflow_count", "ss_profile_events",
                    "ss_profile_next", "ss_debug_phase_times", "ss_debug_distribution_paths", "ss_debug_match_lanes",
-                   "ss_debug_capture_samples", "ss_brute_map_prepare", "ss_orb_extract_frames"):
+                   "ss_debug_capture_samples", "ss_brute_map_prepare", "ss_orb_extract_frames", "ss_track_run"):
             getattr(L, fn).restype = C.c_int
         _lib = L
     return _lib
@@ -136,7 +138,8 @@ EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "s
             "ss_match_projection", "ss_project_points", "ss_stereo_match", "ss_track_tick", "ss_set_distribution",
             "ss_match_last_frame", "ss_match_brute_partial", "ss_match_brute_merge", "ss_profile_events", "ss_profile_next", "ss_debug_level",
             "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times", "ss_debug_distribution_paths",
-            "ss_debug_match_lanes", "ss_debug_capture_samples", "ss_brute_map_prepare", "ss_orb_extract_frames")
+            "ss_debug_match_lanes", "ss_debug_capture_samples", "ss_brute_map_prepare", "ss_orb_extract_frames",
+            "ss_track_run")
 
 
 def _check(status: int, ctx=None):
@@ -295,6 +298,22 @@ def ss_debug_overflow_count(ctx) -> int:
     n = C.c_int32()
     _check(lib().ss_debug_overflow_count(ctx, C.byref(n)), ctx)
     return n.value
+
+
+class TrackRun:
+    """Marshalled arguments of ss_track_run (built once, run many times): ctxs / streams [P],
+    ios [P][n_io] (ss_tick_io structures)."""
+
+    def __init__(self, ctxs, streams, n_frames: int, cfg: "ss_match_cfg", ios):
+        P, n_io = len(ctxs), len(ios[0])
+        self.ctxs = (C.c_void_p * P)(*ctxs)
+        self.streams = (C.c_void_p * P)(*[_stream(s) for s in streams])
+        self.ios = (ss_tick_io * (P * n_io))(*[io for row in ios for io in row])
+        self.cfg, self.n_frames, self.P, self.n_io = cfg, n_frames, P, n_io
+
+    def run(self, n_ticks: int) -> None:
+        _check(lib().ss_track_run(self.ctxs, self.P, self.streams, self.n_frames, C.byref(self.cfg), self.ios,
+                                  self.n_io, n_ticks))
 
 
 def ss_orb_extract_frames(ctx, frames, d_kps, d_desc, d_counts, stream=None):

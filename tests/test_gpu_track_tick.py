@@ -225,3 +225,46 @@ def test_track_tick_graph_reuse(torch_cuda, ref):
         want = ref.match_window(p, rk, rd, rc, None, q, qd)
         np.testing.assert_array_equal(o["matches"].numpy().view(ref.MATCH_DTYPE).reshape(-1), want)
     pipe.close()
+
+
+def test_track_run_native_loop(torch_cuda, ref):
+    """ss_track_run (the native tick loop): 6 ticks over 2 contexts x 3 io slots (graph reuse
+    on), each slot's outputs equal the oracle's extraction of its frames."""
+    torch = torch_cuda
+    from paper_conf_conext_dhakalrwcr22_b200 import ss
+    from paper_conf_conext_dhakalrwcr22_b200.pipeline import OrbPipeline
+    w, h = synth.SHAPES["tum"]
+    B, nf, P, NIO = 2, 1000, 2, 3
+    p = ref.params(w, h, nf)
+    cap = p.kp_capacity
+    frames = [synth.make_frames(w, h, B, cfg=80 + i) for i in range(NIO)]
+    pipes = [OrbPipeline(w, h, nf, 8, max_frames=B) for _ in range(P)]
+    streams = [torch.cuda.Stream() for _ in range(P)]
+    keep, ios = [], []
+    for q in range(P):
+        row = []
+        for i in range(NIO):
+            hf = torch.from_numpy(frames[i].reshape(-1).copy()).pin_memory()
+            hk = torch.zeros(B * cap * 20, dtype=torch.uint8).pin_memory()
+            hc = torch.zeros(B * 9 * 4, dtype=torch.uint8).pin_memory()
+            hd = torch.zeros(B * cap * 32, dtype=torch.uint8).pin_memory()
+            keep.append((hf, hk, hc, hd))
+            io = ss.ss_tick_io()
+            io.frames, io.frame_stride, io.pitch, io.reuse_graph = hf.data_ptr(), h * w, w, 1
+            io.kps, io.counts, io.desc = hk.data_ptr(), hc.data_ptr(), hd.data_ptr()
+            row.append(io)
+        ios.append(row)
+    run = ss.TrackRun([pp.ctx for pp in pipes], streams, B, ss.brute_cfg(), ios)
+    run.run(6)  # ticks t = 0..5: ctx t % 2, slot t % 3 -> every (ctx, slot) pair once
+    torch.cuda.synchronize()
+    for i in range(NIO):
+        rk, rd, rc = ref.orb_extract_batch(p, frames[i])
+        for q in range(P):
+            hf, hk, hc, hd = keep[q * NIO + i]
+            counts = hc.numpy().view(np.int32).reshape(B, 9)
+            kps = hk.numpy().reshape(B, cap, 20)
+            desc = hd.numpy().reshape(B, cap, 32)
+            # every (ctx q, slot i) pair ran exactly once: t < 6 with t % 2 == q, t % 3 == i (CRT)
+            _check_extract(p, kps, desc, counts, frames[i], ref)
+    for pp in pipes:
+        pp.close()
