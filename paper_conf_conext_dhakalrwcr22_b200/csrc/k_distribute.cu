@@ -425,19 +425,37 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
     int nz[7] = {0, 0, 0, 0, 0, 0, 0}, mu[7] = {0, 0, 0, 0, 0, 0, 0};
     uint32_t stride = 1031u;
     while ((uint32_t)n % stride == 0u) stride += 2u;  // an odd prime-ish step coprime with n
+    // only the deepest depth R takes atomics (its bins are sparse, so they rarely collide);
+    // depths r_lo .. R-1 are sums of their 4 children, formed level by level afterwards
+    int nzR = 0, muR = 0;
     for (int j = tid; j < n; j += DT) {
       const int i = (int)(((uint32_t)j * stride) % (uint32_t)n);  // j < 8192: no overflow
       const uint32_t k = make_key(g, l, cand[i], R + 1);
       key[i] = k;
-#pragma unroll
-      for (int r = 0; r < 7; r++) {
-        if (r < r_lo || r > R) continue;
-        const uint32_t old = atomicAdd(&cnt[off(r) + (int)(k >> (26 - 2 * r))], 1u);
-        nz[r] += old == 0u;
-        mu[r] += old == 1u;
-      }
+      const uint32_t old = atomicAdd(&cnt[off(R) + (int)(k >> (26 - 2 * R))], 1u);
+      nzR += old == 0u;
+      muR += old == 1u;
     }
+#pragma unroll
+    for (int r = 0; r < 7; r++)
+      if (r == R) {
+        nz[r] = nzR;
+        mu[r] = muR;
+      }
     __syncthreads();
+#pragma unroll
+    for (int r = 5; r >= 0; r--) {  // depths R-1 .. r_lo, block-parallel
+      if (r >= R || r < r_lo) continue;
+      const int sz = nini << (2 * r);
+      for (int b = tid; b < sz; b += DT) {
+        const uint32_t* ch = cnt + off(r + 1) + 4 * b;
+        const uint32_t c = ch[0] + ch[1] + ch[2] + ch[3];
+        cnt[off(r) + b] = c;
+        nz[r] += c > 0u;
+        mu[r] += c > 1u;
+      }
+      __syncthreads();
+    }
     // the few shallow bins (nini * (1 + 4 + 16)) by warp 0 alone, depth by depth with warp
     // syncs instead of three block barriers; the barrier after the partials orders them
     if (tid < 32) {
@@ -480,9 +498,11 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
   }
   __syncthreads();
   SS_PHASE(4);
-  if (tid == 0) {
-    // ORB-SLAM's loop on node counts (as in the sort path); -1 = a depth > R is needed
-    int D = -1, partial = 0, r = 0;
+  // ORB-SLAM's loop on node counts (as in the sort path); -1 = a depth > R is needed.  Every
+  // thread evaluates it (a handful of shared reads) instead of thread 0 + a barrier.
+  int D = -1, partial_i = 0;
+  {
+    int r = 0;
     for (;;) {
       if (r + 1 > R) break;
       const int nx = S_.H[r + 1];
@@ -492,7 +512,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
         for (;;) {
           if (d + 1 > R) { d = -1; break; }
           const int s2 = S_.H[d + 1];
-          if (s2 >= N) { partial = 1; break; }
+          if (s2 >= N) { partial_i = 1; break; }
           if (s2 == S_.H[d]) { d = d + 1; break; }
           d++;
         }
@@ -501,25 +521,13 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
       }
       r++;
     }
-    S_.sh[3] = D;
-    S_.sh[4] = partial;
-    S_.sh[1] = 0;  // records
-    S_.sh[2] = 0;  // kept keys
   }
-  __syncthreads();
-  const int D = S_.sh[3];
   SS_PHASE(5);
   if (D < 0) return false;
-  const bool partial = S_.sh[4] != 0;
+  const bool partial = partial_i != 0;
   const int szD = nini << (2 * D);
-  for (int b = tid; b < szD; b += DT) best0[b] = 0u;
+  // best0 / best1 / first / split were initialised at the kernel's start (S_.sh[1], [2] = 0 too)
   if (partial) {
-    for (int b = tid; b < 4 * szD; b += DT) best1[b] = 0u;
-    for (int b = tid; b < szD; b += DT) {
-      first[b] = 0xFFFFFFFFu;
-      split[b] = 0;
-    }
-    __syncthreads();
     for (int i = tid; i < n; i += DT) atomicMin(&first[key[i] >> (26 - 2 * D)], (uint32_t)i);
     __syncthreads();
     // the multi-key nodes at depth D, ordered by (size desc, UL.y, UL.x, first-key rank)
@@ -664,6 +672,16 @@ __global__ void __launch_bounds__(DT, 1)
       uint32_t* bins = reinterpret_cast<uint32_t*>(sm + kSmemCells) + 2 * DCAP;
       const int o = g.nini[l] * (((1 << (2 * (R + 1))) - 1) / 3);
       for (int i = tid; i < o; i += DT) bins[i] = 0u;
+      // best0 [DENSE_BINS], best1 [DENSE_BINS], first [DENSE_BINS / 4] (= none), split bytes
+      uint32_t* b0 = bins + DENSE_TOTAL;
+      for (int i = tid; i < 2 * DENSE_BINS; i += DT) b0[i] = 0u;
+      for (int i = tid; i < DENSE_BINS / 4; i += DT) b0[2 * DENSE_BINS + i] = 0xFFFFFFFFu;
+      // split = recch + DENSE_REC, recch = order + DENSE_REC ... as laid out in dense_body
+      const uint64_t* rec = reinterpret_cast<const uint64_t*>(b0 + 2 * DENSE_BINS + DENSE_BINS / 4);
+      const int32_t* recnode = reinterpret_cast<const int32_t*>(rec + DENSE_REC);
+      const int32_t* order = recnode + DENSE_REC;
+      uint8_t* spl = const_cast<uint8_t*>(reinterpret_cast<const uint8_t*>(order + DENSE_REC)) + DENSE_REC;
+      for (int i = tid; i < DENSE_BINS / 4; i += DT) spl[i] = 0;
     }
     __syncthreads();
   }
