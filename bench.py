@@ -512,6 +512,8 @@ def run_ours(args, cfg):
                                   max_map=cfg["map"], device=local) for _ in range(P - 1)]
     for pp in pipes:
         pp.set_distribution(dist_mode)
+        if args.match_lanes:
+            ss.ss_debug_match_lanes(pp.ctx, args.match_lanes)
         if not window and pp is not pipe:
             pp.prepare_map(map_desc)
     outs = [out] + [torch.zeros_like(out) for _ in range(P - 1)]
@@ -1198,6 +1200,8 @@ def main(argv=None):
                     help="N > 1: NCCL gather on a side stream, or gloo with host-staged slots (ranks may share a GPU)")
     ap.add_argument("--same-device", action="store_true", help="every rank on cuda:0 (multi-rank test on one GPU)")
     ap.add_argument("--clients", type=int, default=0, help="override the config's clients per rank")
+    ap.add_argument("--match-lanes", type=int, default=0, choices=[0, 1, 2, 4, 8],
+                    help="lanes per WINDOW query (0 = chosen per launch)")
     ap.add_argument("--dump-gather", default="", help="write the last tick's gathered / own slots to PATH.*.npy")
     ap.add_argument("--dist", choices=["quadtree", "grid"], default="quadtree",
                     help="keypoint distribution: ORB-SLAM quadtree (O4) or grid top-N (O4g)")

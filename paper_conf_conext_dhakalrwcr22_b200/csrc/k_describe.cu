@@ -117,8 +117,13 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
   // Constant inputs (set at ss_create) are read before the dependency wait, overlapping the
   // predecessor kernel's tail.  Lane = output byte: its 8 pairs are the 32 pattern bytes
   // 32 * lane .. 32 * lane + 31, one word (px0, py0, px1, py1) per bit, held in registers.
-  const uint4 pa = __ldg(reinterpret_cast<const uint4*>(pattern) + 2 * lane);
-  const uint4 pb = __ldg(reinterpret_cast<const uint4*>(pattern) + 2 * lane + 1);
+  // the lane's 16 pattern points as floats in shared memory, point j of lane at [j][lane]
+  // (conflict-free LDS.64): point 2t + e of output byte `lane` is pattern point 16 lane + j
+  __shared__ float2 s_pat[16 * 32];
+  for (int i = threadIdx.x; i < 16 * 32; i += DESC_WARPS * 32) {
+    const int ln = i & 31, j = i >> 5, pt = 16 * ln + j;
+    s_pat[i] = make_float2((float)__ldg(pattern + 2 * pt), (float)__ldg(pattern + 2 * pt + 1));
+  }
   if (threadIdx.x < 256) {  // byte j = u + 15 of row |v|: inside the disk -> (1, u + 15), else 0
     const int t = threadIdx.x >> 7, av = (threadIdx.x >> 3) & 15, k = threadIdx.x & 7;
     uint32_t word = 0;
@@ -283,7 +288,6 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
   const float inv_r = r2 ? rsqrtf((float)r2) : 0.f;
   // r2 == 0 (no rotation): (cs, sn) = (1, 0) gives t = px, py exactly, never near a tie
   const float cs = r2 ? (float)m10 * inv_r : 1.f, sn = r2 ? (float)m01 * inv_r : 0.f;  // |m| < 2^24: exact
-  const uint32_t pw[8] = {pa.x, pa.y, pa.z, pa.w, pb.x, pb.y, pb.z, pb.w};
   // horizontal pass at one sample: the 7 V values v0..v6 from the 4 words covering them
   // (funnel shift by 16 when they start at an odd u16; V is word aligned, the 4th word may be
   // the padding after V), weighted by dp2a on 16-bit pairs (v <= 65280, weights < 256)
@@ -310,13 +314,13 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
     int v[2];
 #pragma unroll
     for (int e = 0; e < 2; e++) {
-      // signed bytes 2e (x) and 2e + 1 (y) of the pair's word
-      const int px = (int)(pw[t] << (24 - 16 * e)) >> 24, py = (int)(pw[t] << (16 - 16 * e)) >> 24;
-      const float tx = __fmaf_rn((float)px, cs, __fmul_rn((float)-py, sn));  // (px m10 - py m01) / r
-      const float ty = __fmaf_rn((float)px, sn, __fmul_rn((float)py, cs));   // (px m01 + py m10) / r
+      const float2 pp = s_pat[(2 * t + e) * 32 + lane];  // exact small integers
+      const float tx = __fmaf_rn(pp.x, cs, __fmul_rn(-pp.y, sn));  // (px m10 - py m01) / r
+      const float ty = __fmaf_rn(pp.x, sn, __fmul_rn(pp.y, cs));   // (px m01 + py m10) / r
       const float bx = __fadd_rn(tx, 12582912.0f), by = __fadd_rn(ty, 12582912.0f);
       const float dx = __fsub_rn(tx, __fsub_rn(bx, 12582912.0f)), dy = __fsub_rn(ty, __fsub_rn(by, 12582912.0f));
-      near |= (fabsf(fabsf(dx) - 0.5f) <= 1e-4f) | (fabsf(fabsf(dy) - 0.5f) <= 1e-4f);
+      // |d| <= 1/2 always (t minus its nearest integer): a near-tie is |d| >= 1/2 - 1e-4
+      near |= (fabsf(dx) >= 0.4999f) | (fabsf(dy) >= 0.4999f);
       v[e] = blurred(__float_as_int(bx) - 0x4B400000, __float_as_int(by) - 0x4B400000);
       if (SAMPLES) smp[2 * t + e] = (uint8_t)v[e];
     }

@@ -252,12 +252,14 @@ cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* 
                                 const uint8_t* qdesc, ss_match_cfg cfg, unsigned long long* claim, ss_match* out,
                                 const uint16_t* rowidx, int lanes, cudaStream_t s) {
   if (n_queries <= 0) return cudaSuccess;
-  // lanes per query: enough groups to fill ~2 waves of the GPU (148 SMs x 2048 threads); a
-  // query's window holds a handful of candidates, so with many queries fewer lanes per query
-  // (less redundant per-query work) win: c3 (800 k queries) 1-2 lanes, c2 (20 k) 8
-  // (measured c3: 8 lanes 130 us, 4: 97, 2: 83, 1: 64)
+  // lanes per query: the fewest that still give 1/16 of a wave of the GPU (148 SMs x 2048
+  // threads).  A query's window holds a handful of candidates (0.13 on c2), so extra lanes
+  // mostly repeat the per-query work: with several ticks in flight (throughput) fewer lanes
+  // win even where the kernel alone gets slower.  Measured (scripts/sweep_lanes.sh): c2 (20 k
+  // queries) 1 lane 78.9k vs 8 lanes 76.0k frames/s (steady state), c1 (5 k) 2 lanes 22.9k vs
+  // 8 lanes 22.1k; c3 (800 k) 8 lanes 130 us, 4: 97, 2: 83, 1: 64 per launch.
   int wg = 8;
-  const int64_t want = 2LL * 148 * 2048;
+  const int64_t want = 148LL * 2048 / 16;
   while (wg > 1 && (int64_t)n_queries * (wg / 2) >= want) wg /= 2;
   if (lanes == 1 || lanes == 2 || lanes == 4 || lanes == 8) wg = lanes;  // test hook override
   auto kern = wg == 1 ? match_window_kernel<1> : wg == 2 ? match_window_kernel<2> : wg == 4 ? match_window_kernel<4>
