@@ -556,7 +556,7 @@ def run_ours(args, cfg):
         # concurrently with the extraction; measured on c2 with 4 ticks in flight that cost 7 %
         # of throughput (63.0k -> 58.9k frames/s), so the ring graphs keep it serial (the
         # per-tick executor ss_track_tick forks it: +1-2 % there)
-        fork = False
+        fork = bool(args.fork_project) and window and not prof
         with torch.cuda.graph(g, stream=st):
             if fork:
                 ev0, ev1 = torch.cuda.Event(), torch.cuda.Event()
@@ -1200,6 +1200,8 @@ def main(argv=None):
                     help="N > 1: NCCL gather on a side stream, or gloo with host-staged slots (ranks may share a GPU)")
     ap.add_argument("--same-device", action="store_true", help="every rank on cuda:0 (multi-rank test on one GPU)")
     ap.add_argument("--clients", type=int, default=0, help="override the config's clients per rank")
+    ap.add_argument("--fork-project", type=int, default=0, choices=[0, 1],
+                    help="ring graphs: run the local-map projection on a forked branch concurrent with the extraction")
     ap.add_argument("--match-lanes", type=int, default=0, choices=[0, 1, 2, 4, 8],
                     help="lanes per WINDOW query (0 = chosen per launch)")
     ap.add_argument("--dump-gather", default="", help="write the last tick's gathered / own slots to PATH.*.npy")

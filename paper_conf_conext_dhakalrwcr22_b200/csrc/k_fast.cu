@@ -29,9 +29,16 @@ namespace ss {
 
 namespace {
 
-constexpr int FB_WARPS = 8;
+#ifndef SS_FAST_WARPS
+#define SS_FAST_WARPS 8
+#endif
+#ifndef SS_FAST_ROWS
+#define SS_FAST_ROWS 8
+#endif
+constexpr int FB_WARPS = SS_FAST_WARPS;
 constexpr int FB_THREADS = FB_WARPS * 32;
-constexpr int ROWS_PER_TASK = 8;
+constexpr int ROWS_PER_TASK = SS_FAST_ROWS;  // rows per score task (sliding 7-row window)
+constexpr int FB_MIN_BLOCKS = 24 / FB_WARPS > 1 ? 24 / FB_WARPS : 1;  // 80 registers
 
 // The band is staged with every byte XOR 0x80, so a byte read as a signed char is I - 128
 // (order preserving).  A PRMT whose selector nibbles set the sign-replicate bit turns two
@@ -135,7 +142,7 @@ __device__ __forceinline__ uint32_t nibble4(uint32_t h0, uint32_t h1) {
   return (t | (t >> 14)) & 0xFu;
 }
 
-__global__ void __launch_bounds__(FB_THREADS, 3) fast_bands_kernel(const __grid_constant__ Geom g, FrameSrc src,
+__global__ void __launch_bounds__(FB_THREADS, FB_MIN_BLOCKS) fast_bands_kernel(const __grid_constant__ Geom g, FrameSrc src,
                                                                 const BandInfo* __restrict__ bands,
                                                                 const CellInfo* __restrict__ cells,
                                                                 uint32_t* __restrict__ slots,

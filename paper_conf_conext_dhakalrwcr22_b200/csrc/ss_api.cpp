@@ -366,7 +366,11 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   // FAST work units: runs of <= kSegCells consecutive cells of one row (same level and detect
   // rows; their windows tile [x0, x1)), biggest levels first in the grid.  8 measured best
   // on B200 (c2: 2..24 swept; smaller runs pay more halo, larger ones lose parallelism).
-  const int kSegCells = 8;
+  // level 0: runs of <= 4 (168 -> 336 CTAs for 4 EuRoC frames: the 8-cell runs left 20 SMs with two
+  // CTAs and the rest idle half the launch; fast_l0 18.2 -> 15.6 us, scripts/sweep_seg.sh)
+  int kSegCells = 8, kSegCells0 = 4;  // levels >= 1 / level 0 (SS_SEG / SS_SEG0 override: experiments)
+  if (const char* e = std::getenv("SS_SEG")) kSegCells = imax(1, std::atoi(e));
+  if (const char* e = std::getenv("SS_SEG0")) kSegCells0 = imax(1, std::atoi(e));
   g.max_band_w = g.max_band_h = g.max_cell_w = 0;
   // a row of n cells is cut into nseg = ceil(n / S) near-equal runs: cell k of the row goes
   // to run floor(k * nseg / n)
@@ -375,7 +379,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     size_t r1 = r0;
     while (r1 < c->cells_h.size() && c->cells_h[r1].level == c->cells_h[r0].level && c->cells_h[r1].y0 == c->cells_h[r0].y0)
       r1++;
-    const int n = (int)(r1 - r0), S = kSegCells;
+    const int n = (int)(r1 - r0), S = c->cells_h[r0].level == 0 ? kSegCells0 : kSegCells;
     const int nseg = (n + S - 1) / S;
     for (int k = 0; k < n; k++) run_of[r0 + k] = (int)((int64_t)k * nseg / n);
     r0 = r1;
@@ -448,9 +452,24 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     return fail(SS_EUNSUPPORTED, "scale_factor above 4/3 is not supported by the pyramid kernel");
   }
   // fused pyramid: blocks of about 128 x 96 level-0 pixels (more, smaller blocks if a
-  // block does not fit)
+  // block does not fit).  One 1024-thread CTA per SM: while a full batch (max_frames) still
+  // fits in one wave, smaller blocks shorten the launch (at most 2x the blocks per axis; c2:
+  // 6x5 -> 6x6 blocks for 4 frames, 17.9 -> 16.3 us, scripts/sweep_pyr.sh)
   if (L > 1) {
     int gx = (g.w[0] + 127) / 128, gy = (g.h[0] + 95) / 96;
+    {
+      int nsm = 0;
+      if (cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, device) != cudaSuccess || nsm < 1) nsm = 148;
+      const int gx0 = gx, gy0 = gy;
+      for (;;) {
+        const int nx = gy >= gx ? gx + 1 : gx, ny = gy >= gx ? gy : gy + 1;
+        if ((int64_t)max_frames * nx * ny > nsm || nx > 2 * gx0 || ny > 2 * gy0) break;
+        gx = nx;
+        gy = ny;
+      }
+    }
+    if (const char* e = std::getenv("SS_PYR_GX")) gx = imax(1, std::atoi(e));  // experiments
+    if (const char* e = std::getenv("SS_PYR_GY")) gy = imax(1, std::atoi(e));
     while (!pyramid_plan(g, tab.data(), c->xoff.data(), c->yoff.data(), goff, gx, gy, &plan, &c->pyr_buf0,
                          &c->pyr_buf1, &c->pyr_smem)) {
       if (gx >= g.w[L - 1] / 4 || gy >= g.h[L - 1]) {

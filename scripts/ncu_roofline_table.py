@@ -5,6 +5,7 @@ utilisation for the matchers).
 usage: python scripts/ncu_roofline_table.py OUT.json REPORT.ncu-rep [REPORT2.ncu-rep ...]
 Peaks: MEASURED_PEAKS.json hbm_gbs when present (else the B200_PROFILING.md fallback)."""
 import csv
+import re
 import io
 import json
 import os
@@ -44,7 +45,10 @@ def main():
         hdr, units = r[0], r[1]
         for row in r[2:]:
             d = dict(zip(hdr, row))
-            name = d["Kernel Name"].split("(")[0].split("::")[-1]
+            full = d["Kernel Name"].replace("(anonymous namespace)", "anon").replace("<unnamed>", "anon")
+            while re.search(r"<[^<>]*>", full):  # template arguments, e.g. describe_kernel<(bool)0>
+                full = re.sub(r"<[^<>]*>", "", full)
+            name = full.split("(")[0].split("::")[-1]
             rec = {}
             for k, m in M.items():
                 if m not in d or d[m] in ("", "n/a", "no data"):

@@ -34,7 +34,9 @@ def main():
     launches = []
     for r in rows[2:]:
         d = dict(zip(hdr, r))
-        name = d["Kernel Name"].split("(")[0].split("::")[-1]
+        full = d["Kernel Name"]
+        hits = [k for k in SHORT if k in full]  # template instances, e.g. describe_kernel<(bool)0>
+        name = max(hits, key=len) if hits else full.split("(")[0].split("::")[-1]
         rec = {"kernel": SHORT.get(name, name)}
         for m in METRICS:
             u = units[hdr.index(m)]
