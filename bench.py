@@ -789,7 +789,9 @@ def run_ours(args, cfg):
         for r_ in rooflines:
             if r_["kernel"] == "match_window":
                 r_["popc"] = popc
-    traffic_file = os.path.join(ROOT, "profiles", "dram_traffic_r01.json")
+    traffic_file = os.path.join(ROOT, "profiles", "dram_traffic_r02.json")
+    if not os.path.exists(traffic_file):
+        traffic_file = os.path.join(ROOT, "profiles", "dram_traffic_r01.json")
     if os.path.exists(traffic_file):
         try:
             with open(traffic_file) as f:
@@ -797,6 +799,7 @@ def run_ours(args, cfg):
             trs = [tab.get(n_) for n_ in members]
             if all(t_ is not None for t_ in trs):
                 roof["traffic"] = sum(trs)  # DRAM bytes of the roofline's launches (ncu, per step)
+                roof["traffic_src"] = os.path.relpath(traffic_file, ROOT)
         except Exception:
             pass
 

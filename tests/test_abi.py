@@ -78,3 +78,14 @@ def test_product_does_not_import_oracle():
                 txt = open(os.path.join(dirpath, fn)).read()
                 assert "import oracle" not in txt and "from oracle" not in txt, fn
                 assert "ss_oracle" not in txt and "brief_pattern_ref" not in txt, fn
+
+
+def test_new_entry_points_reject_bad_args(sslib):
+    """Round-2 entry points validate before touching the GPU."""
+    L = sslib.lib()
+    assert L.ss_track_run(None, 0, None, 1, None, None, 0, 1) == sslib.SS_EINVAL
+    assert L.ss_brute_map_prepare(None, None, 10, None) == sslib.SS_EINVAL
+    assert L.ss_orb_extract_frames(None, 1, None, None, None, None, None, None) == sslib.SS_EINVAL
+    assert L.ss_debug_match_lanes(None, 3) == sslib.SS_EINVAL
+    assert L.ss_debug_capture_samples(None, None) == sslib.SS_EINVAL
+    assert L.ss_debug_distribution_paths(None, None, None) == sslib.SS_EINVAL
