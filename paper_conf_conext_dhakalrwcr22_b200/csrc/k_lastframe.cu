@@ -3,10 +3,12 @@
 // "ORB-Matching" step of the paper's tracking breakdown (§5, Fig. 8;
 // DESIGN.md §3 item 14, include/ss.h ss_match_last_frame).
 //
-// ONE launch for the whole step: a thread-block cluster of kCluster CTAs per frame.  The step
-// has three frame-wide dependencies (the dedup of keypoints claimed by several points, the
-// rotation histogram's three maxima, and the "fewer than min_matches -> redo with 2*th"
-// retry), which are cluster barriers here instead of kernel boundaries:
+// ONE launch for the whole step: one 1024-thread CTA per frame (kCluster = 1, the default; a
+// build with SS_LF_CLUSTER=8 spreads a frame over a thread-block cluster of 8 x 512 threads
+// with DSMEM histograms instead).  The step has three frame-wide dependencies (the dedup of
+// keypoints claimed by several points, the rotation histogram's three maxima, and the "fewer
+// than min_matches -> redo with 2*th" retry), which are block (or cluster) barriers here
+// instead of kernel boundaries:
 //   P0  every CTA stages the frame's keypoint positions and builds its row index (first
 //       keypoint per (level, row)) in shared memory; claims reset; the cluster also writes
 //       the window matcher's global row index and resets its claims (match_prepare's work,
@@ -33,9 +35,18 @@ namespace ss {
 
 namespace {
 
-constexpr int kCluster = 8;    // CTAs per frame (portable cluster size)
-constexpr int kThreads = 512;   // per CTA (16 warps)
-constexpr int kLanes = 4;      // lanes per point in P1
+#ifndef SS_LF_CLUSTER
+#define SS_LF_CLUSTER 1
+#endif
+constexpr int kCluster = SS_LF_CLUSTER;           // CTAs per frame (1: one CTA, block barriers)
+#ifndef SS_LF_THREADS
+#define SS_LF_THREADS 1024
+#endif
+constexpr int kThreads = SS_LF_THREADS;  // per CTA
+#ifndef SS_LF_LANES
+#define SS_LF_LANES 1
+#endif
+constexpr int kLanes = SS_LF_LANES;  // lanes per point in P1
 constexpr int kHisto = 30;     // ORB-SLAM HISTO_LENGTH
 constexpr size_t kLfSmemMax = 200 * 1024;
 
@@ -77,13 +88,18 @@ struct LfArgs {
   int rows_per_frame;
 };
 
-__global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
+// frame-wide barrier: the cluster's when a frame spans several CTAs, else the block's
+__device__ __forceinline__ void frame_sync() {
+  if constexpr (kCluster > 1) cg::this_cluster().sync();
+  else __syncthreads();
+}
+
+__global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
   __shared__ int s_hist[2][32];
   __shared__ int s_count[2];
   __shared__ int s_keep[3];
   __shared__ int s_roff[kMaxLevels];
-  cg::cluster_group cluster = cg::this_cluster();
-  const int rank = (int)cluster.block_rank();
+  const int rank = kCluster > 1 ? (int)cg::this_cluster().block_rank() : 0;
   const int f = blockIdx.x / kCluster;
   const int ct = rank * kThreads + threadIdx.x, nct = kCluster * kThreads;
   const Geom& g = a.g;
@@ -93,21 +109,37 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
   if (threadIdx.x < kMaxLevels) s_roff[threadIdx.x] = threadIdx.x < a.g.L ? row_off(a.g, threadIdx.x) : 0;
   pdl_wait();
   pdl_trigger();
-  int* lead_hist = cluster.map_shared_rank(&s_hist[0][0], 0);
-  int* lead_count = cluster.map_shared_rank(&s_count[0], 0);
+  int* lead_hist = &s_hist[0][0];
+  int* lead_count = &s_count[0];
+  if constexpr (kCluster > 1) {
+    lead_hist = cg::this_cluster().map_shared_rank(&s_hist[0][0], 0);
+    lead_count = cg::this_cluster().map_shared_rank(&s_count[0], 0);
+  }
 
   const ss_keypoint* fk = a.kps + (int64_t)f * cap;
   const int32_t* cnt = a.counts + f * (L + 1);
   // every CTA keeps its own copy of the frame's keypoint positions and row index in shared
-  // memory, so the window walk of P1 touches global memory only for descriptors
-  extern __shared__ float2 s_xy[];                                        // [cap]
-  uint16_t* fri = reinterpret_cast<uint16_t*>(s_xy + cap);                // [rows_per_frame]
+  // memory; with one CTA per frame also the descriptors and the taken mask, so the window
+  // walk of P1 never waits on global memory (a cluster CTA reads descriptors from L2)
+  extern __shared__ __align__(16) uint4 s_dyn[];
+  uint4* s_desc = s_dyn;                                                          // [cap][2] (kCluster == 1)
+  float2* s_xy = reinterpret_cast<float2*>(s_dyn + (kCluster == 1 ? 2 * cap : 0));  // [cap]
+  uint16_t* fri = reinterpret_cast<uint16_t*>(s_xy + cap);                        // [rows_per_frame]
+  uint8_t* s_taken = reinterpret_cast<uint8_t*>(fri + a.rows_per_frame);          // [cap] (kCluster == 1)
   unsigned long long* fclaim = a.claim + (int64_t)f * cap;
   uint8_t* fmask = a.matched ? a.matched + (int64_t)f * cap : nullptr;
   const int nk = cnt[L];
+  const uint4* gdesc = reinterpret_cast<const uint4*>(a.desc + (int64_t)f * cap * SS_DESC_BYTES);
   for (int k = threadIdx.x; k < cap; k += kThreads) {  // P0
     rowidx_fill(g, fk, cnt, fri, k);
     if (k < nk) s_xy[k] = make_float2(fk[k].x, fk[k].y);
+    if constexpr (kCluster == 1) {
+      if (k < nk) {
+        s_desc[2 * k] = gdesc[2 * k];
+        s_desc[2 * k + 1] = gdesc[2 * k + 1];
+      }
+      s_taken[k] = a.taken ? a.taken[(int64_t)f * cap + k] : 0;
+    }
   }
   for (int k = ct; k < cap; k += nct) {
     fclaim[k] = ~0ull;
@@ -117,7 +149,7 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
       a.win_claim[(int64_t)f * cap + k] = ~0ull;
     }
   }
-  cluster.sync();
+  frame_sync();
 
   const ss_camera& c = a.cams[f];
   int dir = 0;  // 1 = forward [o, L-1], 2 = backward [0, o], 0 = [o-1, o+1]
@@ -127,8 +159,8 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
     dir = tz > a.mb ? 1 : (-tz > a.mb ? 2 : 0);
   }
   const int i0 = a.pt_off[f], i1 = a.pt_off[f + 1];
-  const uint4* fd = reinterpret_cast<const uint4*>(a.desc + (int64_t)f * cap * SS_DESC_BYTES);
-  const uint8_t* ft = a.taken ? a.taken + (int64_t)f * cap : nullptr;
+  const uint4* fd = kCluster == 1 ? s_desc : gdesc;
+  const uint8_t* ft = kCluster == 1 ? (a.taken ? s_taken : nullptr) : (a.taken ? a.taken + (int64_t)f * cap : nullptr);
   const int sub = threadIdx.x % kLanes;
   const unsigned gmask = ((1u << kLanes) - 1u) << ((threadIdx.x & 31) & ~(kLanes - 1));
   int kept = 0;
@@ -190,7 +222,7 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
           atomicMin(fclaim + m.idx, tag | ((unsigned long long)m.dist << 32) | (unsigned)(i - i0));
       }
     }
-    cluster.sync();
+    frame_sync();
     // P2: dedup (min (distance, point) per keypoint) + rotation histogram
     for (int i = i0 + ct; i < i1; i += nct) {
       const ss_match m = a.out[i];
@@ -204,7 +236,7 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
         atomicAdd(lead_count + pass, 1);
       }
     }
-    cluster.sync();
+    frame_sync();
     // P3: ComputeThreeMaxima, reject the other bins, count the survivors
     if (a.check_orientation) {
       if (threadIdx.x == 0) {
@@ -244,7 +276,7 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
         else
           atomicAdd(lead_count + pass, 1);
       }
-      cluster.sync();
+      frame_sync();
     }
     kept = lead_count[pass];
     if (a.min_matches <= 0 || kept >= a.min_matches) break;  // uniform over the cluster
@@ -255,7 +287,7 @@ __global__ void __cluster_dims__(kCluster, 1, 1) __launch_bounds__(kThreads) las
       const int idx = a.out[i].idx;
       if (idx >= 0) fmask[idx] = 1;
     }
-  cluster.sync();  // the leader's shared memory must outlive every remote access
+  frame_sync();  // the leader's shared memory must outlive every remote access
 }
 
 }  // namespace
@@ -265,7 +297,8 @@ cudaError_t lastframe_init() {  // at ss_create (never inside a stream capture)
 }
 
 size_t lastframe_smem_bytes(const Geom& g) {
-  return sizeof(float2) * (size_t)g.kp_capacity + sizeof(uint16_t) * (size_t)match_rows_per_frame(g);
+  const size_t base = sizeof(float2) * (size_t)g.kp_capacity + sizeof(uint16_t) * (size_t)match_rows_per_frame(g);
+  return kCluster == 1 ? base + (size_t)SS_DESC_BYTES * g.kp_capacity + (size_t)g.kp_capacity : base;
 }
 
 cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams, const ss_camera* last_cams, float mb,
@@ -280,7 +313,26 @@ cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams,
            min_matches, out, n_matches, matched, claim, rowidx, win_claim, match_rows_per_frame(g)};
   const size_t smem = lastframe_smem_bytes(g);
   if (smem > kLfSmemMax) return cudaErrorInvalidValue;
-  cudaError_t e = launch_pdl(lastframe_kernel, dim3(n_frames * kCluster), dim3(kThreads), smem, s, a);
+  cudaError_t e;
+  if constexpr (kCluster > 1) {  // a thread-block cluster per frame (+ programmatic serialisation)
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(n_frames * kCluster);
+    cfg.blockDim = dim3(kThreads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[2];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = kCluster;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[1].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 2;
+    e = cudaLaunchKernelEx(&cfg, lastframe_kernel, a);
+  } else {
+    e = launch_pdl(lastframe_kernel, dim3(n_frames), dim3(kThreads), smem, s, a);
+  }
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 
