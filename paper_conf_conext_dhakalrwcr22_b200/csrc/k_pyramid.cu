@@ -21,7 +21,7 @@ namespace ss {
 namespace {
 
 #ifndef SS_PYR_THREADS
-#define SS_PYR_THREADS 1024
+#define SS_PYR_THREADS 256
 #endif
 constexpr int PT = SS_PYR_THREADS;  // threads per CTA (a block of every level per CTA)
 
@@ -66,7 +66,10 @@ __device__ __forceinline__ uint32_t lerp4(const uint8_t* r0, const uint8_t* r1, 
   return __byte_perm(__byte_perm(a[0], a[1], 0x0062), __byte_perm(a[2], a[3], 0x0062), 0x5410);
 }
 
-__global__ void __launch_bounds__(PT, 1) pyramid_fused_kernel(const __grid_constant__ Geom g, FrameSrc src,
+#ifndef SS_PYR_MINB
+#define SS_PYR_MINB 1
+#endif
+__global__ void __launch_bounds__(PT, SS_PYR_MINB) pyramid_fused_kernel(const __grid_constant__ Geom g, FrameSrc src,
                                                               const uint4* __restrict__ gtab,
                                                               const uint32_t* __restrict__ ytab,
                                                               const PyrLvl* __restrict__ plan, int buf0_bytes,
