@@ -156,6 +156,7 @@ struct ss_ctx {
   PatchMaps maps{};                  // TMA maps of the describe kernel (levels >= 1 at ss_create)
   // test hooks: lanes per WINDOW query (0 = chosen per launch), blurred-sample capture buffer
   int win_lanes = 0;
+  bool tick_fork = true;  // ss_track_tick: local-map projection on the aux branch (SS_TICK_FORK=0: serial)
   uint8_t* dbg_samples = nullptr;
   int32_t* stereo_sad = nullptr;  // O12: accepted SAD per left keypoint [max_frames/2][cap]
   // ss_track_tick staging (device copies of the host inputs / outputs of a tick)
@@ -291,6 +292,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (!c) return fail(SS_ECUDA, "host allocation failed");
   c->device = device;
   c->p = q;
+  if (const char* e = std::getenv("SS_TICK_FORK")) c->tick_fork = std::atoi(e) != 0;
   c->max_frames = max_frames;
   c->max_queries = max_queries;
   c->max_map = max_map;
@@ -985,7 +987,7 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
   // profiling events are installed, which time every kernel alone on `stream`) it forks onto
   // the ctx's aux stream and overlaps the extraction; the WINDOW match joins it.
   ss_status st;
-  const bool fork_project = window && c->prof.empty();
+  const bool fork_project = window && c->prof.empty() && c->tick_fork;
   if (fork_project) {
     SS_CUDA_TRY(cudaEventRecord(c->ev_aux0, s));
     SS_CUDA_TRY(cudaStreamWaitEvent(c->aux, c->ev_aux0, 0));
