@@ -621,30 +621,56 @@ __global__ void __launch_bounds__(DT, 1)
                       int32_t* __restrict__ sel_counts, uint8_t* ovf, int64_t ovf_frame_bytes,
                       const int64_t* __restrict__ ovf_level_off, int32_t* ovf_counter, int level0,
                       uint64_t* phase_base) {
-  pdl_wait();
-  pdl_trigger();
   extern __shared__ __align__(16) uint8_t sm[];
   __shared__ Shared S_;
   const int l = level0 + blockIdx.x, f = blockIdx.y, tid = threadIdx.x;
   uint64_t* phase_ts = phase_base ? phase_base + ((int64_t)f * g.L + l) * 16 : nullptr;
-  SS_PHASE(0);
   const int ncells = g.ncells[l];
   const int c0 = g.cell_first[l];
   int32_t* cell_off = reinterpret_cast<int32_t*>(sm);
   int32_t* cell_slot = cell_off + MAX_CELLS + 1;
   const int32_t* cc = cell_counts + (int64_t)f * g.total_cells + c0;
+  // Work that does not depend on the FAST kernel runs before the dependency wait, overlapping
+  // its tail: the static cell table's slot offsets and the dense path's table initialisation.
+  const int cpt = (ncells + DT - 1) / DT;  // <= 5 (MAX_CELLS)
+  int slot[5];
+#pragma unroll
+  for (int j = 0; j < 5; j++) {
+    const int c = tid * cpt + j;
+    slot[j] = j < cpt && c < ncells ? cells[c0 + c].slot_off : 0;
+  }
+  if (tid < 16) S_.H[tid] = 0;
+  if (tid < 17) S_.G[tid] = 0;
+  {  // the dense path's per-depth bins, zeroed here so its first phase needs no barrier of
+     // its own (the region is past the candidate / key arrays; other paths overwrite it)
+    int R = 0;
+    while (R < 6 && g.nini[l] << (2 * (R + 1)) <= DENSE_BINS) R++;
+    uint32_t* bins = reinterpret_cast<uint32_t*>(sm + kSmemCells) + 2 * DCAP;
+    const int o = g.nini[l] * (((1 << (2 * (R + 1))) - 1) / 3);
+    for (int i = tid; i < o; i += DT) bins[i] = 0u;
+    // best0 [DENSE_BINS], best1 [DENSE_BINS], first [DENSE_BINS / 4] (= none), split bytes
+    uint32_t* b0 = bins + DENSE_TOTAL;
+    for (int i = tid; i < 2 * DENSE_BINS; i += DT) b0[i] = 0u;
+    for (int i = tid; i < DENSE_BINS / 4; i += DT) b0[2 * DENSE_BINS + i] = 0xFFFFFFFFu;
+    // split = recch + DENSE_REC, recch = order + DENSE_REC ... as laid out in dense_body
+    const uint64_t* rec = reinterpret_cast<const uint64_t*>(b0 + 2 * DENSE_BINS + DENSE_BINS / 4);
+    const int32_t* recnode = reinterpret_cast<const int32_t*>(rec + DENSE_REC);
+    const int32_t* order = recnode + DENSE_REC;
+    uint8_t* spl = const_cast<uint8_t*>(reinterpret_cast<const uint8_t*>(order + DENSE_REC)) + DENSE_REC;
+    for (int i = tid; i < DENSE_BINS / 4; i += DT) spl[i] = 0;
+  }
+  pdl_wait();
+  pdl_trigger();
+  SS_PHASE(0);
 
   // ---- 1. candidate offsets per cell (rank order = cells row-major, then raster) ----
   {
-    const int cpt = (ncells + DT - 1) / DT;  // <= 5 (MAX_CELLS)
-    int cnt[5], slot[5];
+    int cnt[5];
     int s = 0;
 #pragma unroll
-    for (int j = 0; j < 5; j++) {  // both loads issued before the scan (one global round trip)
+    for (int j = 0; j < 5; j++) {
       const int c = tid * cpt + j;
-      const bool in = j < cpt && c < ncells;
-      cnt[j] = in ? cc[c] : 0;
-      slot[j] = in ? cells[c0 + c].slot_off : 0;
+      cnt[j] = j < cpt && c < ncells ? cc[c] : 0;
       s += cnt[j];
     }
     int ex, tot;
@@ -662,26 +688,6 @@ __global__ void __launch_bounds__(DT, 1)
       S_.sh[0] = tot;
       S_.sh[1] = 0;  // partial-round record count
       S_.sh[2] = 0;  // kept keys
-    }
-    if (tid < 16) S_.H[tid] = 0;
-    if (tid < 17) S_.G[tid] = 0;
-    {  // the dense path's per-depth bins, zeroed here so its first phase needs no barrier of
-       // its own (the region is past the candidate / key arrays; other paths overwrite it)
-      int R = 0;
-      while (R < 6 && g.nini[l] << (2 * (R + 1)) <= DENSE_BINS) R++;
-      uint32_t* bins = reinterpret_cast<uint32_t*>(sm + kSmemCells) + 2 * DCAP;
-      const int o = g.nini[l] * (((1 << (2 * (R + 1))) - 1) / 3);
-      for (int i = tid; i < o; i += DT) bins[i] = 0u;
-      // best0 [DENSE_BINS], best1 [DENSE_BINS], first [DENSE_BINS / 4] (= none), split bytes
-      uint32_t* b0 = bins + DENSE_TOTAL;
-      for (int i = tid; i < 2 * DENSE_BINS; i += DT) b0[i] = 0u;
-      for (int i = tid; i < DENSE_BINS / 4; i += DT) b0[2 * DENSE_BINS + i] = 0xFFFFFFFFu;
-      // split = recch + DENSE_REC, recch = order + DENSE_REC ... as laid out in dense_body
-      const uint64_t* rec = reinterpret_cast<const uint64_t*>(b0 + 2 * DENSE_BINS + DENSE_BINS / 4);
-      const int32_t* recnode = reinterpret_cast<const int32_t*>(rec + DENSE_REC);
-      const int32_t* order = recnode + DENSE_REC;
-      uint8_t* spl = const_cast<uint8_t*>(reinterpret_cast<const uint8_t*>(order + DENSE_REC)) + DENSE_REC;
-      for (int i = tid; i < DENSE_BINS / 4; i += DT) spl[i] = 0;
     }
     __syncthreads();
   }
