@@ -85,7 +85,8 @@ struct LfArgs {
   unsigned long long* claim;       // this matcher's dedup claims [F][cap]
   uint16_t* rowidx;                // if set: the window matcher's global row index, built here too
   unsigned long long* win_claim;   // ... and its dedup claims, reset here (match_prepare's work)
-  int rows_per_frame;
+  int rows_per_frame;              // row-index entries (the shared-memory copy)
+  int index_stride;                // per-frame stride of the global index (rows + lx section)
 };
 
 // frame-wide barrier: the cluster's when a frame spans several CTAs, else the block's
@@ -145,7 +146,8 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
     fclaim[k] = ~0ull;
     if (fmask) fmask[k] = (a.taken && a.taken[(int64_t)f * cap + k]) ? 1 : 0;
     if (a.rowidx) {  // the following search-local-points match reuses this index (no match_prepare)
-      rowidx_fill(g, fk, cnt, a.rowidx + (int64_t)f * a.rows_per_frame, k);
+      uint16_t* gri = a.rowidx + (int64_t)f * a.index_stride;
+      rowidx_fill(g, fk, cnt, gri, k, gri + lx_off(g));
       a.win_claim[(int64_t)f * cap + k] = ~0ull;
     }
   }
@@ -310,7 +312,8 @@ cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams,
   if (n_frames <= 0) return cudaSuccess;
   LfArgs a{g,     n_frames, cams,    last_cams,         mb,          kps, desc, counts,
            taken, pt_off,   pts,     pdesc,             th,          th_high, check_orientation,
-           min_matches, out, n_matches, matched, claim, rowidx, win_claim, match_rows_per_frame(g)};
+           min_matches, out, n_matches, matched, claim, rowidx, win_claim, match_rows_per_frame(g),
+           match_index_stride(g)};
   const size_t smem = lastframe_smem_bytes(g);
   if (smem > kLfSmemMax) return cudaErrorInvalidValue;
   cudaError_t e;

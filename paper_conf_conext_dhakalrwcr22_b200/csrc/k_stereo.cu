@@ -52,7 +52,7 @@ __global__ void __launch_bounds__(ST_WARPS * 32) stereo_match_kernel(Geom g, int
                                                                       const uint8_t* __restrict__ desc,
                                                                       const int32_t* __restrict__ counts,
                                                                       const uint16_t* __restrict__ rowidx,
-                                                                      int rows_per_frame, float bf, float maxD,
+                                                                      int index_stride, float bf, float maxD,
                                                                       float* __restrict__ uright,
                                                                       float* __restrict__ depth,
                                                                       int32_t* __restrict__ sad) {
@@ -81,7 +81,7 @@ __global__ void __launch_bounds__(ST_WARPS * 32) stereo_match_kernel(Geom g, int
     const uint4 a0 = dl[0], a1 = dl[1];
     const ss_keypoint* kr = kps + (int64_t)fr * cap;
     const uint4* dr = reinterpret_cast<const uint4*>(desc + (int64_t)fr * cap * SS_DESC_BYTES);
-    const uint16_t* fri = rowidx + (int64_t)fr * rows_per_frame;
+    const uint16_t* fri = rowidx + (int64_t)fr * index_stride;
     for (int lr = max(lev - 1, 0); lr <= min(lev + 1, L - 1); lr++) {
       const float s = g.scale[lr], r = __fmul_rn(2.0f, s);
       const int hl = g.h[lr];
@@ -225,12 +225,12 @@ __global__ void __launch_bounds__(1024) stereo_outlier_kernel(Geom g, const int3
 }  // namespace
 
 cudaError_t launch_stereo(const Geom& g, int n_pairs, FrameSrc src, const ss_keypoint* kps, const uint8_t* desc,
-                          const int32_t* counts, const uint16_t* rowidx, int rows_per_frame, float bf, float maxD,
+                          const int32_t* counts, const uint16_t* rowidx, int index_stride, float bf, float maxD,
                           float* uright, float* depth, int32_t* sad, cudaStream_t s) {
   if (n_pairs <= 0) return cudaSuccess;
   const int64_t warps = (int64_t)n_pairs * g.kp_capacity;
   cudaError_t e = launch_pdl(stereo_match_kernel, dim3((unsigned)((warps + ST_WARPS - 1) / ST_WARPS)),
-                             dim3(ST_WARPS * 32), 0, s, g, n_pairs, src, kps, desc, counts, rowidx, rows_per_frame,
+                             dim3(ST_WARPS * 32), 0, s, g, n_pairs, src, kps, desc, counts, rowidx, index_stride,
                              bf, maxD, uright, depth, sad);
   return e != cudaSuccess ? e : cudaGetLastError();
 }

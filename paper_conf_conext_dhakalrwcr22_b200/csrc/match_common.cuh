@@ -14,12 +14,18 @@ __host__ __device__ __forceinline__ int row_off(const Geom& g, int l) {  // star
   return l < g.L ? g.row_off[l] : g.row_off[g.L - 1] + g.h[g.L - 1] + 1;
 }
 
+// A frame's segment of the global keypoint index (stride match_index_stride): the row index
+// ([row_off(g, L)] entries), then from lx_off(g) (16-B aligned) every keypoint's lx as u16 in
+// canonical order, which the window matcher prefilters eight at a time.
+__host__ __device__ __forceinline__ int lx_off(const Geom& g) { return (row_off(g, g.L) + 7) & ~7; }
+
 // Row-index entries owned by slot k of one frame (keypoints in canonical (level, ly, lx)
 // order): ri_l[r] = index of the first keypoint of level l with ly >= r, r in [0, h_l].
 // Slot k < L also fills the rows of an empty level k.  fk = the frame's keypoints, cnt = its
 // prefix counts, fr = its row index.
 __device__ __forceinline__ void rowidx_fill(const Geom& g, const ss_keypoint* __restrict__ fk,
-                                            const int32_t* __restrict__ cnt, uint16_t* __restrict__ fr, int k) {
+                                            const int32_t* __restrict__ cnt, uint16_t* __restrict__ fr, int k,
+                                            uint16_t* __restrict__ flx = nullptr) {
   const int L = g.L;
   if (k < L && cnt[k] == cnt[k + 1]) {  // empty level k: every row points at its (empty) range
     uint16_t* ri = fr + row_off(g, k);
@@ -28,6 +34,7 @@ __device__ __forceinline__ void rowidx_fill(const Geom& g, const ss_keypoint* __
   if (k >= cnt[L]) return;
   const ss_keypoint kp = fk[k];
   const int l = kp.level, ly = kp.ly;
+  if (flx) flx[k] = kp.lx;
   uint16_t* ri = fr + row_off(g, l);
   const int prev = k > cnt[l] ? (int)fk[k - 1].ly : -1;
   for (int r = prev + 1; r <= ly; r++) ri[r] = (uint16_t)k;

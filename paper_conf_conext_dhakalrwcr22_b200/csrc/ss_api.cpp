@@ -518,7 +518,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->pattern, 1024);
   ALLOC(c->claim, sizeof(unsigned long long) * F * g.kp_capacity);
   ALLOC(c->claim_lf, sizeof(unsigned long long) * F * g.kp_capacity);
-  ALLOC(c->rowidx, sizeof(uint16_t) * F * match_rows_per_frame(g));
+  ALLOC(c->rowidx, sizeof(uint16_t) * F * match_index_stride(g));
   ALLOC(c->phase_ts, sizeof(uint64_t) * F * L * 16);
   ALLOC(c->stereo_sad, sizeof(int32_t) * ((F + 1) / 2) * g.kp_capacity);
   c->io_pitch = (g.W + 15) & ~15;
@@ -851,7 +851,7 @@ ss_status ss_stereo_match(ss_ctx* c, int32_t n_pairs, const uint8_t* d_frames, i
   SS_CUDA_TRY(launch_match_prepare(c->g, 2 * n_pairs, d_kps, d_counts, c->rowidx, c->claim, 0, s));
   prof_mark(c, s);
   prof_mark(c, s);
-  SS_CUDA_TRY(launch_stereo(c->g, n_pairs, src, d_kps, d_desc, d_counts, c->rowidx, match_rows_per_frame(c->g), bf,
+  SS_CUDA_TRY(launch_stereo(c->g, n_pairs, src, d_kps, d_desc, d_counts, c->rowidx, match_index_stride(c->g), bf,
                             maxD, d_uright, d_depth, c->stereo_sad, s));
   prof_mark(c, s);
   prof_mark(c, s);

@@ -182,6 +182,8 @@ cudaError_t launch_describe(const Geom& g, int n_frames, FrameSrc src, const uin
 const int* brief_pattern_host();
 // Row index of the keypoints (first keypoint per (frame, level, row)) + dedup claim reset.
 int match_rows_per_frame(const Geom& g);
+// per-frame stride of the global index buffer: the row index, then the keypoints' lx (u16)
+int match_index_stride(const Geom& g);
 cudaError_t launch_match_prepare(const Geom& g, int n_frames, const ss_keypoint* kps, const int32_t* counts,
                                  uint16_t* rowidx, unsigned long long* claim, int dedup, cudaStream_t s);
 cudaError_t launch_match_window(const Geom& g, int n_frames, const ss_keypoint* kps, const uint8_t* desc,
@@ -224,7 +226,7 @@ cudaError_t launch_distribute_grid(const Geom& g, int n_frames, int level0, int 
 
 // O12 stereo matching (k_stereo.cu): one warp per left keypoint, then the per-pair outlier cut.
 cudaError_t launch_stereo(const Geom& g, int n_pairs, FrameSrc src, const ss_keypoint* kps, const uint8_t* desc,
-                          const int32_t* counts, const uint16_t* rowidx, int rows_per_frame, float bf, float maxD,
+                          const int32_t* counts, const uint16_t* rowidx, int index_stride, float bf, float maxD,
                           float* uright, float* depth, int32_t* sad, cudaStream_t s);
 cudaError_t launch_stereo_outliers(const Geom& g, int n_pairs, const int32_t* counts, const int32_t* sad,
                                    float* uright, float* depth, cudaStream_t s);
