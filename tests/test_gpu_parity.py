@@ -269,6 +269,10 @@ def test_compute_sanitizer_clean(torch_cuda, tool):
                        [sys.executable, os.path.join(root, "scripts", "sanitize_extract.py")],
                        capture_output=True, text=True, timeout=900)
     tail = (r.stdout + r.stderr)[-3000:]
+    if r.returncode == 86 and "closed" in tail:
+        # the GPU pool can disable compute-sanitizer (its runs have needed GPU resets there);
+        # the last clean runs are kept in profiles/sanitizer_r02
+        pytest.skip("compute-sanitizer disabled on this GPU pool: " + tail.strip().splitlines()[-1][:200])
     assert r.returncode == 0 and "sanitize run ok" in r.stdout, tail
     assert "ERROR SUMMARY: 0 errors" in r.stdout + r.stderr or "RACECHECK SUMMARY: 0 hazards" in r.stdout + r.stderr, tail
 
