@@ -348,9 +348,8 @@ def kernel_work(name: str, p, B: int, cand_l: list, kps_l: list, nq: int, n_map:
         ls = [0] if name == "fast_l0" else list(range(1, L))
         det = sum(B * (p.level_w[l] - 38) * (p.level_h[l] - 38) for l in ls)
         return "alu", float(det) * FAST_OPS_PER_PX
-    if name in ("distribute_l0", "distribute_l1plus"):  # read candidates, write kept keys
-        ls = [0] if name == "distribute_l0" else list(range(1, L))
-        return "hbm", float(sum(4 * cand_l[l] + 4 * kps_l[l] for l in ls))
+    if name == "distribute":  # read candidates, write kept keys (all levels, one launch)
+        return "hbm", float(sum(4 * cand_l[l] + 4 * kps_l[l] for l in range(L)))
     if name == "describe":  # 43x43 patch per keypoint (L2 gathers) + 52 B written per keypoint
         return "hbm", float(sum(kps_l) * (43 * 43 + 4 + 52))
     if name == "match_window":  # query 20 B + descriptor 32 B read, 12 B written
@@ -699,7 +698,7 @@ def run_ours(args, cfg):
     def group(n):  # report per-level launches as level-0 / levels >= 1 / whole-pyramid totals
         if n.startswith("pyramid_l"):
             return "pyramid"
-        for k in ("fast", "distribute"):
+        for k in ("fast",):
             if n.startswith(k + "_l"):
                 return f"{k}_l0" if n == f"{k}_l0" else f"{k}_l1plus"
         return n
@@ -732,11 +731,9 @@ def run_ours(args, cfg):
     kps_h, desc_h, counts_h = pipe.results(B)  # last step's outputs
     kps_l = [int((counts_h[:, l + 1] - counts_h[:, l]).sum()) for l in range(L)]
     cand_l = [sum(len(ss.ss_debug_candidates(pipe.ctx, b, l)[0]) for b in range(B)) for l in range(L)]
-    # dominant kernel = the kernel FUNCTION with the most device time per step (FAST and the
-    # distribution run as two launches each: level 0 on the side branch, levels >= 1 after the
-    # pyramid); its roofline = the algorithmic work of all its launches / their summed time
-    func_of = {"fast_l0": "fast_bands", "fast_l1plus": "fast_bands", "distribute_l0": "distribute",
-               "distribute_l1plus": "distribute"}
+    # dominant kernel = the kernel FUNCTION with the most device time per step (FAST runs as
+    # two launches: level 0 on the side branch, levels >= 1 after the pyramid); its roofline = the algorithmic work of all its launches / their summed time
+    func_of = {"fast_l0": "fast_bands", "fast_l1plus": "fast_bands"}
     per_func = {}
     for n_, t_ in avg_us.items():
         per_func.setdefault(func_of.get(n_, n_), []).append(n_)

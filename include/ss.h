@@ -398,8 +398,8 @@ ss_status ss_track_run(ss_ctx* const* ctxs, int32_t n_ctx, const ss_stream_t* st
  * kernel it launches, continuing across calls until the next ss_profile_events call
  * (n_events = 0 disables; events beyond n_events are not recorded).  One extract records a
  * start event, then a (before, after) pair around every kernel launch, in this order:
- * fast(level 0), distribute(level 0), pyramid (levels 1..L-1, one launch), fast(levels >= 1),
- * distribute(levels >= 1), describe -- 13 events (while events are installed the level-0
+ * fast(level 0), pyramid (levels 1..L-1, one launch), fast(levels >= 1), distribute (all
+ * levels, one launch), describe -- 11 events (while events are installed the level-0
  * branch runs in line on `stream` instead of on its side stream, so each kernel is timed
  * alone).  WINDOW match: a pair per kernel
  * (match_prepare, match_window[, match_resolve if dedup]; the match_prepare pair encloses

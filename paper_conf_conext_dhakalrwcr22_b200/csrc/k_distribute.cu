@@ -46,8 +46,13 @@ constexpr size_t kUnion = cmax(cmax(sizeof(BRS8::TempStorage), sizeof(BRS4::Temp
                                cmax(sizeof(BRS2::TempStorage), kUnionPost));
 constexpr size_t kSmemTotal = kSmemCells + kSmemArrays + kUnion;
 static_assert(kSmemTotal <= 220 * 1024, "distribution smem budget");
-static_assert((size_t)DCAP * 4 + kUnion >= (5464 + 4096 * 2 + 1024) * 4 + 1024 * (8 + 4 + 4 + 1) + 1024,
-              "dense fast-path workspace must fit in the rank + union region");
+constexpr int kRowsMax = 2048;  // level rows (ss_create: H <= 2048)
+constexpr int kTabMax = 2048;   // quadtree key-table entries per axis (qw + 1, qh + 1 <= 2017)
+// dense fast-path workspace (dense_body): per-depth bins, best0 / best1 / first, the partial
+// round's records, the canonical-order row counts / cursors and the key tables
+constexpr size_t kDenseWs = (size_t)(5464 + 4096 * 2 + 1024) * 4 + 1024 * (8 + 4 + 4 + 1) + 1024 +
+                            (size_t)kRowsMax * 8 + (size_t)kTabMax * 8;
+static_assert((size_t)DCAP * 4 + kUnion >= kDenseWs, "dense fast-path workspace must fit in the rank + union region");
 
 __device__ __forceinline__ uint64_t gtimer() {
   uint64_t t;
@@ -394,47 +399,74 @@ constexpr int DENSE_BINS = 4096;      // nIni * 4^R <= DENSE_BINS
 constexpr int DENSE_TOTAL = 5464;     // sum_{r<=R} nIni * 4^r <= 4/3 DENSE_BINS
 constexpr int DENSE_REC = 1024;       // multi-key bins at the partial depth (<= DENSE_BINS / 4 = DT)
 
-__device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* cand, uint32_t* key, uint8_t* ws,
+// The dense path's workspace (starts right after the key array; kDenseWs bytes).
+struct DenseWs {
+  uint32_t* cnt;      // [DENSE_TOTAL] per-depth bins; depth r starts at nini (4^r - 1) / 3
+  uint32_t* best0;    // [DENSE_BINS] depth D
+  uint32_t* best1;    // [DENSE_BINS] depth D + 1
+  uint32_t* first;    // [DENSE_BINS / 4] first rank, depth D
+  uint64_t* rec;      // [DENSE_REC]
+  int32_t* recnode;   // [DENSE_REC]
+  int32_t* order;     // [DENSE_REC]
+  uint8_t* recch;     // [DENSE_REC]
+  uint8_t* split;     // [DENSE_BINS / 4]
+  uint32_t* rowcnt;   // [kRowsMax] kept keys per level row
+  uint32_t* rowpos;   // [kRowsMax] row start, then the row's scatter cursor
+  uint32_t* tabx;     // [kTabMax] quadtree key table, x part
+  uint32_t* taby;     // [kTabMax] ... y part
+  __device__ explicit DenseWs(uint8_t* ws) {
+    cnt = reinterpret_cast<uint32_t*>(ws);
+    best0 = cnt + DENSE_TOTAL;
+    best1 = best0 + DENSE_BINS;
+    first = best1 + DENSE_BINS;
+    rec = reinterpret_cast<uint64_t*>(first + DENSE_BINS / 4);
+    recnode = reinterpret_cast<int32_t*>(rec + DENSE_REC);
+    order = recnode + DENSE_REC;
+    recch = reinterpret_cast<uint8_t*>(order + DENSE_REC);
+    split = recch + DENSE_REC;
+    rowcnt = reinterpret_cast<uint32_t*>(split + DENSE_BINS / 4);
+    rowpos = rowcnt + kRowsMax;
+    tabx = rowpos + kRowsMax;
+    taby = tabx + kTabMax;
+  }
+};
+
+__device__ bool dense_body(const Geom& g, int l, int f, int n, uint32_t* cand, uint32_t* key, uint8_t* ws_bytes,
                            Shared& S_, uint32_t* __restrict__ selected, int32_t* __restrict__ sel_counts,
                            int32_t* ovf_counter, uint64_t* phase_ts) {
   typedef cub::BlockScan<int, DT> Scan;
-  const int tid = threadIdx.x, lane = tid & 31;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int N = g.N[l];
   const int nini = g.nini[l];
-  int R = 0;
-  while (R < 6 && nini << (2 * (R + 1)) <= DENSE_BINS) R++;
-  uint32_t* cnt = reinterpret_cast<uint32_t*>(ws);          // [DENSE_TOTAL] per-depth bins
-  uint32_t* best0 = cnt + DENSE_TOTAL;                        // [DENSE_BINS] depth D
-  uint32_t* best1 = best0 + DENSE_BINS;                       // [DENSE_BINS] depth D + 1
-  uint32_t* first = best1 + DENSE_BINS;                       // [DENSE_BINS / 4] first rank, depth D
-  uint64_t* rec = reinterpret_cast<uint64_t*>(first + DENSE_BINS / 4);  // [DENSE_REC]
-  int32_t* recnode = reinterpret_cast<int32_t*>(rec + DENSE_REC);
-  int32_t* order = recnode + DENSE_REC;
-  uint8_t* recch = reinterpret_cast<uint8_t*>(order + DENSE_REC);
-  uint8_t* split = recch + DENSE_REC;                         // [DENSE_BINS / 4]
+  const int R = g.dense_r[l];
+  const DenseWs w(ws_bytes);
+  uint32_t* cnt = w.cnt;
   // bins of depth r start at off(r) = nini (4^r - 1) / 3
   auto off = [&](int r) { return nini * (((1 << (2 * r)) - 1) / 3); };
-  // the bins were zeroed (and S_.H / S_.G reset) at the kernel's start, before its first barrier
+  // the bins, rows and tables were set up at the kernel's start, before its first barrier
   SS_PHASE(3);
-  // one pass over the keys in a scattered order (consecutive candidates share cells, hence
-  // bins): key to depth R (+1 spare round), one increment per depth >= r_lo; the value an
-  // increment returns says whether it opened a bin (S_r) or made it multi-key (E_r).  The few
-  // shallow bins (depth < r_lo) are sums of their 4 children, formed afterwards.
+  // one pass over the keys: key = X[kx] | Y[ky] (two table reads), one increment at depth R;
+  // the value an increment returns says whether it opened a bin (S_R) or made it multi-key
+  // (E_R).  Lane j of a warp takes candidate j * P + w (P odd: conflict-free shared reads),
+  // so the lanes of one atomic are spread over the level instead of sharing a cell's bins.
+  // Depths r_lo .. R-1 are sums of their 4 children, formed level by level afterwards, and
+  // the few shallow bins (depth < r_lo) by warp 0.
   const int r_lo = R < 3 ? R : 3;
   {
     int nz[7] = {0, 0, 0, 0, 0, 0, 0}, mu[7] = {0, 0, 0, 0, 0, 0, 0};
-    uint32_t stride = 1031u;
-    while ((uint32_t)n % stride == 0u) stride += 2u;  // an odd prime-ish step coprime with n
-    // only the deepest depth R takes atomics (its bins are sparse, so they rarely collide);
-    // depths r_lo .. R-1 are sums of their 4 children, formed level by level afterwards
+    const int P = ((n + 31) >> 5) | 1;
+    const int offR = off(R), shR = 26 - 2 * R;
     int nzR = 0, muR = 0;
-    for (int j = tid; j < n; j += DT) {
-      const int i = (int)(((uint32_t)j * stride) % (uint32_t)n);  // j < 8192: no overflow
-      const uint32_t k = make_key(g, l, cand[i], R + 1);
-      key[i] = k;
-      const uint32_t old = atomicAdd(&cnt[off(R) + (int)(k >> (26 - 2 * R))], 1u);
-      nzR += old == 0u;
-      muR += old == 1u;
+    for (int wi = warp; wi < P; wi += DT / 32) {
+      const int i = lane * P + wi;
+      if (i < n) {
+        const uint32_t c = cand[i];
+        const uint32_t k = w.tabx[key_lx(c) - kMinBorder] | w.taby[key_ly(c) - kMinBorder];
+        key[i] = k;
+        const uint32_t old = atomicAdd(&cnt[offR + (int)(k >> shR)], 1u);
+        nzR += old == 0u;
+        muR += old == 1u;
+      }
     }
 #pragma unroll
     for (int r = 0; r < 7; r++)
@@ -448,7 +480,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
       if (r >= R || r < r_lo) continue;
       const int sz = nini << (2 * r);
       for (int b = tid; b < sz; b += DT) {
-        const uint32_t* ch = cnt + off(r + 1) + 4 * b;
+        const uint32_t* ch = cnt + off(r + 1) + 4 * b;  // off(r) is not 16-B aligned for every nini
         const uint32_t c = ch[0] + ch[1] + ch[2] + ch[3];
         cnt[off(r) + b] = c;
         nz[r] += c > 0u;
@@ -473,27 +505,21 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
         __syncwarp();
       }
     }
+    // per-warp partials, one warp reduction (REDUX) per depth of the packed (a | m << 16)
 #pragma unroll
     for (int r = 0; r < 7; r++) {
       if (r > R) break;
-      int a = nz[r], m = mu[r];
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) {
-        a += __shfl_xor_sync(0xFFFFFFFFu, a, o);
-        m += __shfl_xor_sync(0xFFFFFFFFu, m, o);
-      }
-      if (lane == 0) S_.W[tid >> 5][r] = a | (m << 16);  // per-warp partials (a, m <= 8192)
+      const unsigned s = __reduce_add_sync(0xFFFFFFFFu, (unsigned)(nz[r] | (mu[r] << 16)));  // a, m <= 8192
+      if (lane == 0) S_.W[warp][r] = (int)s;
     }
   }
   __syncthreads();
   // warp r sums depth r's 32 warp partials (no same-address shared atomics across 32 warps)
-  if ((tid >> 5) <= R) {
-    int s = S_.W[lane][tid >> 5];
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xFFFFFFFFu, s, o);
+  if (warp <= R) {
+    const unsigned s = __reduce_add_sync(0xFFFFFFFFu, (unsigned)S_.W[lane][warp]);
     if (lane == 0) {
-      S_.H[tid >> 5] = s & 0xFFFF;
-      S_.G[tid >> 5] = s >> 16;
+      S_.H[warp] = (int)(s & 0xFFFFu);
+      S_.G[warp] = (int)(s >> 16);
     }
   }
   __syncthreads();
@@ -526,9 +552,10 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
   if (D < 0) return false;
   const bool partial = partial_i != 0;
   const int szD = nini << (2 * D);
+  const int shD = 26 - 2 * D;
   // best0 / best1 / first / split were initialised at the kernel's start (S_.sh[1], [2] = 0 too)
   if (partial) {
-    for (int i = tid; i < n; i += DT) atomicMin(&first[key[i] >> (26 - 2 * D)], (uint32_t)i);
+    for (int i = tid; i < n; i += DT) atomicMin(&w.first[key[i] >> shD], (uint32_t)i);
     __syncthreads();
     // the multi-key nodes at depth D, ordered by (size desc, UL.y, UL.x, first-key rank)
     const uint32_t* cD = cnt + off(D);
@@ -536,33 +563,44 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
     for (int b = tid; b < szD; b += DT) {
       const uint32_t c = cD[b];
       if (c > 1u) {
-        const int ch = (cD1[4 * b] > 0u) + (cD1[4 * b + 1] > 0u) + (cD1[4 * b + 2] > 0u) + (cD1[4 * b + 3] > 0u);
+        const uint32_t* q = cD1 + 4 * b;
+        const int ch = (q[0] > 0u) + (q[1] > 0u) + (q[2] > 0u) + (q[3] > 0u);
         int ulx, uly;
-        node_ul(g, l, (uint32_t)b << (26 - 2 * D), D, ulx, uly);
+        node_ul(g, l, (uint32_t)b << shD, D, ulx, uly);
         const int e = atomicAdd(&S_.sh[1], 1);
-        rec[e] = ((uint64_t)(0x1FFFFF - c) << 43) | ((uint64_t)uly << 32) | ((uint64_t)ulx << 20) | (uint64_t)first[b];
-        recnode[e] = b;
-        recch[e] = (uint8_t)ch;
+        w.rec[e] = ((uint64_t)(0x1FFFFF - c) << 43) | ((uint64_t)uly << 32) | ((uint64_t)ulx << 20) | (uint64_t)w.first[b];
+        w.recnode[e] = b;
+        w.recch[e] = (uint8_t)ch;
       }
     }
     __syncthreads();
     const int ne = S_.sh[1];
-    for (int e = tid; e < ne; e += DT) {
-      const uint64_t k = rec[e];
-      int pos = 0;
-      for (int e2 = 0; e2 < ne; e2++) pos += rec[e2] < k;
-      order[pos] = e;
+    {  // rank = #smaller records; G = DT / ne rounded down to a power of two (<= 32) lanes
+       // per record, each counting a 1/G share of the list (shuffle-summed)
+      int G = 1;
+      while (G < 32 && 2 * G * ne <= DT) G *= 2;
+      const int part = tid & (G - 1);
+      for (int e0 = 0; e0 < ne; e0 += DT / G) {
+        const int e = e0 + tid / G;
+        const bool act = e < ne;
+        const uint64_t k = act ? w.rec[e] : 0ull;
+        int pos = 0;
+        if (act)
+          for (int e2 = part; e2 < ne; e2 += G) pos += w.rec[e2] < k;
+        for (int o = 1; o < G; o <<= 1) pos += __shfl_xor_sync(0xFFFFFFFFu, pos, o);
+        if (act && part == 0) w.order[pos] = e;
+      }
     }
     __syncthreads();
     // split the prefix of that order that first brings the node count to >= N: an inclusive
     // scan of (children - 1) over the sorted nodes (ne <= DENSE_REC = DT)
     {
-      const int e = tid < ne ? order[tid] : 0;
-      const int inc = tid < ne ? (int)recch[e] - 1 : 0;
+      const int e = tid < ne ? w.order[tid] : 0;
+      const int inc = tid < ne ? (int)w.recch[e] - 1 : 0;
       int ex, tot;
       Scan(S_.scan).ExclusiveSum(inc, ex, tot);
       // node t is split iff the nodes before it have not yet reached N
-      if (tid < ne && S_.H[D] + ex < N) split[recnode[e]] = 1;
+      if (tid < ne && S_.H[D] + ex < N) w.split[w.recnode[e]] = 1;
     }
   }
   __syncthreads();
@@ -571,41 +609,65 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
   for (int i = tid; i < n; i += DT) {
     const uint32_t k = key[i];
     const uint32_t v = ((uint32_t)key_m(cand[i]) << 20) | (0xFFFFFu - (uint32_t)i);
-    const int b = (int)(k >> (26 - 2 * D));
-    if (partial && split[b]) atomicMax(&best1[k >> (26 - 2 * (D + 1))], v);
-    else atomicMax(&best0[b], v);
+    const int b = (int)(k >> shD);
+    if (partial && w.split[b]) atomicMax(&w.best1[k >> (shD - 2)], v);
+    else atomicMax(&w.best0[b], v);
   }
   __syncthreads();
   SS_PHASE(7);
+  // kept keys (in no particular order) + their level rows' counts
   uint32_t* kept = key;  // keys are no longer needed
-  const uint32_t* cD = cnt + off(D);
-  for (int b = tid; b < szD; b += DT) {
-    if (cD[b] == 0u) continue;
-    if (partial && split[b]) {
-      for (int q = 0; q < 4; q++) {
-        const uint32_t v = best1[4 * b + q];
-        if (v) kept[atomicAdd(&S_.sh[2], 1)] = cand[0xFFFFFu - (v & 0xFFFFFu)];
+  {
+    const uint32_t* cD = cnt + off(D);
+    for (int b = tid; b < szD; b += DT) {
+      if (cD[b] == 0u) continue;
+      if (partial && w.split[b]) {
+        const uint4 q = *reinterpret_cast<const uint4*>(w.best1 + 4 * b);  // best1: 16-B aligned
+        const uint32_t v4[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+        for (int j = 0; j < 4; j++)
+          if (v4[j]) {
+            const uint32_t c = cand[0xFFFFFu - (v4[j] & 0xFFFFFu)];
+            kept[atomicAdd(&S_.sh[2], 1)] = c;
+            atomicAdd(&w.rowcnt[key_ly(c)], 1u);
+          }
+      } else {
+        const uint32_t c = cand[0xFFFFFu - (w.best0[b] & 0xFFFFFu)];
+        kept[atomicAdd(&S_.sh[2], 1)] = c;
+        atomicAdd(&w.rowcnt[key_ly(c)], 1u);
       }
-    } else {
-      kept[atomicAdd(&S_.sh[2], 1)] = cand[0xFFFFFu - (best0[b] & 0xFFFFFu)];
     }
   }
   __syncthreads();
   const int nk = S_.sh[2];
   const int nk_w = min(nk, g.cap[l]);
   SS_PHASE(8);
+  // canonical (ly, lx) order: row starts by a block scan of the row counts, keys scattered
+  // into their row's bucket, then ranked by lx among the (few) keys of the same row
+  {
+    const int h = g.h[l];
+    const int y0 = 2 * tid;
+    const int a0 = y0 < h ? (int)w.rowcnt[y0] : 0, a1 = y0 + 1 < h ? (int)w.rowcnt[y0 + 1] : 0;
+    int ex, tot;
+    Scan(S_.scan).ExclusiveSum(a0 + a1, ex, tot);
+    if (y0 < h) w.rowpos[y0] = (uint32_t)ex;
+    if (y0 + 1 < h) w.rowpos[y0 + 1] = (uint32_t)(ex + a0);
+  }
+  __syncthreads();
+  uint32_t* bucket = cand;  // candidates are no longer needed
+  for (int t = tid; t < nk; t += DT) {
+    const uint32_t k = kept[t];
+    bucket[atomicAdd(&w.rowpos[key_ly(k)], 1u)] = k;
+  }
+  __syncthreads();
   uint32_t* sel_out = selected + (int64_t)f * g.kp_capacity + g.cap_off[l];
-  // rank of each kept key = #smaller keys; 4 lanes per key each count a quarter of the list
-  for (int t0 = 0; t0 < nk; t0 += DT / 4) {
-    const int t = t0 + (tid >> 2), part = tid & 3;
-    const bool act = t < nk;
-    const uint32_t k = act ? kept[t] >> 8 : 0u;
-    int pos = 0;
-    if (act)
-      for (int u = part; u < nk; u += 4) pos += (kept[u] >> 8) < k;
-    pos += __shfl_xor_sync(0xFFFFFFFFu, pos, 1);
-    pos += __shfl_xor_sync(0xFFFFFFFFu, pos, 2);
-    if (act && part == 0 && pos < nk_w) sel_out[pos] = kept[t];
+  for (int t = tid; t < nk; t += DT) {
+    const uint32_t k = bucket[t];
+    const int y = key_ly(k);
+    const int e = (int)w.rowpos[y], s0 = e - (int)w.rowcnt[y];  // the row's bucket [s0, e)
+    int pos = s0;
+    for (int u = s0; u < e; u++) pos += (bucket[u] >> 8) < (k >> 8);
+    if (pos < nk_w) sel_out[pos] = k;
   }
   if (tid == 0) {
     sel_counts[f * g.L + l] = nk_w;
@@ -616,11 +678,11 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, const uint32_t* c
 }
 
 __global__ void __launch_bounds__(DT, 1)
-    distribute_kernel(const __grid_constant__ Geom g, const CellInfo* __restrict__ cells, const uint32_t* __restrict__ slots,
-                      const int32_t* __restrict__ cell_counts, uint32_t* __restrict__ selected,
-                      int32_t* __restrict__ sel_counts, uint8_t* ovf, int64_t ovf_frame_bytes,
-                      const int64_t* __restrict__ ovf_level_off, int32_t* ovf_counter, int level0,
-                      uint64_t* phase_base) {
+    distribute_kernel(const __grid_constant__ Geom g, const CellInfo* __restrict__ cells, const uint32_t* __restrict__ qtab,
+                      const uint32_t* __restrict__ slots, const int32_t* __restrict__ cell_counts,
+                      uint32_t* __restrict__ selected, int32_t* __restrict__ sel_counts, uint8_t* ovf,
+                      int64_t ovf_frame_bytes, const int64_t* __restrict__ ovf_level_off, int32_t* ovf_counter,
+                      int level0, uint64_t* phase_base) {
   extern __shared__ __align__(16) uint8_t sm[];
   __shared__ Shared S_;
   const int l = level0 + blockIdx.x, f = blockIdx.y, tid = threadIdx.x;
@@ -629,9 +691,15 @@ __global__ void __launch_bounds__(DT, 1)
   const int c0 = g.cell_first[l];
   int32_t* cell_off = reinterpret_cast<int32_t*>(sm);
   int32_t* cell_slot = cell_off + MAX_CELLS + 1;
+  uint32_t* cand = reinterpret_cast<uint32_t*>(sm + kSmemCells);
+  uint32_t* key = cand + DCAP;
+  uint8_t* ws = reinterpret_cast<uint8_t*>(key + DCAP);
   const int32_t* cc = cell_counts + (int64_t)f * g.total_cells + c0;
+  SS_PHASE(10);  // kernel entry
   // Work that does not depend on the FAST kernel runs before the dependency wait, overlapping
-  // its tail: the static cell table's slot offsets and the dense path's table initialisation.
+  // its tail: the static cell table's slot offsets, the key tables and the dense path's
+  // table initialisation (its region is past the candidate / key arrays; other paths
+  // overwrite it).
   const int cpt = (ncells + DT - 1) / DT;  // <= 5 (MAX_CELLS)
   int slot[5];
 #pragma unroll
@@ -641,29 +709,34 @@ __global__ void __launch_bounds__(DT, 1)
   }
   if (tid < 16) S_.H[tid] = 0;
   if (tid < 17) S_.G[tid] = 0;
-  {  // the dense path's per-depth bins, zeroed here so its first phase needs no barrier of
-     // its own (the region is past the candidate / key arrays; other paths overwrite it)
-    int R = 0;
-    while (R < 6 && g.nini[l] << (2 * (R + 1)) <= DENSE_BINS) R++;
-    uint32_t* bins = reinterpret_cast<uint32_t*>(sm + kSmemCells) + 2 * DCAP;
-    const int o = g.nini[l] * (((1 << (2 * (R + 1))) - 1) / 3);
-    for (int i = tid; i < o; i += DT) bins[i] = 0u;
-    // best0 [DENSE_BINS], best1 [DENSE_BINS], first [DENSE_BINS / 4] (= none), split bytes
-    uint32_t* b0 = bins + DENSE_TOTAL;
-    for (int i = tid; i < 2 * DENSE_BINS; i += DT) b0[i] = 0u;
-    for (int i = tid; i < DENSE_BINS / 4; i += DT) b0[2 * DENSE_BINS + i] = 0xFFFFFFFFu;
-    // split = recch + DENSE_REC, recch = order + DENSE_REC ... as laid out in dense_body
-    const uint64_t* rec = reinterpret_cast<const uint64_t*>(b0 + 2 * DENSE_BINS + DENSE_BINS / 4);
-    const int32_t* recnode = reinterpret_cast<const int32_t*>(rec + DENSE_REC);
-    const int32_t* order = recnode + DENSE_REC;
-    uint8_t* spl = const_cast<uint8_t*>(reinterpret_cast<const uint8_t*>(order + DENSE_REC)) + DENSE_REC;
-    for (int i = tid; i < DENSE_BINS / 4; i += DT) spl[i] = 0;
+  if (tid == 0) {
+    S_.sh[1] = 0;  // partial-round record count
+    S_.sh[2] = 0;  // kept keys
   }
+  {
+    const DenseWs w(ws);
+    const int R = g.dense_r[l];
+    const int o = g.nini[l] * (((1 << (2 * (R + 1))) - 1) / 3);
+    for (int i = tid; i < o; i += DT) w.cnt[i] = 0u;
+    for (int i = tid; i < 2 * DENSE_BINS; i += DT) w.best0[i] = 0u;  // best0, best1
+    for (int i = tid; i < DENSE_BINS / 4; i += DT) {
+      w.first[i] = 0xFFFFFFFFu;
+      w.split[i] = 0;
+    }
+    for (int i = tid; i < g.h[l]; i += DT) w.rowcnt[i] = 0u;
+    const uint32_t* qt = qtab + g.qtab_off[l];
+    const int nx = g.qw[l] + 1, ny = g.qh[l] + 1;
+    for (int i = tid; i < nx; i += DT) w.tabx[i] = __ldg(qt + i);
+    for (int i = tid; i < ny; i += DT) w.taby[i] = __ldg(qt + nx + i);
+  }
+  SS_PHASE(11);  // static set-up issued
   pdl_wait();
   pdl_trigger();
   SS_PHASE(0);
 
-  // ---- 1. candidate offsets per cell (rank order = cells row-major, then raster) ----
+  // ---- 1. candidate counts per cell, their offsets (rank order = cells row-major, then
+  // raster inside a cell) and, for the usual case, the gather: every thread copies its own
+  // cells' candidates (no per-candidate search for its cell) ----
   {
     int cnt[5];
     int s = 0;
@@ -675,20 +748,37 @@ __global__ void __launch_bounds__(DT, 1)
     }
     int ex, tot;
     BScan(S_.scan).ExclusiveSum(s, ex, tot);
+    if (tot <= DCAP) {
+      const uint32_t* fs = slots + (int64_t)f * g.slots_per_frame;
 #pragma unroll
-    for (int j = 0; j < 5; j++) {
-      const int c = tid * cpt + j;
-      if (j < cpt && c < ncells) {
-        cell_off[c] = ex;
-        cell_slot[c] = slot[j];
-        ex += cnt[j];
+      for (int j = 0; j < 5; j++) {
+        if (j >= cpt) break;
+        const uint32_t* src = fs + slot[j];
+        uint32_t* dst = cand + ex;
+        const int cn = cnt[j];
+        int q = 0;
+        for (; q + 4 <= cn; q += 4) {  // four independent loads in flight
+          const uint32_t v0 = src[q], v1 = src[q + 1], v2 = src[q + 2], v3 = src[q + 3];
+          dst[q] = v0;
+          dst[q + 1] = v1;
+          dst[q + 2] = v2;
+          dst[q + 3] = v3;
+        }
+        for (; q < cn; q++) dst[q] = src[q];
+        ex += cn;
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < 5; j++) {
+        const int c = tid * cpt + j;
+        if (j < cpt && c < ncells) {
+          cell_off[c] = ex;
+          cell_slot[c] = slot[j];
+          ex += cnt[j];
+        }
       }
     }
-    if (tid == 0) {
-      S_.sh[0] = tot;
-      S_.sh[1] = 0;  // partial-round record count
-      S_.sh[2] = 0;  // kept keys
-    }
+    if (tid == 0) S_.sh[0] = tot;
     __syncthreads();
   }
   const int n = S_.sh[0];
@@ -698,31 +788,8 @@ __global__ void __launch_bounds__(DT, 1)
     return;
   }
   if (n <= DCAP) {
-    uint32_t* cand = reinterpret_cast<uint32_t*>(sm + kSmemCells);
-    uint32_t* key = cand + DCAP;
-    {  // gather candidates into rank order (cells row-major, raster inside a cell)
-      const uint32_t* fs = slots + (int64_t)f * g.slots_per_frame;
-      auto src = [&](int i) {  // slot of rank i: last cell with cell_off[c] <= i
-        int lo = 0, hi = ncells - 1;
-        while (lo < hi) {
-          const int mid = (lo + hi + 1) >> 1;
-          if (cell_off[mid] <= i) lo = mid; else hi = mid - 1;
-        }
-        return cell_slot[lo] + (i - cell_off[lo]);
-      };
-      for (int i = tid; i < n; i += 2 * DT) {  // two independent global loads in flight per thread
-        const int i1 = i + DT;
-        const uint32_t v0 = fs[src(i)];
-        const uint32_t v1 = i1 < n ? fs[src(i1)] : 0u;
-        cand[i] = v0;
-        if (i1 < n) cand[i1] = v1;
-      }
-      __syncthreads();
-    }
     SS_PHASE(2);
-    if (dense_body(g, l, f, n, cand, key, reinterpret_cast<uint8_t*>(key + DCAP), S_, selected, sel_counts,
-                   ovf_counter, phase_ts))
-      return;
+    if (dense_body(g, l, f, n, cand, key, ws, S_, selected, sel_counts, ovf_counter, phase_ts)) return;
     if (tid == 0) atomicAdd(ovf_counter + 2, 1);  // counted for the tests (ss_debug_distribution_paths)
     __syncthreads();
     if (tid < 16) S_.H[tid] = 0;
@@ -749,17 +816,39 @@ int64_t distribute_ovf_bytes(int64_t slots) {
   return (b + 255) & ~(int64_t)255;
 }
 
+// Quadtree key tables: make_key's x decisions depend on kx only and its y decisions on ky
+// only (the node's x interval evolves with the "right" bits alone, its y interval with the
+// "down" bits), so key = X[kx] | Y[ky] with X = root << 26 | the right bits (bit 0 of every
+// 2-bit quadrant code) and Y = the down bits (bit 1).  Built once per ctx by make_key itself.
+__global__ void distribute_tables_kernel(const __grid_constant__ Geom g, uint32_t* qtab) {
+  const int l = blockIdx.y;
+  if (l >= g.L) return;
+  const int nx = g.qw[l] + 1, ny = g.qh[l] + 1;
+  uint32_t* t = qtab + g.qtab_off[l];
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nx + ny; i += gridDim.x * blockDim.x) {
+    if (i < nx)
+      t[i] = make_key(g, l, pack_key(i + kMinBorder, kMinBorder, 0)) & 0xFD555555u;  // root (bits 26+) + right bits
+    else
+      t[i] = make_key(g, l, pack_key(kMinBorder, i - nx + kMinBorder, 0)) & 0x02AAAAAAu;  // down bits
+  }
+}
+
+cudaError_t launch_distribute_tables(const Geom& g, uint32_t* qtab, cudaStream_t s) {
+  distribute_tables_kernel<<<dim3(8, g.L), 256, 0, s>>>(g, qtab);
+  return cudaGetLastError();
+}
+
 cudaError_t distribute_init() {  // ss_create, per device
   return cudaFuncSetAttribute(distribute_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemTotal);
 }
 
 cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_levels, const CellInfo* cells,
-                              const uint32_t* slots, const int32_t* cell_counts, uint32_t* selected, int32_t* sel_counts,
+                              const uint32_t* qtab, const uint32_t* slots, const int32_t* cell_counts, uint32_t* selected, int32_t* sel_counts,
                               uint8_t* ovf, int64_t ovf_frame_bytes, const int64_t* ovf_level_off, int32_t* ovf_counter,
                               uint64_t* phase_ts, cudaStream_t s) {
   if (n_levels <= 0) return cudaSuccess;
   dim3 grid(n_levels, n_frames);
-  cudaError_t e = launch_pdl(distribute_kernel, grid, dim3(DT), kSmemTotal, s, g, cells, slots, cell_counts, selected,
+  cudaError_t e = launch_pdl(distribute_kernel, grid, dim3(DT), kSmemTotal, s, g, cells, qtab, slots, cell_counts, selected,
                              sel_counts, ovf, ovf_frame_bytes, ovf_level_off, ovf_counter, level0, phase_ts);
   return e != cudaSuccess ? e : cudaGetLastError();
 }

@@ -127,6 +127,7 @@ struct ss_ctx {
   CellInfo* cells = nullptr;
   BandInfo* bands = nullptr;
   uint32_t* xytab = nullptr;  // per level l >= 1: xtab [w_l], ytab [h_l]
+  uint32_t* qtab = nullptr;   // quadtree key tables (launch_distribute_tables)
   PyrLvl* pyr_plan = nullptr;   // [pyr_blocks][L] fused-pyramid block records
   uint4* pyr_gtab = nullptr;    // per level >= 1: 4-column group coefficients
   int pyr_blocks = 0, pyr_buf0 = 0, pyr_buf1 = 0, pyr_smem = 0;
@@ -232,7 +233,7 @@ inline void prof_mark(ss_ctx* c, cudaStream_t s) {
 void free_ctx(ss_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->device);
-  void* ptrs[] = {c->cells, c->bands, c->xytab, c->pyr_plan, c->pyr_gtab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
+  void* ptrs[] = {c->cells, c->bands, c->xytab, c->qtab, c->pyr_plan, c->pyr_gtab, c->pyr, c->slots, c->cell_counts, c->selected, c->sel_counts, c->ovf,
                   c->ovf_level_off, c->ovf_counter, c->pattern, c->claim, c->claim_lf, c->partial, c->rowidx, c->phase_ts,
                   c->brute_qexp, c->brute_mexp, c->stereo_sad, c->io_frames, c->io_frames_lin, c->io_kps, c->io_desc, c->io_counts,
                   c->io_cams, c->io_points, c->io_pf, c->io_pdesc, c->io_taken, c->io_queries, c->io_matches,
@@ -328,6 +329,13 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     volatile float hx = (float)g.qw[l] / (float)g.nini[l];
     g.hX[l] = hx;
     g.qrounds[l] = kQuadRounds;
+    g.qtab_off[l] = l == 0 ? 0 : g.qtab_off[l - 1] + g.qw[l - 1] + 1 + g.qh[l - 1] + 1;
+    g.qtab_total = g.qtab_off[l] + g.qw[l] + 1 + g.qh[l] + 1;
+    {
+      int R = 0;
+      while (R < 6 && (g.nini[l] << (2 * (R + 1))) <= 4096) R++;
+      g.dense_r[l] = R;
+    }
     // active FAST cells, row-major (DESIGN.md §3 O3)
     g.cell_first[l] = (int)c->cells_h.size();
     g.level_slot_off[l] = slot_off;
@@ -505,6 +513,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   ALLOC(c->cells, sizeof(CellInfo) * c->cells_h.size());
   ALLOC(c->bands, sizeof(BandInfo) * c->bands_h.size());
   ALLOC(c->xytab, sizeof(uint32_t) * tab.size());
+  ALLOC(c->qtab, sizeof(uint32_t) * g.qtab_total);
   if (!plan.empty()) ALLOC(c->pyr_plan, sizeof(PyrLvl) * plan.size());
   if (!gtab.empty()) ALLOC(c->pyr_gtab, sizeof(uint4) * gtab.size());
   ALLOC(c->pyr, F * g.pyr_frame_bytes);
@@ -569,6 +578,8 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (e == cudaSuccess) e = cudaMemcpy(c->ovf_level_off, ovf_off.data(), sizeof(int64_t) * L, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->pattern, pat.data(), 1024, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemset(c->ovf_counter, 0, sizeof(int32_t) * 4);
+  if (e == cudaSuccess) e = launch_distribute_tables(g, c->qtab, 0);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
   for (int i = 0; i < ss_ctx::kSide && e == cudaSuccess; i++) {
     e = cudaStreamCreateWithFlags(&c->side[i], cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_join[i], cudaEventDisableTiming);
@@ -617,11 +628,12 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   SS_CUDA_TRY(check_stream(s));
   const Geom& g = c->g;
   FrameSrc src{d_frames, frame_stride, pitch, c->pyr};
-  // DAG: level 0's FAST + distribution run on side stream 0 (they need no pyramid) while the
-  // caller's stream builds levels 1..L-1 and runs their FAST + distribution (one launch each:
-  // per-level launches cost more in launch latency than the overlap saves); describe joins.
+  // DAG: level 0's FAST runs on side stream 0 (it needs no pyramid) while the caller's stream
+  // builds levels 1..L-1 and runs their FAST (one launch each: per-level launches cost more in
+  // launch latency than the overlap saves); the distribution of ALL levels is one launch after
+  // the join (one (level, frame) CTA each), then describe.
   // Profiling events: start, then a (before, after) pair around every launch in this order:
-  // fast l0, distribute l0, pyramid (levels 1..L-1, one launch), fast l>=1, distribute l>=1, describe.
+  // fast l0, pyramid (levels 1..L-1, one launch), fast l>=1, distribute (all levels), describe.
   prof_mark(c, s);
   SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 4, s));
   SS_CUDA_TRY(cudaEventRecord(c->ev_fork, s));
@@ -631,14 +643,6 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   if (q != s) SS_CUDA_TRY(cudaStreamWaitEvent(q, c->ev_fork, 0));
   prof_mark(c, q);
   SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands, g.band_count[0], c->cells, c->slots, c->cell_counts, q));
-  prof_mark(c, q);
-  prof_mark(c, q);
-  if (c->dist_mode == SS_DIST_GRID_TOPN)
-    SS_CUDA_TRY(launch_distribute_grid(g, n_frames, 0, 1, c->cells, c->slots, c->cell_counts, c->selected,
-                                       c->sel_counts, q));
-  else
-    SS_CUDA_TRY(launch_distribute(g, n_frames, 0, 1, c->cells, c->slots, c->cell_counts, c->selected, c->sel_counts,
-                                  c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter, c->phase_ts, q));
   prof_mark(c, q);
   if (q != s) SS_CUDA_TRY(cudaEventRecord(c->ev_join[0], q));
   prof_mark(c, s);
@@ -650,16 +654,16 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands + g.band_count[0], g.total_bands - g.band_count[0],
                                 c->cells, c->slots, c->cell_counts, s));
   prof_mark(c, s);
+  if (q != s) SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[0], 0));
   prof_mark(c, s);
   if (c->dist_mode == SS_DIST_GRID_TOPN)
-    SS_CUDA_TRY(launch_distribute_grid(g, n_frames, 1, g.L - 1, c->cells, c->slots, c->cell_counts, c->selected,
+    SS_CUDA_TRY(launch_distribute_grid(g, n_frames, 0, g.L, c->cells, c->slots, c->cell_counts, c->selected,
                                        c->sel_counts, s));
   else
-    SS_CUDA_TRY(launch_distribute(g, n_frames, 1, g.L - 1, c->cells, c->slots, c->cell_counts, c->selected,
+    SS_CUDA_TRY(launch_distribute(g, n_frames, 0, g.L, c->cells, c->qtab, c->slots, c->cell_counts, c->selected,
                                   c->sel_counts, c->ovf, c->ovf_frame_bytes, c->ovf_level_off, c->ovf_counter,
                                   c->phase_ts, s));
   prof_mark(c, s);
-  if (q != s) SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[0], 0));
   prof_mark(c, s);
   // level 0: the caller's frames, encoded for this call (TMA when 16-B aligned, else LDG)
   c->maps.valid &= ~1u;

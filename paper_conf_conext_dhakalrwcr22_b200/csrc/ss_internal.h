@@ -68,6 +68,11 @@ struct Geom {
   int32_t band_first[kMaxLevels], band_count[kMaxLevels];  // FAST work units of level l
   int32_t max_band_w, max_band_h;   // widest band (detect columns) / tallest band (detect rows)
   int32_t max_cell_w;               // widest cell detect window
+  // quadtree key tables (k_distribute.cu): level l's x part (root + right bits) for kx in
+  // [0, qw] at qtab_off[l], its y part (down bits) for ky in [0, qh] right after
+  int32_t qtab_off[kMaxLevels];
+  int32_t qtab_total;
+  int32_t dense_r[kMaxLevels];      // deepest dense-histogram depth R of level l (nIni * 4^R <= 4096)
 };
 
 // Where the frames of one call live.  Level 0 is the caller's frame (no copy).
@@ -170,7 +175,7 @@ cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const B
                               const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s);
 size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int* mband_bytes, int* nball);
 cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_levels, const CellInfo* cells,
-                              const uint32_t* slots, const int32_t* cell_counts, uint32_t* selected,
+                              const uint32_t* qtab, const uint32_t* slots, const int32_t* cell_counts, uint32_t* selected,
                               int32_t* sel_counts, uint8_t* ovf, int64_t ovf_frame_bytes,
                               const int64_t* ovf_level_off, int32_t* ovf_counter, uint64_t* phase_ts,
                               cudaStream_t s);
@@ -251,6 +256,8 @@ cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams,
                              uint8_t* matched, unsigned long long* claim, uint16_t* rowidx,
                              unsigned long long* win_claim, cudaStream_t s);
 
+// Quadtree key tables of every level (ss_create, once): qtab[g.qtab_total] u32.
+cudaError_t launch_distribute_tables(const Geom& g, uint32_t* qtab, cudaStream_t s);
 // Overflow scratch bytes the distribution needs for a level with `slots` candidate slots.
 int64_t distribute_ovf_bytes(int64_t slots);
 

@@ -257,7 +257,7 @@ def ss_profile_next(ctx) -> int:
 
 def extract_kernels(n_levels: int) -> list[str]:
     """Kernel launches of one ss_orb_extract in profiling-event order (include/ss.h)."""
-    return ["fast_l0", "distribute_l0", "pyramid", "fast_l1plus", "distribute_l1plus", "describe"]
+    return ["fast_l0", "pyramid", "fast_l1plus", "distribute", "describe"]
 
 
 def extract_events(n_levels: int) -> int:

@@ -16,9 +16,9 @@ fr = torch.from_numpy(synth.make_frames(w, h, 4, cfg=2)).cuda()
 for _ in range(5):
     pipe.extract(fr)
 torch.cuda.synchronize()
-names = ["start", "n", "gather", "zeroed", "keys+hist", "rules", "partial", "best", "kept", "written"]
+names = ["start", "n", "gather", "zeroed", "keys+hist", "rules", "partial", "best", "kept", "written", "entry", "setup"]
 for l in range(8):
-    t = ss.ss_debug_phase_times(pipe.ctx, 0, l)
-    rel = [(names[i], int(t[i] - t[0])) for i in range(len(t)) if t[i] >= t[0]]
+    t = ss.ss_debug_phase_times(pipe.ctx, 0, l, 12)
+    rel = [(names[i], int(t[i] - t[0])) for i in range(len(t)) if t[i] >= t[0] or i >= 10]
     n = len(ss.ss_debug_candidates(pipe.ctx, 0, l)[0])
     print(f"level {l} n={n}", rel)
