@@ -344,8 +344,8 @@ def kernel_work(name: str, p, B: int, cand_l: list, kps_l: list, nq: int, n_map:
     L = p.n_levels
     if name == "pyramid":  # every level l >= 1 reads level l-1 once and is written once
         return "hbm", float(B * sum(W[l - 1] + W[l] for l in range(1, L)))
-    if name in ("fast_l0", "fast_l1plus"):  # ALU-bound: exact FAST-9 score of every detect pixel
-        ls = [0] if name == "fast_l0" else list(range(1, L))
+    if name in ("fast", "fast_l0", "fast_l1plus"):  # ALU-bound: exact FAST-9 score of every detect pixel
+        ls = {"fast": list(range(L)), "fast_l0": [0]}.get(name, list(range(1, L)))
         det = sum(B * (p.level_w[l] - 38) * (p.level_h[l] - 38) for l in ls)
         return "alu", float(det) * FAST_OPS_PER_PX
     if name == "distribute":  # read candidates, write kept keys (all levels, one launch)
@@ -731,9 +731,10 @@ def run_ours(args, cfg):
     kps_h, desc_h, counts_h = pipe.results(B)  # last step's outputs
     kps_l = [int((counts_h[:, l + 1] - counts_h[:, l]).sum()) for l in range(L)]
     cand_l = [sum(len(ss.ss_debug_candidates(pipe.ctx, b, l)[0]) for b in range(B)) for l in range(L)]
-    # dominant kernel = the kernel FUNCTION with the most device time per step (FAST runs as
-    # two launches: level 0 on the side branch, levels >= 1 after the pyramid); its roofline = the algorithmic work of all its launches / their summed time
-    func_of = {"fast_l0": "fast_bands", "fast_l1plus": "fast_bands"}
+    # dominant kernel = the kernel FUNCTION with the most device time per step (with
+    # SS_FAST_SPLIT=1 FAST runs as two launches: level 0 beside the pyramid, levels >= 1 after
+    # it); its roofline = the algorithmic work of all its launches / their summed time
+    func_of = {"fast": "fast_bands", "fast_l0": "fast_bands", "fast_l1plus": "fast_bands"}
     per_func = {}
     for n_, t_ in avg_us.items():
         per_func.setdefault(func_of.get(n_, n_), []).append(n_)

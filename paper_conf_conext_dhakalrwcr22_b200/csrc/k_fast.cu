@@ -27,6 +27,22 @@
 
 namespace ss {
 
+#ifdef SS_FAST_PHASES  // per-CTA phase timestamps (scripts/fast_phases.py; instrumented builds only)
+__device__ unsigned long long g_fast_ts[2][4096][8];
+#define FAST_TS(i)                                                                                     \
+  do {                                                                                                 \
+    if (threadIdx.x == 0 && blockIdx.y * gridDim.x + blockIdx.x < 4096) {                              \
+      unsigned long long t_;                                                                           \
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                                           \
+      g_fast_ts[bd.level != 0][blockIdx.y * gridDim.x + blockIdx.x][i] = t_;                           \
+    }                                                                                                  \
+  } while (0)
+#else
+#define FAST_TS(i) \
+  do {             \
+  } while (0)
+#endif
+
 namespace {
 
 #ifndef SS_FAST_WARPS
@@ -142,18 +158,121 @@ __device__ __forceinline__ uint32_t nibble4(uint32_t h0, uint32_t h1) {
   return (t | (t >> 14)) & 0xFu;
 }
 
+// Scores of a staged band: task t = (4-pixel group t % ng, rows [ROWS * (t / ng), + ROWS)),
+// a sliding 7-row register window per task (3 shared loads per row step).
+template <int ROWS>
+__device__ __forceinline__ void score_band(const uint8_t* reg, int rp, uint8_t* Mb, int mbw, int g0, int ng, int Dh) {
+  const int nrt = (Dh + ROWS - 1) / ROWS;
+  for (int t = threadIdx.x; t < ng * nrt; t += FB_THREADS) {
+    const int gc = g0 + 4 * (t % ng);
+    const int ys = (t / ng) * ROWS;
+    uint32_t W[7][3];
+    // staged row of band row y is y + 3; rows y-3..y+3 -> staged rows y..y+6
+#pragma unroll
+    for (int r = 0; r < 6; r++) {
+      const uint32_t* p = reinterpret_cast<const uint32_t*>(reg + (ys + r) * rp + gc - 4);
+      W[r + 1][0] = p[0];
+      W[r + 1][1] = p[1];
+      W[r + 1][2] = p[2];
+    }
+#pragma unroll
+    for (int i = 0; i < ROWS; i++) {  // fully unrolled: the window shift is renaming
+      const int y = ys + i;
+      if (y >= Dh) break;
+#pragma unroll
+      for (int r = 0; r < 6; r++) {
+        W[r][0] = W[r + 1][0];
+        W[r][1] = W[r + 1][1];
+        W[r][2] = W[r + 1][2];
+      }
+      const uint32_t* p = reinterpret_cast<const uint32_t*>(reg + (y + 6) * rp + gc - 4);
+      W[6][0] = p[0];
+      W[6][1] = p[1];
+      W[6][2] = p[2];
+      *reinterpret_cast<uint32_t*>(Mb + (y + 1) * mbw + gc) = fast_M4(W);
+    }
+  }
+}
+
+// Strict 8-neighbour maxima of a band's score map into the bit planes (same task layout as
+// score_band): see step 3 of the kernel.
+template <int ROWS>
+__device__ __forceinline__ void nms_band(const uint8_t* Mb, int mbw, uint32_t* bits, int bw, const uint32_t* starts,
+                                         int g0, int ng, int Dh, int tmin, int tini) {
+  const int nrt = (Dh + ROWS - 1) / ROWS;
+  const uint32_t tmin1 = (uint32_t)(tmin + 1) * 0x10001u, tini1 = (uint32_t)(tini + 1) * 0x10001u;
+  for (int t = threadIdx.x; t < ng * nrt; t += FB_THREADS) {
+    const int gc = g0 + 4 * (t % ng);
+    const int ys = (t / ng) * ROWS;
+    // cell starts at columns gc .. gc + 4 -> lane masks of valid left / right neighbours
+    const uint32_t sw5 = (uint32_t)(__funnelshift_r(starts[gc >> 5], starts[(gc >> 5) + 1], gc & 31)) & 0x1Fu;
+    uint32_t mL[2], mR[2];
+#pragma unroll
+    for (int hv = 0; hv < 2; hv++) {  // pixels (hv, hv + 2)
+      mL[hv] = ((sw5 >> hv) & 1u ? 0u : 0xFFFFu) | ((sw5 >> (hv + 2)) & 1u ? 0u : 0xFFFF0000u);
+      mR[hv] = ((sw5 >> (hv + 1)) & 1u ? 0u : 0xFFFFu) | ((sw5 >> (hv + 3)) & 1u ? 0u : 0xFFFF0000u);
+    }
+    // per half: hf / hlr of rows y - 1 and y, the centre of row y
+    uint32_t hfp[2], hf0[2], hl0[2], c0[2];
+    auto rowq = [&](int y, uint32_t (&hf)[2], uint32_t (&hl)[2], uint32_t (&cc)[2]) {
+      const uint32_t* pr = reinterpret_cast<const uint32_t*>(Mb + (y + 1) * mbw + gc - 4);
+      const uint32_t wp = pr[0], wc = pr[1], wn = pr[2];
+      const uint32_t Lw = __byte_perm(wp, wc, 0x6543), Rw = __byte_perm(wc, wn, 0x4321);
+#pragma unroll
+      for (int hv = 0; hv < 2; hv++) {
+        const uint32_t sel = hv ? 0x7371u : 0x7270u;
+        const uint32_t Ch = __byte_perm(wc, 0, sel);
+        const uint32_t Lh = __byte_perm(Lw, 0, sel) & mL[hv], Rh = __byte_perm(Rw, 0, sel) & mR[hv];
+        hl[hv] = __vmaxu2(Lh, Rh);
+        hf[hv] = __vimax3_u16x2(Lh, Rh, Ch);
+        cc[hv] = Ch;
+      }
+    };
+    {
+      uint32_t dummy[2];
+      rowq(ys - 1, hfp, dummy, dummy);  // row -1 reads the zero row
+      rowq(ys, hf0, hl0, c0);
+    }
+    uint32_t* bmin = bits + gc / 32;
+    const int bsh = gc & 31;
+#pragma unroll
+    for (int i = 0; i < ROWS; i++) {
+      const int y = ys + i;
+      if (y >= Dh) break;
+      uint32_t hfn[2], hln[2], cn[2];
+      rowq(y + 1, hfn, hln, cn);  // row Dh reads the zero row
+      uint32_t ok[2], oi[2];
+#pragma unroll
+      for (int hv = 0; hv < 2; hv++) {
+        const uint32_t nb = __vimax3_u16x2(hfp[hv], hl0[hv], hfn[hv]);
+        const uint32_t C = c0[hv] | 0x80008000u;
+        ok[hv] = (C - nb - 0x00010001u) & (C - tmin1) & 0x80008000u;  // > neighbours, > minTh
+        oi[hv] = ok[hv] & (C - tini1);                                // and > iniTh
+        hfp[hv] = hf0[hv];
+        hf0[hv] = hfn[hv];
+        hl0[hv] = hln[hv];
+        c0[hv] = cn[hv];
+      }
+      const uint32_t km = nibble4(ok[0], ok[1]), ki = nibble4(oi[0], oi[1]);
+      if (km) atomicOr(bmin + y * bw, km << bsh);
+      if (ki) atomicOr(bmin + (Dh + y) * bw, ki << bsh);
+    }
+  }
+}
+
 __global__ void __launch_bounds__(FB_THREADS, FB_MIN_BLOCKS) fast_bands_kernel(const __grid_constant__ Geom g, FrameSrc src,
                                                                 const BandInfo* __restrict__ bands,
                                                                 const CellInfo* __restrict__ cells,
                                                                 uint32_t* __restrict__ slots,
                                                                 int32_t* __restrict__ cell_counts, int rp, int mbw,
-                                                                int region_bytes) {
+                                                                int region_bytes, int bits_off) {
   pdl_wait();
   pdl_trigger();
   extern __shared__ __align__(16) uint8_t smem[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const BandInfo bd = bands[blockIdx.x];
   const int f = blockIdx.y;
+  FAST_TS(0);
   const int l = bd.level;
   const int tmin = g.min_th, tini = g.ini_th;
   const uint8_t* img;
@@ -174,9 +293,16 @@ __global__ void __launch_bounds__(FB_THREADS, FB_MIN_BLOCKS) fast_bands_kernel(c
   const uint8_t* row0 = img + (int64_t)(bd.y0 - 3) * ip + xa;
   // ---- 1. stage rows y0-3 .. y1+2, columns xa .. xa+sw-1 (all inside the level row) ----
   const int nchunk = sw >> 4;
+  // NMS bit planes: [2][Dh][bw] words (bit s of row y = staged column s is a maximum above
+  // minTh / above iniTh), then the cell-start columns [bw]; zeroed here, set by atomicOr
+  const int bw = (mbw + 31) / 32 + 2;
+  uint32_t* bits = reinterpret_cast<uint32_t*>(smem + bits_off);
+  uint32_t* starts = bits + 2 * Dh * bw;
+  for (int i = threadIdx.x; i < (2 * Dh + 1) * bw; i += FB_THREADS) bits[i] = 0u;
   if ((ip & 15) == 0 && (reinterpret_cast<uintptr_t>(img) & 15) == 0) {
+    const uint32_t inv = 0xFFFFFFFFu / (uint32_t)nchunk + 1u;  // i / nchunk = umulhi(i, inv) for i < 2^16
     for (int i = threadIdx.x; i < (Dh + 6) * nchunk; i += FB_THREADS) {
-      const int r = i / nchunk, c = i - r * nchunk;
+      const int r = (int)__umulhi((uint32_t)i, inv), c = i - r * nchunk;
       uint4 v = __ldg(reinterpret_cast<const uint4*>(row0 + (int64_t)r * ip) + c);
       v.x ^= 0x80808080u, v.y ^= 0x80808080u, v.z ^= 0x80808080u, v.w ^= 0x80808080u;  // bytes as I - 128
       *reinterpret_cast<uint4*>(reg + r * rp + 16 * c) = v;
@@ -193,130 +319,55 @@ __global__ void __launch_bounds__(FB_THREADS, FB_MIN_BLOCKS) fast_bands_kernel(c
     reinterpret_cast<uint32_t*>(Mb + (Dh + 1) * mbw)[i] = 0u;
   }
   __syncthreads();
-  // ---- 2. scores of all band pixels, 4 per thread, ROWS_PER_TASK rows per task ----
+  FAST_TS(1);
+  // cell-start columns (and the band's end): a pixel's left neighbour is in its cell unless its
+  // column starts a cell, its right neighbour unless the next column does
+  if (threadIdx.x <= bd.ncells) {
+    const int sc = (threadIdx.x < bd.ncells ? cells[bd.cell_first + threadIdx.x].x0 : bd.x1) - xa;
+    atomicOr(&starts[sc >> 5], 1u << (sc & 31));
+  }
+  // ---- 2. scores of all band pixels, 4 per thread, ROWS rows per task: 8, or 4 when 8-row
+  // tasks would leave half the CTA's threads without one (level-0 segments of <= 4 cells) ----
   {
     const int ng = (g1 - g0) >> 2;
-    const int nrt = (Dh + ROWS_PER_TASK - 1) / ROWS_PER_TASK;
-    for (int t = threadIdx.x; t < ng * nrt; t += FB_THREADS) {
-      const int gc = g0 + 4 * (t % ng);
-      const int ys = (t / ng) * ROWS_PER_TASK;
-      uint32_t W[7][3];
-      // staged row of band row y is y + 3; rows y-3..y+3 -> staged rows y..y+6
-#pragma unroll
-      for (int r = 0; r < 6; r++) {
-        const uint32_t* p = reinterpret_cast<const uint32_t*>(reg + (ys + r) * rp + gc - 4);
-        W[r + 1][0] = p[0];
-        W[r + 1][1] = p[1];
-        W[r + 1][2] = p[2];
-      }
-#pragma unroll
-      for (int i = 0; i < ROWS_PER_TASK; i++) {  // fully unrolled: the window shift is renaming
-        const int y = ys + i;
-        if (y >= Dh) break;
-#pragma unroll
-        for (int r = 0; r < 6; r++) {
-          W[r][0] = W[r + 1][0];
-          W[r][1] = W[r + 1][1];
-          W[r][2] = W[r + 1][2];
-        }
-        const uint32_t* p = reinterpret_cast<const uint32_t*>(reg + (y + 6) * rp + gc - 4);
-        W[6][0] = p[0];
-        W[6][1] = p[1];
-        W[6][2] = p[2];
-        *reinterpret_cast<uint32_t*>(Mb + (y + 1) * mbw + gc) = fast_M4(W);
-      }
-    }
+    if (ng * ((Dh + 7) / 8) * 2 <= FB_THREADS)
+      score_band<4>(reg, rp, Mb, mbw, g0, ng, Dh);
+    else
+      score_band<ROWS_PER_TASK>(reg, rp, Mb, mbw, g0, ng, Dh);
   }
   __syncthreads();
-  // ---- 3. per cell (warp), per row (lane): strict maxima, threshold choice, raster output ----
+  FAST_TS(2);
+  // ---- 3. strict 8-neighbour maxima above minTh / iniTh, every thread on 4-pixel groups of
+  // ROWS_PER_TASK rows (the score tasks' layout), into the bit planes: per 16x2 half (pixels
+  // 0, 2 or 1, 3) the horizontal 3-max hf and left/right max hlr of each row are formed once
+  // (neighbours in another cell masked to 0: per-cell ROI semantics; rows -1 and Dh are the
+  // score map's zero rows) and row y tests C > max(hf(y-1), hlr(y), hf(y+1)) ----
+  {
+    const int ng = (g1 - g0) >> 2;
+    if (ng * ((Dh + 7) / 8) * 2 <= FB_THREADS)
+      nms_band<4>(Mb, mbw, bits, bw, starts, g0, ng, Dh, tmin, tini);
+    else
+      nms_band<ROWS_PER_TASK>(Mb, mbw, bits, bw, starts, g0, ng, Dh, tmin, tini);
+  }
+  __syncthreads();
+  FAST_TS(3);
+  // ---- 4. per cell (warp), per row (lane): the cell's threshold (iniTh if any maximum beats
+  // it, else minTh) and the survivors in raster order (warp prefix sum of the row counts) ----
   for (int j = warp; j < bd.ncells; j += FB_WARPS) {
     const int ci = bd.cell_first + j;
     const CellInfo c = cells[ci];
     const int cx0 = c.x0 - xa, cw = c.x1 - c.x0;  // staged columns [cx0, cx0 + cw), cw < 64
+    const unsigned long long cm = cw >= 64 ? ~0ull : (1ull << cw) - 1ull;
     unsigned long long kmin[2] = {0ull, 0ull}, kini[2] = {0ull, 0ull};
-    // words A_j (cell columns [4j-4, 4j)) are whole for j < nk, partial at j = nk (lastmask),
-    // outside the cell beyond
-    const int nk = (cw + 3) >> 2;
-    const uint32_t lastmask = 0xFFFFFFFFu >> (8 * (4 * nk - cw));
-    if (Dh <= 32) {
-      // one pass, lane = row: only the row's own words are read; the neighbour rows' 3-wide
-      // maxima come from lanes y - 1 and y + 1 by shuffles (rows -1 and Dh are the zero rows
-      // of the score map, hence the lane masks); lanes >= Dh read the zero row below the band
-      const int base = cx0 - 4, a0 = base & ~3;
-      const uint32_t sh = 8u * (uint32_t)(base & 3);
-      const uint32_t* pr = reinterpret_cast<const uint32_t*>(Mb + ((lane < Dh ? lane : Dh) + 1) * mbw + a0);
-      auto aword = [&](int j) -> uint32_t {
-        const uint32_t v = __funnelshift_r(pr[j], pr[j + 1], sh);
-        return j < nk ? v : (j == nk ? v & lastmask : 0u);
-      };
-      const uint32_t upm = lane > 0 ? 0xFFFFFFFFu : 0u, dnm = lane + 1 < Dh ? 0xFFFFFFFFu : 0u;
-      const uint32_t tmin1 = (uint32_t)(tmin + 1) * 0x10001u, tini1 = (uint32_t)(tini + 1) * 0x10001u;
-      uint32_t pw = 0u, cwd = aword(1);
-      for (int k = 0; k < nk; k++) {
-        const uint32_t nw = aword(k + 2);
-        const uint32_t Lw = __byte_perm(pw, cwd, 0x6543), Rw = __byte_perm(cwd, nw, 0x4321);
-        uint32_t ok[2], oi[2];
-#pragma unroll
-        for (int half = 0; half < 2; half++) {  // lanes: pixels (0, 2), then (1, 3)
-          const uint32_t sel = half ? 0x7371u : 0x7270u;
-          const uint32_t Ch = __byte_perm(cwd, 0, sel), Lh = __byte_perm(Lw, 0, sel), Rh = __byte_perm(Rw, 0, sel);
-          const uint32_t hlr = __vimax3_u16x2(Lh, Rh, Lh), hf = __vimax3_u16x2(Lh, Rh, Ch);
-          const uint32_t up = __shfl_up_sync(0xFFFFFFFFu, hf, 1) & upm;
-          const uint32_t dn = __shfl_down_sync(0xFFFFFFFFu, hf, 1) & dnm;
-          const uint32_t nb = __vimax3_u16x2(hlr, up, dn);
-          const uint32_t C = Ch | 0x80008000u;
-          ok[half] = (C - nb - 0x00010001u) & (C - tmin1) & 0x80008000u;  // > neighbours, > minTh
-          oi[half] = ok[half] & (C - tini1);                                // and > iniTh
-        }
-        kmin[0] |= (unsigned long long)nibble4(ok[0], ok[1]) << (4 * k);
-        kini[0] |= (unsigned long long)nibble4(oi[0], oi[1]) << (4 * k);
-        pw = cwd;
-        cwd = nw;
-      }
-      if (lane >= Dh) kmin[0] = kini[0] = 0ull;
-    } else
 #pragma unroll
     for (int hh = 0; hh < 2; hh++) {
       const int y = lane + 32 * hh;
       if (y < Dh) {
-        // strict 8-neighbour maxima of the row, four columns per step on 16x2 lanes: words
-        // A_j = cell columns [4j-4, 4j) of rows y-1, y, y+1 with every byte outside the cell
-        // zeroed (ROI semantics: neighbours in other cells are ignored; a zero never beats a
-        // score > minTh), so the test needs no edge cases.
-        const int base = cx0 - 4, a0 = base & ~3;
-        const uint32_t sh = 8u * (uint32_t)(base & 3);
-        const uint32_t* pr0 = reinterpret_cast<const uint32_t*>(Mb + y * mbw + a0);
-        const uint32_t* pr1 = reinterpret_cast<const uint32_t*>(Mb + (y + 1) * mbw + a0);
-        const uint32_t* pr2 = reinterpret_cast<const uint32_t*>(Mb + (y + 2) * mbw + a0);
-        auto aword = [&](const uint32_t* pr, int j) -> uint32_t {
-          const uint32_t v = __funnelshift_r(pr[j], pr[j + 1], sh);
-          return j < nk ? v : (j == nk ? v & lastmask : 0u);
-        };
-        uint32_t p0 = 0u, p1 = 0u, p2 = 0u;  // A_k of rows y-1, y, y+1
-        uint32_t c0w = aword(pr0, 1), c1w = aword(pr1, 1), c2w = aword(pr2, 1);  // A_{k+1}
-        const uint32_t tmin1 = (uint32_t)(tmin + 1) * 0x10001u, tini1 = (uint32_t)(tini + 1) * 0x10001u;
-        for (int k = 0; k < nk; k++) {
-          const uint32_t n0 = aword(pr0, k + 2), n1 = aword(pr1, k + 2), n2 = aword(pr2, k + 2);
-          const uint32_t L0 = __byte_perm(p0, c0w, 0x6543), R0 = __byte_perm(c0w, n0, 0x4321);
-          const uint32_t L1 = __byte_perm(p1, c1w, 0x6543), R1 = __byte_perm(c1w, n1, 0x4321);
-          const uint32_t L2 = __byte_perm(p2, c2w, 0x6543), R2 = __byte_perm(c2w, n2, 0x4321);
-          uint32_t ok[2], oi[2];
-#pragma unroll
-          for (int half = 0; half < 2; half++) {  // lanes: pixels (0, 2), then (1, 3)
-            const uint32_t sel = half ? 0x7371u : 0x7270u;
-            const uint32_t C = __byte_perm(c1w, 0, sel) | 0x80008000u;
-            const uint32_t nb =
-                __vimax3_u16x2(__vimax3_u16x2(__byte_perm(c0w, 0, sel), __byte_perm(L0, 0, sel), __byte_perm(R0, 0, sel)),
-                               __vimax3_u16x2(__byte_perm(c2w, 0, sel), __byte_perm(L2, 0, sel), __byte_perm(R2, 0, sel)),
-                               __vimax3_u16x2(__byte_perm(L1, 0, sel), __byte_perm(R1, 0, sel), 0u));
-            ok[half] = (C - nb - 0x00010001u) & (C - tmin1) & 0x80008000u;  // > neighbours, > minTh
-            oi[half] = ok[half] & (C - tini1);                                // and > iniTh
-          }
-          kmin[hh] |= (unsigned long long)nibble4(ok[0], ok[1]) << (4 * k);
-          kini[hh] |= (unsigned long long)nibble4(oi[0], oi[1]) << (4 * k);
-          p0 = c0w, p1 = c1w, p2 = c2w;
-          c0w = n0, c1w = n1, c2w = n2;
-        }
+        const uint32_t* r0 = bits + y * bw + (cx0 >> 5);
+        const uint32_t* r1 = bits + (Dh + y) * bw + (cx0 >> 5);
+        const int sh = cx0 & 31;
+        kmin[hh] = (((unsigned long long)__funnelshift_r(r0[1], r0[2], sh) << 32) | __funnelshift_r(r0[0], r0[1], sh)) & cm;
+        kini[hh] = (((unsigned long long)__funnelshift_r(r1[1], r1[2], sh) << 32) | __funnelshift_r(r1[0], r1[1], sh)) & cm;
       }
     }
     const bool any_ini = __any_sync(0xFFFFFFFFu, (kini[0] | kini[1]) != 0ull);
@@ -343,6 +394,15 @@ __global__ void __launch_bounds__(FB_THREADS, FB_MIN_BLOCKS) fast_bands_kernel(c
     }
     if (lane == 0) cell_counts[(int64_t)f * g.total_cells + ci] = base;
   }
+#ifdef SS_FAST_PHASES
+  __syncthreads();
+  FAST_TS(4);
+  if (threadIdx.x == 0 && blockIdx.y * gridDim.x + blockIdx.x < 4096) {
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    g_fast_ts[bd.level != 0][blockIdx.y * gridDim.x + blockIdx.x][5] = smid;
+  }
+#endif
 }
 
 }  // namespace
@@ -356,9 +416,16 @@ size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int*
   if (((m >> 2) & 1) == 0) m += 4;  // odd word pitch: lane-per-row reads hit distinct banks
   *mbw = m;
   *mband_bytes = ((g.max_band_h + 2) * m + 16 + 15) & ~15;  // + 16: the NMS word reads pass the last row
-  *nball = 0;
-  return (size_t)*region_bytes + *mband_bytes;
+  const int bw = (m + 31) / 32 + 2;  // bit-plane words per row (+ 2: the 64-bit cell reads)
+  *nball = *region_bytes + *mband_bytes;  // bit planes [2][max_band_h][bw] + cell starts [bw]
+  return (size_t)*nball + (size_t)(2 * g.max_band_h + 1) * bw * 4;
 }
+
+#ifdef SS_FAST_PHASES
+extern "C" int ss_dbg_fast_ts(unsigned long long* out) {  // [2][4096][8]
+  return (int)cudaMemcpyFromSymbol(out, g_fast_ts, sizeof(g_fast_ts));
+}
+#endif
 
 cudaError_t fast_init() {  // ss_create, per device; ss_create rejects bands above 227 KB
   return set_max_dynamic_smem(fast_bands_kernel);
@@ -371,7 +438,7 @@ cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const B
   const size_t smem = fast_smem_bytes(g, &rp, &mbw, &rb, &mb, &nb);
   dim3 grid(n_bands, n_frames);
   cudaError_t e = launch_pdl(fast_bands_kernel, grid, dim3(FB_THREADS), smem, s, g, src, bands, cells, slots,
-                             cell_counts, rp, mbw, rb);
+                             cell_counts, rp, mbw, rb, nb);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 

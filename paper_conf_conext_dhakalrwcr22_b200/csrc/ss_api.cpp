@@ -157,6 +157,7 @@ struct ss_ctx {
   PatchMaps maps{};                  // TMA maps of the describe kernel (levels >= 1 at ss_create)
   // test hooks: lanes per WINDOW query (0 = chosen per launch), blurred-sample capture buffer
   int win_lanes = 0;
+  bool fast_split = false;  // SS_FAST_SPLIT=1: level 0's FAST on a side branch beside the pyramid (A/B)
   bool tick_fork = true;  // ss_track_tick: local-map projection on the aux branch (SS_TICK_FORK=0: serial)
   uint8_t* dbg_samples = nullptr;
   int32_t* stereo_sad = nullptr;  // O12: accepted SAD per left keypoint [max_frames/2][cap]
@@ -511,7 +512,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
 #define ALLOC(ptr, bytes)                          \
   if (e == cudaSuccess) e = dalloc(&(ptr), (bytes));
   ALLOC(c->cells, sizeof(CellInfo) * c->cells_h.size());
-  ALLOC(c->bands, sizeof(BandInfo) * c->bands_h.size());
+  ALLOC(c->bands, sizeof(BandInfo) * c->bands_h.size() * 2);  // [ordered by level | merged-launch order]
   ALLOC(c->xytab, sizeof(uint32_t) * tab.size());
   ALLOC(c->qtab, sizeof(uint32_t) * g.qtab_total);
   if (!plan.empty()) ALLOC(c->pyr_plan, sizeof(PyrLvl) * plan.size());
@@ -570,6 +571,14 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (e == cudaSuccess) e = grid_init();
   if (e == cudaSuccess) e = cudaMemcpy(c->cells, c->cells_h.data(), sizeof(CellInfo) * c->cells_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->bands, c->bands_h.data(), sizeof(BandInfo) * c->bands_h.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) {
+    // the one-launch FAST order: levels >= 1 (segments of up to 8 cells) before level 0's (up
+    // to 4), larger work units first so the last wave is the shorter one
+    std::vector<BandInfo> mo(c->bands_h.begin() + g.band_count[0], c->bands_h.end());
+    mo.insert(mo.end(), c->bands_h.begin(), c->bands_h.begin() + g.band_count[0]);
+    e = cudaMemcpy(c->bands + c->bands_h.size(), mo.data(), sizeof(BandInfo) * mo.size(), cudaMemcpyHostToDevice);
+  }
+  c->fast_split = std::getenv("SS_FAST_SPLIT") && std::atoi(std::getenv("SS_FAST_SPLIT")) != 0;
   if (e == cudaSuccess && !tab.empty()) e = cudaMemcpy(c->xytab, tab.data(), sizeof(uint32_t) * tab.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess && !plan.empty())
     e = cudaMemcpy(c->pyr_plan, plan.data(), sizeof(PyrLvl) * plan.size(), cudaMemcpyHostToDevice);
@@ -628,33 +637,46 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
   SS_CUDA_TRY(check_stream(s));
   const Geom& g = c->g;
   FrameSrc src{d_frames, frame_stride, pitch, c->pyr};
-  // DAG: level 0's FAST runs on side stream 0 (it needs no pyramid) while the caller's stream
-  // builds levels 1..L-1 and runs their FAST (one launch each: per-level launches cost more in
-  // launch latency than the overlap saves); the distribution of ALL levels is one launch after
-  // the join (one (level, frame) CTA each), then describe.
+  // The chain: pyramid (levels 1..L-1, one launch), FAST of all levels (one launch; its grid
+  // fills the GPU better than two launches of which level 0's ran beside the pyramid), the
+  // distribution of all levels (one launch, one (level, frame) CTA each), describe.  With
+  // SS_FAST_SPLIT=1 level 0's FAST runs on side stream 0 beside the pyramid instead (A/B).
   // Profiling events: start, then a (before, after) pair around every launch in this order:
-  // fast l0, pyramid (levels 1..L-1, one launch), fast l>=1, distribute (all levels), describe.
+  // pyramid, fast (all levels), distribute, describe; with SS_FAST_SPLIT: fast l0, pyramid,
+  // fast l>=1, distribute, describe.
   prof_mark(c, s);
   SS_CUDA_TRY(cudaMemsetAsync(c->ovf_counter, 0, sizeof(int32_t) * 4, s));
-  SS_CUDA_TRY(cudaEventRecord(c->ev_fork, s));
-  // with profiling events installed the level-0 branch runs in line on `stream`, so every
-  // kernel is timed alone (the fork/join only changes overlap, not any kernel's work)
-  cudaStream_t q = c->prof.empty() ? c->side[0] : s;
-  if (q != s) SS_CUDA_TRY(cudaStreamWaitEvent(q, c->ev_fork, 0));
-  prof_mark(c, q);
-  SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands, g.band_count[0], c->cells, c->slots, c->cell_counts, q));
-  prof_mark(c, q);
-  if (q != s) SS_CUDA_TRY(cudaEventRecord(c->ev_join[0], q));
-  prof_mark(c, s);
-  if (g.L > 1)
-    SS_CUDA_TRY(launch_pyramid(g, n_frames, src, c->pyr_gtab, c->xytab, c->pyr_plan, c->pyr_blocks, c->pyr_buf0,
-                               c->pyr_buf1, c->pyr_smem, s));
-  prof_mark(c, s);
-  prof_mark(c, s);
-  SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands + g.band_count[0], g.total_bands - g.band_count[0],
-                                c->cells, c->slots, c->cell_counts, s));
-  prof_mark(c, s);
-  if (q != s) SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[0], 0));
+  if (c->fast_split) {
+    SS_CUDA_TRY(cudaEventRecord(c->ev_fork, s));
+    // with profiling events installed the level-0 branch runs in line on `stream`, so every
+    // kernel is timed alone (the fork/join only changes overlap, not any kernel's work)
+    cudaStream_t q = c->prof.empty() ? c->side[0] : s;
+    if (q != s) SS_CUDA_TRY(cudaStreamWaitEvent(q, c->ev_fork, 0));
+    prof_mark(c, q);
+    SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands, g.band_count[0], c->cells, c->slots, c->cell_counts, q));
+    prof_mark(c, q);
+    if (q != s) SS_CUDA_TRY(cudaEventRecord(c->ev_join[0], q));
+    prof_mark(c, s);
+    if (g.L > 1)
+      SS_CUDA_TRY(launch_pyramid(g, n_frames, src, c->pyr_gtab, c->xytab, c->pyr_plan, c->pyr_blocks, c->pyr_buf0,
+                                 c->pyr_buf1, c->pyr_smem, s));
+    prof_mark(c, s);
+    prof_mark(c, s);
+    SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands + g.band_count[0], g.total_bands - g.band_count[0],
+                                  c->cells, c->slots, c->cell_counts, s));
+    prof_mark(c, s);
+    if (q != s) SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[0], 0));
+  } else {
+    prof_mark(c, s);
+    if (g.L > 1)
+      SS_CUDA_TRY(launch_pyramid(g, n_frames, src, c->pyr_gtab, c->xytab, c->pyr_plan, c->pyr_blocks, c->pyr_buf0,
+                                 c->pyr_buf1, c->pyr_smem, s));
+    prof_mark(c, s);
+    prof_mark(c, s);
+    SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands + g.total_bands, g.total_bands, c->cells, c->slots,
+                                  c->cell_counts, s));
+    prof_mark(c, s);
+  }
   prof_mark(c, s);
   if (c->dist_mode == SS_DIST_GRID_TOPN)
     SS_CUDA_TRY(launch_distribute_grid(g, n_frames, 0, g.L, c->cells, c->slots, c->cell_counts, c->selected,

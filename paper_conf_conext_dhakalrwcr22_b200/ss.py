@@ -257,7 +257,9 @@ def ss_profile_next(ctx) -> int:
 
 def extract_kernels(n_levels: int) -> list[str]:
     """Kernel launches of one ss_orb_extract in profiling-event order (include/ss.h)."""
-    return ["fast_l0", "pyramid", "fast_l1plus", "distribute", "describe"]
+    if os.environ.get("SS_FAST_SPLIT", "0") not in ("", "0"):  # level 0's FAST beside the pyramid (A/B)
+        return ["fast_l0", "pyramid", "fast_l1plus", "distribute", "describe"]
+    return ["pyramid", "fast", "distribute", "describe"]
 
 
 def extract_events(n_levels: int) -> int:
