@@ -358,6 +358,10 @@ def kernel_work(name: str, p, B: int, cand_l: list, kps_l: list, nq: int, n_map:
         return "hbm", float(sum(kps_l)) / 2 * (20 + 32 + 121 + 231)  # half of the images are left ones
     if name == "lastframe":  # per last-frame point: 24 B point + 32 B descriptor read, 12 B written
         return "hbm", float(nlf * 68)
+    if name == "lf_prepare":  # per keypoint slot: 20 B keypoint + 1 B taken read; 2 x 8 B claims, 1 B mask, 4 B index written
+        return "hbm", float(B * p.kp_capacity * (20 + 1 + 16 + 1 + 4))
+    if name == "lf_finish":  # per last-frame point: 12 B match + 8 B claim + 8 B angles read, 12 B written
+        return "hbm", float(nlf * 40)
     if name == "project":  # map point 32 B + frame index 4 B read, query 20 B written
         return "hbm", float(nq * 56)
     if name == "match_resolve":

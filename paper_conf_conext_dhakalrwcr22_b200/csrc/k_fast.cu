@@ -54,7 +54,10 @@ namespace {
 constexpr int FB_WARPS = SS_FAST_WARPS;
 constexpr int FB_THREADS = FB_WARPS * 32;
 constexpr int ROWS_PER_TASK = SS_FAST_ROWS;  // rows per score task (sliding 7-row window)
-constexpr int FB_MIN_BLOCKS = 24 / FB_WARPS > 1 ? 24 / FB_WARPS : 1;  // 80 registers
+#ifndef SS_FAST_MINB
+#define SS_FAST_MINB (24 / FB_WARPS > 1 ? 24 / FB_WARPS : 1)
+#endif
+constexpr int FB_MIN_BLOCKS = SS_FAST_MINB;  // 3: 80 registers
 
 // The band is staged with every byte XOR 0x80, so a byte read as a signed char is I - 128
 // (order preserving).  A PRMT whose selector nibbles set the sign-replicate bit turns two

@@ -123,8 +123,10 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
   // memory; with one CTA per frame also the descriptors and the taken mask, so the window
   // walk of P1 never waits on global memory (a cluster CTA reads descriptors from L2)
   extern __shared__ __align__(16) uint4 s_dyn[];
+  const int cap8 = (cap + 7) & ~7;
   uint4* s_desc = s_dyn;                                                          // [cap][2] (kCluster == 1)
-  float2* s_xy = reinterpret_cast<float2*>(s_dyn + (kCluster == 1 ? 2 * cap : 0));  // [cap]
+  uint16_t* s_lx = reinterpret_cast<uint16_t*>(s_dyn + (kCluster == 1 ? 2 * cap : 0));  // [cap8] keypoint lx
+  float2* s_xy = reinterpret_cast<float2*>(s_lx + cap8);                          // [cap]
   uint16_t* fri = reinterpret_cast<uint16_t*>(s_xy + cap);                        // [rows_per_frame]
   uint8_t* s_taken = reinterpret_cast<uint8_t*>(fri + a.rows_per_frame);          // [cap] (kCluster == 1)
   unsigned long long* fclaim = a.claim + (int64_t)f * cap;
@@ -133,7 +135,11 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
   const uint4* gdesc = reinterpret_cast<const uint4*>(a.desc + (int64_t)f * cap * SS_DESC_BYTES);
   for (int k = threadIdx.x; k < cap; k += kThreads) {  // P0
     rowidx_fill(g, fk, cnt, fri, k);
-    if (k < nk) s_xy[k] = make_float2(fk[k].x, fk[k].y);
+    if (k < nk) {
+      const ss_keypoint kp = fk[k];
+      s_xy[k] = make_float2(kp.x, kp.y);
+      s_lx[k] = (uint16_t)kp.lx;
+    }
     if constexpr (kCluster == 1) {
       if (k < nk) {
         s_desc[2 * k] = gdesc[2 * k];
@@ -192,18 +198,33 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
             window_rows(g, l, v, r, &rlo, &rhi);
             const uint16_t* ri = fri + s_roff[l];
             const int kb = ri[rlo], ke = ri[rhi];
-            for (int k = kb + sub; k < ke; k += kLanes) {
-              const float2 xy = s_xy[k];
-              const float dx = __fsub_rn(xy.x, u), dy = __fsub_rn(xy.y, v);
-              if (!(fabsf(dx) < r && fabsf(dy) < r)) continue;
-              if (ft && ft[k]) continue;
-              const int d = hamming256(qa, qb, fd[2 * k], fd[2 * k + 1]);
-              const unsigned long long key = ((unsigned long long)d << 32) | (unsigned)k;
-              if (key < b1) {
-                b2 = b1;
-                b1 = key;
-              } else if (key < b2) {
-                b2 = key;
+            // the rows' keypoints in 8-keypoint chunks of the lx array, prefiltered against the
+            // level's column range (a superset of |x - u| < r); survivors take the exact tests
+            const unsigned cr = col_range(g, l, u, r);
+            const unsigned lo = cr & 0xFFFFu, span = (cr >> 16) - lo;
+            for (int ch = (kb >> 3) + sub; ch < (ke + 7) >> 3; ch += kLanes) {
+              const int k0 = ch * 8;
+              const uint4 x8 = reinterpret_cast<const uint4*>(s_lx)[ch];
+              unsigned m = ((x8.x & 0xFFFFu) - lo <= span ? 0x01u : 0u) | ((x8.x >> 16) - lo <= span ? 0x02u : 0u) |
+                           ((x8.y & 0xFFFFu) - lo <= span ? 0x04u : 0u) | ((x8.y >> 16) - lo <= span ? 0x08u : 0u) |
+                           ((x8.z & 0xFFFFu) - lo <= span ? 0x10u : 0u) | ((x8.z >> 16) - lo <= span ? 0x20u : 0u) |
+                           ((x8.w & 0xFFFFu) - lo <= span ? 0x40u : 0u) | ((x8.w >> 16) - lo <= span ? 0x80u : 0u);
+              m &= (0xFFu << max(kb - k0, 0)) & (0xFFu >> max(k0 + 8 - ke, 0));
+              while (m) {
+                const int k = k0 + __ffs(m) - 1;
+                m &= m - 1;
+                const float2 xy = s_xy[k];
+                const float dx = __fsub_rn(xy.x, u), dy = __fsub_rn(xy.y, v);
+                if (!(fabsf(dx) < r && fabsf(dy) < r)) continue;
+                if (ft && ft[k]) continue;
+                const int d = hamming256(qa, qb, fd[2 * k], fd[2 * k + 1]);
+                const unsigned long long key = ((unsigned long long)d << 32) | (unsigned)k;
+                if (key < b1) {
+                  b2 = b1;
+                  b1 = key;
+                } else if (key < b2) {
+                  b2 = key;
+                }
               }
             }
           }
@@ -299,7 +320,8 @@ cudaError_t lastframe_init() {  // at ss_create (never inside a stream capture)
 }
 
 size_t lastframe_smem_bytes(const Geom& g) {
-  const size_t base = sizeof(float2) * (size_t)g.kp_capacity + sizeof(uint16_t) * (size_t)match_rows_per_frame(g);
+  const size_t base = sizeof(float2) * (size_t)g.kp_capacity + sizeof(uint16_t) * (size_t)match_rows_per_frame(g) +
+                      sizeof(uint16_t) * (size_t)((g.kp_capacity + 7) & ~7);
   return kCluster == 1 ? base + (size_t)SS_DESC_BYTES * g.kp_capacity + (size_t)g.kp_capacity : base;
 }
 
@@ -308,7 +330,9 @@ cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams,
                              const int32_t* pt_off, const ss_frame_point* pts, const uint8_t* pdesc, float th,
                              int th_high, int check_orientation, int min_matches, ss_match* out, int32_t* n_matches,
                              uint8_t* matched, unsigned long long* claim, uint16_t* rowidx,
-                             unsigned long long* win_claim, cudaStream_t s) {
+                             unsigned long long* win_claim, int n_sm, cudaStream_t s, void (*mark)(void*),
+                             void* mark_arg) {
+  (void)n_sm;
   if (n_frames <= 0) return cudaSuccess;
   LfArgs a{g,     n_frames, cams,    last_cams,         mb,          kps, desc, counts,
            taken, pt_off,   pts,     pdesc,             th,          th_high, check_orientation,
@@ -316,6 +340,7 @@ cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams,
            match_index_stride(g)};
   const size_t smem = lastframe_smem_bytes(g);
   if (smem > kLfSmemMax) return cudaErrorInvalidValue;
+  if (mark) mark(mark_arg);
   cudaError_t e;
   if constexpr (kCluster > 1) {  // a thread-block cluster per frame (+ programmatic serialisation)
     cudaLaunchConfig_t cfg = {};
@@ -336,6 +361,7 @@ cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams,
   } else {
     e = launch_pdl(lastframe_kernel, dim3(n_frames), dim3(kThreads), smem, s, a);
   }
+  if (mark) mark(mark_arg);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 

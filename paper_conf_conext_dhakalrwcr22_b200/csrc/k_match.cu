@@ -52,12 +52,6 @@ __global__ void __launch_bounds__(256) match_prepare(Geom g, int F, const ss_key
 // atomicMin on packed (distance << 16 | index) keys (index < 65536): b1 takes min(b1, key), b2
 // takes min(b2, max(old b1, key)) -- keys are distinct (the index), so b1 ends as the minimum
 // and b2 as the second (the minimum is never the larger of a pair).
-__device__ __forceinline__ unsigned col_range(const Geom& g, int l, float u, float r) {  // lo | hi << 16
-  const float is_l = g.inv_scale[l];
-  const float lo = fminf(fmaxf(floorf(__fsub_rn(u, r) * is_l) - 1.0f, 0.0f), 65535.0f);
-  const float hi = fminf(fmaxf(ceilf(__fadd_rn(u, r) * is_l) + 1.0f, 0.0f), 65535.0f);
-  return (unsigned)lo | ((unsigned)hi << 16);
-}
 
 template <int QW>
 __global__ void __launch_bounds__(256) match_window_kernel(Geom g, int F, const ss_keypoint* __restrict__ kps,

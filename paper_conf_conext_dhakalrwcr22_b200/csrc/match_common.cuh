@@ -53,6 +53,16 @@ __device__ __forceinline__ void window_rows(const Geom& g, int l, float v, float
   *rhi = max(0, min(hl, (int)ceilf(__fadd_rn(v, r) * is_l) + 2));
 }
 
+// Columns [lo, hi] of level l (lo | hi << 16) that can hold |x - u| < r: floor / ceil of
+// (u -+ r) / scale, widened by one column (a superset, as window_rows is for the rows); the
+// exact f32 test decides.
+__device__ __forceinline__ unsigned col_range(const Geom& g, int l, float u, float r) {  // lo | hi << 16
+  const float is_l = g.inv_scale[l];
+  const float lo = fminf(fmaxf(floorf(__fsub_rn(u, r) * is_l) - 1.0f, 0.0f), 65535.0f);
+  const float hi = fminf(fmaxf(ceilf(__fadd_rn(u, r) * is_l) + 1.0f, 0.0f), 65535.0f);
+  return (unsigned)lo | ((unsigned)hi << 16);
+}
+
 // top-2 of two packed (distance << 32 | index) pairs
 __device__ __forceinline__ void merge_top2(unsigned long long& a1, unsigned long long& a2, unsigned long long b1,
                                            unsigned long long b2) {

@@ -11,6 +11,7 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <utility>
 #include <vector>
 
 #include "ss_internal.h"
@@ -920,11 +921,15 @@ ss_status ss_match_last_frame(ss_ctx* c, int32_t n_frames, const ss_camera* d_ca
   SS_CUDA_TRY(cudaSetDevice(c->device));
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   SS_CUDA_TRY(check_stream(s));
-  prof_mark(c, s);
+  std::pair<ss_ctx*, cudaStream_t> pm{c, s};
   SS_CUDA_TRY(launch_lastframe(c->g, n_frames, d_cams, mb > 0.0f ? d_last_cams : nullptr, mb, d_kps, d_desc, d_counts,
                                d_kp_taken, d_point_offsets, d_points, d_point_desc, th, th_high, check_orientation,
-                               min_matches, d_out, d_n_matches, d_kp_matched, c->claim_lf, c->rowidx, c->claim, s));
-  prof_mark(c, s);
+                               min_matches, d_out, d_n_matches, d_kp_matched, c->claim_lf, c->rowidx, c->claim, c->n_sm, s,
+                               [](void* p) {
+                                 auto* q = static_cast<std::pair<ss_ctx*, cudaStream_t>*>(p);
+                                 prof_mark(q->first, q->second);
+                               },
+                               &pm));
   c->win_ready = true;
   c->win_kps = d_kps;
   c->win_counts = d_counts;

@@ -236,8 +236,8 @@ cudaError_t launch_stereo(const Geom& g, int n_pairs, FrameSrc src, const ss_key
 cudaError_t launch_stereo_outliers(const Geom& g, int n_pairs, const int32_t* counts, const int32_t* sad,
                                    float* uright, float* depth, cudaStream_t s);
 
-// O13 frame-to-frame projection matching (k_lastframe.cu): one cluster of CTAs per frame;
-// dynamic shared memory per CTA (keypoint positions + row index), at most 200 KB.
+// O13 frame-to-frame projection matching (k_lastframe.cu): one CTA (or cluster) per frame;
+// dynamic shared memory per CTA (keypoint positions + lx + row index [+ descriptors]), <= 200 KB.
 size_t lastframe_smem_bytes(const Geom& g);
 cudaError_t lastframe_init();  // kernel attributes (ss_create)
 // Kernel attributes (the >48 KB dynamic shared-memory opt-in) of the other kernels.  Attributes
@@ -254,7 +254,8 @@ cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams,
                              const int32_t* pt_off, const ss_frame_point* pts, const uint8_t* pdesc, float th,
                              int th_high, int check_orientation, int min_matches, ss_match* out, int32_t* n_matches,
                              uint8_t* matched, unsigned long long* claim, uint16_t* rowidx,
-                             unsigned long long* win_claim, cudaStream_t s);
+                             unsigned long long* win_claim, int n_sm, cudaStream_t s, void (*mark)(void*),
+                             void* mark_arg);  // mark: profiling-event hook before / after each launch
 
 // Quadtree key tables of every level (ss_create, once): qtab[g.qtab_total] u32.
 cudaError_t launch_distribute_tables(const Geom& g, uint32_t* qtab, cudaStream_t s);
