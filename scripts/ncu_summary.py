@@ -2,8 +2,8 @@
 per-launch DRAM traffic bench.py reports as roofline.traffic).
 
 usage: python scripts/ncu_summary.py REPORT.ncu-rep CONFIG OUT_SUMMARY.json [TRAFFIC.json]
-Kernel launches are grouped like bench.py's per-kernel events: fast / distribute launches
-with the smaller grid of their pair are the level-0 ones (fast_l0, distribute_l0).
+Kernel launches are grouped like bench.py's per-kernel events: when fast / distribute run as
+two launches per extract (SS_FAST_SPLIT=1, round 1), the smaller grid of the pair is level 0's.
 """
 import csv
 import io
@@ -52,6 +52,8 @@ def main():
     # level-0 vs levels >= 1 by grid size within each kind
     for kind in ("fast", "distribute"):
         grids = sorted({x["launch__grid_size"] for x in launches if x["kernel"] == kind})
+        if len(grids) < 2:  # one launch per extract (the default since round 2): keep the name
+            continue
         for x in launches:
             if x["kernel"] == kind:
                 x["kernel"] = f"{kind}_l0" if x["launch__grid_size"] == grids[0] else f"{kind}_l1plus"

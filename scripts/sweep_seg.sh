@@ -6,9 +6,9 @@ python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
 for V in ${SEGS:-"8 8" "4 8" "3 8" "4 4" "2 4" "8 4"}; do
   set -- $V
   for rep in 1 2; do
-    SS_SEG0=$1 SS_SEG=$2 timeout 600 python bench.py --no-cpu-baseline > $OUT/seg_$1_$2_$rep.json 2> /dev/null
+    SS_SEG0=$1 SS_SEG=$2 timeout 600 python bench.py --config ${CFG:-c2} --no-cpu-baseline > $OUT/seg_$1_$2_$rep.json 2> /dev/null
     python -c "
 import json; d=json.loads(open('$OUT/seg_$1_$2_$rep.json').read().strip().splitlines()[-1])
-k=d['kernels_us']; print('seg0=$1 seg=$2', round(d['value']), 'steady', round(d['steady_state']['value']), 'fast', round(k['fast_l0'],1), round(k['fast_l1plus'],1), 'p50', round(d['latency_ms']['p50'],4), [round(r['frac'],3) for r in d['rooflines'] if r['kernel'].startswith('fast')])"
+k=d['kernels_us']; print('seg0=$1 seg=$2 ${CFG:-c2}', round(d['value']), 'steady', round(d['steady_state']['value']), 'fast', [round(v,1) for n,v in k.items() if n.startswith('fast')], 'p50', round(d['latency_ms']['p50'],4), [round(r['frac'],3) for r in d['rooflines'] if r['kernel'].startswith('fast')])"
   done
 done
