@@ -378,9 +378,11 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   // FAST work units: runs of <= kSegCells consecutive cells of one row (same level and detect
   // rows; their windows tile [x0, x1)), biggest levels first in the grid.  8 measured best
   // on B200 (c2: 2..24 swept; smaller runs pay more halo, larger ones lose parallelism).
-  // level 0: runs of <= 4 (168 -> 336 CTAs for 4 EuRoC frames: the 8-cell runs left 20 SMs with two
-  // CTAs and the rest idle half the launch; fast_l0 18.2 -> 15.6 us, scripts/sweep_seg.sh)
-  int kSegCells = 8, kSegCells0 = 4;  // levels >= 1 / level 0 (SS_SEG / SS_SEG0 override: experiments)
+  // Level 0 too since FAST is one launch for all levels (round 2: 8-cell level-0 runs give
+  // fewer, longer CTAs after the levels >= 1 ones; c2 fast 30.4 -> 28.1 us, 92.0k -> 94-96k
+  // frames/s on one box, scripts/sweep_seg.sh; the 4-cell runs had paid off only while level 0
+  // was a launch of its own beside the pyramid).
+  int kSegCells = 8, kSegCells0 = 8;  // levels >= 1 / level 0 (SS_SEG / SS_SEG0 override: experiments)
   if (const char* e = std::getenv("SS_SEG")) kSegCells = imax(1, std::atoi(e));
   if (const char* e = std::getenv("SS_SEG0")) kSegCells0 = imax(1, std::atoi(e));
   g.max_band_w = g.max_band_h = g.max_cell_w = 0;

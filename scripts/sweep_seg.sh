@@ -3,7 +3,7 @@
 set -u
 OUT=gpurun_out; mkdir -p $OUT
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
-for V in ${SEGS:-"8 8" "4 8" "3 8" "4 4" "2 4" "8 4"}; do
+for V in ${SEGS:-"8 8" "12 8" "8 12" "12 12" "24 8"}; do
   set -- $V
   for rep in 1 2; do
     SS_SEG0=$1 SS_SEG=$2 timeout 600 python bench.py --config ${CFG:-c2} --no-cpu-baseline > $OUT/seg_$1_$2_$rep.json 2> /dev/null
