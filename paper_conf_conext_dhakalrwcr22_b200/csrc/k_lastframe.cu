@@ -3,51 +3,37 @@
 // "ORB-Matching" step of the paper's tracking breakdown (§5, Fig. 8;
 // DESIGN.md §3 item 14, include/ss.h ss_match_last_frame).
 //
-// ONE launch for the whole step: one 1024-thread CTA per frame (kCluster = 1, the default; a
-// build with SS_LF_CLUSTER=8 spreads a frame over a thread-block cluster of 8 x 512 threads
-// with DSMEM histograms instead).  The step has three frame-wide dependencies (the dedup of
-// keypoints claimed by several points, the rotation histogram's three maxima, and the "fewer
-// than min_matches -> redo with 2*th" retry), which are block (or cluster) barriers here
-// instead of kernel boundaries:
-//   P0  every CTA stages the frame's keypoint positions and builds its row index (first
-//       keypoint per (level, row)) in shared memory; claims reset; the cluster also writes
-//       the window matcher's global row index and resets its claims (match_prepare's work,
-//       so the following search-local-points match skips that launch); | cluster.sync
-//   P1  four lanes per point: pose transform + pinhole projection + bounds (single-rounded
-//       f32 ops in the oracle's order), octave-scaled window, level gate, exact |x-u| < r,
-//       |y-v| < r, 8 x POPC Hamming over the candidate runs of the row index, shuffle merge
-//       of packed (d << 32 | k) top-2; accepted -> atomicMin claim (pass tag | d | point);
-//                                                                              | cluster.sync
-//   P2  claim lost -> rejected; else rotation bin -> histogram in the leader CTA's shared
-//       memory (DSMEM atomics);                                                | cluster.sync
-//   P3  ComputeThreeMaxima of the 30 bins (each CTA once), other bins rejected, survivors
-//       counted in the leader's shared memory;                                 | cluster.sync
+// ONE launch for the whole step: one 1024-thread CTA per frame.  The step has three
+// frame-wide dependencies (the dedup of keypoints claimed by several points, the rotation
+// histogram's three maxima, and the "fewer than min_matches -> redo with 2*th" retry), which
+// are block barriers here instead of kernel boundaries:
+//   P0  stage the frame's keypoint positions, lx, angles, descriptors and taken mask and its
+//       row index (first keypoint per (level, row)) in shared memory; write the window
+//       matcher's global row index and reset its claims (match_prepare's work, so the
+//       following search-local-points match skips that launch); reset this matcher's claims;
+//       each thread's first point is loaded meanwhile;                   | barrier
+//   P1  one thread per point: pose transform + pinhole projection + bounds (single-rounded
+//       f32 ops in the oracle's order), octave-scaled window, level gate, the window rows'
+//       keypoints in 8-keypoint lx chunks prefiltered against the level's column range, exact
+//       |x-u| < r, |y-v| < r, taken mask, 8 x POPC Hamming, top-2 of packed (d << 32 | k);
+//       accepted -> atomicMin claim (pass tag | d | point); the match index and the point's
+//       angle stay in shared memory for P2 / P3;                         | barrier
+//   P2  claim lost -> rejected; else rotation bin -> histogram;          | barrier
+//   P3  ComputeThreeMaxima of the 30 bins, other bins rejected, survivors counted; | barrier
 //   retry: if the count is below min_matches, P1-P3 again with 2*th.  Pass-2 claim keys
 //   carry a smaller tag, so they win over stale pass-1 claims without a reset barrier.
-// Latency-bound (a few hundred points per frame, a handful of candidates each).
-#include <cooperative_groups.h>
-
+// Latency-bound (a few hundred points per frame, a handful of candidates each).  Round 1 also
+// had a thread-block-cluster form (8 x 512 threads per frame, DSMEM histograms): slower with
+// ticks in flight, removed in round 2.
 #include "match_common.cuh"
-
-namespace cg = cooperative_groups;
 
 namespace ss {
 
 namespace {
 
-#ifndef SS_LF_CLUSTER
-#define SS_LF_CLUSTER 1
-#endif
-constexpr int kCluster = SS_LF_CLUSTER;           // CTAs per frame (1: one CTA, block barriers)
-#ifndef SS_LF_THREADS
-#define SS_LF_THREADS 1024
-#endif
-constexpr int kThreads = SS_LF_THREADS;  // per CTA
-#ifndef SS_LF_LANES
-#define SS_LF_LANES 1
-#endif
-constexpr int kLanes = SS_LF_LANES;  // lanes per point in P1
-constexpr int kHisto = 30;     // ORB-SLAM HISTO_LENGTH
+constexpr int kThreads = 1024;   // per CTA (one CTA per frame)
+constexpr int kPtCache = 2048;   // points per frame whose P1 results stay in shared memory
+constexpr int kHisto = 30;       // ORB-SLAM HISTO_LENGTH
 constexpr size_t kLfSmemMax = 200 * 1024;
 
 __device__ __forceinline__ float dot3r(const float* a, float b0, float b1, float b2) {
@@ -89,75 +75,69 @@ struct LfArgs {
   int index_stride;                // per-frame stride of the global index (rows + lx section)
 };
 
-// frame-wide barrier: the cluster's when a frame spans several CTAs, else the block's
-__device__ __forceinline__ void frame_sync() {
-  if constexpr (kCluster > 1) cg::this_cluster().sync();
-  else __syncthreads();
-}
-
 __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
   __shared__ int s_hist[2][32];
   __shared__ int s_count[2];
   __shared__ int s_keep[3];
   __shared__ int s_roff[kMaxLevels];
-  const int rank = kCluster > 1 ? (int)cg::this_cluster().block_rank() : 0;
-  const int f = blockIdx.x / kCluster;
-  const int ct = rank * kThreads + threadIdx.x, nct = kCluster * kThreads;
+  __shared__ int s_midx[kPtCache];    // P1's match index of local point j (-1: none / rejected)
+  __shared__ float s_pang[kPtCache];  // the point's angle
+  __shared__ uint8_t s_bin[kPtCache]; // its rotation bin (P2)
+  const int f = blockIdx.x, tid = threadIdx.x;
   const Geom& g = a.g;
   const int L = g.L, cap = g.kp_capacity;
-  if (threadIdx.x < 64) (&s_hist[0][0])[threadIdx.x] = 0;
-  if (threadIdx.x < 2) s_count[threadIdx.x] = 0;
-  if (threadIdx.x < kMaxLevels) s_roff[threadIdx.x] = threadIdx.x < a.g.L ? row_off(a.g, threadIdx.x) : 0;
+  if (tid < 64) (&s_hist[0][0])[tid] = 0;
+  if (tid < 2) s_count[tid] = 0;
+  if (tid < kMaxLevels) s_roff[tid] = tid < a.g.L ? row_off(a.g, tid) : 0;
   pdl_wait();
   pdl_trigger();
-  int* lead_hist = &s_hist[0][0];
-  int* lead_count = &s_count[0];
-  if constexpr (kCluster > 1) {
-    lead_hist = cg::this_cluster().map_shared_rank(&s_hist[0][0], 0);
-    lead_count = cg::this_cluster().map_shared_rank(&s_count[0], 0);
-  }
-
   const ss_keypoint* fk = a.kps + (int64_t)f * cap;
   const int32_t* cnt = a.counts + f * (L + 1);
-  // every CTA keeps its own copy of the frame's keypoint positions and row index in shared
-  // memory; with one CTA per frame also the descriptors and the taken mask, so the window
-  // walk of P1 never waits on global memory (a cluster CTA reads descriptors from L2)
+  const int i0 = a.pt_off[f], i1 = a.pt_off[f + 1];
+  // the thread's first point, loaded while P0 stages the frame
+  ss_frame_point P0v;
+  uint4 qa0 = make_uint4(0, 0, 0, 0), qb0 = qa0;
+  if (i0 + tid < i1) {
+    P0v = a.pts[i0 + tid];
+    const uint4* qd = reinterpret_cast<const uint4*>(a.pdesc + (int64_t)(i0 + tid) * SS_DESC_BYTES);
+    qa0 = qd[0];
+    qb0 = qd[1];
+  }
+  // the frame's keypoints, descriptors, taken mask and row index in shared memory, so the
+  // window walk of P1 never waits on global memory
   extern __shared__ __align__(16) uint4 s_dyn[];
   const int cap8 = (cap + 7) & ~7;
-  uint4* s_desc = s_dyn;                                                          // [cap][2] (kCluster == 1)
-  uint16_t* s_lx = reinterpret_cast<uint16_t*>(s_dyn + (kCluster == 1 ? 2 * cap : 0));  // [cap8] keypoint lx
-  float2* s_xy = reinterpret_cast<float2*>(s_lx + cap8);                          // [cap]
-  uint16_t* fri = reinterpret_cast<uint16_t*>(s_xy + cap);                        // [rows_per_frame]
-  uint8_t* s_taken = reinterpret_cast<uint8_t*>(fri + a.rows_per_frame);          // [cap] (kCluster == 1)
+  uint4* s_desc = s_dyn;                                                      // [cap][2]
+  uint16_t* s_lx = reinterpret_cast<uint16_t*>(s_dyn + 2 * cap);              // [cap8] keypoint lx
+  float2* s_xy = reinterpret_cast<float2*>(s_lx + cap8);                      // [cap]
+  float* s_ang = reinterpret_cast<float*>(s_xy + cap);                        // [cap] keypoint angle
+  uint16_t* fri = reinterpret_cast<uint16_t*>(s_ang + cap);                   // [rows_per_frame]
+  uint8_t* s_taken = reinterpret_cast<uint8_t*>(fri + a.rows_per_frame);      // [cap]
   unsigned long long* fclaim = a.claim + (int64_t)f * cap;
   uint8_t* fmask = a.matched ? a.matched + (int64_t)f * cap : nullptr;
   const int nk = cnt[L];
   const uint4* gdesc = reinterpret_cast<const uint4*>(a.desc + (int64_t)f * cap * SS_DESC_BYTES);
-  for (int k = threadIdx.x; k < cap; k += kThreads) {  // P0
+  for (int k = tid; k < cap; k += kThreads) {  // P0
     rowidx_fill(g, fk, cnt, fri, k);
     if (k < nk) {
       const ss_keypoint kp = fk[k];
       s_xy[k] = make_float2(kp.x, kp.y);
       s_lx[k] = (uint16_t)kp.lx;
+      s_ang[k] = kp.angle_deg;
+      s_desc[2 * k] = gdesc[2 * k];
+      s_desc[2 * k + 1] = gdesc[2 * k + 1];
     }
-    if constexpr (kCluster == 1) {
-      if (k < nk) {
-        s_desc[2 * k] = gdesc[2 * k];
-        s_desc[2 * k + 1] = gdesc[2 * k + 1];
-      }
-      s_taken[k] = a.taken ? a.taken[(int64_t)f * cap + k] : 0;
-    }
-  }
-  for (int k = ct; k < cap; k += nct) {
+    const uint8_t tk = a.taken ? a.taken[(int64_t)f * cap + k] : 0;
+    s_taken[k] = tk;
     fclaim[k] = ~0ull;
-    if (fmask) fmask[k] = (a.taken && a.taken[(int64_t)f * cap + k]) ? 1 : 0;
+    if (fmask) fmask[k] = tk ? 1 : 0;
     if (a.rowidx) {  // the following search-local-points match reuses this index (no match_prepare)
       uint16_t* gri = a.rowidx + (int64_t)f * a.index_stride;
       rowidx_fill(g, fk, cnt, gri, k, gri + lx_off(g));
       a.win_claim[(int64_t)f * cap + k] = ~0ull;
     }
   }
-  frame_sync();
+  __syncthreads();
 
   const ss_camera& c = a.cams[f];
   int dir = 0;  // 1 = forward [o, L-1], 2 = backward [0, o], 0 = [o-1, o+1]
@@ -166,19 +146,27 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
     const float tz = __fadd_rn(dot3r(cl.R + 6, c.ow[0], c.ow[1], c.ow[2]), cl.t[2]);
     dir = tz > a.mb ? 1 : (-tz > a.mb ? 2 : 0);
   }
-  const int i0 = a.pt_off[f], i1 = a.pt_off[f + 1];
-  const uint4* fd = kCluster == 1 ? s_desc : gdesc;
-  const uint8_t* ft = kCluster == 1 ? (a.taken ? s_taken : nullptr) : (a.taken ? a.taken + (int64_t)f * cap : nullptr);
-  const int sub = threadIdx.x % kLanes;
-  const unsigned gmask = ((1u << kLanes) - 1u) << ((threadIdx.x & 31) & ~(kLanes - 1));
+  const uint8_t* ft = a.taken ? s_taken : nullptr;
   int kept = 0;
 
   for (int pass = 0; pass < 2; pass++) {
     const float th = pass ? __fmul_rn(2.0f, a.th) : a.th;
     const unsigned long long tag = pass ? 0ull : (1ull << 62);
-    // P1: search (all lanes of a group run the same trip count)
-    for (int i = i0 + ct / kLanes; i < i1; i += nct / kLanes) {
-      const ss_frame_point P = a.pts[i];
+    // P1: search
+    for (int i = i0 + tid; i < i1; i += kThreads) {
+      const int j = i - i0;
+      ss_frame_point P;
+      uint4 qa, qb;
+      if (pass == 0 && j == tid) {
+        P = P0v;
+        qa = qa0;
+        qb = qb0;
+      } else {
+        P = a.pts[i];
+        const uint4* qd = reinterpret_cast<const uint4*>(a.pdesc + (int64_t)i * SS_DESC_BYTES);
+        qa = qd[0];
+        qb = qd[1];
+      }
       unsigned long long b1 = ~0ull, b2 = ~0ull;
       const int o = P.octave;
       if (o >= 0 && o < L) {
@@ -191,8 +179,6 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
           const float r = __fmul_rn(th, g.scale[o]);
           const int l0 = dir == 1 ? o : (dir == 2 ? 0 : max(o - 1, 0));
           const int l1 = dir == 1 ? L - 1 : (dir == 2 ? o : min(o + 1, L - 1));
-          const uint4* qd = reinterpret_cast<const uint4*>(a.pdesc + (int64_t)i * SS_DESC_BYTES);
-          const uint4 qa = qd[0], qb = qd[1];
           for (int l = l0; l <= l1; l++) {
             int rlo, rhi;
             window_rows(g, l, v, r, &rlo, &rhi);
@@ -202,7 +188,7 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
             // level's column range (a superset of |x - u| < r); survivors take the exact tests
             const unsigned cr = col_range(g, l, u, r);
             const unsigned lo = cr & 0xFFFFu, span = (cr >> 16) - lo;
-            for (int ch = (kb >> 3) + sub; ch < (ke + 7) >> 3; ch += kLanes) {
+            for (int ch = kb >> 3; ch < (ke + 7) >> 3; ch++) {
               const int k0 = ch * 8;
               const uint4 x8 = reinterpret_cast<const uint4*>(s_lx)[ch];
               unsigned m = ((x8.x & 0xFFFFu) - lo <= span ? 0x01u : 0u) | ((x8.x >> 16) - lo <= span ? 0x02u : 0u) |
@@ -217,7 +203,7 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
                 const float dx = __fsub_rn(xy.x, u), dy = __fsub_rn(xy.y, v);
                 if (!(fabsf(dx) < r && fabsf(dy) < r)) continue;
                 if (ft && ft[k]) continue;
-                const int d = hamming256(qa, qb, fd[2 * k], fd[2 * k + 1]);
+                const int d = hamming256(qa, qb, s_desc[2 * k], s_desc[2 * k + 1]);
                 const unsigned long long key = ((unsigned long long)d << 32) | (unsigned)k;
                 if (key < b1) {
                   b2 = b1;
@@ -230,42 +216,44 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
           }
         }
       }
-#pragma unroll
-      for (int s = kLanes / 2; s > 0; s >>= 1) {
-        const unsigned long long o1 = __shfl_xor_sync(gmask, b1, s), o2 = __shfl_xor_sync(gmask, b2, s);
-        merge_top2(b1, b2, o1, o2);
+      ss_match m;
+      m.dist = b1 == ~0ull ? 256 : (int)(b1 >> 32);
+      m.dist2 = b2 == ~0ull ? 256 : (int)(b2 >> 32);
+      m.idx = (b1 != ~0ull && m.dist <= a.th_high) ? (int)(b1 & 0xFFFFFFFFu) : -1;
+      a.out[i] = m;
+      if (j < kPtCache) {
+        s_midx[j] = m.idx;
+        s_pang[j] = P.angle_deg;
       }
-      if (sub == 0) {
-        ss_match m;
-        m.dist = b1 == ~0ull ? 256 : (int)(b1 >> 32);
-        m.dist2 = b2 == ~0ull ? 256 : (int)(b2 >> 32);
-        m.idx = (b1 != ~0ull && m.dist <= a.th_high) ? (int)(b1 & 0xFFFFFFFFu) : -1;
-        a.out[i] = m;
-        if (m.idx >= 0)
-          atomicMin(fclaim + m.idx, tag | ((unsigned long long)m.dist << 32) | (unsigned)(i - i0));
-      }
+      if (m.idx >= 0) atomicMin(fclaim + m.idx, tag | ((unsigned long long)m.dist << 32) | (unsigned)j);
     }
-    frame_sync();
+    __syncthreads();
     // P2: dedup (min (distance, point) per keypoint) + rotation histogram
-    for (int i = i0 + ct; i < i1; i += nct) {
-      const ss_match m = a.out[i];
-      if (m.idx < 0) continue;
-      const unsigned long long mine = tag | ((unsigned long long)m.dist << 32) | (unsigned)(i - i0);
-      if (fclaim[m.idx] != mine) {
+    for (int i = i0 + tid; i < i1; i += kThreads) {
+      const int j = i - i0;
+      const bool cached = j < kPtCache;
+      const int idx = cached ? s_midx[j] : a.out[i].idx;
+      if (idx < 0) continue;
+      const int dist = a.out[i].dist;
+      const unsigned long long mine = tag | ((unsigned long long)dist << 32) | (unsigned)j;
+      if (fclaim[idx] != mine) {
         a.out[i].idx = -1;
+        if (cached) s_midx[j] = -1;
       } else if (a.check_orientation) {
-        atomicAdd(lead_hist + pass * 32 + rot_bin(a.pts[i].angle_deg, fk[m.idx].angle_deg), 1);
+        const int bin = rot_bin(cached ? s_pang[j] : a.pts[i].angle_deg, s_ang[idx]);
+        if (cached) s_bin[j] = (uint8_t)bin;
+        atomicAdd(&s_hist[pass][bin], 1);
       } else {
-        atomicAdd(lead_count + pass, 1);
+        atomicAdd(&s_count[pass], 1);
       }
     }
-    frame_sync();
+    __syncthreads();
     // P3: ComputeThreeMaxima, reject the other bins, count the survivors
     if (a.check_orientation) {
-      if (threadIdx.x == 0) {
+      if (tid == 0) {
         int max1 = 0, max2 = 0, max3 = 0, ind1 = -1, ind2 = -1, ind3 = -1;
         for (int b = 0; b < kHisto; b++) {
-          const int s = lead_hist[pass * 32 + b];
+          const int s = s_hist[pass][b];
           if (s > max1) {
             max3 = max2; max2 = max1; max1 = s;
             ind3 = ind2; ind2 = ind1; ind1 = b;
@@ -290,27 +278,31 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
       }
       __syncthreads();
       const int k1 = s_keep[0], k2 = s_keep[1], k3 = s_keep[2];
-      for (int i = i0 + ct; i < i1; i += nct) {
-        const int idx = a.out[i].idx;
+      for (int i = i0 + tid; i < i1; i += kThreads) {
+        const int j = i - i0;
+        const bool cached = j < kPtCache;
+        const int idx = cached ? s_midx[j] : a.out[i].idx;
         if (idx < 0) continue;
-        const int bin = rot_bin(a.pts[i].angle_deg, fk[idx].angle_deg);
-        if (bin != k1 && bin != k2 && bin != k3)
+        const int bin = cached ? (int)s_bin[j] : rot_bin(a.pts[i].angle_deg, s_ang[idx]);
+        if (bin != k1 && bin != k2 && bin != k3) {
           a.out[i].idx = -1;
-        else
-          atomicAdd(lead_count + pass, 1);
+          if (cached) s_midx[j] = -1;
+        } else {
+          atomicAdd(&s_count[pass], 1);
+        }
       }
-      frame_sync();
+      __syncthreads();
     }
-    kept = lead_count[pass];
-    if (a.min_matches <= 0 || kept >= a.min_matches) break;  // uniform over the cluster
+    kept = s_count[pass];
+    if (a.min_matches <= 0 || kept >= a.min_matches) break;  // uniform over the CTA
   }
-  if (a.n_matches && rank == 0 && threadIdx.x == 0) a.n_matches[f] = kept;
+  if (a.n_matches && tid == 0) a.n_matches[f] = kept;
   if (fmask)  // kept matches are unique per keypoint (dedup), so these stores never collide
-    for (int i = i0 + ct; i < i1; i += nct) {
-      const int idx = a.out[i].idx;
+    for (int i = i0 + tid; i < i1; i += kThreads) {
+      const int j = i - i0;
+      const int idx = j < kPtCache ? s_midx[j] : a.out[i].idx;
       if (idx >= 0) fmask[idx] = 1;
     }
-  frame_sync();  // the leader's shared memory must outlive every remote access
 }
 
 }  // namespace
@@ -319,10 +311,10 @@ cudaError_t lastframe_init() {  // at ss_create (never inside a stream capture)
   return cudaFuncSetAttribute(lastframe_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kLfSmemMax);
 }
 
-size_t lastframe_smem_bytes(const Geom& g) {
-  const size_t base = sizeof(float2) * (size_t)g.kp_capacity + sizeof(uint16_t) * (size_t)match_rows_per_frame(g) +
-                      sizeof(uint16_t) * (size_t)((g.kp_capacity + 7) & ~7);
-  return kCluster == 1 ? base + (size_t)SS_DESC_BYTES * g.kp_capacity + (size_t)g.kp_capacity : base;
+size_t lastframe_smem_bytes(const Geom& g) {  // dynamic part (static: ~19 KB)
+  const size_t cap = (size_t)g.kp_capacity;
+  return (size_t)SS_DESC_BYTES * cap + sizeof(uint16_t) * ((cap + 7) & ~(size_t)7) + sizeof(float2) * cap +
+         sizeof(float) * cap + sizeof(uint16_t) * (size_t)match_rows_per_frame(g) + cap;
 }
 
 cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams, const ss_camera* last_cams, float mb,
@@ -342,25 +334,7 @@ cudaError_t launch_lastframe(const Geom& g, int n_frames, const ss_camera* cams,
   if (smem > kLfSmemMax) return cudaErrorInvalidValue;
   if (mark) mark(mark_arg);
   cudaError_t e;
-  if constexpr (kCluster > 1) {  // a thread-block cluster per frame (+ programmatic serialisation)
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(n_frames * kCluster);
-    cfg.blockDim = dim3(kThreads);
-    cfg.dynamicSmemBytes = smem;
-    cfg.stream = s;
-    cudaLaunchAttribute at[2];
-    at[0].id = cudaLaunchAttributeClusterDimension;
-    at[0].val.clusterDim.x = kCluster;
-    at[0].val.clusterDim.y = 1;
-    at[0].val.clusterDim.z = 1;
-    at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    at[1].val.programmaticStreamSerializationAllowed = 1;
-    cfg.attrs = at;
-    cfg.numAttrs = 2;
-    e = cudaLaunchKernelEx(&cfg, lastframe_kernel, a);
-  } else {
-    e = launch_pdl(lastframe_kernel, dim3(n_frames), dim3(kThreads), smem, s, a);
-  }
+  e = launch_pdl(lastframe_kernel, dim3(n_frames), dim3(kThreads), smem, s, a);
   if (mark) mark(mark_arg);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
