@@ -19,6 +19,23 @@
 
 namespace ss {
 
+#ifdef SS_DESC_PHASES  // per-warp phase timestamps (scripts/desc_phases.py; instrumented builds only)
+__device__ unsigned long long g_desc_ts[16384][8];
+#define DESC_TS(i)                                                                   \
+  do {                                                                               \
+    const int w_ = (blockIdx.y * gridDim.x + blockIdx.x) * DESC_WARPS + (threadIdx.x >> 5); \
+    if ((threadIdx.x & 31) == 0 && w_ < 16384) {                                     \
+      unsigned long long t_;                                                         \
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                         \
+      g_desc_ts[w_][i] = t_;                                                         \
+    }                                                                                \
+  } while (0)
+#else
+#define DESC_TS(i) \
+  do {             \
+  } while (0)
+#endif
+
 namespace {
 
 constexpr int DESC_WARPS = 8;
@@ -105,6 +122,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
                                                                    uint8_t* __restrict__ samples,
                                                                    const __grid_constant__ PatchMaps maps) {
   pdl_trigger();
+  DESC_TS(0);
   extern __shared__ __align__(128) uint8_t sm_raw[];  // DESC_WARPS * PER_WARP + 128
   // 128-B aligned warp buffers (TMA destinations)
   uint8_t* const sm = sm_raw + ((128 - (smem_addr(sm_raw) & 127)) & 127);
@@ -134,6 +152,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
     (t ? s_wu : s_wmask)[(threadIdx.x & 127)] = word;
   }
   pdl_wait();
+  DESC_TS(1);
   if (warp == 0) {  // level offsets: the L counts loaded at once, inclusive warp scan
     int s = lane < L ? sel_counts[f * L + lane] : 0;
 #pragma unroll
@@ -148,6 +167,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
   if (blockIdx.x == 0 && threadIdx.x <= L) counts[f * (L + 1) + threadIdx.x] = off[threadIdx.x];
   const int i = blockIdx.x * DESC_WARPS + warp;
   if (i >= off[L]) return;  // warp-uniform; only warp-level sync below
+  DESC_TS(2);
   int l = 0;
   while (i >= off[l + 1]) l++;
   const uint32_t packed = selected[(int64_t)f * g.kp_capacity + g.cap_off[l] + (i - off[l])];
@@ -197,8 +217,35 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
       if (i < PR * 4) *reinterpret_cast<uint4*>(Pw + (i >> 2) * PP + 16 * (i & 3)) = chunk[k];
     }
     P = Pw + sh;
+  } else if ((ip & 15) == 0 && ip >= 64 && w >= 22) {
+    // near the left/right level border (round 2; was per-byte REFLECT_101 loads in 8 dependent
+    // batches, the describe launch's slowest warps): the 64-column aligned window holding every
+    // in-level column of the patch, rows mapped by REFLECT_101, staged with 16-B loads into the
+    // V region (written only later), then the patch gathered with REFLECT_101 columns
+    const int xl = max(lx - 21, 0), xr = min(lx + 21, w - 1);
+    const int a0 = min(xl & ~15, ip - 64);  // a0 <= xl, xr < a0 + 64 (xr - xl <= 42)
+    uint8_t* Wb = reinterpret_cast<uint8_t*>(V);
+    const uint8_t* cb = img + a0;
+    constexpr int NCH = (PR * 4 + 31) / 32;
+    uint4 chunk[NCH];
+#pragma unroll
+    for (int k = 0; k < NCH; k++) {
+      const int i = lane + 32 * k;
+      if (i < PR * 4) chunk[k] = __ldg(reinterpret_cast<const uint4*>(cb + (int64_t)reflect101(ly - 21 + (i >> 2), h) * ip) + (i & 3));
+    }
+#pragma unroll
+    for (int k = 0; k < NCH; k++) {
+      const int i = lane + 32 * k;
+      if (i < PR * 4) *reinterpret_cast<uint4*>(Wb + (i >> 2) * 64 + 16 * (i & 3)) = chunk[k];
+    }
+    __syncwarp();
+    for (int i = lane; i < PR * PR; i += 32) {
+      const int r = i / PR, c = i - r * PR;
+      Pw[r * PP + c] = Wb[r * 64 + reflect101(lx - 21 + c, w) - a0];
+    }
+    P = Pw;
   } else {
-    // near the left/right level border: REFLECT_101 (the blur's border rule) byte loads, 8 per
+    // tiny levels or an unaligned pitch: REFLECT_101 (the blur's border rule) byte loads, 8 per
     // lane in flight per batch
     constexpr int BB = 8;
 #pragma unroll 1
@@ -221,6 +268,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
     P = Pw;
   }
   __syncwarp();
+  DESC_TS(3);
   // moments over the disk |u| <= umax[|v|] (always inside the level: 19 <= lx < w-19):
   // lane = row v; the row's 31 pixels (plus one zero-weight byte) as 8 words, dotted 4 bytes
   // at a time with the disk mask (S0 = sum I) and with weights u + 15 (S1); m10 = sum of
@@ -278,6 +326,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
     }
   }
   __syncwarp();  // V complete
+  DESC_TS(4);
   // rotated BRIEF: lane = output byte; bit t compares points 2b, 2b+1 with b = 8*lane + t.
   // The blurred value is needed only at the 512 sample points, so the horizontal pass runs
   // there alone: B(oy, ox) = (sum_j k_j V[18 + oy][18 + ox + j] + 2^15) >> 16.
@@ -345,6 +394,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
     }
   }
   desc[o * SS_DESC_BYTES + lane] = (uint8_t)byte;
+  DESC_TS(5);
   if (lane == 0) {
     float ang = 0.f;
     if (m10 != 0 || m01 != 0) {
@@ -364,9 +414,14 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
     kp.reserved = 0;
     kps[o] = kp;
   }
+  DESC_TS(6);
 }
 
 }  // namespace
+
+#ifdef SS_DESC_PHASES
+extern "C" int ss_dbg_desc_ts(unsigned long long* out) { return (int)cudaMemcpyFromSymbol(out, g_desc_ts, sizeof(g_desc_ts)); }
+#endif
 
 const int* brief_pattern_host() { return SS_BRIEF_PATTERN_HOST; }
 
