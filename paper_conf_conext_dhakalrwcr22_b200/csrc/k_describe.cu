@@ -30,9 +30,17 @@ __device__ unsigned long long g_desc_ts[16384][8];
       g_desc_ts[w_][i] = t_;                                                         \
     }                                                                                \
   } while (0)
+#define DESC_PATH(v)                                                                 \
+  do {                                                                               \
+    const int w_ = (blockIdx.y * gridDim.x + blockIdx.x) * DESC_WARPS + (threadIdx.x >> 5); \
+    if ((threadIdx.x & 31) == 0 && w_ < 16384) g_desc_ts[w_][7] = (v) | ((unsigned long long)l << 8); \
+  } while (0)
 #else
 #define DESC_TS(i) \
   do {             \
+  } while (0)
+#define DESC_PATH(v) \
+  do {               \
   } while (0)
 #endif
 
@@ -195,6 +203,7 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
     const int x0 = lx - 21;
     tma_patch(&maps.level[l], Pw, &s_bar[warp], x0 & ~15, ly - 21, f, lane);
     P = Pw + (x0 & 15);
+    DESC_PATH(1);
   } else if ((ip & 15) == 0 && lx >= 21 && lx + 21 < w && lx - 21 - sh + 64 <= ip) {
     // columns inside the level: 43 rows x four aligned 16-B chunks, rows mapped by REFLECT_101
     // (identity away from the top/bottom border); all six loads of a lane are issued before
@@ -217,33 +226,39 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
       if (i < PR * 4) *reinterpret_cast<uint4*>(Pw + (i >> 2) * PP + 16 * (i & 3)) = chunk[k];
     }
     P = Pw + sh;
-  } else if ((ip & 15) == 0 && ip >= 64 && w >= 22) {
+    DESC_PATH(2);
+  } else if ((ip & 15) == 0 && w >= 22) {
     // near the left/right level border (round 2; was per-byte REFLECT_101 loads in 8 dependent
-    // batches, the describe launch's slowest warps): the 64-column aligned window holding every
-    // in-level column of the patch, rows mapped by REFLECT_101, staged with 16-B loads into the
-    // V region (written only later), then the patch gathered with REFLECT_101 columns
-    const int xl = max(lx - 21, 0), xr = min(lx + 21, w - 1);
-    const int a0 = min(xl & ~15, ip - 64);  // a0 <= xl, xr < a0 + 64 (xr - xl <= 42)
-    uint8_t* Wb = reinterpret_cast<uint8_t*>(V);
+    // batches, the describe launch's slowest warps): the 16-B chunks of the aligned 64-column
+    // window from the patch's first in-level column (chunks past the row's end skipped), rows
+    // mapped by REFLECT_101, stored 16 B to the right when the patch starts left of column 0;
+    // then the <= 3 reflected columns per row are copied in shared memory (a row's slot is
+    // 64 B: the shifted row's unused last columns and the next row's left pad overlap)
+    const int a0 = max(lx - 21, 0) & ~15;
+    const int sft = lx < 21 ? 16 : 0;
     const uint8_t* cb = img + a0;
     constexpr int NCH = (PR * 4 + 31) / 32;
     uint4 chunk[NCH];
 #pragma unroll
     for (int k = 0; k < NCH; k++) {
       const int i = lane + 32 * k;
-      if (i < PR * 4) chunk[k] = __ldg(reinterpret_cast<const uint4*>(cb + (int64_t)reflect101(ly - 21 + (i >> 2), h) * ip) + (i & 3));
+      if (i < PR * 4 && a0 + 16 * (i & 3) < ip)
+        chunk[k] = __ldg(reinterpret_cast<const uint4*>(cb + (int64_t)reflect101(ly - 21 + (i >> 2), h) * ip) + (i & 3));
     }
 #pragma unroll
     for (int k = 0; k < NCH; k++) {
       const int i = lane + 32 * k;
-      if (i < PR * 4) *reinterpret_cast<uint4*>(Wb + (i >> 2) * 64 + 16 * (i & 3)) = chunk[k];
+      if (i < PR * 4 && a0 + 16 * (i & 3) < ip) *reinterpret_cast<uint4*>(Pw + (i >> 2) * PP + sft + 16 * (i & 3)) = chunk[k];
     }
     __syncwarp();
-    for (int i = lane; i < PR * PR; i += 32) {
-      const int r = i / PR, c = i - r * PR;
-      Pw[r * PP + c] = Wb[r * 64 + reflect101(lx - 21 + c, w) - a0];
+    for (int r = lane; r < PR; r += 32) {
+      uint8_t* row = Pw + r * PP + sft - a0;  // row[x] = pixel column x of this patch row
+      for (int x = lx - 21; x < 0; x++) row[x] = row[-x];                     // REFLECT_101, left
+      for (int x = w; x <= lx + 21; x++) row[x] = row[2 * w - 2 - x];        // REFLECT_101, right
     }
-    P = Pw;
+    __syncwarp();
+    P = Pw + sft + (lx - 21 - a0);
+    DESC_PATH(3);
   } else {
     // tiny levels or an unaligned pitch: REFLECT_101 (the blur's border rule) byte loads, 8 per
     // lane in flight per batch

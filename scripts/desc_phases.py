@@ -40,3 +40,13 @@ for j, n in enumerate(names):
     print(f"  {n:10s} median {np.median(d[:, j]):.2f}  p90 {np.percentile(d[:, j], 90):.2f}  max {d[:, j].max():.2f} us")
 tot = (t[:, 6] - t[:, 0]) / 1000
 print(f"  warp total median {np.median(tot):.2f} max {tot.max():.2f} us")
+path = t[:, 7] & 0xFF
+lev = (t[:, 7] >> 8) & 0xFF
+for pv, pn in [(0, "bytes"), (1, "tma"), (2, "chunks"), (3, "border")]:
+    m = path == pv
+    if m.any():
+        print(f"  path {pn:7s}: {int(m.sum())} warps, patch median {np.median(d[m, 2]):.2f} max {d[m, 2].max():.2f} us, "
+              f"levels {sorted(set(lev[m].tolist()))}")
+post = (t[:, 6] - t[:, 1]) / 1000
+slow = np.argsort(post)[-8:]
+print("  slowest (post-wait us, path, level, phases):", [(round(post[k], 1), int(path[k]), int(lev[k]), [round(x, 1) for x in d[k, 1:]]) for k in slow])
