@@ -628,8 +628,33 @@ def run_ours(args, cfg):
     W_, K = args.warmup, args.steps
     ev_start = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
     ev_end = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
+    for e in ev_start + ev_end:  # torch creates the CUDA event lazily, at its first record
+        e.record(streams[0])
+    torch.cuda.synchronize(dev)
+
+    # the timed loop launches through the runtime directly (one cudaEventRecord + cudaGraphLaunch
+    # + cudaEventRecord per tick, ~4 us of host time): torch's stream context + Event.record +
+    # CUDAGraph.replay cost ~28 us per tick, and in a short run the GPU waited on that enqueue
+    _launch = _rt.cudaGraphLaunch
+    _record = _rt.cudaEventRecord
+    _launch.argtypes = [ctypes.c_void_p, ctypes.c_void_p]
+    _record.argtypes = [ctypes.c_void_p, ctypes.c_void_p]
+    raw_exec = [[ctypes.c_void_p(g_.raw_cuda_graph_exec()) for g_ in graphs[q]] for q in range(P)]
+    raw_stream = [ctypes.c_void_p(streams[q].cuda_stream) for q in range(P)]
+
+    def run_steps_raw(s0, n, marks):
+        es = [ctypes.c_void_p(e.cuda_event) for e in marks[0][:n]]
+        ee = [ctypes.c_void_p(e.cuda_event) for e in marks[1][:n]]
+        for i in range(n):
+            s = (s0 + i) % n_slots
+            q = (s0 + i) % P
+            st = raw_stream[q]
+            if _record(es[i], st) or _launch(raw_exec[q][s], st) or _record(ee[i], st):
+                raise RuntimeError("cudaGraphLaunch / cudaEventRecord failed")
 
     def run_steps(s0, n, marks=None):
+        if marks is not None and world == 1 and not eager_tail:
+            return run_steps_raw(s0, n, marks)
         for i in range(n):
             s = (s0 + i) % n_slots
             q = (s0 + i) % P
@@ -657,7 +682,9 @@ def run_ours(args, cfg):
         t0.record(streams[0])
         for q in range(1, P):
             streams[q].wait_event(t0)
+        t_host = time.perf_counter()
         run_steps(W_, K, (ev_start, ev_end))
+        host_enqueue_ms = (time.perf_counter() - t_host) * 1e3
         for q in range(1, P):
             streams[0].wait_stream(streams[q])
         t1.record(streams[0])
@@ -880,6 +907,7 @@ def run_ours(args, cfg):
         "rooflines": rooflines,
         "e2e": e2e,
         "gpu_launches": launches_per_step * K * world,
+        "host_enqueue_ms": host_enqueue_ms,  # host time to enqueue the K timed ticks (graph launches + events)
         "clocks": sampler.summary(),
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
