@@ -555,14 +555,14 @@ def run_ours(args, cfg):
         pp, st, ot = pipes[q], streams[q], outs[q]
         if prof:
             ss.ss_profile_events(pp.ctx, events[s])
-        # the local-map projection (cameras + map points only) could run on a forked branch
-        # concurrently with the extraction; measured on c2 with 4 ticks in flight that cost 7 %
-        # of throughput (63.0k -> 58.9k frames/s), so the ring graphs keep it serial (the
-        # per-tick executor ss_track_tick forks it: +1-2 % there)
-        fork = bool(args.fork_project) and window and not prof
+        # the local-map projection (cameras + map points only) runs on a forked branch beside
+        # the frame-to-frame matcher (whose one CTA per frame leaves most SMs free): c2 K=20
+        # 83.5k -> 86.0k frames/s, K=200 unchanged (scripts/ab_forkproj.sh); forked beside the
+        # extraction instead (--fork-project 1) it cost 7 % (94.5k -> 87.4k), serial = 0
+        fork = args.fork_project if window and not prof else 0
         with torch.cuda.graph(g, stream=st):
-            if fork:
-                ev0, ev1 = torch.cuda.Event(), torch.cuda.Event()
+            ev0, ev1 = torch.cuda.Event(), torch.cuda.Event()
+            if fork == 1:  # beside the extraction
                 ev0.record(st)
                 aux_streams[q].wait_event(ev0)
                 pp.project(B, cams[s], points[s], point_frame[s], qbufs[q], th=cfg["th"], stream=aux_streams[q])
@@ -570,6 +570,11 @@ def run_ours(args, cfg):
             pp.extract(frames[s], stream=st)
             if stereo:
                 pp.stereo(frames[s], BF, BASE_M, st_out[q][0], st_out[q][1], stream=st)
+            if fork == 2:  # beside the frame-to-frame matcher (one CTA per frame leaves SMs free)
+                ev0.record(st)
+                aux_streams[q].wait_event(ev0)
+                pp.project(B, cams[s], points[s], point_frame[s], qbufs[q], th=cfg["th"], stream=aux_streams[q])
+                ev1.record(aux_streams[q])
             if window:  # ORB-Matching (O13), then search local points skipping its matches (O11 + O9)
                 pp.match_last_frame(B, cams[s], lf_off[s], lf_pts[s], lf_desc[s], lf_out[q], lf_n[q],
                                     last_cams=lf_last[s] if MB > 0 else None, mb=MB, th=cfg["lf_th"],
@@ -1242,8 +1247,9 @@ def main(argv=None):
                     help="N > 1: NCCL gather on a side stream, or gloo with host-staged slots (ranks may share a GPU)")
     ap.add_argument("--same-device", action="store_true", help="every rank on cuda:0 (multi-rank test on one GPU)")
     ap.add_argument("--clients", type=int, default=0, help="override the config's clients per rank")
-    ap.add_argument("--fork-project", type=int, default=0, choices=[0, 1],
-                    help="ring graphs: run the local-map projection on a forked branch concurrent with the extraction")
+    ap.add_argument("--fork-project", type=int, default=2, choices=[0, 1, 2],
+                    help="ring graphs: run the local-map projection on a forked branch concurrent with the "
+                         "extraction (1) or with the frame-to-frame matcher (2)")
     ap.add_argument("--match-lanes", type=int, default=0, choices=[0, 1, 2, 4, 8],
                     help="lanes per WINDOW query (0 = chosen per launch)")
     ap.add_argument("--dump-gather", default="", help="write the last tick's gathered / own slots to PATH.*.npy")

@@ -5,7 +5,7 @@ OUT=gpurun_out; mkdir -p $OUT
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
 for rep in 1 2; do
   for K in 20 200; do
-    for F in 0 1; do
+    for F in 0 2; do
       timeout 600 python bench.py --steps $K --warmup 5 --fork-project $F --no-cpu-baseline > $OUT/fp_${K}_$F.json 2> /dev/null
       python -c "
 import json; d=json.loads(open('$OUT/fp_${K}_$F.json').read().strip().splitlines()[-1])
