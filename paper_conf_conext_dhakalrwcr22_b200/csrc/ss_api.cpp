@@ -1018,9 +1018,17 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
   }
   // the hot path.  The local-map projection needs only the cameras and map points, so (unless
   // profiling events are installed, which time every kernel alone on `stream`) it forks onto
-  // the ctx's aux stream and overlaps the extraction; the WINDOW match joins it.
+  // the ctx's aux stream after the extraction and overlaps the frame-to-frame matcher (one CTA
+  // per frame: most SMs are free); the WINDOW match joins it.
   ss_status st;
   const bool fork_project = window && c->prof.empty() && c->tick_fork;
+  st = ss_orb_extract(c, n_frames, c->io_frames, fstride, P, c->io_kps, c->io_desc, c->io_counts, stream);
+  if (st != SS_OK) return st;
+  if (stereo) {
+    st = ss_stereo_match(c, n_frames / 2, c->io_frames, fstride, P, c->io_kps, c->io_desc, c->io_counts, io->bf,
+                         io->baseline, c->io_uright, c->io_depth, stream);
+    if (st != SS_OK) return st;
+  }
   if (fork_project) {
     SS_CUDA_TRY(cudaEventRecord(c->ev_aux0, s));
     SS_CUDA_TRY(cudaStreamWaitEvent(c->aux, c->ev_aux0, 0));
@@ -1028,13 +1036,6 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
                            reinterpret_cast<ss_stream_t>(c->aux));
     if (st != SS_OK) return st;
     SS_CUDA_TRY(cudaEventRecord(c->ev_aux1, c->aux));
-  }
-  st = ss_orb_extract(c, n_frames, c->io_frames, fstride, P, c->io_kps, c->io_desc, c->io_counts, stream);
-  if (st != SS_OK) return st;
-  if (stereo) {
-    st = ss_stereo_match(c, n_frames / 2, c->io_frames, fstride, P, c->io_kps, c->io_desc, c->io_counts, io->bf,
-                         io->baseline, c->io_uright, c->io_depth, stream);
-    if (st != SS_OK) return st;
   }
   int64_t n_matches = 0;
   const uint8_t* win_taken = d_taken;
