@@ -764,6 +764,10 @@ def run_ours(args, cfg):
         k0, _, c0 = pipe.results(B)
         qrec = qbufs[0].cpu().numpy().reshape(-1).view(ss.QUERY_DTYPE)
         win_sample = (k0, c0, lf_mask[0].cpu().numpy(), qrec)
+    if getattr(args, "dump_lf_ts", None):  # instrumented builds only (scripts/lf_phases.py)
+        buf = np.zeros(64 * 8 + 64 * 32 + 64 * 64, np.uint64)
+        ss.lib().ss_dbg_lf_ts(buf.ctypes.data_as(ctypes.c_void_p))
+        np.save(args.dump_lf_ts, buf)
     kps_h, desc_h, counts_h = pipe.results(B)  # last step's outputs
     kps_l = [int((counts_h[:, l + 1] - counts_h[:, l]).sum()) for l in range(L)]
     cand_l = [sum(len(ss.ss_debug_candidates(pipe.ctx, b, l)[0]) for b in range(B)) for l in range(L)]
@@ -1241,6 +1245,7 @@ def main(argv=None):
     ap.add_argument("--e2e-inflight", type=int, default=8, help="ticks in flight on the end-to-end (host memory) path")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--dump-lf-ts", default=None, help=argparse.SUPPRESS)  # scripts/lf_phases.py (instrumented build)
     ap.add_argument("--map-shard", action="store_true",
                     help="brute configs: partition the map over the ranks (F4: shard top-2, all-to-all, merge)")
     ap.add_argument("--backend", choices=["nccl", "gloo"], default="nccl",

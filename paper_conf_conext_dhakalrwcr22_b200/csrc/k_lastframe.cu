@@ -29,6 +29,52 @@
 
 namespace ss {
 
+#ifdef SS_LF_PHASES  // phase timestamps per frame CTA + per-warp P1 ends (scripts/lf_phases.py; instrumented builds)
+__device__ unsigned long long g_lf_ts[64][8];
+__device__ unsigned long long g_lf_w[64][32];
+__device__ unsigned long long g_lf_w2[64][32][2];
+#define LF_WTS2(q)                                                                        \
+  do {                                                                                    \
+    if ((threadIdx.x & 31) == 0 && blockIdx.x < 64) {                                     \
+      unsigned long long t_;                                                              \
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                              \
+      g_lf_w2[blockIdx.x][threadIdx.x >> 5][q] = t_;                                      \
+    }                                                                                     \
+  } while (0)
+#define LF_TS(i)                                                   \
+  do {                                                             \
+    if (threadIdx.x == 0 && blockIdx.x < 64) {                     \
+      unsigned long long t_;                                       \
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));       \
+      g_lf_ts[blockIdx.x][i] = t_;                                 \
+    }                                                              \
+  } while (0)
+#define LF_WTS()                                                                          \
+  do {                                                                                    \
+    if ((threadIdx.x & 31) == 0 && blockIdx.x < 64) {                                     \
+      unsigned long long t_;                                                              \
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                              \
+      g_lf_w[blockIdx.x][threadIdx.x >> 5] = t_;                                          \
+    }                                                                                     \
+  } while (0)
+extern "C" int ss_dbg_lf_ts(unsigned long long* out) {
+  cudaError_t e = cudaMemcpyFromSymbol(out, g_lf_ts, sizeof(g_lf_ts));
+  if (e == cudaSuccess) e = cudaMemcpyFromSymbol(out + 64 * 8, g_lf_w, sizeof(g_lf_w));
+  if (e == cudaSuccess) e = cudaMemcpyFromSymbol(out + 64 * 8 + 64 * 32, g_lf_w2, sizeof(g_lf_w2));
+  return (int)e;
+}
+#else
+#define LF_TS(i) \
+  do {           \
+  } while (0)
+#define LF_WTS() \
+  do {           \
+  } while (0)
+#define LF_WTS2(q) \
+  do {             \
+  } while (0)
+#endif
+
 namespace {
 
 constexpr int kThreads = 1024;   // per CTA (one CTA per frame)
@@ -89,8 +135,10 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
   if (tid < 64) (&s_hist[0][0])[tid] = 0;
   if (tid < 2) s_count[tid] = 0;
   if (tid < kMaxLevels) s_roff[tid] = tid < a.g.L ? row_off(a.g, tid) : 0;
+  LF_TS(0);
   pdl_wait();
   pdl_trigger();
+  LF_TS(1);
   const ss_keypoint* fk = a.kps + (int64_t)f * cap;
   const int32_t* cnt = a.counts + f * (L + 1);
   const int i0 = a.pt_off[f], i1 = a.pt_off[f + 1];
@@ -138,6 +186,7 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
     }
   }
   __syncthreads();
+  LF_TS(2);
 
   const ss_camera& c = a.cams[f];
   int dir = 0;  // 1 = forward [o, L-1], 2 = backward [0, o], 0 = [o-1, o+1]
@@ -175,6 +224,7 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
         const float Z = __fadd_rn(dot3r(c.R + 6, P.pos[0], P.pos[1], P.pos[2]), c.t[2]);
         const float u = __fadd_rn(__fdiv_rn(__fmul_rn(c.fx, X), Z), c.cx);
         const float v = __fadd_rn(__fdiv_rn(__fmul_rn(c.fy, Y), Z), c.cy);
+        if (pass == 0 && j == tid) LF_WTS2(0);
         if (!(Z < 0.0f) && !(u < c.min_x || u > c.max_x) && !(v < c.min_y || v > c.max_y)) {
           const float r = __fmul_rn(th, g.scale[o]);
           const int l0 = dir == 1 ? o : (dir == 2 ? 0 : max(o - 1, 0));
@@ -216,6 +266,7 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
           }
         }
       }
+      if (pass == 0 && j == tid) LF_WTS2(1);
       ss_match m;
       m.dist = b1 == ~0ull ? 256 : (int)(b1 >> 32);
       m.dist2 = b2 == ~0ull ? 256 : (int)(b2 >> 32);
@@ -227,7 +278,9 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
       }
       if (m.idx >= 0) atomicMin(fclaim + m.idx, tag | ((unsigned long long)m.dist << 32) | (unsigned)j);
     }
+    if (pass == 0) LF_WTS();
     __syncthreads();
+    if (pass == 0) LF_TS(3);
     // P2: dedup (min (distance, point) per keypoint) + rotation histogram
     for (int i = i0 + tid; i < i1; i += kThreads) {
       const int j = i - i0;
@@ -293,6 +346,7 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
       }
       __syncthreads();
     }
+    if (pass == 0) LF_TS(4);
     kept = s_count[pass];
     if (a.min_matches <= 0 || kept >= a.min_matches) break;  // uniform over the CTA
   }
@@ -303,6 +357,7 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
       const int idx = j < kPtCache ? s_midx[j] : a.out[i].idx;
       if (idx >= 0) fmask[idx] = 1;
     }
+  LF_TS(5);
 }
 
 }  // namespace
