@@ -216,7 +216,7 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
         qa = qd[0];
         qb = qd[1];
       }
-      unsigned long long b1 = ~0ull, b2 = ~0ull;
+      unsigned b1 = ~0u, b2 = ~0u;  // top-2 keys (distance << 16 | keypoint), keypoints < 65536
       const int o = P.octave;
       if (o >= 0 && o < L) {
         const float X = __fadd_rn(dot3r(c.R, P.pos[0], P.pos[1], P.pos[2]), c.t[0]);
@@ -238,14 +238,16 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
             // level's column range (a superset of |x - u| < r); survivors take the exact tests
             const unsigned cr = col_range(g, l, u, r);
             const unsigned lo = cr & 0xFFFFu, span = (cr >> 16) - lo;
-            for (int ch = kb >> 3; ch < (ke + 7) >> 3; ch++) {
-              const int k0 = ch * 8;
-              const uint4 x8 = reinterpret_cast<const uint4*>(s_lx)[ch];
-              unsigned m = ((x8.x & 0xFFFFu) - lo <= span ? 0x01u : 0u) | ((x8.x >> 16) - lo <= span ? 0x02u : 0u) |
-                           ((x8.y & 0xFFFFu) - lo <= span ? 0x04u : 0u) | ((x8.y >> 16) - lo <= span ? 0x08u : 0u) |
-                           ((x8.z & 0xFFFFu) - lo <= span ? 0x10u : 0u) | ((x8.z >> 16) - lo <= span ? 0x20u : 0u) |
-                           ((x8.w & 0xFFFFu) - lo <= span ? 0x40u : 0u) | ((x8.w >> 16) - lo <= span ? 0x80u : 0u);
-              m &= (0xFFu << max(kb - k0, 0)) & (0xFFu >> max(k0 + 8 - ke, 0));
+            // two chunks per step: both lx loads in flight before either's survivors are tested
+            const uint4* lx4 = reinterpret_cast<const uint4*>(s_lx);
+            auto pref = [&](const uint4 x8, int k0) -> unsigned {
+              const unsigned mm = ((x8.x & 0xFFFFu) - lo <= span ? 0x01u : 0u) | ((x8.x >> 16) - lo <= span ? 0x02u : 0u) |
+                                  ((x8.y & 0xFFFFu) - lo <= span ? 0x04u : 0u) | ((x8.y >> 16) - lo <= span ? 0x08u : 0u) |
+                                  ((x8.z & 0xFFFFu) - lo <= span ? 0x10u : 0u) | ((x8.z >> 16) - lo <= span ? 0x20u : 0u) |
+                                  ((x8.w & 0xFFFFu) - lo <= span ? 0x40u : 0u) | ((x8.w >> 16) - lo <= span ? 0x80u : 0u);
+              return mm & (0xFFu << max(kb - k0, 0)) & (0xFFu >> max(k0 + 8 - ke, 0));
+            };
+            auto survivors = [&](unsigned m, int k0) {
               while (m) {
                 const int k = k0 + __ffs(m) - 1;
                 m &= m - 1;
@@ -253,8 +255,7 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
                 const float dx = __fsub_rn(xy.x, u), dy = __fsub_rn(xy.y, v);
                 if (!(fabsf(dx) < r && fabsf(dy) < r)) continue;
                 if (ft && ft[k]) continue;
-                const int d = hamming256(qa, qb, s_desc[2 * k], s_desc[2 * k + 1]);
-                const unsigned long long key = ((unsigned long long)d << 32) | (unsigned)k;
+                const unsigned key = ((unsigned)hamming256(qa, qb, s_desc[2 * k], s_desc[2 * k + 1]) << 16) | (unsigned)k;
                 if (key < b1) {
                   b2 = b1;
                   b1 = key;
@@ -262,15 +263,24 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
                   b2 = key;
                 }
               }
+            };
+            const int ce = (ke + 7) >> 3;
+            for (int ch = kb >> 3; ch < ce; ch += 2) {
+              const bool two = ch + 1 < ce;
+              const uint4 xa = lx4[ch];
+              const uint4 xb = two ? lx4[ch + 1] : make_uint4(0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu);
+              const unsigned ma = pref(xa, ch * 8), mb = two ? pref(xb, ch * 8 + 8) : 0u;
+              survivors(ma, ch * 8);
+              survivors(mb, ch * 8 + 8);
             }
           }
         }
       }
       if (pass == 0 && j == tid) LF_WTS2(1);
       ss_match m;
-      m.dist = b1 == ~0ull ? 256 : (int)(b1 >> 32);
-      m.dist2 = b2 == ~0ull ? 256 : (int)(b2 >> 32);
-      m.idx = (b1 != ~0ull && m.dist <= a.th_high) ? (int)(b1 & 0xFFFFFFFFu) : -1;
+      m.dist = b1 == ~0u ? 256 : (int)(b1 >> 16);
+      m.dist2 = b2 == ~0u ? 256 : (int)(b2 >> 16);
+      m.idx = (b1 != ~0u && m.dist <= a.th_high) ? (int)(b1 & 0xFFFFu) : -1;
       a.out[i] = m;
       if (j < kPtCache) {
         s_midx[j] = m.idx;
