@@ -69,30 +69,37 @@ constexpr int FB_MIN_BLOCKS = SS_FAST_MINB;  // 3: 80 registers
 //   M = max( max_s min9(r)[s] - c,  c - min_s max9(r)[s],  0 ).
 // Returns M + 256 in both lanes (the low byte of each lane is M).
 __device__ __forceinline__ uint32_t arc_score2(const uint32_t (&r)[16], uint32_t c) {
-  uint32_t mn3[16], mx3[16];
+  // the bright side (min over arcs, max over starts) first, then the dark side, so only one
+  // side's 16 three-way partials are live at a time (register pressure: 4 CTAs per SM)
+  uint32_t maxmin, minmax;
+  {
+    uint32_t mn3[16];
 #pragma unroll
-  for (int k = 0; k < 16; k++) {
-    mn3[k] = __vimin3_s16x2(r[k], r[(k + 1) & 15], r[(k + 2) & 15]);
-    mx3[k] = __vimax3_s16x2(r[k], r[(k + 1) & 15], r[(k + 2) & 15]);
-  }
-  uint32_t mn9[16], mx9[16];
+    for (int k = 0; k < 16; k++) mn3[k] = __vimin3_s16x2(r[k], r[(k + 1) & 15], r[(k + 2) & 15]);
+    uint32_t mn9[16];
 #pragma unroll
-  for (int s = 0; s < 16; s++) {
-    mn9[s] = __vimin3_s16x2(mn3[s], mn3[(s + 3) & 15], mn3[(s + 6) & 15]);
-    mx9[s] = __vimax3_s16x2(mx3[s], mx3[(s + 3) & 15], mx3[(s + 6) & 15]);
+    for (int s = 0; s < 16; s++) mn9[s] = __vimin3_s16x2(mn3[s], mn3[(s + 3) & 15], mn3[(s + 6) & 15]);
+    const uint32_t a1 = __vimax3_s16x2(__vimax3_s16x2(mn9[0], mn9[1], mn9[2]), __vimax3_s16x2(mn9[3], mn9[4], mn9[5]),
+                                       __vimax3_s16x2(mn9[6], mn9[7], mn9[8]));
+    const uint32_t a2 = __vimax3_s16x2(__vimax3_s16x2(mn9[9], mn9[10], mn9[11]),
+                                       __vimax3_s16x2(mn9[12], mn9[13], mn9[14]), mn9[15]);
+    maxmin = __vimax3_s16x2(a1, a2, a2) ^ 0x80008000u;  // max_s min9(r), offset-binary
   }
-  const uint32_t a1 = __vimax3_s16x2(__vimax3_s16x2(mn9[0], mn9[1], mn9[2]), __vimax3_s16x2(mn9[3], mn9[4], mn9[5]),
-                                     __vimax3_s16x2(mn9[6], mn9[7], mn9[8]));
-  const uint32_t a2 = __vimax3_s16x2(__vimax3_s16x2(mn9[9], mn9[10], mn9[11]),
-                                     __vimax3_s16x2(mn9[12], mn9[13], mn9[14]), mn9[15]);
-  const uint32_t z1 = __vimin3_s16x2(__vimin3_s16x2(mx9[0], mx9[1], mx9[2]), __vimin3_s16x2(mx9[3], mx9[4], mx9[5]),
-                                     __vimin3_s16x2(mx9[6], mx9[7], mx9[8]));
-  const uint32_t z2 = __vimin3_s16x2(__vimin3_s16x2(mx9[9], mx9[10], mx9[11]),
-                                     __vimin3_s16x2(mx9[12], mx9[13], mx9[14]), mx9[15]);
-  // to offset-binary (s16 + 32768, order preserving) so the differences below are lane-local:
+  {
+    uint32_t mx3[16];
+#pragma unroll
+    for (int k = 0; k < 16; k++) mx3[k] = __vimax3_s16x2(r[k], r[(k + 1) & 15], r[(k + 2) & 15]);
+    uint32_t mx9[16];
+#pragma unroll
+    for (int s = 0; s < 16; s++) mx9[s] = __vimax3_s16x2(mx3[s], mx3[(s + 3) & 15], mx3[(s + 6) & 15]);
+    const uint32_t z1 = __vimin3_s16x2(__vimin3_s16x2(mx9[0], mx9[1], mx9[2]), __vimin3_s16x2(mx9[3], mx9[4], mx9[5]),
+                                       __vimin3_s16x2(mx9[6], mx9[7], mx9[8]));
+    const uint32_t z2 = __vimin3_s16x2(__vimin3_s16x2(mx9[9], mx9[10], mx9[11]),
+                                       __vimin3_s16x2(mx9[12], mx9[13], mx9[14]), mx9[15]);
+    minmax = __vimin3_s16x2(z1, z2, z2) ^ 0x80008000u;  // min_s max9(r), offset-binary
+  }
+  // offset-binary (s16 + 32768, order preserving) makes the differences lane-local:
   // (x + 32768) + 256 - (y + 32768) = x - y + 256 in [1, 511], never borrowing across lanes
-  const uint32_t maxmin = __vimax3_s16x2(a1, a2, a2) ^ 0x80008000u;  // max_s min9(r)
-  const uint32_t minmax = __vimin3_s16x2(z1, z2, z2) ^ 0x80008000u;  // min_s max9(r)
   const uint32_t cb = c ^ 0x80008000u;
   const uint32_t bright = maxmin + 0x01000100u - cb;                 // 256 + max_s min9(r) - c
   const uint32_t dark = cb + 0x01000100u - minmax;                   // 256 + c - min_s max9(r)

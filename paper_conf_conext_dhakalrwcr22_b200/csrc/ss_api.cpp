@@ -575,10 +575,12 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (e == cudaSuccess) e = cudaMemcpy(c->cells, c->cells_h.data(), sizeof(CellInfo) * c->cells_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->bands, c->bands_h.data(), sizeof(BandInfo) * c->bands_h.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) {
-    // the one-launch FAST order: levels >= 1 (segments of up to 8 cells) before level 0's (up
-    // to 4), larger work units first so the last wave is the shorter one
-    std::vector<BandInfo> mo(c->bands_h.begin() + g.band_count[0], c->bands_h.end());
-    mo.insert(mo.end(), c->bands_h.begin(), c->bands_h.begin() + g.band_count[0]);
+    // the one-launch FAST order: larger work units (detect pixels of the segment) first, so
+    // the CTAs that start last are the short ones (longest-processing-time first)
+    std::vector<BandInfo> mo(c->bands_h.begin(), c->bands_h.end());
+    std::stable_sort(mo.begin(), mo.end(), [](const BandInfo& x, const BandInfo& y) {
+      return (int64_t)(x.x1 - x.x0) * (x.y1 - x.y0) > (int64_t)(y.x1 - y.x0) * (y.y1 - y.y0);
+    });
     e = cudaMemcpy(c->bands + c->bands_h.size(), mo.data(), sizeof(BandInfo) * mo.size(), cudaMemcpyHostToDevice);
   }
   c->fast_split = std::getenv("SS_FAST_SPLIT") && std::atoi(std::getenv("SS_FAST_SPLIT")) != 0;
