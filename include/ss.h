@@ -368,7 +368,25 @@ typedef struct {
    * buffers' CONTENTS may change freely between calls.  Ignored while profiling events are
    * installed or when the stream is already capturing. */
   int32_t reuse_graph;
+  /* NULL, or ONE host block (page-locked) that receives every output of the tick in a single
+   * device-to-host copy instead of one copy per output (each copy costs the DMA engine a few
+   * microseconds whatever its size: c2 end to end 75k -> 92k frames/s).  When set, the
+   * separate output pointers above (kps ... lf_n_matches) are ignored and the block holds, in
+   * this order and packed: kps [n_frames][kp_capacity], desc [n_frames][kp_capacity][32],
+   * counts [n_frames][n_levels+1], lf_n_matches [n_frames], lf_matches
+   * [lf_offsets[n_frames]] (0 without O13), matches [n_points] (WINDOW) or
+   * [n_frames][kp_capacity] (BRUTE), uright / depth [n_frames/2][kp_capacity] (stereo only),
+   * each section starting on a 256-byte boundary; ss_tick_packed_layout gives the offsets. */
+  void* out_packed;
 } ss_tick_io;
+
+/* Byte offsets of the sections of ss_tick_io.out_packed for a tick: offsets[0..7] = kps,
+ * desc, counts, lf_n_matches, lf_matches, matches, uright, depth; offsets[8] = total bytes.
+ * n_lf = lf_offsets[n_frames] (0 without O13), brute = 1 for a BRUTE tick (matches per
+ * keypoint slot), stereo = 1 when bf > 0 and baseline > 0.  Host only; SS_EINVAL on NULL or
+ * negative sizes. */
+ss_status ss_tick_packed_layout(const ss_ctx* ctx, int32_t n_frames, int32_t n_points, int64_t n_lf, int32_t brute,
+                                int32_t stereo, int64_t* offsets);
 
 /* One tick of the hot path for a batch of client frames, enqueued on `stream` from a single
  * call: host -> device copies into ctx-owned staging buffers (sized at ss_create: max_frames

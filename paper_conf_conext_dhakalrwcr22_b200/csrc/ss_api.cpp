@@ -184,6 +184,7 @@ struct ss_ctx {
   ss_camera* io_last_cams = nullptr;
   ss_match* io_lf_matches = nullptr;
   int32_t* io_lf_n = nullptr;
+  uint8_t* io_packed = nullptr;  // ss_tick_io.out_packed: every output of a tick, packed (one D2H copy)
   uint8_t* io_lf_mask = nullptr;
   // ss_track_tick graph cache (io->reuse_graph): LRU of instantiated tick graphs by argument key
   struct TickGraph {
@@ -240,7 +241,7 @@ void free_ctx(ss_ctx* c) {
                   c->brute_qexp, c->brute_mexp, c->stereo_sad, c->io_frames, c->io_frames_lin, c->io_kps, c->io_desc, c->io_counts,
                   c->io_cams, c->io_points, c->io_pf, c->io_pdesc, c->io_taken, c->io_queries, c->io_matches,
                   c->io_uright, c->io_depth, c->io_lf_off, c->io_lf_pts, c->io_lf_desc, c->io_last_cams,
-                  c->io_lf_matches, c->io_lf_n, c->io_lf_mask};
+                  c->io_lf_matches, c->io_lf_n, c->io_lf_mask, c->io_packed};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   for (ss_ctx::TickGraph& tg : c->tick_graphs)
@@ -256,6 +257,28 @@ void free_ctx(ss_ctx* c) {
   for (cudaStream_t q : c->side)
     if (q) cudaStreamDestroy(q);
   delete c;
+}
+
+// Byte offsets of a tick's packed outputs (ss_tick_io.out_packed; ss.h documents the order):
+// o[0..7] = kps, desc, counts, lf_n, lf_matches, matches, uright, depth; o[8] = total.
+void packed_layout(const Geom& g, int64_t n_frames, int64_t n_match, int64_t n_lf, bool stereo, int64_t* o) {
+  const int64_t cap = g.kp_capacity;
+  const int64_t ns = stereo ? (n_frames / 2) * cap : 0;
+  const int64_t len[8] = {(int64_t)sizeof(ss_keypoint) * n_frames * cap, n_frames * cap * SS_DESC_BYTES,
+                          4 * n_frames * (g.L + 1), 4 * n_frames, (int64_t)sizeof(ss_match) * n_lf,
+                          (int64_t)sizeof(ss_match) * n_match, 4 * ns, 4 * ns};
+  int64_t b = 0;
+  for (int i = 0; i < 8; i++) {  // every section starts on a 256-byte boundary (vector loads of desc)
+    o[i] = b;
+    b = (b + len[i] + 255) & ~(int64_t)255;
+  }
+  o[8] = o[7] + len[7];
+}
+
+int64_t packed_capacity(const Geom& g, int64_t F, int64_t Qm) {
+  int64_t o[9];
+  packed_layout(g, F, std::max<int64_t>(Qm, F * g.kp_capacity), Qm, true, o);
+  return o[8] + 256;
 }
 
 template <typename T>
@@ -557,6 +580,7 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     ALLOC(c->io_last_cams, sizeof(ss_camera) * F);
     ALLOC(c->io_lf_matches, sizeof(ss_match) * Qm);
     ALLOC(c->io_lf_n, sizeof(int32_t) * F);
+    ALLOC(c->io_packed, packed_capacity(g, F, Qm));
     ALLOC(c->io_lf_mask, (size_t)F * g.kp_capacity);
   }
   if (max_map > 0) {
@@ -966,6 +990,18 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
   const Geom& g = c->g;
   ss_stream_t stream = reinterpret_cast<ss_stream_t>(s);
   const int cap = g.kp_capacity, L = g.L;
+  // outputs: the ctx's buffers, or sections of the packed block (ss_tick_io.out_packed: one D2H)
+  const bool packed = io->out_packed != nullptr;
+  int64_t po[9];
+  packed_layout(g, n_frames, window ? io->n_points : (int64_t)n_frames * cap, lastf ? n_lf : 0, stereo, po);
+  ss_keypoint* o_kps = packed ? reinterpret_cast<ss_keypoint*>(c->io_packed + po[0]) : c->io_kps;
+  uint8_t* o_desc = packed ? c->io_packed + po[1] : c->io_desc;
+  int32_t* o_counts = packed ? reinterpret_cast<int32_t*>(c->io_packed + po[2]) : c->io_counts;
+  int32_t* o_lf_n = packed ? reinterpret_cast<int32_t*>(c->io_packed + po[3]) : c->io_lf_n;
+  ss_match* o_lf_matches = packed ? reinterpret_cast<ss_match*>(c->io_packed + po[4]) : c->io_lf_matches;
+  ss_match* o_matches = packed ? reinterpret_cast<ss_match*>(c->io_packed + po[5]) : c->io_matches;
+  float* o_uright = packed ? reinterpret_cast<float*>(c->io_packed + po[6]) : c->io_uright;
+  float* o_depth = packed ? reinterpret_cast<float*>(c->io_packed + po[7]) : c->io_depth;
   // host -> device.  Frames stored densely (pitch <= the staging pitch, frame_stride = H *
   // pitch) go in ONE linear copy and keep their pitch; anything else is repacked by 2-D
   // copies (a 2-D copy moves row by row, several times slower for 0.3-0.5 MB frames).
@@ -1024,11 +1060,11 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
   // per frame: most SMs are free); the WINDOW match joins it.
   ss_status st;
   const bool fork_project = window && c->prof.empty() && c->tick_fork;
-  st = ss_orb_extract(c, n_frames, c->io_frames, fstride, P, c->io_kps, c->io_desc, c->io_counts, stream);
+  st = ss_orb_extract(c, n_frames, c->io_frames, fstride, P, o_kps, o_desc, o_counts, stream);
   if (st != SS_OK) return st;
   if (stereo) {
-    st = ss_stereo_match(c, n_frames / 2, c->io_frames, fstride, P, c->io_kps, c->io_desc, c->io_counts, io->bf,
-                         io->baseline, c->io_uright, c->io_depth, stream);
+    st = ss_stereo_match(c, n_frames / 2, c->io_frames, fstride, P, o_kps, o_desc, o_counts, io->bf,
+                         io->baseline, o_uright, o_depth, stream);
     if (st != SS_OK) return st;
   }
   if (fork_project) {
@@ -1042,9 +1078,9 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
   int64_t n_matches = 0;
   const uint8_t* win_taken = d_taken;
   if (lastf) {
-    st = ss_match_last_frame(c, n_frames, c->io_cams, io->mb > 0.0f ? d_last : nullptr, io->mb, c->io_kps,
-                             c->io_desc, c->io_counts, win_taken, c->io_lf_off, d_lf_pts, d_lf_desc,
-                             io->lf_th, 100, 1, io->lf_min_matches, c->io_lf_matches, c->io_lf_n, c->io_lf_mask,
+    st = ss_match_last_frame(c, n_frames, c->io_cams, io->mb > 0.0f ? d_last : nullptr, io->mb, o_kps,
+                             o_desc, o_counts, win_taken, c->io_lf_off, d_lf_pts, d_lf_desc,
+                             io->lf_th, 100, 1, io->lf_min_matches, o_lf_matches, o_lf_n, c->io_lf_mask,
                              stream);
     if (st != SS_OK) return st;
     win_taken = c->io_lf_mask;
@@ -1056,17 +1092,21 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
       st = ss_project_points(c, n_frames, c->io_cams, io->n_points, d_points, d_pf, io->th, c->io_queries, stream);
       if (st != SS_OK) return st;
     }
-    st = ss_match_projection(c, n_frames, c->io_kps, c->io_desc, c->io_counts, win_taken, io->n_points, c->io_queries,
-                             d_pdesc, 0, cfg, c->io_matches, stream);
+    st = ss_match_projection(c, n_frames, o_kps, o_desc, o_counts, win_taken, io->n_points, c->io_queries,
+                             d_pdesc, 0, cfg, o_matches, stream);
     if (st != SS_OK) return st;
     n_matches = io->n_points;
   } else if (cfg->mode == SS_MATCH_BRUTE) {
-    st = ss_match_projection(c, n_frames, c->io_kps, c->io_desc, c->io_counts, nullptr, 0, nullptr, io->d_map_desc,
-                             io->n_map, cfg, c->io_matches, stream);
+    st = ss_match_projection(c, n_frames, o_kps, o_desc, o_counts, nullptr, 0, nullptr, io->d_map_desc,
+                             io->n_map, cfg, o_matches, stream);
     if (st != SS_OK) return st;
     n_matches = (int64_t)n_frames * cap;
   }
   // device -> host
+  if (packed) {  // every output in ONE copy
+    SS_CUDA_TRY(cudaMemcpyAsync(io->out_packed, c->io_packed, (size_t)po[8], cudaMemcpyDeviceToHost, s));
+    return SS_OK;
+  }
   if (io->kps)
     SS_CUDA_TRY(cudaMemcpyAsync(io->kps, c->io_kps, sizeof(ss_keypoint) * n_frames * cap, cudaMemcpyDeviceToHost, s));
   if (io->desc)
@@ -1104,11 +1144,20 @@ std::vector<unsigned char> tick_key(int32_t n_frames, const ss_match_cfg* cfg, c
   ptr(io->kps); ptr(io->desc); ptr(io->counts); ptr(io->matches); ptr(io->uright); ptr(io->depth);
   ptr(io->lf_offsets); ptr(io->lf_points); ptr(io->lf_desc); ptr(io->last_cams); put(&io->mb, 4); put(&io->lf_th, 4);
   put(&io->lf_min_matches, 4); ptr(io->lf_matches); ptr(io->lf_n_matches); put(&io->map_resident, 4);
+  ptr(io->out_packed);
   put(&n_lf, 8);
   return k;
 }
 
 }  // namespace
+
+ss_status ss_tick_packed_layout(const ss_ctx* c, int32_t n_frames, int32_t n_points, int64_t n_lf, int32_t brute,
+                                int32_t stereo, int64_t* offsets) {
+  if (!c || !offsets) return fail(SS_EINVAL, "NULL ctx/offsets");
+  if (n_frames < 0 || n_points < 0 || n_lf < 0) return fail(SS_EINVAL, "negative size");
+  packed_layout(c->g, n_frames, brute ? (int64_t)n_frames * c->g.kp_capacity : n_points, n_lf, stereo != 0, offsets);
+  return SS_OK;
+}
 
 ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, const ss_tick_io* io,
                         ss_stream_t stream) {

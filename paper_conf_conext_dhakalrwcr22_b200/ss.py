@@ -65,7 +65,7 @@ class ss_tick_io(C.Structure):
                 ("lf_offsets", C.c_void_p), ("lf_points", C.c_void_p), ("lf_desc", C.c_void_p),
                 ("last_cams", C.c_void_p), ("mb", C.c_float), ("lf_th", C.c_float), ("lf_min_matches", C.c_int32),
                 ("lf_matches", C.c_void_p), ("lf_n_matches", C.c_void_p), ("map_resident", C.c_int32),
-                ("reuse_graph", C.c_int32)]
+                ("reuse_graph", C.c_int32), ("out_packed", C.c_void_p)]
 
 
 # numpy views of the 20-/20-/12-byte records of ss.h
@@ -115,6 +115,7 @@ def lib():
                                    C.POINTER(ss_tick_io), i32, i32]
         L.ss_set_distribution.argtypes = [P, i32]
         L.ss_track_tick.argtypes = [P, i32, C.POINTER(ss_match_cfg), C.POINTER(ss_tick_io), P]
+        L.ss_tick_packed_layout.argtypes = [P, i32, i32, i64, i32, i32, P]
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
         L.ss_debug_candidates.argtypes = [P, i32, i32, P, P, P, i32, C.POINTER(i32)]
         L.ss_debug_overflow_count.argtypes = [P, C.POINTER(i32)]
@@ -139,7 +140,7 @@ EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "s
             "ss_match_last_frame", "ss_match_brute_partial", "ss_match_brute_merge", "ss_profile_events", "ss_profile_next", "ss_debug_level",
             "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times", "ss_debug_distribution_paths",
             "ss_debug_match_lanes", "ss_debug_capture_samples", "ss_brute_map_prepare", "ss_orb_extract_frames",
-            "ss_track_run")
+            "ss_track_run", "ss_tick_packed_layout")
 
 
 def _check(status: int, ctx=None):
@@ -202,6 +203,14 @@ def ss_match_projection(ctx, n_frames, d_kps, d_desc, d_counts, d_kp_taken, n_qu
 
 def ss_set_distribution(ctx, mode: int) -> None:
     _check(lib().ss_set_distribution(ctx, mode), ctx)
+
+
+def ss_tick_packed_layout(ctx, n_frames, n_points, n_lf, brute=False, stereo=False) -> np.ndarray:
+    """Byte offsets of ss_tick_io.out_packed's sections (kps, desc, counts, lf_n_matches,
+    lf_matches, matches, uright, depth) and the total (index 8)."""
+    out = np.zeros(9, np.int64)
+    _check(lib().ss_tick_packed_layout(ctx, n_frames, n_points, n_lf, int(brute), int(stereo), out.ctypes.data), ctx)
+    return out
 
 
 def ss_track_tick(ctx, n_frames, cfg: ss_match_cfg, io: ss_tick_io, stream=None):

@@ -117,11 +117,12 @@ def test_track_tick_brute(torch_cuda, ref):
     pipe.close()
 
 
-@pytest.mark.parametrize("resident", [0, 1])
-def test_track_tick_lastframe_window(torch_cuda, ref, resident):
+@pytest.mark.parametrize("resident,packed", [(0, 0), (1, 0), (1, 1)])
+def test_track_tick_lastframe_window(torch_cuda, ref, resident, packed):
     """Mono tick with frame-to-frame matching (O13) before search local points: the window
     match skips keypoints that are taken or kept by O13.  Oracle chain: extract -> O13 ->
-    taken | kept -> O11 -> O9."""
+    taken | kept -> O11 -> O9.  packed: every output through ss_tick_io.out_packed (one D2H
+    copy; ss_tick_packed_layout's sections), direct and replayed from the cached graph."""
     torch = torch_cuda
     from paper_conf_conext_dhakalrwcr22_b200 import ss
     from paper_conf_conext_dhakalrwcr22_b200.pipeline import OrbPipeline
@@ -153,8 +154,23 @@ def test_track_tick_lastframe_window(torch_cuda, ref, resident):
     for k in o:
         setattr(io, k, o[k].data_ptr())
     pipe = OrbPipeline(w, h, nf, 8, max_frames=B, max_queries=B * Qm)
-    ss.ss_track_tick(pipe.ctx, B, ss.window_cfg(), io)
-    torch.cuda.synchronize()
+    if packed:
+        lay = ss.ss_tick_packed_layout(pipe.ctx, B, B * Qm, int(off[-1]))
+        assert (lay[:8] % 256 == 0).all()
+        blk = torch.full((int(lay[8]),), 0xAB, dtype=torch.uint8).pin_memory()
+        io.out_packed = blk.data_ptr()
+        io.reuse_graph = 1
+        st = torch.cuda.Stream()
+        for _ in range(3):  # direct, capture, replay: the block is rewritten every time
+            blk.fill_(0xAB)
+            ss.ss_track_tick(pipe.ctx, B, ss.window_cfg(), io, st)
+            torch.cuda.synchronize()
+        names = ["kps", "desc", "counts", "lf_n_matches", "lf_matches", "matches"]
+        for j, k in enumerate(names):
+            o[k] = blk[int(lay[j]):int(lay[j]) + o[k].numel()]
+    else:
+        ss.ss_track_tick(pipe.ctx, B, ss.window_cfg(), io)
+        torch.cuda.synchronize()
     kps = o["kps"].numpy().reshape(B, cap, 20)
     desc = o["desc"].numpy().reshape(B, cap, 32)
     counts = o["counts"].numpy().view(np.int32).reshape(B, 9)
