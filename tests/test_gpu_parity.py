@@ -309,3 +309,26 @@ def test_search_local_points_chain(torch_cuda, ref, shape, th):
     np.testing.assert_array_equal(got, want)
     assert (got["idx"] >= 0).sum() > 200
     pipe.close()
+
+
+@pytest.mark.parametrize("env", [{"SS_FAST_SPLIT": "1"}, {"SS_SEG0": "4", "SS_SEG": "4"},
+                                 {"SS_SEG0": "2", "SS_SEG": "3"}, {"SS_SEG0": "24", "SS_SEG": "24"}],
+                         ids=["split-launch", "seg4", "seg2-3", "seg24"])
+def test_extract_launch_layouts(torch_cuda, ref, env, monkeypatch):
+    """The FAST launch layouts the A/B switches select (level 0 beside the pyramid; 2..24-cell
+    segments, i.e. other cell-start columns for the NMS's neighbour masks and other band
+    widths) give the same bit-exact extraction on EuRoC and KITTI frames."""
+    torch = torch_cuda
+    for k, v in env.items():  # read by ss_create
+        monkeypatch.setenv(k, v)
+    for (w, h), nf in ((synth.SHAPES["euroc"], 1000), (synth.SHAPES["kitti"], 2000)):
+        B = 2
+        frames = synth.make_frames(w, h, B, cfg=17, client0=3)
+        pipe = _pipe(torch, w, h, nf, 8, max_frames=B)
+        pipe.extract(_upload(torch, frames))
+        gk, gd, gc = pipe.results(B)
+        p = ref.params(w, h, nf)
+        for b in range(B):
+            rk, rd, rc = ref.orb_extract(p, frames[b])
+            assert_extract_equal(gk[b], gd[b], gc[b], rk, rd, rc, f"{env} {w}x{h} frame {b}")
+        pipe.close()
