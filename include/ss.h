@@ -378,7 +378,18 @@ typedef struct {
    * [n_frames][kp_capacity] (BRUTE), uright / depth [n_frames/2][kp_capacity] (stereo only),
    * each section starting on a 256-byte boundary; ss_tick_packed_layout gives the offsets. */
   void* out_packed;
+  /* NULL, or ONE host block (page-locked) holding the tick's per-tick host inputs, copied in a
+   * single host-to-device copy: frames [n_frames][frame_stride] (dense: frame_stride = height
+   * * pitch, pitch a multiple of 16 and <= the width rounded up to 16), cams [n_frames], and
+   * lf_offsets [n_frames+1] (read only with O13), each section on a 256-byte boundary
+   * (ss_tick_packed_in_layout).  When set, frames, cams and lf_offsets above are ignored; the
+   * other inputs (the map state, last_cams) are unchanged. */
+  const void* in_packed;
 } ss_tick_io;
+
+/* Byte offsets of ss_tick_io.in_packed's sections for n_frames frames of frame_stride bytes:
+ * offsets[0..2] = frames, cams, lf_offsets; offsets[3] = total bytes.  Host only. */
+ss_status ss_tick_packed_in_layout(const ss_ctx* ctx, int32_t n_frames, int64_t frame_stride, int64_t* offsets);
 
 /* Byte offsets of the sections of ss_tick_io.out_packed for a tick: offsets[0..7] = kps,
  * desc, counts, lf_n_matches, lf_matches, matches, uright, depth; offsets[8] = total bytes.

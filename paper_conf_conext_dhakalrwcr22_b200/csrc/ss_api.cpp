@@ -185,6 +185,7 @@ struct ss_ctx {
   ss_match* io_lf_matches = nullptr;
   int32_t* io_lf_n = nullptr;
   uint8_t* io_packed = nullptr;  // ss_tick_io.out_packed: every output of a tick, packed (one D2H copy)
+  uint8_t* io_inpacked = nullptr;  // ss_tick_io.in_packed: frames + cams + lf_offsets (one H2D copy)
   uint8_t* io_lf_mask = nullptr;
   // ss_track_tick graph cache (io->reuse_graph): LRU of instantiated tick graphs by argument key
   struct TickGraph {
@@ -241,7 +242,7 @@ void free_ctx(ss_ctx* c) {
                   c->brute_qexp, c->brute_mexp, c->stereo_sad, c->io_frames, c->io_frames_lin, c->io_kps, c->io_desc, c->io_counts,
                   c->io_cams, c->io_points, c->io_pf, c->io_pdesc, c->io_taken, c->io_queries, c->io_matches,
                   c->io_uright, c->io_depth, c->io_lf_off, c->io_lf_pts, c->io_lf_desc, c->io_last_cams,
-                  c->io_lf_matches, c->io_lf_n, c->io_lf_mask, c->io_packed};
+                  c->io_lf_matches, c->io_lf_n, c->io_lf_mask, c->io_packed, c->io_inpacked};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   for (ss_ctx::TickGraph& tg : c->tick_graphs)
@@ -273,6 +274,18 @@ void packed_layout(const Geom& g, int64_t n_frames, int64_t n_match, int64_t n_l
     b = (b + len[i] + 255) & ~(int64_t)255;
   }
   o[8] = o[7] + len[7];
+}
+
+// Byte offsets of a tick's packed host inputs (ss_tick_io.in_packed): frames, cams,
+// lf_offsets (each on a 256-byte boundary); o[3] = total.
+void packed_in_layout(int64_t n_frames, int64_t frame_stride, int64_t* o) {
+  const int64_t len[3] = {n_frames * frame_stride, (int64_t)sizeof(ss_camera) * n_frames, 4 * (n_frames + 1)};
+  int64_t b = 0;
+  for (int i = 0; i < 3; i++) {
+    o[i] = b;
+    b = (b + len[i] + 255) & ~(int64_t)255;
+  }
+  o[3] = o[2] + len[2];
 }
 
 int64_t packed_capacity(const Geom& g, int64_t F, int64_t Qm) {
@@ -581,6 +594,11 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
     ALLOC(c->io_lf_matches, sizeof(ss_match) * Qm);
     ALLOC(c->io_lf_n, sizeof(int32_t) * F);
     ALLOC(c->io_packed, packed_capacity(g, F, Qm));
+    {
+      int64_t o[4];
+      packed_in_layout(F, (int64_t)g.H * c->io_pitch, o);
+      ALLOC(c->io_inpacked, o[3] + 256);
+    }
     ALLOC(c->io_lf_mask, (size_t)F * g.kp_capacity);
   }
   if (max_map > 0) {
@@ -1008,7 +1026,21 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
   int P = c->io_pitch;
   int64_t fstride = (int64_t)g.H * P;
   const bool dense = io->pitch <= c->io_pitch && (n_frames == 1 || io->frame_stride == (int64_t)io->pitch * g.H);
-  if (dense && io->pitch % 16 == 0) {
+  // device copies of the per-tick host inputs: the ctx's buffers, or sections of the packed
+  // input block (ss_tick_io.in_packed: frames + cams + lf_offsets in ONE copy)
+  uint8_t* d_frames_in = c->io_frames;
+  ss_camera* d_cams_in = c->io_cams;
+  int32_t* d_lfoff_in = c->io_lf_off;
+  if (io->in_packed) {
+    int64_t o[4];
+    packed_in_layout(n_frames, io->frame_stride, o);
+    P = io->pitch;
+    fstride = io->frame_stride;
+    SS_CUDA_TRY(cudaMemcpyAsync(c->io_inpacked, io->in_packed, (size_t)o[3], cudaMemcpyHostToDevice, s));
+    d_frames_in = c->io_inpacked + o[0];
+    d_cams_in = reinterpret_cast<ss_camera*>(c->io_inpacked + o[1]);
+    d_lfoff_in = reinterpret_cast<int32_t*>(c->io_inpacked + o[2]);
+  } else if (dense && io->pitch % 16 == 0) {
     P = io->pitch;
     fstride = (int64_t)g.H * P;
     SS_CUDA_TRY(cudaMemcpyAsync(c->io_frames, io->frames, (size_t)fstride * n_frames, cudaMemcpyHostToDevice, s));
@@ -1036,7 +1068,8 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
   const ss_camera* d_last = res ? io->last_cams : c->io_last_cams;
   if (window) {
     const int64_t n = io->n_points;
-    SS_CUDA_TRY(cudaMemcpyAsync(c->io_cams, io->cams, sizeof(ss_camera) * n_frames, cudaMemcpyHostToDevice, s));
+    if (!io->in_packed)
+      SS_CUDA_TRY(cudaMemcpyAsync(c->io_cams, io->cams, sizeof(ss_camera) * n_frames, cudaMemcpyHostToDevice, s));
     if (!res) {
       SS_CUDA_TRY(cudaMemcpyAsync(c->io_points, io->points, sizeof(ss_map_point) * n, cudaMemcpyHostToDevice, s));
       SS_CUDA_TRY(cudaMemcpyAsync(c->io_pf, io->point_frame, sizeof(int32_t) * n, cudaMemcpyHostToDevice, s));
@@ -1046,7 +1079,8 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
     }
   }
   if (lastf) {
-    SS_CUDA_TRY(cudaMemcpyAsync(c->io_lf_off, io->lf_offsets, sizeof(int32_t) * (n_frames + 1), cudaMemcpyHostToDevice, s));
+    if (!io->in_packed)
+      SS_CUDA_TRY(cudaMemcpyAsync(c->io_lf_off, io->lf_offsets, sizeof(int32_t) * (n_frames + 1), cudaMemcpyHostToDevice, s));
     if (n_lf > 0 && !res) {
       SS_CUDA_TRY(cudaMemcpyAsync(c->io_lf_pts, io->lf_points, sizeof(ss_frame_point) * n_lf, cudaMemcpyHostToDevice, s));
       SS_CUDA_TRY(cudaMemcpyAsync(c->io_lf_desc, io->lf_desc, (size_t)n_lf * SS_DESC_BYTES, cudaMemcpyHostToDevice, s));
@@ -1060,17 +1094,17 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
   // per frame: most SMs are free); the WINDOW match joins it.
   ss_status st;
   const bool fork_project = window && c->prof.empty() && c->tick_fork;
-  st = ss_orb_extract(c, n_frames, c->io_frames, fstride, P, o_kps, o_desc, o_counts, stream);
+  st = ss_orb_extract(c, n_frames, d_frames_in, fstride, P, o_kps, o_desc, o_counts, stream);
   if (st != SS_OK) return st;
   if (stereo) {
-    st = ss_stereo_match(c, n_frames / 2, c->io_frames, fstride, P, o_kps, o_desc, o_counts, io->bf,
+    st = ss_stereo_match(c, n_frames / 2, d_frames_in, fstride, P, o_kps, o_desc, o_counts, io->bf,
                          io->baseline, o_uright, o_depth, stream);
     if (st != SS_OK) return st;
   }
   if (fork_project) {
     SS_CUDA_TRY(cudaEventRecord(c->ev_aux0, s));
     SS_CUDA_TRY(cudaStreamWaitEvent(c->aux, c->ev_aux0, 0));
-    st = ss_project_points(c, n_frames, c->io_cams, io->n_points, d_points, d_pf, io->th, c->io_queries,
+    st = ss_project_points(c, n_frames, d_cams_in, io->n_points, d_points, d_pf, io->th, c->io_queries,
                            reinterpret_cast<ss_stream_t>(c->aux));
     if (st != SS_OK) return st;
     SS_CUDA_TRY(cudaEventRecord(c->ev_aux1, c->aux));
@@ -1078,8 +1112,8 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
   int64_t n_matches = 0;
   const uint8_t* win_taken = d_taken;
   if (lastf) {
-    st = ss_match_last_frame(c, n_frames, c->io_cams, io->mb > 0.0f ? d_last : nullptr, io->mb, o_kps,
-                             o_desc, o_counts, win_taken, c->io_lf_off, d_lf_pts, d_lf_desc,
+    st = ss_match_last_frame(c, n_frames, d_cams_in, io->mb > 0.0f ? d_last : nullptr, io->mb, o_kps,
+                             o_desc, o_counts, win_taken, d_lfoff_in, d_lf_pts, d_lf_desc,
                              io->lf_th, 100, 1, io->lf_min_matches, o_lf_matches, o_lf_n, c->io_lf_mask,
                              stream);
     if (st != SS_OK) return st;
@@ -1089,7 +1123,7 @@ ss_status tick_enqueue(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, con
     if (fork_project) {
       SS_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_aux1, 0));
     } else {
-      st = ss_project_points(c, n_frames, c->io_cams, io->n_points, d_points, d_pf, io->th, c->io_queries, stream);
+      st = ss_project_points(c, n_frames, d_cams_in, io->n_points, d_points, d_pf, io->th, c->io_queries, stream);
       if (st != SS_OK) return st;
     }
     st = ss_match_projection(c, n_frames, o_kps, o_desc, o_counts, win_taken, io->n_points, c->io_queries,
@@ -1144,7 +1178,7 @@ std::vector<unsigned char> tick_key(int32_t n_frames, const ss_match_cfg* cfg, c
   ptr(io->kps); ptr(io->desc); ptr(io->counts); ptr(io->matches); ptr(io->uright); ptr(io->depth);
   ptr(io->lf_offsets); ptr(io->lf_points); ptr(io->lf_desc); ptr(io->last_cams); put(&io->mb, 4); put(&io->lf_th, 4);
   put(&io->lf_min_matches, 4); ptr(io->lf_matches); ptr(io->lf_n_matches); put(&io->map_resident, 4);
-  ptr(io->out_packed);
+  ptr(io->out_packed); ptr(io->in_packed);
   put(&n_lf, 8);
   return k;
 }
@@ -1159,14 +1193,36 @@ ss_status ss_tick_packed_layout(const ss_ctx* c, int32_t n_frames, int32_t n_poi
   return SS_OK;
 }
 
+ss_status ss_tick_packed_in_layout(const ss_ctx* c, int32_t n_frames, int64_t frame_stride, int64_t* offsets) {
+  if (!c || !offsets) return fail(SS_EINVAL, "NULL ctx/offsets");
+  if (n_frames < 0 || frame_stride < 0) return fail(SS_EINVAL, "negative size");
+  packed_in_layout(n_frames, frame_stride, offsets);
+  return SS_OK;
+}
+
 ss_status ss_track_tick(ss_ctx* c, int32_t n_frames, const ss_match_cfg* cfg, const ss_tick_io* io,
                         ss_stream_t stream) {
   if (!c || !cfg || !io) return fail(SS_EINVAL, "NULL ctx/cfg/io");
   if (n_frames < 0 || io->n_points < 0 || io->n_map < 0) return fail(SS_EINVAL, "negative size");
   if (n_frames > c->max_frames) return fail(SS_ECAPACITY, "n_frames exceeds the ctx's max_frames");
   if (n_frames == 0) return SS_OK;
-  if (!io->frames) return fail(SS_EINVAL, "NULL frames");
   const Geom& g = c->g;
+  // packed host inputs: frames, cams and lf_offsets are sections of io->in_packed (one H2D
+  // copy, tick_enqueue); O13 then runs when lf_points is set
+  ss_tick_io eff = *io;
+  if (io->in_packed) {
+    if (io->pitch % 16 != 0 || io->pitch > c->io_pitch || io->pitch < g.W || io->frame_stride != (int64_t)io->pitch * g.H)
+      return fail(SS_EINVAL, "in_packed needs dense frames (frame_stride = height * pitch, pitch a multiple of 16, "
+                             "<= width rounded up to 16)");
+    int64_t o[4];
+    packed_in_layout(n_frames, io->frame_stride, o);
+    const uint8_t* b = static_cast<const uint8_t*>(io->in_packed);
+    eff.frames = b + o[0];
+    eff.cams = reinterpret_cast<const ss_camera*>(b + o[1]);
+    eff.lf_offsets = io->lf_points ? reinterpret_cast<const int32_t*>(b + o[2]) : nullptr;
+  }
+  io = &eff;
+  if (!io->frames) return fail(SS_EINVAL, "NULL frames");
   if (io->pitch < g.W || (n_frames > 1 && io->frame_stride < (int64_t)io->pitch * g.H))
     return fail(SS_EINVAL, "bad pitch / frame stride");
   const bool stereo = io->bf > 0.0f;

@@ -65,7 +65,7 @@ class ss_tick_io(C.Structure):
                 ("lf_offsets", C.c_void_p), ("lf_points", C.c_void_p), ("lf_desc", C.c_void_p),
                 ("last_cams", C.c_void_p), ("mb", C.c_float), ("lf_th", C.c_float), ("lf_min_matches", C.c_int32),
                 ("lf_matches", C.c_void_p), ("lf_n_matches", C.c_void_p), ("map_resident", C.c_int32),
-                ("reuse_graph", C.c_int32), ("out_packed", C.c_void_p)]
+                ("reuse_graph", C.c_int32), ("out_packed", C.c_void_p), ("in_packed", C.c_void_p)]
 
 
 # numpy views of the 20-/20-/12-byte records of ss.h
@@ -116,6 +116,7 @@ def lib():
         L.ss_set_distribution.argtypes = [P, i32]
         L.ss_track_tick.argtypes = [P, i32, C.POINTER(ss_match_cfg), C.POINTER(ss_tick_io), P]
         L.ss_tick_packed_layout.argtypes = [P, i32, i32, i64, i32, i32, P]
+        L.ss_tick_packed_in_layout.argtypes = [P, i32, i64, P]
         L.ss_debug_level.argtypes = [P, i32, i32, C.POINTER(P), C.POINTER(i32)]
         L.ss_debug_candidates.argtypes = [P, i32, i32, P, P, P, i32, C.POINTER(i32)]
         L.ss_debug_overflow_count.argtypes = [P, C.POINTER(i32)]
@@ -140,7 +141,7 @@ EXPORTED = ("ss_orb_params_init", "ss_create", "ss_destroy", "ss_last_error", "s
             "ss_match_last_frame", "ss_match_brute_partial", "ss_match_brute_merge", "ss_profile_events", "ss_profile_next", "ss_debug_level",
             "ss_debug_candidates", "ss_debug_overflow_count", "ss_debug_phase_times", "ss_debug_distribution_paths",
             "ss_debug_match_lanes", "ss_debug_capture_samples", "ss_brute_map_prepare", "ss_orb_extract_frames",
-            "ss_track_run", "ss_tick_packed_layout")
+            "ss_track_run", "ss_tick_packed_layout", "ss_tick_packed_in_layout")
 
 
 def _check(status: int, ctx=None):
@@ -210,6 +211,13 @@ def ss_tick_packed_layout(ctx, n_frames, n_points, n_lf, brute=False, stereo=Fal
     lf_matches, matches, uright, depth) and the total (index 8)."""
     out = np.zeros(9, np.int64)
     _check(lib().ss_tick_packed_layout(ctx, n_frames, n_points, n_lf, int(brute), int(stereo), out.ctypes.data), ctx)
+    return out
+
+
+def ss_tick_packed_in_layout(ctx, n_frames, frame_stride) -> np.ndarray:
+    """Byte offsets of ss_tick_io.in_packed's sections (frames, cams, lf_offsets) and the total."""
+    out = np.zeros(4, np.int64)
+    _check(lib().ss_tick_packed_in_layout(ctx, n_frames, frame_stride, out.ctypes.data), ctx)
     return out
 
 

@@ -122,7 +122,8 @@ def test_track_tick_lastframe_window(torch_cuda, ref, resident, packed):
     """Mono tick with frame-to-frame matching (O13) before search local points: the window
     match skips keypoints that are taken or kept by O13.  Oracle chain: extract -> O13 ->
     taken | kept -> O11 -> O9.  packed: every output through ss_tick_io.out_packed (one D2H
-    copy; ss_tick_packed_layout's sections), direct and replayed from the cached graph."""
+    copy; ss_tick_packed_layout's sections) and the frames, cameras and last-frame offsets
+    through ss_tick_io.in_packed (one H2D copy), direct and replayed from the cached graph."""
     torch = torch_cuda
     from paper_conf_conext_dhakalrwcr22_b200 import ss
     from paper_conf_conext_dhakalrwcr22_b200.pipeline import OrbPipeline
@@ -159,6 +160,13 @@ def test_track_tick_lastframe_window(torch_cuda, ref, resident, packed):
         assert (lay[:8] % 256 == 0).all()
         blk = torch.full((int(lay[8]),), 0xAB, dtype=torch.uint8).pin_memory()
         io.out_packed = blk.data_ptr()
+        # inputs too: frames + cams + lf_offsets in one block; the separate pointers are ignored
+        ilay = ss.ss_tick_packed_in_layout(pipe.ctx, B, h * w)
+        iblk = torch.zeros(int(ilay[3]), dtype=torch.uint8).pin_memory()
+        for j, t_ in enumerate((hf, hc, hoff)):
+            iblk[int(ilay[j]):int(ilay[j]) + t_.numel()].copy_(t_)
+        io.in_packed = iblk.data_ptr()
+        io.frames, io.cams, io.lf_offsets = None, None, None
         io.reuse_graph = 1
         st = torch.cuda.Stream()
         for _ in range(3):  # direct, capture, replay: the block is rewritten every time
