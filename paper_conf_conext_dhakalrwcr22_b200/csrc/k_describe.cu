@@ -441,7 +441,10 @@ extern "C" int ss_dbg_desc_ts(unsigned long long* out) { return (int)cudaMemcpyF
 const int* brief_pattern_host() { return SS_BRIEF_PATTERN_HOST; }
 
 cudaError_t describe_init() {  // ss_create, per device (never under stream capture)
-  cudaError_t e = cudaFuncSetAttribute(describe_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  cudaError_t e = carveout_from_env(describe_kernel<false>);
+  if (e == cudaSuccess) e = carveout_from_env(describe_kernel<true>);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(describe_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)(DESC_WARPS * PER_WARP + 128));
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(describe_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,

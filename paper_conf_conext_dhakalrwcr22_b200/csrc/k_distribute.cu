@@ -839,6 +839,8 @@ cudaError_t launch_distribute_tables(const Geom& g, uint32_t* qtab, cudaStream_t
 }
 
 cudaError_t distribute_init() {  // ss_create, per device
+  cudaError_t e = carveout_from_env(distribute_kernel);
+  if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(distribute_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemTotal);
 }
 

@@ -438,6 +438,8 @@ extern "C" int ss_dbg_fast_ts(unsigned long long* out) {  // [2][4096][8]
 #endif
 
 cudaError_t fast_init() {  // ss_create, per device; ss_create rejects bands above 227 KB
+  cudaError_t e = carveout_from_env(fast_bands_kernel);
+  if (e != cudaSuccess) return e;
   return set_max_dynamic_smem(fast_bands_kernel);
 }
 

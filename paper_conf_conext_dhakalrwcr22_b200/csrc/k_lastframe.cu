@@ -373,6 +373,8 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
 }  // namespace
 
 cudaError_t lastframe_init() {  // at ss_create (never inside a stream capture)
+  cudaError_t e = carveout_from_env(lastframe_kernel);
+  if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(lastframe_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kLfSmemMax);
 }
 

@@ -300,6 +300,8 @@ bool pyramid_plan(const Geom& g, const uint32_t* tab, const int64_t* xoff, const
 }
 
 cudaError_t pyramid_init() {  // ss_create, per device; pyramid_plan keeps every plan within kPyrSmemMax
+  cudaError_t e = carveout_from_env(pyramid_fused_kernel);
+  if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(pyramid_fused_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kPyrSmemMax);
 }
 

@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <cstdlib>
 #include <vector>
 
 #include "../../include/ss.h"
@@ -139,6 +140,15 @@ inline cudaError_t set_max_dynamic_smem(K kernel) {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, kernel);
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, optin - (int)fa.sharedSizeBytes);
+}
+// Shared-memory carveout (percent of the unified L1/shared array) from SS_CARVEOUT, for the
+// A/B of one fixed carveout across the extraction kernels (no reconfiguration between them);
+// unset = the driver's choice.
+template <typename K>
+inline cudaError_t carveout_from_env(K kernel) {
+  const char* e = std::getenv("SS_CARVEOUT");
+  if (!e) return cudaSuccess;
+  return cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout, std::atoi(e));
 }
 #endif
 
