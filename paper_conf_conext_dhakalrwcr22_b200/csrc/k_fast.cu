@@ -276,11 +276,15 @@ __global__ void __launch_bounds__(FB_THREADS, FB_MIN_BLOCKS) fast_bands_kernel(c
                                                                 uint32_t* __restrict__ slots,
                                                                 int32_t* __restrict__ cell_counts, int rp, int mbw,
                                                                 int region_bytes, int bits_off) {
-  pdl_wait();
-  pdl_trigger();
   extern __shared__ __align__(16) uint8_t smem[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const BandInfo bd = bands[blockIdx.x];
+  const BandInfo bd = bands[blockIdx.x];  // static (ss_create): readable before the dependency wait
+  // Level 0 reads only the caller's frames, which are complete before the pyramid (the kernel
+  // this one depends on) passed its own dependency wait -- and this grid launches only after
+  // the pyramid's trigger -- so level-0 CTAs run beside the pyramid; the other levels wait for
+  // it (as level 0's separate launch on a side branch did in round 1, without the extra launch).
+  if (bd.level != 0) pdl_wait();
+  pdl_trigger();
   const int f = blockIdx.y;
   FAST_TS(0);
   const int l = bd.level;
