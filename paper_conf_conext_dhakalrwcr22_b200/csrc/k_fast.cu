@@ -2,9 +2,10 @@
 // iniThFAST -> minThFAST fallback (DESIGN.md §3 O2, O3; "parallelization of
 // FAST corner detection ... with the GPU").
 //
-// One CTA per *segment* = up to 8 consecutive 30-px FAST cells of one cell row of one level
-// of one frame (the cells of a row share their detect rows and their detect windows tile
-// [x0, x1) without gaps):
+// ONE launch for every level of every frame (levels >= 1 wait for the pyramid; level 0 reads
+// only the caller's frames and runs beside it), one CTA per *segment* = up to 8 consecutive
+// 30-px FAST cells of one cell row of one level of one frame (the cells of a row share their
+// detect rows and their detect windows tile [x0, x1) without gaps), largest segments first:
 //  1. stage the band + ring halo in shared memory with 16-byte coalesced loads;
 //  2. the score M of EVERY band pixel, four horizontally adjacent pixels per thread: the band
 //     is staged as I - 128 (bytes XOR 0x80); each ring value PAIR of pixels (0, 2) or (1, 3)
@@ -13,11 +14,13 @@
 //     the 16 arcs of 9 of the RAW ring values runs on DPX three-way min/max (VIMNMX3.S16x2);
 //     the centre enters only at the end (min_k (c - r_k) = c - max_k r_k) -- no pre-test, no
 //     divergence, one 32-bit store of 4 scores;
-//  3. one warp per cell, one lane per cell row: strict 8-neighbour maxima inside the cell's
-//     window (neighbours in the next cell are ignored: per-cell ROI semantics), four columns
-//     per step as 16x2 three-way max trees over cell-masked neighbour words, as 64-bit row
-//     masks; the cell's threshold (iniTh if any maximum beats it, else minTh), and the
-//     survivors written in raster order (warp prefix sum of the row counts).
+//  3. strict 8-neighbour maxima above minTh / iniTh, every thread on 4-pixel groups (the score
+//     tasks' layout): each row's horizontal 3-max and left/right max per 16x2 half, with
+//     neighbours in another cell masked to 0 by a cell-start column bitmap (per-cell ROI
+//     semantics), into two shared-memory bit planes;
+//  4. one warp per cell, one lane per cell row: the row's 64-bit masks from the bit planes, the
+//     cell's threshold (iniTh if any maximum beats it, else minTh), and the survivors written
+//     in raster order (warp prefix sum of the row counts).
 //
 //   M(p) = max_s max( min_{k<9} d_{s+k}, min_{k<9} -d_{s+k} ),  d_k = I(p) - I(p + R_k)
 //        = max( I(p) - min_s max_{k<9} I(p + R_{s+k}),  max_s min_{k<9} I(p + R_{s+k}) - I(p) )
