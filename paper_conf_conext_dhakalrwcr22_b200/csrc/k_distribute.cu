@@ -1,12 +1,18 @@
 // k_distribute.cu -- S4: per-(frame, level) quadtree keypoint distribution
-// (ORB-SLAM DistributeOctTree reading, DESIGN.md §3 O4), one 1024-thread CTA per
-// (level, frame), round-synchronous reformulation:
+// (ORB-SLAM DistributeOctTree reading, DESIGN.md §3 O4), ONE launch for all levels, one
+// 1024-thread CTA per (level, frame), round-synchronous reformulation:
 //
 //  * Each candidate's quadtree path is a function of its position only: the root is
 //    trunc(f32 kx / hX) and at every round the child is chosen against the node's ceil
-//    half-split.  We precompute 13 rounds of 2-bit quadrant codes per key
-//    (key = root << 26 | path) and radix-sort the keys once (stable, CUB, in shared
-//    memory).  Every depth-r node is then a contiguous run of keys sharing an r-prefix.
+//    half-split; the x decisions depend on kx alone and the y decisions on ky alone, so the
+//    13-round key (key = root << 26 | path of 2-bit quadrant codes) is X[kx] | Y[ky] from two
+//    per-level tables built once by make_key (distribute_tables_kernel, at ss_create).
+//  * Dense fast path (dense_body, the usual case): the depth-r node of a key is the dense
+//    index key >> (26 - 2r), so per-depth node counts are shared-memory histograms -- S_r and
+//    E_r below without any sort; the kept keys are ordered by row buckets.
+//  * Sort fallback (a stop rule needs a depth beyond the dense table, or > 8192 candidates):
+//    the keys radix-sorted once (stable, CUB, in shared memory); every depth-r node is then a
+//    contiguous run of keys sharing an r-prefix, and:
 //  * dd_i = the round at which sorted neighbours i-1, i separate.  Histograms of dd and of
 //    max(dd_i, dd_i+1) give, for every depth r at once, S_r = #nodes and E_r = #nodes
 //    with > 1 key -- exactly the quantities ORB-SLAM's phase-1/phase-2 stop rules test
