@@ -151,7 +151,6 @@ __global__ void __launch_bounds__(PT, SS_PYR_MINB) pyramid_fused_kernel(const __
     // last group can pass its right edge
     const int x = nx0 + 4 * cx;
     const bool own_x = x >= B.x && x < B.y;
-    const int dw = g.w[l];
     uint8_t* const d = src.pyr + (int64_t)f * g.pyr_frame_bytes + g.lvl_off[l] + x;
     const int gp = g.pitch[l];
     const uint32_t* const yc = s_y + (D.y >> 16);
@@ -161,14 +160,11 @@ __global__ void __launch_bounds__(PT, SS_PYR_MINB) pyramid_fused_kernel(const __
       const uint32_t packed = lerp4(sa + y0 * spitch, sa + y1 * spitch, sh, sel, W, (cy >> 16) & 0x1FF);
       *reinterpret_cast<uint32_t*>(da + r * dpitch) = packed;
       const int y = ny0 + r;
-      if (own_x && y >= B.z && y < B.w) {
-        uint8_t* drow = d + (int64_t)y * gp;
-        if (x + 4 <= dw) {
-          *reinterpret_cast<uint32_t*>(drow) = packed;  // x and the pitch are multiples of 4
-        } else {
-          for (int q = 0; x + q < dw; q++) drow[q] = (uint8_t)(packed >> (8 * q));
-        }
-      }
+      if (own_x && y >= B.z && y < B.w)  // x and the pitch are multiples of 4 and x < w <= pitch:
+        // the level's last group may write up to 3 bytes of the row's pitch padding, which no
+        // reader uses (FAST and stereo stay inside the level; describe's TMA boxes are bounded
+        // by the level width)
+        *reinterpret_cast<uint32_t*>(d + (int64_t)y * gp) = packed;
     }
   }
 }
