@@ -372,10 +372,11 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
   const int64_t o = (int64_t)f * g.kp_capacity + i;
   uint8_t* smp = SAMPLES ? samples + o * 512 + 16 * lane : nullptr;
   uint32_t byte = 0;
-  bool near = false;
+  uint32_t near = 0;  // bit t: pair t had an estimate within 1e-4 of a half-integer
 #pragma unroll
   for (int t = 0; t < 8; t++) {
     int v[2];
+    bool nr = false;
 #pragma unroll
     for (int e = 0; e < 2; e++) {
       const float2 pp = s_pat[(2 * t + e) * 32 + lane];  // exact small integers
@@ -384,29 +385,32 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
       const float bx = __fadd_rn(tx, 12582912.0f), by = __fadd_rn(ty, 12582912.0f);
       const float dx = __fsub_rn(tx, __fsub_rn(bx, 12582912.0f)), dy = __fsub_rn(ty, __fsub_rn(by, 12582912.0f));
       // |d| <= 1/2 always (t minus its nearest integer): a near-tie is |d| >= 1/2 - 1e-4
-      near |= (fabsf(dx) >= 0.4999f) | (fabsf(dy) >= 0.4999f);
+      nr |= (fabsf(dx) >= 0.4999f) | (fabsf(dy) >= 0.4999f);
       v[e] = blurred(__float_as_int(bx) - 0x4B400000, __float_as_int(by) - 0x4B400000);
       if (SAMPLES) smp[2 * t + e] = (uint8_t)v[e];
     }
     byte |= (uint32_t)(v[0] < v[1]) << t;
+    near |= (uint32_t)nr << t;
   }
-  if (__any_sync(0xFFFFFFFFu, near)) {  // rare: redo the byte with the exact tie test
-    byte = 0;
-    for (int t = 0; t < 8; t++) {
-      int v[2];
-      for (int e = 0; e < 2; e++) {
-        const uint32_t wd = __ldg(reinterpret_cast<const uint32_t*>(pattern) + 8 * lane + t);
-        const int px = (int)(wd << (24 - 16 * e)) >> 24, py = (int)(wd << (16 - 16 * e)) >> 24;
-        int ox = px, oy = py;
-        if (r2) {
-          ox = rhe_rot(px, -py, cs, sn, m10, m01, r2);
-          oy = rhe_rot(px, py, sn, cs, m01, m10, r2);
-        }
-        v[e] = blurred(ox, oy);
-        if (SAMPLES) smp[2 * t + e] = (uint8_t)v[e];
+  // rare: only the pairs with a near-tie estimate are redone with the exact tie test (round
+  // 1 redid all 16 samples of every lane of the warp: those warps were the launch's slowest)
+  while (near) {
+    const int t = __ffs(near) - 1;
+    near &= near - 1;
+    int v[2];
+#pragma unroll
+    for (int e = 0; e < 2; e++) {
+      const float2 pp = s_pat[(2 * t + e) * 32 + lane];
+      const int px = (int)pp.x, py = (int)pp.y;
+      int ox = px, oy = py;
+      if (r2) {
+        ox = rhe_rot(px, -py, cs, sn, m10, m01, r2);
+        oy = rhe_rot(px, py, sn, cs, m01, m10, r2);
       }
-      byte |= (uint32_t)(v[0] < v[1]) << t;
+      v[e] = blurred(ox, oy);
+      if (SAMPLES) smp[2 * t + e] = (uint8_t)v[e];
     }
+    byte = (byte & ~(1u << t)) | ((uint32_t)(v[0] < v[1]) << t);
   }
   desc[o * SS_DESC_BYTES + lane] = (uint8_t)byte;
   DESC_TS(5);
