@@ -31,8 +31,8 @@ buf = np.zeros((2, 4096, 8), np.uint64)
 assert ss.lib().ss_dbg_fast_ts(buf.ctypes.data_as(ctypes.c_void_p)) == 0
 for li, name in enumerate(["level 0", "levels >= 1"]):
     t = buf[li].astype(np.int64)
-    n = int((t[:, 0] > 0).sum())
-    t = t[:n]
+    t = t[t[:, 0] > 0]  # the launch's CTAs of this group (indices follow the launch's band order)
+    n = len(t)
     t0 = t[:, 0].min()
     ph = np.diff(t[:, 0:5], axis=1)
     print(f"{name}: {n} CTAs, span {(t[:, 4].max() - t0) / 1000:.2f} us, last start {(t[:, 0].max() - t0) / 1000:.2f} us, "
