@@ -46,7 +46,10 @@ __device__ unsigned long long g_desc_ts[16384][8];
 
 namespace {
 
-constexpr int DESC_WARPS = 8;
+#ifndef SS_DESC_WARPS
+#define SS_DESC_WARPS 4  // 4 vs 6 vs 8: c2 describe 18.9 / 19.6 / 19.8 us (scripts/ab_descwarps.sh)
+#endif
+constexpr int DESC_WARPS = SS_DESC_WARPS;  // warps (keypoints in flight) per CTA
 constexpr int PR = 43;  // raw patch: radius 21 (18 max sample offset + 3 blur taps)
 constexpr int PP = 64;  // raw patch pitch: a 16-B aligned 64-B window covers the 43 B row
 constexpr int BR = 37;  // blurred patch: radius 18
@@ -120,7 +123,7 @@ __device__ __forceinline__ void tma_patch(const CUtensorMap* map, uint8_t* dst, 
 // SAMPLES (test hook, ss_debug_capture_samples): also write the blurred value of every sample
 // point the comparisons read, samples[slot][b][e] for bit b = 8 * lane + t, point e
 template <bool SAMPLES>
-__global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, FrameSrc src,
+__global__ void __launch_bounds__(DESC_WARPS * 32, 32 / DESC_WARPS) describe_kernel(Geom g, FrameSrc src,
                                                                    const uint32_t* __restrict__ selected,
                                                                    const int32_t* __restrict__ sel_counts,
                                                                    const int8_t* __restrict__ pattern,
@@ -150,14 +153,14 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 4) describe_kernel(Geom g, Fr
     const int ln = i & 31, j = i >> 5, pt = 16 * ln + j;
     s_pat[i] = make_float2((float)__ldg(pattern + 2 * pt), (float)__ldg(pattern + 2 * pt + 1));
   }
-  if (threadIdx.x < 256) {  // byte j = u + 15 of row |v|: inside the disk -> (1, u + 15), else 0
-    const int t = threadIdx.x >> 7, av = (threadIdx.x >> 3) & 15, k = threadIdx.x & 7;
+  for (int it = threadIdx.x; it < 256; it += DESC_WARPS * 32) {  // byte j = u + 15 of row |v|: inside the disk -> (1, u + 15), else 0
+    const int t = it >> 7, av = (it >> 3) & 15, k = it & 7;
     uint32_t word = 0;
     for (int b = 0; b < 4; b++) {
       const int j = 4 * k + b, u = j - 15;
       if (j <= 30 && u >= -c_umax[av] && u <= c_umax[av]) word |= (uint32_t)(t ? j : 1) << (8 * b);
     }
-    (t ? s_wu : s_wmask)[(threadIdx.x & 127)] = word;
+    (t ? s_wu : s_wmask)[(it & 127)] = word;
   }
   pdl_wait();
   DESC_TS(1);
