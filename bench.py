@@ -979,12 +979,18 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
     packed_out = [torch.empty(int(lay[8]), dtype=torch.uint8).pin_memory() for _ in range(P)]
     # ... and the per-tick host inputs (frames, cameras, last-frame offsets) in ONE pinned block
     # per input slot (ss_tick_io.in_packed: one H2D copy per tick instead of three)
-    ilay = ss.ss_tick_packed_in_layout(pipes[0].ctx, B, H * W)
+    # (frames whose width is not a multiple of 16 B, e.g. KITTI's 1241, sit in the block with
+    # the row pitch rounded up to 16: the host's receive buffer layout, so the library needs no
+    # unaligned copy or on-device repack)
+    WP = (W + 15) // 16 * 16
+    ilay = ss.ss_tick_packed_in_layout(pipes[0].ctx, B, H * WP)
     inblk = []
     for i in range(n_host):
         blk_ = torch.zeros(int(ilay[3]), dtype=torch.uint8).pin_memory()
-        parts = [fr[i]] + ([hin[i][0], hin[i][6]] if window else [])
-        for j, t_ in enumerate(parts):
+        fview = blk_[:B * H * WP].view(B, H, WP)
+        fview[:, :, :W].copy_(fr[i].view(B, H, W))
+        parts = [hin[i][0], hin[i][6]] if window else []
+        for j, t_ in enumerate(parts, start=1):
             blk_[int(ilay[j]):int(ilay[j]) + t_.numel()].copy_(t_)
         inblk.append(blk_)
 
@@ -1020,8 +1026,8 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
                     io.uright, io.depth = o["uright"].data_ptr(), o["depth"].data_ptr()
                 if packed:
                     io.out_packed = packed_out[q].data_ptr()
-                    if W % 16 == 0:  # dense frames with a 16-B pitch: the packed input block applies
-                        io.in_packed = inblk[i].data_ptr()
+                    io.in_packed = inblk[i].data_ptr()
+                    io.frame_stride, io.pitch = H * WP, WP
                 row.append(io)
             ios.append(row)
         # bytes actually copied per tick (hin: cams, points, point_frame, qdesc, taken, last_cams,
@@ -1032,7 +1038,7 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
             h2d = fr[0].numel() + hin[0][0].numel() + hin[0][6].numel()
         else:
             h2d = fr[0].numel() + sum(a.numel() for j, a in enumerate(hin[0]) if j != 5 or lf[0] > 0)
-        if packed and W % 16 == 0:  # the packed block replaces frames + cams + offsets (256-B aligned sections)
+        if packed:  # the packed block replaces frames + cams + offsets (256-B aligned sections, 16-B row pitch)
             h2d += int(ilay[3]) - (fr[0].numel() + ((hin[0][0].numel() + hin[0][6].numel()) if window else 0))
 
         # the tick loop runs natively (ss_track_run: tick t = ss_track_tick on ctx t % P with
@@ -1056,8 +1062,8 @@ def run_e2e(args, pipes, frames_h, q_host, map_desc, outs, B, Q, window, dev, st
         return {"value": B * world * K / (ms / 1000.0), "unit": "frames/s", "h2d_bytes_per_step": int(h2d),
                 "d2h_bytes_per_step": int(lay[8] if packed else d2h_sep), "steps": K, "ms_per_step": ms / K,
                 "ticks_in_flight": P, "host_us_per_call": 1e6 * (h1 - h0) / K,
-                "io": ("packed: one H2D (ss_tick_io.in_packed) + one D2H (out_packed) per tick" if packed and W % 16 == 0
-                       else "packed outputs (one D2H per tick)" if packed else "one copy per input / output")}
+                "io": ("packed: one H2D (ss_tick_io.in_packed, frame rows at a 16-B pitch) + one D2H (out_packed) per tick"
+                       if packed else "one copy per input / output")}
 
     path = ("ss_track_run: one ss_track_tick per tick in native code: H2D, ss_orb_extract, " +
             ("ss_stereo_match, " if stereo else "") +
