@@ -676,13 +676,13 @@ def run_ours(args, cfg):
                 ev.record(streams[q])
                 gather_step(ev, q)
 
-    run_steps(0, W_)
-    torch.cuda.synchronize(dev)
-    if world > 1:
-        dist.barrier()
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     sampler = ClockSampler(local)
-    with sampler:
+    with sampler:  # started before the warm-up, so its start-up (a subprocess) leaves no idle gap before t0
+        run_steps(0, W_)
+        torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier()
         torch.cuda.synchronize(dev)
         t0.record(streams[0])
         for q in range(1, P):
