@@ -890,18 +890,9 @@ def run_ours(args, cfg):
         "metric": METRIC, "value": value, "unit": "frames/s", "n_gpus": world, "steps": K, "warmup": W_,
         "ms_per_step": T_max / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "u8", "data": "synthetic",
-        "config": {"workload": cfg["desc"], "config": args.config, "frames_per_step": frames_per_step,
-                   "images_per_step_per_gpu": B, "features_per_image": cfg["nf"],
-                   "map_points_per_step_per_gpu": Q if window else 0, "map_size": cfg["map"],
-                   "parallelism": f"dp{world} (clients sharded over GPUs)" +
-                                  (f"; result gather over {backend}" if world > 1 else "") +
-                                  ("; all ranks on one GPU (--same-device)" if args.same_device and world > 1 else ""),
-                   "l2": f"inputs ring of {n_slots} distinct slots = {n_slots * slot_bytes / 2**20:.0f} MiB "
-                         f"> L2 {l2 / 2**20:.0f} MiB (no flush)",
-                   "cuda_graphs": True, "ticks_in_flight": P, "setup_s": round(setup_s, 1),
-                   "distribution": "grid top-N (O4g)" if args.dist == "grid" else "quadtree (O4)",
-                   "map": ("sharded over ranks (F4: shard top-2 for all ranks' frames, all-to-all, merge)"
-                           if shard else ("replicated" if not window else None))},
+        "config": workload_config(args, cfg, world),
+        "run": {"cuda_graphs": True, "ticks_in_flight": P, "setup_s": round(setup_s, 1),
+                "input_ring": {"slots": n_slots, "MiB": round(n_slots * slot_bytes / 2**20), "l2_MiB": round(l2 / 2**20)}},
         "steady_state": steady,
         "latency_ms": {"p50": float(np.percentile(step_ms, 50)), "p99": float(np.percentile(step_ms, 99)),
                        "samples": len(step_ms),
@@ -1204,6 +1195,28 @@ def _cpu_model():
     return "unknown"
 
 
+def workload_config(args, cfg, world):
+    """The JSON line's `config`: the workload alone, identical on both arms (`--impl ours` and
+    `--impl reference`), so the driver's ratio compares the same workload.  How an arm runs it
+    (graphs, ticks in flight, the input ring's size, the oracle's sample) is in `run` /
+    `cpu_baseline`."""
+    window = cfg["mode"] == "window"
+    per_client = 2 if cfg.get("stereo") else 1
+    n_clients = cfg["clients"]  # per GPU (weak scaling)
+    B = n_clients * per_client
+    return {"workload": cfg["desc"], "config": args.config, "frames_per_step": B * world,
+            "images_per_step_per_gpu": B, "features_per_image": cfg["nf"],
+            "map_points_per_step_per_gpu": cfg["queries"] * n_clients if window else 0, "map_size": cfg["map"],
+            "parallelism": f"dp{world} (clients sharded over GPUs)" +
+                           (f"; result gather over {args.backend}" if world > 1 else "") +
+                           ("; all ranks on one GPU (--same-device)" if args.same_device and world > 1 else ""),
+            "l2": "no flush: the timed steps cycle through an input ring larger than the L2 "
+                  "(sizes in run.input_ring)",
+            "distribution": "grid top-N (O4g)" if args.dist == "grid" else "quadtree (O4)",
+            "map": ("sharded over ranks (F4: shard top-2 for all ranks' frames, all-to-all, merge)"
+                    if getattr(args, "map_shard", False) and not window else ("replicated" if not window else None))}
+
+
 def run_reference(args, cfg):
     """The CPU oracle as the reference arm: each step = one bounded sample of the workload."""
     rank = int(os.environ.get("RANK", 0))
@@ -1253,8 +1266,7 @@ def run_reference(args, cfg):
     res = {"impl": "reference", "metric": METRIC, "value": value, "unit": "frames/s", "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * T / len(times),
            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-           "config": {"workload": cfg["desc"], "config": args.config, "frames_per_step": n_frames,
-                      "parallelism": "CPU oracle, one single-threaded process per core"},
+           "config": workload_config(args, cfg, world),
            "cpu_baseline": {"value": value, "unit": "frames/s", "cores": min(cores, n_frames), "kind": "oracle",
                             "sample": f"{n_frames} of the tick's {B} frames per step (extract + " +
                                       (f"{cfg.get('lf', 0)} last-frame points matched + {cfg['queries']}-point "
@@ -1295,6 +1307,8 @@ def main(argv=None):
     args = ap.parse_args(argv)
     assert args.warmup >= 3, "at least 3 warm-up steps"
     cfg = CONFIGS[args.config]
+    if args.clients:
+        cfg = dict(cfg, clients=args.clients)
     if args.impl == "reference":
         run_reference(args, cfg)
     else:
