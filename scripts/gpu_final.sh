@@ -14,7 +14,7 @@ if [ "${SKIP_TESTS:-0}" != "1" ]; then
   timeout 300 python __graft_entry__.py smoke > $OUT/smoke_$TAG.txt 2>&1; echo "smoke rc=$?"; tail -1 $OUT/smoke_$TAG.txt
 fi
 timeout 900 python bench.py > $OUT/bench_$TAG.json 2> $OUT/bench_$TAG.err; echo "bench c2 rc=$?"
-timeout 900 python bench.py --steps 20 --warmup 3 --no-cpu-baseline > $OUT/bench_${TAG}_k20.json 2> /dev/null; echo "bench c2 K=20 rc=$?"
+timeout 900 python bench.py --steps 20 --warmup 5 --no-cpu-baseline > $OUT/bench_${TAG}_k20.json 2> /dev/null; echo "bench c2 K=20 rc=$?"
 for C in c1 c3 c4 c5; do
   PYTHONFAULTHANDLER=1 timeout -s ABRT 600 python bench.py --config $C --no-cpu-baseline > $OUT/bench_${TAG}_$C.json 2> $OUT/bench_${TAG}_$C.err
   echo "bench $C rc=$?"
