@@ -132,7 +132,9 @@ __global__ void __launch_bounds__(DESC_WARPS * 32, 32 / DESC_WARPS) describe_ker
                                                                    int32_t* __restrict__ counts,
                                                                    uint8_t* __restrict__ samples,
                                                                    const __grid_constant__ PatchMaps maps) {
+#ifndef SS_DESC_LATE_TRIGGER
   pdl_trigger();
+#endif
   DESC_TS(0);
   extern __shared__ __align__(128) uint8_t sm_raw[];  // DESC_WARPS * PER_WARP + 128
   // 128-B aligned warp buffers (TMA destinations)

@@ -65,6 +65,17 @@ __device__ __forceinline__ uint64_t gtimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
+// Where the CTA lets the dependent grid (describe) launch: at phase SS_DIST_TRIGGER of the
+// dense path (0 = right after the dependency wait; -1 = only at exit).  Describe's ~1000 CTAs
+// become resident as soon as every distribution CTA has triggered and then wait, holding their
+// shared memory, for the whole distribution -- SM space other ticks in flight could use.
+#ifndef SS_DIST_TRIGGER
+#define SS_DIST_TRIGGER 8
+#endif
+#define DIST_TRIGGER_AT(k)                  \
+  do {                                      \
+    if (SS_DIST_TRIGGER == (k)) pdl_trigger(); \
+  } while (0)
 // phase timestamps of one (frame, level) CTA (debug hook ss_debug_phase_times), thread 0 only
 #define SS_PHASE(i)                                  \
   do {                                               \
@@ -611,6 +622,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, uint32_t* cand, u
   }
   __syncthreads();
   SS_PHASE(6);
+  DIST_TRIGGER_AT(6);
   // best key of every final node: max score, ties -> lowest rank
   for (int i = tid; i < n; i += DT) {
     const uint32_t k = key[i];
@@ -621,6 +633,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, uint32_t* cand, u
   }
   __syncthreads();
   SS_PHASE(7);
+  DIST_TRIGGER_AT(7);
   // kept keys (in no particular order) + their level rows' counts
   uint32_t* kept = key;  // keys are no longer needed
   {
@@ -648,6 +661,7 @@ __device__ bool dense_body(const Geom& g, int l, int f, int n, uint32_t* cand, u
   const int nk = S_.sh[2];
   const int nk_w = min(nk, g.cap[l]);
   SS_PHASE(8);
+  DIST_TRIGGER_AT(8);
   // canonical (ly, lx) order: row starts by a block scan of the row counts, keys scattered
   // into their row's bucket, then ranked by lx among the (few) keys of the same row
   {
@@ -737,7 +751,7 @@ __global__ void __launch_bounds__(DT, 1)
   }
   SS_PHASE(11);  // static set-up issued
   pdl_wait();
-  pdl_trigger();
+  DIST_TRIGGER_AT(0);
   SS_PHASE(0);
 
   // ---- 1. candidate counts per cell, their offsets (rank order = cells row-major, then

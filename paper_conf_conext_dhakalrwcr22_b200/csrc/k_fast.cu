@@ -287,7 +287,9 @@ __global__ void __launch_bounds__(FB_THREADS, FB_MIN_BLOCKS) fast_bands_kernel(c
   // the pyramid's trigger -- so level-0 CTAs run beside the pyramid; the other levels wait for
   // it (as level 0's separate launch on a side branch did in round 1, without the extra launch).
   if (bd.level != 0) pdl_wait();
+#ifndef SS_FAST_LATE_TRIGGER
   pdl_trigger();
+#endif
   const int f = blockIdx.y;
   FAST_TS(0);
   const int l = bd.level;

@@ -66,6 +66,12 @@ __device__ __forceinline__ uint32_t lerp4(const uint8_t* r0, const uint8_t* r1, 
   return __byte_perm(__byte_perm(a[0], a[1], 0x0062), __byte_perm(a[2], a[3], 0x0062), 0x5410);
 }
 
+// the level whose start lets the dependent grid (FAST) launch: <= 1 = the kernel's start (FAST's
+// level-0 CTAs run beside the pyramid; its other CTAs sit resident until the pyramid ends),
+// k = once levels < k are built, > L - 1 = only at exit
+#ifndef SS_PYR_TRIGGER
+#define SS_PYR_TRIGGER 3
+#endif
 #ifndef SS_PYR_MINB
 #define SS_PYR_MINB 1
 #endif
@@ -75,7 +81,7 @@ __global__ void __launch_bounds__(PT, SS_PYR_MINB) pyramid_fused_kernel(const __
                                                               const PyrLvl* __restrict__ plan, int buf0_bytes,
                                                               int buf1_bytes) {
   pdl_wait();
-  pdl_trigger();
+  if (SS_PYR_TRIGGER <= 1) pdl_trigger();
   extern __shared__ __align__(16) uint8_t smem[];
   // [buffer 0 | pad | buffer 1 | pad | plan | group coefficients | row coefficients]; level l
   // lives in buffer l & 1; the pads absorb the source windows' over-read past a buffer's
@@ -131,6 +137,7 @@ __global__ void __launch_bounds__(PT, SS_PYR_MINB) pyramid_fused_kernel(const __
   const uint32_t* const s_y = reinterpret_cast<const uint32_t*>(s_g) + P[0].soff;
   for (int l = 1; l < L; l++) {
     __syncthreads();  // staged / the previous level's buffer complete
+    if (l == SS_PYR_TRIGGER && l > 1) pdl_trigger();
     const int4 A = s_plan[4 * l], B = s_plan[4 * l + 1], C = s_plan[4 * l + 2], D = s_plan[4 * l + 3];
     const int nx0 = A.x, ngx = A.y, ny0 = A.z, rows = A.w;
     const int ry = (int)(((uint32_t)tid * (uint32_t)(D.x & 0x1FFFFF)) >> 20);  // tid / ngx (host-verified)
