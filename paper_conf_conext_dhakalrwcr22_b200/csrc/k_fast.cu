@@ -57,6 +57,12 @@ namespace {
 constexpr int FB_WARPS = SS_FAST_WARPS;
 constexpr int FB_THREADS = FB_WARPS * 32;
 constexpr int ROWS_PER_TASK = SS_FAST_ROWS;  // rows per score task (sliding 7-row window)
+// when the dependent grid (the distribution: 32 CTAs of 215 KB shared memory at c2, resident from
+// then until this grid ends) may launch: 0 = the CTA's start, 2 = after its scores, 3 = after
+// its NMS, -1 = at exit (measured: exit -3.5 % at c2)
+#ifndef SS_FAST_TRIGGER
+#define SS_FAST_TRIGGER 0
+#endif
 #ifndef SS_FAST_MINB
 #define SS_FAST_MINB (24 / FB_WARPS > 1 ? 24 / FB_WARPS : 1)
 #endif
@@ -278,19 +284,20 @@ __global__ void __launch_bounds__(FB_THREADS, FB_MIN_BLOCKS) fast_bands_kernel(c
                                                                 const CellInfo* __restrict__ cells,
                                                                 uint32_t* __restrict__ slots,
                                                                 int32_t* __restrict__ cell_counts, int rp, int mbw,
-                                                                int region_bytes, int bits_off) {
+                                                                int region_bytes, int bits_off, int flat_frames) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const BandInfo bd = bands[blockIdx.x];  // static (ss_create): readable before the dependency wait
+  // 2-D grid (band, frame), or flat band-major (flat_frames = F: CTA i = band i / F, frame i % F,
+  // so the band order -- longest first -- holds across frames too)
+  const int bi = flat_frames ? (int)blockIdx.x / flat_frames : (int)blockIdx.x;
+  const BandInfo bd = bands[bi];  // static (ss_create): readable before the dependency wait
   // Level 0 reads only the caller's frames, which are complete before the pyramid (the kernel
   // this one depends on) passed its own dependency wait -- and this grid launches only after
   // the pyramid's trigger -- so level-0 CTAs run beside the pyramid; the other levels wait for
   // it (as level 0's separate launch on a side branch did in round 1, without the extra launch).
   if (bd.level != 0) pdl_wait();
-#ifndef SS_FAST_LATE_TRIGGER
-  pdl_trigger();
-#endif
-  const int f = blockIdx.y;
+  if (SS_FAST_TRIGGER == 0) pdl_trigger();
+  const int f = flat_frames ? (int)blockIdx.x % flat_frames : (int)blockIdx.y;
   FAST_TS(0);
   const int l = bd.level;
   const int tmin = g.min_th, tini = g.ini_th;
@@ -356,6 +363,7 @@ __global__ void __launch_bounds__(FB_THREADS, FB_MIN_BLOCKS) fast_bands_kernel(c
   }
   __syncthreads();
   FAST_TS(2);
+  if (SS_FAST_TRIGGER == 2) pdl_trigger();
   // ---- 3. strict 8-neighbour maxima above minTh / iniTh, every thread on 4-pixel groups of
   // ROWS_PER_TASK rows (the score tasks' layout), into the bit planes: per 16x2 half (pixels
   // 0, 2 or 1, 3) the horizontal 3-max hf and left/right max hlr of each row are formed once
@@ -370,6 +378,7 @@ __global__ void __launch_bounds__(FB_THREADS, FB_MIN_BLOCKS) fast_bands_kernel(c
   }
   __syncthreads();
   FAST_TS(3);
+  if (SS_FAST_TRIGGER == 3) pdl_trigger();
   // ---- 4. per cell (warp), per row (lane): the cell's threshold (iniTh if any maximum beats
   // it, else minTh) and the survivors in raster order (warp prefix sum of the row counts) ----
   for (int j = warp; j < bd.ncells; j += FB_WARPS) {
@@ -453,13 +462,14 @@ cudaError_t fast_init() {  // ss_create, per device; ss_create rejects bands abo
 }
 
 cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands, int n_bands,
-                              const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s) {
+                              const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s,
+                              bool flat) {
   if (n_bands <= 0) return cudaSuccess;
   int rp, mbw, rb, mb, nb;
   const size_t smem = fast_smem_bytes(g, &rp, &mbw, &rb, &mb, &nb);
-  dim3 grid(n_bands, n_frames);
+  const dim3 grid = flat ? dim3(n_bands * n_frames) : dim3(n_bands, n_frames);
   cudaError_t e = launch_pdl(fast_bands_kernel, grid, dim3(FB_THREADS), smem, s, g, src, bands, cells, slots,
-                             cell_counts, rp, mbw, rb, nb);
+                             cell_counts, rp, mbw, rb, nb, flat ? n_frames : 0);
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 

@@ -77,6 +77,11 @@ extern "C" int ss_dbg_lf_ts(unsigned long long* out) {
 
 namespace {
 
+// when the dependent grid (the window matcher) may launch: 0 = after the dependency wait, 1 = after
+// the first pass's search (P1), -1 = at exit; its CTAs sit resident from then until this ends
+#ifndef SS_LF_TRIGGER
+#define SS_LF_TRIGGER 0
+#endif
 constexpr int kThreads = 1024;   // per CTA (one CTA per frame)
 constexpr int kPtCache = 2048;   // points per frame whose P1 results stay in shared memory
 constexpr int kHisto = 30;       // ORB-SLAM HISTO_LENGTH
@@ -137,7 +142,7 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
   if (tid < kMaxLevels) s_roff[tid] = tid < a.g.L ? row_off(a.g, tid) : 0;
   LF_TS(0);
   pdl_wait();
-  pdl_trigger();
+  if (SS_LF_TRIGGER == 0) pdl_trigger();
   LF_TS(1);
   const ss_keypoint* fk = a.kps + (int64_t)f * cap;
   const int32_t* cnt = a.counts + f * (L + 1);
@@ -290,6 +295,7 @@ __global__ void __launch_bounds__(kThreads) lastframe_kernel(const LfArgs a) {
     }
     if (pass == 0) LF_WTS();
     __syncthreads();
+    if (pass == 0 && SS_LF_TRIGGER == 1) pdl_trigger();
     if (pass == 0) LF_TS(3);
     // P2: dedup (min (distance, point) per keypoint) + rotation histogram
     for (int i = i0 + tid; i < i1; i += kThreads) {

@@ -158,6 +158,7 @@ struct ss_ctx {
   PatchMaps maps{};                  // TMA maps of the describe kernel (levels >= 1 at ss_create)
   // test hooks: lanes per WINDOW query (0 = chosen per launch), blurred-sample capture buffer
   int win_lanes = 0;
+  int fast_flat = 0;         // SS_FAST_FLAT (A/B): flat band-major FAST grid, 2 = level 0 first
   bool fast_split = false;  // SS_FAST_SPLIT=1: level 0's FAST on a side branch beside the pyramid (A/B)
   bool tick_fork = true;  // ss_track_tick: local-map projection on the aux branch (SS_TICK_FORK=0: serial)
   uint8_t* dbg_samples = nullptr;
@@ -619,8 +620,14 @@ ss_status ss_create(int32_t device, const ss_orb_params* p, int32_t max_frames, 
   if (e == cudaSuccess) {
     // the one-launch FAST order: larger work units (detect pixels of the segment) first, so
     // the CTAs that start last are the short ones (longest-processing-time first)
+    // SS_FAST_FLAT (A/B): 1 = a flat band-major grid (the order holds across frames), 2 = that
+    // with level 0's bands first (they need not wait for the pyramid)
+    const char* ff = std::getenv("SS_FAST_FLAT");
+    c->fast_flat = ff ? std::atoi(ff) : 0;
+    const bool l0first = c->fast_flat == 2;
     std::vector<BandInfo> mo(c->bands_h.begin(), c->bands_h.end());
-    std::stable_sort(mo.begin(), mo.end(), [](const BandInfo& x, const BandInfo& y) {
+    std::stable_sort(mo.begin(), mo.end(), [l0first](const BandInfo& x, const BandInfo& y) {
+      if (l0first && (x.level == 0) != (y.level == 0)) return x.level == 0;
       return (int64_t)(x.x1 - x.x0) * (x.y1 - x.y0) > (int64_t)(y.x1 - y.x0) * (y.y1 - y.y0);
     });
     e = cudaMemcpy(c->bands + c->bands_h.size(), mo.data(), sizeof(BandInfo) * mo.size(), cudaMemcpyHostToDevice);
@@ -721,7 +728,7 @@ ss_status ss_orb_extract(ss_ctx* c, int32_t n_frames, const uint8_t* d_frames, i
     prof_mark(c, s);
     prof_mark(c, s);
     SS_CUDA_TRY(launch_fast_bands(g, n_frames, src, c->bands + g.total_bands, g.total_bands, c->cells, c->slots,
-                                  c->cell_counts, s));
+                                  c->cell_counts, s, c->fast_flat != 0));
     prof_mark(c, s);
   }
   prof_mark(c, s);

@@ -182,7 +182,8 @@ bool pyramid_plan(const Geom& g, const uint32_t* tab, const int64_t* xoff, const
 cudaError_t launch_pyramid(const Geom& g, int n_frames, FrameSrc src, const uint4* gtab, const uint32_t* ytab,
                            const PyrLvl* plan, int n_blocks, int buf0, int buf1, int smem, cudaStream_t s);
 cudaError_t launch_fast_bands(const Geom& g, int n_frames, FrameSrc src, const BandInfo* bands, int n_bands,
-                              const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s);
+                              const CellInfo* cells, uint32_t* slots, int32_t* cell_counts, cudaStream_t s,
+                              bool flat = false);
 size_t fast_smem_bytes(const Geom& g, int* rp, int* mbw, int* region_bytes, int* mband_bytes, int* nball);
 cudaError_t launch_distribute(const Geom& g, int n_frames, int level0, int n_levels, const CellInfo* cells,
                               const uint32_t* qtab, const uint32_t* slots, const int32_t* cell_counts, uint32_t* selected,

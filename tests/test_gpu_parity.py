@@ -312,12 +312,14 @@ def test_search_local_points_chain(torch_cuda, ref, shape, th):
 
 
 @pytest.mark.parametrize("env", [{"SS_FAST_SPLIT": "1"}, {"SS_SEG0": "4", "SS_SEG": "4"},
-                                 {"SS_SEG0": "2", "SS_SEG": "3"}, {"SS_SEG0": "24", "SS_SEG": "24"}],
-                         ids=["split-launch", "seg4", "seg2-3", "seg24"])
+                                 {"SS_SEG0": "2", "SS_SEG": "3"}, {"SS_SEG0": "24", "SS_SEG": "24"},
+                                 {"SS_FAST_FLAT": "1"}, {"SS_FAST_FLAT": "2"}],
+                         ids=["split-launch", "seg4", "seg2-3", "seg24", "flat", "flat-l0-first"])
 def test_extract_launch_layouts(torch_cuda, ref, env, monkeypatch):
     """The FAST launch layouts the A/B switches select (level 0 beside the pyramid; 2..24-cell
     segments, i.e. other cell-start columns for the NMS's neighbour masks and other band
-    widths) give the same bit-exact extraction on EuRoC and KITTI frames."""
+    widths; a flat band-major grid, with or without level 0 first) give the same bit-exact
+    extraction on EuRoC and KITTI frames."""
     torch = torch_cuda
     for k, v in env.items():  # read by ss_create
         monkeypatch.setenv(k, v)
