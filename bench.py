@@ -293,7 +293,8 @@ def measured_peaks() -> dict:
 # ----------------------------------------------------------------------------- algorithmic work
 # FAST-9 work model of SURVEY.md §8(d) (N2+N3 row): >= 32 compares per detect pixel (16 ring
 # pixels x 2 polarities) + the contiguity test ~= 40 integer ops per detect pixel.  (The
-# kernel's own exact-score formulation issues ~52 ALU-pipe ops per pixel: DESIGN.md §5.)
+# kernel's own exact-score formulation issues ~52 ALU-pipe ops per pixel, the whole kernel ~95
+# thread instructions per pixel with staging, NMS and output: DESIGN.md §5.)
 FAST_OPS_PER_PX = 40.0
 FAST_KERNEL_OPS_PER_PX = 51.5
 # Hamming distance of two 256-bit descriptors: 8 POPC (XU pipe) per candidate (O9 / O13)
@@ -805,8 +806,9 @@ def run_ours(args, cfg):
                              "frac": achieved / alu_peak_tops, "traffic": None, "kernel": name,
                              "peak_src": f"{ipk['src']}: {ipk['alu']:.0f} ALU-pipe ops/clk/SM x {n_sm} SMs x "
                                          f"{clk_mhz:.0f} MHz (SM clock under load in this run)",
-                             "work": f"{FAST_OPS_PER_PX:g} int ops per detect pixel (SURVEY.md §8(d)); the kernel "
-                                     f"issues ~{FAST_KERNEL_OPS_PER_PX:g}", "share_of_step": share}
+                             "work": f"{FAST_OPS_PER_PX:g} int ops per detect pixel (SURVEY.md §8(d)); the kernel's "
+                                     f"score core issues ~{FAST_KERNEL_OPS_PER_PX:g} ALU-pipe ops per pixel and the "
+                                     f"whole kernel ~95 thread instructions per pixel (ncu)", "share_of_step": share}
         # tensor: int8 dense peak = measured bf16 dense x 2 (the guide's nominal i8 : bf16 ratio)
         achieved = work / (us * 1e-6) / 1e12
         return members, {"bound": "tensor", "achieved": achieved, "peak": peaks["i8_tops"], "unit": "TOPS",
