@@ -1287,7 +1287,7 @@ def main(argv=None):
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--config", choices=sorted(CONFIGS), default="c2")
     ap.add_argument("--ring", type=int, default=0, help="override the number of input ring slots")
-    ap.add_argument("--inflight", type=int, default=6, help="ticks in flight (contexts/streams)")
+    ap.add_argument("--inflight", type=int, default=8, help="ticks in flight (contexts/streams); 8 = the e2e depth")
     ap.add_argument("--e2e-inflight", type=int, default=8, help="ticks in flight on the end-to-end (host memory) path")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
